@@ -1,0 +1,103 @@
+/*
+ * arb_oracle.h — plain, slow, sequential CPU oracle for the ARBALEST replay.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and
+ * bench.py's cpu_baseline / --impl reference legs may load this library.
+ * It shares no code, header, table or constant generator with the CUDA path
+ * (paper_conf_ipps_yuphs21_b200/csrc); every constant below is restated here
+ * from the paper and from the trace format in DESIGN.md §3.
+ *
+ * Paper: L. Yu, J. Protze, O. Hernandez, V. Sarkar, "ARBALEST: Dynamic
+ * Detection of Data Mapping Issues in Heterogeneous OpenMP Applications",
+ * IPDPS 2021.  Citations "P:n" are lines of /root/reference/PAPER.md.
+ *
+ * What it computes:
+ *   for every record i in trace order, expand it into word-ops; for every
+ *   (word x, op o): MIR check against the log of unjoined async ops on x,
+ *   VSM check, VSM transition (bits of Table II),
+ *   log the op if it runs inside a nowait task.  Output: the sorted unique
+ *   (word, record, kind) triples and the final 4-bit state of every word.
+ *
+ * Parity status of each part:
+ *   VSM edges / fault condition          pinned (prose edges + Definition-1 brute force)
+ *   UUM-vs-USD split (init bits, Z2)      pinned to Definition 1 (value simulator);
+ *                                         parity unpinned BY THE PAPER (Fig.1/Fig.2 do not split readings)
+ *   Table I refcount resolution (Z5-Z7)   pinned (hand scenarios + brute force vs independent model)
+ *   MIR predicate (Theorem 1, Z10)        pinned (schedule enumeration)
+ *   MIR attribution to later event (Z11)  parity unpinned (definition only)
+ *   dedup-first mode (Z3)                 parity unpinned (definition only)
+ *   sub-word semantics (Z4)               parity unpinned (definition only)
+ */
+#ifndef ARB_ORACLE_H
+#define ARB_ORACLE_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Trace record: two little-endian 64-bit words.
+ * w0: [0,48) byte address | [48,56) op | [56,64) arg (map-type or update dir)
+ * w1: [0,48) length in bytes          | [48,64) task id (TASK_BEGIN/END, SYNC) */
+typedef struct { uint64_t w0, w1; } orc_record;
+
+/* ops (P:242-245 read/write host/target; P:106-123 device directives) */
+enum { ORC_RH = 0, ORC_WH = 1, ORC_RT = 2, ORC_WT = 3,
+       ORC_MAP_ENTER = 8, ORC_MAP_EXIT = 9, ORC_UPDATE = 10,
+       ORC_TASK_BEGIN = 12, ORC_TASK_END = 13, ORC_SYNC = 14 };
+/* map-types (Table I) */
+enum { ORC_TO = 0, ORC_FROM = 1, ORC_TOFROM = 2, ORC_ALLOC = 3,
+       ORC_RELEASE = 4, ORC_DELETE = 5 };
+/* update direction */
+enum { ORC_UPD_TO = 0, ORC_UPD_FROM = 1 };
+#define ORC_SYNC_ALL 0xFFFFu
+/* report kinds */
+enum { ORC_UUM = 1, ORC_USD = 2, ORC_MIR = 3 };
+/* status codes (same values as the library's, restated) */
+enum { ORC_OK = 0, ORC_EINVAL = -1, ORC_ENOMEM = -2, ORC_EMAP = -4,
+       ORC_ETRACE = -5, ORC_EOPEN = -7 };
+
+typedef struct {
+  uint64_t word;    /* absolute word index = byte address / 8 */
+  uint64_t record;  /* record index (global_index[i] if given, else i) */
+  uint32_t kind;    /* ORC_UUM / ORC_USD / ORC_MIR */
+  uint32_t pad;
+} orc_report;
+
+typedef struct {
+  uint64_t addr_base;    /* tracked byte range [addr_base, addr_base+addr_bytes), 8-B aligned */
+  uint64_t addr_bytes;
+  int      dedup_first;  /* Z3: keep only the first report per (word, kind) */
+  /* Sparse mode: if tracked_words != NULL only these absolute word indices
+   * (sorted ascending, unique, inside the range) carry state and reports.
+   * Words of the range that are not listed are ignored.  Dense mode
+   * (tracked_words == NULL) tracks every word of the range (Z12). */
+  const uint64_t* tracked_words;
+  uint64_t        n_tracked;
+} orc_config;
+
+typedef struct {
+  uint64_t records;        /* records replayed */
+  uint64_t word_events;    /* (tracked word, data-op) pairs */
+  uint64_t transitions;    /* VSM transitions applied; invariant: == word_events */
+  uint64_t control_records;
+  uint64_t ignored_word_events; /* word-ops on untracked words */
+  uint64_t tasks;          /* task instances */
+  uint64_t error_record;   /* index of the offending record when rc < 0 */
+} orc_stats;
+
+/* Replay n records.  global_index may be NULL (record index = position).
+ * On success *out / *n_out receive a malloc'ed array of reports in canonical
+ * order (word, record, kind ascending) that the caller frees with
+ * orc_free(); shadow_out (dense: addr_bytes/8 bytes, sparse: n_tracked
+ * bytes, may be NULL) receives the final states (bit0 OVv, bit1 CVv,
+ * bit2 OVi, bit3 CVi — Table II).  Returns ORC_OK or an error. */
+int  orc_replay(const orc_config* cfg, const orc_record* rec, uint64_t n,
+                const uint64_t* global_index, orc_report** out, uint64_t* n_out,
+                uint8_t* shadow_out, orc_stats* stats);
+void orc_free(void* p);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

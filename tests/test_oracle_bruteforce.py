@@ -1,0 +1,138 @@
+"""Brute-force pins: oracle vs the Definition-1 value simulator (tests/valuesim.py).
+
+SURVEY §4 / §8(c): every record sequence of bounded length over the access +
+map + update alphabet, on 1-word and 2-word arrays (sections [0,1), [1,2),
+[0,2)), must give the same UUM/USD reports and the same final per-word state
+(Table II bits P:330-333) as the value-level simulator, which knows nothing
+about the state machine and implements Table I's reference counting on its own.
+"""
+import itertools
+
+import numpy as np
+import pytest
+
+from gen.trace import MAP, OP, UPD, encode
+from valuesim import MapError, ValueSim
+
+ACC = [OP.RH, OP.WH, OP.RT, OP.WT]
+ENTER_T = [MAP.TO, MAP.FROM, MAP.TOFROM, MAP.ALLOC]
+EXIT_T = [MAP.TO, MAP.FROM, MAP.TOFROM, MAP.ALLOC, MAP.RELEASE, MAP.DELETE]
+
+
+def alphabet(nwords):
+    sections = [(0, 1)] if nwords == 1 else [(0, 1), (1, 2), (0, 2)]
+    sym = []
+    for op in ACC:
+        for w in range(nwords):
+            sym.append(("acc", op, w * 8, 8))
+    for lo, hi in sections:
+        for t in ENTER_T:
+            sym.append(("ctl", OP.MAP_ENTER, lo * 8, (hi - lo) * 8, t))
+        for t in EXIT_T:
+            sym.append(("ctl", OP.MAP_EXIT, lo * 8, (hi - lo) * 8, t))
+        for d in (UPD.TO, UPD.FROM):
+            sym.append(("ctl", OP.UPDATE, lo * 8, (hi - lo) * 8, d))
+    return sym
+
+
+def encode_seq(seq, base):
+    out = []
+    for s in seq:
+        if s[0] == "acc":
+            out.append(encode(s[1], base + s[2], s[3]))
+        else:
+            out.append(encode(s[1], base + s[2], s[3], arg=s[4]))
+    return out
+
+
+def check_batch(orc, seqs, nwords):
+    """Concatenate the sequences on disjoint arrays, run the oracle once, compare per array."""
+    stride = 8 * nwords
+    recs, expect, states, offsets = [], [], [], []
+    for j, seq in enumerate(seqs):
+        base = stride * j
+        enc = encode_seq(seq, base)
+        vs = ValueSim()
+        try:
+            issues = vs.run(enc)
+        except MapError:
+            continue
+        off = len(recs)
+        offsets.append(off)
+        recs.extend(enc)
+        expect.extend((w, i + off, k) for (w, i, k) in issues)
+        states.extend(vs.state_bits(base // 8 + w) for w in range(nwords))
+    arr = np.array(recs, dtype=np.uint64).reshape(-1, 2)
+    nseq = len(offsets)
+    res = orc.replay(arr, 0, stride * (len(seqs)))
+    assert res.rc == 0
+    assert res.triples() == sorted(expect)
+    # final states: only the arrays that were kept
+    got = []
+    kept = 0
+    for j, seq in enumerate(seqs):
+        try:
+            ValueSim().run(encode_seq(seq, stride * j))
+        except MapError:
+            continue
+        got.extend(int(res.shadow[(stride * j) // 8 + w]) for w in range(nwords))
+        kept += 1
+    assert got == states
+    assert res.stats["transitions"] == res.stats["word_events"]
+    return nseq
+
+
+def test_one_word_exhaustive(orc):
+    sym = alphabet(1)
+    seqs = [s for L in range(1, 5) for s in itertools.product(sym, repeat=L)]
+    assert check_batch(orc, seqs, 1) > 60000
+
+
+def test_one_word_random_long(orc):
+    sym = alphabet(1)
+    rs = np.random.default_rng(11)
+    seqs = [tuple(sym[i] for i in rs.integers(0, len(sym), rs.integers(5, 9))) for _ in range(40000)]
+    check_batch(orc, seqs, 1)
+
+
+def test_two_words_exhaustive(orc):
+    sym = alphabet(2)
+    seqs = [s for L in range(1, 4) for s in itertools.product(sym, repeat=L)]
+    assert check_batch(orc, seqs, 2) > 50000
+
+
+def test_two_words_random_long(orc):
+    sym = alphabet(2)
+    rs = np.random.default_rng(12)
+    seqs = [tuple(sym[i] for i in rs.integers(0, len(sym), rs.integers(4, 8))) for _ in range(40000)]
+    check_batch(orc, seqs, 2)
+
+
+def test_emap_agrees(orc):
+    """Sequences the independent refcount model rejects are rejected by the oracle (ARB_EMAP)."""
+    sym = alphabet(2)
+    n_bad = 0
+    for seq in itertools.product(sym, repeat=2):
+        enc = encode_seq(seq, 0)
+        try:
+            ValueSim().run(enc)
+            bad = False
+        except MapError:
+            bad = True
+        rc = orc.replay(np.array(enc, dtype=np.uint64).reshape(-1, 2), 0, 16).rc
+        assert (rc == -4) == bad
+        n_bad += bad
+    assert n_bad > 0
+
+
+def test_one_word_len6_reduced(orc):
+    """Length <= 6 (north_star) over a 10-symbol alphabet: accesses, enter to/alloc,
+    exit from/release, update to/from."""
+    full = alphabet(1)
+    keep = [s for s in full if s[0] == "acc" or
+            (s[1] == OP.MAP_ENTER and s[4] in (MAP.TO, MAP.ALLOC)) or
+            (s[1] == OP.MAP_EXIT and s[4] in (MAP.FROM, MAP.RELEASE)) or s[1] == OP.UPDATE]
+    assert len(keep) == 10
+    seqs = list(itertools.product(keep, repeat=6))
+    for k in range(0, len(seqs), 250000):
+        check_batch(orc, seqs[k:k + 250000], 1)

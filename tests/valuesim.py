@@ -1,0 +1,148 @@
+"""Definition-1 value simulator — an independent ground truth used to PIN the oracle.
+
+Definition 1: "For a read on the host that can receive a value
+from a write to the same variable on the accelerator (or vice versa), a data
+mapping issue occurs if the read does not observe the write; namely, the read
+fails to return the value placed by the write."
+
+This simulator does not use the state machine at all.  Every write gets a
+fresh id; OV and CV of each 8-byte word hold the id of the value they contain
+(BOT = never defined, "the variable's CV has not been created and its
+OV has not been explicitly initialized"); transfers copy contents (P:117,
+P:121, Table I memcpy); new/delete CV make the CV content undefined.  A read
+is an issue iff the side it reads does not hold the latest write; it is a use
+of uninitialized memory iff the side holds no defined value at all, else a use
+of stale data.
+
+The map-clause reference counting is re-implemented here from Table I
+ and OpenMP 5.1 independently of the oracle's code.
+"""
+from __future__ import annotations
+
+BOT = 0  # undefined content
+
+RH, WH, RT, WT, MAP_ENTER, MAP_EXIT, UPDATE = 0, 1, 2, 3, 8, 9, 10
+TASK_BEGIN, TASK_END, SYNC = 12, 13, 14
+TO, FROM, TOFROM, ALLOC, RELEASE, DELETE = 0, 1, 2, 3, 4, 5
+UUM, USD = 1, 2
+
+
+class MapError(Exception):
+    pass
+
+
+class ValueSim:
+    def __init__(self):
+        self.ov: dict[int, int] = {}
+        self.cv: dict[int, int] = {}
+        self.latest: dict[int, int] = {}
+        self.next_id = 1
+        self.present: list[list[int]] = []  # [lo, hi, refcount] byte intervals
+        self.issues: set[tuple[int, int, int]] = set()
+
+    # -- per-word primitive operations ---------------------------------------
+    def _write(self, side, w):
+        vid = self.next_id
+        self.next_id += 1
+        side[w] = vid
+        self.latest[w] = vid
+
+    def _read(self, side, w, idx):
+        lat = self.latest.get(w)
+        got = side.get(w, BOT)
+        if lat is None or got != lat:
+            self.issues.add((w, idx, UUM if got == BOT else USD))
+
+    def word_op(self, name, w, idx):
+        if name == "RH":
+            self._read(self.ov, w, idx)
+        elif name == "RT":
+            self._read(self.cv, w, idx)
+        elif name == "WH":
+            self._write(self.ov, w)
+        elif name == "WT":
+            self._write(self.cv, w)
+        elif name == "UPT":   # memcpy(CV, OV)
+            self.cv[w] = self.ov.get(w, BOT)
+        elif name == "UPH":   # memcpy(OV, CV)
+            self.ov[w] = self.cv.get(w, BOT)
+        elif name in ("NEW", "DEL"):  # fresh or deleted CV holds nothing
+            self.cv[w] = BOT
+        else:
+            raise ValueError(name)
+
+    @staticmethod
+    def words(addr, length):
+        return range(addr // 8, (addr + length - 1) // 8 + 1)
+
+    # -- map clauses (Table I) ------------------------------------------------
+    def _lookup(self, lo, hi):
+        hit = None
+        for ent in self.present:
+            if ent[0] <= lo and hi <= ent[1]:
+                hit = ent
+            elif lo < ent[1] and ent[0] < hi:
+                raise MapError("partial overlap")
+        return hit
+
+    def record(self, op, addr, length, arg, idx):
+        if op in (RH, WH, RT, WT):
+            name = {RH: "RH", WH: "WH", RT: "RT", WT: "WT"}[op]
+            for w in self.words(addr, length):
+                self.word_op(name, w, idx)
+        elif op == MAP_ENTER:
+            ent = self._lookup(addr, addr + length)
+            if ent is not None:
+                ent[2] += 1
+                return
+            self.present.append([addr, addr + length, 1])
+            for w in self.words(addr, length):
+                self.word_op("NEW", w, idx)
+            if arg in (TO, TOFROM):
+                for w in self.words(addr, length):
+                    self.word_op("UPT", w, idx)
+        elif op == MAP_EXIT:
+            ent = self._lookup(addr, addr + length)
+            if ent is None:
+                return
+            ent[2] = 0 if arg == DELETE else ent[2] - 1
+            if ent[2] == 0:
+                if arg in (FROM, TOFROM):
+                    for w in self.words(addr, length):
+                        self.word_op("UPH", w, idx)
+                for w in self.words(ent[0], ent[1] - ent[0]):
+                    self.word_op("DEL", w, idx)
+                self.present.remove(ent)
+        elif op == UPDATE:
+            ent = self._lookup(addr, addr + length)
+            if ent is None:
+                return
+            for w in self.words(addr, length):
+                self.word_op("UPT" if arg == 0 else "UPH", w, idx)
+        # TASK_BEGIN / TASK_END / SYNC: no data effect
+
+    def run(self, records):
+        """records: iterable of (w0, w1); returns the set of UUM/USD issues."""
+        for idx, (w0, w1) in enumerate(records):
+            w0 = int(w0)
+            w1 = int(w1)
+            self.record((w0 >> 48) & 0xFF, w0 & ((1 << 48) - 1), w1 & ((1 << 48) - 1),
+                        w0 >> 56, idx)
+        return self.issues
+
+    def state_bits(self, w):
+        """The 4 quantities of Table II as observed on values (for final-state pins)."""
+        lat = self.latest.get(w)
+        ov = self.ov.get(w, BOT)
+        cv = self.cv.get(w, BOT)
+        ovv = lat is not None and ov == lat
+        cvv = lat is not None and cv == lat
+        return int(ovv) | (int(cvv) << 1) | (int(ov != BOT) << 2) | (int(cv != BOT) << 3)
+
+
+def schedule_issues(ops):
+    """Definition-1 check of one schedule given as a list of (word_op_name, word)."""
+    vs = ValueSim()
+    for k, (name, w) in enumerate(ops):
+        vs.word_op(name, w, k)
+    return vs.issues
