@@ -1,0 +1,98 @@
+"""Seeded random offload programs for parity fuzzing (structure only).
+
+A program works on a few arrays; it opens and closes data regions on whole
+arrays or halves, runs host and device loops with random unaligned 1..8-byte
+accesses, target updates, nowait blocks (some joined late or never) and
+taskwaits.  The generator keeps a little bookkeeping so that most programs
+stay well-formed; it computes nothing the replay computes.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+from .trace import MAP, OP, UPD, SYNC_ALL, TraceBuilder, encode_np
+
+
+def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: int = 60,
+                   base: int = 0x10000, loop_max: int = 48, p_task: float = 0.15):
+    rs = np.random.default_rng(seed)
+    tb = TraceBuilder()
+    arrays = [base + i * array_words * 8 * 2 for i in range(n_arrays)]   # gap between arrays
+    present = {i: [] for i in range(n_arrays)}   # list of (lo, hi) byte sections entered
+    in_task = 0
+    next_task = 1
+    unjoined = []
+
+    def section(i):
+        a = arrays[i]
+        n = array_words * 8
+        kind = rs.integers(0, 4)
+        if kind == 0:
+            return a, n
+        if kind == 1:
+            return a, n // 2
+        if kind == 2:
+            return a + n // 2, n - n // 2
+        lo = int(rs.integers(0, array_words - 1)) * 8
+        return a + lo, int(rs.integers(1, array_words - lo // 8)) * 8
+
+    def loop(op):
+        i = int(rs.integers(n_arrays))
+        cnt = int(rs.integers(1, loop_max))
+        start = int(rs.integers(0, array_words * 8 - 8))
+        stride = int(rs.choice([1, 4, 8, 8, 8, 12]))
+        size = int(rs.choice([1, 2, 4, 8, 8, 8]))
+        addr = arrays[i] + start + stride * np.arange(cnt, dtype=np.uint64)
+        addr = addr[addr + size <= arrays[i] + array_words * 8 + 8]
+        if addr.size:
+            tb.add_array(encode_np(op, addr, size))
+
+    for _ in range(steps):
+        r = rs.random()
+        if r < 0.35:
+            loop(int(rs.choice([OP.RH, OP.WH, OP.RT, OP.WT])))
+        elif r < 0.5:
+            i = int(rs.integers(n_arrays))
+            lo, n = section(i)
+            hi = lo + n
+            ok = all(hi <= a or lo >= b or (a <= lo and hi <= b) for a, b in present[i])
+            if ok:
+                tb.enter(int(rs.choice([MAP.TO, MAP.FROM, MAP.TOFROM, MAP.ALLOC])), lo, n)
+                present[i].append((lo, hi))
+        elif r < 0.65:
+            i = int(rs.integers(n_arrays))
+            if present[i]:
+                k = int(rs.integers(len(present[i])))
+                lo, hi = present[i][k]
+                # exit only sections that contain no other present section
+                if all(not (lo <= a and b <= hi and (a, b) != (lo, hi)) for a, b in present[i]):
+                    tb.exit(int(rs.choice([MAP.TO, MAP.FROM, MAP.TOFROM, MAP.ALLOC,
+                                           MAP.RELEASE, MAP.DELETE])), lo, hi - lo)
+                    present[i].pop(k)
+        elif r < 0.72:
+            i = int(rs.integers(n_arrays))
+            if present[i]:
+                lo, hi = present[i][int(rs.integers(len(present[i])))]
+                tb.update(int(rs.choice([UPD.TO, UPD.FROM])), lo, hi - lo)
+            elif rs.random() < 0.3:
+                tb.update(int(rs.choice([UPD.TO, UPD.FROM])), arrays[i], array_words * 8)
+        elif r < 0.72 + p_task and not in_task:
+            k = next_task
+            next_task = next_task + 1 if next_task < 60000 else 1
+            tb.task_begin(k)
+            in_task = k
+        elif in_task and r < 0.95:
+            tb.task_end(in_task)
+            unjoined.append(in_task)
+            in_task = 0
+        elif not in_task and unjoined and r >= 0.95:
+            if rs.random() < 0.5:
+                tb.sync(SYNC_ALL)
+                unjoined = []
+            else:
+                k = unjoined.pop(int(rs.integers(len(unjoined))))
+                tb.sync(k)
+    if in_task:
+        tb.task_end(in_task)
+    span = n_arrays * array_words * 8 * 2
+    return tb.array(), base, span

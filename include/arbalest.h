@@ -1,0 +1,170 @@
+/*
+ * arbalest.h — C ABI of the B200-native ARBALEST replay library (libarbalest.so).
+ *
+ * Problem statement: given an execution trace
+ * of host/device memory accesses and OpenMP device directives, replay it through
+ * the per-location variable state machine (VSM) over 1 byte of shadow
+ * per 8-byte word (Table II) and report every read that
+ * fails to observe the latest write (Definition 1) — as a use of
+ * uninitialized memory (UUM) or a use of stale data (USD) — and
+ * every race between mapping-relevant operations of an unjoined nowait region
+ * and another operation (Theorem 1) as a mapping-induced race (MIR).
+ * The readings of the paper that fix every silent case are listed in
+ * DESIGN.md §2 (Z1-Z18).
+ *
+ * Conventions
+ *  - All integers little-endian.  No C++ exception crosses the ABI.
+ *  - Every call returns an int: ARB_OK (0), a negative error, or a positive
+ *    warning (ARB_TRUNCATED).
+ *  - One host thread per context.  Work is ordered on the CUDA stream passed
+ *    to the call (NULL = the legacy default stream); arb_flush synchronizes
+ *    that stream before it returns (the report counts cross to the host).
+ *  - Device pointers must be CUDA device (or managed) memory of the context's
+ *    device; "host" pointers are ordinary (pageable or pinned) host memory.
+ */
+#ifndef ARBALEST_H
+#define ARBALEST_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- trace records ---------------------------------------- */
+/* 16 B, 16-B aligned so that one 128-bit load reads one record.
+ * w0: [0,48) byte address | [48,56) op | [56,64) arg (map-type / update dir)
+ * w1: [0,48) length in bytes | [48,64) task id (TASK_BEGIN / TASK_END / SYNC) */
+typedef struct { uint64_t w0, w1; } arb_event;
+
+/* ops: accesses and device directives */
+enum arb_op {
+  ARB_RH = 0, ARB_WH = 1, ARB_RT = 2, ARB_WT = 3,       /* read/write host/target, 1..8 bytes */
+  ARB_MAP_ENTER = 8, ARB_MAP_EXIT = 9,                  /* map clause on region entry / exit   */
+  ARB_UPDATE = 10,                                      /* target update to/from       */
+  ARB_TASK_BEGIN = 12, ARB_TASK_END = 13,               /* nowait region block (Z8)     */
+  ARB_SYNC = 14                                         /* taskwait: joins task k, 0xFFFF = all */
+};
+/* map-types (Table I) */
+enum arb_map { ARB_TO = 0, ARB_FROM = 1, ARB_TOFROM = 2, ARB_ALLOC = 3,
+               ARB_RELEASE = 4, ARB_DELETE = 5 };
+/* target update direction */
+enum arb_upd { ARB_UPD_TO = 0, ARB_UPD_FROM = 1 };
+#define ARB_SYNC_ALL 0xFFFFu
+
+/* ---- reports ---------------------------------------------------------------- */
+enum arb_kind { ARB_UUM = 1, ARB_USD = 2, ARB_MIR = 3 };
+/* w0: [0,48) absolute word index (= byte address / 8) | [48,56) kind
+ * w1: global record index (0-based; see arb_submit_events)
+ * Canonical order: word, then record, then kind, ascending; no duplicates. */
+typedef struct { uint64_t w0, w1; } arb_report;
+
+/* ---- status codes -------------------------------------------------------------- */
+enum arb_status {
+  ARB_OK = 0,
+  ARB_TRUNCATED = 1,  /* warning: more reports than the buffer; the count is exact   */
+  ARB_EINVAL = -1,    /* bad argument                                                 */
+  ARB_ENOMEM = -2,    /* device or host allocation failed                             */
+  ARB_ECUDA = -3,     /* CUDA / NCCL failure: destroy the context                     */
+  ARB_EMAP = -4,      /* map clause partially overlaps a present entry (Z6)          */
+  ARB_ETRACE = -5,    /* malformed trace (Z18)                              */
+  ARB_ESTATE = -6,    /* call out of order (e.g. get_reports before any flush)        */
+  ARB_EOPEN = -7      /* a TASK_BEGIN block is still open at the end of the flush     */
+};
+/* After ARB_EMAP / ARB_ETRACE / ARB_EOPEN the pending batch is discarded, the
+ * committed shadow is unchanged and the context stays usable.  After ARB_ECUDA
+ * the context must be destroyed. */
+
+/* ---- configuration ------------------------------------------------------------- */
+#define ARB_F_DEDUP_FIRST 0x1u  /* keep only the first report per (word, kind) (Z3)      */
+#define ARB_F_TIMING      0x2u  /* record CUDA events around every kernel (arb_get_stats) */
+
+typedef struct {
+  uint64_t addr_base;        /* tracked OV byte range [addr_base, addr_base+addr_bytes);   */
+  uint64_t addr_bytes;       /*   both multiples of 8; shadow = addr_bytes/8 bytes of HBM. */
+                             /*   Words outside the range are ignored (Z12): in sharded    */
+                             /*   mode the range is this rank's shard.                     */
+  int      device;           /* CUDA ordinal                                               */
+  int      rank, world;      /* address shard of this process; world == 1: single GPU      */
+  const void* nccl_unique_id;/* ncclUniqueId* (128 B) when world > 1, else NULL            */
+  uint64_t report_capacity;  /* device report-candidate capacity, 0 = default (2^24)       */
+  uint32_t flags;            /* ARB_F_*                                                    */
+  uint32_t bucket_bits;      /* log2 words per address bucket, 0 = automatic               */
+} arb_config;
+
+/* Statistics of the last flush (and totals since arb_init). */
+typedef struct {
+  uint64_t records;          /* records in the last flush                                  */
+  uint64_t access_words;     /* word-events from access records (tracked words only)       */
+  uint64_t range_words;      /* word-events from MAP / UPDATE data ops (tracked words)     */
+  uint64_t control_records;  /* MAP / UPDATE / TASK / SYNC records                         */
+  uint64_t range_ops;        /* resolved ALLOC/UPT/UPH/REL range ops                       */
+  uint64_t tasks;            /* nowait task instances                                      */
+  uint64_t reports;          /* reports of the last flush (exact)                          */
+  uint64_t reports_by_kind[4];
+  uint64_t ignored_words;    /* word-ops outside the tracked range                        */
+  uint64_t buckets, bucket_bits, max_bucket_events;
+  uint64_t total_records, total_word_events, total_reports, flushes;
+  /* device time of each phase of the last flush in milliseconds (ARB_F_TIMING) */
+  double   ms_partition, ms_control, ms_replay, ms_mir, ms_reports, ms_total;
+  uint64_t kernel_launches;  /* kernels launched by the last flush                         */
+} arb_stats;
+
+typedef struct arb_ctx_s* arb_ctx;
+
+/* Create a context on cfg->device: allocates and zeroes the shadow (all words
+ * start invalid), workspaces, and (world > 1) the NCCL communicator from
+ * cfg->nccl_unique_id.  Returns ARB_OK and *out, or an error (*out = NULL).
+ * Ownership: the context owns the shadow, workspaces and report buffer. */
+int arb_init(const arb_config* cfg, arb_ctx* out);
+
+/* Append n records to the pending batch.
+ *  ev           device pointer (ev_on_device = 1): used zero-copy, must stay valid
+ *               and unmodified until arb_flush returns; host pointer (0): copied
+ *               (stream-ordered) before the call returns.
+ *  global_index NULL: record i of the batch gets the index (records submitted
+ *               since arb_init) + i; else an array of n u64 global indices in the
+ *               same memory space as ev (sharded mode: the rank sees a subset of
+ *               the global trace, in order).  Read only on the report path.
+ *  stream       cudaStream_t (NULL = legacy default stream).
+ * Records of one batch keep their relative order; a batch holds at most 2^30
+ * records.  Errors: ARB_EINVAL, ARB_ENOMEM, ARB_ECUDA. */
+int arb_submit_events(arb_ctx ctx, const arb_event* ev, uint64_t n,
+                      const uint64_t* global_index, int ev_on_device, void* stream);
+
+/* Replay the pending batch: decode + partition, control resolution (Table I),
+ * per-address segmented scan + classification, MIR join, canonical report
+ * compaction, and (world > 1) the allgather of per-rank report counts.
+ *  n_reports_local       this rank's report count (exact even if truncated)
+ *  report_offset_global  exclusive prefix of the counts over ranks (0 if world 1)
+ * Both may be NULL.  Synchronizes `stream`.  The batch is consumed.  Returns
+ * ARB_OK, ARB_TRUNCATED (more candidates than report_capacity; the count is
+ * exact, the stored set is the canonical order of the retained candidates),
+ * ARB_EMAP / ARB_ETRACE / ARB_EOPEN (batch discarded, shadow unchanged) or
+ * ARB_ECUDA / ARB_ENOMEM. */
+int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local,
+              uint64_t* report_offset_global);
+
+/* Copy up to cap reports of the last flush, in canonical order, to out
+ * (out_on_device = 1: device pointer, else host).  *n_written = copied count.
+ * Returns ARB_OK, ARB_TRUNCATED if cap < count, ARB_ESTATE before any flush. */
+int arb_get_reports(arb_ctx ctx, arb_report* out, uint64_t cap, uint64_t* n_written,
+                    int out_on_device);
+
+/* Copy the final shadow byte of words [word_lo, word_lo + n) (absolute word
+ * indices inside the tracked range) to out (host or device).  Bits: 0 OVv,
+ * 1 CVv, 2 OVi, 3 CVi (Table II).  Synchronous. */
+int arb_get_shadow(arb_ctx ctx, uint64_t word_lo, uint64_t n, uint8_t* out, int out_on_device);
+
+/* Statistics of the last flush and totals. */
+int arb_get_stats(arb_ctx ctx, arb_stats* out);
+
+/* Human-readable description of the last error of ctx (never NULL). */
+const char* arb_last_error(arb_ctx ctx);
+
+/* Release every resource of ctx (NULL is a no-op). */
+int arb_destroy(arb_ctx ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,492 @@
+// api.cpp — the C ABI of libarbalest (include/arbalest.h).
+#include "arbalest.h"
+#include "arb_internal.h"
+#include "control.h"
+
+#include <dlfcn.h>
+#include <algorithm>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+using namespace arb;
+
+namespace {
+
+// ---- NCCL through dlopen (only needed when world > 1) ---------------------
+// ncclUniqueId is a 128-byte struct passed by value
+struct NcclId { char internal[128]; };
+typedef int (*nccl_init_fn)(void** comm, int nranks, NcclId id, int rank);
+typedef int (*nccl_allgather_fn)(const void* send, void* recv, size_t count, int dtype, void* comm, cudaStream_t s);
+typedef int (*nccl_destroy_fn)(void* comm);
+constexpr int kNcclUint64 = 5;  // ncclUint64
+
+template <class T>
+struct DevBuf {
+  T* p = nullptr;
+  size_t cap = 0;
+  cudaError_t ensure(size_t n) {
+    if (n <= cap) return cudaSuccess;
+    size_t c = std::max(n, (size_t)(cap * 3 / 2));
+    if (p) cudaFree(p);
+    p = nullptr; cap = 0;
+    cudaError_t e = cudaMalloc(&p, c * sizeof(T) + 16);
+    if (e == cudaSuccess) cap = c;
+    return e;
+  }
+  // grow keeping the first `keep` elements (staging buffers filled across submits)
+  cudaError_t ensure_keep(size_t n, size_t keep) {
+    if (n <= cap) return cudaSuccess;
+    size_t c = std::max(n, (size_t)(cap * 3 / 2));
+    T* q = nullptr;
+    cudaError_t e = cudaMalloc(&q, c * sizeof(T) + 16);
+    if (e != cudaSuccess) return e;
+    keep = std::min(keep, cap);
+    if (p && keep) e = cudaMemcpy(q, p, keep * sizeof(T), cudaMemcpyDeviceToDevice);
+    if (p) cudaFree(p);
+    p = q; cap = c;
+    return e;
+  }
+  void release() { if (p) cudaFree(p); p = nullptr; cap = 0; }
+};
+
+template <class T>
+cudaError_t upload(DevBuf<T>& b, const std::vector<T>& v, cudaStream_t s) {
+  cudaError_t e = b.ensure(std::max<size_t>(v.size(), 1));
+  if (e != cudaSuccess || v.empty()) return e;
+  return cudaMemcpyAsync(b.p, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice, s);
+}
+
+struct Submit { const void* ev; uint64_t n; const uint64_t* gidx; int on_device; };
+
+}  // namespace
+
+struct arb_ctx_s {
+  arb_config cfg{};
+  uint64_t base_word = 0, n_words = 0;
+  uint32_t bucket_bits = 0, n_buckets = 0;
+  int n_sms = 148;
+  uint8_t* shadow = nullptr;
+  std::vector<Submit> subs;
+  uint64_t pending = 0;
+  bool any_gidx = false, any_nogidx = false;
+  DevBuf<uint4> staging;
+  DevBuf<uint64_t> gidx_staging;
+  DevBuf<uint2> part_ev;
+  DevBuf<uint16_t> part_off;
+  DevBuf<CtlRec> ctl;
+  DevBuf<uint4> cand, cand_tmp, reports;
+  DevBuf<uint32_t> blk;
+  DevBuf<uint32_t> ops_start;
+  DevBuf<BucketOp> ops;
+  DevBuf<DevStats> dstats;
+  DevBuf<unsigned long long> dcount;
+  // MIR
+  DevBuf<uint64_t> m_ins_lo, m_ins_cum, m_qry_lo, m_qry_cum, m_rr_cum;
+  DevBuf<uint32_t> m_ins_inst, m_qry_open_start, m_open_list, m_own_start, m_win_start;
+  DevBuf<RangeRef> m_own, m_win, m_rr;
+  DevBuf<unsigned long long> hkeys;
+  DevBuf<uint32_t> hvals;
+  uint64_t ctl_cap = 1 << 16;
+  uint64_t cand_cap = 1 << 24;
+  MapTable map;
+  uint64_t next_index = 0;
+  uint64_t n_reports = 0;      // exact count of the last flush
+  uint64_t n_stored = 0;       // reports held in `reports`
+  bool flushed = false;
+  std::string err;
+  arb_stats stats{};
+  cudaEvent_t ev[8] = {};
+  // NCCL
+  void* nccl_lib = nullptr;
+  void* comm = nullptr;
+  nccl_allgather_fn nccl_allgather = nullptr;
+  nccl_destroy_fn nccl_destroy = nullptr;
+  DevBuf<uint64_t> counts;
+};
+
+static int fail(arb_ctx c, int rc, const std::string& msg) {
+  if (c) c->err = msg;
+  return rc;
+}
+static int cuda_fail(arb_ctx c, cudaError_t e, const char* where) {
+  return fail(c, ARB_ECUDA, std::string(where) + ": " + cudaGetErrorString(e));
+}
+#define CK(call, where)                                    \
+  do {                                                     \
+    cudaError_t _e = (call);                               \
+    if (_e != cudaSuccess) return cuda_fail(ctx, _e, where); \
+  } while (0)
+
+extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
+  if (!out) return ARB_EINVAL;
+  *out = nullptr;
+  if (!cfg || (cfg->addr_base & 7) || (cfg->addr_bytes & 7) || cfg->addr_bytes == 0 ||
+      cfg->addr_base + cfg->addr_bytes > (1ull << 48) || cfg->world < 1 || cfg->rank < 0 ||
+      cfg->rank >= cfg->world || (cfg->world > 1 && !cfg->nccl_unique_id))
+    return ARB_EINVAL;
+  arb_ctx ctx = new (std::nothrow) arb_ctx_s();
+  if (!ctx) return ARB_ENOMEM;
+  ctx->cfg = *cfg;
+  ctx->base_word = cfg->addr_base >> 3;
+  ctx->n_words = cfg->addr_bytes >> 3;
+  // address buckets: <= 1024 buckets, >= 2^12 words each, <= 2^30 words each
+  uint32_t bits = cfg->bucket_bits;
+  if (bits == 0) {
+    bits = 12;
+    while (bits < 30 && ((ctx->n_words + (1ull << bits) - 1) >> bits) > (uint64_t)kMaxBuckets) ++bits;
+  }
+  if (bits > 30 || ((ctx->n_words + (1ull << bits) - 1) >> bits) > (uint64_t)kMaxBuckets) {
+    delete ctx;
+    return ARB_EINVAL;
+  }
+  ctx->bucket_bits = bits;
+  ctx->n_buckets = (uint32_t)((ctx->n_words + (1ull << bits) - 1) >> bits);
+  if (cfg->report_capacity) ctx->cand_cap = cfg->report_capacity;
+  cudaError_t e = cudaSetDevice(cfg->device);
+  if (e != cudaSuccess) { delete ctx; return ARB_ECUDA; }
+  cudaDeviceGetAttribute(&ctx->n_sms, cudaDevAttrMultiProcessorCount, cfg->device);
+  e = cudaMalloc(&ctx->shadow, ctx->n_words + 16);
+  if (e != cudaSuccess) { delete ctx; return ARB_ENOMEM; }
+  e = cudaMemset(ctx->shadow, 0, ctx->n_words);                 // all invalid
+  if (e == cudaSuccess) e = ctx->dstats.ensure(1);
+  if (e == cudaSuccess) e = ctx->dcount.ensure(4);
+  if (e == cudaSuccess) e = ctx->ctl.ensure(ctx->ctl_cap);
+  for (int i = 0; i < 8 && e == cudaSuccess; ++i) e = cudaEventCreate(&ctx->ev[i]);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) { arb_destroy(ctx); return ARB_ENOMEM; }
+  if (cfg->world > 1) {
+    ctx->nccl_lib = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!ctx->nccl_lib) { arb_destroy(ctx); return ARB_ECUDA; }
+    auto init = (nccl_init_fn)dlsym(ctx->nccl_lib, "ncclCommInitRank");
+    ctx->nccl_allgather = (nccl_allgather_fn)dlsym(ctx->nccl_lib, "ncclAllGather");
+    ctx->nccl_destroy = (nccl_destroy_fn)dlsym(ctx->nccl_lib, "ncclCommDestroy");
+    if (!init || !ctx->nccl_allgather || !ctx->nccl_destroy) { arb_destroy(ctx); return ARB_ECUDA; }
+    NcclId id;
+    std::memcpy(id.internal, cfg->nccl_unique_id, sizeof(id.internal));
+    if (init(&ctx->comm, cfg->world, id, cfg->rank) != 0 || ctx->counts.ensure(cfg->world + 1) != cudaSuccess) {
+      arb_destroy(ctx);
+      return ARB_ECUDA;
+    }
+  }
+  *out = ctx;
+  return ARB_OK;
+}
+
+extern "C" int arb_destroy(arb_ctx ctx) {
+  if (!ctx) return ARB_OK;
+  if (ctx->comm && ctx->nccl_destroy) ctx->nccl_destroy(ctx->comm);
+  if (ctx->shadow) cudaFree(ctx->shadow);
+  ctx->staging.release(); ctx->gidx_staging.release(); ctx->part_ev.release(); ctx->part_off.release();
+  ctx->ctl.release(); ctx->cand.release(); ctx->cand_tmp.release(); ctx->reports.release(); ctx->blk.release();
+  ctx->ops_start.release(); ctx->ops.release(); ctx->dstats.release(); ctx->dcount.release();
+  ctx->m_ins_lo.release(); ctx->m_ins_cum.release(); ctx->m_qry_lo.release(); ctx->m_qry_cum.release();
+  ctx->m_rr_cum.release(); ctx->m_ins_inst.release(); ctx->m_qry_open_start.release(); ctx->m_open_list.release();
+  ctx->m_own_start.release(); ctx->m_win_start.release(); ctx->m_own.release(); ctx->m_win.release();
+  ctx->m_rr.release(); ctx->hkeys.release(); ctx->hvals.release(); ctx->counts.release();
+  for (auto& e : ctx->ev) if (e) cudaEventDestroy(e);
+  if (ctx->nccl_lib) dlclose(ctx->nccl_lib);
+  delete ctx;
+  return ARB_OK;
+}
+
+extern "C" const char* arb_last_error(arb_ctx ctx) {
+  if (!ctx) return "null context";
+  return ctx->err.c_str();
+}
+
+extern "C" int arb_submit_events(arb_ctx ctx, const arb_event* ev, uint64_t n, const uint64_t* global_index,
+                                 int ev_on_device, void* stream) {
+  if (!ctx) return ARB_EINVAL;
+  if (n == 0) return ARB_OK;
+  if (!ev) return fail(ctx, ARB_EINVAL, "null event pointer");
+  if (ctx->pending + n > kMaxBatchRecords) return fail(ctx, ARB_EINVAL, "batch exceeds 2^30 records");
+  if ((global_index != nullptr && ctx->any_nogidx) || (global_index == nullptr && ctx->any_gidx))
+    return fail(ctx, ARB_EINVAL, "global_index must be given for every submit of a batch or for none");
+  cudaSetDevice(ctx->cfg.device);
+  cudaStream_t s = (cudaStream_t)stream;
+  if (!ev_on_device) {
+    // host records are copied now (stream-ordered) into the staging buffer
+    uint64_t off = ctx->pending;
+    // keep earlier device submits: move them into staging first
+    cudaError_t e = cudaStreamSynchronize(s);
+    if (e == cudaSuccess) e = ctx->staging.ensure_keep(off + n, off);
+    if (e != cudaSuccess) return fail(ctx, ARB_ENOMEM, "staging buffer");
+    e = cudaMemcpyAsync(ctx->staging.p + off, ev, n * sizeof(arb_event), cudaMemcpyHostToDevice, s);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "copy host records");
+    if (global_index) {
+      if ((e = ctx->gidx_staging.ensure_keep(off + n, off)) != cudaSuccess) return fail(ctx, ARB_ENOMEM, "gidx staging");
+      e = cudaMemcpyAsync(ctx->gidx_staging.p + off, global_index, n * 8, cudaMemcpyHostToDevice, s);
+      if (e != cudaSuccess) return cuda_fail(ctx, e, "copy host global_index");
+    }
+    e = cudaStreamSynchronize(s);  // the caller may free the host buffer on return
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "submit sync");
+    ctx->subs.push_back(Submit{nullptr, n, nullptr, 0});
+  } else {
+    ctx->subs.push_back(Submit{ev, n, global_index, 1});
+  }
+  if (global_index) ctx->any_gidx = true; else ctx->any_nogidx = true;
+  ctx->pending += n;
+  return ARB_OK;
+}
+
+static void reset_batch(arb_ctx ctx) {
+  ctx->subs.clear();
+  ctx->pending = 0;
+  ctx->any_gidx = ctx->any_nogidx = false;
+}
+
+extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, uint64_t* report_offset_global) {
+  if (!ctx) return ARB_EINVAL;
+  cudaSetDevice(ctx->cfg.device);
+  cudaStream_t s = (cudaStream_t)stream;
+  const bool timing = ctx->cfg.flags & ARB_F_TIMING;
+  int launches = 0;
+  const uint64_t n = ctx->pending;
+  arb_stats& S = ctx->stats;
+  S.records = n; S.access_words = S.range_words = S.control_records = S.range_ops = S.tasks = 0;
+  S.reports = 0; std::memset(S.reports_by_kind, 0, sizeof(S.reports_by_kind)); S.ignored_words = 0;
+  S.ms_partition = S.ms_control = S.ms_replay = S.ms_mir = S.ms_reports = S.ms_total = 0;
+  S.buckets = ctx->n_buckets; S.bucket_bits = ctx->bucket_bits; S.max_bucket_events = 0;
+
+  // ---- resolve the batch into one device array ---------------------------
+  const uint4* ev = nullptr;
+  const uint64_t* gidx = nullptr;
+  if (n) {
+    bool single_dev = ctx->subs.size() == 1 && ctx->subs[0].on_device;
+    if (single_dev) {
+      ev = reinterpret_cast<const uint4*>(ctx->subs[0].ev);
+      gidx = ctx->subs[0].gidx;
+    } else {
+      // gather device submits into staging (host submits are already there)
+      uint64_t off = 0;
+      CK(cudaStreamSynchronize(s), "staging sync");
+      CK(ctx->staging.ensure_keep(n, n), "staging");
+      if (ctx->any_gidx) CK(ctx->gidx_staging.ensure_keep(n, n), "gidx staging");
+      for (const Submit& sb : ctx->subs) {
+        if (sb.on_device) {
+          CK(cudaMemcpyAsync(ctx->staging.p + off, sb.ev, sb.n * 16, cudaMemcpyDeviceToDevice, s), "gather");
+          if (sb.gidx) CK(cudaMemcpyAsync(ctx->gidx_staging.p + off, sb.gidx, sb.n * 8, cudaMemcpyDeviceToDevice, s), "gather gidx");
+        }
+        off += sb.n;
+      }
+      ev = ctx->staging.p;
+      gidx = ctx->any_gidx ? ctx->gidx_staging.p : nullptr;
+    }
+  }
+  const uint64_t index_base = ctx->next_index;
+
+  if (timing) cudaEventRecord(ctx->ev[0], s);
+  // ---- A1/A3a: decode + partition ------------------------------------------
+  const uint32_t n_chunks = (uint32_t)((n + kChunkRecords - 1) / kChunkRecords);
+  CK(ctx->part_ev.ensure((size_t)std::max<uint32_t>(n_chunks, 1) * kChunkCap), "alloc part_ev");
+  CK(ctx->part_off.ensure((size_t)(ctx->n_buckets + 1) * std::max<uint32_t>(n_chunks, 1)), "alloc part_off");
+  DevStats hst;
+  PartParams pp{};
+  for (int attempt = 0; attempt < 2; ++attempt) {
+    std::memset(&hst, 0, sizeof(hst));
+    hst.err_pos = ~0ull;
+    CK(cudaMemcpyAsync(ctx->dstats.p, &hst, sizeof(hst), cudaMemcpyHostToDevice, s), "stats init");
+    pp.ev = ev; pp.n = n; pp.base_word = ctx->base_word; pp.n_words = ctx->n_words;
+    pp.bucket_bits = ctx->bucket_bits; pp.n_buckets = ctx->n_buckets; pp.n_chunks = n_chunks;
+    pp.part_ev = ctx->part_ev.p; pp.part_off = ctx->part_off.p; pp.ctl = ctx->ctl.p; pp.ctl_cap = ctx->ctl_cap;
+    pp.st = ctx->dstats.p;
+    CK(launch_partition(pp, s), "k_partition");
+    launches += n_chunks ? 1 : 0;
+    CK(cudaMemcpyAsync(&hst, ctx->dstats.p, sizeof(hst), cudaMemcpyDeviceToHost, s), "stats d2h");
+    CK(cudaStreamSynchronize(s), "partition sync");
+    if (hst.n_ctl <= ctx->ctl_cap) break;
+    ctx->ctl_cap = hst.n_ctl + hst.n_ctl / 2;
+    CK(ctx->ctl.ensure(ctx->ctl_cap), "grow ctl");
+  }
+  if (timing) cudaEventRecord(ctx->ev[1], s);
+  if (hst.err_pos != ~0ull) {
+    reset_batch(ctx);
+    return fail(ctx, ARB_ETRACE, "malformed record at batch position " + std::to_string(hst.err_pos));
+  }
+  S.access_words = hst.access_words;
+  S.control_records = hst.n_ctl;
+
+  // ---- A2: control resolution on the host -------------------------------------
+  std::vector<CtlRec> ctl(hst.n_ctl);
+  if (hst.n_ctl) {
+    CK(cudaMemcpy(ctl.data(), ctx->ctl.p, hst.n_ctl * sizeof(CtlRec), cudaMemcpyDeviceToHost), "ctl d2h");
+    std::sort(ctl.begin(), ctl.end(), [](const CtlRec& a, const CtlRec& b) { return a.pos < b.pos; });
+  }
+  MapTable map = ctx->map;
+  FlushPlan plan;
+  resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_bits, ctx->n_buckets, map, plan);
+  if (plan.rc != 0) {
+    reset_batch(ctx);
+    return fail(ctx, plan.rc, plan.err + " (batch position " + std::to_string(plan.err_pos) + ")");
+  }
+  S.range_words = plan.range_words;
+  S.range_ops = plan.range_ops.size();
+  S.tasks = plan.tasks;
+  S.ignored_words = hst.ignored_words + plan.ignored_words;
+  CK(upload(ctx->ops_start, plan.ops_start, s), "upload ops_start");
+  CK(upload(ctx->ops, plan.ops, s), "upload ops");
+  CK(ctx->cand.ensure(ctx->cand_cap), "alloc candidates");
+  if (timing) cudaEventRecord(ctx->ev[2], s);
+
+  // ---- A3b/A4/A5: replay ---------------------------------------------------------
+  ReplayParams rp{};
+  rp.part_ev = ctx->part_ev.p; rp.part_off = ctx->part_off.p; rp.n_chunks = n_chunks;
+  rp.n_buckets = ctx->n_buckets; rp.bucket_bits = ctx->bucket_bits; rp.n_words = ctx->n_words;
+  rp.shadow = ctx->shadow; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
+  rp.cand = ctx->cand.p; rp.cand_cap = ctx->cand_cap; rp.st = ctx->dstats.p;
+  int n_ctas = std::min<int>((int)ctx->n_buckets, ctx->n_sms * 2);
+  CK(launch_replay(rp, std::max(n_ctas, 1), s), "k_replay");
+  launches += 1;
+  if (timing) cudaEventRecord(ctx->ev[3], s);
+  CK(cudaMemcpyAsync(&hst, ctx->dstats.p, sizeof(hst), cudaMemcpyDeviceToHost, s), "stats d2h");
+  CK(cudaStreamSynchronize(s), "replay sync");
+  const uint64_t n_vsm = hst.n_cand;                 // exact: VSM candidates are unique
+  uint64_t kept_vsm = std::min(n_vsm, ctx->cand_cap);
+  S.max_bucket_events = hst.max_bucket_events;
+
+  // ---- A6: MIR join ---------------------------------------------------------------
+  uint64_t n_mir = 0;
+  if (!plan.mir.empty()) {
+    MirPlanH& M = plan.mir;
+    uint64_t hcap = 1;
+    while (hcap < 2 * (2 * M.n_ins_pos + 1)) hcap <<= 1;
+    CK(ctx->hkeys.ensure(hcap), "alloc hash");
+    CK(ctx->hvals.ensure(hcap), "alloc hash");
+    CK(upload(ctx->m_ins_lo, M.ins_lo, s), "mir"); CK(upload(ctx->m_ins_cum, M.ins_cum, s), "mir");
+    CK(upload(ctx->m_ins_inst, M.ins_inst, s), "mir"); CK(upload(ctx->m_qry_lo, M.qry_lo, s), "mir");
+    CK(upload(ctx->m_qry_cum, M.qry_cum, s), "mir"); CK(upload(ctx->m_qry_open_start, M.qry_open_start, s), "mir");
+    CK(upload(ctx->m_open_list, M.open_list, s), "mir"); CK(upload(ctx->m_own_start, M.own_start, s), "mir");
+    CK(upload(ctx->m_win_start, M.win_start, s), "mir"); CK(upload(ctx->m_own, M.own_ops, s), "mir");
+    CK(upload(ctx->m_win, M.win_ops, s), "mir"); CK(upload(ctx->m_rr, M.rr, s), "mir");
+    CK(upload(ctx->m_rr_cum, M.rr_cum, s), "mir");
+    for (int attempt = 0; attempt < 2; ++attempt) {
+      CK(cudaMemsetAsync(ctx->hkeys.p, 0, hcap * sizeof(unsigned long long), s), "hash clear");
+      CK(cudaMemsetAsync(ctx->hvals.p, 0, hcap * sizeof(uint32_t), s), "hash clear");
+      CK(cudaMemsetAsync(&ctx->dstats.p->n_mir_cand, 0, sizeof(unsigned long long), s), "mir count");
+      MirParams mp{};
+      mp.ev = ev; mp.base_word = ctx->base_word; mp.n_words = ctx->n_words;
+      mp.ins_lo = ctx->m_ins_lo.p; mp.ins_cum = ctx->m_ins_cum.p; mp.ins_inst = ctx->m_ins_inst.p;
+      mp.n_ins = (uint32_t)M.ins_lo.size();
+      mp.qry_lo = ctx->m_qry_lo.p; mp.qry_cum = ctx->m_qry_cum.p; mp.qry_open_start = ctx->m_qry_open_start.p;
+      mp.n_qry = (uint32_t)M.qry_lo.size(); mp.open_list = ctx->m_open_list.p;
+      mp.own_start = ctx->m_own_start.p; mp.own_ops = ctx->m_own.p;
+      mp.win_start = ctx->m_win_start.p; mp.win_ops = ctx->m_win.p;
+      mp.hkeys = ctx->hkeys.p; mp.hvals = ctx->hvals.p; mp.hmask = hcap - 1;
+      mp.rr = ctx->m_rr.p; mp.rr_cum = ctx->m_rr_cum.p; mp.n_rr = (uint32_t)M.rr.size();
+      mp.cand = ctx->cand.p + kept_vsm; mp.cand_cap = ctx->cand.cap - kept_vsm; mp.st = ctx->dstats.p;
+      CK(launch_mir(mp, M.n_ins_pos, M.n_qry_pos, M.n_rr_words, s, &launches), "k_mir");
+      unsigned long long c = 0;
+      CK(cudaMemcpyAsync(&c, &ctx->dstats.p->n_mir_cand, sizeof(c), cudaMemcpyDeviceToHost, s), "mir d2h");
+      CK(cudaStreamSynchronize(s), "mir sync");
+      n_mir = c;
+      if (kept_vsm + n_mir <= ctx->cand.cap) break;
+      // MIR kernels only read: grow and run them again
+      DevBuf<uint4> bigger;
+      CK(bigger.ensure(kept_vsm + n_mir), "grow candidates");
+      if (kept_vsm) CK(cudaMemcpyAsync(bigger.p, ctx->cand.p, kept_vsm * 16, cudaMemcpyDeviceToDevice, s), "copy cand");
+      CK(cudaStreamSynchronize(s), "copy sync");
+      ctx->cand.release();
+      ctx->cand = bigger;
+    }
+  }
+  if (timing) cudaEventRecord(ctx->ev[4], s);
+
+  // ---- canonical order + unique ---------------------------------------------------
+  const uint64_t n_cand = kept_vsm + n_mir;
+  CK(ctx->cand_tmp.ensure(std::max<uint64_t>(n_cand, 1)), "alloc cand tmp");
+  CK(ctx->reports.ensure(std::max<uint64_t>(n_cand, 1)), "alloc reports");
+  uint64_t nblk = (n_cand + 4095) / 4096;
+  CK(ctx->blk.ensure(std::max<uint64_t>(nblk * 256, 1)), "alloc blk");
+  CompactParams cp{};
+  cp.cand = ctx->cand.p; cp.n_cand = n_cand; cp.tmp = ctx->cand_tmp.p; cp.blk = ctx->blk.p;
+  cp.blk_cap = ctx->blk.cap; cp.base_word = ctx->base_word;
+  int wb = 1; while (wb < 64 && (ctx->n_words - 1) >> wb) ++wb;
+  int pb = 1; while (pb < 32 && (n ? (n - 1) >> pb : 0)) ++pb;
+  cp.word_bits = wb; cp.pos_bits = pb;
+  cp.dedup_first = (ctx->cfg.flags & ARB_F_DEDUP_FIRST) ? 1 : 0;
+  cp.gidx = gidx; cp.index_base = index_base;
+  cp.out = ctx->reports.p; cp.n_out = ctx->dcount.p;
+  CK(launch_compact(cp, s, &launches), "compact");
+  unsigned long long cnt4[4] = {0, 0, 0, 0};
+  CK(cudaMemcpyAsync(cnt4, ctx->dcount.p, sizeof(cnt4), cudaMemcpyDeviceToHost, s), "count d2h");
+  if (timing) cudaEventRecord(ctx->ev[5], s);
+  CK(cudaStreamSynchronize(s), "compact sync");
+  const uint64_t n_out = cnt4[0];
+  ctx->n_stored = n_out;
+  for (int k = 1; k < 4; ++k) S.reports_by_kind[k] = cnt4[k];
+  // dropped VSM candidates are unique and distinct from every retained one
+  ctx->n_reports = n_out + (n_vsm - kept_vsm);
+  int rc = n_vsm > kept_vsm ? ARB_TRUNCATED : ARB_OK;
+  if (rc == ARB_TRUNCATED) ctx->err = "report candidates exceeded report_capacity";
+
+  // ---- A7: multi-GPU count exchange ----------------------------------------------
+  uint64_t offset = 0;
+  if (ctx->cfg.world > 1) {
+    uint64_t mine = ctx->n_reports;
+    CK(cudaMemcpyAsync(ctx->counts.p + ctx->cfg.world, &mine, 8, cudaMemcpyHostToDevice, s), "counts");
+    if (ctx->nccl_allgather(ctx->counts.p + ctx->cfg.world, ctx->counts.p, 1, kNcclUint64, ctx->comm, s) != 0)
+      return fail(ctx, ARB_ECUDA, "ncclAllGather failed");
+    std::vector<uint64_t> all(ctx->cfg.world);
+    CK(cudaMemcpyAsync(all.data(), ctx->counts.p, 8 * ctx->cfg.world, cudaMemcpyDeviceToHost, s), "counts d2h");
+    CK(cudaStreamSynchronize(s), "counts sync");
+    for (int r = 0; r < ctx->cfg.rank; ++r) offset += all[r];
+    launches += 1;
+  }
+  if (timing) {
+    cudaEventRecord(ctx->ev[6], s);
+    cudaEventSynchronize(ctx->ev[6]);
+    float ms;
+    cudaEventElapsedTime(&ms, ctx->ev[0], ctx->ev[1]); S.ms_partition = ms;
+    cudaEventElapsedTime(&ms, ctx->ev[1], ctx->ev[2]); S.ms_control = ms;
+    cudaEventElapsedTime(&ms, ctx->ev[2], ctx->ev[3]); S.ms_replay = ms;
+    cudaEventElapsedTime(&ms, ctx->ev[3], ctx->ev[4]); S.ms_mir = ms;
+    cudaEventElapsedTime(&ms, ctx->ev[4], ctx->ev[5]); S.ms_reports = ms;
+    cudaEventElapsedTime(&ms, ctx->ev[0], ctx->ev[6]); S.ms_total = ms;
+  }
+  ctx->map.swap(map);
+  ctx->next_index += n;
+  ctx->flushed = true;
+  S.reports = ctx->n_reports;
+  S.kernel_launches = launches;
+  S.total_records += n;
+  S.total_word_events += S.access_words + S.range_words;
+  S.total_reports += ctx->n_reports;
+  S.flushes += 1;
+  reset_batch(ctx);
+  if (n_reports_local) *n_reports_local = ctx->n_reports;
+  if (report_offset_global) *report_offset_global = offset;
+  return rc;
+}
+
+extern "C" int arb_get_reports(arb_ctx ctx, arb_report* out, uint64_t cap, uint64_t* n_written, int out_on_device) {
+  if (!ctx) return ARB_EINVAL;
+  if (!ctx->flushed) return fail(ctx, ARB_ESTATE, "no flush yet");
+  uint64_t k = std::min(cap, ctx->n_stored);
+  if (k) {
+    if (!out) return fail(ctx, ARB_EINVAL, "null output");
+    cudaError_t e = cudaMemcpy(out, ctx->reports.p, k * sizeof(arb_report),
+                               out_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "get_reports");
+  }
+  if (n_written) *n_written = k;
+  return cap < ctx->n_reports ? ARB_TRUNCATED : ARB_OK;
+}
+
+extern "C" int arb_get_shadow(arb_ctx ctx, uint64_t word_lo, uint64_t n, uint8_t* out, int out_on_device) {
+  if (!ctx) return ARB_EINVAL;
+  if (word_lo < ctx->base_word || word_lo + n > ctx->base_word + ctx->n_words || (n && !out))
+    return fail(ctx, ARB_EINVAL, "shadow range outside the tracked range");
+  if (!n) return ARB_OK;
+  cudaError_t e = cudaMemcpy(out, ctx->shadow + (word_lo - ctx->base_word), n,
+                             out_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return cuda_fail(ctx, e, "get_shadow");
+  return ARB_OK;
+}
+
+extern "C" int arb_get_stats(arb_ctx ctx, arb_stats* out) {
+  if (!ctx || !out) return ARB_EINVAL;
+  *out = ctx->stats;
+  return ARB_OK;
+}

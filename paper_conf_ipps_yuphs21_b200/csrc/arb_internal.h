@@ -1,0 +1,142 @@
+// arb_internal.h — internal declarations of libarbalest (product path).
+// Nothing here is shared with oracle/ (DESIGN.md §4 keeps the two independent).
+#pragma once
+#include <cstdint>
+#include <cstddef>
+#include <cuda_runtime.h>
+
+namespace arb {
+
+// ---- trace format ------------------------------------------
+constexpr uint64_t kMask48 = (1ull << 48) - 1;
+enum Op : uint32_t { OP_RH = 0, OP_WH = 1, OP_RT = 2, OP_WT = 3,
+                     OP_MAP_ENTER = 8, OP_MAP_EXIT = 9, OP_UPDATE = 10,
+                     OP_TASK_BEGIN = 12, OP_TASK_END = 13, OP_SYNC = 14 };
+enum MapType : uint32_t { MT_TO = 0, MT_FROM = 1, MT_TOFROM = 2, MT_ALLOC = 3,
+                          MT_RELEASE = 4, MT_DELETE = 5 };
+constexpr uint32_t kSyncAll = 0xFFFFu;
+
+// ---- VSM bits (Table II) ----------------------------------------
+constexpr uint32_t kOVv = 1, kCVv = 2, kOVi = 4, kCVi = 8;
+
+// A transition function of the VSM in "selector" form: output bit j of the
+// 4-bit state is taken from source sel_j (0..3 = input bit, 4 = constant 0,
+// 5 = constant 1); 3 bits per output bit.  Every transition of P:255-261 is
+// a set-constant or copy-a-bit map, so the form is closed under composition.
+using Sel = uint32_t;
+constexpr Sel sel_make(uint32_t s0, uint32_t s1, uint32_t s2, uint32_t s3) {
+  return s0 | (s1 << 3) | (s2 << 6) | (s3 << 9);
+}
+constexpr Sel kSelId    = sel_make(0, 1, 2, 3);
+constexpr Sel kSelUPT   = sel_make(0, 0, 2, 2);   // CV takes OV's validity and init (update_target)
+constexpr Sel kSelUPH   = sel_make(1, 1, 3, 3);   // OV takes CV's (update_host)
+constexpr Sel kSelALLOC = sel_make(0, 4, 2, 4);   // fresh CV: not valid, not initialised
+constexpr Sel kSelREL   = sel_make(0, 4, 2, 4);   // released CV: same bits as allocate
+
+// ---- compact event (partition output, 8 B) ---------------------------------
+// x: [0,30) word offset inside the address bucket | [30,32) access op (RH/WH/RT/WT)
+// y: record position inside the batch (< 2^30)
+constexpr uint32_t kMaxBatchRecords = 1u << 30;
+
+// ---- partition geometry ----------------------------------------------------
+constexpr int kPartThreads = 512;
+constexpr int kPartWarps = kPartThreads / 32;
+constexpr int kChunkRecords = 4096;                 // records per chunk (one CTA)
+constexpr int kChunkCap = 2 * kChunkRecords;        // events per chunk (<= 2 words per access)
+constexpr int kMaxBuckets = 1024;
+
+// ---- replay geometry -------------------------------------------------------
+constexpr int kReplayThreads = 512;
+constexpr int kReplayItems = 8;
+constexpr int kStep = kReplayThreads * kReplayItems;  // events per step
+
+// device-side counters and error flags of one flush
+struct DevStats {
+  unsigned long long access_words;    // tracked access word-events
+  unsigned long long ignored_words;   // access word-ops outside the tracked range
+  unsigned long long n_ctl;           // control records seen
+  unsigned long long err_pos;         // first malformed record (UINT64_MAX = none)
+  unsigned long long n_cand;          // report candidates produced (may exceed capacity)
+  unsigned long long work;            // replay work counter
+  unsigned long long max_bucket_events;
+  unsigned long long range_words_applied;
+  unsigned long long n_mir_cand;
+  unsigned long long pad[7];
+};
+
+// control record extracted by the partition kernel
+struct CtlRec { uint64_t pos, w0, w1; };
+
+// a resolved range op restricted to one address bucket
+struct BucketOp {
+  uint32_t pos;      // record position in the batch
+  uint32_t sel;      // transition function (selector form)
+  uint64_t lo, hi;   // word range [lo, hi) relative to the tracked base
+};
+
+// a range op for the MIR join (absolute relative words, instance of its block)
+struct RangeRef { uint64_t lo, hi; uint32_t pos; uint32_t inst; };
+
+struct PartParams {
+  const uint4* ev; uint64_t n;            // batch records
+  uint64_t base_word, n_words;            // tracked words [base_word, base_word + n_words)
+  uint32_t bucket_bits, n_buckets;
+  uint32_t n_chunks;
+  uint2* part_ev;                         // [n_chunks][kChunkCap]
+  uint16_t* part_off;                     // [n_buckets + 1][n_chunks] start of bucket in chunk
+  CtlRec* ctl; uint64_t ctl_cap;
+  DevStats* st;
+};
+
+struct ReplayParams {
+  const uint2* part_ev; const uint16_t* part_off;
+  uint32_t n_chunks, n_buckets, bucket_bits;
+  uint64_t n_words;
+  uint8_t* shadow;                        // n_words bytes
+  const uint32_t* ops_start;              // [n_buckets + 1]
+  const BucketOp* ops;
+  uint4* cand; uint64_t cand_cap;         // report candidates {word lo, word hi, pos, kind}
+  DevStats* st;
+};
+
+struct MirParams {
+  const uint4* ev;                         // batch records
+  uint64_t base_word, n_words;
+  // position ranges to insert (racy task blocks) / query (windows)
+  const uint64_t* ins_lo; const uint64_t* ins_cum; const uint32_t* ins_inst; uint32_t n_ins;
+  const uint64_t* qry_lo; const uint64_t* qry_cum; const uint32_t* qry_open_start; uint32_t n_qry;
+  const uint32_t* open_list;                // instances open in each query segment
+  // per racy instance (dense index): own range ops and window range ops
+  const uint32_t* own_start; const RangeRef* own_ops;
+  const uint32_t* win_start; const RangeRef* win_ops;
+  const uint32_t* inst_dense;               // instance -> dense index (or 0xFFFFFFFF)
+  // hash table (word, instance) -> write flag
+  unsigned long long* hkeys; uint32_t* hvals; uint64_t hmask;
+  // (ii) range-vs-range emission list
+  const RangeRef* rr; const uint64_t* rr_cum; uint32_t n_rr;
+  uint4* cand; uint64_t cand_cap;
+  DevStats* st;
+};
+
+// ---- kernel launchers (kernels.cu) -----------------------------------------
+cudaError_t launch_partition(const PartParams& p, cudaStream_t s);
+cudaError_t launch_replay(const ReplayParams& p, int n_ctas, cudaStream_t s);
+cudaError_t launch_mir(const MirParams& p, uint64_t n_ins_pos, uint64_t n_qry_pos, uint64_t n_rr_words,
+                       cudaStream_t s, int* launches);
+// report compaction: sorts candidates, removes duplicates, optional dedup-first,
+// maps positions to global indices and writes arb_report records.
+struct CompactParams {
+  uint4* cand; uint64_t n_cand;           // in/out scratch
+  uint4* tmp;                             // same size scratch
+  uint32_t* blk; uint64_t blk_cap;        // block counters scratch
+  uint64_t base_word;
+  int word_bits, pos_bits;
+  int dedup_first;
+  const uint64_t* gidx;                   // device global index per batch position, or null
+  uint64_t index_base;                    // used when gidx is null
+  uint4* out;                             // arb_report output (w0 lo/hi, w1 lo/hi)
+  unsigned long long* n_out;              // device count
+};
+cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches);
+
+}  // namespace arb

@@ -1,0 +1,231 @@
+// control.cpp — host control plane (see control.h).
+#include "control.h"
+#include <algorithm>
+#include <set>
+
+namespace arb {
+
+namespace {
+
+// 1 = [lo,hi) contained in an entry (it = entry), 0 = disjoint from every
+// entry, -1 = partial overlap (reading Z6).
+int map_find(MapTable& m, uint64_t lo, uint64_t hi, MapTable::iterator& it) {
+  auto nx = m.upper_bound(lo);
+  if (nx != m.begin()) {
+    auto pv = std::prev(nx);
+    if (lo < pv->second.hi) {
+      if (hi <= pv->second.hi) { it = pv; return 1; }
+      return -1;
+    }
+  }
+  if (nx != m.end() && nx->first < hi) return -1;
+  return 0;
+}
+
+struct Emitter {
+  uint64_t base_word, n_words;
+  FlushPlan* out;
+  void emit(uint32_t pos, Sel sel, uint64_t byte_lo, uint64_t byte_hi, uint32_t inst) {
+    uint64_t w0 = byte_lo >> 3, w1 = ((byte_hi - 1) >> 3) + 1;    // [w0, w1) absolute
+    uint64_t total = w1 - w0;
+    uint64_t lo = std::max(w0, base_word), hi = std::min(w1, base_word + n_words);
+    if (lo >= hi) { out->ignored_words += total; return; }
+    out->ignored_words += total - (hi - lo);
+    out->range_words += hi - lo;
+    out->range_ops.push_back(RangeOpH{pos, sel, lo - base_word, hi - base_word, inst});
+  }
+};
+
+}  // namespace
+
+void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
+                     uint64_t n_words, uint32_t bucket_bits, uint32_t n_buckets, MapTable& map,
+                     FlushPlan& out) {
+  out = FlushPlan();
+  Emitter em{base_word, n_words, &out};
+  // task instances (1-based; 0 = host)
+  std::vector<uint64_t> t_begin{0}, t_end{0}, t_join{0};
+  std::vector<uint32_t> t_id{0};
+  std::vector<uint32_t> unjoined;
+  uint32_t open = 0;
+  auto fail = [&](int rc, uint64_t pos, const char* why) {
+    out.rc = rc; out.err_pos = pos; out.err = why;
+  };
+  for (const CtlRec& c : ctl) {
+    uint32_t op = (uint32_t)(c.w0 >> 48) & 0xFFu, arg = (uint32_t)(c.w0 >> 56);
+    uint64_t addr = c.w0 & kMask48, len = c.w1 & kMask48;
+    uint32_t tid = (uint32_t)(c.w1 >> 48);
+    uint32_t pos = (uint32_t)c.pos;
+    switch (op) {
+      case OP_TASK_BEGIN:
+        if (open) return fail(ARB_ETRACE, c.pos, "TASK_BEGIN inside an open task block");
+        if (tid == 0 || tid == kSyncAll) return fail(ARB_ETRACE, c.pos, "TASK_BEGIN with task id 0 or 0xFFFF");
+        t_begin.push_back(c.pos); t_end.push_back(0); t_join.push_back(UINT64_MAX); t_id.push_back(tid);
+        open = (uint32_t)(t_begin.size() - 1);
+        break;
+      case OP_TASK_END:
+        if (!open || t_id[open] != tid) return fail(ARB_ETRACE, c.pos, "TASK_END does not match the open block");
+        t_end[open] = c.pos;
+        unjoined.push_back(open);
+        open = 0;
+        break;
+      case OP_SYNC: {
+        if (open) return fail(ARB_ETRACE, c.pos, "SYNC inside a task block");
+        size_t k = 0;
+        for (size_t j = 0; j < unjoined.size(); ++j) {
+          uint32_t q = unjoined[j];
+          if (tid == kSyncAll || t_id[q] == tid) t_join[q] = c.pos;
+          else unjoined[k++] = q;
+        }
+        unjoined.resize(k);
+        break;
+      }
+      case OP_MAP_ENTER: {                          // Table I, entry
+        if (arg > MT_ALLOC || len == 0 || addr + len > (1ull << 48))
+          return fail(ARB_ETRACE, c.pos, "bad MAP_ENTER record");
+        MapTable::iterator it;
+        int f = map_find(map, addr, addr + len, it);
+        if (f < 0) return fail(ARB_EMAP, c.pos, "map clause partially overlaps a present entry");
+        if (f == 1) { it->second.rc += 1; break; }  // exist(CV): ref_count += 1
+        map.emplace(addr, MapEntry{addr + len, 1});  // new CV, ref_count = 1
+        em.emit(pos, kSelALLOC, addr, addr + len, open);
+        if (arg == MT_TO || arg == MT_TOFROM) em.emit(pos, kSelUPT, addr, addr + len, open);
+        break;
+      }
+      case OP_MAP_EXIT: {                           // Table I, exit (reading Z5)
+        if (arg > MT_DELETE || len == 0 || addr + len > (1ull << 48))
+          return fail(ARB_ETRACE, c.pos, "bad MAP_EXIT record");
+        MapTable::iterator it;
+        int f = map_find(map, addr, addr + len, it);
+        if (f < 0) return fail(ARB_EMAP, c.pos, "map clause partially overlaps a present entry");
+        if (f == 0) break;                          // not present: no-op (Z7)
+        if (arg == MT_DELETE) it->second.rc = 0; else it->second.rc -= 1;
+        if (it->second.rc == 0) {
+          if (arg == MT_FROM || arg == MT_TOFROM) em.emit(pos, kSelUPH, addr, addr + len, open);
+          em.emit(pos, kSelREL, it->first, it->second.hi, open);
+          map.erase(it);
+        }
+        break;
+      }
+      case OP_UPDATE: {
+        if (arg > 1 || len == 0 || addr + len > (1ull << 48))
+          return fail(ARB_ETRACE, c.pos, "bad UPDATE record");
+        MapTable::iterator it;
+        int f = map_find(map, addr, addr + len, it);
+        if (f < 0) return fail(ARB_EMAP, c.pos, "target update partially overlaps a present entry");
+        if (f == 0) break;                          // not present: no-op (Z7)
+        em.emit(pos, arg == 0 ? kSelUPT : kSelUPH, addr, addr + len, open);
+        break;
+      }
+      default:
+        return fail(ARB_ETRACE, c.pos, "unknown control op");
+    }
+  }
+  if (open) return fail(ARB_EOPEN, n_records, "a task block is still open at the end of the flush");
+  const uint32_t ninst = (uint32_t)t_begin.size() - 1;
+  out.tasks = ninst;
+  for (uint32_t q = 1; q <= ninst; ++q)
+    if (t_join[q] == UINT64_MAX) t_join[q] = n_records;   // never joined in this flush
+
+  // ---- per-bucket CSR of range ops (trace order kept inside each bucket) ----
+  out.ops_start.assign(n_buckets + 1, 0);
+  for (const RangeOpH& r : out.range_ops) {
+    uint64_t b0 = r.lo >> bucket_bits, b1 = (r.hi - 1) >> bucket_bits;
+    for (uint64_t b = b0; b <= b1; ++b) out.ops_start[b + 1]++;
+  }
+  for (uint32_t b = 0; b < n_buckets; ++b) out.ops_start[b + 1] += out.ops_start[b];
+  out.ops.resize(out.ops_start[n_buckets]);
+  {
+    std::vector<uint32_t> fill(out.ops_start.begin(), out.ops_start.end() - 1);
+    for (const RangeOpH& r : out.range_ops) {
+      uint64_t b0 = r.lo >> bucket_bits, b1 = (r.hi - 1) >> bucket_bits;
+      for (uint64_t b = b0; b <= b1; ++b) {
+        uint64_t blo = b << bucket_bits, bhi = (b + 1) << bucket_bits;
+        out.ops[fill[b]++] = BucketOp{r.pos, r.sel, std::max(r.lo, blo), std::min(r.hi, bhi)};
+      }
+    }
+  }
+
+  // ---- MIR join plan (Theorem 1) -------------------------------
+  // An instance q is racy if its window (end_q, join_q) holds at least one record.
+  MirPlanH& M = out.mir;
+  std::vector<uint32_t> dense(ninst + 1, 0xFFFFFFFFu);
+  std::vector<uint32_t> racy;
+  for (uint32_t q = 1; q <= ninst; ++q)
+    if (t_join[q] > t_end[q] + 1) { dense[q] = (uint32_t)racy.size(); racy.push_back(q); }
+  M.n_racy = (uint32_t)racy.size();
+  if (racy.empty()) return;
+  // insert ranges: records strictly inside each racy block
+  M.ins_cum.push_back(0);
+  for (uint32_t q : racy) {
+    if (t_end[q] > t_begin[q] + 1) {
+      M.ins_lo.push_back(t_begin[q] + 1);
+      M.ins_inst.push_back(dense[q]);
+      M.ins_cum.push_back(M.ins_cum.back() + (t_end[q] - t_begin[q] - 1));
+    }
+  }
+  M.n_ins_pos = M.ins_cum.back();
+  M.ins_cum.pop_back();
+  // own and window range ops per racy instance
+  M.own_start.assign(racy.size() + 1, 0);
+  M.win_start.assign(racy.size() + 1, 0);
+  std::vector<std::vector<RangeRef>> own(racy.size()), win(racy.size());
+  for (const RangeOpH& r : out.range_ops) {
+    if (r.inst && dense[r.inst] != 0xFFFFFFFFu)
+      own[dense[r.inst]].push_back(RangeRef{r.lo, r.hi, r.pos, r.inst});
+  }
+  for (size_t d = 0; d < racy.size(); ++d) {
+    uint32_t q = racy[d];
+    // range ops are in trace order: binary search the window
+    auto first = std::upper_bound(out.range_ops.begin(), out.range_ops.end(), (uint32_t)t_end[q],
+                                  [](uint32_t p, const RangeOpH& r) { return p < r.pos; });
+    for (auto it = first; it != out.range_ops.end() && it->pos < t_join[q]; ++it)
+      win[d].push_back(RangeRef{it->lo, it->hi, it->pos, it->inst});
+  }
+  for (size_t d = 0; d < racy.size(); ++d) {
+    M.own_start[d + 1] = M.own_start[d] + (uint32_t)own[d].size();
+    M.win_start[d + 1] = M.win_start[d] + (uint32_t)win[d].size();
+    M.own_ops.insert(M.own_ops.end(), own[d].begin(), own[d].end());
+    M.win_ops.insert(M.win_ops.end(), win[d].begin(), win[d].end());
+    // (ii) a window range op against the instance's own range ops
+    for (const RangeRef& r : win[d])
+      for (const RangeRef& a : own[d]) {
+        uint64_t lo = std::max(r.lo, a.lo), hi = std::min(r.hi, a.hi);
+        if (lo < hi) M.rr.push_back(RangeRef{lo, hi, r.pos, 0});
+      }
+  }
+  M.rr_cum.push_back(0);
+  for (const RangeRef& r : M.rr) M.rr_cum.push_back(M.rr_cum.back() + (r.hi - r.lo));
+  M.n_rr_words = M.rr_cum.back();
+  M.rr_cum.pop_back();
+  // query segments: positions covered by at least one window, with the open set
+  std::vector<std::pair<uint64_t, int64_t>> evs;   // (position, +/-(dense+1))
+  for (size_t d = 0; d < racy.size(); ++d) {
+    uint32_t q = racy[d];
+    evs.push_back({t_end[q] + 1, (int64_t)d + 1});
+    evs.push_back({t_join[q], -((int64_t)d + 1)});
+  }
+  std::sort(evs.begin(), evs.end());
+  std::set<uint32_t> active;
+  M.qry_cum.push_back(0);
+  M.qry_open_start.push_back(0);
+  for (size_t k = 0; k < evs.size();) {
+    uint64_t p = evs[k].first;
+    while (k < evs.size() && evs[k].first == p) {
+      if (evs[k].second > 0) active.insert((uint32_t)(evs[k].second - 1));
+      else active.erase((uint32_t)(-evs[k].second - 1));
+      ++k;
+    }
+    if (k < evs.size() && !active.empty() && evs[k].first > p) {
+      uint64_t len = evs[k].first - p;
+      M.qry_lo.push_back(p);
+      M.qry_cum.push_back(M.qry_cum.back() + len);
+      for (uint32_t d : active) M.open_list.push_back(d);
+      M.qry_open_start.push_back((uint32_t)M.open_list.size());
+    }
+  }
+  M.n_qry_pos = M.qry_cum.back();
+  M.qry_cum.pop_back();
+}
+
+}  // namespace arb

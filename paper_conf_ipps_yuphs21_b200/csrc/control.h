@@ -1,0 +1,51 @@
+// control.h — host control plane of libarbalest.
+//
+// Input: the control records of one batch (MAP_ENTER / MAP_EXIT / UPDATE /
+// TASK_BEGIN / TASK_END / SYNC) with their positions, extracted on the device
+// by k_partition.  Output: resolved range ops (Table I),
+// task instances with their joins (Theorem 1, reading Z8),
+// the per-bucket range-op lists consumed by k_replay and the MIR join plan
+// consumed by k_mir_*.  O(C log C) for C control records.
+#pragma once
+#include <cstdint>
+#include <map>
+#include <string>
+#include <vector>
+#include "arb_internal.h"
+#include "arbalest.h"
+
+namespace arb {
+
+struct MapEntry { uint64_t hi; uint64_t rc; };        // keyed by lo (bytes), [lo, hi)
+using MapTable = std::map<uint64_t, MapEntry>;
+
+struct RangeOpH { uint32_t pos; uint32_t sel; uint64_t lo, hi; uint32_t inst; };  // rel words [lo, hi)
+
+struct MirPlanH {
+  std::vector<uint64_t> ins_lo, ins_cum; std::vector<uint32_t> ins_inst;
+  std::vector<uint64_t> qry_lo, qry_cum; std::vector<uint32_t> qry_open_start, open_list;
+  std::vector<uint32_t> own_start, win_start;
+  std::vector<RangeRef> own_ops, win_ops;
+  std::vector<RangeRef> rr; std::vector<uint64_t> rr_cum;
+  uint64_t n_ins_pos = 0, n_qry_pos = 0, n_rr_words = 0;
+  uint32_t n_racy = 0;
+  bool empty() const { return n_ins_pos == 0 && n_qry_pos == 0 && n_rr_words == 0; }
+};
+
+struct FlushPlan {
+  std::vector<RangeOpH> range_ops;       // in trace order
+  std::vector<uint32_t> ops_start;       // per bucket CSR
+  std::vector<BucketOp> ops;
+  MirPlanH mir;
+  uint64_t range_words = 0, ignored_words = 0, tasks = 0;
+  int rc = 0; uint64_t err_pos = 0; std::string err;
+};
+
+// Resolve the control records `ctl` (sorted by position) of a batch of
+// n_records records.  `map` is the persistent mapping table; it is modified in
+// place only on success (the caller passes a copy and commits it).
+void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
+                     uint64_t n_words, uint32_t bucket_bits, uint32_t n_buckets, MapTable& map,
+                     FlushPlan& out);
+
+}  // namespace arb

@@ -1,0 +1,198 @@
+"""GPU parity: libarbalest (through the C ABI) vs the CPU oracle, element by element.
+
+Report sets must be identical triples (word, record, kind) — bit-exact, this is
+integer work — and the final shadow must be identical byte for byte.
+"""
+import numpy as np
+import pytest
+
+from golden_io import load
+from gpu_util import run_gpu
+
+pytestmark = pytest.mark.gpu
+
+
+def check(orc, rec, base, size, **kw):
+    okw = {k: kw.pop(k) for k in ("dedup_first",) if k in kw}
+    exp = orc.replay(rec, base, size, **okw)
+    flags = 1 if okw.get("dedup_first") else 0
+    rc, got, shadow, st = run_gpu(rec, base, size, flags=flags, **kw)
+    assert rc == exp.rc
+    if rc == 0:
+        assert got == exp.triples()
+        assert np.array_equal(shadow, exp.shadow)
+        assert st["access_words"] + st["range_words"] == exp.stats["word_events"]
+    return exp, st
+
+
+@pytest.mark.parametrize("name", ["fig1_n3.trace", "fig2_no_sync.trace", "fig2_sync.trace"])
+@pytest.mark.parametrize("bb", [0, 3])
+def test_golden(orc, name, bb):
+    rec, base, size, expect = load(name)
+    exp, _ = check(orc, rec, base, size, bucket_bits=bb)
+    assert exp.triples() == expect
+
+
+def test_config1(orc):
+    from gen.configs import config1
+    rec, base, size = config1()
+    exp, st = check(orc, rec, base, size)
+    assert len(exp.triples()) == 1024
+    assert st["reports"] == 1024 and st["reports_by_kind"][2] == 1024
+
+
+@pytest.mark.parametrize("bb", [0, 14])
+def test_config2(orc, bb):
+    from gen.configs import config2
+    rec, base, size = config2()
+    check(orc, rec, base, size, bucket_bits=bb)
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_fuzz_small(orc, seed):
+    from gen.fuzz import random_program
+    rec, base, span = random_program(seed)
+    for bb in (0, 2, 5):
+        check(orc, rec, base, span, bucket_bits=bb)
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_fuzz_large_steps(orc, seed):
+    """Buckets with many steps (> 4096 events), range ops cutting steps, ragged tails."""
+    from gen.fuzz import random_program
+    rec, base, span = random_program(1000 + seed, n_arrays=6, array_words=8192, steps=500,
+                                     loop_max=20000)
+    for bb in (0, 11):
+        check(orc, rec, base, span, bucket_bits=bb)
+
+
+def test_hot_word(orc):
+    """One word with ~10^5 events spanning many steps (the bfs `stop` flag shape)."""
+    from gen.trace import MAP, OP, TraceBuilder
+    tb = TraceBuilder()
+    A = 0x8000
+    tb.wh(A)
+    tb.enter(MAP.TO, A, 64)
+    rs = np.random.default_rng(5)
+    ops = rs.choice([OP.RT, OP.WT, OP.RH, OP.WH], size=100000, p=[.4, .2, .3, .1])
+    for chunk in np.array_split(ops, 10):
+        arr = np.zeros((chunk.size, 2), dtype=np.uint64)
+        arr[:, 0] = np.uint64(A) | (chunk.astype(np.uint64) << np.uint64(48))
+        arr[:, 1] = 8
+        tb.add_array(arr)
+        tb.update(0, A, 64)
+    tb.exit(MAP.TOFROM, A, 64)
+    check(orc, tb.array(), A, 64)
+
+
+def test_multi_flush_quiescent(orc):
+    """Flushes cut where no task is open or unjoined give the oracle's whole-trace result."""
+    from gen.configs import config2
+    rec, base, size, inst, spans = config2(reps=2, with_index=True)
+    exp = orc.replay(rec, base, size)
+    cuts = [s[2] for s in spans[1:]][::7]          # pattern boundaries are quiescent
+    rc, got, shadow, st = run_gpu(rec, base, size, flush_points=cuts)
+    # each flush is in canonical order; the union over flushes is the oracle's set
+    assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+    assert st["flushes"] == len(cuts) + 1
+
+
+def test_host_submit_and_global_index(orc):
+    from gen.fuzz import random_program
+    rec, base, span = random_program(77)
+    gi = np.arange(rec.shape[0], dtype=np.uint64) * 3 + 1000
+    exp = orc.replay(rec, base, span, global_index=gi)
+    for host in (True, False):
+        rc, got, shadow, _ = run_gpu(rec, base, span, host=host, global_index=gi)
+        assert rc == 0 and got == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+def test_several_submits_one_flush(orc):
+    import torch
+    from gpu_util import to_device
+    from paper_conf_ipps_yuphs21_b200 import Context, reports_to_triples
+    from gen.fuzz import random_program
+    rec, base, span = random_program(78)
+    exp = orc.replay(rec, base, span)
+    ctx = Context(base, span)
+    k = rec.shape[0] // 3
+    d0, d2 = to_device(rec[:k]), to_device(rec[2 * k:])   # device buffers stay alive until flush
+    ctx.submit_events(d0)
+    ctx.submit_events(np.ascontiguousarray(rec[k:2 * k]))
+    ctx.submit_events(d2)
+    rc, n, _ = ctx.flush()
+    assert reports_to_triples(ctx.get_reports(n)) == exp.triples()
+    assert np.array_equal(ctx.get_shadow(base // 8, span // 8), exp.shadow)
+    ctx.close()
+    torch.cuda.synchronize()
+
+
+def test_dedup_first(orc):
+    from gen.configs import config2
+    rec, base, size = config2(reps=2)
+    check(orc, rec, base, size, dedup_first=True)
+
+
+@pytest.mark.parametrize("bad", ["op", "len", "emap", "eopen", "nested"])
+def test_errors_leave_state_unchanged(orc, bad):
+    from gen.trace import MAP, TraceBuilder
+    from paper_conf_ipps_yuphs21_b200 import Context, reports_to_triples
+    from gpu_util import to_device
+    A = 0x4000
+    good = TraceBuilder()
+    good.wh(A); good.enter(MAP.TO, A, 64); good.wt(A + 8)
+    tb = TraceBuilder()
+    tb.rt(A)
+    if bad == "op":
+        tb._add(7, A, 8)
+    elif bad == "len":
+        tb.rh(A, 0)
+    elif bad == "emap":
+        tb.enter(MAP.TO, A + 32, 64)
+    elif bad == "eopen":
+        tb.task_begin(3); tb.wt(A)
+    elif bad == "nested":
+        tb.task_begin(3); tb.task_begin(4)
+    ctx = Context(A, 256)
+    dg = to_device(good.array())
+    ctx.submit_events(dg)
+    ctx.flush()
+    before = ctx.get_shadow(A // 8, 32).copy()
+    db = to_device(tb.array())
+    ctx.submit_events(db)
+    rc, _, _ = ctx.flush(check=False)
+    whole = np.concatenate([good.array(), tb.array()])
+    assert rc == orc.replay(whole, A, 256).rc
+    assert rc in (-4, -5, -7)
+    assert np.array_equal(ctx.get_shadow(A // 8, 32), before)
+    # the context stays usable: the same good continuation works
+    nxt = TraceBuilder(); nxt.rt(A + 8); nxt.rh(A)
+    dn = to_device(nxt.array())
+    ctx.submit_events(dn)
+    rc, n, _ = ctx.flush()
+    exp = orc.replay(np.concatenate([good.array(), nxt.array()]), A, 256)
+    assert reports_to_triples(ctx.get_reports(n)) == [t for t in exp.triples() if t[1] >= 3]
+    ctx.close()
+
+
+def test_truncation_count_exact(orc):
+    from gen.configs import config1
+    from paper_conf_ipps_yuphs21_b200 import Context, reports_to_triples, ARB_TRUNCATED
+    from gpu_util import to_device
+    rec, base, size = config1()
+    exp = orc.replay(rec, base, size)
+    ctx = Context(base, size, report_capacity=100)
+    dr = to_device(rec)
+    ctx.submit_events(dr)
+    rc, n, _ = ctx.flush()
+    assert rc == ARB_TRUNCATED and n == len(exp.triples()) == 1024
+    got = reports_to_triples(ctx.get_reports(100))
+    assert len(got) == 100 and set(got) <= set(exp.triples())
+    ctx.close()
+
+
+def test_untracked_words_ignored(orc):
+    """Z12: words outside the tracked range are ignored by both sides."""
+    from gen.fuzz import random_program
+    rec, base, span = random_program(91)
+    check(orc, rec, base + 256, span // 2)
