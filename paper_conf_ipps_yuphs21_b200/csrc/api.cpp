@@ -65,7 +65,11 @@ struct Submit { const void* ev; uint64_t n; const uint64_t* gidx; int on_device;
 struct arb_ctx_s {
   arb_config cfg{};
   uint64_t base_word = 0, n_words = 0;
-  uint32_t bucket_bits = 0, n_buckets = 0;
+  uint32_t bucket_bits = 0, n_buckets = 0, coarse_bits = 0, n_bins = 0;
+  std::vector<uint32_t> bin_map, order, hist;
+  std::vector<uint64_t> bucket_start;
+  DevBuf<uint32_t> d_bin_map, d_order, d_hist;
+  DevBuf<uint64_t> d_bucket_start;
   int n_sms = 148;
   uint8_t* shadow = nullptr;
   std::vector<Submit> subs;
@@ -131,18 +135,28 @@ extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
   ctx->cfg = *cfg;
   ctx->base_word = cfg->addr_base >> 3;
   ctx->n_words = cfg->addr_bytes >> 3;
-  // address buckets: <= 1024 buckets, >= 2^12 words each, <= 2^30 words each
+  // Address buckets.  bucket_bits != 0: fixed buckets of 2^bits words (<= 1024
+  // of them).  0: buckets balanced per flush on a sampled address histogram over
+  // <= 2^16 coarse bins (<= 1024 buckets of <= 2^30 words).
+  if (ctx->n_words > (1ull << 38)) { delete ctx; return ARB_EINVAL; }
   uint32_t bits = cfg->bucket_bits;
-  if (bits == 0) {
-    bits = 12;
-    while (bits < 30 && ((ctx->n_words + (1ull << bits) - 1) >> bits) > (uint64_t)kMaxBuckets) ++bits;
-  }
-  if (bits > 30 || ((ctx->n_words + (1ull << bits) - 1) >> bits) > (uint64_t)kMaxBuckets) {
-    delete ctx;
-    return ARB_EINVAL;
+  if (bits) {
+    uint64_t nb = (ctx->n_words + (1ull << bits) - 1) >> bits;
+    if (bits > 30 || nb > (uint64_t)kMaxBuckets) { delete ctx; return ARB_EINVAL; }
+    ctx->coarse_bits = bits;
+    ctx->bin_map.resize(nb);
+    ctx->bucket_start.clear();
+    for (uint64_t b = 0; b < nb; ++b) { ctx->bin_map[b] = (uint32_t)b; ctx->bucket_start.push_back(b << bits); }
+    ctx->bucket_start.push_back(ctx->n_words);
+    ctx->order.resize(nb);
+    for (uint64_t b = 0; b < nb; ++b) ctx->order[b] = (uint32_t)b;
+  } else {
+    uint32_t cb = 0;
+    while (((ctx->n_words + (1ull << cb) - 1) >> cb) > (uint64_t)kMaxCoarseBins) ++cb;
+    ctx->coarse_bits = cb;
   }
   ctx->bucket_bits = bits;
-  ctx->n_buckets = (uint32_t)((ctx->n_words + (1ull << bits) - 1) >> bits);
+  ctx->n_bins = (uint32_t)((ctx->n_words + (1ull << ctx->coarse_bits) - 1) >> ctx->coarse_bits);
   if (cfg->report_capacity) ctx->cand_cap = cfg->report_capacity;
   cudaError_t e = cudaSetDevice(cfg->device);
   if (e != cudaSuccess) { delete ctx; return ARB_ECUDA; }
@@ -185,6 +199,7 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   ctx->m_rr_cum.release(); ctx->m_ins_inst.release(); ctx->m_qry_open_start.release(); ctx->m_open_list.release();
   ctx->m_own_start.release(); ctx->m_win_start.release(); ctx->m_own.release(); ctx->m_win.release();
   ctx->m_rr.release(); ctx->hkeys.release(); ctx->hvals.release(); ctx->counts.release();
+  ctx->d_bin_map.release(); ctx->d_order.release(); ctx->d_hist.release(); ctx->d_bucket_start.release();
   for (auto& e : ctx->ev) if (e) cudaEventDestroy(e);
   if (ctx->nccl_lib) dlclose(ctx->nccl_lib);
   delete ctx;
@@ -278,6 +293,31 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   const uint64_t index_base = ctx->next_index;
 
   if (timing) cudaEventRecord(ctx->ev[0], s);
+  // ---- bucket balancing on a sampled address histogram ------------------------
+  if (ctx->bucket_bits == 0) {
+    CK(ctx->d_hist.ensure(ctx->n_bins), "alloc hist");
+    CK(cudaMemsetAsync(ctx->d_hist.p, 0, ctx->n_bins * sizeof(uint32_t), s), "hist clear");
+    SampleParams sp{};
+    sp.ev = ev; sp.n = n; sp.stride = std::max<uint64_t>(1, n / kSampleCap);
+    sp.base_word = ctx->base_word; sp.n_words = ctx->n_words; sp.coarse_bits = ctx->coarse_bits;
+    sp.hist = ctx->d_hist.p;
+    const uint64_t n_samples = n ? (n + sp.stride - 1) / sp.stride : 0;
+    CK(launch_sample(sp, n_samples, s), "k_sample");
+    launches += n_samples ? 1 : 0;
+    ctx->hist.resize(ctx->n_bins);
+    CK(cudaMemcpyAsync(ctx->hist.data(), ctx->d_hist.p, ctx->n_bins * sizeof(uint32_t), cudaMemcpyDeviceToHost, s),
+       "hist d2h");
+    CK(cudaStreamSynchronize(s), "sample sync");
+    balance_buckets(ctx->hist, ctx->coarse_bits, ctx->n_words, kMaxBuckets, ctx->bin_map, ctx->bucket_start,
+                    ctx->order);
+  }
+  if (ctx->bucket_bits == 0 || ctx->d_bin_map.cap == 0) {
+    CK(upload(ctx->d_bin_map, ctx->bin_map, s), "upload bin map");
+    CK(upload(ctx->d_bucket_start, ctx->bucket_start, s), "upload bucket starts");
+    CK(upload(ctx->d_order, ctx->order, s), "upload order");
+  }
+  ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;
+  S.buckets = ctx->n_buckets;
   // ---- A1/A3a: decode + partition ------------------------------------------
   const uint32_t n_chunks = (uint32_t)((n + kChunkRecords - 1) / kChunkRecords);
   CK(ctx->part_ev.ensure((size_t)std::max<uint32_t>(n_chunks, 1) * kChunkCap), "alloc part_ev");
@@ -289,6 +329,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     hst.err_pos = ~0ull;
     CK(cudaMemcpyAsync(ctx->dstats.p, &hst, sizeof(hst), cudaMemcpyHostToDevice, s), "stats init");
     pp.ev = ev; pp.n = n; pp.base_word = ctx->base_word; pp.n_words = ctx->n_words;
+    pp.coarse_bits = ctx->coarse_bits; pp.bin_map = ctx->d_bin_map.p;
     pp.bucket_bits = ctx->bucket_bits; pp.n_buckets = ctx->n_buckets; pp.n_chunks = n_chunks;
     pp.part_ev = ctx->part_ev.p; pp.part_off = ctx->part_off.p; pp.ctl = ctx->ctl.p; pp.ctl_cap = ctx->ctl_cap;
     pp.st = ctx->dstats.p;
@@ -316,7 +357,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   }
   MapTable map = ctx->map;
   FlushPlan plan;
-  resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_bits, ctx->n_buckets, map, plan);
+  resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_start, map, plan);
   if (plan.rc != 0) {
     reset_batch(ctx);
     return fail(ctx, plan.rc, plan.err + " (batch position " + std::to_string(plan.err_pos) + ")");
@@ -334,6 +375,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   ReplayParams rp{};
   rp.part_ev = ctx->part_ev.p; rp.part_off = ctx->part_off.p; rp.n_chunks = n_chunks;
   rp.n_buckets = ctx->n_buckets; rp.bucket_bits = ctx->bucket_bits; rp.n_words = ctx->n_words;
+  rp.bucket_start = ctx->d_bucket_start.p; rp.order = ctx->d_order.p;
   rp.shadow = ctx->shadow; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
   rp.cand = ctx->cand.p; rp.cand_cap = ctx->cand_cap; rp.st = ctx->dstats.p;
   int n_ctas = std::min<int>((int)ctx->n_buckets, ctx->n_sms * 2);

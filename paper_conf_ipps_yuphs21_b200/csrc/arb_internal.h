@@ -77,9 +77,23 @@ struct BucketOp {
 // a range op for the MIR join (absolute relative words, instance of its block)
 struct RangeRef { uint64_t lo, hi; uint32_t pos; uint32_t inst; };
 
+// Address buckets are contiguous word ranges made of whole "coarse bins" of
+// 2^coarse_bits words.  bin_map[bin] = bucket | (bin - first bin of bucket) << 10,
+// so one lookup gives both the bucket and the word offset inside it.  The map
+// is balanced on a sampled histogram of the batch's access addresses.
+constexpr int kMaxCoarseBins = 1 << 16;
+constexpr uint32_t kSampleCap = 1u << 22;
+
+struct SampleParams {
+  const uint4* ev; uint64_t n; uint64_t stride;   // sample records 0, stride, 2*stride, ...
+  uint64_t base_word, n_words; uint32_t coarse_bits;
+  uint32_t* hist;                                 // [n_bins]
+};
+
 struct PartParams {
   const uint4* ev; uint64_t n;            // batch records
   uint64_t base_word, n_words;            // tracked words [base_word, base_word + n_words)
+  uint32_t coarse_bits; const uint32_t* bin_map;
   uint32_t bucket_bits, n_buckets;
   uint32_t n_chunks;
   uint2* part_ev;                         // [n_chunks][kChunkCap]
@@ -91,6 +105,8 @@ struct PartParams {
 struct ReplayParams {
   const uint2* part_ev; const uint16_t* part_off;
   uint32_t n_chunks, n_buckets, bucket_bits;
+  const uint64_t* bucket_start;           // [n_buckets + 1] first relative word of each bucket
+  const uint32_t* order;                  // buckets in scheduling order (largest first)
   uint64_t n_words;
   uint8_t* shadow;                        // n_words bytes
   const uint32_t* ops_start;              // [n_buckets + 1]
@@ -119,6 +135,7 @@ struct MirParams {
 };
 
 // ---- kernel launchers (kernels.cu) -----------------------------------------
+cudaError_t launch_sample(const SampleParams& p, uint64_t n_samples, cudaStream_t s);
 cudaError_t launch_partition(const PartParams& p, cudaStream_t s);
 cudaError_t launch_replay(const ReplayParams& p, int n_ctas, cudaStream_t s);
 cudaError_t launch_mir(const MirParams& p, uint64_t n_ins_pos, uint64_t n_qry_pos, uint64_t n_rr_words,

@@ -38,9 +38,44 @@ struct Emitter {
 
 }  // namespace
 
+void balance_buckets(const std::vector<uint32_t>& hist, uint32_t coarse_bits, uint64_t n_words,
+                     uint32_t max_buckets, std::vector<uint32_t>& bin_map,
+                     std::vector<uint64_t>& bucket_start, std::vector<uint32_t>& order) {
+  const uint64_t n_bins = hist.size();
+  uint64_t total = 0;
+  for (uint32_t h : hist) total += h;
+  const uint64_t max_span_bins = std::max<uint64_t>(1, (1ull << 30) >> coarse_bits);
+  // span cuts (buckets of <= 2^30 words) are always taken; weight cuts use the
+  // rest of the budget (n_words <= 2^38 keeps the span cuts <= 256)
+  const uint64_t span_reserve = (n_words >> 30) + 2;
+  const uint64_t target = std::max<uint64_t>(1, total / std::max<uint32_t>(1, max_buckets * 3 / 8));
+  bin_map.assign(n_bins, 0);
+  bucket_start.clear();
+  std::vector<uint64_t> weight;
+  uint64_t first = 0, acc = 0;
+  for (uint64_t i = 0; i < n_bins; ++i) {
+    bool full = acc > 0 && acc + hist[i] > target && bucket_start.size() + 1 + span_reserve < max_buckets;
+    bool too_long = i - first >= max_span_bins;
+    if (full || too_long) {
+      bucket_start.push_back(first << coarse_bits);
+      weight.push_back(acc);
+      first = i; acc = 0;
+    }
+    acc += hist[i];
+    bin_map[i] = (uint32_t)bucket_start.size() | (uint32_t)((i - first) << 10);
+  }
+  bucket_start.push_back(first << coarse_bits);
+  weight.push_back(acc);
+  bucket_start.push_back(n_words);
+  order.resize(weight.size());
+  for (uint32_t b = 0; b < order.size(); ++b) order[b] = b;
+  std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return weight[a] > weight[b]; });
+}
+
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
-                     uint64_t n_words, uint32_t bucket_bits, uint32_t n_buckets, MapTable& map,
+                     uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
                      FlushPlan& out) {
+  const uint32_t n_buckets = (uint32_t)bucket_start.size() - 1;
   out = FlushPlan();
   Emitter em{base_word, n_words, &out};
   // task instances (1-based; 0 = host)
@@ -128,22 +163,20 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
     if (t_join[q] == UINT64_MAX) t_join[q] = n_records;   // never joined in this flush
 
   // ---- per-bucket CSR of range ops (trace order kept inside each bucket) ----
+  auto first_bucket = [&](uint64_t w) {   // bucket holding relative word w
+    return (uint32_t)(std::upper_bound(bucket_start.begin(), bucket_start.end() - 1, w) - bucket_start.begin() - 1);
+  };
   out.ops_start.assign(n_buckets + 1, 0);
-  for (const RangeOpH& r : out.range_ops) {
-    uint64_t b0 = r.lo >> bucket_bits, b1 = (r.hi - 1) >> bucket_bits;
-    for (uint64_t b = b0; b <= b1; ++b) out.ops_start[b + 1]++;
-  }
+  for (const RangeOpH& r : out.range_ops)
+    for (uint32_t b = first_bucket(r.lo); b < n_buckets && bucket_start[b] < r.hi; ++b) out.ops_start[b + 1]++;
   for (uint32_t b = 0; b < n_buckets; ++b) out.ops_start[b + 1] += out.ops_start[b];
   out.ops.resize(out.ops_start[n_buckets]);
   {
     std::vector<uint32_t> fill(out.ops_start.begin(), out.ops_start.end() - 1);
-    for (const RangeOpH& r : out.range_ops) {
-      uint64_t b0 = r.lo >> bucket_bits, b1 = (r.hi - 1) >> bucket_bits;
-      for (uint64_t b = b0; b <= b1; ++b) {
-        uint64_t blo = b << bucket_bits, bhi = (b + 1) << bucket_bits;
-        out.ops[fill[b]++] = BucketOp{r.pos, r.sel, std::max(r.lo, blo), std::min(r.hi, bhi)};
-      }
-    }
+    for (const RangeOpH& r : out.range_ops)
+      for (uint32_t b = first_bucket(r.lo); b < n_buckets && bucket_start[b] < r.hi; ++b)
+        out.ops[fill[b]++] = BucketOp{r.pos, r.sel, std::max(r.lo, bucket_start[b]),
+                                      std::min(r.hi, bucket_start[b + 1])};
   }
 
   // ---- MIR join plan (Theorem 1) -------------------------------

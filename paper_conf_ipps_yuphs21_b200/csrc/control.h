@@ -44,8 +44,19 @@ struct FlushPlan {
 // Resolve the control records `ctl` (sorted by position) of a batch of
 // n_records records.  `map` is the persistent mapping table; it is modified in
 // place only on success (the caller passes a copy and commits it).
+// `bucket_start` holds the first relative word of every address bucket plus
+// n_words at the end (ascending).
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
-                     uint64_t n_words, uint32_t bucket_bits, uint32_t n_buckets, MapTable& map,
+                     uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
                      FlushPlan& out);
+
+// Balance address buckets on a sampled histogram of coarse bins: contiguous
+// bins are grouped greedily so that each bucket holds about total/target
+// samples (a bucket spans at most 2^30 words).  Fills bin_map (see
+// arb_internal.h), bucket_start (n_buckets + 1 entries) and a largest-first
+// scheduling order.
+void balance_buckets(const std::vector<uint32_t>& hist, uint32_t coarse_bits, uint64_t n_words,
+                     uint32_t max_buckets, std::vector<uint32_t>& bin_map,
+                     std::vector<uint64_t>& bucket_start, std::vector<uint32_t>& order);
 
 }  // namespace arb

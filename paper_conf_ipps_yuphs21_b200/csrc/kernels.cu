@@ -86,12 +86,14 @@ __device__ __forceinline__ Decoded decode(uint4 r, bool valid, const PartParams&
     uint64_t addr = w0 & kMask48, len = w1 & kMask48;
     if (len < 1 || len > 8 || addr + len > (1ull << 48)) { d.bad = true; return d; }
     uint64_t x0 = addr >> 3, x1 = (addr + len - 1) >> 3;
-    uint32_t bmask = (1u << p.bucket_bits) - 1u;
+    const uint32_t cmask = (1u << p.coarse_bits) - 1u;
     for (uint64_t x = x0; x <= x1; ++x) {
       uint64_t rel = x - p.base_word;
       if (x >= p.base_word && rel < p.n_words) {
-        uint32_t b = (uint32_t)(rel >> p.bucket_bits);
-        uint32_t k = (op << 30) | ((uint32_t)rel & bmask);
+        uint32_t m = __ldg(p.bin_map + (rel >> p.coarse_bits));
+        uint32_t b = m & 1023u;
+        uint32_t off = ((m >> 10) << p.coarse_bits) | ((uint32_t)rel & cmask);
+        uint32_t k = (op << 30) | off;
         if (d.cnt == 0) { d.b0 = b; d.k0 = k; } else { d.b1 = b; d.k1 = k; }
         d.cnt++;
       } else {
@@ -269,6 +271,25 @@ __global__ void __launch_bounds__(kPartThreads, 2) k_partition(PartParams p) {
     if (n_acc) atomicAdd(&p.st->access_words, (unsigned long long)n_acc);
     if (n_ign) atomicAdd(&p.st->ignored_words, (unsigned long long)n_ign);
   }
+}
+
+// Sampled histogram of access addresses over coarse bins (bucket balancing).
+__global__ void k_sample(SampleParams p, uint64_t n_samples) {
+  for (uint64_t k = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; k < n_samples;
+       k += (uint64_t)gridDim.x * blockDim.x) {
+    uint4 r = ld_stream(p.ev + k * p.stride);
+    uint64_t w0 = (uint64_t)r.x | ((uint64_t)r.y << 32);
+    if (((w0 >> 48) & 0xFFu) >= 4) continue;
+    uint64_t rel = ((w0 & kMask48) >> 3) - p.base_word;
+    if ((w0 & kMask48) >> 3 >= p.base_word && rel < p.n_words) atomicAdd(&p.hist[rel >> p.coarse_bits], 1u);
+  }
+}
+
+cudaError_t launch_sample(const SampleParams& p, uint64_t n_samples, cudaStream_t s) {
+  if (!n_samples) return cudaSuccess;
+  uint64_t g = (n_samples + 255) / 256;
+  k_sample<<<(unsigned)(g > 148 * 16 ? 148 * 16 : g), 256, 0, s>>>(p, n_samples);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_partition(const PartParams& p, cudaStream_t s) {
@@ -516,7 +537,7 @@ __device__ void process_step(ReplaySmem& S, const ReplayParams& p, uint32_t m) {
     t = pin; pin = pout; pout = t;
   }
   // blocked arrangement: thread t owns sorted elements [8t, 8t+8)
-  const uint64_t bucket_base = (uint64_t)S.bucket << p.bucket_bits;
+  const uint64_t bucket_base = p.bucket_start[S.bucket];
   uint32_t val[kReplayItems], s0[kReplayItems], key[kReplayItems];
   bool head[kReplayItems];
   uint32_t agg = 0;
@@ -606,7 +627,10 @@ __global__ void __launch_bounds__(kReplayThreads, 1) k_replay(ReplayParams p) {
   ReplaySmem& S = *reinterpret_cast<ReplaySmem*>(smem_raw);
   const uint32_t tid = threadIdx.x;
   for (;;) {
-    if (tid == 0) S.bucket = (uint32_t)atomicAdd(&p.st->work, 1ull);
+    if (tid == 0) {
+      unsigned long long w = atomicAdd(&p.st->work, 1ull);
+      S.bucket = w < p.n_buckets ? p.order[w] : 0xFFFFFFFFu;
+    }
     __syncthreads();
     const uint32_t b = S.bucket;
     if (b >= p.n_buckets) return;
