@@ -107,6 +107,7 @@ typedef struct {
   /* device time of each phase of the last flush in milliseconds (ARB_F_TIMING) */
   double   ms_partition, ms_control, ms_replay, ms_mir, ms_reports, ms_total;
   uint64_t kernel_launches;  /* kernels launched by the last flush                         */
+  double   ms_sample;        /* address sampling + bucket balancing (inside ms_partition)  */
 } arb_stats;
 
 typedef struct arb_ctx_s* arb_ctx;

@@ -311,6 +311,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     balance_buckets(ctx->hist, ctx->coarse_bits, ctx->n_words, kMaxBuckets, ctx->bin_map, ctx->bucket_start,
                     ctx->order);
   }
+  if (timing) cudaEventRecord(ctx->ev[7], s);
   if (ctx->bucket_bits == 0 || ctx->d_bin_map.cap == 0) {
     CK(upload(ctx->d_bin_map, ctx->bin_map, s), "upload bin map");
     CK(upload(ctx->d_bucket_start, ctx->bucket_start, s), "upload bucket starts");
@@ -481,6 +482,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     cudaEventSynchronize(ctx->ev[6]);
     float ms;
     cudaEventElapsedTime(&ms, ctx->ev[0], ctx->ev[1]); S.ms_partition = ms;
+    cudaEventElapsedTime(&ms, ctx->ev[0], ctx->ev[7]); S.ms_sample = ms;
     cudaEventElapsedTime(&ms, ctx->ev[1], ctx->ev[2]); S.ms_control = ms;
     cudaEventElapsedTime(&ms, ctx->ev[2], ctx->ev[3]); S.ms_replay = ms;
     cudaEventElapsedTime(&ms, ctx->ev[3], ctx->ev[4]); S.ms_mir = ms;

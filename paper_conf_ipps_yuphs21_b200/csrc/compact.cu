@@ -1,0 +1,232 @@
+// compact.cu — canonical report order (word, record, kind) + unique:
+// LSD radix sort of the report candidates, then stream compaction.
+#include "kcommon.cuh"
+
+namespace arb {
+
+constexpr int kRsThreads = 512, kRsItems = 8, kRsTile = kRsThreads * kRsItems;
+
+struct RsPass { int field; int shift; int bits; };
+__device__ __forceinline__ uint32_t rs_digit(uint4 c, RsPass ps) {
+  uint32_t f = ps.field == 0 ? c.w : ps.field == 1 ? c.z : ps.field == 2 ? c.x : c.y;
+  return (f >> ps.shift) & ((1u << ps.bits) - 1u);
+}
+
+__global__ void __launch_bounds__(kRsThreads) k_rs_hist(const uint4* in, uint64_t n, RsPass ps, uint32_t* cnt,
+                                                        uint32_t nblk) {
+  __shared__ uint32_t h[256];
+  for (int i = threadIdx.x; i < 256; i += kRsThreads) h[i] = 0;
+  __syncthreads();
+  uint64_t base = (uint64_t)blockIdx.x * kRsTile;
+  for (int j = 0; j < kRsItems; ++j) {
+    uint64_t i = base + (uint64_t)j * kRsThreads + threadIdx.x;
+    if (i < n) atomicAdd(&h[rs_digit(in[i], ps)], 1u);
+  }
+  __syncthreads();
+  for (int d = threadIdx.x; d < 256; d += kRsThreads) cnt[(uint64_t)d * nblk + blockIdx.x] = h[d];
+}
+
+// exclusive scan of n u32 values in place (single CTA)
+__global__ void __launch_bounds__(1024) k_scan_inplace(uint32_t* a, uint64_t n) {
+  __shared__ uint32_t ws[32];
+  __shared__ uint32_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (uint64_t base = 0; base < n; base += 1024) {
+    uint64_t i = base + threadIdx.x;
+    uint32_t v = i < n ? a[i] : 0, incl = v;
+    for (int d = 1; d < 32; d <<= 1) {
+      uint32_t o = __shfl_up_sync(FULL, incl, d);
+      if (lane >= (uint32_t)d) incl += o;
+    }
+    if (lane == 31) ws[warp] = incl;
+    __syncthreads();
+    if (warp == 0) {
+      uint32_t x = ws[lane], xi = x;
+      for (int d = 1; d < 32; d <<= 1) {
+        uint32_t o = __shfl_up_sync(FULL, xi, d);
+        if (lane >= (uint32_t)d) xi += o;
+      }
+      ws[lane] = xi - x;
+    }
+    __syncthreads();
+    uint32_t c = carry;
+    if (i < n) a[i] = c + ws[warp] + incl - v;
+    __syncthreads();
+    if (threadIdx.x == 1023) carry = c + ws[warp] + incl;
+    __syncthreads();
+  }
+}
+
+__global__ void __launch_bounds__(kRsThreads) k_rs_scatter(const uint4* in, uint4* out, uint64_t n, RsPass ps,
+                                                           const uint32_t* cnt, uint32_t nblk) {
+  __shared__ uint16_t hist[kRsThreads / 32][256];
+  __shared__ uint32_t dbase[256];
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  uint32_t* h32 = reinterpret_cast<uint32_t*>(&hist[0][0]);
+  for (uint32_t i = tid; i < (kRsThreads / 32) * 128; i += kRsThreads) h32[i] = 0;
+  __syncthreads();
+  uint64_t base = (uint64_t)blockIdx.x * kRsTile;
+  uint4 c[kRsItems]; uint32_t rk[kRsItems], dg[kRsItems];
+  const uint32_t lt = lanemask_lt();
+  for (int r = 0; r < kRsItems; ++r) {
+    uint64_t i = base + warp * (32 * kRsItems) + r * 32 + lane;
+    bool valid = i < n;
+    c[r] = valid ? in[i] : make_uint4(0, 0, 0, 0);
+    uint32_t d = valid ? rs_digit(c[r], ps) : 0xFFFFu;
+    uint32_t grp = __match_any_sync(FULL, d);
+    uint32_t b = valid ? hist[warp][d] : 0;
+    __syncwarp();
+    if (valid && lane == 31u - __clz(grp)) hist[warp][d] = (uint16_t)(b + __popc(grp));
+    __syncwarp();
+    dg[r] = d; rk[r] = b + __popc(grp & lt);
+  }
+  __syncthreads();
+  if (tid < 256) {
+    uint32_t s = 0;
+    for (int w = 0; w < kRsThreads / 32; ++w) { uint32_t x = hist[w][tid]; hist[w][tid] = (uint16_t)s; s += x; }
+    dbase[tid] = cnt[(uint64_t)tid * nblk + blockIdx.x];
+  }
+  __syncthreads();
+  for (int r = 0; r < kRsItems; ++r) {
+    uint64_t i = base + warp * (32 * kRsItems) + r * 32 + lane;
+    if (i < n) out[dbase[dg[r]] + hist[warp][dg[r]] + rk[r]] = c[r];
+  }
+}
+
+// keep flags: unique (all fields differ from the predecessor), or dedup-first
+// (word, kind differ from the predecessor) for the (word, kind, pos) order.
+__device__ __forceinline__ bool keep_elem(const uint4* a, uint64_t i, int mode) {
+  if (i == 0) return true;
+  uint4 x = a[i], y = a[i - 1];
+  if (mode == 0) return x.x != y.x || x.y != y.y || x.z != y.z || x.w != y.w;
+  return x.x != y.x || x.y != y.y || x.w != y.w;
+}
+__global__ void __launch_bounds__(kRsThreads) k_keep_count(const uint4* a, uint64_t n, int mode, uint32_t* blk) {
+  __shared__ uint32_t red[kRsThreads / 32];
+  uint32_t c = 0;
+  uint64_t base = (uint64_t)blockIdx.x * kRsTile;
+  for (int j = 0; j < kRsItems; ++j) {
+    uint64_t i = base + (uint64_t)threadIdx.x * kRsItems + j;
+    if (i < n) c += keep_elem(a, i, mode);
+  }
+  for (int d = 16; d; d >>= 1) c += __shfl_xor_sync(FULL, c, d);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = c;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t t = 0;
+    for (int w = 0; w < kRsThreads / 32; ++w) t += red[w];
+    blk[blockIdx.x] = t;
+  }
+}
+// write kept elements; final != 0: convert to arb_report records
+__global__ void __launch_bounds__(kRsThreads) k_keep_write(const uint4* a, uint64_t n, int mode, const uint32_t* blk,
+                                                           uint4* out, int final_out, uint64_t base_word,
+                                                           const uint64_t* gidx, uint64_t index_base,
+                                                           unsigned long long* n_out, uint32_t nblk) {
+  __shared__ uint32_t ws[kRsThreads / 32];
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint64_t base = (uint64_t)blockIdx.x * kRsTile;
+  bool kp[kRsItems];
+  uint32_t c = 0;
+  for (int j = 0; j < kRsItems; ++j) {
+    uint64_t i = base + (uint64_t)threadIdx.x * kRsItems + j;
+    kp[j] = i < n && keep_elem(a, i, mode);
+    c += kp[j];
+  }
+  uint32_t incl = c;
+  for (int d = 1; d < 32; d <<= 1) {
+    uint32_t o = __shfl_up_sync(FULL, incl, d);
+    if (lane >= (uint32_t)d) incl += o;
+  }
+  if (lane == 31) ws[warp] = incl;
+  __syncthreads();
+  uint32_t wpre = 0;
+  for (uint32_t w = 0; w < warp; ++w) wpre += ws[w];
+  uint64_t o = blk[blockIdx.x] + wpre + incl - c;
+  for (int j = 0; j < kRsItems; ++j) {
+    uint64_t i = base + (uint64_t)threadIdx.x * kRsItems + j;
+    if (!kp[j]) continue;
+    uint4 x = a[i];
+    if (final_out) {
+      uint64_t word = ((uint64_t)x.x | ((uint64_t)x.y << 32)) + base_word;
+      uint64_t w0 = (word & kMask48) | ((uint64_t)x.w << 48);
+      uint64_t w1 = gidx ? gidx[x.z] : index_base + x.z;
+      out[o] = make_uint4((uint32_t)w0, (uint32_t)(w0 >> 32), (uint32_t)w1, (uint32_t)(w1 >> 32));
+      atomicAdd(&n_out[x.w & 3u], 1ull);   // per-kind counts in n_out[1..3]
+    } else {
+      out[o] = x;
+    }
+    ++o;
+  }
+  if (blockIdx.x == nblk - 1 && threadIdx.x == kRsThreads - 1) *n_out = o;
+}
+
+static cudaError_t radix_sort(uint4*& a, uint4*& b, uint64_t n, const RsPass* passes, int np, uint32_t* cnt,
+                              cudaStream_t s, int* launches) {
+  uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
+  for (int k = 0; k < np; ++k) {
+    k_rs_hist<<<nblk, kRsThreads, 0, s>>>(a, n, passes[k], cnt, nblk);
+    k_scan_inplace<<<1, 1024, 0, s>>>(cnt, (uint64_t)nblk * 256);
+    k_rs_scatter<<<nblk, kRsThreads, 0, s>>>(a, b, n, passes[k], cnt, nblk);
+    *launches += 3;
+    uint4* t = a; a = b; b = t;
+  }
+  return cudaGetLastError();
+}
+
+static int add_field_passes(RsPass* ps, int np, int field, int bits) {
+  for (int sh = 0; sh < bits; sh += 8) ps[np++] = RsPass{field, sh, bits - sh < 8 ? bits - sh : 8};
+  return np;
+}
+
+cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches) {
+  cudaMemsetAsync(p.n_out, 0, 4 * sizeof(unsigned long long), s);
+  if (p.n_cand == 0) return cudaGetLastError();
+  uint4* a = p.cand;
+  uint4* b = p.tmp;
+  uint64_t n = p.n_cand;
+  RsPass ps[24];
+  int np = 0;
+  int wb_lo = p.word_bits > 32 ? 32 : p.word_bits, wb_hi = p.word_bits > 32 ? p.word_bits - 32 : 0;
+  cudaError_t e;
+  if (p.dedup_first) {
+    // (word, kind, pos): keep the first of each (word, kind)
+    np = add_field_passes(ps, np, 1, p.pos_bits);
+    np = add_field_passes(ps, np, 0, 2);
+    np = add_field_passes(ps, np, 2, wb_lo);
+    np = add_field_passes(ps, np, 3, wb_hi);
+    if ((e = radix_sort(a, b, n, ps, np, p.blk, s, launches)) != cudaSuccess) return e;
+    uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
+    k_keep_count<<<nblk, kRsThreads, 0, s>>>(a, n, 1, p.blk);
+    k_scan_inplace<<<1, 1024, 0, s>>>(p.blk, nblk);
+    k_keep_write<<<nblk, kRsThreads, 0, s>>>(a, n, 1, p.blk, b, 0, 0, nullptr, 0, p.n_out, nblk);
+    *launches += 3;
+    // the number kept is needed on the host side to continue; read it back
+    unsigned long long kept = 0;
+    cudaMemcpyAsync(&kept, p.n_out, sizeof(kept), cudaMemcpyDeviceToHost, s);
+    cudaStreamSynchronize(s);
+    n = kept;
+    uint4* t = a; a = b; b = t;
+    np = 0;
+  }
+  np = add_field_passes(ps, np, 0, 2);
+  np = add_field_passes(ps, np, 1, p.pos_bits);
+  np = add_field_passes(ps, np, 2, wb_lo);
+  np = add_field_passes(ps, np, 3, wb_hi);
+  if ((e = radix_sort(a, b, n, ps, np, p.blk, s, launches)) != cudaSuccess) return e;
+  uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
+  if (n == 0) {
+    cudaMemsetAsync(p.n_out, 0, 4 * sizeof(unsigned long long), s);
+    return cudaGetLastError();
+  }
+  k_keep_count<<<nblk, kRsThreads, 0, s>>>(a, n, 0, p.blk);
+  k_scan_inplace<<<1, 1024, 0, s>>>(p.blk, nblk);
+  k_keep_write<<<nblk, kRsThreads, 0, s>>>(a, n, 0, p.blk, p.out, 1, p.base_word, p.gidx, p.index_base,
+                                           p.n_out, nblk);
+  *launches += 3;
+  return cudaGetLastError();
+}
+
+}  // namespace arb

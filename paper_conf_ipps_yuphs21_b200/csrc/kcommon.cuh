@@ -1,0 +1,58 @@
+// kcommon.cuh — device helpers shared by the libarbalest kernels.
+#pragma once
+#include "arb_internal.h"
+
+namespace arb {
+
+#define FULL 0xFFFFFFFFu
+
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
+// streaming (evict-first) loads of data read exactly once
+__device__ __forceinline__ uint4 ld_stream(const uint4* p) {
+  uint4 r;
+  asm volatile("ld.global.cs.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ uint2 ld_stream2(const uint2* p) {
+  uint2 r;
+  asm volatile("ld.global.cs.v2.u32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
+  return r;
+}
+
+// ---- selector-form transition functions (see arb_internal.h) -------------
+// x holds 4 states, one per byte (low nibble); returns the 4 images.
+__device__ __forceinline__ uint32_t sel_apply4(Sel s, uint32_t x) {
+  uint32_t out = 0;
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    uint32_t src = (s >> (3 * j)) & 7u;
+    uint32_t v = src < 4 ? (x >> src) & 0x01010101u : (src == 5 ? 0x01010101u : 0u);
+    out |= v << j;
+  }
+  return out;
+}
+__device__ __forceinline__ Sel sel_compose(Sel g, Sel f) {  // g after f
+  Sel r = 0;
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    uint32_t gj = (g >> (3 * j)) & 7u;
+    uint32_t v = gj < 4 ? (f >> (3 * gj)) & 7u : gj;
+    r |= v << (3 * j);
+  }
+  return r;
+}
+
+// ---- the two access writes of the VSM on a 4-bit state --------
+__device__ __forceinline__ uint32_t vsm_write(uint32_t kind, uint32_t s) {
+  // kind 1 = write_host: OV holds the latest value, CV does not, OV initialised
+  // kind 2 = write_target: CV holds the latest value, OV does not, CV initialised
+  return kind == 1 ? ((s & kCVi) | kOVv | kOVi) : ((s & kOVi) | kCVv | kCVi);
+}
+
+}  // namespace arb

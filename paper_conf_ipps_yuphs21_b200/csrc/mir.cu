@@ -1,0 +1,113 @@
+// mir.cu — MIR join kernels (Theorem 1; reading Z10 of DESIGN.md).
+#include "kcommon.cuh"
+
+namespace arb {
+
+__device__ __forceinline__ uint32_t seg_of(const uint64_t* cum, uint32_t n, uint64_t g) {
+  uint32_t a = 0, z = n;          // last cum[a] <= g
+  while (z - a > 1) { uint32_t mid = (a + z) >> 1; if (cum[mid] <= g) a = mid; else z = mid; }
+  return a;
+}
+__device__ __forceinline__ uint64_t hslot(unsigned long long key, uint64_t mask) {
+  unsigned long long h = key * 0x9E3779B97F4A7C15ull;
+  return (h ^ (h >> 29)) & mask;
+}
+__device__ __forceinline__ void emit_mir(const MirParams& p, uint64_t word_rel, uint32_t pos) {
+  unsigned long long slot = atomicAdd(&p.st->n_mir_cand, 1ull);
+  if (slot < p.cand_cap) p.cand[slot] = make_uint4((uint32_t)word_rel, (uint32_t)(word_rel >> 32), pos, 3u);
+}
+// words of an access record inside the tracked range: returns count (0..2)
+__device__ __forceinline__ int access_words(const MirParams& p, uint4 r, uint64_t* w, uint32_t* op) {
+  uint64_t w0 = (uint64_t)r.x | ((uint64_t)r.y << 32), w1 = (uint64_t)r.z | ((uint64_t)r.w << 32);
+  *op = (uint32_t)(w0 >> 48) & 0xFFu;
+  if (*op >= 4) return 0;
+  uint64_t addr = w0 & kMask48, len = w1 & kMask48;
+  int n = 0;
+  for (uint64_t x = addr >> 3; x <= (addr + len - 1) >> 3; ++x) {
+    if (x >= p.base_word && x - p.base_word < p.n_words) w[n++] = x - p.base_word;
+  }
+  return n;
+}
+
+// (iv) insert the access word-ops of racy task blocks; (iii) range ops in the
+// instance's window that cover an inserted word race with it.
+__global__ void k_mir_insert(MirParams p, uint64_t n_pos) {
+  for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < n_pos;
+       g += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t s = seg_of(p.ins_cum, p.n_ins, g);
+    uint64_t pos = p.ins_lo[s] + (g - p.ins_cum[s]);
+    uint32_t qd = p.ins_inst[s];
+    uint4 r = p.ev[pos];
+    uint64_t w[2]; uint32_t op;
+    int n = access_words(p, r, w, &op);
+    for (int k = 0; k < n; ++k) {
+      unsigned long long key = ((unsigned long long)w[k] << 20) | (qd + 1);
+      uint64_t h = hslot(key, p.hmask);
+      for (;;) {
+        unsigned long long old = atomicCAS(&p.hkeys[h], 0ull, key);
+        if (old == 0ull || old == key) break;
+        h = (h + 1) & p.hmask;
+      }
+      if (op == OP_WH || op == OP_WT) atomicOr(&p.hvals[h], 1u);
+      for (uint32_t j = p.win_start[qd]; j < p.win_start[qd + 1]; ++j) {
+        RangeRef rr = p.win_ops[j];
+        if (w[k] >= rr.lo && w[k] < rr.hi) emit_mir(p, w[k], rr.pos);
+      }
+    }
+  }
+}
+
+// (iv) + (i): access ops inside race windows against the open instances'
+// access ops (hash) and range ops (lists).
+__global__ void k_mir_query(MirParams p, uint64_t n_pos) {
+  for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < n_pos;
+       g += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t s = seg_of(p.qry_cum, p.n_qry, g);
+    uint64_t pos = p.qry_lo[s] + (g - p.qry_cum[s]);
+    uint4 r = p.ev[pos];
+    uint64_t w[2]; uint32_t op;
+    int n = access_words(p, r, w, &op);
+    bool is_write = op == OP_WH || op == OP_WT;
+    for (int k = 0; k < n; ++k) {
+      bool mir = false;
+      for (uint32_t j = p.qry_open_start[s]; j < p.qry_open_start[s + 1] && !mir; ++j) {
+        uint32_t qd = p.open_list[j];
+        unsigned long long key = ((unsigned long long)w[k] << 20) | (qd + 1);
+        uint64_t h = hslot(key, p.hmask);
+        for (;;) {
+          unsigned long long kk = p.hkeys[h];
+          if (kk == 0ull) break;
+          if (kk == key) { if (is_write || (p.hvals[h] & 1u)) mir = true; break; }
+          h = (h + 1) & p.hmask;
+        }
+        for (uint32_t t = p.own_start[qd]; t < p.own_start[qd + 1] && !mir; ++t) {
+          RangeRef rr = p.own_ops[t];
+          if (w[k] >= rr.lo && w[k] < rr.hi) mir = true;   // range ops are write-class
+        }
+      }
+      if (mir) emit_mir(p, w[k], (uint32_t)pos);
+    }
+  }
+}
+
+// (ii) range op in a window vs the instance's own range ops: every word of
+// the overlap (precomputed on the host) races.
+__global__ void k_mir_ranges(MirParams p, uint64_t n_words) {
+  for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < n_words;
+       g += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t s = seg_of(p.rr_cum, p.n_rr, g);
+    RangeRef rr = p.rr[s];
+    emit_mir(p, rr.lo + (g - p.rr_cum[s]), rr.pos);
+  }
+}
+
+cudaError_t launch_mir(const MirParams& p, uint64_t n_ins_pos, uint64_t n_qry_pos, uint64_t n_rr_words,
+                       cudaStream_t s, int* launches) {
+  auto grid = [](uint64_t n) { uint64_t g = (n + 255) / 256; return (unsigned)(g > 148 * 64 ? 148 * 64 : (g ? g : 1)); };
+  if (n_ins_pos) { k_mir_insert<<<grid(n_ins_pos), 256, 0, s>>>(p, n_ins_pos); ++*launches; }
+  if (n_qry_pos) { k_mir_query<<<grid(n_qry_pos), 256, 0, s>>>(p, n_qry_pos); ++*launches; }
+  if (n_rr_words) { k_mir_ranges<<<grid(n_rr_words), 256, 0, s>>>(p, n_rr_words); ++*launches; }
+  return cudaGetLastError();
+}
+
+}  // namespace arb
