@@ -108,6 +108,7 @@ typedef struct {
   double   ms_partition, ms_control, ms_replay, ms_mir, ms_reports, ms_total;
   uint64_t kernel_launches;  /* kernels launched by the last flush                         */
   double   ms_sample;        /* address sampling + bucket balancing (inside ms_partition)  */
+  uint64_t steps_fast, steps_sort;  /* replay steps by kind                  */
 } arb_stats;
 
 typedef struct arb_ctx_s* arb_ctx;

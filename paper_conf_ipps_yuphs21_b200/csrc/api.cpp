@@ -68,7 +68,7 @@ struct arb_ctx_s {
   uint32_t bucket_bits = 0, n_buckets = 0, coarse_bits = 0, n_bins = 0;
   std::vector<uint32_t> bin_map, order, hist;
   std::vector<uint64_t> bucket_start;
-  DevBuf<uint32_t> d_bin_map, d_order, d_hist;
+  DevBuf<uint32_t> d_bin_map, d_order, d_hist, d_seg;
   DevBuf<uint64_t> d_bucket_start;
   int n_sms = 148;
   uint8_t* shadow = nullptr;
@@ -199,7 +199,7 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   ctx->m_rr_cum.release(); ctx->m_ins_inst.release(); ctx->m_qry_open_start.release(); ctx->m_open_list.release();
   ctx->m_own_start.release(); ctx->m_win_start.release(); ctx->m_own.release(); ctx->m_win.release();
   ctx->m_rr.release(); ctx->hkeys.release(); ctx->hvals.release(); ctx->counts.release();
-  ctx->d_bin_map.release(); ctx->d_order.release(); ctx->d_hist.release(); ctx->d_bucket_start.release();
+  ctx->d_bin_map.release(); ctx->d_order.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_seg.release();
   for (auto& e : ctx->ev) if (e) cudaEventDestroy(e);
   if (ctx->nccl_lib) dlclose(ctx->nccl_lib);
   delete ctx;
@@ -379,7 +379,10 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   rp.bucket_start = ctx->d_bucket_start.p; rp.order = ctx->d_order.p;
   rp.shadow = ctx->shadow; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
   rp.cand = ctx->cand.p; rp.cand_cap = ctx->cand_cap; rp.st = ctx->dstats.p;
-  int n_ctas = std::min<int>((int)ctx->n_buckets, ctx->n_sms * 2);
+  int n_ctas = std::max(1, std::min<int>((int)ctx->n_buckets, ctx->n_sms * kReplayCtasPerSm));
+  CK(ctx->d_seg.ensure((size_t)2 * n_ctas * (n_chunks + 1)), "alloc segment lists");
+  rp.seg_start = ctx->d_seg.p;
+  rp.seg_cum = ctx->d_seg.p + (size_t)n_ctas * (n_chunks + 1);
   CK(launch_replay(rp, std::max(n_ctas, 1), s), "k_replay");
   launches += 1;
   if (timing) cudaEventRecord(ctx->ev[3], s);
@@ -388,6 +391,8 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   const uint64_t n_vsm = hst.n_cand;                 // exact: VSM candidates are unique
   uint64_t kept_vsm = std::min(n_vsm, ctx->cand_cap);
   S.max_bucket_events = hst.max_bucket_events;
+  S.steps_fast = hst.steps_fast;
+  S.steps_sort = hst.steps_sort;
 
   // ---- A6: MIR join ---------------------------------------------------------------
   uint64_t n_mir = 0;

@@ -46,9 +46,10 @@ constexpr int kChunkCap = 2 * kChunkRecords;        // events per chunk (<= 2 wo
 constexpr int kMaxBuckets = 1024;
 
 // ---- replay geometry -------------------------------------------------------
-constexpr int kReplayThreads = 512;
+constexpr int kReplayThreads = 256;
 constexpr int kReplayItems = 8;
 constexpr int kStep = kReplayThreads * kReplayItems;  // events per step
+constexpr int kReplayCtasPerSm = 3;
 
 // device-side counters and error flags of one flush
 struct DevStats {
@@ -61,7 +62,8 @@ struct DevStats {
   unsigned long long max_bucket_events;
   unsigned long long range_words_applied;
   unsigned long long n_mir_cand;
-  unsigned long long pad[7];
+  unsigned long long steps_fast, steps_sort;
+  unsigned long long pad[5];
 };
 
 // control record extracted by the partition kernel
@@ -81,8 +83,8 @@ struct RangeRef { uint64_t lo, hi; uint32_t pos; uint32_t inst; };
 // 2^coarse_bits words.  bin_map[bin] = bucket | (bin - first bin of bucket) << 10,
 // so one lookup gives both the bucket and the word offset inside it.  The map
 // is balanced on a sampled histogram of the batch's access addresses.
-constexpr int kMaxCoarseBins = 1 << 16;
-constexpr uint32_t kSampleCap = 1u << 22;
+constexpr int kMaxCoarseBins = 1 << 18;
+constexpr uint32_t kSampleCap = 1u << 23;
 
 struct SampleParams {
   const uint4* ev; uint64_t n; uint64_t stride;   // sample records 0, stride, 2*stride, ...
@@ -107,6 +109,7 @@ struct ReplayParams {
   uint32_t n_chunks, n_buckets, bucket_bits;
   const uint64_t* bucket_start;           // [n_buckets + 1] first relative word of each bucket
   const uint32_t* order;                  // buckets in scheduling order (largest first)
+  uint32_t* seg_start; uint32_t* seg_cum; // per-CTA scratch: [gridDim][n_chunks + 1] segment list
   uint64_t n_words;
   uint8_t* shadow;                        // n_words bytes
   const uint32_t* ops_start;              // [n_buckets + 1]

@@ -48,7 +48,9 @@ void balance_buckets(const std::vector<uint32_t>& hist, uint32_t coarse_bits, ui
   // span cuts (buckets of <= 2^30 words) are always taken; weight cuts use the
   // rest of the budget (n_words <= 2^38 keeps the span cuts <= 256)
   const uint64_t span_reserve = (n_words >> 30) + 2;
-  const uint64_t target = std::max<uint64_t>(1, total / std::max<uint32_t>(1, max_buckets * 3 / 8));
+  // ~2/3 of the budget by weight leaves room for the cuts a greedy pass adds
+  // around heavy bins, so the last bucket never absorbs a large remainder
+  const uint64_t target = std::max<uint64_t>(1, total / std::max<uint64_t>(1, max_buckets * 2 / 3));
   bin_map.assign(n_bins, 0);
   bucket_start.clear();
   std::vector<uint64_t> weight;

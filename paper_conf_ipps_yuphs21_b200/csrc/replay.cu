@@ -1,10 +1,11 @@
 // replay.cu — A3b + A4 + A5: per-address replay of each bucket.
 //
 // One CTA per address bucket at a time (persistent; buckets in largest-first
-// order).  For its bucket the CTA gathers the word-events in trace order from
-// the chunk-major partition output (segment queue), applies the resolved range
-// ops (Table I transfers / allocate / release; target update P:121)
-// to the bucket's shadow at their trace positions, and processes the events in
+// order).  For its bucket the CTA first compacts the bucket's non-empty chunk
+// segments (from the partition's offset table) into a segment list, then walks
+// the bucket's word-events in trace order, applies the resolved range ops
+// (Table I transfers / allocate / release; target update P:121) to
+// the bucket's shadow at their trace positions, and processes the events in
 // steps of <= 2048 that never straddle a range op:
 //
 //   fast step  (every word has at most one write in the step): a shared-memory
@@ -23,30 +24,28 @@
 
 namespace arb {
 
-constexpr int RT = kReplayThreads;           // 512 threads
-constexpr int RI = 4;                        // events per thread per step
+constexpr int RT = kReplayThreads;           // 256 threads
+constexpr int RI = kReplayItems;             // 8 events per thread per step
 constexpr int STEP = RT * RI;                // 2048 events per step
-constexpr int kQCap = 1024;                  // segment queue (circular)
-constexpr int kScanChunks = 512;             // chunks examined per refill round
+constexpr int kWin = 2 * RT;                 // segment descriptors staged per step
 constexpr int kHSlots = 4096;                // hash slots (load <= 1/2)
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
 constexpr uint32_t kWordMask = 0x3FFFFFFFu;
 
 struct ReplaySmem {
-  uint32_t keyA[STEP], posA[STEP];
+  uint2 ev[2][STEP];              // double-buffered step events {key, pos} (cp.async)
   union {
-    struct { uint32_t keyB[STEP], posB[STEP]; uint16_t hist[RT / 32][256]; } s;   // sort step
+    struct { uint32_t keyA[STEP], posA[STEP], keyB[STEP], posB[STEP]; uint16_t hist[RT / 32][256]; } s;
     struct { uint32_t key[kHSlots], wpos[kHSlots]; uint8_t st[kHSlots]; } h;      // fast step
   } u;
-  uint32_t q_start[kQCap];        // global event index of a segment
-  uint32_t q_len[kQCap];
-  uint32_t pref[kQCap];           // prefix of queue lengths (also radix scratch)
+  uint32_t wstart[kWin];          // staged segment list window: global event index
+  uint32_t wcum[kWin + 1];        //   and bucket-relative first event of each segment
+  uint32_t pref[256];             // radix digit scratch
   uint32_t red[RT / 32], red2[RT / 32], wscan[RT / 32];
-  uint32_t bucket;
-  uint32_t q_head, q_tail, q_head_off;
-  uint64_t q_events;
-  uint32_t chunk_cur, n_gather, op_cur, op_end;
-  uint64_t bucket_events, bucket_base;
+  uint32_t wcnt[RT / 32], wev[RT / 32];
+  uint32_t bucket, op_cur, op_end, next_op;
+  uint32_t n_segs, n_events, wsc, nwin;
+  uint64_t bucket_base;
 };
 
 // ---- block-level helpers ----------------------------------------------------
@@ -75,28 +74,6 @@ __device__ __forceinline__ void block_minmax(uint32_t& lo, uint32_t& hi, uint32_
   lo = 0xFFFFFFFFu; hi = 0;
 #pragma unroll
   for (int w = 0; w < RT / 32; ++w) { lo = min(lo, r1[w]); hi = max(hi, r2[w]); }
-}
-// exclusive block scan (sum); *total = sum
-__device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t* wscan, uint32_t* total) {
-  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  uint32_t incl = v;
-#pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {
-    const uint32_t o = __shfl_up_sync(FULL, incl, d);
-    if (lane >= (uint32_t)d) incl += o;
-  }
-  __syncthreads();
-  if (lane == 31) wscan[warp] = incl;
-  __syncthreads();
-  uint32_t wpre = 0, tot = 0;
-#pragma unroll
-  for (int w = 0; w < RT / 32; ++w) {
-    const uint32_t x = wscan[w];
-    if ((uint32_t)w < warp) wpre += x;
-    tot += x;
-  }
-  *total = tot;
-  return wpre + incl - v;
 }
 
 // ---- range ops ----------------------------------------------------------------
@@ -132,8 +109,9 @@ __device__ void stream_apply(uint8_t* shadow, uint64_t lo, uint64_t hi, Sel sel)
 
 // Apply every pending range op of the bucket with position < limit; runs of
 // ops on the identical range with no event in between are composed first.
+// S.next_op caches the position of the first pending op.
 __device__ void apply_ops_before(ReplaySmem& S, const ReplayParams& p, uint32_t limit) {
-  while (S.op_cur < S.op_end && p.ops[S.op_cur].pos < limit) {
+  while (S.next_op < limit) {
     const uint32_t k = S.op_cur;
     const BucketOp o = p.ops[k];
     Sel sel = o.sel;
@@ -148,6 +126,7 @@ __device__ void apply_ops_before(ReplaySmem& S, const ReplayParams& p, uint32_t 
     __syncthreads();
     if (threadIdx.x == 0) {
       S.op_cur = k2;
+      S.next_op = k2 < S.op_end ? p.ops[k2].pos : 0xFFFFFFFFu;
       atomicAdd(&p.st->range_words_applied, (unsigned long long)(o.hi - o.lo));
     }
     __syncthreads();
@@ -161,6 +140,7 @@ __device__ __forceinline__ void emit_faults(const ReplayParams& p, const uint32_
   uint32_t nf = 0;
 #pragma unroll
   for (int j = 0; j < RI; ++j) nf += fk[j] != 0;
+  if (!__any_sync(FULL, nf != 0)) return;
   uint32_t wf = nf;
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {
@@ -168,7 +148,6 @@ __device__ __forceinline__ void emit_faults(const ReplayParams& p, const uint32_
     if (lane >= (uint32_t)d) wf += o;
   }
   const uint32_t wtot = __shfl_sync(FULL, wf, 31);
-  if (!wtot) return;
   unsigned long long base = 0;
   if (lane == 31) base = atomicAdd(&p.st->n_cand, (unsigned long long)wtot);
   base = __shfl_sync(FULL, base, 31);
@@ -196,17 +175,24 @@ __device__ __forceinline__ void hash_clear(ReplaySmem& S) {
 
 // ---- fast step: at most one write per word -------------------------------------------
 // Returns false (and leaves the shadow untouched) if some word has two writes.
-__device__ bool step_fast(ReplaySmem& S, const ReplayParams& p, uint32_t m) {
-  uint32_t slot[RI], word[RI], pos[RI], op[RI];
+__device__ bool step_fast(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
+  uint32_t slot[RI], word[RI], pos[RI], op[RI], s_pre[RI];
   bool own[RI];
   bool multi = false;
+  const uint64_t bb = S.bucket_base;
+#pragma unroll
+  for (int j = 0; j < RI; ++j) {   // shadow loads first: their latency overlaps the hashing
+    const uint32_t i = threadIdx.x + j * RT;
+    own[j] = false; slot[j] = 0; word[j] = 0; pos[j] = 0; op[j] = 0xFFu; s_pre[j] = 0;
+    if (i < m) {
+      const uint2 e = ev[i];
+      word[j] = e.x & kWordMask; op[j] = e.x >> 30; pos[j] = e.y;
+      s_pre[j] = __ldcg(p.shadow + bb + word[j]);
+    }
+  }
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
-    const uint32_t i = threadIdx.x + j * RT;
-    own[j] = false; slot[j] = 0; word[j] = 0; pos[j] = 0; op[j] = 0xFFu;
-    if (i < m) {
-      const uint32_t k = S.keyA[i];
-      word[j] = k & kWordMask; op[j] = k >> 30; pos[j] = S.posA[i];
+    if (op[j] != 0xFFu) {
       uint32_t h = (word[j] * 2654435761u) >> 20;          // 12 bits
       for (;;) {
         const uint32_t old = atomicCAS(&S.u.h.key[h], kEmpty, word[j]);
@@ -228,10 +214,9 @@ __device__ bool step_fast(ReplaySmem& S, const ReplayParams& p, uint32_t m) {
     __syncthreads();
     return false;
   }
-  const uint64_t bb = S.bucket_base;
 #pragma unroll
   for (int j = 0; j < RI; ++j)
-    if (own[j]) S.u.h.st[slot[j]] = __ldcg(p.shadow + bb + word[j]) & 15u;
+    if (own[j]) S.u.h.st[slot[j]] = s_pre[j] & 15u;
   __syncthreads();
   uint32_t fk[RI];
 #pragma unroll
@@ -279,7 +264,7 @@ __device__ void sort_pass(ReplaySmem& S, const uint32_t* kin, const uint32_t* pi
     kk[r] = k; pp[r] = pv; dg[r] = d; rk[r] = base + __popc(grp & lt);
   }
   __syncthreads();
-  if (tid < 256) {
+  {
     uint32_t s = 0;
 #pragma unroll
     for (int w = 0; w < RT / 32; ++w) {
@@ -305,7 +290,7 @@ __device__ void sort_pass(ReplaySmem& S, const uint32_t* kin, const uint32_t* pi
     for (int j = 0; j < 8; ++j) { S.pref[tid * 8 + j] = run; run += v[j]; }
   }
   __syncthreads();
-  if (tid < 256) {
+  {
     const uint32_t b = S.pref[tid];
 #pragma unroll
     for (int w = 0; w < RT / 32; ++w) S.u.s.hist[w][tid] = (uint16_t)(S.u.s.hist[w][tid] + b);
@@ -342,17 +327,19 @@ __device__ __forceinline__ uint32_t acc_summary(uint32_t op) {
   return op == OP_WH ? (1u | 4u) : (op == OP_WT ? (2u | 8u) : 0u);
 }
 
-__device__ void step_sort(ReplaySmem& S, const ReplayParams& p, uint32_t m) {
+__device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   uint32_t lo = 0xFFFFFFFFu, hi = 0;
   for (uint32_t i = tid; i < m; i += RT) {
-    const uint32_t w = S.keyA[i] & kWordMask;
+    const uint2 e = ev[i];
+    S.u.s.keyA[i] = e.x; S.u.s.posA[i] = e.y;
+    const uint32_t w = e.x & kWordMask;
     lo = min(lo, w); hi = max(hi, w);
   }
   block_minmax(lo, hi, S.red, S.red2);
   const uint32_t span = hi - lo;
   const uint32_t bits = span ? 32 - __clz(span) : 0;
-  uint32_t* kin = S.keyA; uint32_t* pin = S.posA; uint32_t* kout = S.u.s.keyB; uint32_t* pout = S.u.s.posB;
+  uint32_t* kin = S.u.s.keyA; uint32_t* pin = S.u.s.posA; uint32_t* kout = S.u.s.keyB; uint32_t* pout = S.u.s.posB;
   for (uint32_t sh = 0; sh < bits; sh += 8) {
     sort_pass(S, kin, pin, kout, pout, m, lo, sh, (1u << min(8u, bits - sh)) - 1u);
     uint32_t* t = kin; kin = kout; kout = t;
@@ -414,11 +401,130 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, uint32_t m) {
   __syncthreads();
 }
 
+// ---- per-bucket segment list ---------------------------------------------------------------
+// Compact the bucket's non-empty chunk segments, in chunk order, into the CTA's
+// scratch: seg_start[i] = global index of the segment's first event,
+// seg_cum[i] = bucket-relative index of that event; seg_cum[n] = event total.
+__device__ void build_segments(ReplaySmem& S, const ReplayParams& p, uint32_t b, uint32_t* sstart,
+                               uint32_t* scum) {
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint16_t* row0 = p.part_off + (uint64_t)b * p.n_chunks;
+  const uint16_t* row1 = row0 + p.n_chunks;
+  const uint32_t per = (p.n_chunks + RT / 32 - 1) / (RT / 32);
+  const uint32_t c0 = warp * per, c1 = min(p.n_chunks, c0 + per);
+  uint32_t cnt = 0, evs = 0;
+  for (uint32_t c = c0 + lane; c < c1; c += 32) {
+    const uint32_t len = (uint32_t)row1[c] - row0[c];
+    cnt += len != 0;
+    evs += len;
+  }
+#pragma unroll
+  for (int d = 16; d; d >>= 1) {
+    cnt += __shfl_xor_sync(FULL, cnt, d);
+    evs += __shfl_xor_sync(FULL, evs, d);
+  }
+  if (lane == 0) { S.wcnt[warp] = cnt; S.wev[warp] = evs; }
+  __syncthreads();
+  uint32_t cbase = 0, ebase = 0, ctot = 0, etot = 0;
+#pragma unroll
+  for (int w = 0; w < RT / 32; ++w) {
+    if ((uint32_t)w < warp) { cbase += S.wcnt[w]; ebase += S.wev[w]; }
+    ctot += S.wcnt[w]; etot += S.wev[w];
+  }
+  const uint32_t lt = lanemask_lt();
+  for (uint32_t c = c0; c < c1; c += 32) {
+    const uint32_t cc = c + lane;
+    uint32_t st = 0, len = 0;
+    if (cc < c1) { st = row0[cc]; len = (uint32_t)row1[cc] - st; }
+    const uint32_t nz = __ballot_sync(FULL, len != 0);
+    uint32_t incl = len;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t o = __shfl_up_sync(FULL, incl, d);
+      if (lane >= (uint32_t)d) incl += o;
+    }
+    if (len) {
+      const uint32_t idx = cbase + __popc(nz & lt);
+      sstart[idx] = cc * (uint32_t)kChunkCap + st;
+      scum[idx] = ebase + incl - len;
+    }
+    cbase += __popc(nz);
+    ebase += __shfl_sync(FULL, incl, 31);
+  }
+  if (threadIdx.x == 0) { scum[ctot] = etot; S.n_segs = ctot; S.n_events = etot; }
+  __syncthreads();
+}
+
 // ---- the kernel ------------------------------------------------------------------------
-__global__ void __launch_bounds__(RT, 2) k_replay(ReplayParams p) {
+__device__ __forceinline__ void cp_async8(void* smem_dst, const void* gsrc) {
+  const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(d), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+
+// Make the staged window of segment descriptors contain event e0 (rarely reloads).
+__device__ void ensure_window(ReplaySmem& S, const uint32_t* sstart, const uint32_t* scum, uint32_t e0) {
+  if (e0 >= S.wcum[0] && e0 < S.wcum[S.nwin]) return;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t a = 0, z = S.n_segs;                 // last segment with scum <= e0
+    while (z - a > 1) { const uint32_t mid = (a + z) >> 1; if (scum[mid] <= e0) a = mid; else z = mid; }
+    S.wsc = a;
+    S.nwin = min((uint32_t)kWin, S.n_segs - a);
+  }
+  __syncthreads();
+  const uint32_t sc = S.wsc, nwin = S.nwin;
+  for (uint32_t k = threadIdx.x; k < nwin; k += RT) { S.wstart[k] = sstart[sc + k]; S.wcum[k] = scum[sc + k]; }
+  if (threadIdx.x == 0) S.wcum[nwin] = scum[sc + nwin];
+  __syncthreads();
+}
+
+// Issue cp.async copies of events [e0, e0 + m) of the bucket into dst; the
+// window must contain e0.  Returns m (<= STEP, clipped to the window).
+__device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t e0, uint32_t total, uint2* dst) {
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t nwin = S.nwin;
+  const uint32_t m = min(min((uint32_t)STEP, total - e0), S.wcum[nwin] - e0);
+  uint32_t a0, a1;                                  // window segments [a0, a1) hold the events
+  {
+    uint32_t a = 0, z = nwin;
+    while (z - a > 1) { const uint32_t mid = (a + z) >> 1; if (S.wcum[mid] <= e0) a = mid; else z = mid; }
+    a0 = a;
+    a = a0; z = nwin;
+    while (z - a > 1) { const uint32_t mid = (a + z) >> 1; if (S.wcum[mid] < e0 + m) a = mid; else z = mid; }
+    a1 = a + 1;
+  }
+  if ((a1 - a0) * 16 <= m) {
+    // long segments: one warp streams one segment at a time
+    for (uint32_t j = a0 + warp; j < a1; j += RT / 32) {
+      const uint32_t lo = max(S.wcum[j], e0), hi = min(S.wcum[j + 1], e0 + m);
+      const uint2* src = p.part_ev + (uint64_t)S.wstart[j] + (lo - S.wcum[j]);
+      uint2* d = dst + (lo - e0);
+      for (uint32_t k = lane; k < hi - lo; k += 32) cp_async8(d + k, src + k);
+    }
+  } else {
+    // short segments: every thread locates the segments of its events
+#pragma unroll
+    for (int k = 0; k < RI; ++k) {
+      const uint32_t e = e0 + threadIdx.x + k * RT;
+      if (e < e0 + m) {
+        uint32_t a = a0, z = a1;
+        while (z - a > 1) { const uint32_t mid = (a + z) >> 1; if (S.wcum[mid] <= e) a = mid; else z = mid; }
+        cp_async8(dst + (e - e0), p.part_ev + (uint64_t)S.wstart[a] + (e - S.wcum[a]));
+      }
+    }
+  }
+  cp_async_commit();
+  return m;
+}
+
+__global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   ReplaySmem& S = *reinterpret_cast<ReplaySmem*>(smem_raw);
-  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t tid = threadIdx.x;
+  uint32_t* sstart = p.seg_start + (uint64_t)blockIdx.x * (p.n_chunks + 1);
+  uint32_t* scum = p.seg_cum + (uint64_t)blockIdx.x * (p.n_chunks + 1);
   hash_clear(S);
   for (;;) {
     if (tid == 0) {
@@ -429,127 +535,56 @@ __global__ void __launch_bounds__(RT, 2) k_replay(ReplayParams p) {
     const uint32_t b = S.bucket;
     if (b >= p.n_buckets) return;
     if (tid == 0) {
-      S.q_head = S.q_tail = S.q_head_off = 0;
-      S.q_events = 0;
-      S.chunk_cur = 0;
       S.op_cur = p.ops_start[b];
       S.op_end = p.ops_start[b + 1];
-      S.bucket_events = 0;
+      S.next_op = S.op_cur < S.op_end ? p.ops[S.op_cur].pos : 0xFFFFFFFFu;
       S.bucket_base = p.bucket_start[b];
+      S.wcum[0] = 1; S.nwin = 0; S.wcum[0] = 1;   // empty window: forces a load
     }
-    __syncthreads();
-    const uint16_t* row0 = p.part_off + (uint64_t)b * p.n_chunks;
-    const uint16_t* row1 = row0 + p.n_chunks;
-    for (;;) {
-      // ---- refill the segment queue ----------------------------------------
-      while (S.q_events < STEP && S.chunk_cur < p.n_chunks && (S.q_tail - S.q_head) + kScanChunks <= kQCap) {
-        const uint32_t c = S.chunk_cur + tid;
-        uint32_t len = 0, st = 0;
-        if (c < p.n_chunks) { st = row0[c]; len = (uint32_t)row1[c] - st; }
-        uint32_t tot;
-        const uint32_t rank = block_excl_scan(len ? 1u : 0u, S.wscan, &tot);
-        const uint32_t evs = block_sum(len, S.red);
-        if (len) {
-          const uint32_t q = (S.q_tail + rank) % kQCap;
-          S.q_start[q] = c * (uint32_t)kChunkCap + st;
-          S.q_len[q] = len;
-        }
-        __syncthreads();
-        if (tid == 0) {
-          S.q_tail += tot;
-          S.q_events += evs;
-          S.chunk_cur += kScanChunks;
-          S.bucket_events += evs;
-        }
-        __syncthreads();
+    build_segments(S, p, b, sstart, scum);
+    const uint32_t total = S.n_events;
+    uint32_t e0 = 0, cur = 0, m_cur = 0;
+    if (total) {
+      ensure_window(S, sstart, scum, 0);
+      m_cur = issue_gather(S, p, 0, total, S.ev[0]);
+    }
+    while (e0 < total) {
+      cp_async_wait_all();
+      __syncthreads();
+      const uint2* ev = S.ev[cur];
+      const uint32_t m = m_cur;
+      // ---- prefetch the next step's events (assumes the step is not cut) ---------
+      const uint32_t nxt = e0 + m;
+      uint32_t m_nxt = 0;
+      if (nxt < total) {
+        ensure_window(S, sstart, scum, nxt);
+        m_nxt = issue_gather(S, p, nxt, total, S.ev[cur ^ 1]);
       }
-      if (S.q_events == 0) {
-        apply_ops_before(S, p, 0xFFFFFFFFu);
-        break;
+      // ---- range ops before the first event, then cut at the next one -------------
+      apply_ops_before(S, p, ev[0].y);
+      uint32_t cut = m;
+      if (S.next_op != 0xFFFFFFFFu && ev[m - 1].y > S.next_op) {
+        uint32_t cnt = 0;
+        for (uint32_t e = tid; e < m; e += RT) cnt += ev[e].y < S.next_op;
+        cut = block_sum(cnt, S.red);
       }
-      // ---- gather up to STEP events in trace order ---------------------------
-      const uint32_t nseg = min(S.q_tail - S.q_head, (uint32_t)kQCap);
-      {
-        uint32_t v[2];
-#pragma unroll
-        for (int k = 0; k < 2; ++k) {
-          const uint32_t e = 2 * tid + k;
-          v[k] = 0;
-          if (e < nseg) v[k] = S.q_len[(S.q_head + e) % kQCap] - (e == 0 ? S.q_head_off : 0);
-        }
-        uint32_t tot;
-        const uint32_t ex = block_excl_scan(v[0] + v[1], S.wscan, &tot);
-        if (2 * tid < nseg) S.pref[2 * tid] = ex;
-        if (2 * tid + 1 < nseg) S.pref[2 * tid + 1] = ex + v[0];
-        if (tid == 0) S.n_gather = min(tot, (uint32_t)STEP);
-        __syncthreads();
-      }
-      const uint32_t m = S.n_gather;
-      // number of segments that hold the first m events
-      uint32_t nseg_m;
-      {
-        uint32_t a = 0, z = nseg;
-        while (z - a > 1) { const uint32_t mid = (a + z) >> 1; if (S.pref[mid] < m) a = mid; else z = mid; }
-        nseg_m = a + 1;
-      }
-      if (nseg_m * 8 <= m) {
-        // long segments: one warp copies one segment at a time, coalesced
-        for (uint32_t sgi = warp; sgi < nseg_m; sgi += RT / 32) {
-          const uint32_t q = (S.q_head + sgi) % kQCap;
-          const uint32_t dst = S.pref[sgi];
-          const uint32_t len = min((sgi + 1 < nseg ? S.pref[sgi + 1] : m), m) - dst;
-          const uint2* src = p.part_ev + (uint64_t)S.q_start[q] + (sgi == 0 ? S.q_head_off : 0);
-          for (uint32_t k = lane; k < len; k += 64) {
-            const uint2 e0 = ld_stream2(src + k);
-            uint2 e1 = make_uint2(0, 0);
-            if (k + 32 < len) e1 = ld_stream2(src + k + 32);
-            S.keyA[dst + k] = e0.x; S.posA[dst + k] = e0.y;
-            if (k + 32 < len) { S.keyA[dst + k + 32] = e1.x; S.posA[dst + k + 32] = e1.y; }
-          }
-        }
+      const bool fast = step_fast(S, p, ev, cut);
+      if (!fast) step_sort(S, p, ev, cut);
+      if (tid == 0) atomicAdd(fast ? &p.st->steps_fast : &p.st->steps_sort, 1ull);
+      e0 += cut;
+      if (cut == m) {
+        cur ^= 1;
+        m_cur = m_nxt;
       } else {
-        // short segments: every thread finds its events' segments
-        uint2 evv[RI];
-#pragma unroll
-        for (int k = 0; k < RI; ++k) {
-          const uint32_t e = tid + k * RT;
-          evv[k] = make_uint2(0, 0);
-          if (e < m) {
-            uint32_t a = 0, z = nseg_m;
-            while (z - a > 1) { const uint32_t mid = (a + z) >> 1; if (S.pref[mid] <= e) a = mid; else z = mid; }
-            const uint32_t q = (S.q_head + a) % kQCap;
-            const uint32_t off = e - S.pref[a] + (a == 0 ? S.q_head_off : 0);
-            evv[k] = ld_stream2(p.part_ev + (uint64_t)S.q_start[q] + off);
-          }
-        }
-#pragma unroll
-        for (int k = 0; k < RI; ++k) {
-          const uint32_t e = tid + k * RT;
-          if (e < m) { S.keyA[e] = evv[k].x; S.posA[e] = evv[k].y; }
-        }
+        // the prefetch started at e0_old + m: drain it and gather from e0
+        cp_async_wait_all();
+        __syncthreads();
+        ensure_window(S, sstart, scum, e0);
+        m_cur = issue_gather(S, p, e0, total, S.ev[cur]);
       }
-      __syncthreads();
-      // ---- range ops before the first gathered event ---------------------------
-      apply_ops_before(S, p, S.posA[0]);
-      // ---- cut the step at the next pending range op -----------------------------
-      const uint32_t next_op = S.op_cur < S.op_end ? p.ops[S.op_cur].pos : 0xFFFFFFFFu;
-      uint32_t cnt = 0;
-      for (uint32_t e = tid; e < m; e += RT) cnt += S.posA[e] < next_op;
-      const uint32_t cut = block_sum(cnt, S.red);
-      // ---- consume `cut` events from the queue (before pref is reused) -----------
-      if (tid == 0) {
-        uint32_t a = 0, z = nseg;
-        while (z - a > 1) { const uint32_t mid = (a + z) >> 1; if (S.pref[mid] <= cut) a = mid; else z = mid; }
-        const uint32_t q = (S.q_head + a) % kQCap;
-        const uint32_t consumed = cut - S.pref[a] + (a == 0 ? S.q_head_off : 0);
-        if (consumed >= S.q_len[q]) { S.q_head += a + 1; S.q_head_off = 0; }
-        else { S.q_head += a; S.q_head_off = consumed; }
-        S.q_events -= cut;
-      }
-      __syncthreads();
-      if (!step_fast(S, p, cut)) step_sort(S, p, cut);
     }
-    if (tid == 0 && S.bucket_events) atomicMax(&p.st->max_bucket_events, (unsigned long long)S.bucket_events);
+    apply_ops_before(S, p, 0xFFFFFFFFu);
+    if (tid == 0 && total) atomicMax(&p.st->max_bucket_events, (unsigned long long)total);
     __syncthreads();
   }
 }
