@@ -68,7 +68,7 @@ struct arb_ctx_s {
   uint32_t bucket_bits = 0, n_buckets = 0, coarse_bits = 0, n_bins = 0;
   std::vector<uint32_t> bin_map, order, hist;
   std::vector<uint64_t> bucket_start;
-  DevBuf<uint32_t> d_bin_map, d_order, d_hist, d_seg;
+  DevBuf<uint32_t> d_bin_map, d_order, d_hist, d_seg, d_cut;
   DevBuf<uint64_t> d_bucket_start;
   int n_sms = 148;
   uint8_t* shadow = nullptr;
@@ -199,7 +199,7 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   ctx->m_rr_cum.release(); ctx->m_ins_inst.release(); ctx->m_qry_open_start.release(); ctx->m_open_list.release();
   ctx->m_own_start.release(); ctx->m_win_start.release(); ctx->m_own.release(); ctx->m_win.release();
   ctx->m_rr.release(); ctx->hkeys.release(); ctx->hvals.release(); ctx->counts.release();
-  ctx->d_bin_map.release(); ctx->d_order.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_seg.release();
+  ctx->d_bin_map.release(); ctx->d_order.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_seg.release(); ctx->d_cut.release();
   for (auto& e : ctx->ev) if (e) cudaEventDestroy(e);
   if (ctx->nccl_lib) dlclose(ctx->nccl_lib);
   delete ctx;
@@ -304,19 +304,32 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     const uint64_t n_samples = n ? (n + sp.stride - 1) / sp.stride : 0;
     CK(launch_sample(sp, n_samples, s), "k_sample");
     launches += n_samples ? 1 : 0;
-    ctx->hist.resize(ctx->n_bins);
-    CK(cudaMemcpyAsync(ctx->hist.data(), ctx->d_hist.p, ctx->n_bins * sizeof(uint32_t), cudaMemcpyDeviceToHost, s),
-       "hist d2h");
-    CK(cudaStreamSynchronize(s), "sample sync");
-    balance_buckets(ctx->hist, ctx->coarse_bits, ctx->n_words, kMaxBuckets, ctx->bin_map, ctx->bucket_start,
-                    ctx->order);
-  }
-  if (timing) cudaEventRecord(ctx->ev[7], s);
-  if (ctx->bucket_bits == 0 || ctx->d_bin_map.cap == 0) {
+    // cut balanced buckets on the device; the histogram becomes the bin map in place
+    CK(ctx->d_bucket_start.ensure(kMaxBuckets + 1), "alloc buckets");
+    CK(ctx->d_cut.ensure(2 * kMaxBuckets + 2), "alloc cut scratch");
+    CK(launch_cut(ctx->d_hist.p, ctx->n_bins, ctx->coarse_bits, ctx->n_words, kMaxBuckets, ctx->d_bucket_start.p,
+                  ctx->d_cut.p, ctx->d_cut.p + kMaxBuckets, ctx->d_cut.p + 2 * kMaxBuckets, s), "k_cut");
+    launches += 1;
+    uint32_t nb = 0;
+    CK(cudaMemcpyAsync(&nb, ctx->d_cut.p + 2 * kMaxBuckets, 4, cudaMemcpyDeviceToHost, s), "nb d2h");
+    CK(cudaStreamSynchronize(s), "cut sync");
+    ctx->bucket_start.resize(nb + 1);
+    std::vector<uint32_t> weight(nb);
+    CK(cudaMemcpyAsync(ctx->bucket_start.data(), ctx->d_bucket_start.p, (nb + 1) * 8, cudaMemcpyDeviceToHost, s),
+       "buckets d2h");
+    CK(cudaMemcpyAsync(weight.data(), ctx->d_cut.p, nb * 4, cudaMemcpyDeviceToHost, s), "weights d2h");
+    CK(cudaStreamSynchronize(s), "cut sync");
+    ctx->order.resize(nb);
+    for (uint32_t b = 0; b < nb; ++b) ctx->order[b] = b;
+    std::stable_sort(ctx->order.begin(), ctx->order.end(),
+                     [&](uint32_t a, uint32_t b) { return weight[a] > weight[b]; });
+    CK(upload(ctx->d_order, ctx->order, s), "upload order");
+  } else if (ctx->d_bin_map.cap == 0) {
     CK(upload(ctx->d_bin_map, ctx->bin_map, s), "upload bin map");
     CK(upload(ctx->d_bucket_start, ctx->bucket_start, s), "upload bucket starts");
     CK(upload(ctx->d_order, ctx->order, s), "upload order");
   }
+  if (timing) cudaEventRecord(ctx->ev[7], s);
   ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;
   S.buckets = ctx->n_buckets;
   // ---- A1/A3a: decode + partition ------------------------------------------
@@ -330,7 +343,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     hst.err_pos = ~0ull;
     CK(cudaMemcpyAsync(ctx->dstats.p, &hst, sizeof(hst), cudaMemcpyHostToDevice, s), "stats init");
     pp.ev = ev; pp.n = n; pp.base_word = ctx->base_word; pp.n_words = ctx->n_words;
-    pp.coarse_bits = ctx->coarse_bits; pp.bin_map = ctx->d_bin_map.p;
+    pp.coarse_bits = ctx->coarse_bits; pp.bin_map = ctx->bucket_bits ? ctx->d_bin_map.p : ctx->d_hist.p;
     pp.bucket_bits = ctx->bucket_bits; pp.n_buckets = ctx->n_buckets; pp.n_chunks = n_chunks;
     pp.part_ev = ctx->part_ev.p; pp.part_off = ctx->part_off.p; pp.ctl = ctx->ctl.p; pp.ctl_cap = ctx->ctl_cap;
     pp.st = ctx->dstats.p;

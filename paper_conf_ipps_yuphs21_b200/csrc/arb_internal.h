@@ -84,7 +84,7 @@ struct RangeRef { uint64_t lo, hi; uint32_t pos; uint32_t inst; };
 // so one lookup gives both the bucket and the word offset inside it.  The map
 // is balanced on a sampled histogram of the batch's access addresses.
 constexpr int kMaxCoarseBins = 1 << 18;
-constexpr uint32_t kSampleCap = 1u << 23;
+constexpr uint32_t kSampleCap = 1u << 20;
 
 struct SampleParams {
   const uint4* ev; uint64_t n; uint64_t stride;   // sample records 0, stride, 2*stride, ...
@@ -139,6 +139,9 @@ struct MirParams {
 
 // ---- kernel launchers (kernels.cu) -----------------------------------------
 cudaError_t launch_sample(const SampleParams& p, uint64_t n_samples, cudaStream_t s);
+cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits, uint64_t n_words,
+                       uint32_t max_buckets, uint64_t* bucket_start, uint32_t* weight, uint32_t* first_bin,
+                       uint32_t* nb_out, cudaStream_t s);
 cudaError_t launch_partition(const PartParams& p, cudaStream_t s);
 cudaError_t launch_replay(const ReplayParams& p, int n_ctas, cudaStream_t s);
 cudaError_t launch_mir(const MirParams& p, uint64_t n_ins_pos, uint64_t n_qry_pos, uint64_t n_rr_words,

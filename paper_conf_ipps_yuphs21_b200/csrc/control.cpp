@@ -38,42 +38,6 @@ struct Emitter {
 
 }  // namespace
 
-void balance_buckets(const std::vector<uint32_t>& hist, uint32_t coarse_bits, uint64_t n_words,
-                     uint32_t max_buckets, std::vector<uint32_t>& bin_map,
-                     std::vector<uint64_t>& bucket_start, std::vector<uint32_t>& order) {
-  const uint64_t n_bins = hist.size();
-  uint64_t total = 0;
-  for (uint32_t h : hist) total += h;
-  const uint64_t max_span_bins = std::max<uint64_t>(1, (1ull << 30) >> coarse_bits);
-  // span cuts (buckets of <= 2^30 words) are always taken; weight cuts use the
-  // rest of the budget (n_words <= 2^38 keeps the span cuts <= 256)
-  const uint64_t span_reserve = (n_words >> 30) + 2;
-  // ~2/3 of the budget by weight leaves room for the cuts a greedy pass adds
-  // around heavy bins, so the last bucket never absorbs a large remainder
-  const uint64_t target = std::max<uint64_t>(1, total / std::max<uint64_t>(1, max_buckets * 2 / 3));
-  bin_map.assign(n_bins, 0);
-  bucket_start.clear();
-  std::vector<uint64_t> weight;
-  uint64_t first = 0, acc = 0;
-  for (uint64_t i = 0; i < n_bins; ++i) {
-    bool full = acc > 0 && acc + hist[i] > target && bucket_start.size() + 1 + span_reserve < max_buckets;
-    bool too_long = i - first >= max_span_bins;
-    if (full || too_long) {
-      bucket_start.push_back(first << coarse_bits);
-      weight.push_back(acc);
-      first = i; acc = 0;
-    }
-    acc += hist[i];
-    bin_map[i] = (uint32_t)bucket_start.size() | (uint32_t)((i - first) << 10);
-  }
-  bucket_start.push_back(first << coarse_bits);
-  weight.push_back(acc);
-  bucket_start.push_back(n_words);
-  order.resize(weight.size());
-  for (uint32_t b = 0; b < order.size(); ++b) order[b] = b;
-  std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return weight[a] > weight[b]; });
-}
-
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
                      FlushPlan& out) {

@@ -50,13 +50,4 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
                      FlushPlan& out);
 
-// Balance address buckets on a sampled histogram of coarse bins: contiguous
-// bins are grouped greedily so that each bucket holds about total/target
-// samples (a bucket spans at most 2^30 words).  Fills bin_map (see
-// arb_internal.h), bucket_start (n_buckets + 1 entries) and a largest-first
-// scheduling order.
-void balance_buckets(const std::vector<uint32_t>& hist, uint32_t coarse_bits, uint64_t n_words,
-                     uint32_t max_buckets, std::vector<uint32_t>& bin_map,
-                     std::vector<uint64_t>& bucket_start, std::vector<uint32_t>& order);
-
 }  // namespace arb
