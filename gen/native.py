@@ -250,3 +250,182 @@ def config5(total_records: int = 9 * 10**9, groups: int = 4096, seed: int = BASE
         p.quiescent.append(p.n)
     p.meta = dict(groups=groups, total_records=total_records)
     return p.finish()
+
+
+# ---------------------------------------------------------------------------
+# config 3: "Rodinia-like offload loops (hotspot/lud/bfs shapes) with target
+# data regions and nowait, ~10^9 events"
+# ---------------------------------------------------------------------------
+C3_BASE = 0x2000_0000_0000        # byte address of the first array
+
+
+def _arrays(base, sizes, gap=1 << 20):
+    out, a = [], base
+    for s in sizes:
+        out.append(a)
+        a += (s + gap + 4095) & ~4095
+    return out, a - base
+
+
+def config3(scale: float = 1.0, seed: int = BASE_SEED + 3, hotspot_iters: int = 6) -> Program:
+    """hotspot: 4096^2 float temp/power/result, 5-point stencil, target data
+    map(to:power) map(tofrom:temp) map(alloc:result), per iteration a nowait
+    kernel + taskwait; one iteration reads a result row on the host before the
+    taskwait (MIR).  lud: 1024^2 doubles in 64x64 blocks (diagonal, perimeter,
+    internal kernels), tofrom.  bfs: R-MAT-like (skewed) graph, V=2^22, E=2^25,
+    CSR mapped to, mask/visited/cost tofrom, per level kernel + target update
+    from(stop) + host read of `stop` (a hot word); one level omits the update
+    (USD).  `scale` shrinks the grids / graph for tests."""
+    N = max(64, int(4096 * scale ** 0.5)) & ~63
+    LN = max(128, int(1024 * scale ** 0.5)) & ~63
+    V = max(1 << 10, int((1 << 22) * scale))
+    E = 8 * V
+    F4, F8 = 4, 8
+    sizes = [N * N * F4] * 3 + [LN * LN * F8] + [(V + 1) * F4, E * F4, V * F4, V * F4, V * F4, 64]
+    (temp, power, result, lud, rowp, col, mask, visited, cost, stop), span = _arrays(C3_BASE, sizes)
+    p = Program("config3", C3_BASE, span)
+    L, S = OP, MAP
+    # ---------------- hotspot ----------------
+    p.loop([(L.WH, F4, M_LINEAR, temp, F4, 0), (L.WH, F4, M_LINEAR, power, F4, 0)], N * N)
+    for a, mt in ((power, S.TO), (temp, S.TOFROM), (result, S.ALLOC)):
+        p.sections.append((a // 8, (a + N * N * F4 + 7) // 8, p.n))
+        p.lit(encode(OP.MAP_ENTER, a, N * N * F4, arg=mt))
+    src, dst = temp, result
+    task = 1
+    for it in range(hotspot_iters):
+        p.lit(encode(OP.TASK_BEGIN, task=task))
+        c0 = N                                           # interior rows 1 .. N-2
+        p.loop([(L.RT, F4, M_LINEAR, src + c0 * F4, F4, 0), (L.RT, F4, M_LINEAR, src + (c0 - 1) * F4, F4, 0),
+                (L.RT, F4, M_LINEAR, src + (c0 + 1) * F4, F4, 0), (L.RT, F4, M_LINEAR, src + (c0 - N) * F4, F4, 0),
+                (L.RT, F4, M_LINEAR, src + (c0 + N) * F4, F4, 0), (L.RT, F4, M_LINEAR, power + c0 * F4, F4, 0),
+                (L.WT, F4, M_LINEAR, dst + c0 * F4, F4, 0)], N * (N - 2))
+        # boundary rows: copied through (clamped stencil)
+        p.loop([(L.RT, F4, M_LINEAR, src, F4, 0), (L.WT, F4, M_LINEAR, dst, F4, 0),
+                (L.RT, F4, M_LINEAR, src + (N - 1) * N * F4, F4, 0),
+                (L.WT, F4, M_LINEAR, dst + (N - 1) * N * F4, F4, 0)], N)
+        p.lit(encode(OP.TASK_END, task=task))
+        if it == 2:   # host reads a boundary row of the result before the taskwait (MIR + stale)
+            p.loop([(L.RH, F4, M_LINEAR, dst + N * F4, F4, 0)], N)
+        p.lit(encode(OP.SYNC, task=task))
+        p.quiescent.append(p.n)
+        task += 1
+        src, dst = dst, src
+    for a, mt in ((power, S.TO), (temp, S.TOFROM), (result, S.ALLOC)):
+        p.lit(encode(OP.MAP_EXIT, a, N * N * F4, arg=mt))
+    p.loop([(L.RH, F4, M_LINEAR, temp + (N // 2) * N * F4, F4, 0)], N)   # host prints a row
+    p.quiescent.append(p.n)
+    # ---------------- lud ----------------
+    B = 64
+    nb = LN // B
+    p.loop([(L.WH, F8, M_LINEAR, lud, F8, 0)], LN * LN)
+    p.sections.append((lud // 8, lud // 8 + LN * LN, p.n))
+    p.lit(encode(OP.MAP_ENTER, lud, LN * LN * F8, arg=S.TOFROM))
+    blk = lambda bi, bj: lud + (bi * B * LN + bj * B) * F8
+    for k in range(nb):
+        p.loop([(L.RT, F8, M_2D, blk(k, k), F8, LN * F8), (L.WT, F8, M_2D, blk(k, k), F8, LN * F8)], B * B, width=B)
+        for j in range(k + 1, nb):
+            p.loop([(L.RT, F8, M_2D, blk(k, k), F8, LN * F8), (L.RT, F8, M_2D, blk(k, j), F8, LN * F8),
+                    (L.WT, F8, M_2D, blk(k, j), F8, LN * F8)], B * B, width=B)
+            p.loop([(L.RT, F8, M_2D, blk(k, k), F8, LN * F8), (L.RT, F8, M_2D, blk(j, k), F8, LN * F8),
+                    (L.WT, F8, M_2D, blk(j, k), F8, LN * F8)], B * B, width=B)
+        for i in range(k + 1, nb):
+            for j in range(k + 1, nb):
+                p.loop([(L.RT, F8, M_2D, blk(i, k), F8, LN * F8), (L.RT, F8, M_2D, blk(k, j), F8, LN * F8),
+                        (L.RT, F8, M_2D, blk(i, j), F8, LN * F8), (L.WT, F8, M_2D, blk(i, j), F8, LN * F8)],
+                       B * B, width=B)
+    p.lit(encode(OP.MAP_EXIT, lud, LN * LN * F8, arg=S.TOFROM))
+    p.loop([(L.RH, F8, M_LINEAR, lud, F8, 0)], LN)
+    p.quiescent.append(p.n)
+    # ---------------- bfs ----------------
+    p.loop([(L.WH, F4, M_LINEAR, rowp, F4, 0)], V + 1)
+    p.loop([(L.WH, F4, M_LINEAR, col, F4, 0)], E)
+    p.loop([(L.WH, F4, M_LINEAR, mask, F4, 0), (L.WH, F4, M_LINEAR, visited, F4, 0),
+            (L.WH, F4, M_LINEAR, cost, F4, 0)], V)
+    p.wh_stop = stop
+    p.lit(encode(OP.WH, stop, 4))
+    for a, n, mt in ((rowp, V + 1, S.TO), (col, E, S.TO), (mask, V, S.TOFROM), (visited, V, S.TOFROM),
+                     (cost, V, S.TOFROM), (stop, 1, S.TOFROM)):
+        p.sections.append((a // 8, (a + n * F4 + 7) // 8, p.n))
+        p.lit(encode(OP.MAP_ENTER, a, n * F4, arg=mt))
+    frac = [0.001, 0.01, 0.05, 0.15, 0.25, 0.25, 0.15, 0.08, 0.04, 0.015, 0.004, 0.001]
+    e0 = 0
+    for lvl, f in enumerate(frac):
+        ne = min(E, max(8, int(E * f))) & ~7
+        e0 = min(e0, E - ne)
+        p.lit(encode(OP.WH, stop, 4), encode(OP.UPDATE, stop, 4, arg=0))       # stop = false; update to
+        p.loop([(L.RT, F4, M_LINEAR, mask, F4, 0)], V)                          # scan the frontier mask
+        body = [(L.RT, F4, M_SKEW, rowp, F4, V)]                               # frontier vertex's row_ptr
+        for k in range(8):   # 8 edges per iteration: col[e], visited[u], cost[u], mask[u]
+            body += [(L.RT, F4, M_LINEAR, col + (e0 + k) * F4, 8 * F4, 0),
+                     (L.RT, F4, M_SKEW, visited, F4, V), (L.WT, F4, M_SKEW, cost, F4, V),
+                     (L.WT, F4, M_SKEW, mask, F4, V)]
+        body.append((L.WT, F4, M_LINEAR, stop, 0, 0))                          # the hot `stop` flag
+        p.loop(body, ne // 8, seed=rng(seed, lvl))
+        e0 = e0 + ne
+        if lvl != 5:
+            p.lit(encode(OP.UPDATE, stop, 4, arg=1))                            # update from(stop)
+        p.lit(encode(OP.RH, stop, 4))                                           # host reads stop
+        p.quiescent.append(p.n)
+    for a, n, mt in ((rowp, V + 1, S.TO), (col, E, S.TO), (mask, V, S.TOFROM), (visited, V, S.TOFROM),
+                     (cost, V, S.TOFROM), (stop, 1, S.TOFROM)):
+        p.lit(encode(OP.MAP_EXIT, a, n * F4, arg=mt))
+    p.meta = dict(N=N, LN=LN, V=V, E=E)
+    return p.finish()
+
+
+# ---------------------------------------------------------------------------
+# config 4: "SPEC-ACCEL-like multi-array stencil with repeated target update
+# and array-section maps, 16 GB shadow" (SURVEY §8(d); 503.postencil P:386)
+# ---------------------------------------------------------------------------
+C4_BASE = 0x4000_0000_0000
+
+
+def config4(scale: float = 1.0, iters: int = 3) -> Program:
+    """8 arrays of NX*NY*NZ doubles (2048x2048x512 = 2^31 at scale 1 -> 2^34
+    words of shadow).  X (mapped tofrom) and Y (mapped to) by target data; six
+    more arrays by target enter/exit data.  Each of `iters` (3)
+    iterations runs a 7-point stencil over a 1/64 z-slab, src -> dst with a host
+    pointer swap (503.postencil), then `target update from` the slab's
+    top halo plane of dst and `target update to` its bottom halo plane of src.
+    With an odd count the result stays in the `to`-mapped Y: the host's final
+    reads (a sample of the output) are stale (USD)."""
+    NX = NY = max(64, int(2048 * scale ** (1 / 3))) & ~15
+    NZ = max(64, int(512 * scale ** (1 / 3))) & ~63
+    plane = NX * NY
+    n = plane * NZ
+    F8 = 8
+    arrs, span = _arrays(C4_BASE, [n * F8] * 8, gap=0)
+    X, Y = arrs[0], arrs[1]
+    p = Program("config4", C4_BASE, span)
+    L, S = OP, MAP
+    z0, nz = NZ // 2, max(2, NZ // 64)
+    c0, cells = (z0 * plane), nz * plane
+    # host initialises the slab (and its halo planes) of X and Y
+    p.loop([(L.WH, F8, M_LINEAR, X + (c0 - plane) * F8, F8, 0),
+            (L.WH, F8, M_LINEAR, Y + (c0 - plane) * F8, F8, 0)], cells + 2 * plane)
+    for a, mt in zip(arrs, [S.TOFROM, S.TO] + [S.TO] * 6):
+        p.sections.append((a // 8, a // 8 + n, p.n))
+        p.lit(encode(OP.MAP_ENTER, a, n * F8, arg=mt))
+    src, dst = X, Y
+    for it in range(iters):
+        offs = [0, -1, 1, -NX, NX, -plane, plane]
+        body = [(L.RT, F8, M_LINEAR, src + (c0 + o) * F8, F8, 0) for o in offs]
+        body.append((L.WT, F8, M_LINEAR, dst + c0 * F8, F8, 0))
+        p.loop(body, cells)
+        p.lit(encode(OP.UPDATE, dst + (c0 + cells - plane) * F8, plane * F8, arg=1),   # update from: top halo
+              encode(OP.UPDATE, src + (c0 - plane) * F8, plane * F8, arg=0))           # update to: bottom halo
+        src, dst = dst, src
+    for a, mt in zip(arrs, [S.TOFROM, S.TO] + [S.TO] * 6):
+        p.lit(encode(OP.MAP_EXIT, a, n * F8, arg=mt))
+    p.loop([(L.RH, F8, M_LINEAR, src + c0 * F8, 64 * F8, 0)], min(65536, cells // 64))  # sampled output reads
+    p.meta = dict(NX=NX, NY=NY, NZ=NZ, words=8 * n)
+    return p.finish()
+
+
+def from_records(name, rec, addr_base, addr_bytes) -> Program:
+    """Wrap a host-built trace (configs 1-2) as a literal program."""
+    p = Program(name, addr_base, addr_bytes)
+    for k in range(0, rec.shape[0], 1 << 16):
+        p.lit(*[(int(a), int(b)) for a, b in rec[k:k + (1 << 16)]])
+    p.sections.append((addr_base // 8, (addr_base + addr_bytes) // 8, 0))
+    return p.finish()
