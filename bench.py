@@ -215,7 +215,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--cpu-records", type=int, default=60_000_000)
+    ap.add_argument("--cpu-records", type=int, default=300_000_000)
     ap.add_argument("--ref-sample", type=int, default=15_000_000)
     args = ap.parse_args()
     if args.impl == "reference":
@@ -316,8 +316,18 @@ def main():
     # record once (16 R); the replay owns the shadow term (2 W) and the report writes (16 Rep)
     alg = {"k_partition": 16 * s0["records"], "k_replay": 2 * W + 16 * s0["reports"]}
     achieved = alg[dom] / (phases[dom] / 1e3) / 1e9 if phases[dom] > 0 else 0.0
+    # DRAM traffic of the dominant kernel from the committed `ncu --set full`
+    # capture (profiles/traffic.json), scaled per launch to this step's records
+    traffic = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as fh:
+            tj = json.load(fh)[dom]
+        traffic = tj["dram_bytes_per_launch"] / tj["records_in_launch"] * s0["records"] / len(flushes)
+    except Exception:
+        pass
     roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": hbm_gbs, "unit": "GB/s",
-            "frac": achieved / hbm_gbs, "traffic": None, "peak_source": peak_src,
+            "frac": achieved / hbm_gbs, "traffic": traffic, "traffic_unit": "bytes per launch (ncu)",
+            "alg_bytes_per_launch": alg[dom] / len(flushes), "peak_source": peak_src,
             "kernel_ms_per_step": phases[dom], "phase_ms_per_step": phases,
             "path": {"b_alg_bytes_per_step": b_alg, "achieved": b_alg / (ms_per_step / 1e3) / 1e9,
                      "frac": b_alg / (ms_per_step / 1e3) / 1e9 / hbm_gbs}}
