@@ -78,7 +78,9 @@ struct arb_ctx_s {
   DevBuf<uint4> staging;
   DevBuf<uint64_t> gidx_staging;
   DevBuf<uint2> part_ev;
-  DevBuf<uint16_t> part_off;
+  DevBuf<uint4> seg_a, seg_b;
+  DevBuf<uint32_t> seg_first;
+  uint64_t seg_cap = 0;
   DevBuf<CtlRec> ctl;
   DevBuf<uint4> cand, cand_tmp, reports;
   DevBuf<uint32_t> blk;
@@ -192,7 +194,7 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   if (!ctx) return ARB_OK;
   if (ctx->comm && ctx->nccl_destroy) ctx->nccl_destroy(ctx->comm);
   if (ctx->shadow) cudaFree(ctx->shadow);
-  ctx->staging.release(); ctx->gidx_staging.release(); ctx->part_ev.release(); ctx->part_off.release();
+  ctx->staging.release(); ctx->gidx_staging.release(); ctx->part_ev.release(); ctx->seg_a.release(); ctx->seg_b.release(); ctx->seg_first.release();
   ctx->ctl.release(); ctx->cand.release(); ctx->cand_tmp.release(); ctx->reports.release(); ctx->blk.release();
   ctx->ops_start.release(); ctx->ops.release(); ctx->dstats.release(); ctx->dcount.release();
   ctx->m_ins_lo.release(); ctx->m_ins_cum.release(); ctx->m_qry_lo.release(); ctx->m_qry_cum.release();
@@ -335,7 +337,8 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   // ---- A1/A3a: decode + partition ------------------------------------------
   const uint32_t n_chunks = (uint32_t)((n + kChunkRecords - 1) / kChunkRecords);
   CK(ctx->part_ev.ensure((size_t)std::max<uint32_t>(n_chunks, 1) * kChunkCap), "alloc part_ev");
-  CK(ctx->part_off.ensure((size_t)(ctx->n_buckets + 1) * std::max<uint32_t>(n_chunks, 1)), "alloc part_off");
+  if (ctx->seg_cap < (uint64_t)n_chunks * 16) ctx->seg_cap = (uint64_t)n_chunks * 16;
+  CK(ctx->seg_a.ensure(std::max<uint64_t>(ctx->seg_cap, 1)), "alloc segments");
   DevStats hst;
   PartParams pp{};
   for (int attempt = 0; attempt < 2; ++attempt) {
@@ -345,15 +348,18 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     pp.ev = ev; pp.n = n; pp.base_word = ctx->base_word; pp.n_words = ctx->n_words;
     pp.coarse_bits = ctx->coarse_bits; pp.bin_map = ctx->bucket_bits ? ctx->d_bin_map.p : ctx->d_hist.p;
     pp.bucket_bits = ctx->bucket_bits; pp.n_buckets = ctx->n_buckets; pp.n_chunks = n_chunks;
-    pp.part_ev = ctx->part_ev.p; pp.part_off = ctx->part_off.p; pp.ctl = ctx->ctl.p; pp.ctl_cap = ctx->ctl_cap;
+    pp.part_ev = ctx->part_ev.p; pp.seg_out = ctx->seg_a.p; pp.seg_cap = ctx->seg_cap;
+    pp.ctl = ctx->ctl.p; pp.ctl_cap = ctx->ctl_cap;
     pp.st = ctx->dstats.p;
     CK(launch_partition(pp, s), "k_partition");
     launches += n_chunks ? 1 : 0;
     CK(cudaMemcpyAsync(&hst, ctx->dstats.p, sizeof(hst), cudaMemcpyDeviceToHost, s), "stats d2h");
     CK(cudaStreamSynchronize(s), "partition sync");
-    if (hst.n_ctl <= ctx->ctl_cap) break;
-    ctx->ctl_cap = hst.n_ctl + hst.n_ctl / 2;
+    if (hst.n_ctl <= ctx->ctl_cap && hst.n_segs <= ctx->seg_cap) break;
+    if (hst.n_ctl > ctx->ctl_cap) ctx->ctl_cap = hst.n_ctl + hst.n_ctl / 2;
+    if (hst.n_segs > ctx->seg_cap) ctx->seg_cap = hst.n_segs + hst.n_segs / 4;
     CK(ctx->ctl.ensure(ctx->ctl_cap), "grow ctl");
+    CK(ctx->seg_a.ensure(ctx->seg_cap), "grow segments");
   }
   if (timing) cudaEventRecord(ctx->ev[1], s);
   if (hst.err_pos != ~0ull) {
@@ -387,7 +393,21 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
 
   // ---- A3b/A4/A5: replay ---------------------------------------------------------
   ReplayParams rp{};
-  rp.part_ev = ctx->part_ev.p; rp.part_off = ctx->part_off.p; rp.n_chunks = n_chunks;
+  // segment entries sorted by (bucket, chunk) and each bucket's first entry
+  uint4* segs_sorted = ctx->seg_a.p;
+  {
+    const uint64_t ns = hst.n_segs;
+    CK(ctx->seg_b.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
+    CK(ctx->seg_first.ensure(ctx->n_buckets + 1), "alloc seg_first");
+    CK(ctx->blk.ensure(std::max<uint64_t>((ns + 4095) / 4096 * 256, 1)), "alloc blk");
+    int cb = 1;
+    while (cb < 32 && ((uint64_t)n_chunks >> cb)) ++cb;
+    uint4* a = ctx->seg_a.p;
+    uint4* b2 = ctx->seg_b.p;
+    CK(launch_sort_segments(a, b2, ns, cb, ctx->n_buckets, ctx->blk.p, ctx->seg_first.p, &segs_sorted, s, &launches),
+       "sort segments");
+  }
+  rp.part_ev = ctx->part_ev.p; rp.segs = segs_sorted; rp.seg_first = ctx->seg_first.p; rp.n_chunks = n_chunks;
   rp.n_buckets = ctx->n_buckets; rp.bucket_bits = ctx->bucket_bits; rp.n_words = ctx->n_words;
   rp.bucket_start = ctx->d_bucket_start.p; rp.order = ctx->d_order.p;
   rp.shadow = ctx->shadow; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;

@@ -63,7 +63,8 @@ struct DevStats {
   unsigned long long range_words_applied;
   unsigned long long n_mir_cand;
   unsigned long long steps_fast, steps_sort;
-  unsigned long long pad[5];
+  unsigned long long n_segs;          // (chunk, bucket) segment entries written by k_partition
+  unsigned long long pad[4];
 };
 
 // control record extracted by the partition kernel
@@ -99,13 +100,15 @@ struct PartParams {
   uint32_t bucket_bits, n_buckets;
   uint32_t n_chunks;
   uint2* part_ev;                         // [n_chunks][kChunkCap]
-  uint16_t* part_off;                     // [n_buckets + 1][n_chunks] start of bucket in chunk
+  uint4* seg_out; uint64_t seg_cap;       // {chunk, bucket, start | len << 16, 0} per touched bucket
   CtlRec* ctl; uint64_t ctl_cap;
   DevStats* st;
 };
 
 struct ReplayParams {
-  const uint2* part_ev; const uint16_t* part_off;
+  const uint2* part_ev;
+  const uint4* segs;                      // segment entries sorted by (bucket, chunk)
+  const uint32_t* seg_first;              // [n_buckets + 1] first entry of each bucket
   uint32_t n_chunks, n_buckets, bucket_bits;
   const uint64_t* bucket_start;           // [n_buckets + 1] first relative word of each bucket
   const uint32_t* order;                  // buckets in scheduling order (largest first)
@@ -143,6 +146,8 @@ cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits
                        uint32_t max_buckets, uint64_t* bucket_start, uint32_t* weight, uint32_t* first_bin,
                        uint32_t* nb_out, cudaStream_t s);
 cudaError_t launch_partition(const PartParams& p, cudaStream_t s);
+cudaError_t launch_sort_segments(uint4* a, uint4* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
+                                 uint32_t* first, uint4** sorted, cudaStream_t s, int* launches);
 cudaError_t launch_replay(const ReplayParams& p, int n_ctas, cudaStream_t s);
 cudaError_t launch_mir(const MirParams& p, uint64_t n_ins_pos, uint64_t n_qry_pos, uint64_t n_rr_words,
                        cudaStream_t s, int* launches);

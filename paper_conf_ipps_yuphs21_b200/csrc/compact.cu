@@ -181,6 +181,32 @@ static int add_field_passes(RsPass* ps, int np, int field, int bits) {
   return np;
 }
 
+// first entry of every bucket in the (bucket, chunk)-sorted segment entries
+__global__ void k_seg_first(const uint4* segs, uint64_t n, uint32_t n_buckets, uint32_t* first) {
+  for (uint32_t b = blockIdx.x * blockDim.x + threadIdx.x; b <= n_buckets; b += gridDim.x * blockDim.x) {
+    uint64_t a = 0, z = n;                 // first entry with bucket >= b
+    while (a < z) { const uint64_t mid = (a + z) >> 1; if (segs[mid].y < b) a = mid + 1; else z = mid; }
+    first[b] = (uint32_t)a;
+  }
+}
+
+// Sort the partition's segment entries {chunk, bucket, start|len<<16, 0} by
+// (bucket, chunk) — stable LSD passes on the chunk then the bucket field — and
+// compute each bucket's first entry.  *sorted points at the result (a or b).
+cudaError_t launch_sort_segments(uint4* a, uint4* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
+                                 uint32_t* first, uint4** sorted, cudaStream_t s, int* launches) {
+  RsPass ps[8];
+  int np = add_field_passes(ps, 0, 2, chunk_bits);
+  np = add_field_passes(ps, np, 3, 10);
+  cudaError_t e = cudaSuccess;
+  if (n) e = radix_sort(a, b, n, ps, np, cnt, s, launches);
+  if (e != cudaSuccess) return e;
+  *sorted = a;
+  k_seg_first<<<(n_buckets + 256) / 256, 256, 0, s>>>(a, n, n_buckets, first);
+  *launches += 1;
+  return cudaGetLastError();
+}
+
 cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches) {
   cudaMemsetAsync(p.n_out, 0, 4 * sizeof(unsigned long long), s);
   if (p.n_cand == 0) return cudaGetLastError();

@@ -24,6 +24,7 @@ struct PartSmem {
   uint32_t tstart[kMaxBuckets + 1];         // their first event in the chunk
   uint32_t wsum[PW];
   uint32_t n_touched, total;
+  unsigned long long seg_base;
 };
 
 // Decoded access record: info = cnt | b0 << 2 | b1 << 12 (cnt = tracked words
@@ -255,11 +256,13 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
       if (tid == 0) { S.total = all0 + all1; S.tstart[T] = all0 + all1; }
     }
     __syncthreads();
-    // ---- table row: start of every bucket in the chunk ------------------------------
-    for (uint32_t b = tid; b <= NB; b += PT) {
-      uint32_t a = 0, z = T;                       // touched buckets below b
-      while (a < z) { const uint32_t mid = (a + z) >> 1; if (S.tlist[mid] < b) a = mid + 1; else z = mid; }
-      p.part_off[(uint64_t)b * p.n_chunks + chunk] = (uint16_t)S.tstart[a];
+    // ---- one segment entry per touched bucket: {chunk, bucket, start | len << 16} ----
+    if (tid == 0) S.seg_base = atomicAdd(&p.st->n_segs, (unsigned long long)T);
+    __syncthreads();
+    for (uint32_t t = tid; t < T; t += PT) {
+      const unsigned long long slot = S.seg_base + t;
+      const uint32_t st = S.tstart[t], len = S.tstart[t + 1] - st;
+      if (slot < p.seg_cap) p.seg_out[slot] = make_uint4((uint32_t)chunk, S.tlist[t], st | (len << 16), 0);
     }
     // ---- pass B: scatter into shared memory -------------------------------------------
 #pragma unroll

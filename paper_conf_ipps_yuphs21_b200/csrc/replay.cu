@@ -44,7 +44,7 @@ struct ReplaySmem {
   uint32_t red[RT / 32], red2[RT / 32], wscan[RT / 32];
   uint32_t wcnt[RT / 32], wev[RT / 32];
   uint32_t bucket, op_cur, op_end, next_op;
-  uint32_t n_segs, n_events, wsc, nwin;
+  uint32_t n_segs, n_events, wsc, nwin, ga0, ga1;
   uint64_t bucket_base;
 };
 
@@ -408,50 +408,32 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
 __device__ void build_segments(ReplaySmem& S, const ReplayParams& p, uint32_t b, uint32_t* sstart,
                                uint32_t* scum) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const uint16_t* row0 = p.part_off + (uint64_t)b * p.n_chunks;
-  const uint16_t* row1 = row0 + p.n_chunks;
-  const uint32_t per = (p.n_chunks + RT / 32 - 1) / (RT / 32);
-  const uint32_t c0 = warp * per, c1 = min(p.n_chunks, c0 + per);
-  uint32_t cnt = 0, evs = 0;
-  for (uint32_t c = c0 + lane; c < c1; c += 32) {
-    const uint32_t len = (uint32_t)row1[c] - row0[c];
-    cnt += len != 0;
-    evs += len;
-  }
-#pragma unroll
-  for (int d = 16; d; d >>= 1) {
-    cnt += __shfl_xor_sync(FULL, cnt, d);
-    evs += __shfl_xor_sync(FULL, evs, d);
-  }
-  if (lane == 0) { S.wcnt[warp] = cnt; S.wev[warp] = evs; }
-  __syncthreads();
-  uint32_t cbase = 0, ebase = 0, ctot = 0, etot = 0;
-#pragma unroll
-  for (int w = 0; w < RT / 32; ++w) {
-    if ((uint32_t)w < warp) { cbase += S.wcnt[w]; ebase += S.wev[w]; }
-    ctot += S.wcnt[w]; etot += S.wev[w];
-  }
-  const uint32_t lt = lanemask_lt();
-  for (uint32_t c = c0; c < c1; c += 32) {
-    const uint32_t cc = c + lane;
-    uint32_t st = 0, len = 0;
-    if (cc < c1) { st = row0[cc]; len = (uint32_t)row1[cc] - st; }
-    const uint32_t nz = __ballot_sync(FULL, len != 0);
+  const uint32_t f0 = p.seg_first[b], ne = p.seg_first[b + 1] - f0;
+  uint32_t carry = 0;
+  for (uint32_t base = 0; base < ne; base += RT) {
+    const uint32_t i = base + threadIdx.x;
+    uint32_t len = 0, gs = 0;
+    if (i < ne) {
+      const uint4 e = p.segs[f0 + i];                  // {chunk, bucket, start | len << 16, 0}
+      len = e.z >> 16;
+      gs = e.x * (uint32_t)kChunkCap + (e.z & 0xFFFFu);
+    }
     uint32_t incl = len;
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
       const uint32_t o = __shfl_up_sync(FULL, incl, d);
       if (lane >= (uint32_t)d) incl += o;
     }
-    if (len) {
-      const uint32_t idx = cbase + __popc(nz & lt);
-      sstart[idx] = cc * (uint32_t)kChunkCap + st;
-      scum[idx] = ebase + incl - len;
-    }
-    cbase += __popc(nz);
-    ebase += __shfl_sync(FULL, incl, 31);
+    if (lane == 31) S.wev[warp] = incl;
+    __syncthreads();
+    uint32_t wpre = 0, tot = 0;
+#pragma unroll
+    for (int w = 0; w < RT / 32; ++w) { const uint32_t x = S.wev[w]; if ((uint32_t)w < warp) wpre += x; tot += x; }
+    if (i < ne) { sstart[i] = gs; scum[i] = carry + wpre + incl - len; }
+    carry += tot;
+    __syncthreads();
   }
-  if (threadIdx.x == 0) { scum[ctot] = etot; S.n_segs = ctot; S.n_events = etot; }
+  if (threadIdx.x == 0) { scum[ne] = carry; S.n_segs = ne; S.n_events = carry; }
   __syncthreads();
 }
 
@@ -486,15 +468,22 @@ __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t 
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t nwin = S.nwin;
   const uint32_t m = min(min((uint32_t)STEP, total - e0), S.wcum[nwin] - e0);
-  uint32_t a0, a1;                                  // window segments [a0, a1) hold the events
-  {
-    uint32_t a = 0, z = nwin;
-    while (z - a > 1) { const uint32_t mid = (a + z) >> 1; if (S.wcum[mid] <= e0) a = mid; else z = mid; }
-    a0 = a;
-    a = a0; z = nwin;
-    while (z - a > 1) { const uint32_t mid = (a + z) >> 1; if (S.wcum[mid] < e0 + m) a = mid; else z = mid; }
-    a1 = a + 1;
+  // window segments [a0, a1) hold the events: warp 0 searches, everyone reads
+  if (warp == 0) {
+    // lane-parallel search: segment j holds e iff wcum[j] <= e < wcum[j+1]
+    uint32_t a0 = 0, a1 = 0;
+    for (uint32_t base = 0; base < nwin; base += 32) {
+      const uint32_t j = base + lane;
+      const bool le0 = j < nwin && S.wcum[j] <= e0;
+      const bool lt1 = j < nwin && S.wcum[j] < e0 + m;
+      a0 += __popc(__ballot_sync(FULL, le0));
+      a1 += __popc(__ballot_sync(FULL, lt1));
+      if (!__any_sync(FULL, lt1)) break;
+    }
+    if (lane == 0) { S.ga0 = a0 - 1; S.ga1 = a1; }
   }
+  __syncthreads();
+  const uint32_t a0 = S.ga0, a1 = S.ga1;
   if ((a1 - a0) * 16 <= m) {
     // long segments: one warp streams one segment at a time
     for (uint32_t j = a0 + warp; j < a1; j += RT / 32) {
