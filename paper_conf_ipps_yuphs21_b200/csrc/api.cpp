@@ -68,7 +68,7 @@ struct arb_ctx_s {
   uint32_t bucket_bits = 0, n_buckets = 0, coarse_bits = 0, n_bins = 0;
   std::vector<uint32_t> bin_map, order, hist;
   std::vector<uint64_t> bucket_start;
-  DevBuf<uint32_t> d_bin_map, d_order, d_hist, d_seg, d_cut;
+  DevBuf<uint32_t> d_bin_map, d_order, d_hist, d_seg, d_cut, d_cutscr;
   DevBuf<uint64_t> d_bucket_start;
   int n_sms = 148;
   uint8_t* shadow = nullptr;
@@ -309,9 +309,10 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     // cut balanced buckets on the device; the histogram becomes the bin map in place
     CK(ctx->d_bucket_start.ensure(kMaxBuckets + 1), "alloc buckets");
     CK(ctx->d_cut.ensure(2 * kMaxBuckets + 2), "alloc cut scratch");
+    CK(ctx->d_cutscr.ensure(2 * ((ctx->n_bins + 1023) / 1024) + 4 + ctx->n_bins), "alloc cut scratch");
     CK(launch_cut(ctx->d_hist.p, ctx->n_bins, ctx->coarse_bits, ctx->n_words, kMaxBuckets, ctx->d_bucket_start.p,
-                  ctx->d_cut.p, ctx->d_cut.p + kMaxBuckets, ctx->d_cut.p + 2 * kMaxBuckets, s), "k_cut");
-    launches += 1;
+                  ctx->d_cut.p, ctx->d_cut.p + kMaxBuckets, ctx->d_cut.p + 2 * kMaxBuckets, ctx->d_cutscr.p, s,
+                  &launches), "k_cut");
     uint32_t nb = 0;
     CK(cudaMemcpyAsync(&nb, ctx->d_cut.p + 2 * kMaxBuckets, 4, cudaMemcpyDeviceToHost, s), "nb d2h");
     CK(cudaStreamSynchronize(s), "cut sync");

@@ -142,9 +142,10 @@ struct MirParams {
 
 // ---- kernel launchers (kernels.cu) -----------------------------------------
 cudaError_t launch_sample(const SampleParams& p, uint64_t n_samples, cudaStream_t s);
+// scratch: 2 * ceil(n_bins / 1024) + 4 + n_bins u32
 cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits, uint64_t n_words,
                        uint32_t max_buckets, uint64_t* bucket_start, uint32_t* weight, uint32_t* first_bin,
-                       uint32_t* nb_out, cudaStream_t s);
+                       uint32_t* nb_out, uint32_t* scratch, cudaStream_t s, int* launches);
 cudaError_t launch_partition(const PartParams& p, cudaStream_t s);
 cudaError_t launch_sort_segments(uint4* a, uint4* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
                                  uint32_t* first, uint4** sorted, cudaStream_t s, int* launches);

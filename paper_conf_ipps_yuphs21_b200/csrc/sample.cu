@@ -1,40 +1,40 @@
 // sample.cu — address sampling and device-side bucket cutting (bucket balancing).
 //
-// k_sample  sampled histogram of access addresses over coarse bins.
-// k_cut     single CTA: contiguous, event-balanced address buckets (quantile
-//           cuts of the sampled histogram + span cuts), bin map in place.
+// k_sample   sampled histogram of access addresses over coarse bins.
+// k_cut_*    contiguous, event-balanced address buckets: a bucket starts at
+//            bin 0, at every bin whose exclusive sample prefix enters a new
+//            quantile level (a heavy bin gets a bucket of its own) and at every
+//            2^30-word span boundary.  The histogram is rewritten in place as
+//            the bin map (bucket | offset-in-bins << 10, see arb_internal.h).
+//            Tiles of 1024 bins are handled by separate CTAs; two one-CTA
+//            scans carry the prefixes between tiles.
 #include "kcommon.cuh"
 
 namespace arb {
 
-// Sampled histogram of access addresses over coarse bins (bucket balancing).
 __global__ void k_sample(SampleParams p, uint64_t n_samples) {
   for (uint64_t k = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; k < n_samples;
        k += (uint64_t)gridDim.x * blockDim.x) {
-    uint4 r = ld_stream(p.ev + k * p.stride);
-    uint64_t w0 = (uint64_t)r.x | ((uint64_t)r.y << 32);
+    const uint4 r = ld_stream(p.ev + k * p.stride);
+    const uint64_t w0 = (uint64_t)r.x | ((uint64_t)r.y << 32);
     if (((w0 >> 48) & 0xFFu) >= 4) continue;
-    uint64_t x = (w0 & kMask48) >> 3;
-    uint64_t rel = x - p.base_word;
+    const uint64_t x = (w0 & kMask48) >> 3;
+    const uint64_t rel = x - p.base_word;
     if (x >= p.base_word && rel < p.n_words) atomicAdd(&p.hist[rel >> p.coarse_bits], 1u);
   }
 }
 
 cudaError_t launch_sample(const SampleParams& p, uint64_t n_samples, cudaStream_t s) {
   if (!n_samples) return cudaSuccess;
-  uint64_t g = (n_samples + 255) / 256;
+  const uint64_t g = (n_samples + 255) / 256;
   k_sample<<<(unsigned)(g > 148 * 16 ? 148 * 16 : g), 256, 0, s>>>(p, n_samples);
   return cudaGetLastError();
 }
 
-// ---- bucket cutting on the device (single CTA) ------------------------------
-// Buckets start at bin 0, at every bin whose exclusive sample prefix crosses a
-// multiple of `target` (quantile cuts: a heavy bin gets a bucket of its own),
-// and at every multiple of 2^30 words (span cap).  Writes bin_map (see
-// arb_internal.h), bucket_start [nb + 1], bucket weights [nb] and nb.
-constexpr int kCutThreads = 1024;
+constexpr int kT = 1024;   // bins per tile = threads per CTA
 
-__device__ uint32_t cta_excl_scan(uint32_t v, uint32_t* ws, uint32_t* total) {
+// exclusive block scan of one value per thread (1024 threads)
+__device__ __forceinline__ uint32_t scan1024(uint32_t v, uint32_t* ws, uint32_t* total) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   uint32_t incl = v;
 #pragma unroll
@@ -42,7 +42,6 @@ __device__ uint32_t cta_excl_scan(uint32_t v, uint32_t* ws, uint32_t* total) {
     const uint32_t o = __shfl_up_sync(FULL, incl, d);
     if (lane >= (uint32_t)d) incl += o;
   }
-  __syncthreads();
   if (lane == 31) ws[warp] = incl;
   __syncthreads();
   if (warp == 0) {
@@ -58,84 +57,135 @@ __device__ uint32_t cta_excl_scan(uint32_t v, uint32_t* ws, uint32_t* total) {
   }
   __syncthreads();
   *total = ws[32];
-  return ws[warp] + incl - v;
+  const uint32_t r = ws[warp] + incl - v;
+  __syncthreads();
+  return r;
 }
 
-__global__ void __launch_bounds__(kCutThreads) k_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits,
-                                                      uint64_t n_words, uint32_t max_buckets,
-                                                      uint64_t* bucket_start, uint32_t* weight,
-                                                      uint32_t* first_bin, uint32_t* nb_out) {
+struct CutArgs {
+  uint32_t* hist_map; uint32_t n_bins; uint32_t coarse_bits; uint64_t n_words; uint32_t max_buckets;
+  uint64_t* bucket_start; uint32_t* weight; uint32_t* first_bin; uint32_t* nb_out;
+  uint32_t* tile_a; uint32_t* tile_b;          // per-tile scratch (sums / flag counts, then prefixes)
+  uint32_t* misc;                              // [0] total, [1] target, [2] span bins
+  uint32_t* bucket_of;                         // per bin bucket index
+};
+
+__global__ void __launch_bounds__(kT) k_cut_sum(CutArgs a) {
   __shared__ uint32_t ws[33];
-  const uint32_t per = (n_bins + kCutThreads - 1) / kCutThreads;
-  const uint32_t i0 = min(n_bins, threadIdx.x * per), i1 = min(n_bins, i0 + per);
-  uint32_t s = 0;
-  for (uint32_t i = i0; i < i1; ++i) s += hist_map[i];
-  uint32_t total;
-  const uint32_t pre = cta_excl_scan(s, ws, &total);
-  const uint32_t levels = max(1u, max_buckets - 124);            // <= levels quantile cuts (+ span cuts <= 1024)
-  const uint32_t target = max(1u, (total + levels - 1) / levels);
-  const uint64_t span64 = (1ull << 30) >> coarse_bits;
-  const uint32_t span_bins = span64 == 0 ? 1u : (span64 > 0xFFFFFFFFull ? 0xFFFFFFFFu : (uint32_t)span64);
-  // a bucket starts at bin i when the quantile level of its exclusive prefix
-  // differs from the previous bin's, or at a span boundary
-  const uint32_t lev0 = (i0 == 0 || i0 >= n_bins) ? 0xFFFFFFFFu : (pre - hist_map[i0 - 1]) / target;
-  uint32_t nflag = 0;
-  {
-    uint32_t p = pre, prev = lev0;
-    for (uint32_t i = i0; i < i1; ++i) {
-      const uint32_t lev = p / target;
-      nflag += (i == 0 || i % span_bins == 0 || lev != prev);
-      prev = lev;
-      p += hist_map[i];
+  const uint32_t i = blockIdx.x * kT + threadIdx.x;
+  uint32_t tot;
+  scan1024(i < a.n_bins ? a.hist_map[i] : 0, ws, &tot);
+  if (threadIdx.x == 0) a.tile_a[blockIdx.x] = tot;
+}
+
+// one CTA: exclusive scan of n per-tile values in place; optional totals
+__global__ void __launch_bounds__(kT) k_cut_scan(uint32_t* v, uint32_t n, uint32_t* total_out, CutArgs a,
+                                                 int first) {
+  __shared__ uint32_t ws[33];
+  uint32_t carry = 0;
+  for (uint32_t base = 0; base < n; base += kT) {
+    const uint32_t i = base + threadIdx.x;
+    uint32_t tot;
+    const uint32_t ex = scan1024(i < n ? v[i] : 0, ws, &tot);
+    if (i < n) v[i] = carry + ex;
+    carry += tot;
+  }
+  if (threadIdx.x == 0) {
+    *total_out = carry;
+    if (first) {   // quantile target and span cap
+      const uint32_t levels = max(1u, a.max_buckets - 124);
+      a.misc[1] = max(1u, (carry + levels - 1) / levels);
+      const uint64_t span64 = (1ull << 30) >> a.coarse_bits;
+      a.misc[2] = span64 == 0 ? 1u : (span64 > 0xFFFFFFFFull ? 0xFFFFFFFFu : (uint32_t)span64);
     }
   }
-  uint32_t nb;
-  uint32_t b = cta_excl_scan(nflag, ws, &nb);
-  {
-    uint32_t p = pre, prev = lev0;
-    for (uint32_t i = i0; i < i1; ++i) {
-      const uint32_t lev = p / target;
-      if (i == 0 || i % span_bins == 0 || lev != prev) { first_bin[b] = i; weight[b] = p; ++b; }
-      prev = lev;
-      p += hist_map[i];
-    }
+}
+
+// flags of the bins of one tile (needs the tile's exclusive sample prefix)
+__device__ __forceinline__ bool cut_flag(const CutArgs& a, uint32_t i, uint32_t p, uint32_t h_prev_known,
+                                         uint32_t* levs) {
+  const uint32_t target = a.misc[1], span = a.misc[2];
+  const uint32_t lev = p / target;
+  levs[threadIdx.x] = lev;
+  __syncthreads();
+  uint32_t prev;
+  if (threadIdx.x > 0) prev = levs[threadIdx.x - 1];
+  else prev = i == 0 ? 0xFFFFFFFFu : (p - h_prev_known) / target;   // level of the previous tile's last bin
+  __syncthreads();
+  return i < a.n_bins && (i == 0 || i % span == 0 || lev != prev);
+}
+
+__global__ void __launch_bounds__(kT) k_cut_flags(CutArgs a) {
+  __shared__ uint32_t ws[33];
+  __shared__ uint32_t levs[kT];
+  const uint32_t i = blockIdx.x * kT + threadIdx.x;
+  const uint32_t h = i < a.n_bins ? a.hist_map[i] : 0;
+  uint32_t tot;
+  const uint32_t p = a.tile_a[blockIdx.x] + scan1024(h, ws, &tot);
+  const uint32_t hprev = (i > 0 && threadIdx.x == 0) ? a.hist_map[i - 1] : 0;
+  const bool f = cut_flag(a, i, p, hprev, levs);
+  uint32_t nf;
+  scan1024(f ? 1u : 0u, ws, &nf);
+  if (threadIdx.x == 0) a.tile_b[blockIdx.x] = nf;
+}
+
+__global__ void __launch_bounds__(kT) k_cut_write(CutArgs a) {
+  __shared__ uint32_t ws[33];
+  __shared__ uint32_t levs[kT];
+  const uint32_t i = blockIdx.x * kT + threadIdx.x;
+  const uint32_t h = i < a.n_bins ? a.hist_map[i] : 0;
+  uint32_t tot;
+  const uint32_t p = a.tile_a[blockIdx.x] + scan1024(h, ws, &tot);
+  const uint32_t hprev = (i > 0 && threadIdx.x == 0) ? a.hist_map[i - 1] : 0;
+  const bool f = cut_flag(a, i, p, hprev, levs);
+  uint32_t nf;
+  const uint32_t b = a.tile_b[blockIdx.x] + scan1024(f ? 1u : 0u, ws, &nf);
+  if (f) { a.first_bin[b] = i; a.weight[b] = p; }
+  if (i < a.n_bins) a.bucket_of[i] = f ? b : b - 1;
+}
+
+__global__ void k_cut_map(CutArgs a) {
+  const uint32_t nb = *a.nb_out, total = a.misc[0];
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < a.n_bins; i += gridDim.x * blockDim.x) {
+    const uint32_t b = a.bucket_of[i];
+    a.hist_map[i] = b | ((i - a.first_bin[b]) << 10);
   }
-  __syncthreads();
-  for (uint32_t k = threadIdx.x; k < nb; k += kCutThreads) bucket_start[k] = (uint64_t)first_bin[k] << coarse_bits;
-  __syncthreads();
-  uint32_t wk[4];   // weights = differences of the prefixes at the starts (nb <= 4096)
+  for (uint32_t b = blockIdx.x * blockDim.x + threadIdx.x; b <= nb; b += gridDim.x * blockDim.x) {
+    if (b < nb) a.bucket_start[b] = (uint64_t)a.first_bin[b] << a.coarse_bits;
+    else a.bucket_start[nb] = a.n_words;
+  }
+}
+
+__global__ void k_cut_weights(CutArgs a) {   // one CTA: prefix differences
+  const uint32_t nb = *a.nb_out, total = a.misc[0];
+  uint32_t w[4];
 #pragma unroll
   for (int j = 0; j < 4; ++j) {
-    const uint32_t k = threadIdx.x + j * kCutThreads;
-    wk[j] = k < nb ? (k + 1 < nb ? weight[k + 1] : total) - weight[k] : 0;
+    const uint32_t b = threadIdx.x + j * blockDim.x;
+    w[j] = b < nb ? (b + 1 < nb ? a.weight[b + 1] : total) - a.weight[b] : 0;
   }
   __syncthreads();
 #pragma unroll
   for (int j = 0; j < 4; ++j) {
-    const uint32_t k = threadIdx.x + j * kCutThreads;
-    if (k < nb) weight[k] = wk[j];
+    const uint32_t b = threadIdx.x + j * blockDim.x;
+    if (b < nb) a.weight[b] = w[j];
   }
-  {
-    // bin map: walk this thread's bins again; b = number of bucket starts before i0
-    uint32_t p = pre, prev = lev0;
-    int cur = (int)(b - nflag) - 1;                         // bucket open at i0 - 1 (-1: none)
-    uint32_t first = (cur >= 0 && i0 < i1) ? first_bin[cur] : 0;
-    for (uint32_t i = i0; i < i1; ++i) {
-      const uint32_t lev = p / target;
-      if (i == 0 || i % span_bins == 0 || lev != prev) { ++cur; first = i; }
-      prev = lev;
-      p += hist_map[i];
-      hist_map[i] = cur | ((i - first) << 10);
-    }
-  }
-  if (threadIdx.x == 0) { bucket_start[nb] = n_words; *nb_out = nb; }
 }
 
 cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits, uint64_t n_words,
                        uint32_t max_buckets, uint64_t* bucket_start, uint32_t* weight, uint32_t* first_bin,
-                       uint32_t* nb_out, cudaStream_t s) {
-  k_cut<<<1, kCutThreads, 0, s>>>(hist_map, n_bins, coarse_bits, n_words, max_buckets, bucket_start, weight,
-                                  first_bin, nb_out);
+                       uint32_t* nb_out, uint32_t* scratch, cudaStream_t s, int* launches) {
+  const uint32_t nt = (n_bins + kT - 1) / kT;
+  CutArgs a{hist_map, n_bins, coarse_bits, n_words, max_buckets, bucket_start, weight, first_bin, nb_out,
+            scratch, scratch + nt, scratch + 2 * nt, scratch + 2 * nt + 4};
+  k_cut_sum<<<nt, kT, 0, s>>>(a);
+  k_cut_scan<<<1, kT, 0, s>>>(a.tile_a, nt, a.misc, a, 1);
+  k_cut_flags<<<nt, kT, 0, s>>>(a);
+  k_cut_scan<<<1, kT, 0, s>>>(a.tile_b, nt, nb_out, a, 0);
+  k_cut_write<<<nt, kT, 0, s>>>(a);
+  k_cut_map<<<148, 1024, 0, s>>>(a);
+  k_cut_weights<<<1, kT, 0, s>>>(a);
+  *launches += 7;
   return cudaGetLastError();
 }
 
