@@ -9,7 +9,7 @@
 // steps of <= 2048 that never straddle a range op:
 //
 //   fast step  (every word has at most one write in the step): a shared-memory
-//              hash word -> (first write, state before the step).  A read's
+//              hash of the written words, word -> write position.  A read's
 //              state-before is the initial state, or the image of the one
 //              write when that write precedes it; the word's final state is
 //              the image of the write (reads do not change the state).
@@ -36,7 +36,7 @@ struct ReplaySmem {
   uint2 ev[2][STEP];              // double-buffered step events {key, pos} (cp.async)
   union {
     struct { uint32_t keyA[STEP], posA[STEP], keyB[STEP], posB[STEP]; uint16_t hist[RT / 32][256]; } s;
-    struct { uint32_t key[kHSlots], wpos[kHSlots]; uint8_t st[kHSlots]; } h;      // fast step
+    struct { uint32_t key[kHSlots], wpos[kHSlots]; } h;      // fast step: written words only
   } u;
   uint32_t wstart[kWin];          // staged segment list window: global event index
   uint32_t wcum[kWin + 1];        //   and bucket-relative first event of each segment
@@ -175,15 +175,19 @@ __device__ __forceinline__ void hash_clear(ReplaySmem& S) {
 
 // ---- fast step: at most one write per word -------------------------------------------
 // Returns false (and leaves the shadow untouched) if some word has two writes.
+//
+// Only writes enter the hash (word -> first write position | kind): reads do
+// not change the state, so a read's state-before is the state loaded
+// at the start of the step, or — if its word's single write precedes it — the
+// image of that write; the write event itself commits the word's final state.
 __device__ bool step_fast(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
   uint32_t slot[RI], word[RI], pos[RI], op[RI], s_pre[RI];
-  bool own[RI];
   bool multi = false;
   const uint64_t bb = S.bucket_base;
 #pragma unroll
   for (int j = 0; j < RI; ++j) {   // shadow loads first: their latency overlaps the hashing
     const uint32_t i = threadIdx.x + j * RT;
-    own[j] = false; slot[j] = 0; word[j] = 0; pos[j] = 0; op[j] = 0xFFu; s_pre[j] = 0;
+    slot[j] = 0; word[j] = 0; pos[j] = 0; op[j] = 0xFFu; s_pre[j] = 0;
     if (i < m) {
       const uint2 e = ev[i];
       word[j] = e.x & kWordMask; op[j] = e.x >> 30; pos[j] = e.y;
@@ -192,50 +196,53 @@ __device__ bool step_fast(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
   }
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
-    if (op[j] != 0xFFu) {
+    if (op[j] == OP_WH || op[j] == OP_WT) {
       uint32_t h = (word[j] * 2654435761u) >> 20;          // 12 bits
       for (;;) {
         const uint32_t old = atomicCAS(&S.u.h.key[h], kEmpty, word[j]);
-        if (old == kEmpty) { own[j] = true; break; }
-        if (old == word[j]) break;
+        if (old == kEmpty) break;
+        if (old == word[j]) { multi = true; break; }        // a second write of the word
         h = (h + 1) & (kHSlots - 1);
       }
       slot[j] = h;
-      if (op[j] == OP_WH || op[j] == OP_WT) {
-        const uint32_t o = atomicMin(&S.u.h.wpos[h], (pos[j] << 2) | (op[j] == OP_WH ? 1u : 2u));
-        if (o != kEmpty) multi = true;
-      }
+      S.u.h.wpos[h] = (pos[j] << 2) | (op[j] == OP_WH ? 1u : 2u);
     }
   }
   if (__syncthreads_or(multi)) {
 #pragma unroll
     for (int j = 0; j < RI; ++j)
-      if (own[j]) { S.u.h.key[slot[j]] = kEmpty; S.u.h.wpos[slot[j]] = kEmpty; }
+      if (op[j] == OP_WH || op[j] == OP_WT) { S.u.h.key[slot[j]] = kEmpty; S.u.h.wpos[slot[j]] = kEmpty; }
     __syncthreads();
     return false;
   }
-#pragma unroll
-  for (int j = 0; j < RI; ++j)
-    if (own[j]) S.u.h.st[slot[j]] = s_pre[j] & 15u;
-  __syncthreads();
   uint32_t fk[RI];
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
     fk[j] = 0;
-    if (op[j] == 0xFFu) continue;
-    const uint32_t s0 = S.u.h.st[slot[j]], wp = S.u.h.wpos[slot[j]];
-    const bool hasw = wp != kEmpty;
-    const uint32_t after = hasw ? vsm_write(wp & 3u, s0) : s0;
-    const uint32_t before = (hasw && (wp >> 2) < pos[j]) ? after : s0;
-    fk[j] = classify(op[j], before);
-    if (own[j]) __stcg(p.shadow + bb + word[j], (uint8_t)after);
+    const uint32_t s0 = s_pre[j] & 15u;
+    if (op[j] == OP_RH || op[j] == OP_RT) {
+      uint32_t h = (word[j] * 2654435761u) >> 20, before = s0;
+      for (;;) {                                            // probe for the word's write
+        const uint32_t k = S.u.h.key[h];
+        if (k == kEmpty) break;
+        if (k == word[j]) {
+          const uint32_t wp = S.u.h.wpos[h];
+          if ((wp >> 2) < pos[j]) before = vsm_write(wp & 3u, s0);
+          break;
+        }
+        h = (h + 1) & (kHSlots - 1);
+      }
+      fk[j] = classify(op[j], before);
+    } else if (op[j] != 0xFFu) {
+      __stcg(p.shadow + bb + word[j], (uint8_t)vsm_write(op[j] == OP_WH ? 1u : 2u, s0));
+    }
   }
   emit_faults(p, fk, word, pos, bb);
   __syncthreads();
 #pragma unroll
   for (int j = 0; j < RI; ++j)
-    if (own[j]) { S.u.h.key[slot[j]] = kEmpty; S.u.h.wpos[slot[j]] = kEmpty; }
-  __syncthreads();
+    if (op[j] == OP_WH || op[j] == OP_WT) { S.u.h.key[slot[j]] = kEmpty; S.u.h.wpos[slot[j]] = kEmpty; }
+  // the caller's next barrier orders this reset before the next step's inserts
   return true;
 }
 
