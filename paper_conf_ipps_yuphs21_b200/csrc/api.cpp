@@ -68,7 +68,7 @@ struct arb_ctx_s {
   uint32_t bucket_bits = 0, n_buckets = 0, coarse_bits = 0, n_bins = 0;
   std::vector<uint32_t> bin_map, order, hist;
   std::vector<uint64_t> bucket_start;
-  DevBuf<uint32_t> d_bin_map, d_order, d_hist, d_seg, d_cut, d_cutscr;
+  DevBuf<uint32_t> d_bin_map, d_order, d_hist, d_cut, d_cutscr;
   DevBuf<uint64_t> d_bucket_start;
   int n_sms = 148;
   uint8_t* shadow = nullptr;
@@ -201,7 +201,7 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   ctx->m_rr_cum.release(); ctx->m_ins_inst.release(); ctx->m_qry_open_start.release(); ctx->m_open_list.release();
   ctx->m_own_start.release(); ctx->m_win_start.release(); ctx->m_own.release(); ctx->m_win.release();
   ctx->m_rr.release(); ctx->hkeys.release(); ctx->hvals.release(); ctx->counts.release();
-  ctx->d_bin_map.release(); ctx->d_order.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_seg.release(); ctx->d_cut.release();
+  ctx->d_bin_map.release(); ctx->d_order.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_cut.release();
   for (auto& e : ctx->ev) if (e) cudaEventDestroy(e);
   if (ctx->nccl_lib) dlclose(ctx->nccl_lib);
   delete ctx;
@@ -338,7 +338,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   // ---- A1/A3a: decode + partition ------------------------------------------
   const uint32_t n_chunks = (uint32_t)((n + kChunkRecords - 1) / kChunkRecords);
   CK(ctx->part_ev.ensure((size_t)std::max<uint32_t>(n_chunks, 1) * kChunkCap), "alloc part_ev");
-  if (ctx->seg_cap < (uint64_t)n_chunks * 16) ctx->seg_cap = (uint64_t)n_chunks * 16;
+  if (ctx->seg_cap < (uint64_t)n_chunks * 2 + 4096) ctx->seg_cap = (uint64_t)n_chunks * 2 + 4096;
   CK(ctx->seg_a.ensure(std::max<uint64_t>(ctx->seg_cap, 1)), "alloc segments");
   DevStats hst;
   PartParams pp{};
@@ -400,7 +400,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     const uint64_t ns = hst.n_segs;
     CK(ctx->seg_b.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
     CK(ctx->seg_first.ensure(ctx->n_buckets + 1), "alloc seg_first");
-    CK(ctx->blk.ensure(std::max<uint64_t>((ns + 4095) / 4096 * 256, 1)), "alloc blk");
+    CK(ctx->blk.ensure((ns + 4095) / 4096 * 256 + 4096), "alloc blk");
     int cb = 1;
     while (cb < 32 && ((uint64_t)n_chunks >> cb)) ++cb;
     uint4* a = ctx->seg_a.p;
@@ -408,15 +408,12 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     CK(launch_sort_segments(a, b2, ns, cb, ctx->n_buckets, ctx->blk.p, ctx->seg_first.p, &segs_sorted, s, &launches),
        "sort segments");
   }
-  rp.part_ev = ctx->part_ev.p; rp.segs = segs_sorted; rp.seg_first = ctx->seg_first.p; rp.n_chunks = n_chunks;
+  rp.part_ev = ctx->part_ev.p; rp.segs = segs_sorted; rp.seg_first = ctx->seg_first.p;
   rp.n_buckets = ctx->n_buckets; rp.bucket_bits = ctx->bucket_bits; rp.n_words = ctx->n_words;
   rp.bucket_start = ctx->d_bucket_start.p; rp.order = ctx->d_order.p;
   rp.shadow = ctx->shadow; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
   rp.cand = ctx->cand.p; rp.cand_cap = ctx->cand_cap; rp.st = ctx->dstats.p;
   int n_ctas = std::max(1, std::min<int>((int)ctx->n_buckets, ctx->n_sms * kReplayCtasPerSm));
-  CK(ctx->d_seg.ensure((size_t)2 * n_ctas * (n_chunks + 1)), "alloc segment lists");
-  rp.seg_start = ctx->d_seg.p;
-  rp.seg_cum = ctx->d_seg.p + (size_t)n_ctas * (n_chunks + 1);
   CK(launch_replay(rp, std::max(n_ctas, 1), s), "k_replay");
   launches += 1;
   if (timing) cudaEventRecord(ctx->ev[3], s);
@@ -480,7 +477,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   CK(ctx->cand_tmp.ensure(std::max<uint64_t>(n_cand, 1)), "alloc cand tmp");
   CK(ctx->reports.ensure(std::max<uint64_t>(n_cand, 1)), "alloc reports");
   uint64_t nblk = (n_cand + 4095) / 4096;
-  CK(ctx->blk.ensure(std::max<uint64_t>(nblk * 256, 1)), "alloc blk");
+  CK(ctx->blk.ensure(nblk * 256 + 4096), "alloc blk");
   CompactParams cp{};
   cp.cand = ctx->cand.p; cp.n_cand = n_cand; cp.tmp = ctx->cand_tmp.p; cp.blk = ctx->blk.p;
   cp.blk_cap = ctx->blk.cap; cp.base_word = ctx->base_word;

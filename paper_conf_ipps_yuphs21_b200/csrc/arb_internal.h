@@ -41,7 +41,7 @@ constexpr uint32_t kMaxBatchRecords = 1u << 30;
 // ---- partition geometry ----------------------------------------------------
 constexpr int kPartThreads = 512;
 constexpr int kPartWarps = kPartThreads / 32;
-constexpr int kChunkRecords = 4096;                 // records per chunk (one CTA)
+constexpr int kChunkRecords = 256;                  // records per chunk (one warp, independently)
 constexpr int kChunkCap = 2 * kChunkRecords;        // events per chunk (<= 2 words per access)
 constexpr int kMaxBuckets = 1024;
 
@@ -100,19 +100,19 @@ struct PartParams {
   uint32_t bucket_bits, n_buckets;
   uint32_t n_chunks;
   uint2* part_ev;                         // [n_chunks][kChunkCap]
-  uint4* seg_out; uint64_t seg_cap;       // {chunk, bucket, start | len << 16, 0} per touched bucket
+  uint4* seg_out; uint64_t seg_cap;       // {chunk, bucket, start | len << 16, -} per touched bucket
   CtlRec* ctl; uint64_t ctl_cap;
   DevStats* st;
 };
 
 struct ReplayParams {
   const uint2* part_ev;
-  const uint4* segs;                      // segment entries sorted by (bucket, chunk)
+  const uint4* segs;                      // segment entries sorted by (bucket, chunk); .w = exclusive
+                                          // prefix of the event counts over the sorted array
   const uint32_t* seg_first;              // [n_buckets + 1] first entry of each bucket
-  uint32_t n_chunks, n_buckets, bucket_bits;
+  uint32_t n_buckets, bucket_bits;
   const uint64_t* bucket_start;           // [n_buckets + 1] first relative word of each bucket
   const uint32_t* order;                  // buckets in scheduling order (largest first)
-  uint32_t* seg_start; uint32_t* seg_cum; // per-CTA scratch: [gridDim][n_chunks + 1] segment list
   uint64_t n_words;
   uint8_t* shadow;                        // n_words bytes
   const uint32_t* ops_start;              // [n_buckets + 1]
@@ -147,6 +147,8 @@ cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits
                        uint32_t max_buckets, uint64_t* bucket_start, uint32_t* weight, uint32_t* first_bin,
                        uint32_t* nb_out, uint32_t* scratch, cudaStream_t s, int* launches);
 cudaError_t launch_partition(const PartParams& p, cudaStream_t s);
+// sorts the segment entries by (bucket, chunk), writes each entry's exclusive
+// event prefix into .w and each bucket's first entry; cnt: (n / 4096 + 1) * 256 u32
 cudaError_t launch_sort_segments(uint4* a, uint4* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
                                  uint32_t* first, uint4** sorted, cudaStream_t s, int* launches);
 cudaError_t launch_replay(const ReplayParams& p, int n_ctas, cudaStream_t s);

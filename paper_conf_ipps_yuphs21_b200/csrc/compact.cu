@@ -26,37 +26,79 @@ __global__ void __launch_bounds__(kRsThreads) k_rs_hist(const uint4* in, uint64_
   for (int d = threadIdx.x; d < 256; d += kRsThreads) cnt[(uint64_t)d * nblk + blockIdx.x] = h[d];
 }
 
-// exclusive scan of n u32 values in place (single CTA)
-__global__ void __launch_bounds__(1024) k_scan_inplace(uint32_t* a, uint64_t n) {
-  __shared__ uint32_t ws[32];
-  __shared__ uint32_t carry;
-  if (threadIdx.x == 0) carry = 0;
-  __syncthreads();
+// ---- exclusive scan of u32 values in place ------------------------------------------
+// A tile is 16K values: 1024 threads owning 16 consecutive values each.
+constexpr int kScanV = 16;
+constexpr uint64_t kScanTile = 1024 * kScanV;
+
+// scans a[base, base + kScanTile) ∩ [0, n) starting from `carry`; returns the
+// running total after the tile (valid in every thread)
+__device__ uint32_t scan_tile(uint32_t* a, uint64_t base, uint64_t n, uint32_t carry, uint32_t* ws) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  for (uint64_t base = 0; base < n; base += 1024) {
-    uint64_t i = base + threadIdx.x;
-    uint32_t v = i < n ? a[i] : 0, incl = v;
-    for (int d = 1; d < 32; d <<= 1) {
-      uint32_t o = __shfl_up_sync(FULL, incl, d);
-      if (lane >= (uint32_t)d) incl += o;
-    }
-    if (lane == 31) ws[warp] = incl;
-    __syncthreads();
-    if (warp == 0) {
-      uint32_t x = ws[lane], xi = x;
-      for (int d = 1; d < 32; d <<= 1) {
-        uint32_t o = __shfl_up_sync(FULL, xi, d);
-        if (lane >= (uint32_t)d) xi += o;
-      }
-      ws[lane] = xi - x;
-    }
-    __syncthreads();
-    uint32_t c = carry;
-    if (i < n) a[i] = c + ws[warp] + incl - v;
-    __syncthreads();
-    if (threadIdx.x == 1023) carry = c + ws[warp] + incl;
-    __syncthreads();
+  const uint64_t i0 = base + (uint64_t)threadIdx.x * kScanV;
+  uint32_t v[kScanV], s = 0;
+#pragma unroll
+  for (int j = 0; j < kScanV; ++j) { v[j] = i0 + j < n ? a[i0 + j] : 0; s += v[j]; }
+  uint32_t incl = s;
+  for (int d = 1; d < 32; d <<= 1) {
+    uint32_t o = __shfl_up_sync(FULL, incl, d);
+    if (lane >= (uint32_t)d) incl += o;
   }
+  if (lane == 31) ws[warp] = incl;
+  __syncthreads();
+  if (warp == 0) {
+    uint32_t x = ws[lane], xi = x;
+    for (int d = 1; d < 32; d <<= 1) {
+      uint32_t o = __shfl_up_sync(FULL, xi, d);
+      if (lane >= (uint32_t)d) xi += o;
+    }
+    ws[lane] = xi - x;
+    if (lane == 31) ws[32] = xi;
+  }
+  __syncthreads();
+  uint32_t run = carry + ws[warp] + incl - s;
+#pragma unroll
+  for (int j = 0; j < kScanV; ++j) {
+    if (i0 + j < n) a[i0 + j] = run;
+    run += v[j];
+  }
+  const uint32_t total = carry + ws[32];
+  __syncthreads();
+  return total;
+}
+
+// single CTA, tile after tile
+__global__ void __launch_bounds__(1024) k_scan_inplace(uint32_t* a, uint64_t n) {
+  __shared__ uint32_t ws[33];
+  uint32_t carry = 0;
+  for (uint64_t base = 0; base < n; base += kScanTile) carry = scan_tile(a, base, n, carry, ws);
+}
+// one CTA per tile: local scan, tile totals to tot[]
+__global__ void __launch_bounds__(1024) k_scan_tiles(uint32_t* a, uint64_t n, uint32_t* tot) {
+  __shared__ uint32_t ws[33];
+  const uint32_t t = scan_tile(a, blockIdx.x * kScanTile, n, 0, ws);
+  if (threadIdx.x == 0) tot[blockIdx.x] = t;
+}
+__global__ void __launch_bounds__(1024) k_scan_add(uint32_t* a, uint64_t n, const uint32_t* off) {
+  const uint32_t o = off[blockIdx.x];
+  if (!o) return;
+  const uint64_t i0 = blockIdx.x * kScanTile + (uint64_t)threadIdx.x * kScanV;
+#pragma unroll
+  for (int j = 0; j < kScanV; ++j)
+    if (i0 + j < n) a[i0 + j] += o;
+}
+// scratch: n / kScanTile + 1 values
+static void scan_u32(uint32_t* a, uint64_t n, uint32_t* scratch, cudaStream_t s, int* launches) {
+  const uint64_t nt = (n + kScanTile - 1) / kScanTile;
+  if (nt <= 1) {
+    k_scan_inplace<<<1, 1024, 0, s>>>(a, n);
+    *launches += 1;
+    return;
+  }
+  k_scan_tiles<<<(unsigned)nt, 1024, 0, s>>>(a, n, scratch);
+  k_scan_inplace<<<1, 1024, 0, s>>>(scratch, nt);
+  k_scan_add<<<(unsigned)nt, 1024, 0, s>>>(a, n, scratch);
+  *launches += 3;
 }
 
 __global__ void __launch_bounds__(kRsThreads) k_rs_scatter(const uint4* in, uint4* out, uint64_t n, RsPass ps,
@@ -145,6 +187,7 @@ __global__ void __launch_bounds__(kRsThreads) k_keep_write(const uint4* a, uint6
   uint32_t wpre = 0;
   for (uint32_t w = 0; w < warp; ++w) wpre += ws[w];
   uint64_t o = blk[blockIdx.x] + wpre + incl - c;
+  uint32_t kc[4] = {0, 0, 0, 0};
   for (int j = 0; j < kRsItems; ++j) {
     uint64_t i = base + (uint64_t)threadIdx.x * kRsItems + j;
     if (!kp[j]) continue;
@@ -154,11 +197,19 @@ __global__ void __launch_bounds__(kRsThreads) k_keep_write(const uint4* a, uint6
       uint64_t w0 = (word & kMask48) | ((uint64_t)x.w << 48);
       uint64_t w1 = gidx ? gidx[x.z] : index_base + x.z;
       out[o] = make_uint4((uint32_t)w0, (uint32_t)(w0 >> 32), (uint32_t)w1, (uint32_t)(w1 >> 32));
-      atomicAdd(&n_out[x.w & 3u], 1ull);   // per-kind counts in n_out[1..3]
+      kc[x.w & 3u]++;                      // per-kind counts in n_out[1..3]
     } else {
       out[o] = x;
     }
     ++o;
+  }
+  if (final_out) {
+#pragma unroll
+    for (int k = 1; k < 4; ++k) {
+      uint32_t v = kc[k];
+      for (int d = 16; d; d >>= 1) v += __shfl_xor_sync(FULL, v, d);
+      if (lane == 0 && v) atomicAdd(&n_out[k], (unsigned long long)v);
+    }
   }
   if (blockIdx.x == nblk - 1 && threadIdx.x == kRsThreads - 1) *n_out = o;
 }
@@ -168,9 +219,9 @@ static cudaError_t radix_sort(uint4*& a, uint4*& b, uint64_t n, const RsPass* pa
   uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
   for (int k = 0; k < np; ++k) {
     k_rs_hist<<<nblk, kRsThreads, 0, s>>>(a, n, passes[k], cnt, nblk);
-    k_scan_inplace<<<1, 1024, 0, s>>>(cnt, (uint64_t)nblk * 256);
+    scan_u32(cnt, (uint64_t)nblk * 256, cnt + (uint64_t)nblk * 256, s, launches);
     k_rs_scatter<<<nblk, kRsThreads, 0, s>>>(a, b, n, passes[k], cnt, nblk);
-    *launches += 3;
+    *launches += 2;
     uint4* t = a; a = b; b = t;
   }
   return cudaGetLastError();
@@ -190,9 +241,54 @@ __global__ void k_seg_first(const uint4* segs, uint64_t n, uint32_t n_buckets, u
   }
 }
 
-// Sort the partition's segment entries {chunk, bucket, start|len<<16, 0} by
-// (bucket, chunk) — stable LSD passes on the chunk then the bucket field — and
-// compute each bucket's first entry.  *sorted points at the result (a or b).
+// event count of each tile of segment entries (blocked: thread t owns 8 entries)
+__global__ void __launch_bounds__(kRsThreads) k_seg_tile_sum(const uint4* segs, uint64_t n, uint32_t* blk) {
+  __shared__ uint32_t red[kRsThreads / 32];
+  const uint64_t base = (uint64_t)blockIdx.x * kRsTile + (uint64_t)threadIdx.x * kRsItems;
+  uint32_t c = 0;
+#pragma unroll
+  for (int j = 0; j < kRsItems; ++j)
+    if (base + j < n) c += segs[base + j].z >> 16;
+  for (int d = 16; d; d >>= 1) c += __shfl_xor_sync(FULL, c, d);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = c;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t t = 0;
+    for (int w = 0; w < kRsThreads / 32; ++w) t += red[w];
+    blk[blockIdx.x] = t;
+  }
+}
+// .w = exclusive prefix of the event counts over the whole array
+__global__ void __launch_bounds__(kRsThreads) k_seg_cum(uint4* segs, uint64_t n, const uint32_t* blk) {
+  __shared__ uint32_t ws[kRsThreads / 32];
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint64_t base = (uint64_t)blockIdx.x * kRsTile + (uint64_t)threadIdx.x * kRsItems;
+  uint32_t len[kRsItems], c = 0;
+#pragma unroll
+  for (int j = 0; j < kRsItems; ++j) {
+    len[j] = base + j < n ? segs[base + j].z >> 16 : 0;
+    c += len[j];
+  }
+  uint32_t incl = c;
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint32_t o = __shfl_up_sync(FULL, incl, d);
+    if (lane >= (uint32_t)d) incl += o;
+  }
+  if (lane == 31) ws[warp] = incl;
+  __syncthreads();
+  uint32_t run = blk[blockIdx.x] + incl - c;
+  for (uint32_t w = 0; w < warp; ++w) run += ws[w];
+#pragma unroll
+  for (int j = 0; j < kRsItems; ++j) {
+    if (base + j < n) segs[base + j].w = run;
+    run += len[j];
+  }
+}
+
+// Sort the partition's segment entries {chunk, bucket, start|len<<16, -} by
+// (bucket, chunk) — stable LSD passes on the chunk then the bucket field —
+// write the exclusive event prefix into .w and compute each bucket's first
+// entry.  *sorted points at the result (a or b).
 cudaError_t launch_sort_segments(uint4* a, uint4* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
                                  uint32_t* first, uint4** sorted, cudaStream_t s, int* launches) {
   RsPass ps[8];
@@ -202,6 +298,13 @@ cudaError_t launch_sort_segments(uint4* a, uint4* b, uint64_t n, int chunk_bits,
   if (n) e = radix_sort(a, b, n, ps, np, cnt, s, launches);
   if (e != cudaSuccess) return e;
   *sorted = a;
+  if (n) {
+    const uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
+    k_seg_tile_sum<<<nblk, kRsThreads, 0, s>>>(a, n, cnt);
+    scan_u32(cnt, nblk, cnt + nblk, s, launches);
+    k_seg_cum<<<nblk, kRsThreads, 0, s>>>(a, n, cnt);
+    *launches += 2;
+  }
   k_seg_first<<<(n_buckets + 256) / 256, 256, 0, s>>>(a, n, n_buckets, first);
   *launches += 1;
   return cudaGetLastError();
@@ -226,9 +329,9 @@ cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches
     if ((e = radix_sort(a, b, n, ps, np, p.blk, s, launches)) != cudaSuccess) return e;
     uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
     k_keep_count<<<nblk, kRsThreads, 0, s>>>(a, n, 1, p.blk);
-    k_scan_inplace<<<1, 1024, 0, s>>>(p.blk, nblk);
+    scan_u32(p.blk, nblk, p.blk + nblk, s, launches);
     k_keep_write<<<nblk, kRsThreads, 0, s>>>(a, n, 1, p.blk, b, 0, 0, nullptr, 0, p.n_out, nblk);
-    *launches += 3;
+    *launches += 2;
     // the number kept is needed on the host side to continue; read it back
     unsigned long long kept = 0;
     cudaMemcpyAsync(&kept, p.n_out, sizeof(kept), cudaMemcpyDeviceToHost, s);
@@ -248,10 +351,10 @@ cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches
     return cudaGetLastError();
   }
   k_keep_count<<<nblk, kRsThreads, 0, s>>>(a, n, 0, p.blk);
-  k_scan_inplace<<<1, 1024, 0, s>>>(p.blk, nblk);
+  scan_u32(p.blk, nblk, p.blk + nblk, s, launches);
   k_keep_write<<<nblk, kRsThreads, 0, s>>>(a, n, 0, p.blk, p.out, 1, p.base_word, p.gidx, p.index_base,
                                            p.n_out, nblk);
-  *launches += 3;
+  *launches += 2;
   return cudaGetLastError();
 }
 

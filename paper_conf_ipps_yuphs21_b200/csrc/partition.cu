@@ -1,18 +1,20 @@
 // partition.cu — A1 (ingest/decode) + A3a (stable partition by address bucket).
 //
-// k_partition  persistent CTAs (one per SM), one 4096-record chunk at a time.
-//              The chunk's 16-B records are staged in shared memory by
-//              cp.async (the next chunk is fetched while the current one is
-//              ranked and written).  Each warp owns 256 consecutive records, in
-//              two groups of 128: lane L decodes records L, L+32, L+64, L+96 of
-//              the group (access vs control; byte range -> its 1 or 2 8-byte
-//              words; word -> address bucket via the bin map), and the
-//              group is ranked stably into the warp's per-bucket counters with a
-//              single check when all its events hit one bucket (the common case
-//              for real access streams).  Events are then written straight to
-//              the chunk's slot of the output, grouped by bucket in trace order,
-//              and one {chunk, bucket, start, len} entry per touched bucket is
-//              appended for the replay.
+// k_partition  persistent CTAs (one per SM, 16 warps).  Every warp works on its
+//              own 256-record chunks with no block-level synchronisation: the
+//              chunk's 16-B records are staged in the warp's shared memory by
+//              cp.async (double-buffered: the next chunk streams in while the
+//              current one is processed).  Lane L decodes records L, L+32, ...
+//              (access vs control; byte range -> its 1 or 2 8-byte words, P:267;
+//              word -> address bucket via the bin map) in two groups of 128, and
+//              each group is ranked stably into the warp's per-bucket counters —
+//              a single check when all its events hit one bucket, the common
+//              case for real access streams.  First touches of a bucket append
+//              it to the warp's touched list; a warp scan over that list turns
+//              the counts into offsets.  Events are written straight to the
+//              chunk's 512-event slot of the output, grouped by bucket in trace
+//              order, and one {chunk, bucket, start | len << 16} entry per touched
+//              bucket is appended (batched per warp) for the replay.
 #include "kcommon.cuh"
 #include <algorithm>
 
@@ -20,24 +22,15 @@ namespace arb {
 
 constexpr int PT = kPartThreads;            // 512 threads
 constexpr int PW = kPartWarps;              // 16 warps
-constexpr int GROUPS = kChunkRecords / PT / 4;  // 2 groups of 128 records per warp
-constexpr int RPT = kChunkRecords / PT;     // 8 records per thread
+constexpr int WREC = kChunkRecords;         // 256 records per chunk
+constexpr int RPL = WREC / 32;              // 8 records per lane (two groups of 4 x 32)
+constexpr int kSegBuf = 64;                 // segment entries buffered per warp
 
-struct PartSmem {
-  uint32_t touched[kMaxBuckets / 32];       // bitmap of buckets hit by the chunk
-  uint16_t tlist[kMaxBuckets];              // touched buckets, ascending
-  uint32_t tstart[kMaxBuckets + 1];         // their first event in the chunk
-  uint32_t wsum[PW];
-  uint32_t n_touched, total;
-  unsigned long long seg_base;
-};
-
-__device__ __forceinline__ void cp_async16(void* smem_dst, const void* gsrc) {
-  const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(gsrc) : "memory");
+// per-warp shared memory: stage[2][WREC] uint4, segbuf[kSegBuf] uint4,
+// tlist[2 * WREC] u16, row[NB] u16 (padded to 16 B)
+__host__ __device__ constexpr size_t warp_smem_bytes(uint32_t nb) {
+  return sizeof(uint4) * (2 * WREC + kSegBuf) + 2 * (2 * WREC) + (((size_t)nb * 2 + 15) & ~(size_t)15);
 }
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
 // Decoded record: info = cnt | b0 << 2 | b1 << 12 (cnt = tracked words 0..2),
 // keys k0/k1 = op << 30 | word offset inside the bucket.
@@ -79,34 +72,40 @@ __device__ __forceinline__ Dec decode(uint4 q, const PartParams& p, uint32_t& ig
   return d;
 }
 
-__device__ __forceinline__ void mark(uint32_t* touched, uint32_t b) { atomicOr(&touched[b >> 5], 1u << (b & 31)); }
+// append the buckets of lanes with `is_new` to the warp's touched list
+__device__ __forceinline__ void touch(uint16_t* tlist, uint32_t& nT, bool is_new, uint32_t b, uint32_t lt) {
+  const uint32_t m = __ballot_sync(FULL, is_new);
+  if (is_new) tlist[nT + __popc(m & lt)] = (uint16_t)b;
+  nT += __popc(m);
+}
 
 // Generic stable rank of one 32-record round (record order, word0 before word1).
-__device__ __forceinline__ void rank_round(uint32_t info, uint16_t* row, uint32_t* touched, uint32_t lane,
-                                           uint32_t& r0, uint32_t& r1) {
+__device__ __forceinline__ void rank_round(uint32_t info, uint16_t* row, uint16_t* tlist, uint32_t& nT,
+                                           uint32_t lane, uint32_t lt, uint32_t& r0, uint32_t& r1) {
   const uint32_t cnt = info & 3u, b0 = (info >> 2) & 1023u, b1 = (info >> 12) & 1023u;
   r0 = r1 = 0;
-  const uint32_t lt = lanemask_lt();
   if (__any_sync(FULL, cnt == 2 && b0 != b1)) {
     // a record crossing a bucket boundary: serial over lanes
+    bool n0 = false, n1 = false;
     for (uint32_t L = 0; L < 32; ++L) {
       if (lane == L) {
-        if (cnt >= 1) { r0 = row[b0]; row[b0] = (uint16_t)(r0 + 1); mark(touched, b0); }
-        if (cnt == 2) { r1 = row[b1]; row[b1] = (uint16_t)(r1 + 1); mark(touched, b1); }
+        if (cnt >= 1) { r0 = row[b0]; row[b0] = (uint16_t)(r0 + 1); n0 = r0 == 0; }
+        if (cnt == 2) { r1 = row[b1]; row[b1] = (uint16_t)(r1 + 1); n1 = r1 == 0; }
       }
       __syncwarp();
     }
+    touch(tlist, nT, n0, b0, lt);
+    touch(tlist, nT, n1, b1, lt);
     return;
   }
   const uint32_t two = __ballot_sync(FULL, cnt == 2);
   const uint32_t grp = __match_any_sync(FULL, cnt ? b0 : 0xFFFFFFFFu);
   const uint32_t base = cnt ? row[b0] : 0;
   __syncwarp();
-  if (cnt && lane == 31u - __clz(grp)) {
-    row[b0] = (uint16_t)(base + __popc(grp) + __popc(grp & two));
-    mark(touched, b0);
-  }
+  const bool leader = cnt && lane == 31u - __clz(grp);
+  if (leader) row[b0] = (uint16_t)(base + __popc(grp) + __popc(grp & two));
   __syncwarp();
+  touch(tlist, nT, leader && base == 0, b0, lt);
   r0 = base + __popc(grp & lt) + __popc(grp & lt & two);
   r1 = r0 + 1;
 }
@@ -114,46 +113,63 @@ __device__ __forceinline__ void rank_round(uint32_t info, uint16_t* row, uint32_
 __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   extern __shared__ __align__(16) uint8_t smem[];
   const uint32_t NB = p.n_buckets;
-  uint4* stage = reinterpret_cast<uint4*>(smem);                            // [kChunkRecords]
-  uint16_t* cnt = reinterpret_cast<uint16_t*>(smem + kChunkRecords * sizeof(uint4));   // [PW][NB]
-  __shared__ PartSmem S;
-
-  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t lt = lanemask_lt();
-  for (uint32_t i = tid; i < PW * NB; i += PT) cnt[i] = 0;
-  if (tid < kMaxBuckets / 32) S.touched[tid] = 0;
-  uint16_t* row = cnt + warp * NB;
-  uint32_t n_acc = 0, n_ign = 0;
+  uint8_t* wbase = smem + warp * warp_smem_bytes(NB);
+  uint4* stage = reinterpret_cast<uint4*>(wbase);                   // [2][WREC]
+  uint4* segbuf = stage + 2 * WREC;                                  // [kSegBuf]
+  uint16_t* tlist = reinterpret_cast<uint16_t*>(segbuf + kSegBuf);   // [2 * WREC]
+  uint16_t* row = tlist + 2 * WREC;                                  // [NB]
+  for (uint32_t i = lane; i < NB; i += 32) row[i] = 0;
+  uint32_t n_acc = 0, n_ign = 0, nbuf = 0;
 
-  auto fetch = [&](uint64_t c) {
-    if (c >= p.n_chunks) return;
-    const uint64_t r0 = c * kChunkRecords;
+  auto fetch = [&](uint64_t c, uint4* dst) {
+    if (c < p.n_chunks) {
+      const uint64_t r0 = c * WREC;
 #pragma unroll
-    for (int k = 0; k < RPT; ++k) {
-      const uint32_t j = tid + k * PT;
-      if (r0 + j < p.n) cp_async16(stage + j, p.ev + r0 + j);
+      for (int k = 0; k < RPL; ++k) {
+        const uint32_t j = lane + k * 32;
+        if (r0 + j < p.n) cp_async16(dst + j, p.ev + r0 + j);
+      }
     }
-    cp_async_commit();
+    cp_async_commit();                 // possibly empty: keeps the group count uniform
+  };
+  auto flush_segs = [&]() {
+    __syncwarp();
+    unsigned long long sb = 0;
+    if (lane == 0 && nbuf) sb = atomicAdd(&p.st->n_segs, (unsigned long long)nbuf);
+    sb = __shfl_sync(FULL, sb, 0);
+    for (uint32_t i = lane; i < nbuf; i += 32)
+      if (sb + i < p.seg_cap) p.seg_out[sb + i] = segbuf[i];
+    __syncwarp();
+    nbuf = 0;
   };
 
-  uint64_t chunk = blockIdx.x;
-  fetch(chunk);
-  for (; chunk < p.n_chunks; chunk += gridDim.x) {
-    const uint64_t rec0 = chunk * kChunkRecords;
-    cp_async_wait_all();
-    __syncthreads();
-    // ---- pass A: decode + rank, 2 groups of 4 x 32 records per warp ---------------
-    Dec dec[RPT];
-    uint32_t rk[RPT];
+  const uint64_t nwarps = (uint64_t)gridDim.x * PW;
+  uint32_t cur = 0;
+  uint64_t chunk = (uint64_t)blockIdx.x * PW + warp;
+  fetch(chunk, stage);
+  __syncwarp();
+  for (; chunk < p.n_chunks; chunk += nwarps) {
+    fetch(chunk + nwarps, stage + (cur ^ 1) * WREC);
+    cp_async_wait_group<1>();
+    __syncwarp();
+    const uint4* st = stage + cur * WREC;
+    const uint64_t rec0 = chunk * WREC;
+    const uint32_t nvalid = p.n - rec0 < (uint64_t)WREC ? (uint32_t)(p.n - rec0) : (uint32_t)WREC;
+    uint32_t nT = 0;
+    // ---- pass A: decode + rank, 2 groups of 4 x 32 records ----------------------------
+    Dec dec[RPL];
+    uint32_t rk[RPL];
 #pragma unroll
-    for (int g = 0; g < GROUPS; ++g) {
+    for (int g = 0; g < 2; ++g) {
       uint32_t any_flag = 0;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
-        const uint32_t j = warp * 256 + g * 128 + k * 32 + lane;      // record inside the chunk
+        const uint32_t j = g * 128 + k * 32 + lane;
         uint32_t flags = 0;
         dec[g * 4 + k] = Dec{0, 0, 0};
-        if (rec0 + j < p.n) dec[g * 4 + k] = decode(stage[j], p, n_ign, flags);
+        if (j < nvalid) dec[g * 4 + k] = decode(st[j], p, n_ign, flags);
         any_flag |= flags << (2 * k);
         n_acc += dec[g * 4 + k].info & 3u;
       }
@@ -161,7 +177,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
         // control / malformed records in the group (rare)
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
-          const uint32_t j = warp * 256 + g * 128 + k * 32 + lane;
+          const uint32_t j = g * 128 + k * 32 + lane;
           const uint32_t f = (any_flag >> (2 * k)) & 3u;
           if (f & 2u) atomicMin(&p.st->err_pos, (unsigned long long)(rec0 + j));
           const uint32_t cm = __ballot_sync(FULL, f & 1u);
@@ -172,7 +188,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
             if (f & 1u) {
               const uint64_t slot = base + __popc(cm & lt);
               if (slot < p.ctl_cap) {
-                const uint4 q = stage[j];
+                const uint4 q = st[j];
                 CtlRec c;
                 c.pos = rec0 + j;
                 c.w0 = (uint64_t)q.x | ((uint64_t)q.y << 32);
@@ -197,18 +213,20 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
         for (int k = 0; k < 4; ++k) rk[g * 4 + k] = 0;
         continue;
       }
-      uint32_t kl = 0;
-      while (!vm[kl]) ++kl;
-      const uint32_t lead = __ffs(vm[kl]) - 1;
+      // bucket of the group's first event: round kl = first with a valid lane
+      const uint32_t kl = vm[0] ? 0u : vm[1] ? 1u : vm[2] ? 2u : 3u;
+      const uint32_t vml = vm[0] ? vm[0] : vm[1] ? vm[1] : vm[2] ? vm[2] : vm[3];
+      const uint32_t lead = __ffs(vml) - 1;
       uint32_t bsrc = 0;
 #pragma unroll
       for (int k = 0; k < 4; ++k) if ((uint32_t)k == kl) bsrc = (dec[g * 4 + k].info >> 2) & 1023u;
       const uint32_t bref = __shfl_sync(FULL, bsrc, lead);
+      const uint32_t iref = bref << 2 | bref << 12;
       bool same = true;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
         const uint32_t info = dec[g * 4 + k].info;
-        same &= (info & 3u) == 0 || (((info >> 2) & 1023u) == bref && ((info >> 12) & 1023u) == bref);
+        same &= (info & 3u) == 0 || (info & ~3u) == iref;
       }
       if (__all_sync(FULL, same)) {
         const uint32_t base = row[bref];
@@ -220,147 +238,61 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
           run += __popc(vm[k]) + __popc(tw[k]);
         }
         __syncwarp();
-        if (lane == 0) { row[bref] = (uint16_t)run; mark(S.touched, bref); }
+        if (lane == 0) {
+          row[bref] = (uint16_t)run;
+          if (base == 0) tlist[nT] = (uint16_t)bref;
+        }
+        nT += base == 0;
         __syncwarp();
       } else {
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
           uint32_t r0, r1;
-          rank_round(dec[g * 4 + k].info, row, S.touched, lane, r0, r1);
+          rank_round(dec[g * 4 + k].info, row, tlist, nT, lane, lt, r0, r1);
           rk[g * 4 + k] = r0 | (r1 << 16);
         }
       }
     }
-    __syncthreads();                 // stage consumed; counters complete
-    fetch(chunk + gridDim.x);        // next chunk streams in during the rest
-    // ---- touched buckets, totals, per-warp offsets ------------------------------------
-    if (warp == 0) {
-      uint32_t base = 0;
-      const uint32_t nw = (NB + 31) / 32;
-      for (uint32_t w0 = 0; w0 < nw; w0 += 32) {
-        const uint32_t wi = w0 + lane;
-        const uint32_t bits = wi < nw ? S.touched[wi] : 0;
-        if (wi < nw) S.touched[wi] = 0;
-        const uint32_t pc = __popc(bits);
-        uint32_t incl = pc;
+    __syncwarp();
+    // ---- counts -> offsets over the touched list; segment entries ------------------------
+    uint32_t carry = 0;
+    for (uint32_t t0 = 0; t0 < nT; t0 += 32) {
+      const uint32_t t = t0 + lane;
+      uint32_t b = 0, tot = 0;
+      if (t < nT) { b = tlist[t]; tot = row[b]; }
+      uint32_t incl = tot;
 #pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-          const uint32_t o = __shfl_up_sync(FULL, incl, d);
-          if (lane >= (uint32_t)d) incl += o;
-        }
-        uint32_t k = base + incl - pc;
-        for (uint32_t b = bits; b; b &= b - 1) S.tlist[k++] = (uint16_t)(wi * 32 + __ffs(b) - 1);
-        base += __shfl_sync(FULL, incl, 31);
+      for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t o = __shfl_up_sync(FULL, incl, d);
+        if (lane >= (uint32_t)d) incl += o;
       }
-      if (lane == 0) S.n_touched = base;
+      const uint32_t start = carry + incl - tot;
+      carry += __shfl_sync(FULL, incl, 31);
+      const uint32_t n_new = min(32u, nT - t0);
+      if (nbuf + n_new > kSegBuf) flush_segs();
+      if (t < nT) {
+        row[b] = (uint16_t)start;
+        segbuf[nbuf + lane] = make_uint4((uint32_t)chunk, b, start | (tot << 16), 0);
+      }
+      nbuf += n_new;
     }
-    __syncthreads();
-    const uint32_t T = S.n_touched;
-    if (T <= 32) {
-      // the common case: one warp does the bookkeeping
-      if (warp == 0) {
-        uint32_t tot = 0, b = 0;
-        if (lane < T) {
-          b = S.tlist[lane];
-#pragma unroll
-          for (int w = 0; w < PW; ++w) tot += cnt[w * NB + b];
-        }
-        uint32_t incl = tot;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-          const uint32_t o = __shfl_up_sync(FULL, incl, d);
-          if (lane >= (uint32_t)d) incl += o;
-        }
-        if (lane < T) {
-          uint32_t run = incl - tot;
-          S.tstart[lane] = run;
-#pragma unroll
-          for (int w = 0; w < PW; ++w) { const uint32_t c = cnt[w * NB + b]; cnt[w * NB + b] = (uint16_t)run; run += c; }
-        }
-        if (lane == 31) { S.tstart[T] = incl; S.total = incl; }
-        unsigned long long sb = 0;
-        if (lane == 0) sb = atomicAdd(&p.st->n_segs, (unsigned long long)T);
-        sb = __shfl_sync(FULL, sb, 0);
-        __syncwarp();
-        if (lane < T && sb + lane < p.seg_cap)
-          p.seg_out[sb + lane] = make_uint4((uint32_t)chunk, b, (incl - tot) | (tot << 16), 0);
-      }
-    } else {
-      // many buckets (scattered chunk): all threads
-      uint32_t mytot[2] = {0, 0};
-#pragma unroll
-      for (int k = 0; k < 2; ++k) {
-        const uint32_t t = tid + k * PT;
-        if (t < T) {
-          const uint32_t b = S.tlist[t];
-          uint32_t s = 0;
-#pragma unroll
-          for (int w = 0; w < PW; ++w) s += cnt[w * NB + b];
-          mytot[k] = s;
-        }
-      }
-      uint32_t all0 = 0, s0 = 0, s1 = 0, all1 = 0;
-      {
-        uint32_t v = mytot[0], incl = v;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-          const uint32_t o = __shfl_up_sync(FULL, incl, d);
-          if (lane >= (uint32_t)d) incl += o;
-        }
-        if (lane == 31) S.wsum[warp] = incl;
-        __syncthreads();
-        uint32_t wpre = 0;
-#pragma unroll
-        for (int w = 0; w < PW; ++w) { const uint32_t x = S.wsum[w]; if ((uint32_t)w < warp) wpre += x; all0 += x; }
-        s0 = wpre + incl - v;
-        __syncthreads();
-        uint32_t v1 = mytot[1], incl1 = v1;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-          const uint32_t o = __shfl_up_sync(FULL, incl1, d);
-          if (lane >= (uint32_t)d) incl1 += o;
-        }
-        if (lane == 31) S.wsum[warp] = incl1;
-        __syncthreads();
-        uint32_t wpre1 = 0;
-#pragma unroll
-        for (int w = 0; w < PW; ++w) { const uint32_t x = S.wsum[w]; if ((uint32_t)w < warp) wpre1 += x; all1 += x; }
-        s1 = all0 + wpre1 + incl1 - v1;
-      }
-      if (tid == 0) S.seg_base = atomicAdd(&p.st->n_segs, (unsigned long long)T);
-      __syncthreads();
-#pragma unroll
-      for (int k = 0; k < 2; ++k) {
-        const uint32_t t = tid + k * PT;
-        if (t < T) {
-          const uint32_t b = S.tlist[t];
-          uint32_t run = k ? s1 : s0;
-          const uint32_t st = run;
-          S.tstart[t] = run;
-#pragma unroll
-          for (int w = 0; w < PW; ++w) { const uint32_t c = cnt[w * NB + b]; cnt[w * NB + b] = (uint16_t)run; run += c; }
-          if (S.seg_base + t < p.seg_cap)
-            p.seg_out[S.seg_base + t] = make_uint4((uint32_t)chunk, b, st | ((run - st) << 16), 0);
-        }
-      }
-      if (tid == 0) { S.total = all0 + all1; S.tstart[T] = all0 + all1; }
-    }
-    __syncthreads();
-    // ---- pass B: write the events straight to the chunk's output slot ---------------
+    __syncwarp();
+    // ---- pass B: write the events straight to the chunk's output slot ----------------------
     uint2* out = p.part_ev + chunk * kChunkCap;
 #pragma unroll
-    for (int r = 0; r < RPT; ++r) {
+    for (int r = 0; r < RPL; ++r) {
       const uint32_t info = dec[r].info, c = info & 3u;
-      const uint32_t j = warp * 256 + (r >> 2) * 128 + (r & 3) * 32 + lane;
-      const uint32_t pos = (uint32_t)(rec0 + j);
+      const uint32_t pos = (uint32_t)(rec0 + (r >> 2) * 128 + (r & 3) * 32 + lane);
       if (c >= 1) out[row[(info >> 2) & 1023u] + (rk[r] & 0xFFFFu)] = make_uint2(dec[r].k0, pos);
       if (c == 2) out[row[(info >> 12) & 1023u] + (rk[r] >> 16)] = make_uint2(dec[r].k1, pos);
     }
-    __syncthreads();
-    for (uint32_t t = tid; t < T * PW; t += PT) cnt[(t % PW) * NB + S.tlist[t / PW]] = 0;
-    // the next iteration's wait + barrier orders this reset before the next ranking
+    __syncwarp();
+    for (uint32_t t = lane; t < nT; t += 32) row[tlist[t]] = 0;
+    cur ^= 1;
+    __syncwarp();                      // stage[cur] reads and row resets done before reuse
   }
   cp_async_wait_all();
+  flush_segs();
 
 #pragma unroll
   for (int d = 16; d; d >>= 1) {
@@ -375,13 +307,14 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
 
 cudaError_t launch_partition(const PartParams& p, cudaStream_t s) {
   if (p.n_chunks == 0) return cudaSuccess;
-  const size_t smem = (size_t)kChunkRecords * sizeof(uint4) + (size_t)PW * p.n_buckets * 2;
+  const size_t smem = PW * warp_smem_bytes(p.n_buckets);
   cudaError_t e = cudaFuncSetAttribute(k_partition, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const uint32_t grid = (uint32_t)std::min<uint64_t>(p.n_chunks, (uint64_t)sms);
+  const uint64_t ctas = (p.n_chunks + PW - 1) / PW;
+  const uint32_t grid = (uint32_t)std::min<uint64_t>(ctas, (uint64_t)sms);
   k_partition<<<grid, PT, smem, s>>>(p);
   return cudaGetLastError();
 }

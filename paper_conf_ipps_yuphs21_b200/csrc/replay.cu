@@ -44,7 +44,7 @@ struct ReplaySmem {
   uint32_t red[RT / 32], red2[RT / 32], wscan[RT / 32];
   uint32_t wcnt[RT / 32], wev[RT / 32];
   uint32_t bucket, op_cur, op_end, next_op;
-  uint32_t n_segs, n_events, wsc, nwin, ga0, ga1;
+  uint32_t seg0, cum0, n_segs, n_events, wsc, nwin, ga0, ga1;
   uint64_t bucket_base;
 };
 
@@ -408,64 +408,54 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
   __syncthreads();
 }
 
-// ---- per-bucket segment list ---------------------------------------------------------------
-// Compact the bucket's non-empty chunk segments, in chunk order, into the CTA's
-// scratch: seg_start[i] = global index of the segment's first event,
-// seg_cum[i] = bucket-relative index of that event; seg_cum[n] = event total.
-__device__ void build_segments(ReplaySmem& S, const ReplayParams& p, uint32_t b, uint32_t* sstart,
-                               uint32_t* scum) {
-  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const uint32_t f0 = p.seg_first[b], ne = p.seg_first[b + 1] - f0;
-  uint32_t carry = 0;
-  for (uint32_t base = 0; base < ne; base += RT) {
-    const uint32_t i = base + threadIdx.x;
-    uint32_t len = 0, gs = 0;
-    if (i < ne) {
-      const uint4 e = p.segs[f0 + i];                  // {chunk, bucket, start | len << 16, 0}
-      len = e.z >> 16;
-      gs = e.x * (uint32_t)kChunkCap + (e.z & 0xFFFFu);
+// ---- the bucket's segments -------------------------------------------------------------
+// The sorted entries of bucket b are p.segs[f0, f1) in chunk order (= trace
+// order); entry i covers bucket-relative events [segs[i].w - segs[f0].w, + len)
+// stored at part_ev[chunk * kChunkCap + start].
+__device__ void bucket_setup(ReplaySmem& S, const ReplayParams& p, uint32_t b) {
+  if (threadIdx.x == 0) {
+    const uint32_t f0 = p.seg_first[b], f1 = p.seg_first[b + 1];
+    S.seg0 = f0; S.n_segs = f1 - f0;
+    S.cum0 = 0; S.n_events = 0;
+    if (f1 > f0) {
+      const uint4 first = p.segs[f0], last = p.segs[f1 - 1];
+      S.cum0 = first.w;
+      S.n_events = last.w + (last.z >> 16) - first.w;
     }
-    uint32_t incl = len;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t o = __shfl_up_sync(FULL, incl, d);
-      if (lane >= (uint32_t)d) incl += o;
-    }
-    if (lane == 31) S.wev[warp] = incl;
-    __syncthreads();
-    uint32_t wpre = 0, tot = 0;
-#pragma unroll
-    for (int w = 0; w < RT / 32; ++w) { const uint32_t x = S.wev[w]; if ((uint32_t)w < warp) wpre += x; tot += x; }
-    if (i < ne) { sstart[i] = gs; scum[i] = carry + wpre + incl - len; }
-    carry += tot;
-    __syncthreads();
+    S.wsc = 0; S.nwin = 0; S.wcum[0] = 1;      // empty window: forces a load
   }
-  if (threadIdx.x == 0) { scum[ne] = carry; S.n_segs = ne; S.n_events = carry; }
   __syncthreads();
 }
 
-// ---- the kernel ------------------------------------------------------------------------
-__device__ __forceinline__ void cp_async8(void* smem_dst, const void* gsrc) {
-  const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(d), "l"(gsrc) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
-
-// Make the staged window of segment descriptors contain event e0 (rarely reloads).
-__device__ void ensure_window(ReplaySmem& S, const uint32_t* sstart, const uint32_t* scum, uint32_t e0) {
+// Make the staged window of segment descriptors contain event e0 (reloads
+// about every kWin segments; sequential progress needs no search).
+__device__ void ensure_window(ReplaySmem& S, const ReplayParams& p, uint32_t e0) {
   if (e0 >= S.wcum[0] && e0 < S.wcum[S.nwin]) return;
   __syncthreads();
   if (threadIdx.x == 0) {
-    uint32_t a = 0, z = S.n_segs;                 // last segment with scum <= e0
-    while (z - a > 1) { const uint32_t mid = (a + z) >> 1; if (scum[mid] <= e0) a = mid; else z = mid; }
+    uint32_t a;
+    if (S.nwin && e0 == S.wcum[S.nwin]) {
+      a = S.wsc + S.nwin;                       // the window's successor
+    } else {                                    // last segment starting at or before e0
+      uint32_t lo = 0, z = S.n_segs;
+      while (z - lo > 1) {
+        const uint32_t mid = (lo + z) >> 1;
+        if (p.segs[S.seg0 + mid].w - S.cum0 <= e0) lo = mid; else z = mid;
+      }
+      a = lo;
+    }
     S.wsc = a;
     S.nwin = min((uint32_t)kWin, S.n_segs - a);
   }
   __syncthreads();
   const uint32_t sc = S.wsc, nwin = S.nwin;
-  for (uint32_t k = threadIdx.x; k < nwin; k += RT) { S.wstart[k] = sstart[sc + k]; S.wcum[k] = scum[sc + k]; }
-  if (threadIdx.x == 0) S.wcum[nwin] = scum[sc + nwin];
+  const uint4* segs = p.segs + S.seg0 + sc;
+  for (uint32_t k = threadIdx.x; k < nwin; k += RT) {
+    const uint4 e = segs[k];
+    S.wstart[k] = e.x * (uint32_t)kChunkCap + (e.z & 0xFFFFu);
+    S.wcum[k] = e.w - S.cum0;
+  }
+  if (threadIdx.x == 0) S.wcum[nwin] = sc + nwin < S.n_segs ? segs[nwin].w - S.cum0 : S.n_events;
   __syncthreads();
 }
 
@@ -519,8 +509,6 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
   extern __shared__ __align__(16) uint8_t smem_raw[];
   ReplaySmem& S = *reinterpret_cast<ReplaySmem*>(smem_raw);
   const uint32_t tid = threadIdx.x;
-  uint32_t* sstart = p.seg_start + (uint64_t)blockIdx.x * (p.n_chunks + 1);
-  uint32_t* scum = p.seg_cum + (uint64_t)blockIdx.x * (p.n_chunks + 1);
   hash_clear(S);
   for (;;) {
     if (tid == 0) {
@@ -535,13 +523,12 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       S.op_end = p.ops_start[b + 1];
       S.next_op = S.op_cur < S.op_end ? p.ops[S.op_cur].pos : 0xFFFFFFFFu;
       S.bucket_base = p.bucket_start[b];
-      S.wcum[0] = 1; S.nwin = 0; S.wcum[0] = 1;   // empty window: forces a load
     }
-    build_segments(S, p, b, sstart, scum);
+    bucket_setup(S, p, b);
     const uint32_t total = S.n_events;
     uint32_t e0 = 0, cur = 0, m_cur = 0;
     if (total) {
-      ensure_window(S, sstart, scum, 0);
+      ensure_window(S, p, 0);
       m_cur = issue_gather(S, p, 0, total, S.ev[0]);
     }
     while (e0 < total) {
@@ -553,7 +540,7 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       const uint32_t nxt = e0 + m;
       uint32_t m_nxt = 0;
       if (nxt < total) {
-        ensure_window(S, sstart, scum, nxt);
+        ensure_window(S, p, nxt);
         m_nxt = issue_gather(S, p, nxt, total, S.ev[cur ^ 1]);
       }
       // ---- range ops before the first event, then cut at the next one -------------
@@ -575,7 +562,7 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         // the prefetch started at e0_old + m: drain it and gather from e0
         cp_async_wait_all();
         __syncthreads();
-        ensure_window(S, sstart, scum, e0);
+        ensure_window(S, p, e0);
         m_cur = issue_gather(S, p, e0, total, S.ev[cur]);
       }
     }
