@@ -36,39 +36,33 @@ __host__ __device__ constexpr size_t warp_smem_bytes(uint32_t nb) {
 // keys k0/k1 = op << 30 | word offset inside the bucket.
 struct Dec { uint32_t info, k0, k1; };
 
-__device__ __forceinline__ uint32_t bucket_key(const PartParams& p, uint64_t rel, uint32_t op, uint32_t& b) {
-  const uint32_t m = __ldg(p.bin_map + (uint32_t)(rel >> p.coarse_bits));
-  b = m & 1023u;
-  return (op << 30) | (((m >> 10) << p.coarse_bits) | ((uint32_t)rel & ((1u << p.coarse_bits) - 1u)));
-}
-
-// flags: bit0 control record, bit1 malformed
-__device__ __forceinline__ Dec decode(uint4 q, const PartParams& p, uint32_t& ign, uint32_t& flags) {
-  Dec d{0, 0, 0};
+// Branch-free (predicated) so the four records of a round interleave.
+// flags: bit0 control record, bit1 malformed.  valid = record exists.
+__device__ __forceinline__ Dec decode(uint4 q, bool valid, const PartParams& p, uint32_t& ign, uint32_t& flags) {
   const uint32_t op = (q.y >> 16) & 0xFFu;
-  if (op >= 4) {
-    const bool ctl = op <= 14 && op >= 8 && op != 11;
-    flags = ctl ? 1u : 2u;
-    return d;
-  }
   const uint32_t len = q.z;
   const uint64_t addr = ((uint64_t)(q.y & 0xFFFFu) << 32) | q.x;
-  if ((q.w & 0xFFFFu) | (len - 1u > 7u) | (addr + len > (1ull << 48))) { flags = 2u; return d; }
+  const bool bad_acc = ((q.w & 0xFFFFu) | (uint32_t)(len - 1u > 7u) | (uint32_t)(addr + len > (1ull << 48))) != 0;
+  const bool ctl = op <= 14 && op >= 8 && op != 11;
+  flags = !valid ? 0u : op < 4 ? (bad_acc ? 2u : 0u) : (ctl ? 1u : 2u);
+  const bool ok = valid && op < 4 && !bad_acc;
   const uint64_t rel = (addr >> 3) - p.base_word;                 // wraps when below the range
-  uint32_t cnt = 0, b0 = 0, b1 = 0;
-  if (rel < p.n_words) { d.k0 = bucket_key(p, rel, op, b0); b1 = b0; cnt = 1; } else { ++ign; }
-  if ((q.x & 7u) + len > 8u) {                                     // unaligned: a second word (Z4)
-    const uint64_t r1 = rel + 1;
-    if (r1 < p.n_words) {
-      uint32_t bb;
-      const uint32_t k = bucket_key(p, r1, op, bb);
-      if (cnt == 0) { d.k0 = k; b0 = bb; b1 = bb; } else { d.k1 = k; b1 = bb; }
-      ++cnt;
-    } else {
-      ++ign;
-    }
-  }
-  d.info = cnt | (b0 << 2) | (b1 << 12);
+  const bool in0 = ok && rel < p.n_words;
+  const bool two = ok && (q.x & 7u) + len > 8u;                    // unaligned: a second word (Z4)
+  const bool in1 = two && rel + 1 < p.n_words;
+  ign += (uint32_t)(ok && !in0) + (uint32_t)(two && !in1);
+  const uint32_t cb = p.coarse_bits, msk = (1u << cb) - 1u;
+  uint32_t m0 = 0, m1 = 0;
+  if (in0) m0 = __ldg(p.bin_map + (uint32_t)(rel >> cb));
+  if (in1) m1 = __ldg(p.bin_map + (uint32_t)((rel + 1) >> cb));
+  const uint32_t kk0 = (op << 30) | ((m0 >> 10) << cb) | ((uint32_t)rel & msk);
+  const uint32_t kk1 = (op << 30) | ((m1 >> 10) << cb) | ((uint32_t)(rel + 1) & msk);
+  const uint32_t b0 = in0 ? (m0 & 1023u) : (m1 & 1023u);          // 0 when neither word is tracked
+  const uint32_t b1 = in1 ? (m1 & 1023u) : b0;
+  Dec d;
+  d.k0 = in0 ? kk0 : kk1;
+  d.k1 = kk1;
+  d.info = ((uint32_t)in0 + (uint32_t)in1) | (b0 << 2) | (b1 << 12);
   return d;
 }
 
@@ -126,10 +120,12 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   auto fetch = [&](uint64_t c, uint4* dst) {
     if (c < p.n_chunks) {
       const uint64_t r0 = c * WREC;
+      const uint32_t nv = p.n - r0 < (uint64_t)WREC ? (uint32_t)(p.n - r0) : (uint32_t)WREC;
+      const uint4* src = p.ev + r0;
 #pragma unroll
       for (int k = 0; k < RPL; ++k) {
         const uint32_t j = lane + k * 32;
-        if (r0 + j < p.n) cp_async16(dst + j, p.ev + r0 + j);
+        if (j < nv) cp_async16(dst + j, src + j);
       }
     }
     cp_async_commit();                 // possibly empty: keeps the group count uniform
@@ -167,9 +163,8 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
         const uint32_t j = g * 128 + k * 32 + lane;
-        uint32_t flags = 0;
-        dec[g * 4 + k] = Dec{0, 0, 0};
-        if (j < nvalid) dec[g * 4 + k] = decode(st[j], p, n_ign, flags);
+        uint32_t flags;
+        dec[g * 4 + k] = decode(st[j], j < nvalid, p, n_ign, flags);
         any_flag |= flags << (2 * k);
         n_acc += dec[g * 4 + k].info & 3u;
       }

@@ -1,9 +1,9 @@
 // replay.cu — A3b + A4 + A5: per-address replay of each bucket.
 //
 // One CTA per address bucket at a time (persistent; buckets in largest-first
-// order).  For its bucket the CTA first compacts the bucket's non-empty chunk
-// segments (from the partition's offset table) into a segment list, then walks
-// the bucket's word-events in trace order, applies the resolved range ops
+// order).  The bucket's events are the segments of its sorted segment entries
+// (chunk order = trace order); the CTA gathers them step by step through a
+// staged window of entries (cp.async, double-buffered), applies the resolved range ops
 // (Table I transfers / allocate / release; target update P:121) to
 // the bucket's shadow at their trace positions, and processes the events in
 // steps of <= 2048 that never straddle a range op:
@@ -44,7 +44,7 @@ struct ReplaySmem {
   uint32_t red[RT / 32], red2[RT / 32], wscan[RT / 32];
   uint32_t wcnt[RT / 32], wev[RT / 32];
   uint32_t bucket, op_cur, op_end, next_op;
-  uint32_t seg0, cum0, n_segs, n_events, wsc, nwin, ga0, ga1;
+  uint32_t seg0, cum0, n_segs, n_events, wsc, nwin;
   uint64_t bucket_base;
 };
 
@@ -429,8 +429,9 @@ __device__ void bucket_setup(ReplaySmem& S, const ReplayParams& p, uint32_t b) {
 
 // Make the staged window of segment descriptors contain event e0 (reloads
 // about every kWin segments; sequential progress needs no search).
-__device__ void ensure_window(ReplaySmem& S, const ReplayParams& p, uint32_t e0) {
+__device__ void ensure_window(ReplaySmem& S, const ReplayParams& p, uint32_t e0, uint32_t& hint) {
   if (e0 >= S.wcum[0] && e0 < S.wcum[S.nwin]) return;
+  hint = 0;
   __syncthreads();
   if (threadIdx.x == 0) {
     uint32_t a;
@@ -461,26 +462,27 @@ __device__ void ensure_window(ReplaySmem& S, const ReplayParams& p, uint32_t e0)
 
 // Issue cp.async copies of events [e0, e0 + m) of the bucket into dst; the
 // window must contain e0.  Returns m (<= STEP, clipped to the window).
-__device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t e0, uint32_t total, uint2* dst) {
+// `hint` (per thread, block-uniform) is a window segment index with
+// wcum[hint] <= e0; it is advanced to the last segment gathered.
+__device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t e0, uint32_t total, uint2* dst,
+                                 uint32_t& hint) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t nwin = S.nwin;
   const uint32_t m = min(min((uint32_t)STEP, total - e0), S.wcum[nwin] - e0);
-  // window segments [a0, a1) hold the events: warp 0 searches, everyone reads
-  if (warp == 0) {
-    // lane-parallel search: segment j holds e iff wcum[j] <= e < wcum[j+1]
-    uint32_t a0 = 0, a1 = 0;
-    for (uint32_t base = 0; base < nwin; base += 32) {
-      const uint32_t j = base + lane;
-      const bool le0 = j < nwin && S.wcum[j] <= e0;
-      const bool lt1 = j < nwin && S.wcum[j] < e0 + m;
-      a0 += __popc(__ballot_sync(FULL, le0));
-      a1 += __popc(__ballot_sync(FULL, lt1));
-      if (!__any_sync(FULL, lt1)) break;
-    }
-    if (lane == 0) { S.ga0 = a0 - 1; S.ga1 = a1; }
+  // window segments [a0, a1) hold the events; every warp searches (no barrier):
+  // segment j holds e iff wcum[j] <= e < wcum[j+1]
+  const uint32_t base0 = hint & ~31u;
+  uint32_t c0 = 0, c1 = 0;
+  for (uint32_t base = base0; base < nwin; base += 32) {
+    const uint32_t j = base + lane;
+    const bool le0 = j < nwin && S.wcum[j] <= e0;
+    const bool lt1 = j < nwin && S.wcum[j] < e0 + m;
+    c0 += __popc(__ballot_sync(FULL, le0));
+    c1 += __popc(__ballot_sync(FULL, lt1));
+    if (!__any_sync(FULL, lt1)) break;
   }
-  __syncthreads();
-  const uint32_t a0 = S.ga0, a1 = S.ga1;
+  const uint32_t a0 = base0 + c0 - 1, a1 = base0 + c1;
+  hint = a1 - 1;
   if ((a1 - a0) * 16 <= m) {
     // long segments: one warp streams one segment at a time
     for (uint32_t j = a0 + warp; j < a1; j += RT / 32) {
@@ -526,10 +528,10 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
     }
     bucket_setup(S, p, b);
     const uint32_t total = S.n_events;
-    uint32_t e0 = 0, cur = 0, m_cur = 0;
+    uint32_t e0 = 0, cur = 0, m_cur = 0, hint = 0;
     if (total) {
-      ensure_window(S, p, 0);
-      m_cur = issue_gather(S, p, 0, total, S.ev[0]);
+      ensure_window(S, p, 0, hint);
+      m_cur = issue_gather(S, p, 0, total, S.ev[0], hint);
     }
     while (e0 < total) {
       cp_async_wait_all();
@@ -540,8 +542,8 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       const uint32_t nxt = e0 + m;
       uint32_t m_nxt = 0;
       if (nxt < total) {
-        ensure_window(S, p, nxt);
-        m_nxt = issue_gather(S, p, nxt, total, S.ev[cur ^ 1]);
+        ensure_window(S, p, nxt, hint);
+        m_nxt = issue_gather(S, p, nxt, total, S.ev[cur ^ 1], hint);
       }
       // ---- range ops before the first event, then cut at the next one -------------
       apply_ops_before(S, p, ev[0].y);
@@ -562,8 +564,9 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         // the prefetch started at e0_old + m: drain it and gather from e0
         cp_async_wait_all();
         __syncthreads();
-        ensure_window(S, p, e0);
-        m_cur = issue_gather(S, p, e0, total, S.ev[cur]);
+        hint = 0;
+        ensure_window(S, p, e0, hint);
+        m_cur = issue_gather(S, p, e0, total, S.ev[cur], hint);
       }
     }
     apply_ops_before(S, p, 0xFFFFFFFFu);
