@@ -47,9 +47,9 @@ constexpr int kMaxBuckets = 1024;
 
 // ---- replay geometry -------------------------------------------------------
 constexpr int kReplayThreads = 256;
-constexpr int kReplayItems = 8;
+constexpr int kReplayItems = 4;
 constexpr int kStep = kReplayThreads * kReplayItems;  // events per step
-constexpr int kReplayCtasPerSm = 3;
+constexpr int kReplayCtasPerSm = 4;
 
 // device-side counters and error flags of one flush
 struct DevStats {

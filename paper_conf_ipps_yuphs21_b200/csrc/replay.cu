@@ -24,9 +24,10 @@
 
 namespace arb {
 
-constexpr int RT = kReplayThreads;           // 256 threads
-constexpr int RI = kReplayItems;             // 8 events per thread per step
+constexpr int RT = kReplayThreads;           // threads per CTA (>= 256)
+constexpr int RI = kReplayItems;             // events per thread per step
 constexpr int STEP = RT * RI;                // 2048 events per step
+static_assert(RT >= 256 && STEP <= 4096, "sort_pass digit loop and u16 offsets");
 constexpr int kWin = 2 * RT;                 // segment descriptors staged per step
 constexpr int kHSlots = 4096;                // hash slots (load <= 1/2)
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
@@ -271,7 +272,7 @@ __device__ void sort_pass(ReplaySmem& S, const uint32_t* kin, const uint32_t* pi
     kk[r] = k; pp[r] = pv; dg[r] = d; rk[r] = base + __popc(grp & lt);
   }
   __syncthreads();
-  {
+  if (tid < 256) {   // digit tid: per-warp offsets and total
     uint32_t s = 0;
 #pragma unroll
     for (int w = 0; w < RT / 32; ++w) {
@@ -297,7 +298,7 @@ __device__ void sort_pass(ReplaySmem& S, const uint32_t* kin, const uint32_t* pi
     for (int j = 0; j < 8; ++j) { S.pref[tid * 8 + j] = run; run += v[j]; }
   }
   __syncthreads();
-  {
+  if (tid < 256) {
     const uint32_t b = S.pref[tid];
 #pragma unroll
     for (int w = 0; w < RT / 32; ++w) S.u.s.hist[w][tid] = (uint16_t)(S.u.s.hist[w][tid] + b);
