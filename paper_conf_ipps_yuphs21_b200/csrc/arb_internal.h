@@ -43,7 +43,9 @@ constexpr int kPartThreads = 512;
 constexpr int kPartWarps = kPartThreads / 32;
 constexpr int kChunkRecords = 256;                  // records per chunk (one warp, independently)
 constexpr int kChunkCap = 2 * kChunkRecords;        // events per chunk (<= 2 words per access)
-constexpr int kMaxBuckets = 1024;
+constexpr int kBucketBits = 11;                    // bucket ids are 11-bit
+constexpr int kMaxBuckets = 1 << kBucketBits;
+constexpr uint32_t kBucketMask = kMaxBuckets - 1;
 
 // ---- replay geometry -------------------------------------------------------
 constexpr int kReplayThreads = 256;
@@ -81,7 +83,7 @@ struct BucketOp {
 struct RangeRef { uint64_t lo, hi; uint32_t pos; uint32_t inst; };
 
 // Address buckets are contiguous word ranges made of whole "coarse bins" of
-// 2^coarse_bits words.  bin_map[bin] = bucket | (bin - first bin of bucket) << 10,
+// 2^coarse_bits words.  bin_map[bin] = bucket | (bin - first bin of bucket) << kBucketBits,
 // so one lookup gives both the bucket and the word offset inside it.  The map
 // is balanced on a sampled histogram of the batch's access addresses.
 constexpr int kMaxCoarseBins = 1 << 18;

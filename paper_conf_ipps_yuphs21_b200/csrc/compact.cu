@@ -293,7 +293,7 @@ cudaError_t launch_sort_segments(uint4* a, uint4* b, uint64_t n, int chunk_bits,
                                  uint32_t* first, uint4** sorted, cudaStream_t s, int* launches) {
   RsPass ps[8];
   int np = add_field_passes(ps, 0, 2, chunk_bits);
-  np = add_field_passes(ps, np, 3, 10);
+  np = add_field_passes(ps, np, 3, kBucketBits);
   cudaError_t e = cudaSuccess;
   if (n) e = radix_sort(a, b, n, ps, np, cnt, s, launches);
   if (e != cudaSuccess) return e;

@@ -32,9 +32,10 @@ __host__ __device__ constexpr size_t warp_smem_bytes(uint32_t nb) {
   return sizeof(uint4) * (2 * WREC + kSegBuf) + 2 * (2 * WREC) + (((size_t)nb * 2 + 15) & ~(size_t)15);
 }
 
-// Decoded record: info = cnt | b0 << 2 | b1 << 12 (cnt = tracked words 0..2),
+// Decoded record: info = cnt | b0 << 2 | b1 << kB1Shift (cnt = tracked words 0..2),
 // keys k0/k1 = op << 30 | word offset inside the bucket.
 struct Dec { uint32_t info, k0, k1; };
+constexpr int kB1Shift = 2 + kBucketBits;
 
 // Branch-free (predicated) so the four records of a round interleave.
 // flags: bit0 control record, bit1 malformed.  valid = record exists.
@@ -55,14 +56,14 @@ __device__ __forceinline__ Dec decode(uint4 q, bool valid, const PartParams& p, 
   uint32_t m0 = 0, m1 = 0;
   if (in0) m0 = __ldg(p.bin_map + (uint32_t)(rel >> cb));
   if (in1) m1 = __ldg(p.bin_map + (uint32_t)((rel + 1) >> cb));
-  const uint32_t kk0 = (op << 30) | ((m0 >> 10) << cb) | ((uint32_t)rel & msk);
-  const uint32_t kk1 = (op << 30) | ((m1 >> 10) << cb) | ((uint32_t)(rel + 1) & msk);
-  const uint32_t b0 = in0 ? (m0 & 1023u) : (m1 & 1023u);          // 0 when neither word is tracked
-  const uint32_t b1 = in1 ? (m1 & 1023u) : b0;
+  const uint32_t kk0 = (op << 30) | ((m0 >> kBucketBits) << cb) | ((uint32_t)rel & msk);
+  const uint32_t kk1 = (op << 30) | ((m1 >> kBucketBits) << cb) | ((uint32_t)(rel + 1) & msk);
+  const uint32_t b0 = in0 ? (m0 & kBucketMask) : (m1 & kBucketMask);          // 0 when neither word is tracked
+  const uint32_t b1 = in1 ? (m1 & kBucketMask) : b0;
   Dec d;
   d.k0 = in0 ? kk0 : kk1;
   d.k1 = kk1;
-  d.info = ((uint32_t)in0 + (uint32_t)in1) | (b0 << 2) | (b1 << 12);
+  d.info = ((uint32_t)in0 + (uint32_t)in1) | (b0 << 2) | (b1 << kB1Shift);
   return d;
 }
 
@@ -76,7 +77,7 @@ __device__ __forceinline__ void touch(uint16_t* tlist, uint32_t& nT, bool is_new
 // Generic stable rank of one 32-record round (record order, word0 before word1).
 __device__ __forceinline__ void rank_round(uint32_t info, uint16_t* row, uint16_t* tlist, uint32_t& nT,
                                            uint32_t lane, uint32_t lt, uint32_t& r0, uint32_t& r1) {
-  const uint32_t cnt = info & 3u, b0 = (info >> 2) & 1023u, b1 = (info >> 12) & 1023u;
+  const uint32_t cnt = info & 3u, b0 = (info >> 2) & kBucketMask, b1 = (info >> kB1Shift) & kBucketMask;
   r0 = r1 = 0;
   if (__any_sync(FULL, cnt == 2 && b0 != b1)) {
     // a record crossing a bucket boundary: serial over lanes
@@ -214,9 +215,9 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
       const uint32_t lead = __ffs(vml) - 1;
       uint32_t bsrc = 0;
 #pragma unroll
-      for (int k = 0; k < 4; ++k) if ((uint32_t)k == kl) bsrc = (dec[g * 4 + k].info >> 2) & 1023u;
+      for (int k = 0; k < 4; ++k) if ((uint32_t)k == kl) bsrc = (dec[g * 4 + k].info >> 2) & kBucketMask;
       const uint32_t bref = __shfl_sync(FULL, bsrc, lead);
-      const uint32_t iref = bref << 2 | bref << 12;
+      const uint32_t iref = bref << 2 | bref << kB1Shift;
       bool same = true;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
@@ -278,8 +279,8 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     for (int r = 0; r < RPL; ++r) {
       const uint32_t info = dec[r].info, c = info & 3u;
       const uint32_t pos = (uint32_t)(rec0 + (r >> 2) * 128 + (r & 3) * 32 + lane);
-      if (c >= 1) out[row[(info >> 2) & 1023u] + (rk[r] & 0xFFFFu)] = make_uint2(dec[r].k0, pos);
-      if (c == 2) out[row[(info >> 12) & 1023u] + (rk[r] >> 16)] = make_uint2(dec[r].k1, pos);
+      if (c >= 1) out[row[(info >> 2) & kBucketMask] + (rk[r] & 0xFFFFu)] = make_uint2(dec[r].k0, pos);
+      if (c == 2) out[row[(info >> kB1Shift) & kBucketMask] + (rk[r] >> 16)] = make_uint2(dec[r].k1, pos);
     }
     __syncwarp();
     for (uint32_t t = lane; t < nT; t += 32) row[tlist[t]] = 0;

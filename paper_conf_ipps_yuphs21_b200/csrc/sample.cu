@@ -5,7 +5,7 @@
 //            bin 0, at every bin whose exclusive sample prefix enters a new
 //            quantile level (a heavy bin gets a bucket of its own) and at every
 //            2^30-word span boundary.  The histogram is rewritten in place as
-//            the bin map (bucket | offset-in-bins << 10, see arb_internal.h).
+//            the bin map (bucket | offset-in-bins << kBucketBits, see arb_internal.h).
 //            Tiles of 1024 bins are handled by separate CTAs; two one-CTA
 //            scans carry the prefixes between tiles.
 #include "kcommon.cuh"
@@ -93,7 +93,7 @@ __global__ void __launch_bounds__(kT) k_cut_scan(uint32_t* v, uint32_t n, uint32
   if (threadIdx.x == 0) {
     *total_out = carry;
     if (first) {   // quantile target and span cap
-      const uint32_t levels = max(1u, a.max_buckets - 124);
+      const uint32_t levels = max(1u, a.max_buckets - 257);   // <= 256 span cuts (n_words <= 2^38)
       a.misc[1] = max(1u, (carry + levels - 1) / levels);
       const uint64_t span64 = (1ull << 30) >> a.coarse_bits;
       a.misc[2] = span64 == 0 ? 1u : (span64 > 0xFFFFFFFFull ? 0xFFFFFFFFu : (uint32_t)span64);
@@ -148,7 +148,7 @@ __global__ void k_cut_map(CutArgs a) {
   const uint32_t nb = *a.nb_out, total = a.misc[0];
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < a.n_bins; i += gridDim.x * blockDim.x) {
     const uint32_t b = a.bucket_of[i];
-    a.hist_map[i] = b | ((i - a.first_bin[b]) << 10);
+    a.hist_map[i] = b | ((i - a.first_bin[b]) << kBucketBits);
   }
   for (uint32_t b = blockIdx.x * blockDim.x + threadIdx.x; b <= nb; b += gridDim.x * blockDim.x) {
     if (b < nb) a.bucket_start[b] = (uint64_t)a.first_bin[b] << a.coarse_bits;
