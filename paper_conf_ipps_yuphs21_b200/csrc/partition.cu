@@ -37,34 +37,45 @@ __host__ __device__ constexpr size_t warp_smem_bytes(uint32_t nb) {
 struct Dec { uint32_t info, k0, k1; };
 constexpr int kB1Shift = 2 + kBucketBits;
 
-// Branch-free (predicated) so the four records of a round interleave.
-// flags: bit0 control record, bit1 malformed.  valid = record exists.
-__device__ __forceinline__ Dec decode(uint4 q, bool valid, const PartParams& p, uint32_t& ign, uint32_t& flags) {
+// First word of a record, branch-free (predicated) so the four records of a
+// round interleave.  flags: bit0 control record, bit1 malformed.  valid =
+// record exists; two = an unaligned access that also touches the next word
+// (Z4, rare: handled by decode1).  b1 = b0 until decode1 says otherwise.
+__device__ __forceinline__ Dec decode0(uint4 q, bool valid, const PartParams& p, uint32_t& ign, uint32_t& flags,
+                                       bool& two) {
   const uint32_t op = (q.y >> 16) & 0xFFu;
-  const uint32_t len = q.z;
-  const uint64_t addr = ((uint64_t)(q.y & 0xFFFFu) << 32) | q.x;
-  const bool bad_acc = ((q.w & 0xFFFFu) | (uint32_t)(len - 1u > 7u) | (uint32_t)(addr + len > (1ull << 48))) != 0;
-  const bool ctl = op <= 14 && op >= 8 && op != 11;
-  flags = !valid ? 0u : op < 4 ? (bad_acc ? 2u : 0u) : (ctl ? 1u : 2u);
-  const bool ok = valid && op < 4 && !bad_acc;
-  const uint64_t rel = (addr >> 3) - p.base_word;                 // wraps when below the range
+  const uint32_t len = q.z, hi = q.y & 0xFFFFu;
+  // malformed access: len outside 1..8 or the byte range leaving the 48-bit space
+  const bool bad_acc = (q.w & 0xFFFFu) != 0 || len - 1u > 7u || (hi == 0xFFFFu && q.x > 0u - len);
+  const bool ctl = op < 16 && ((0x7700u >> op) & 1u);            // ops 8, 9, 10, 12, 13, 14
+  const bool acc = op < 4;
+  flags = valid ? (acc ? (bad_acc ? 2u : 0u) : (ctl ? 1u : 2u)) : 0u;
+  const bool ok = valid && acc && !bad_acc;
+  const uint64_t rel = ((((uint64_t)hi) << 29) | (q.x >> 3)) - p.base_word;   // wraps below the range
   const bool in0 = ok && rel < p.n_words;
-  const bool two = ok && (q.x & 7u) + len > 8u;                    // unaligned: a second word (Z4)
-  const bool in1 = two && rel + 1 < p.n_words;
-  ign += (uint32_t)(ok && !in0) + (uint32_t)(two && !in1);
-  const uint32_t cb = p.coarse_bits, msk = (1u << cb) - 1u;
-  uint32_t m0 = 0, m1 = 0;
+  two = ok && (q.x & 7u) + len > 8u;
+  ign += (uint32_t)(ok && !in0);
+  const uint32_t cb = p.coarse_bits;
+  uint32_t m0 = 0;
   if (in0) m0 = __ldg(p.bin_map + (uint32_t)(rel >> cb));
-  if (in1) m1 = __ldg(p.bin_map + (uint32_t)((rel + 1) >> cb));
-  const uint32_t kk0 = (op << 30) | ((m0 >> kBucketBits) << cb) | ((uint32_t)rel & msk);
-  const uint32_t kk1 = (op << 30) | ((m1 >> kBucketBits) << cb) | ((uint32_t)(rel + 1) & msk);
-  const uint32_t b0 = in0 ? (m0 & kBucketMask) : (m1 & kBucketMask);          // 0 when neither word is tracked
-  const uint32_t b1 = in1 ? (m1 & kBucketMask) : b0;
+  const uint32_t b0 = m0 & kBucketMask;                          // 0 when untracked
   Dec d;
-  d.k0 = in0 ? kk0 : kk1;
-  d.k1 = kk1;
-  d.info = ((uint32_t)in0 + (uint32_t)in1) | (b0 << 2) | (b1 << kB1Shift);
+  d.k0 = (op << 30) | ((m0 >> kBucketBits) << cb) | ((uint32_t)rel & ((1u << cb) - 1u));
+  d.k1 = 0;
+  d.info = (uint32_t)in0 | (b0 << 2) | (b0 << kB1Shift);
   return d;
+}
+// Second word of an unaligned access (the record is re-read from the stage).
+__device__ __forceinline__ void decode1(Dec& d, uint4 q, const PartParams& p, uint32_t& ign) {
+  const uint32_t op = (q.y >> 16) & 0xFFu;
+  const uint64_t r1 = ((((uint64_t)(q.y & 0xFFFFu)) << 29) | (q.x >> 3)) - p.base_word + 1;
+  if (r1 >= p.n_words) { ++ign; return; }
+  const uint32_t cb = p.coarse_bits;
+  const uint32_t m = __ldg(p.bin_map + (uint32_t)(r1 >> cb));
+  const uint32_t b = m & kBucketMask;
+  const uint32_t k = (op << 30) | ((m >> kBucketBits) << cb) | ((uint32_t)r1 & ((1u << cb) - 1u));
+  if ((d.info & 3u) == 0) { d.k0 = k; d.info = 1u | (b << 2) | (b << kB1Shift); }
+  else { d.k1 = k; d.info = 2u | (d.info & (kBucketMask << 2)) | (b << kB1Shift); }
 }
 
 // append the buckets of lanes with `is_new` to the warp's touched list
@@ -158,17 +169,27 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     // ---- pass A: decode + rank, 2 groups of 4 x 32 records ----------------------------
     Dec dec[RPL];
     uint32_t rk[RPL];
+    bool any2 = false;                 // some record of the chunk has two words
 #pragma unroll
     for (int g = 0; g < 2; ++g) {
-      uint32_t any_flag = 0;
+      uint32_t any_flag = 0, twos = 0;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
         const uint32_t j = g * 128 + k * 32 + lane;
         uint32_t flags;
-        dec[g * 4 + k] = decode(st[j], j < nvalid, p, n_ign, flags);
+        bool two;
+        dec[g * 4 + k] = decode0(st[j], j < nvalid, p, n_ign, flags, two);
         any_flag |= flags << (2 * k);
-        n_acc += dec[g * 4 + k].info & 3u;
+        twos |= (uint32_t)two << k;
       }
+      if (__any_sync(FULL, twos != 0)) {
+        any2 = true;
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+          if ((twos >> k) & 1u) decode1(dec[g * 4 + k], st[g * 128 + k * 32 + lane], p, n_ign);
+      }
+#pragma unroll
+      for (int k = 0; k < 4; ++k) n_acc += dec[g * 4 + k].info & 3u;
       if (__any_sync(FULL, any_flag != 0)) {
         // control / malformed records in the group (rare)
 #pragma unroll
@@ -275,12 +296,20 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     __syncwarp();
     // ---- pass B: write the events straight to the chunk's output slot ----------------------
     uint2* out = p.part_ev + chunk * kChunkCap;
+    const uint32_t pos0 = (uint32_t)rec0 + lane;
 #pragma unroll
     for (int r = 0; r < RPL; ++r) {
-      const uint32_t info = dec[r].info, c = info & 3u;
-      const uint32_t pos = (uint32_t)(rec0 + (r >> 2) * 128 + (r & 3) * 32 + lane);
-      if (c >= 1) out[row[(info >> 2) & kBucketMask] + (rk[r] & 0xFFFFu)] = make_uint2(dec[r].k0, pos);
-      if (c == 2) out[row[(info >> kB1Shift) & kBucketMask] + (rk[r] >> 16)] = make_uint2(dec[r].k1, pos);
+      const uint32_t info = dec[r].info;
+      const uint32_t pos = pos0 + (r >> 2) * 128 + (r & 3) * 32;
+      if (info & 3u) out[row[(info >> 2) & kBucketMask] + (rk[r] & 0xFFFFu)] = make_uint2(dec[r].k0, pos);
+    }
+    if (any2) {
+#pragma unroll
+      for (int r = 0; r < RPL; ++r) {
+        const uint32_t info = dec[r].info;
+        const uint32_t pos = pos0 + (r >> 2) * 128 + (r & 3) * 32;
+        if ((info & 3u) == 2u) out[row[(info >> kB1Shift) & kBucketMask] + (rk[r] >> 16)] = make_uint2(dec[r].k1, pos);
+      }
     }
     __syncwarp();
     for (uint32_t t = lane; t < nT; t += 32) row[tlist[t]] = 0;
