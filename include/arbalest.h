@@ -104,7 +104,10 @@ typedef struct {
   uint64_t ignored_words;    /* word-ops outside the tracked range                        */
   uint64_t buckets, bucket_bits, max_bucket_events;
   uint64_t total_records, total_word_events, total_reports, flushes;
-  /* device time of each phase of the last flush in milliseconds (ARB_F_TIMING) */
+  /* stream time of each phase of the last flush in milliseconds (ARB_F_TIMING):
+     ms_partition = sampling + partition (+ the counter read-back), ms_control =
+     segment sort on the GPU overlapped with host control resolution + op upload,
+     ms_replay = the replay kernel, ms_mir, ms_reports = compaction, ms_total */
   double   ms_partition, ms_control, ms_replay, ms_mir, ms_reports, ms_total;
   uint64_t kernel_launches;  /* kernels launched by the last flush                         */
   double   ms_sample;        /* address sampling + bucket balancing (inside ms_partition)  */

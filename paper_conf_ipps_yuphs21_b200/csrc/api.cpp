@@ -60,6 +60,34 @@ cudaError_t upload(DevBuf<T>& b, const std::vector<T>& v, cudaStream_t s) {
 
 struct Submit { const void* ev; uint64_t n; const uint64_t* gidx; int on_device; };
 
+// pinned host buffer (async copies, no staging through pageable memory)
+template <class T>
+struct HostBuf {
+  T* p = nullptr;
+  size_t cap = 0;
+  cudaError_t ensure(size_t n) {
+    if (n <= cap) return cudaSuccess;
+    size_t c = std::max(n, (size_t)(cap * 3 / 2));
+    if (p) cudaFreeHost(p);
+    p = nullptr; cap = 0;
+    cudaError_t e = cudaMallocHost(&p, c * sizeof(T));
+    if (e == cudaSuccess) cap = c;
+    return e;
+  }
+  void release() { if (p) cudaFreeHost(p); p = nullptr; cap = 0; }
+};
+
+// upload through a pinned staging buffer; the staging buffer is reused only
+// after the flush's final stream synchronisation
+template <class T>
+cudaError_t upload_pinned(DevBuf<T>& b, HostBuf<T>& h, const std::vector<T>& v, cudaStream_t s) {
+  cudaError_t e = b.ensure(std::max<size_t>(v.size(), 1));
+  if (e != cudaSuccess || v.empty()) return e;
+  if ((e = h.ensure(v.size())) != cudaSuccess) return e;
+  std::memcpy(h.p, v.data(), v.size() * sizeof(T));
+  return cudaMemcpyAsync(b.p, h.p, v.size() * sizeof(T), cudaMemcpyHostToDevice, s);
+}
+
 }  // namespace
 
 struct arb_ctx_s {
@@ -104,6 +132,12 @@ struct arb_ctx_s {
   std::string err;
   arb_stats stats{};
   cudaEvent_t ev[8] = {};
+  cudaStream_t aux = nullptr;                 // control-record copies beside the main stream
+  HostBuf<DevStats> h_stats;
+  HostBuf<uint32_t> h_nb, h_ops_start;
+  HostBuf<uint64_t> h_bstart;
+  HostBuf<CtlRec> h_ctl;
+  HostBuf<BucketOp> h_ops;
   // NCCL
   void* nccl_lib = nullptr;
   void* comm = nullptr;
@@ -170,6 +204,10 @@ extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
   if (e == cudaSuccess) e = ctx->dcount.ensure(4);
   if (e == cudaSuccess) e = ctx->ctl.ensure(ctx->ctl_cap);
   for (int i = 0; i < 8 && e == cudaSuccess; ++i) e = cudaEventCreate(&ctx->ev[i]);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->aux, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = ctx->h_stats.ensure(1);
+  if (e == cudaSuccess) e = ctx->h_nb.ensure(1);
+  if (e == cudaSuccess) e = ctx->h_bstart.ensure(kMaxBuckets + 1);
   if (e == cudaSuccess) e = cudaDeviceSynchronize();
   if (e != cudaSuccess) { arb_destroy(ctx); return ARB_ENOMEM; }
   if (cfg->world > 1) {
@@ -203,6 +241,9 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   ctx->m_rr.release(); ctx->hkeys.release(); ctx->hvals.release(); ctx->counts.release();
   ctx->d_bin_map.release(); ctx->d_order.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_cut.release();
   for (auto& e : ctx->ev) if (e) cudaEventDestroy(e);
+  if (ctx->aux) cudaStreamDestroy(ctx->aux);
+  ctx->h_stats.release(); ctx->h_nb.release(); ctx->h_ops_start.release(); ctx->h_bstart.release();
+  ctx->h_ctl.release(); ctx->h_ops.release();
   if (ctx->nccl_lib) dlclose(ctx->nccl_lib);
   delete ctx;
   return ARB_OK;
@@ -295,8 +336,9 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   const uint64_t index_base = ctx->next_index;
 
   if (timing) cudaEventRecord(ctx->ev[0], s);
-  // ---- bucket balancing on a sampled address histogram ------------------------
-  if (ctx->bucket_bits == 0) {
+  const bool balanced = ctx->bucket_bits == 0;
+  // ---- bucket balancing on a sampled address histogram (all on the device) ----
+  if (balanced) {
     CK(ctx->d_hist.ensure(ctx->n_bins), "alloc hist");
     CK(cudaMemsetAsync(ctx->d_hist.p, 0, ctx->n_bins * sizeof(uint32_t), s), "hist clear");
     SampleParams sp{};
@@ -306,49 +348,39 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     const uint64_t n_samples = n ? (n + sp.stride - 1) / sp.stride : 0;
     CK(launch_sample(sp, n_samples, s), "k_sample");
     launches += n_samples ? 1 : 0;
-    // cut balanced buckets on the device; the histogram becomes the bin map in place
+    // cut balanced buckets; the histogram becomes the bin map in place
     CK(ctx->d_bucket_start.ensure(kMaxBuckets + 1), "alloc buckets");
+    CK(ctx->d_order.ensure(kMaxBuckets), "alloc order");
     CK(ctx->d_cut.ensure(2 * kMaxBuckets + 2), "alloc cut scratch");
     CK(ctx->d_cutscr.ensure(2 * ((ctx->n_bins + 1023) / 1024) + 4 + ctx->n_bins), "alloc cut scratch");
     CK(launch_cut(ctx->d_hist.p, ctx->n_bins, ctx->coarse_bits, ctx->n_words, kMaxBuckets, ctx->d_bucket_start.p,
-                  ctx->d_cut.p, ctx->d_cut.p + kMaxBuckets, ctx->d_cut.p + 2 * kMaxBuckets, ctx->d_cutscr.p, s,
-                  &launches), "k_cut");
-    uint32_t nb = 0;
-    CK(cudaMemcpyAsync(&nb, ctx->d_cut.p + 2 * kMaxBuckets, 4, cudaMemcpyDeviceToHost, s), "nb d2h");
-    CK(cudaStreamSynchronize(s), "cut sync");
-    ctx->bucket_start.resize(nb + 1);
-    std::vector<uint32_t> weight(nb);
-    CK(cudaMemcpyAsync(ctx->bucket_start.data(), ctx->d_bucket_start.p, (nb + 1) * 8, cudaMemcpyDeviceToHost, s),
+                  ctx->d_cut.p, ctx->d_cut.p + kMaxBuckets, ctx->d_cut.p + 2 * kMaxBuckets, ctx->d_cutscr.p,
+                  ctx->d_order.p, s, &launches), "k_cut");
+    // the bucket count and starts come back with the partition's counters (one sync)
+    CK(cudaMemcpyAsync(ctx->h_nb.p, ctx->d_cut.p + 2 * kMaxBuckets, 4, cudaMemcpyDeviceToHost, s), "nb d2h");
+    CK(cudaMemcpyAsync(ctx->h_bstart.p, ctx->d_bucket_start.p, (kMaxBuckets + 1) * 8, cudaMemcpyDeviceToHost, s),
        "buckets d2h");
-    CK(cudaMemcpyAsync(weight.data(), ctx->d_cut.p, nb * 4, cudaMemcpyDeviceToHost, s), "weights d2h");
-    CK(cudaStreamSynchronize(s), "cut sync");
-    ctx->order.resize(nb);
-    for (uint32_t b = 0; b < nb; ++b) ctx->order[b] = b;
-    std::stable_sort(ctx->order.begin(), ctx->order.end(),
-                     [&](uint32_t a, uint32_t b) { return weight[a] > weight[b]; });
-    CK(upload(ctx->d_order, ctx->order, s), "upload order");
   } else if (ctx->d_bin_map.cap == 0) {
     CK(upload(ctx->d_bin_map, ctx->bin_map, s), "upload bin map");
     CK(upload(ctx->d_bucket_start, ctx->bucket_start, s), "upload bucket starts");
     CK(upload(ctx->d_order, ctx->order, s), "upload order");
   }
+  if (!balanced) ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;   // fixed buckets
   if (timing) cudaEventRecord(ctx->ev[7], s);
-  ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;
-  S.buckets = ctx->n_buckets;
   // ---- A1/A3a: decode + partition ------------------------------------------
   const uint32_t n_chunks = (uint32_t)((n + kChunkRecords - 1) / kChunkRecords);
   CK(ctx->part_ev.ensure((size_t)std::max<uint32_t>(n_chunks, 1) * kChunkCap), "alloc part_ev");
   if (ctx->seg_cap < (uint64_t)n_chunks * 2 + 4096) ctx->seg_cap = (uint64_t)n_chunks * 2 + 4096;
   CK(ctx->seg_a.ensure(std::max<uint64_t>(ctx->seg_cap, 1)), "alloc segments");
-  DevStats hst;
+  DevStats& hst = *ctx->h_stats.p;
   PartParams pp{};
   for (int attempt = 0; attempt < 2; ++attempt) {
-    std::memset(&hst, 0, sizeof(hst));
-    hst.err_pos = ~0ull;
-    CK(cudaMemcpyAsync(ctx->dstats.p, &hst, sizeof(hst), cudaMemcpyHostToDevice, s), "stats init");
+    CK(cudaMemsetAsync(ctx->dstats.p, 0, sizeof(DevStats), s), "stats init");
+    CK(cudaMemsetAsync(&ctx->dstats.p->err_pos, 0xFF, sizeof(unsigned long long), s), "stats init");
     pp.ev = ev; pp.n = n; pp.base_word = ctx->base_word; pp.n_words = ctx->n_words;
-    pp.coarse_bits = ctx->coarse_bits; pp.bin_map = ctx->bucket_bits ? ctx->d_bin_map.p : ctx->d_hist.p;
-    pp.bucket_bits = ctx->bucket_bits; pp.n_buckets = ctx->n_buckets; pp.n_chunks = n_chunks;
+    pp.coarse_bits = ctx->coarse_bits; pp.bin_map = balanced ? ctx->d_hist.p : ctx->d_bin_map.p;
+    pp.bucket_bits = ctx->bucket_bits; pp.n_buckets = balanced ? (uint32_t)kMaxBuckets : ctx->n_buckets;
+    pp.n_chunks = n_chunks;
     pp.part_ev = ctx->part_ev.p; pp.seg_out = ctx->seg_a.p; pp.seg_cap = ctx->seg_cap;
     pp.ctl = ctx->ctl.p; pp.ctl_cap = ctx->ctl_cap;
     pp.st = ctx->dstats.p;
@@ -367,34 +399,17 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     reset_batch(ctx);
     return fail(ctx, ARB_ETRACE, "malformed record at batch position " + std::to_string(hst.err_pos));
   }
+  if (balanced) {
+    const uint32_t nb = *ctx->h_nb.p;
+    ctx->bucket_start.assign(ctx->h_bstart.p, ctx->h_bstart.p + nb + 1);
+  }
+  ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;
+  S.buckets = ctx->n_buckets;
   S.access_words = hst.access_words;
   S.control_records = hst.n_ctl;
 
-  // ---- A2: control resolution on the host -------------------------------------
-  std::vector<CtlRec> ctl(hst.n_ctl);
-  if (hst.n_ctl) {
-    CK(cudaMemcpy(ctl.data(), ctx->ctl.p, hst.n_ctl * sizeof(CtlRec), cudaMemcpyDeviceToHost), "ctl d2h");
-    std::sort(ctl.begin(), ctl.end(), [](const CtlRec& a, const CtlRec& b) { return a.pos < b.pos; });
-  }
-  MapTable map = ctx->map;
-  FlushPlan plan;
-  resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_start, map, plan);
-  if (plan.rc != 0) {
-    reset_batch(ctx);
-    return fail(ctx, plan.rc, plan.err + " (batch position " + std::to_string(plan.err_pos) + ")");
-  }
-  S.range_words = plan.range_words;
-  S.range_ops = plan.range_ops.size();
-  S.tasks = plan.tasks;
-  S.ignored_words = hst.ignored_words + plan.ignored_words;
-  CK(upload(ctx->ops_start, plan.ops_start, s), "upload ops_start");
-  CK(upload(ctx->ops, plan.ops, s), "upload ops");
-  CK(ctx->cand.ensure(ctx->cand_cap), "alloc candidates");
-  if (timing) cudaEventRecord(ctx->ev[2], s);
-
-  // ---- A3b/A4/A5: replay ---------------------------------------------------------
-  ReplayParams rp{};
-  // segment entries sorted by (bucket, chunk) and each bucket's first entry
+  // ---- A3b: segment entries sorted by (bucket, chunk) — on the GPU while the
+  // host resolves the control records ------------------------------------------------
   uint4* segs_sorted = ctx->seg_a.p;
   {
     const uint64_t ns = hst.n_segs;
@@ -408,6 +423,36 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     CK(launch_sort_segments(a, b2, ns, cb, ctx->n_buckets, ctx->blk.p, ctx->seg_first.p, &segs_sorted, s, &launches),
        "sort segments");
   }
+
+  // ---- A2: control resolution on the host -------------------------------------
+  std::vector<CtlRec> ctl(hst.n_ctl);
+  if (hst.n_ctl) {
+    CK(ctx->h_ctl.ensure(hst.n_ctl), "pinned ctl");
+    CK(cudaMemcpyAsync(ctx->h_ctl.p, ctx->ctl.p, hst.n_ctl * sizeof(CtlRec), cudaMemcpyDeviceToHost, ctx->aux),
+       "ctl d2h");
+    CK(cudaStreamSynchronize(ctx->aux), "ctl sync");
+    std::memcpy(ctl.data(), ctx->h_ctl.p, hst.n_ctl * sizeof(CtlRec));
+    std::sort(ctl.begin(), ctl.end(), [](const CtlRec& a, const CtlRec& b) { return a.pos < b.pos; });
+  }
+  MapTable map = ctx->map;
+  FlushPlan plan;
+  resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_start, map, plan);
+  if (plan.rc != 0) {
+    CK(cudaStreamSynchronize(s), "sync");
+    reset_batch(ctx);
+    return fail(ctx, plan.rc, plan.err + " (batch position " + std::to_string(plan.err_pos) + ")");
+  }
+  S.range_words = plan.range_words;
+  S.range_ops = plan.range_ops.size();
+  S.tasks = plan.tasks;
+  S.ignored_words = hst.ignored_words + plan.ignored_words;
+  CK(upload_pinned(ctx->ops_start, ctx->h_ops_start, plan.ops_start, s), "upload ops_start");
+  CK(upload_pinned(ctx->ops, ctx->h_ops, plan.ops, s), "upload ops");
+  CK(ctx->cand.ensure(ctx->cand_cap), "alloc candidates");
+  if (timing) cudaEventRecord(ctx->ev[2], s);
+
+  // ---- A3b/A4/A5: replay ---------------------------------------------------------
+  ReplayParams rp{};
   rp.part_ev = ctx->part_ev.p; rp.segs = segs_sorted; rp.seg_first = ctx->seg_first.p;
   rp.n_buckets = ctx->n_buckets; rp.bucket_bits = ctx->bucket_bits; rp.n_words = ctx->n_words;
   rp.bucket_start = ctx->d_bucket_start.p; rp.order = ctx->d_order.p;

@@ -144,10 +144,11 @@ struct MirParams {
 
 // ---- kernel launchers (kernels.cu) -----------------------------------------
 cudaError_t launch_sample(const SampleParams& p, uint64_t n_samples, cudaStream_t s);
-// scratch: 2 * ceil(n_bins / 1024) + 4 + n_bins u32
+// scratch: 2 * ceil(n_bins / 1024) + 4 + n_bins u32.  Writes the bucket count
+// (*nb_out), bucket starts, weights and the replay order (heaviest first).
 cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits, uint64_t n_words,
                        uint32_t max_buckets, uint64_t* bucket_start, uint32_t* weight, uint32_t* first_bin,
-                       uint32_t* nb_out, uint32_t* scratch, cudaStream_t s, int* launches);
+                       uint32_t* nb_out, uint32_t* scratch, uint32_t* order, cudaStream_t s, int* launches);
 cudaError_t launch_partition(const PartParams& p, cudaStream_t s);
 // sorts the segment entries by (bucket, chunk), writes each entry's exclusive
 // event prefix into .w and each bucket's first entry; cnt: (n / 4096 + 1) * 256 u32

@@ -10,4 +10,4 @@ for it in range(2):
     for a, b in flushes:
         ctx.submit_events(recs[a:b], global_index=gidx[a:b]); ctx.flush()
         st = ctx.stats()
-        print({k: st[k] for k in ('records','access_words','range_words','buckets','max_bucket_events','steps_fast','steps_sort','ms_sample','ms_partition','ms_replay','ms_mir','ms_reports','ms_total','range_ops')})
+        print({k: (round(st[k],3) if isinstance(st[k], float) else st[k]) for k in ('records','buckets','max_bucket_events','steps_sort','ms_sample','ms_partition','ms_control','ms_replay','ms_mir','ms_reports','ms_total')})
