@@ -106,7 +106,8 @@ struct arb_ctx_s {
   DevBuf<uint4> staging;
   DevBuf<uint64_t> gidx_staging;
   DevBuf<uint2> part_ev;
-  DevBuf<uint4> seg_a, seg_b;
+  DevBuf<uint2> seg_a, seg_b;                 // partition entries, sort ping-pong
+  DevBuf<uint4> segs;                         // replay form
   DevBuf<uint32_t> seg_first;
   uint64_t seg_cap = 0;
   DevBuf<CtlRec> ctl;
@@ -171,14 +172,14 @@ extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
   ctx->cfg = *cfg;
   ctx->base_word = cfg->addr_base >> 3;
   ctx->n_words = cfg->addr_bytes >> 3;
-  // Address buckets.  bucket_bits != 0: fixed buckets of 2^bits words (<= 1024
+  // Address buckets.  bucket_bits != 0: fixed buckets of 2^bits words (<= 2048
   // of them).  0: buckets balanced per flush on a sampled address histogram over
-  // <= 2^16 coarse bins (<= 1024 buckets of <= 2^30 words).
+  // <= 2^18 coarse bins (<= 2048 buckets of <= 2^30 words).
   if (ctx->n_words > (1ull << 38)) { delete ctx; return ARB_EINVAL; }
   uint32_t bits = cfg->bucket_bits;
   if (bits) {
     uint64_t nb = (ctx->n_words + (1ull << bits) - 1) >> bits;
-    if (bits > 30 || nb > (uint64_t)kMaxBuckets) { delete ctx; return ARB_EINVAL; }
+    if (bits > kMaxBucketSpanBits || nb > (uint64_t)kMaxBuckets) { delete ctx; return ARB_EINVAL; }
     ctx->coarse_bits = bits;
     ctx->bin_map.resize(nb);
     ctx->bucket_start.clear();
@@ -232,7 +233,7 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   if (!ctx) return ARB_OK;
   if (ctx->comm && ctx->nccl_destroy) ctx->nccl_destroy(ctx->comm);
   if (ctx->shadow) cudaFree(ctx->shadow);
-  ctx->staging.release(); ctx->gidx_staging.release(); ctx->part_ev.release(); ctx->seg_a.release(); ctx->seg_b.release(); ctx->seg_first.release();
+  ctx->staging.release(); ctx->gidx_staging.release(); ctx->part_ev.release(); ctx->seg_a.release(); ctx->seg_b.release(); ctx->segs.release(); ctx->seg_first.release();
   ctx->ctl.release(); ctx->cand.release(); ctx->cand_tmp.release(); ctx->reports.release(); ctx->blk.release();
   ctx->ops_start.release(); ctx->ops.release(); ctx->dstats.release(); ctx->dcount.release();
   ctx->m_ins_lo.release(); ctx->m_ins_cum.release(); ctx->m_qry_lo.release(); ctx->m_qry_cum.release();
@@ -259,7 +260,7 @@ extern "C" int arb_submit_events(arb_ctx ctx, const arb_event* ev, uint64_t n, c
   if (!ctx) return ARB_EINVAL;
   if (n == 0) return ARB_OK;
   if (!ev) return fail(ctx, ARB_EINVAL, "null event pointer");
-  if (ctx->pending + n > kMaxBatchRecords) return fail(ctx, ARB_EINVAL, "batch exceeds 2^30 records");
+  if (ctx->pending + n > kMaxBatchRecords) return fail(ctx, ARB_EINVAL, "batch exceeds 2^29 records");
   if ((global_index != nullptr && ctx->any_nogidx) || (global_index == nullptr && ctx->any_gidx))
     return fail(ctx, ARB_EINVAL, "global_index must be given for every submit of a batch or for none");
   cudaSetDevice(ctx->cfg.device);
@@ -410,18 +411,16 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
 
   // ---- A3b: segment entries sorted by (bucket, chunk) — on the GPU while the
   // host resolves the control records ------------------------------------------------
-  uint4* segs_sorted = ctx->seg_a.p;
   {
     const uint64_t ns = hst.n_segs;
     CK(ctx->seg_b.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
+    CK(ctx->segs.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
     CK(ctx->seg_first.ensure(ctx->n_buckets + 1), "alloc seg_first");
     CK(ctx->blk.ensure((ns + 4095) / 4096 * 256 + 4096), "alloc blk");
     int cb = 1;
-    while (cb < 32 && ((uint64_t)n_chunks >> cb)) ++cb;
-    uint4* a = ctx->seg_a.p;
-    uint4* b2 = ctx->seg_b.p;
-    CK(launch_sort_segments(a, b2, ns, cb, ctx->n_buckets, ctx->blk.p, ctx->seg_first.p, &segs_sorted, s, &launches),
-       "sort segments");
+    while (cb < kSegChunkBits && ((uint64_t)n_chunks >> cb)) ++cb;
+    CK(launch_sort_segments(ctx->seg_a.p, ctx->seg_b.p, ns, cb, ctx->n_buckets, ctx->blk.p, ctx->seg_first.p,
+                            ctx->segs.p, s, &launches), "sort segments");
   }
 
   // ---- A2: control resolution on the host -------------------------------------
@@ -453,7 +452,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
 
   // ---- A3b/A4/A5: replay ---------------------------------------------------------
   ReplayParams rp{};
-  rp.part_ev = ctx->part_ev.p; rp.segs = segs_sorted; rp.seg_first = ctx->seg_first.p;
+  rp.part_ev = ctx->part_ev.p; rp.segs = ctx->segs.p; rp.seg_first = ctx->seg_first.p;
   rp.n_buckets = ctx->n_buckets; rp.bucket_bits = ctx->bucket_bits; rp.n_words = ctx->n_words;
   rp.bucket_start = ctx->d_bucket_start.p; rp.order = ctx->d_order.p;
   rp.shadow = ctx->shadow; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;

@@ -35,8 +35,10 @@ constexpr Sel kSelREL   = sel_make(0, 4, 2, 4);   // released CV: same bits as a
 
 // ---- compact event (partition output, 8 B) ---------------------------------
 // x: [0,30) word offset inside the address bucket | [30,32) access op (RH/WH/RT/WT)
-// y: record position inside the batch (< 2^30)
-constexpr uint32_t kMaxBatchRecords = 1u << 30;
+// y: record position inside the batch (< 2^29)
+constexpr int kMaxBucketSpanBits = 30;               // buckets span <= 2^30 words
+constexpr uint32_t kMaxBatchRecords = 1u << 29;
+constexpr int kSegChunkBits = 21;                    // chunk ids of a batch fit 21 bits
 
 // ---- partition geometry ----------------------------------------------------
 constexpr int kPartThreads = 512;
@@ -102,7 +104,8 @@ struct PartParams {
   uint32_t bucket_bits, n_buckets;
   uint32_t n_chunks;
   uint2* part_ev;                         // [n_chunks][kChunkCap]
-  uint4* seg_out; uint64_t seg_cap;       // {chunk, bucket, start | len << 16, -} per touched bucket
+  uint2* seg_out; uint64_t seg_cap;       // {bucket << kSegChunkBits | chunk, start | len << 16} per
+                                          // touched bucket of a chunk
   CtlRec* ctl; uint64_t ctl_cap;
   DevStats* st;
 };
@@ -150,10 +153,12 @@ cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits
                        uint32_t max_buckets, uint64_t* bucket_start, uint32_t* weight, uint32_t* first_bin,
                        uint32_t* nb_out, uint32_t* scratch, uint32_t* order, cudaStream_t s, int* launches);
 cudaError_t launch_partition(const PartParams& p, cudaStream_t s);
-// sorts the segment entries by (bucket, chunk), writes each entry's exclusive
-// event prefix into .w and each bucket's first entry; cnt: (n / 4096 + 1) * 256 u32
-cudaError_t launch_sort_segments(uint4* a, uint4* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
-                                 uint32_t* first, uint4** sorted, cudaStream_t s, int* launches);
+// Sorts the 8-B segment entries {bucket << kSegChunkBits | chunk, start | len << 16}
+// by (bucket, chunk) (a, b: ping-pong buffers), writes the replay form
+// {chunk, bucket, start | len << 16, exclusive event prefix} to out and each
+// bucket's first entry; cnt: (n / 4096 + 1) * 256 + 4096 u32
+cudaError_t launch_sort_segments(uint2* a, uint2* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
+                                 uint32_t* first, uint4* out, cudaStream_t s, int* launches);
 cudaError_t launch_replay(const ReplayParams& p, int n_ctas, cudaStream_t s);
 cudaError_t launch_mir(const MirParams& p, uint64_t n_ins_pos, uint64_t n_qry_pos, uint64_t n_rr_words,
                        cudaStream_t s, int* launches);

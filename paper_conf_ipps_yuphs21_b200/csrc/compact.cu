@@ -7,12 +7,16 @@ namespace arb {
 constexpr int kRsThreads = 512, kRsItems = 8, kRsTile = kRsThreads * kRsItems;
 
 struct RsPass { int field; int shift; int bits; };
-__device__ __forceinline__ uint32_t rs_digit(uint4 c, RsPass ps) {
-  uint32_t f = ps.field == 0 ? c.w : ps.field == 1 ? c.z : ps.field == 2 ? c.x : c.y;
-  return (f >> ps.shift) & ((1u << ps.bits) - 1u);
+// digit fields: uint4 {0: w, 1: z, 2: x, 3: y}; uint2 {0: x, 1: y}
+__device__ __forceinline__ uint32_t rs_field(uint4 c, int f) { return f == 0 ? c.w : f == 1 ? c.z : f == 2 ? c.x : c.y; }
+__device__ __forceinline__ uint32_t rs_field(uint2 c, int f) { return f == 0 ? c.x : c.y; }
+template <class E>
+__device__ __forceinline__ uint32_t rs_digit(E c, RsPass ps) {
+  return (rs_field(c, ps.field) >> ps.shift) & ((1u << ps.bits) - 1u);
 }
 
-__global__ void __launch_bounds__(kRsThreads) k_rs_hist(const uint4* in, uint64_t n, RsPass ps, uint32_t* cnt,
+template <class E>
+__global__ void __launch_bounds__(kRsThreads) k_rs_hist(const E* in, uint64_t n, RsPass ps, uint32_t* cnt,
                                                         uint32_t nblk) {
   __shared__ uint32_t h[256];
   for (int i = threadIdx.x; i < 256; i += kRsThreads) h[i] = 0;
@@ -101,7 +105,8 @@ static void scan_u32(uint32_t* a, uint64_t n, uint32_t* scratch, cudaStream_t s,
   *launches += 3;
 }
 
-__global__ void __launch_bounds__(kRsThreads) k_rs_scatter(const uint4* in, uint4* out, uint64_t n, RsPass ps,
+template <class E>
+__global__ void __launch_bounds__(kRsThreads) k_rs_scatter(const E* in, E* out, uint64_t n, RsPass ps,
                                                            const uint32_t* cnt, uint32_t nblk) {
   __shared__ uint16_t hist[kRsThreads / 32][256];
   __shared__ uint32_t dbase[256];
@@ -110,12 +115,12 @@ __global__ void __launch_bounds__(kRsThreads) k_rs_scatter(const uint4* in, uint
   for (uint32_t i = tid; i < (kRsThreads / 32) * 128; i += kRsThreads) h32[i] = 0;
   __syncthreads();
   uint64_t base = (uint64_t)blockIdx.x * kRsTile;
-  uint4 c[kRsItems]; uint32_t rk[kRsItems], dg[kRsItems];
+  E c[kRsItems]; uint32_t rk[kRsItems], dg[kRsItems];
   const uint32_t lt = lanemask_lt();
   for (int r = 0; r < kRsItems; ++r) {
     uint64_t i = base + warp * (32 * kRsItems) + r * 32 + lane;
     bool valid = i < n;
-    c[r] = valid ? in[i] : make_uint4(0, 0, 0, 0);
+    if (valid) c[r] = in[i];
     uint32_t d = valid ? rs_digit(c[r], ps) : 0xFFFFu;
     uint32_t grp = __match_any_sync(FULL, d);
     uint32_t b = valid ? hist[warp][d] : 0;
@@ -214,15 +219,16 @@ __global__ void __launch_bounds__(kRsThreads) k_keep_write(const uint4* a, uint6
   if (blockIdx.x == nblk - 1 && threadIdx.x == kRsThreads - 1) *n_out = o;
 }
 
-static cudaError_t radix_sort(uint4*& a, uint4*& b, uint64_t n, const RsPass* passes, int np, uint32_t* cnt,
+template <class E>
+static cudaError_t radix_sort(E*& a, E*& b, uint64_t n, const RsPass* passes, int np, uint32_t* cnt,
                               cudaStream_t s, int* launches) {
   uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
   for (int k = 0; k < np; ++k) {
-    k_rs_hist<<<nblk, kRsThreads, 0, s>>>(a, n, passes[k], cnt, nblk);
+    k_rs_hist<E><<<nblk, kRsThreads, 0, s>>>(a, n, passes[k], cnt, nblk);
     scan_u32(cnt, (uint64_t)nblk * 256, cnt + (uint64_t)nblk * 256, s, launches);
-    k_rs_scatter<<<nblk, kRsThreads, 0, s>>>(a, b, n, passes[k], cnt, nblk);
+    k_rs_scatter<E><<<nblk, kRsThreads, 0, s>>>(a, b, n, passes[k], cnt, nblk);
     *launches += 2;
-    uint4* t = a; a = b; b = t;
+    E* t = a; a = b; b = t;
   }
   return cudaGetLastError();
 }
@@ -232,23 +238,27 @@ static int add_field_passes(RsPass* ps, int np, int field, int bits) {
   return np;
 }
 
-// first entry of every bucket in the (bucket, chunk)-sorted segment entries
-__global__ void k_seg_first(const uint4* segs, uint64_t n, uint32_t n_buckets, uint32_t* first) {
+// Segment entries as written by k_partition (8 B): x = bucket << kSegChunkBits |
+// chunk, y = start | len << 16.  Sorted by x they are in (bucket, chunk) order.
+__device__ __forceinline__ uint32_t seg_bucket(uint2 e) { return e.x >> kSegChunkBits; }
+
+// first entry of every bucket in the sorted entries
+__global__ void k_seg_first(const uint2* segs, uint64_t n, uint32_t n_buckets, uint32_t* first) {
   for (uint32_t b = blockIdx.x * blockDim.x + threadIdx.x; b <= n_buckets; b += gridDim.x * blockDim.x) {
     uint64_t a = 0, z = n;                 // first entry with bucket >= b
-    while (a < z) { const uint64_t mid = (a + z) >> 1; if (segs[mid].y < b) a = mid + 1; else z = mid; }
+    while (a < z) { const uint64_t mid = (a + z) >> 1; if (seg_bucket(segs[mid]) < b) a = mid + 1; else z = mid; }
     first[b] = (uint32_t)a;
   }
 }
 
-// event count of each tile of segment entries (blocked: thread t owns 8 entries)
-__global__ void __launch_bounds__(kRsThreads) k_seg_tile_sum(const uint4* segs, uint64_t n, uint32_t* blk) {
+// event count of each tile of sorted entries (blocked: thread t owns 8 entries)
+__global__ void __launch_bounds__(kRsThreads) k_seg_tile_sum(const uint2* segs, uint64_t n, uint32_t* blk) {
   __shared__ uint32_t red[kRsThreads / 32];
   const uint64_t base = (uint64_t)blockIdx.x * kRsTile + (uint64_t)threadIdx.x * kRsItems;
   uint32_t c = 0;
 #pragma unroll
   for (int j = 0; j < kRsItems; ++j)
-    if (base + j < n) c += segs[base + j].z >> 16;
+    if (base + j < n) c += segs[base + j].y >> 16;
   for (int d = 16; d; d >>= 1) c += __shfl_xor_sync(FULL, c, d);
   if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = c;
   __syncthreads();
@@ -258,16 +268,18 @@ __global__ void __launch_bounds__(kRsThreads) k_seg_tile_sum(const uint4* segs, 
     blk[blockIdx.x] = t;
   }
 }
-// .w = exclusive prefix of the event counts over the whole array
-__global__ void __launch_bounds__(kRsThreads) k_seg_cum(uint4* segs, uint64_t n, const uint32_t* blk) {
+// replay form {chunk, bucket, start | len << 16, exclusive event prefix over the array}
+__global__ void __launch_bounds__(kRsThreads) k_seg_cum(const uint2* segs, uint64_t n, const uint32_t* blk,
+                                                        uint4* out) {
   __shared__ uint32_t ws[kRsThreads / 32];
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint64_t base = (uint64_t)blockIdx.x * kRsTile + (uint64_t)threadIdx.x * kRsItems;
-  uint32_t len[kRsItems], c = 0;
+  uint2 e[kRsItems];
+  uint32_t c = 0;
 #pragma unroll
   for (int j = 0; j < kRsItems; ++j) {
-    len[j] = base + j < n ? segs[base + j].z >> 16 : 0;
-    c += len[j];
+    e[j] = base + j < n ? segs[base + j] : make_uint2(0, 0);
+    c += e[j].y >> 16;
   }
   uint32_t incl = c;
   for (int d = 1; d < 32; d <<= 1) {
@@ -280,29 +292,26 @@ __global__ void __launch_bounds__(kRsThreads) k_seg_cum(uint4* segs, uint64_t n,
   for (uint32_t w = 0; w < warp; ++w) run += ws[w];
 #pragma unroll
   for (int j = 0; j < kRsItems; ++j) {
-    if (base + j < n) segs[base + j].w = run;
-    run += len[j];
+    if (base + j < n)
+      out[base + j] = make_uint4(e[j].x & ((1u << kSegChunkBits) - 1u), seg_bucket(e[j]), e[j].y, run);
+    run += e[j].y >> 16;
   }
 }
 
-// Sort the partition's segment entries {chunk, bucket, start|len<<16, -} by
-// (bucket, chunk) — stable LSD passes on the chunk then the bucket field —
-// write the exclusive event prefix into .w and compute each bucket's first
-// entry.  *sorted points at the result (a or b).
-cudaError_t launch_sort_segments(uint4* a, uint4* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
-                                 uint32_t* first, uint4** sorted, cudaStream_t s, int* launches) {
+cudaError_t launch_sort_segments(uint2* a, uint2* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
+                                 uint32_t* first, uint4* out, cudaStream_t s, int* launches) {
   RsPass ps[8];
-  int np = add_field_passes(ps, 0, 2, chunk_bits);
-  np = add_field_passes(ps, np, 3, kBucketBits);
+  int np = 0;
+  for (int sh = 0; sh < chunk_bits; sh += 8) ps[np++] = RsPass{0, sh, chunk_bits - sh < 8 ? chunk_bits - sh : 8};
+  for (int sh = kSegChunkBits; sh < 32; sh += 8) ps[np++] = RsPass{0, sh, 32 - sh < 8 ? 32 - sh : 8};
   cudaError_t e = cudaSuccess;
   if (n) e = radix_sort(a, b, n, ps, np, cnt, s, launches);
   if (e != cudaSuccess) return e;
-  *sorted = a;
   if (n) {
     const uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
     k_seg_tile_sum<<<nblk, kRsThreads, 0, s>>>(a, n, cnt);
     scan_u32(cnt, nblk, cnt + nblk, s, launches);
-    k_seg_cum<<<nblk, kRsThreads, 0, s>>>(a, n, cnt);
+    k_seg_cum<<<nblk, kRsThreads, 0, s>>>(a, n, cnt, out);
     *launches += 2;
   }
   k_seg_first<<<(n_buckets + 256) / 256, 256, 0, s>>>(a, n, n_buckets, first);
@@ -326,7 +335,7 @@ cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches
     np = add_field_passes(ps, np, 0, 2);
     np = add_field_passes(ps, np, 2, wb_lo);
     np = add_field_passes(ps, np, 3, wb_hi);
-    if ((e = radix_sort(a, b, n, ps, np, p.blk, s, launches)) != cudaSuccess) return e;
+    if ((e = radix_sort<uint4>(a, b, n, ps, np, p.blk, s, launches)) != cudaSuccess) return e;
     uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
     k_keep_count<<<nblk, kRsThreads, 0, s>>>(a, n, 1, p.blk);
     scan_u32(p.blk, nblk, p.blk + nblk, s, launches);
@@ -344,7 +353,7 @@ cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches
   np = add_field_passes(ps, np, 1, p.pos_bits);
   np = add_field_passes(ps, np, 2, wb_lo);
   np = add_field_passes(ps, np, 3, wb_hi);
-  if ((e = radix_sort(a, b, n, ps, np, p.blk, s, launches)) != cudaSuccess) return e;
+  if ((e = radix_sort<uint4>(a, b, n, ps, np, p.blk, s, launches)) != cudaSuccess) return e;
   uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
   if (n == 0) {
     cudaMemsetAsync(p.n_out, 0, 4 * sizeof(unsigned long long), s);

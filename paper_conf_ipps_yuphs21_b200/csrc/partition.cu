@@ -13,7 +13,7 @@
 //              it to the warp's touched list; a warp scan over that list turns
 //              the counts into offsets.  Events are written straight to the
 //              chunk's 512-event slot of the output, grouped by bucket in trace
-//              order, and one {chunk, bucket, start | len << 16} entry per touched
+//              order, and one {bucket:chunk, start | len << 16} entry per touched
 //              bucket is appended (batched per warp) for the replay.
 #include "kcommon.cuh"
 #include <algorithm>
@@ -26,10 +26,10 @@ constexpr int WREC = kChunkRecords;         // 256 records per chunk
 constexpr int RPL = WREC / 32;              // 8 records per lane (two groups of 4 x 32)
 constexpr int kSegBuf = 64;                 // segment entries buffered per warp
 
-// per-warp shared memory: stage[2][WREC] uint4, segbuf[kSegBuf] uint4,
+// per-warp shared memory: stage[2][WREC] uint4, segbuf[kSegBuf] uint2,
 // tlist[2 * WREC] u16, row[NB] u16 (padded to 16 B)
 __host__ __device__ constexpr size_t warp_smem_bytes(uint32_t nb) {
-  return sizeof(uint4) * (2 * WREC + kSegBuf) + 2 * (2 * WREC) + (((size_t)nb * 2 + 15) & ~(size_t)15);
+  return sizeof(uint4) * 2 * WREC + sizeof(uint2) * kSegBuf + 2 * (2 * WREC) + (((size_t)nb * 2 + 15) & ~(size_t)15);
 }
 
 // Decoded record: info = cnt | b0 << 2 | b1 << kB1Shift (cnt = tracked words 0..2),
@@ -123,7 +123,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   const uint32_t lt = lanemask_lt();
   uint8_t* wbase = smem + warp * warp_smem_bytes(NB);
   uint4* stage = reinterpret_cast<uint4*>(wbase);                   // [2][WREC]
-  uint4* segbuf = stage + 2 * WREC;                                  // [kSegBuf]
+  uint2* segbuf = reinterpret_cast<uint2*>(stage + 2 * WREC);       // [kSegBuf]
   uint16_t* tlist = reinterpret_cast<uint16_t*>(segbuf + kSegBuf);   // [2 * WREC]
   uint16_t* row = tlist + 2 * WREC;                                  // [NB]
   for (uint32_t i = lane; i < NB; i += 32) row[i] = 0;
@@ -165,7 +165,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     const uint4* st = stage + cur * WREC;
     const uint64_t rec0 = chunk * WREC;
     const uint32_t nvalid = p.n - rec0 < (uint64_t)WREC ? (uint32_t)(p.n - rec0) : (uint32_t)WREC;
-    uint32_t nT = 0;
+    uint32_t nT = 0, e_lane = 0;
     // ---- pass A: decode + rank, 2 groups of 4 x 32 records ----------------------------
     Dec dec[RPL];
     uint32_t rk[RPL];
@@ -189,7 +189,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
           if ((twos >> k) & 1u) decode1(dec[g * 4 + k], st[g * 128 + k * 32 + lane], p, n_ign);
       }
 #pragma unroll
-      for (int k = 0; k < 4; ++k) n_acc += dec[g * 4 + k].info & 3u;
+      for (int k = 0; k < 4; ++k) e_lane += dec[g * 4 + k].info & 3u;
       if (__any_sync(FULL, any_flag != 0)) {
         // control / malformed records in the group (rare)
 #pragma unroll
@@ -272,30 +272,31 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     }
     __syncwarp();
     // ---- counts -> offsets over the touched list; segment entries ------------------------
+    uint2* out = p.part_ev + chunk * kChunkCap;
     uint32_t carry = 0;
     for (uint32_t t0 = 0; t0 < nT; t0 += 32) {
       const uint32_t t = t0 + lane;
       uint32_t b = 0, tot = 0;
       if (t < nT) { b = tlist[t]; tot = row[b]; }
-      uint32_t incl = tot;
+      const uint32_t len = tot;
+      uint32_t incl = len;
 #pragma unroll
       for (int d = 1; d < 32; d <<= 1) {
         const uint32_t o = __shfl_up_sync(FULL, incl, d);
         if (lane >= (uint32_t)d) incl += o;
       }
-      const uint32_t start = carry + incl - tot;
+      const uint32_t start = carry + incl - len;
       carry += __shfl_sync(FULL, incl, 31);
       const uint32_t n_new = min(32u, nT - t0);
       if (nbuf + n_new > kSegBuf) flush_segs();
       if (t < nT) {
         row[b] = (uint16_t)start;
-        segbuf[nbuf + lane] = make_uint4((uint32_t)chunk, b, start | (tot << 16), 0);
+        segbuf[nbuf + lane] = make_uint2((b << kSegChunkBits) | (uint32_t)chunk, start | (len << 16));
       }
       nbuf += n_new;
     }
     __syncwarp();
     // ---- pass B: write the events straight to the chunk's output slot ----------------------
-    uint2* out = p.part_ev + chunk * kChunkCap;
     const uint32_t pos0 = (uint32_t)rec0 + lane;
 #pragma unroll
     for (int r = 0; r < RPL; ++r) {
@@ -313,6 +314,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     }
     __syncwarp();
     for (uint32_t t = lane; t < nT; t += 32) row[tlist[t]] = 0;
+    n_acc += e_lane;
     cur ^= 1;
     __syncwarp();                      // stage[cur] reads and row resets done before reuse
   }

@@ -93,9 +93,11 @@ __global__ void __launch_bounds__(kT) k_cut_scan(uint32_t* v, uint32_t n, uint32
   if (threadIdx.x == 0) {
     *total_out = carry;
     if (first) {   // quantile target and span cap
-      const uint32_t levels = max(1u, a.max_buckets - 257);   // <= 256 span cuts (n_words <= 2^38)
+      // leave room for the span cuts (n_words / 2^30 + 1 of them, <= 257)
+      const uint32_t spans = (uint32_t)(a.n_words >> kMaxBucketSpanBits) + 1;
+      const uint32_t levels = max(1u, a.max_buckets - spans - 1);
       a.misc[1] = max(1u, (carry + levels - 1) / levels);
-      const uint64_t span64 = (1ull << 30) >> a.coarse_bits;
+      const uint64_t span64 = (1ull << kMaxBucketSpanBits) >> a.coarse_bits;
       a.misc[2] = span64 == 0 ? 1u : (span64 > 0xFFFFFFFFull ? 0xFFFFFFFFu : (uint32_t)span64);
     }
   }
