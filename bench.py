@@ -167,7 +167,8 @@ def run_reference(args):
     hi = lo + (native.C5_SHARD_WORDS if prog.name == "config5" else prog.addr_bytes // 8)
     sample = args.ref_sample
     rec, gi = prog.filter_host(word_lo=lo, word_hi=hi, start=0, count=min(prog.n, sample * 8))
-    rec, gi = rec[:sample], gi[:sample]
+    cut = quiescent_prefix(prog, gi, sample)
+    rec, gi = rec[:cut], gi[:cut]
     times, evs = [], 0
     for s in range(args.warmup + args.steps):
         t0 = time.perf_counter()
@@ -190,9 +191,22 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def quiescent_prefix(prog, gidx, budget):
+    """Largest prefix of a rank's records (global indices gidx, ascending) that ends
+    at a quiescent point of the program and holds <= budget records (else the
+    shortest non-empty one): a bounded sample never cuts a nowait block open."""
+    q = np.asarray(prog.quiescent, dtype=np.int64)
+    local = np.unique(np.searchsorted(np.asarray(gidx, dtype=np.int64), q))
+    local = local[local > 0]
+    if local.size == 0:
+        return len(gidx)
+    ok = local[local <= budget]
+    return int(ok[-1]) if ok.size else int(local[0])
+
+
 def cpu_baseline(prog, recs_dev, gidx_dev, lo, hi, budget_records):
     import oracle
-    n = min(budget_records, recs_dev.shape[0])
+    n = quiescent_prefix(prog, gidx_dev.cpu().numpy(), min(budget_records, recs_dev.shape[0]))
     rec = recs_dev[:n].cpu().numpy().view(np.uint64)
     gi = gidx_dev[:n].cpu().numpy().view(np.uint64)
     t0 = time.perf_counter()

@@ -131,7 +131,7 @@ int arb_init(const arb_config* cfg, arb_ctx* out);
  *               same memory space as ev (sharded mode: the rank sees a subset of
  *               the global trace, in order).  Read only on the report path.
  *  stream       cudaStream_t (NULL = legacy default stream).
- * Records of one batch keep their relative order; a batch holds at most 2^29
+ * Records of one batch keep their relative order; a batch holds at most 2^30
  * records.  Errors: ARB_EINVAL, ARB_ENOMEM, ARB_ECUDA. */
 int arb_submit_events(arb_ctx ctx, const arb_event* ev, uint64_t n,
                       const uint64_t* global_index, int ev_on_device, void* stream);

@@ -260,7 +260,7 @@ extern "C" int arb_submit_events(arb_ctx ctx, const arb_event* ev, uint64_t n, c
   if (!ctx) return ARB_EINVAL;
   if (n == 0) return ARB_OK;
   if (!ev) return fail(ctx, ARB_EINVAL, "null event pointer");
-  if (ctx->pending + n > kMaxBatchRecords) return fail(ctx, ARB_EINVAL, "batch exceeds 2^29 records");
+  if (ctx->pending + n > kMaxBatchRecords) return fail(ctx, ARB_EINVAL, "batch exceeds 2^30 records");
   if ((global_index != nullptr && ctx->any_nogidx) || (global_index == nullptr && ctx->any_gidx))
     return fail(ctx, ARB_EINVAL, "global_index must be given for every submit of a batch or for none");
   cudaSetDevice(ctx->cfg.device);
@@ -418,7 +418,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     CK(ctx->seg_first.ensure(ctx->n_buckets + 1), "alloc seg_first");
     CK(ctx->blk.ensure((ns + 4095) / 4096 * 256 + 4096), "alloc blk");
     int cb = 1;
-    while (cb < kSegChunkBits && ((uint64_t)n_chunks >> cb)) ++cb;
+    while (cb < 22 && ((uint64_t)n_chunks >> cb)) ++cb;
     CK(launch_sort_segments(ctx->seg_a.p, ctx->seg_b.p, ns, cb, ctx->n_buckets, ctx->blk.p, ctx->seg_first.p,
                             ctx->segs.p, s, &launches), "sort segments");
   }

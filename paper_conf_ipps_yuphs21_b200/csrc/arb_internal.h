@@ -35,10 +35,10 @@ constexpr Sel kSelREL   = sel_make(0, 4, 2, 4);   // released CV: same bits as a
 
 // ---- compact event (partition output, 8 B) ---------------------------------
 // x: [0,30) word offset inside the address bucket | [30,32) access op (RH/WH/RT/WT)
-// y: record position inside the batch (< 2^29)
+// y: record position inside the batch (< 2^30)
 constexpr int kMaxBucketSpanBits = 30;               // buckets span <= 2^30 words
-constexpr uint32_t kMaxBatchRecords = 1u << 29;
-constexpr int kSegChunkBits = 21;                    // chunk ids of a batch fit 21 bits
+constexpr uint32_t kMaxBatchRecords = 1u << 30;
+constexpr int kSegChunkBits = 21;                    // chunk id bits in the entry key (bit 21 in y)
 
 // ---- partition geometry ----------------------------------------------------
 constexpr int kPartThreads = 512;
@@ -104,8 +104,8 @@ struct PartParams {
   uint32_t bucket_bits, n_buckets;
   uint32_t n_chunks;
   uint2* part_ev;                         // [n_chunks][kChunkCap]
-  uint2* seg_out; uint64_t seg_cap;       // {bucket << kSegChunkBits | chunk, start | len << 16} per
-                                          // touched bucket of a chunk
+  uint2* seg_out; uint64_t seg_cap;       // {bucket << 21 | chunk bits 0-20, start | len << 16 | chunk
+                                          // bit 21 << 31} per touched bucket of a chunk
   CtlRec* ctl; uint64_t ctl_cap;
   DevStats* st;
 };
@@ -153,7 +153,7 @@ cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits
                        uint32_t max_buckets, uint64_t* bucket_start, uint32_t* weight, uint32_t* first_bin,
                        uint32_t* nb_out, uint32_t* scratch, uint32_t* order, cudaStream_t s, int* launches);
 cudaError_t launch_partition(const PartParams& p, cudaStream_t s);
-// Sorts the 8-B segment entries {bucket << kSegChunkBits | chunk, start | len << 16}
+// Sorts the 8-B segment entries {bucket << 21 | chunk, start | len << 16 | chunk bit 21 << 31}
 // by (bucket, chunk) (a, b: ping-pong buffers), writes the replay form
 // {chunk, bucket, start | len << 16, exclusive event prefix} to out and each
 // bucket's first entry; cnt: (n / 4096 + 1) * 256 + 4096 u32

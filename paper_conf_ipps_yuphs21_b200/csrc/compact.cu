@@ -238,9 +238,13 @@ static int add_field_passes(RsPass* ps, int np, int field, int bits) {
   return np;
 }
 
-// Segment entries as written by k_partition (8 B): x = bucket << kSegChunkBits |
-// chunk, y = start | len << 16.  Sorted by x they are in (bucket, chunk) order.
+// Segment entries as written by k_partition (8 B): x = bucket << 21 | chunk bits
+// 0-20, y = start | len << 16 | chunk bit 21 << 31 (start, len <= 512).
 __device__ __forceinline__ uint32_t seg_bucket(uint2 e) { return e.x >> kSegChunkBits; }
+__device__ __forceinline__ uint32_t seg_len(uint2 e) { return (e.y >> 16) & 0x3FFu; }
+__device__ __forceinline__ uint32_t seg_chunk(uint2 e) {
+  return (e.x & ((1u << kSegChunkBits) - 1u)) | ((e.y >> 31) << kSegChunkBits);
+}
 
 // first entry of every bucket in the sorted entries
 __global__ void k_seg_first(const uint2* segs, uint64_t n, uint32_t n_buckets, uint32_t* first) {
@@ -258,7 +262,7 @@ __global__ void __launch_bounds__(kRsThreads) k_seg_tile_sum(const uint2* segs, 
   uint32_t c = 0;
 #pragma unroll
   for (int j = 0; j < kRsItems; ++j)
-    if (base + j < n) c += segs[base + j].y >> 16;
+    if (base + j < n) c += seg_len(segs[base + j]);
   for (int d = 16; d; d >>= 1) c += __shfl_xor_sync(FULL, c, d);
   if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = c;
   __syncthreads();
@@ -279,7 +283,7 @@ __global__ void __launch_bounds__(kRsThreads) k_seg_cum(const uint2* segs, uint6
 #pragma unroll
   for (int j = 0; j < kRsItems; ++j) {
     e[j] = base + j < n ? segs[base + j] : make_uint2(0, 0);
-    c += e[j].y >> 16;
+    c += seg_len(e[j]);
   }
   uint32_t incl = c;
   for (int d = 1; d < 32; d <<= 1) {
@@ -293,8 +297,8 @@ __global__ void __launch_bounds__(kRsThreads) k_seg_cum(const uint2* segs, uint6
 #pragma unroll
   for (int j = 0; j < kRsItems; ++j) {
     if (base + j < n)
-      out[base + j] = make_uint4(e[j].x & ((1u << kSegChunkBits) - 1u), seg_bucket(e[j]), e[j].y, run);
-    run += e[j].y >> 16;
+      out[base + j] = make_uint4(seg_chunk(e[j]), seg_bucket(e[j]), e[j].y & 0x3FFFFFFu, run);
+    run += seg_len(e[j]);
   }
 }
 
@@ -302,7 +306,9 @@ cudaError_t launch_sort_segments(uint2* a, uint2* b, uint64_t n, int chunk_bits,
                                  uint32_t* first, uint4* out, cudaStream_t s, int* launches) {
   RsPass ps[8];
   int np = 0;
-  for (int sh = 0; sh < chunk_bits; sh += 8) ps[np++] = RsPass{0, sh, chunk_bits - sh < 8 ? chunk_bits - sh : 8};
+  const int lo_bits = chunk_bits < kSegChunkBits ? chunk_bits : kSegChunkBits;
+  for (int sh = 0; sh < lo_bits; sh += 8) ps[np++] = RsPass{0, sh, lo_bits - sh < 8 ? lo_bits - sh : 8};
+  if (chunk_bits > kSegChunkBits) ps[np++] = RsPass{1, 31, 1};    // chunk bit 21 (batches > 2^29 records)
   for (int sh = kSegChunkBits; sh < 32; sh += 8) ps[np++] = RsPass{0, sh, 32 - sh < 8 ? 32 - sh : 8};
   cudaError_t e = cudaSuccess;
   if (n) e = radix_sort(a, b, n, ps, np, cnt, s, launches);

@@ -291,7 +291,8 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
       if (nbuf + n_new > kSegBuf) flush_segs();
       if (t < nT) {
         row[b] = (uint16_t)start;
-        segbuf[nbuf + lane] = make_uint2((b << kSegChunkBits) | (uint32_t)chunk, start | (len << 16));
+        segbuf[nbuf + lane] = make_uint2((b << kSegChunkBits) | ((uint32_t)chunk & ((1u << kSegChunkBits) - 1u)),
+                                         start | (len << 16) | (((uint32_t)chunk >> kSegChunkBits) << 31));
       }
       nbuf += n_new;
     }
