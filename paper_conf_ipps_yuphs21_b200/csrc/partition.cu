@@ -116,6 +116,39 @@ __device__ __forceinline__ void rank_round(uint32_t info, uint16_t* row, uint16_
   r1 = r0 + 1;
 }
 
+// The fast chunk test and its output.  One check per record: an access (op < 4)
+// of 1..8 bytes inside one 8-byte word (such an access cannot leave the
+// 48-bit space) whose word is tracked; then every word must map to the bucket of
+// record 0.  Returns false (nothing written) when any record fails.
+__device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p, uint32_t rec0, uint32_t chunk,
+                                           uint2* out, uint2* segbuf, uint32_t& nbuf, uint32_t lane) {
+  const uint32_t cb = p.coarse_bits, cmask = (1u << cb) - 1u;
+  uint32_t key[RPL], b0 = 0;
+  bool ok = true;
+#pragma unroll
+  for (int k = 0; k < RPL; ++k) {
+    const uint4 q = st[k * 32 + lane];
+    const uint32_t bad = (q.y & 0x00FC0000u) | (q.w & 0xFFFFu) | ((q.z - 1u) & ~7u) | (((q.x & 7u) + q.z - 1u) & ~7u);
+    const uint64_t word = ((uint64_t)((q.y & 0xFFFFu) >> 3) << 32) | __funnelshift_r(q.x, q.y, 3);
+    const uint64_t rel = word - p.base_word;
+    const bool okk = bad == 0 && rel < p.n_words;
+    const uint32_t m = okk ? __ldg(p.bin_map + (uint32_t)(rel >> cb)) : 0xFFFFFFFFu;
+    const uint32_t b = m & kBucketMask;
+    if (k == 0) b0 = b;
+    ok = ok && okk && b == b0;
+    key[k] = (((q.y >> 16) & 3u) << 30) | ((m >> kBucketBits) << cb) | ((uint32_t)rel & cmask);
+  }
+  const uint32_t bref = __shfl_sync(FULL, b0, 0);
+  if (!__all_sync(FULL, ok && b0 == bref)) return false;
+#pragma unroll
+  for (int k = 0; k < RPL; ++k) out[k * 32 + lane] = make_uint2(key[k], rec0 + k * 32 + lane);
+  if (lane == 0)
+    segbuf[nbuf] = make_uint2((bref << kSegChunkBits) | (chunk & ((1u << kSegChunkBits) - 1u)),
+                              (uint32_t)WREC << 16 | ((chunk >> kSegChunkBits) << 31));
+  ++nbuf;
+  return true;
+}
+
 __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   extern __shared__ __align__(16) uint8_t smem[];
   const uint32_t NB = p.n_buckets;
@@ -165,6 +198,18 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     const uint4* st = stage + cur * WREC;
     const uint64_t rec0 = chunk * WREC;
     const uint32_t nvalid = p.n - rec0 < (uint64_t)WREC ? (uint32_t)(p.n - rec0) : (uint32_t)WREC;
+    // ---- fast chunk: 256 single-word tracked accesses of one bucket ----------------------
+    // (the common case of real access streams: a run over one array).  The events
+    // keep record order, so event j is record j: one coalesced store per record and
+    // one segment entry for the chunk.  Anything else takes the general path below.
+    if (nbuf == kSegBuf) flush_segs();
+    if (nvalid == WREC && fast_chunk(st, p, (uint32_t)rec0, (uint32_t)chunk, p.part_ev + chunk * kChunkCap,
+                                     segbuf, nbuf, lane)) {
+      n_acc += RPL;
+      cur ^= 1;
+      __syncwarp();                    // stage[cur] reads done before the next fetch overwrites it
+      continue;
+    }
     uint32_t nT = 0, e_lane = 0;
     // ---- pass A: decode + rank, 2 groups of 4 x 32 records ----------------------------
     Dec dec[RPL];

@@ -37,7 +37,7 @@ struct ReplaySmem {
   uint2 ev[2][STEP];              // double-buffered step events {key, pos} (cp.async)
   union {
     struct { uint32_t keyA[STEP], posA[STEP], keyB[STEP], posB[STEP]; uint16_t hist[RT / 32][256]; } s;
-    struct { uint32_t key[kHSlots], wpos[kHSlots]; } h;      // fast step: written words only
+    struct { uint2 slot[kHSlots]; } h;      // fast step: written words {word, pos << 2 | op}
   } u;
   uint32_t wstart[kWin];          // staged segment list window: global event index
   uint32_t wcum[kWin + 1];        //   and bucket-relative first event of each segment
@@ -171,8 +171,24 @@ __device__ __forceinline__ uint32_t classify(uint32_t op, uint32_t before) {
 }
 
 __device__ __forceinline__ void hash_clear(ReplaySmem& S) {
-  for (uint32_t i = threadIdx.x; i < kHSlots; i += RT) { S.u.h.key[i] = kEmpty; S.u.h.wpos[i] = kEmpty; }
+  for (uint32_t i = threadIdx.x; i < kHSlots; i += RT) S.u.h.slot[i] = make_uint2(kEmpty, kEmpty);
 }
+
+// VSM write by access op (WH = 1, WT = 3) on a 4-bit state, branch-free
+__device__ __forceinline__ uint32_t vsm_write_op(uint32_t op, uint32_t s) {
+  return op == OP_WH ? ((s & kCVi) | kOVv | kOVi) : ((s & kOVi) | kCVv | kCVi);
+}
+// fault kind of an access with state-before `before`: a read
+// (RH = 0, RT = 2) whose side (bit op/2) is not valid: UUM (1) if that side was
+// never initialised, else USD (2); 0 for writes and valid reads
+__device__ __forceinline__ uint32_t classify_bits(uint32_t op, uint32_t before) {
+  const uint32_t v = before >> (op >> 1);
+  return (op & 1u) || (v & 1u) || op > 3 ? 0u : 1u + ((v >> 2) & 1u);
+}
+
+// hash slot of a word (Fibonacci hashing: consecutive words land far apart, so
+// the linear probe chains of a run's words stay short)
+__device__ __forceinline__ uint32_t hslot(uint32_t w) { return (w * 2654435761u) >> 20; }
 
 // ---- fast step: at most one write per word -------------------------------------------
 // Returns false (and leaves the shadow untouched) if some word has two writes.
@@ -181,68 +197,76 @@ __device__ __forceinline__ void hash_clear(ReplaySmem& S) {
 // not change the state, so a read's state-before is the state loaded
 // at the start of the step, or — if its word's single write precedes it — the
 // image of that write; the write event itself commits the word's final state.
-__device__ bool step_fast(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
+__device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
   uint32_t slot[RI], word[RI], pos[RI], op[RI], s_pre[RI];
   bool multi = false;
-  const uint64_t bb = S.bucket_base;
+  const uint8_t* sh = p.shadow + S.bucket_base;
+  uint2* hs = S.u.h.slot;
 #pragma unroll
   for (int j = 0; j < RI; ++j) {   // shadow loads first: their latency overlaps the hashing
     const uint32_t i = threadIdx.x + j * RT;
-    slot[j] = 0; word[j] = 0; pos[j] = 0; op[j] = 0xFFu; s_pre[j] = 0;
+    slot[j] = 0; word[j] = 0; pos[j] = 0; op[j] = 4; s_pre[j] = 0;
     if (i < m) {
       const uint2 e = ev[i];
       word[j] = e.x & kWordMask; op[j] = e.x >> 30; pos[j] = e.y;
-      s_pre[j] = __ldcg(p.shadow + bb + word[j]);
+      s_pre[j] = __ldcg(sh + word[j]);
     }
   }
+  // writes (WH = 1, WT = 3: odd ops) enter the table: slot {word, pos << 2 | op}
+  bool any_w = false;
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
-    if (op[j] == OP_WH || op[j] == OP_WT) {
-      uint32_t h = (word[j] * 2654435761u) >> 20;          // 12 bits
+    if (op[j] & 1u) {
+      any_w = true;
+      uint32_t h = hslot(word[j]);
       for (;;) {
-        const uint32_t old = atomicCAS(&S.u.h.key[h], kEmpty, word[j]);
+        const uint32_t old = atomicCAS(&hs[h].x, kEmpty, word[j]);
         if (old == kEmpty) break;
         if (old == word[j]) { multi = true; break; }        // a second write of the word
         h = (h + 1) & (kHSlots - 1);
       }
       slot[j] = h;
-      S.u.h.wpos[h] = (pos[j] << 2) | (op[j] == OP_WH ? 1u : 2u);
+      hs[h].y = (pos[j] << 2) | op[j];
     }
   }
-  if (__syncthreads_or(multi)) {
+  any_w = __syncthreads_or(any_w);
+  if (any_w && __syncthreads_or(multi)) {
 #pragma unroll
     for (int j = 0; j < RI; ++j)
-      if (op[j] == OP_WH || op[j] == OP_WT) { S.u.h.key[slot[j]] = kEmpty; S.u.h.wpos[slot[j]] = kEmpty; }
+      if (op[j] & 1u) hs[slot[j]] = make_uint2(kEmpty, kEmpty);
     __syncthreads();
     return false;
   }
   uint32_t fk[RI];
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
-    fk[j] = 0;
     const uint32_t s0 = s_pre[j] & 15u;
+    uint32_t before = s0;
     if (op[j] == OP_RH || op[j] == OP_RT) {
-      uint32_t h = (word[j] * 2654435761u) >> 20, before = s0;
-      for (;;) {                                            // probe for the word's write
-        const uint32_t k = S.u.h.key[h];
-        if (k == kEmpty) break;
-        if (k == word[j]) {
-          const uint32_t wp = S.u.h.wpos[h];
-          if ((wp >> 2) < pos[j]) before = vsm_write(wp & 3u, s0);
-          break;
+      if (any_w) {
+        uint32_t h = hslot(word[j]);
+        for (;;) {                                          // probe for the word's write
+          const uint2 k = hs[h];
+          if (k.x == word[j]) {
+            if ((k.y >> 2) < pos[j]) before = vsm_write_op(k.y & 3u, s0);
+            break;
+          }
+          if (k.x == kEmpty) break;
+          h = (h + 1) & (kHSlots - 1);
         }
-        h = (h + 1) & (kHSlots - 1);
       }
-      fk[j] = classify(op[j], before);
-    } else if (op[j] != 0xFFu) {
-      __stcg(p.shadow + bb + word[j], (uint8_t)vsm_write(op[j] == OP_WH ? 1u : 2u, s0));
+    } else if (op[j] & 1u) {
+      __stcg(const_cast<uint8_t*>(sh) + word[j], (uint8_t)vsm_write_op(op[j], s0));
     }
+    fk[j] = classify_bits(op[j], before);
   }
-  emit_faults(p, fk, word, pos, bb);
-  __syncthreads();
+  emit_faults(p, fk, word, pos, S.bucket_base);
+  if (any_w) {
+    __syncthreads();
 #pragma unroll
-  for (int j = 0; j < RI; ++j)
-    if (op[j] == OP_WH || op[j] == OP_WT) { S.u.h.key[slot[j]] = kEmpty; S.u.h.wpos[slot[j]] = kEmpty; }
+    for (int j = 0; j < RI; ++j)
+      if (op[j] & 1u) hs[slot[j]] = make_uint2(kEmpty, kEmpty);
+  }
   // the caller's next barrier orders this reset before the next step's inserts
   return true;
 }
@@ -470,37 +494,66 @@ __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t 
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t nwin = S.nwin;
   const uint32_t m = min(min((uint32_t)STEP, total - e0), S.wcum[nwin] - e0);
-  // window segments [a0, a1) hold the events; every warp searches (no barrier):
-  // segment j holds e iff wcum[j] <= e < wcum[j+1]
+  // Warp w gathers the slice [e0 + 32*RI*w, +32*RI) of the step.  Segment j holds
+  // event e iff wcum[j] <= e < wcum[j+1]; every warp counts, from the hint, the
+  // segments starting at or before its slice start and before the step's last
+  // event (ballots, no barrier), then each lane walks forward to the segment of
+  // each of its events (segments are usually longer than the slice).
+  const uint32_t s0 = e0 + warp * (32 * RI), last = e0 + m - 1;
   const uint32_t base0 = hint & ~31u;
   uint32_t c0 = 0, c1 = 0;
   for (uint32_t base = base0; base < nwin; base += 32) {
     const uint32_t j = base + lane;
-    const bool le0 = j < nwin && S.wcum[j] <= e0;
-    const bool lt1 = j < nwin && S.wcum[j] < e0 + m;
-    c0 += __popc(__ballot_sync(FULL, le0));
-    c1 += __popc(__ballot_sync(FULL, lt1));
-    if (!__any_sync(FULL, lt1)) break;
+    const uint32_t w = j < nwin ? S.wcum[j] : 0xFFFFFFFFu;
+    c0 += __popc(__ballot_sync(FULL, w <= s0));
+    const uint32_t b1 = __ballot_sync(FULL, w <= last);
+    c1 += __popc(b1);
+    if (b1 != FULL) break;
   }
-  const uint32_t a0 = base0 + c0 - 1, a1 = base0 + c1;
-  hint = a1 - 1;
-  if ((a1 - a0) * 16 <= m) {
-    // long segments: one warp streams one segment at a time
-    for (uint32_t j = a0 + warp; j < a1; j += RT / 32) {
-      const uint32_t lo = max(S.wcum[j], e0), hi = min(S.wcum[j + 1], e0 + m);
-      const uint2* src = p.part_ev + (uint64_t)S.wstart[j] + (lo - S.wcum[j]);
-      uint2* d = dst + (lo - e0);
-      for (uint32_t k = lane; k < hi - lo; k += 32) cp_async8(d + k, src + k);
+  hint = base0 + c1 - 1;                 // segment of the step's last event
+  if (s0 < e0 + m) {
+    uint32_t seg = base0 + c0 - 1, seg_end = S.wcum[seg + 1];
+    // event e of segment seg sits at part_ev[wstart[seg] + e - wcum[seg]] = bp[e]
+    int64_t bp = (int64_t)S.wstart[seg] - (int64_t)S.wcum[seg];
+    const uint32_t s_end = min(s0 + 32 * RI, e0 + m);
+    if (s_end <= seg_end) {
+      // the whole slice lies in one segment (warp-uniform; the common case):
+      // a contiguous copy, 16 B per lane when both sides are 16-B aligned
+      const uint2* src = p.part_ev + (bp + s0);
+      uint2* d = dst + (s0 - e0);
+      const uint32_t cnt = s_end - s0;
+      if (cnt == 32 * RI && ((reinterpret_cast<uintptr_t>(src) & 15u) == 0)) {
+#pragma unroll
+        for (int k = 0; k < RI / 2; ++k) cp_async16(d + 2 * (lane + 32 * k), src + 2 * (lane + 32 * k));
+      } else {
+#pragma unroll
+        for (int k = 0; k < RI; ++k)
+          if (lane + 32 * k < cnt) cp_async8(d + lane + 32 * k, src + lane + 32 * k);
+      }
+      cp_async_commit();
+      return m;
     }
-  } else {
-    // short segments: every thread locates the segments of its events
+    uint2* d = dst + (s0 - e0) + lane;
+    if (seg + 2 <= nwin && s_end <= S.wcum[seg + 2]) {
+      // two segments: select the base per event
+      const int64_t bp1 = (int64_t)S.wstart[seg + 1] - (int64_t)seg_end;
+#pragma unroll
+      for (int k = 0; k < RI; ++k) {
+        const uint32_t e = s0 + k * 32 + lane;
+        if (e < s_end) cp_async8(d + k * 32, p.part_ev + ((e < seg_end ? bp : bp1) + e));
+      }
+      cp_async_commit();
+      return m;
+    }
 #pragma unroll
     for (int k = 0; k < RI; ++k) {
-      const uint32_t e = e0 + threadIdx.x + k * RT;
+      const uint32_t e = s0 + k * 32 + lane;
       if (e < e0 + m) {
-        uint32_t a = a0, z = a1;
-        while (z - a > 1) { const uint32_t mid = (a + z) >> 1; if (S.wcum[mid] <= e) a = mid; else z = mid; }
-        cp_async8(dst + (e - e0), p.part_ev + (uint64_t)S.wstart[a] + (e - S.wcum[a]));
+        if (e >= seg_end) {
+          do { ++seg; seg_end = S.wcum[seg + 1]; } while (e >= seg_end);
+          bp = (int64_t)S.wstart[seg] - (int64_t)S.wcum[seg];
+        }
+        cp_async8(d + k * 32, p.part_ev + (bp + e));
       }
     }
   }

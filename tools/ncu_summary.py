@@ -79,14 +79,14 @@ def to_num(s):
 
 def main():
     tag, name = sys.argv[1], sys.argv[2]
-    prof = os.path.join(ROOT, "profiles")
-    lib = [(k, ms) for k, ms in launches(os.path.join(tag, "launches.csv"))
-           if k.startswith("arb::")]
+    prof = os.environ.get("OUTDIR", os.path.join(ROOT, "profiles"))
+    lpath = os.path.join(tag, "launches.csv")
+    lib = [(k, ms) for k, ms in launches(lpath) if k.startswith("arb::")] if os.path.exists(lpath) else []
     agg = defaultdict(lambda: [0, 0.0])
     for k, ms in lib:
         agg[k][0] += 1
         agg[k][1] += ms
-    tot = sum(v[1] for v in agg.values())
+    tot = sum(v[1] for v in agg.values()) or 1.0
     lines = [f"# {name} — launch list of one bench step (config 5, rank 0)", "",
              "`ncu --metrics gpu__time_duration.sum --clock-control none` over "
              "`python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu` (cold-cache, serialised; "
