@@ -269,13 +269,15 @@ def main():
     def one_step(collect=False):
         st_acc = {"access_words": 0, "range_words": 0, "reports": 0, "launches": 0, "ms_partition": 0.0,
                   "ms_replay": 0.0, "ms_mir": 0.0, "ms_reports": 0.0, "ms_control": 0.0, "ms_total": 0.0,
-                  "ms_sample": 0.0, "records": 0, "by_kind": [0, 0, 0, 0]}
+                  "ms_sample": 0.0, "ms_segsort": 0.0, "ms_host_control": 0.0, "records": 0,
+                  "by_kind": [0, 0, 0, 0]}
         for (a, b) in flushes:
             ctx.submit_events(recs[a:b], global_index=gidx[a:b], stream=stream)
             rc, n, off = ctx.flush(stream=stream)
             st = ctx.stats()
             for k in ("access_words", "range_words", "reports", "records", "ms_partition", "ms_replay",
-                      "ms_mir", "ms_reports", "ms_control", "ms_total", "ms_sample"):
+                      "ms_mir", "ms_reports", "ms_control", "ms_total", "ms_sample", "ms_segsort",
+                      "ms_host_control"):
                 st_acc[k] += st[k]
             st_acc["launches"] += st["kernel_launches"]
             for k in range(4):
@@ -324,7 +326,9 @@ def main():
     step_ms_lib = s0["ms_total"]
     phases = {"k_sample+balance": s0["ms_sample"], "k_partition": s0["ms_partition"] - s0["ms_sample"],
               "k_replay": s0["ms_replay"], "k_mir": s0["ms_mir"],
-              "report_compaction": s0["ms_reports"], "control_plane": s0["ms_control"]}
+              "report_compaction": s0["ms_reports"], "control_plane": s0["ms_control"],
+              "segment_sort (in control_plane)": s0["ms_segsort"],
+              "host_control_wall (in control_plane)": s0["ms_host_control"]}
     dom = max(("k_partition", "k_replay"), key=lambda k: phases[k])
     # algorithmic bytes of each kernel: the partition kernel reads every
     # record once (16 R); the replay owns the shadow term (2 W) and the report writes (16 Rep)

@@ -112,6 +112,8 @@ typedef struct {
   uint64_t kernel_launches;  /* kernels launched by the last flush                         */
   double   ms_sample;        /* address sampling + bucket balancing (inside ms_partition)  */
   uint64_t steps_fast, steps_sort;  /* replay steps by kind                  */
+  double   ms_segsort;       /* GPU: segment-entry sort (inside ms_control)                 */
+  double   ms_host_control;  /* host wall time of the Table I / task resolution             */
 } arb_stats;
 
 typedef struct arb_ctx_s* arb_ctx;

@@ -5,6 +5,7 @@
 
 #include <dlfcn.h>
 #include <algorithm>
+#include <chrono>
 #include <cstring>
 #include <new>
 #include <string>
@@ -132,7 +133,7 @@ struct arb_ctx_s {
   bool flushed = false;
   std::string err;
   arb_stats stats{};
-  cudaEvent_t ev[8] = {};
+  cudaEvent_t ev[10] = {};
   cudaStream_t aux = nullptr;                 // control-record copies beside the main stream
   HostBuf<DevStats> h_stats;
   HostBuf<uint32_t> h_nb, h_ops_start;
@@ -204,7 +205,7 @@ extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
   if (e == cudaSuccess) e = ctx->dstats.ensure(1);
   if (e == cudaSuccess) e = ctx->dcount.ensure(4);
   if (e == cudaSuccess) e = ctx->ctl.ensure(ctx->ctl_cap);
-  for (int i = 0; i < 8 && e == cudaSuccess; ++i) e = cudaEventCreate(&ctx->ev[i]);
+  for (int i = 0; i < 10 && e == cudaSuccess; ++i) e = cudaEventCreate(&ctx->ev[i]);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->aux, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = ctx->h_stats.ensure(1);
   if (e == cudaSuccess) e = ctx->h_nb.ensure(1);
@@ -307,6 +308,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   S.records = n; S.access_words = S.range_words = S.control_records = S.range_ops = S.tasks = 0;
   S.reports = 0; std::memset(S.reports_by_kind, 0, sizeof(S.reports_by_kind)); S.ignored_words = 0;
   S.ms_partition = S.ms_control = S.ms_replay = S.ms_mir = S.ms_reports = S.ms_total = 0;
+  S.ms_segsort = S.ms_host_control = 0;
   S.buckets = ctx->n_buckets; S.bucket_bits = ctx->bucket_bits; S.max_bucket_events = 0;
 
   // ---- resolve the batch into one device array ---------------------------
@@ -416,12 +418,14 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     CK(ctx->seg_b.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
     CK(ctx->segs.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
     CK(ctx->seg_first.ensure(ctx->n_buckets + 1), "alloc seg_first");
-    CK(ctx->blk.ensure((ns + 4095) / 4096 * 256 + 4096), "alloc blk");
+    CK(ctx->blk.ensure((ns + 4095) / 4096 * 2049 + 4096), "alloc blk");   // 2048-bin digit counters + scan scratch
     int cb = 1;
     while (cb < 22 && ((uint64_t)n_chunks >> cb)) ++cb;
     CK(launch_sort_segments(ctx->seg_a.p, ctx->seg_b.p, ns, cb, ctx->n_buckets, ctx->blk.p, ctx->seg_first.p,
                             ctx->segs.p, s, &launches), "sort segments");
+    if (timing) cudaEventRecord(ctx->ev[8], s);
   }
+  const auto t_host0 = std::chrono::steady_clock::now();
 
   // ---- A2: control resolution on the host -------------------------------------
   std::vector<CtlRec> ctl(hst.n_ctl);
@@ -441,6 +445,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     reset_batch(ctx);
     return fail(ctx, plan.rc, plan.err + " (batch position " + std::to_string(plan.err_pos) + ")");
   }
+  S.ms_host_control = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_host0).count();
   S.range_words = plan.range_words;
   S.range_ops = plan.range_ops.size();
   S.tasks = plan.tasks;
@@ -521,7 +526,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   CK(ctx->cand_tmp.ensure(std::max<uint64_t>(n_cand, 1)), "alloc cand tmp");
   CK(ctx->reports.ensure(std::max<uint64_t>(n_cand, 1)), "alloc reports");
   uint64_t nblk = (n_cand + 4095) / 4096;
-  CK(ctx->blk.ensure(nblk * 256 + 4096), "alloc blk");
+  CK(ctx->blk.ensure(nblk * 2049 + 4096), "alloc blk");
   CompactParams cp{};
   cp.cand = ctx->cand.p; cp.n_cand = n_cand; cp.tmp = ctx->cand_tmp.p; cp.blk = ctx->blk.p;
   cp.blk_cap = ctx->blk.cap; cp.base_word = ctx->base_word;
@@ -564,6 +569,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     cudaEventElapsedTime(&ms, ctx->ev[0], ctx->ev[1]); S.ms_partition = ms;
     cudaEventElapsedTime(&ms, ctx->ev[0], ctx->ev[7]); S.ms_sample = ms;
     cudaEventElapsedTime(&ms, ctx->ev[1], ctx->ev[2]); S.ms_control = ms;
+    cudaEventElapsedTime(&ms, ctx->ev[1], ctx->ev[8]); S.ms_segsort = ms;
     cudaEventElapsedTime(&ms, ctx->ev[2], ctx->ev[3]); S.ms_replay = ms;
     cudaEventElapsedTime(&ms, ctx->ev[3], ctx->ev[4]); S.ms_mir = ms;
     cudaEventElapsedTime(&ms, ctx->ev[4], ctx->ev[5]); S.ms_reports = ms;

@@ -7,8 +7,12 @@ namespace arb {
 constexpr int kRsThreads = 512, kRsItems = 8, kRsTile = kRsThreads * kRsItems;
 
 struct RsPass { int field; int shift; int bits; };
-// digit fields: uint4 {0: w, 1: z, 2: x, 3: y}; uint2 {0: x, 1: y}
-__device__ __forceinline__ uint32_t rs_field(uint4 c, int f) { return f == 0 ? c.w : f == 1 ? c.z : f == 2 ? c.x : c.y; }
+constexpr int kRsMaxBits = 11;                    // digits of up to 11 bits (2048 bins)
+constexpr int kRsBins = 1 << kRsMaxBits;
+// digit fields: uint4 {0: w, 1: z, 2: x, 3: y, 4: z << 2 | w}; uint2 {0: x, 1: y}
+__device__ __forceinline__ uint32_t rs_field(uint4 c, int f) {
+  return f == 0 ? c.w : f == 1 ? c.z : f == 2 ? c.x : f == 3 ? c.y : (c.z << 2) | c.w;
+}
 __device__ __forceinline__ uint32_t rs_field(uint2 c, int f) { return f == 0 ? c.x : c.y; }
 template <class E>
 __device__ __forceinline__ uint32_t rs_digit(E c, RsPass ps) {
@@ -18,8 +22,9 @@ __device__ __forceinline__ uint32_t rs_digit(E c, RsPass ps) {
 template <class E>
 __global__ void __launch_bounds__(kRsThreads) k_rs_hist(const E* in, uint64_t n, RsPass ps, uint32_t* cnt,
                                                         uint32_t nblk) {
-  __shared__ uint32_t h[256];
-  for (int i = threadIdx.x; i < 256; i += kRsThreads) h[i] = 0;
+  __shared__ uint32_t h[kRsBins];
+  const int nd = 1 << ps.bits;
+  for (int i = threadIdx.x; i < nd; i += kRsThreads) h[i] = 0;
   __syncthreads();
   uint64_t base = (uint64_t)blockIdx.x * kRsTile;
   for (int j = 0; j < kRsItems; ++j) {
@@ -27,7 +32,7 @@ __global__ void __launch_bounds__(kRsThreads) k_rs_hist(const E* in, uint64_t n,
     if (i < n) atomicAdd(&h[rs_digit(in[i], ps)], 1u);
   }
   __syncthreads();
-  for (int d = threadIdx.x; d < 256; d += kRsThreads) cnt[(uint64_t)d * nblk + blockIdx.x] = h[d];
+  for (int d = threadIdx.x; d < nd; d += kRsThreads) cnt[(uint64_t)d * nblk + blockIdx.x] = h[d];
 }
 
 // ---- exclusive scan of u32 values in place ------------------------------------------
@@ -105,15 +110,19 @@ static void scan_u32(uint32_t* a, uint64_t n, uint32_t* scratch, cudaStream_t s,
   *launches += 3;
 }
 
+// dynamic shared memory: hist[kRsThreads / 32][2^bits] u16 + dbase[2^bits] u32
 template <class E>
 __global__ void __launch_bounds__(kRsThreads) k_rs_scatter(const E* in, E* out, uint64_t n, RsPass ps,
                                                            const uint32_t* cnt, uint32_t nblk) {
-  __shared__ uint16_t hist[kRsThreads / 32][256];
-  __shared__ uint32_t dbase[256];
+  extern __shared__ __align__(16) uint8_t rs_smem[];
+  const int nd = 1 << ps.bits;
+  uint16_t* hist = reinterpret_cast<uint16_t*>(rs_smem);                     // [warp][nd]
+  uint32_t* dbase = reinterpret_cast<uint32_t*>(rs_smem + (kRsThreads / 32) * nd * 2);
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  uint32_t* h32 = reinterpret_cast<uint32_t*>(&hist[0][0]);
-  for (uint32_t i = tid; i < (kRsThreads / 32) * 128; i += kRsThreads) h32[i] = 0;
+  uint32_t* h32 = reinterpret_cast<uint32_t*>(hist);
+  for (uint32_t i = tid; i < (uint32_t)((kRsThreads / 32) * nd / 2); i += kRsThreads) h32[i] = 0;
   __syncthreads();
+  uint16_t* row = hist + warp * nd;
   uint64_t base = (uint64_t)blockIdx.x * kRsTile;
   E c[kRsItems]; uint32_t rk[kRsItems], dg[kRsItems];
   const uint32_t lt = lanemask_lt();
@@ -123,22 +132,22 @@ __global__ void __launch_bounds__(kRsThreads) k_rs_scatter(const E* in, E* out, 
     if (valid) c[r] = in[i];
     uint32_t d = valid ? rs_digit(c[r], ps) : 0xFFFFu;
     uint32_t grp = __match_any_sync(FULL, d);
-    uint32_t b = valid ? hist[warp][d] : 0;
+    uint32_t b = valid ? row[d] : 0;
     __syncwarp();
-    if (valid && lane == 31u - __clz(grp)) hist[warp][d] = (uint16_t)(b + __popc(grp));
+    if (valid && lane == 31u - __clz(grp)) row[d] = (uint16_t)(b + __popc(grp));
     __syncwarp();
     dg[r] = d; rk[r] = b + __popc(grp & lt);
   }
   __syncthreads();
-  if (tid < 256) {
+  for (int d = tid; d < nd; d += kRsThreads) {
     uint32_t s = 0;
-    for (int w = 0; w < kRsThreads / 32; ++w) { uint32_t x = hist[w][tid]; hist[w][tid] = (uint16_t)s; s += x; }
-    dbase[tid] = cnt[(uint64_t)tid * nblk + blockIdx.x];
+    for (int w = 0; w < kRsThreads / 32; ++w) { uint32_t x = hist[w * nd + d]; hist[w * nd + d] = (uint16_t)s; s += x; }
+    dbase[d] = cnt[(uint64_t)d * nblk + blockIdx.x];
   }
   __syncthreads();
   for (int r = 0; r < kRsItems; ++r) {
     uint64_t i = base + warp * (32 * kRsItems) + r * 32 + lane;
-    if (i < n) out[dbase[dg[r]] + hist[warp][dg[r]] + rk[r]] = c[r];
+    if (i < n) out[dbase[dg[r]] + row[dg[r]] + rk[r]] = c[r];
   }
 }
 
@@ -223,18 +232,30 @@ template <class E>
 static cudaError_t radix_sort(E*& a, E*& b, uint64_t n, const RsPass* passes, int np, uint32_t* cnt,
                               cudaStream_t s, int* launches) {
   uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
+  const size_t smem_max = (kRsThreads / 32) * kRsBins * 2 + kRsBins * 4;
+  cudaError_t e = cudaFuncSetAttribute(k_rs_scatter<E>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_max);
+  if (e != cudaSuccess) return e;
   for (int k = 0; k < np; ++k) {
+    const uint64_t nd = 1ull << passes[k].bits;
     k_rs_hist<E><<<nblk, kRsThreads, 0, s>>>(a, n, passes[k], cnt, nblk);
-    scan_u32(cnt, (uint64_t)nblk * 256, cnt + (uint64_t)nblk * 256, s, launches);
-    k_rs_scatter<E><<<nblk, kRsThreads, 0, s>>>(a, b, n, passes[k], cnt, nblk);
+    scan_u32(cnt, (uint64_t)nblk * nd, cnt + (uint64_t)nblk * nd, s, launches);
+    k_rs_scatter<E><<<nblk, kRsThreads, (kRsThreads / 32) * nd * 2 + nd * 4, s>>>(a, b, n, passes[k], cnt, nblk);
     *launches += 2;
     E* t = a; a = b; b = t;
   }
   return cudaGetLastError();
 }
 
+// LSD passes over `bits` bits of a field, in near-equal digits of <= 11 bits
 static int add_field_passes(RsPass* ps, int np, int field, int bits) {
-  for (int sh = 0; sh < bits; sh += 8) ps[np++] = RsPass{field, sh, bits - sh < 8 ? bits - sh : 8};
+  if (bits <= 0) return np;
+  const int k = (bits + kRsMaxBits - 1) / kRsMaxBits;
+  int sh = 0;
+  for (int j = 0; j < k; ++j) {
+    const int w = (bits - sh + (k - j) - 1) / (k - j);
+    ps[np++] = RsPass{field, sh, w};
+    sh += w;
+  }
   return np;
 }
 
@@ -307,9 +328,13 @@ cudaError_t launch_sort_segments(uint2* a, uint2* b, uint64_t n, int chunk_bits,
   RsPass ps[8];
   int np = 0;
   const int lo_bits = chunk_bits < kSegChunkBits ? chunk_bits : kSegChunkBits;
-  for (int sh = 0; sh < lo_bits; sh += 8) ps[np++] = RsPass{0, sh, lo_bits - sh < 8 ? lo_bits - sh : 8};
+  np = add_field_passes(ps, np, 0, lo_bits);
   if (chunk_bits > kSegChunkBits) ps[np++] = RsPass{1, 31, 1};    // chunk bit 21 (batches > 2^29 records)
-  for (int sh = kSegChunkBits; sh < 32; sh += 8) ps[np++] = RsPass{0, sh, 32 - sh < 8 ? 32 - sh : 8};
+  {
+    int nbb = 1;
+    while ((1u << nbb) < n_buckets) ++nbb;                      // bucket bits actually used
+    for (int sh = kSegChunkBits, k = 0; k < 1; ++k) ps[np++] = RsPass{0, sh, nbb};
+  }
   cudaError_t e = cudaSuccess;
   if (n) e = radix_sort(a, b, n, ps, np, cnt, s, launches);
   if (e != cudaSuccess) return e;
@@ -355,8 +380,12 @@ cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches
     uint4* t = a; a = b; b = t;
     np = 0;
   }
-  np = add_field_passes(ps, np, 0, 2);
-  np = add_field_passes(ps, np, 1, p.pos_bits);
+  if (p.pos_bits <= 30) {
+    np = add_field_passes(ps, np, 4, p.pos_bits + 2);         // record, then kind
+  } else {
+    np = add_field_passes(ps, np, 0, 2);
+    np = add_field_passes(ps, np, 1, p.pos_bits);
+  }
   np = add_field_passes(ps, np, 2, wb_lo);
   np = add_field_passes(ps, np, 3, wb_hi);
   if ((e = radix_sort<uint4>(a, b, n, ps, np, p.blk, s, launches)) != cudaSuccess) return e;

@@ -147,7 +147,7 @@ __global__ void __launch_bounds__(kT) k_cut_write(CutArgs a) {
 }
 
 __global__ void k_cut_map(CutArgs a) {
-  const uint32_t nb = *a.nb_out, total = a.misc[0];
+  const uint32_t nb = *a.nb_out;
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < a.n_bins; i += gridDim.x * blockDim.x) {
     const uint32_t b = a.bucket_of[i];
     a.hist_map[i] = b | ((i - a.first_bin[b]) << kBucketBits);
@@ -174,19 +174,21 @@ __global__ void k_cut_weights(CutArgs a) {   // one CTA: prefix differences
   }
 }
 
-// one CTA: replay scheduling order = buckets by weight, heaviest first (stable:
-// rank = #heavier + #equal with a smaller id)
-__global__ void __launch_bounds__(1024) k_cut_order(CutArgs a, uint32_t* order) {
+// replay scheduling order = buckets by weight, heaviest first (stable: rank =
+// #heavier + #equal with a smaller id); CTA c ranks buckets [256c, 256c + 256)
+constexpr int kOrderT = 256;
+__global__ void __launch_bounds__(kOrderT) k_cut_order(CutArgs a, uint32_t* order) {
   __shared__ uint32_t w[kMaxBuckets];
   const uint32_t nb = *a.nb_out;
+  if (blockIdx.x * kOrderT >= nb) return;
   for (uint32_t b = threadIdx.x; b < nb; b += blockDim.x) w[b] = a.weight[b];
   __syncthreads();
-  for (uint32_t b = threadIdx.x; b < nb; b += blockDim.x) {
-    const uint32_t x = w[b];
-    uint32_t r = 0;
-    for (uint32_t c = 0; c < nb; ++c) r += (w[c] > x) | ((w[c] == x) & (c < b));
-    order[r] = b;
-  }
+  const uint32_t b = blockIdx.x * kOrderT + threadIdx.x;
+  if (b >= nb) return;
+  const uint32_t x = w[b];
+  uint32_t r = 0;
+  for (uint32_t c = 0; c < nb; ++c) r += (w[c] > x) | ((w[c] == x) & (c < b));
+  order[r] = b;
 }
 
 cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits, uint64_t n_words,
@@ -202,7 +204,7 @@ cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits
   k_cut_write<<<nt, kT, 0, s>>>(a);
   k_cut_map<<<148, 1024, 0, s>>>(a);
   k_cut_weights<<<1, kT, 0, s>>>(a);
-  k_cut_order<<<1, kT, 0, s>>>(a, order);
+  k_cut_order<<<kMaxBuckets / kOrderT, kOrderT, 0, s>>>(a, order);
   *launches += 8;
   return cudaGetLastError();
 }

@@ -11,3 +11,6 @@ if [ -n "$NCU" ]; then
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:"$NCU" -c 2 -o $OUT/full python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu > $OUT/ncu_full.log 2>&1
   tail -n 2 $OUT/ncu_full.log
 fi
+if [ -n "$LAUNCHES" ]; then
+  timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu > $OUT/ncu_launch.log 2>&1
+fi
