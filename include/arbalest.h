@@ -77,6 +77,9 @@ enum arb_status {
 /* ---- configuration ------------------------------------------------------------- */
 #define ARB_F_DEDUP_FIRST 0x1u  /* keep only the first report per (word, kind) (Z3)      */
 #define ARB_F_TIMING      0x2u  /* record CUDA events around every kernel (arb_get_stats) */
+#define ARB_F_SMALL_PARTS 0x4u  /* test knob: split every bucket with >= 2048 range-op words
+                                   into word-range parts replayed by separate CTAs (the
+                                   mechanism normally used for range-heavy buckets only)  */
 
 typedef struct {
   uint64_t addr_base;        /* tracked OV byte range [addr_base, addr_base+addr_bytes);   */

@@ -95,9 +95,13 @@ struct arb_ctx_s {
   arb_config cfg{};
   uint64_t base_word = 0, n_words = 0;
   uint32_t bucket_bits = 0, n_buckets = 0, coarse_bits = 0, n_bins = 0;
-  std::vector<uint32_t> bin_map, order, hist;
+  std::vector<uint32_t> bin_map, hist;
   std::vector<uint64_t> bucket_start;
-  DevBuf<uint32_t> d_bin_map, d_order, d_hist, d_cut, d_cutscr;
+  std::vector<uint4> items;                   // replay work items (see build_items)
+  DevBuf<uint4> d_items;
+  HostBuf<uint4> h_items;
+  HostBuf<uint32_t> h_weight;
+  DevBuf<uint32_t> d_bin_map, d_hist, d_cut, d_cutscr;
   DevBuf<uint64_t> d_bucket_start;
   int n_sms = 148;
   uint8_t* shadow = nullptr;
@@ -186,8 +190,6 @@ extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
     ctx->bucket_start.clear();
     for (uint64_t b = 0; b < nb; ++b) { ctx->bin_map[b] = (uint32_t)b; ctx->bucket_start.push_back(b << bits); }
     ctx->bucket_start.push_back(ctx->n_words);
-    ctx->order.resize(nb);
-    for (uint64_t b = 0; b < nb; ++b) ctx->order[b] = (uint32_t)b;
   } else {
     uint32_t cb = 0;
     while (((ctx->n_words + (1ull << cb) - 1) >> cb) > (uint64_t)kMaxCoarseBins) ++cb;
@@ -210,6 +212,7 @@ extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
   if (e == cudaSuccess) e = ctx->h_stats.ensure(1);
   if (e == cudaSuccess) e = ctx->h_nb.ensure(1);
   if (e == cudaSuccess) e = ctx->h_bstart.ensure(kMaxBuckets + 1);
+  if (e == cudaSuccess) e = ctx->h_weight.ensure(kMaxBuckets);
   if (e == cudaSuccess) e = cudaDeviceSynchronize();
   if (e != cudaSuccess) { arb_destroy(ctx); return ARB_ENOMEM; }
   if (cfg->world > 1) {
@@ -241,7 +244,7 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   ctx->m_rr_cum.release(); ctx->m_ins_inst.release(); ctx->m_qry_open_start.release(); ctx->m_open_list.release();
   ctx->m_own_start.release(); ctx->m_win_start.release(); ctx->m_own.release(); ctx->m_win.release();
   ctx->m_rr.release(); ctx->hkeys.release(); ctx->hvals.release(); ctx->counts.release();
-  ctx->d_bin_map.release(); ctx->d_order.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_cut.release();
+  ctx->d_bin_map.release(); ctx->d_items.release(); ctx->h_items.release(); ctx->h_weight.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_cut.release();
   for (auto& e : ctx->ev) if (e) cudaEventDestroy(e);
   if (ctx->aux) cudaStreamDestroy(ctx->aux);
   ctx->h_stats.release(); ctx->h_nb.release(); ctx->h_ops_start.release(); ctx->h_bstart.release();
@@ -295,6 +298,45 @@ static void reset_batch(arb_ctx ctx) {
   ctx->subs.clear();
   ctx->pending = 0;
   ctx->any_gidx = ctx->any_nogidx = false;
+}
+
+// Replay work items, heaviest first.  A bucket whose range ops cover many words
+// compared with its events is split into parts (contiguous word ranges, 16-word
+// aligned): each part replays all of the bucket's events but acts only on its own
+// words, so the range-op streaming of one huge bucket spreads over many CTAs.
+// Cost model (per CTA): ~600 range-op words stream in the time of one event.
+static void build_items(arb_ctx ctx, const FlushPlan& plan, const std::vector<double>& bucket_events) {
+  constexpr double kWordsPerEvent = 600.0;
+  constexpr uint32_t kMaxParts = 64;
+  const bool small = ctx->cfg.flags & ARB_F_SMALL_PARTS;
+  const double kPartWords = small ? 1024.0 : double(1u << 24);
+  const uint32_t nb = ctx->n_buckets;
+  struct It { double cost; uint4 v; };
+  std::vector<It> its;
+  its.reserve(nb);
+  for (uint32_t b = 0; b < nb; ++b) {
+    double rw = 0;
+    for (uint32_t k = plan.ops_start[b]; k < plan.ops_start[b + 1]; ++k) rw += double(plan.ops[k].hi - plan.ops[k].lo);
+    const double ev = b < bucket_events.size() ? bucket_events[b] : 0.0;
+    const uint64_t span = ctx->bucket_start[b + 1] - ctx->bucket_start[b];
+    uint32_t np = 1;
+    if (rw > 2 * kPartWords && span >= 32) {
+      double by_range = rw / kPartWords, by_events = small ? by_range : rw / (ev * kWordsPerEvent + 1.0);
+      double x = std::min(by_range, by_events);
+      np = (uint32_t)std::max(1.0, std::min<double>(x, kMaxParts));
+      np = (uint32_t)std::min<uint64_t>(np, span / 16);
+    }
+    const uint64_t step = ((span + np - 1) / np + 15) & ~15ull;
+    for (uint32_t q = 0; q < np; ++q) {
+      const uint64_t lo = std::min<uint64_t>(span, q * step), hi = std::min<uint64_t>(span, lo + step);
+      if (lo >= hi && np > 1) continue;
+      const double cost = ev * kWordsPerEvent + rw * double(hi - lo) / double(std::max<uint64_t>(span, 1));
+      its.push_back(It{cost, make_uint4(b, (uint32_t)lo, (uint32_t)hi, np > 1 ? 1u : 0u)});
+    }
+  }
+  std::stable_sort(its.begin(), its.end(), [](const It& a, const It& b) { return a.cost > b.cost; });
+  ctx->items.resize(its.size());
+  for (size_t i = 0; i < its.size(); ++i) ctx->items[i] = its[i].v;
 }
 
 extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, uint64_t* report_offset_global) {
@@ -353,20 +395,19 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     launches += n_samples ? 1 : 0;
     // cut balanced buckets; the histogram becomes the bin map in place
     CK(ctx->d_bucket_start.ensure(kMaxBuckets + 1), "alloc buckets");
-    CK(ctx->d_order.ensure(kMaxBuckets), "alloc order");
     CK(ctx->d_cut.ensure(2 * kMaxBuckets + 2), "alloc cut scratch");
     CK(ctx->d_cutscr.ensure(2 * ((ctx->n_bins + 1023) / 1024) + 4 + ctx->n_bins), "alloc cut scratch");
     CK(launch_cut(ctx->d_hist.p, ctx->n_bins, ctx->coarse_bits, ctx->n_words, kMaxBuckets, ctx->d_bucket_start.p,
                   ctx->d_cut.p, ctx->d_cut.p + kMaxBuckets, ctx->d_cut.p + 2 * kMaxBuckets, ctx->d_cutscr.p,
-                  ctx->d_order.p, s, &launches), "k_cut");
+                  s, &launches), "k_cut");
     // the bucket count and starts come back with the partition's counters (one sync)
     CK(cudaMemcpyAsync(ctx->h_nb.p, ctx->d_cut.p + 2 * kMaxBuckets, 4, cudaMemcpyDeviceToHost, s), "nb d2h");
     CK(cudaMemcpyAsync(ctx->h_bstart.p, ctx->d_bucket_start.p, (kMaxBuckets + 1) * 8, cudaMemcpyDeviceToHost, s),
        "buckets d2h");
+    CK(cudaMemcpyAsync(ctx->h_weight.p, ctx->d_cut.p, kMaxBuckets * 4, cudaMemcpyDeviceToHost, s), "weights d2h");
   } else if (ctx->d_bin_map.cap == 0) {
     CK(upload(ctx->d_bin_map, ctx->bin_map, s), "upload bin map");
     CK(upload(ctx->d_bucket_start, ctx->bucket_start, s), "upload bucket starts");
-    CK(upload(ctx->d_order, ctx->order, s), "upload order");
   }
   if (!balanced) ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;   // fixed buckets
   if (timing) cudaEventRecord(ctx->ev[7], s);
@@ -402,9 +443,13 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     reset_batch(ctx);
     return fail(ctx, ARB_ETRACE, "malformed record at batch position " + std::to_string(hst.err_pos));
   }
+  std::vector<double> bucket_events;      // estimated events per bucket (sampled)
   if (balanced) {
     const uint32_t nb = *ctx->h_nb.p;
     ctx->bucket_start.assign(ctx->h_bstart.p, ctx->h_bstart.p + nb + 1);
+    const double stride = (double)std::max<uint64_t>(1, n / kSampleCap);
+    bucket_events.resize(nb);
+    for (uint32_t b = 0; b < nb; ++b) bucket_events[b] = ctx->h_weight.p[b] * stride;
   }
   ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;
   S.buckets = ctx->n_buckets;
@@ -450,6 +495,8 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   S.range_ops = plan.range_ops.size();
   S.tasks = plan.tasks;
   S.ignored_words = hst.ignored_words + plan.ignored_words;
+  build_items(ctx, plan, bucket_events);
+  CK(upload_pinned(ctx->d_items, ctx->h_items, ctx->items, s), "upload work items");
   CK(upload_pinned(ctx->ops_start, ctx->h_ops_start, plan.ops_start, s), "upload ops_start");
   CK(upload_pinned(ctx->ops, ctx->h_ops, plan.ops, s), "upload ops");
   CK(ctx->cand.ensure(ctx->cand_cap), "alloc candidates");
@@ -459,10 +506,11 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   ReplayParams rp{};
   rp.part_ev = ctx->part_ev.p; rp.segs = ctx->segs.p; rp.seg_first = ctx->seg_first.p;
   rp.n_buckets = ctx->n_buckets; rp.bucket_bits = ctx->bucket_bits; rp.n_words = ctx->n_words;
-  rp.bucket_start = ctx->d_bucket_start.p; rp.order = ctx->d_order.p;
+  rp.bucket_start = ctx->d_bucket_start.p;
+  rp.items = ctx->d_items.p; rp.n_items = (uint32_t)ctx->items.size();
   rp.shadow = ctx->shadow; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
   rp.cand = ctx->cand.p; rp.cand_cap = ctx->cand_cap; rp.st = ctx->dstats.p;
-  int n_ctas = std::max(1, std::min<int>((int)ctx->n_buckets, ctx->n_sms * kReplayCtasPerSm));
+  int n_ctas = std::max(1, std::min<int>((int)ctx->items.size(), ctx->n_sms * kReplayCtasPerSm));
   CK(launch_replay(rp, std::max(n_ctas, 1), s), "k_replay");
   launches += 1;
   if (timing) cudaEventRecord(ctx->ev[3], s);

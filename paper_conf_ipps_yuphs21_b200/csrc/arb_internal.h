@@ -117,7 +117,8 @@ struct ReplayParams {
   const uint32_t* seg_first;              // [n_buckets + 1] first entry of each bucket
   uint32_t n_buckets, bucket_bits;
   const uint64_t* bucket_start;           // [n_buckets + 1] first relative word of each bucket
-  const uint32_t* order;                  // buckets in scheduling order (largest first)
+  const uint4* items; uint32_t n_items;   // work items in scheduling order (largest first):
+                                          // {bucket, word lo, word hi (bucket-relative), partial}
   uint64_t n_words;
   uint8_t* shadow;                        // n_words bytes
   const uint32_t* ops_start;              // [n_buckets + 1]
@@ -148,10 +149,10 @@ struct MirParams {
 // ---- kernel launchers (kernels.cu) -----------------------------------------
 cudaError_t launch_sample(const SampleParams& p, uint64_t n_samples, cudaStream_t s);
 // scratch: 2 * ceil(n_bins / 1024) + 4 + n_bins u32.  Writes the bucket count
-// (*nb_out), bucket starts, weights and the replay order (heaviest first).
+// (*nb_out), bucket starts and the sampled event weight of every bucket.
 cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits, uint64_t n_words,
                        uint32_t max_buckets, uint64_t* bucket_start, uint32_t* weight, uint32_t* first_bin,
-                       uint32_t* nb_out, uint32_t* scratch, uint32_t* order, cudaStream_t s, int* launches);
+                       uint32_t* nb_out, uint32_t* scratch, cudaStream_t s, int* launches);
 cudaError_t launch_partition(const PartParams& p, cudaStream_t s);
 // Sorts the 8-B segment entries {bucket << 21 | chunk, start | len << 16 | chunk bit 21 << 31}
 // by (bucket, chunk) (a, b: ping-pong buffers), writes the replay form

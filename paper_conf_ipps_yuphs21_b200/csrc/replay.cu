@@ -45,6 +45,8 @@ struct ReplaySmem {
   uint32_t red[RT / 32], red2[RT / 32], wscan[RT / 32];
   uint32_t wcnt[RT / 32], wev[RT / 32];
   uint32_t bucket, op_cur, op_end, next_op;
+  uint32_t part_lo, part_hi;      // the work item's word range inside the bucket
+  bool partial;                   //   (partial: not the whole bucket)
   uint32_t seg0, cum0, n_segs, n_events, wsc, nwin;
   uint64_t bucket_base;
 };
@@ -123,12 +125,13 @@ __device__ void apply_ops_before(ReplaySmem& S, const ReplayParams& p, uint32_t 
       sel = sel_compose(o2.sel, sel);
       ++k2;
     }
-    stream_apply(p.shadow, o.lo, o.hi, sel);
+    const uint64_t lo = max(o.lo, S.bucket_base + S.part_lo), hi = min(o.hi, S.bucket_base + S.part_hi);
+    stream_apply(p.shadow, lo, hi, sel);
     __syncthreads();
     if (threadIdx.x == 0) {
       S.op_cur = k2;
       S.next_op = k2 < S.op_end ? p.ops[k2].pos : 0xFFFFFFFFu;
-      atomicAdd(&p.st->range_words_applied, (unsigned long long)(o.hi - o.lo));
+      if (hi > lo) atomicAdd(&p.st->range_words_applied, (unsigned long long)(hi - lo));
     }
     __syncthreads();
   }
@@ -209,7 +212,8 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
     if (i < m) {
       const uint2 e = ev[i];
       word[j] = e.x & kWordMask; op[j] = e.x >> 30; pos[j] = e.y;
-      s_pre[j] = __ldcg(sh + word[j]);
+      if (word[j] - S.part_lo < S.part_hi - S.part_lo) s_pre[j] = __ldcg(sh + word[j]);
+      else op[j] = 4;                                       // another work item's word
     }
   }
   // writes (WH = 1, WT = 3: odd ops) enter the table: slot {word, pos << 2 | op}
@@ -362,11 +366,51 @@ __device__ __forceinline__ uint32_t acc_summary(uint32_t op) {
 __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   uint32_t lo = 0xFFFFFFFFu, hi = 0;
-  for (uint32_t i = tid; i < m; i += RT) {
-    const uint2 e = ev[i];
-    S.u.s.keyA[i] = e.x; S.u.s.posA[i] = e.y;
-    const uint32_t w = e.x & kWordMask;
-    lo = min(lo, w); hi = max(hi, w);
+  if (S.partial) {
+    // keep only the events of the work item's words (stable block compaction)
+    uint32_t keep[RI], c = 0;
+#pragma unroll
+    for (int j = 0; j < RI; ++j) {
+      const uint32_t i = tid * RI + j;
+      const uint32_t w = i < m ? (ev[i].x & kWordMask) : 0;
+      keep[j] = i < m && w >= S.part_lo && w < S.part_hi;
+      c += keep[j];
+    }
+    uint32_t incl = c;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t o = __shfl_up_sync(FULL, incl, d);
+      if (lane >= (uint32_t)d) incl += o;
+    }
+    __syncthreads();
+    if (lane == 31) S.wscan[warp] = incl;
+    __syncthreads();
+    uint32_t o = incl - c, tot = 0;
+    for (uint32_t w = 0; w < RT / 32; ++w) { if (w < warp) o += S.wscan[w]; tot += S.wscan[w]; }
+#pragma unroll
+    for (int j = 0; j < RI; ++j) {
+      if (keep[j]) {
+        const uint2 e = ev[tid * RI + j];
+        S.u.s.keyA[o] = e.x; S.u.s.posA[o] = e.y;
+        const uint32_t w = e.x & kWordMask;
+        lo = min(lo, w); hi = max(hi, w);
+        ++o;
+      }
+    }
+    m = tot;
+    if (m == 0) {
+      __syncthreads();
+      hash_clear(S);
+      __syncthreads();
+      return;
+    }
+  } else {
+    for (uint32_t i = tid; i < m; i += RT) {
+      const uint2 e = ev[i];
+      S.u.s.keyA[i] = e.x; S.u.s.posA[i] = e.y;
+      const uint32_t w = e.x & kWordMask;
+      lo = min(lo, w); hi = max(hi, w);
+    }
   }
   block_minmax(lo, hi, S.red, S.red2);
   const uint32_t span = hi - lo;
@@ -569,7 +613,13 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
   for (;;) {
     if (tid == 0) {
       const unsigned long long w = atomicAdd(&p.st->work, 1ull);
-      S.bucket = w < p.n_buckets ? p.order[w] : 0xFFFFFFFFu;
+      if (w < p.n_items) {
+        const uint4 it = p.items[w];
+        S.bucket = it.x; S.part_lo = it.y; S.part_hi = it.z;
+        S.partial = it.w != 0;
+      } else {
+        S.bucket = 0xFFFFFFFFu;
+      }
     }
     __syncthreads();
     const uint32_t b = S.bucket;

@@ -174,26 +174,9 @@ __global__ void k_cut_weights(CutArgs a) {   // one CTA: prefix differences
   }
 }
 
-// replay scheduling order = buckets by weight, heaviest first (stable: rank =
-// #heavier + #equal with a smaller id); CTA c ranks buckets [256c, 256c + 256)
-constexpr int kOrderT = 256;
-__global__ void __launch_bounds__(kOrderT) k_cut_order(CutArgs a, uint32_t* order) {
-  __shared__ uint32_t w[kMaxBuckets];
-  const uint32_t nb = *a.nb_out;
-  if (blockIdx.x * kOrderT >= nb) return;
-  for (uint32_t b = threadIdx.x; b < nb; b += blockDim.x) w[b] = a.weight[b];
-  __syncthreads();
-  const uint32_t b = blockIdx.x * kOrderT + threadIdx.x;
-  if (b >= nb) return;
-  const uint32_t x = w[b];
-  uint32_t r = 0;
-  for (uint32_t c = 0; c < nb; ++c) r += (w[c] > x) | ((w[c] == x) & (c < b));
-  order[r] = b;
-}
-
 cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits, uint64_t n_words,
                        uint32_t max_buckets, uint64_t* bucket_start, uint32_t* weight, uint32_t* first_bin,
-                       uint32_t* nb_out, uint32_t* scratch, uint32_t* order, cudaStream_t s, int* launches) {
+                       uint32_t* nb_out, uint32_t* scratch, cudaStream_t s, int* launches) {
   const uint32_t nt = (n_bins + kT - 1) / kT;
   CutArgs a{hist_map, n_bins, coarse_bits, n_words, max_buckets, bucket_start, weight, first_bin, nb_out,
             scratch, scratch + nt, scratch + 2 * nt, scratch + 2 * nt + 4};
@@ -204,8 +187,7 @@ cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits
   k_cut_write<<<nt, kT, 0, s>>>(a);
   k_cut_map<<<148, 1024, 0, s>>>(a);
   k_cut_weights<<<1, kT, 0, s>>>(a);
-  k_cut_order<<<kMaxBuckets / kOrderT, kOrderT, 0, s>>>(a, order);
-  *launches += 8;
+  *launches += 7;
   return cudaGetLastError();
 }
 

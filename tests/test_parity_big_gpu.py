@@ -14,11 +14,11 @@ import pytest
 pytestmark = pytest.mark.gpu
 
 
-def _gpu_run(prog, lo, hi, flushes=None, recs=None, gidx=None):
+def _gpu_run(prog, lo, hi, flushes=None, recs=None, gidx=None, flags=0):
     import torch
     from paper_conf_ipps_yuphs21_b200 import Context, reports_to_triples
     from gpu_util import to_device
-    ctx = Context(lo * 8, (hi - lo) * 8, report_capacity=1 << 25)
+    ctx = Context(lo * 8, (hi - lo) * 8, report_capacity=1 << 25, flags=flags)
     if recs is None:
         rec = prog.fill_host()
         recs = to_device(rec)
@@ -33,12 +33,12 @@ def _gpu_run(prog, lo, hi, flushes=None, recs=None, gidx=None):
     return ctx, triples
 
 
-def _check_full(orc, prog):
+def _check_full(orc, prog, flags=0):
     rec = prog.fill_host()
     lo, hi = prog.addr_base // 8, (prog.addr_base + prog.addr_bytes) // 8
     exp = orc.replay(rec, prog.addr_base, prog.addr_bytes)
     assert exp.rc == 0
-    ctx, got = _gpu_run(prog, lo, hi)
+    ctx, got = _gpu_run(prog, lo, hi, flags=flags)
     assert sorted(got) == exp.triples()
     assert np.array_equal(ctx.get_shadow(lo, hi - lo), exp.shadow)
     ctx.close()
@@ -52,9 +52,11 @@ def test_config3_scaled(orc):
     assert kinds == {1, 2, 3}          # alloc-mapped row read, stale `stop`, the missing taskwait
 
 
-def test_config4_scaled(orc):
+@pytest.mark.parametrize("flags", [0, 4])
+def test_config4_scaled(orc, flags):
+    """flags=4 (ARB_F_SMALL_PARTS): the range-heavy buckets run as word-range parts."""
     from gen import native
-    exp = _check_full(orc, native.config4(scale=1 / 512))
+    exp = _check_full(orc, native.config4(scale=1 / 512), flags=flags)
     assert {k for _, _, k in exp.triples()} == {2}   # 503.postencil: stale output reads
 
 

@@ -15,7 +15,7 @@ pytestmark = pytest.mark.gpu
 def check(orc, rec, base, size, **kw):
     okw = {k: kw.pop(k) for k in ("dedup_first",) if k in kw}
     exp = orc.replay(rec, base, size, **okw)
-    flags = 1 if okw.get("dedup_first") else 0
+    flags = (1 if okw.get("dedup_first") else 0) | kw.pop("flags", 0)
     rc, got, shadow, st = run_gpu(rec, base, size, flags=flags, **kw)
     assert rc == exp.rc
     if rc == 0:
@@ -64,6 +64,22 @@ def test_fuzz_large_steps(orc, seed):
                                      loop_max=20000)
     for bb in (0, 11):
         check(orc, rec, base, span, bucket_bits=bb)
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_split_parts(orc, seed):
+    """Range-heavy buckets replayed as word-range parts by separate CTAs
+    (ARB_F_SMALL_PARTS forces the split at 1024-word parts)."""
+    from gen.fuzz import random_program
+    rec, base, span = random_program(2000 + seed, n_arrays=4, array_words=8192, steps=200)
+    for bb in (0, 13):
+        _, st = check(orc, rec, base, span, bucket_bits=bb, flags=4)
+
+
+def test_config2_split_parts(orc):
+    from gen.configs import config2
+    rec, base, size = config2()
+    check(orc, rec, base, size, flags=4)
 
 
 def test_hot_word(orc):
