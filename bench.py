@@ -270,7 +270,7 @@ def main():
         st_acc = {"access_words": 0, "range_words": 0, "reports": 0, "launches": 0, "ms_partition": 0.0,
                   "ms_replay": 0.0, "ms_mir": 0.0, "ms_reports": 0.0, "ms_control": 0.0, "ms_total": 0.0,
                   "ms_sample": 0.0, "ms_segsort": 0.0, "ms_host_control": 0.0, "records": 0,
-                  "steps_fast": 0, "steps_sort": 0, "max_bucket_events": 0,
+                  "steps_fast": 0, "steps_sort": 0, "max_bucket_events": 0, "work_items": 0,
                   "by_kind": [0, 0, 0, 0]}
         for (a, b) in flushes:
             ctx.submit_events(recs[a:b], global_index=gidx[a:b], stream=stream)
@@ -278,7 +278,7 @@ def main():
             st = ctx.stats()
             for k in ("access_words", "range_words", "reports", "records", "ms_partition", "ms_replay",
                       "ms_mir", "ms_reports", "ms_control", "ms_total", "ms_sample", "ms_segsort",
-                      "ms_host_control", "steps_fast", "steps_sort"):
+                      "ms_host_control", "steps_fast", "steps_sort", "work_items"):
                 st_acc[k] += st[k]
             st_acc["max_bucket_events"] = max(st_acc["max_bucket_events"], st["max_bucket_events"])
             st_acc["launches"] += st["kernel_launches"]
@@ -394,6 +394,7 @@ def main():
                            "flushes_per_step_rank0": len(flushes), "shard_words": hi - lo,
                            "replay_steps_fast_sort_rank0": [int(s0["steps_fast"]), int(s0["steps_sort"])],
                            "max_bucket_events_rank0": int(s0["max_bucket_events"]),
+                           "replay_work_items_rank0": int(s0["work_items"]),
                            "l2": "inputs larger than L2 (>= 16 GB of records per step)",
                            "generation_s": round(t_gen, 2)},
                 "clocks": clk, "e2e": e2e, "gpu_launches": int(sum(s["launches"] for s in per_step)),

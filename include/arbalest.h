@@ -117,6 +117,7 @@ typedef struct {
   uint64_t steps_fast, steps_sort;  /* replay steps by kind                  */
   double   ms_segsort;       /* GPU: segment-entry sort (inside ms_control)                 */
   double   ms_host_control;  /* host wall time of the Table I / task resolution             */
+  uint64_t work_items;       /* replay work items (buckets, or word-range parts of buckets) */
 } arb_stats;
 
 typedef struct arb_ctx_s* arb_ctx;

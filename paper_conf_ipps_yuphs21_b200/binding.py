@@ -45,7 +45,8 @@ class arb_stats(ctypes.Structure):
                 ("ms_reports", ctypes.c_double), ("ms_total", ctypes.c_double),
                 ("kernel_launches", ctypes.c_uint64), ("ms_sample", ctypes.c_double),
                 ("steps_fast", ctypes.c_uint64), ("steps_sort", ctypes.c_uint64),
-                ("ms_segsort", ctypes.c_double), ("ms_host_control", ctypes.c_double)]
+                ("ms_segsort", ctypes.c_double), ("ms_host_control", ctypes.c_double),
+                ("work_items", ctypes.c_uint64)]
 
     def as_dict(self):
         d = {}

@@ -311,30 +311,55 @@ static void build_items(arb_ctx ctx, const FlushPlan& plan, const std::vector<do
   const bool small = ctx->cfg.flags & ARB_F_SMALL_PARTS;
   const double kPartWords = small ? 1024.0 : double(1u << 24);
   const uint32_t nb = ctx->n_buckets;
+  std::vector<uint32_t> parts(nb, 1);
+  std::vector<double> rws(nb, 0.0);
+  bool any_split = false;
+  for (uint32_t b = 0; b < nb; ++b) {
+    double rw = 0;
+    for (uint32_t k = plan.ops_start[b]; k < plan.ops_start[b + 1]; ++k) rw += double(plan.ops[k].hi - plan.ops[k].lo);
+    rws[b] = rw;
+    const double ev = b < bucket_events.size() ? bucket_events[b] : 0.0;
+    const uint64_t span = ctx->bucket_start[b + 1] - ctx->bucket_start[b];
+    if (rw > 2 * kPartWords && span >= 32) {
+      const double by_range = rw / kPartWords, by_events = small ? by_range : rw / (ev * kWordsPerEvent + 1.0);
+      uint32_t np = (uint32_t)std::max(1.0, std::min<double>(std::min(by_range, by_events), kMaxParts));
+      np = (uint32_t)std::min<uint64_t>(np, span / 16);
+      parts[b] = np;
+      any_split |= np > 1;
+    }
+  }
+  ctx->items.clear();
+  if (!any_split) {
+    // every bucket whole: order by sampled events, heaviest first (ties: bucket id)
+    std::vector<uint64_t> key(nb);
+    for (uint32_t b = 0; b < nb; ++b) {
+      const double ev = b < bucket_events.size() ? bucket_events[b] : 0.0;
+      const uint64_t w = (uint64_t)std::min(ev, 4.0e9);
+      key[b] = ((0xFFFFFFFFull - w) << 32) | b;
+    }
+    std::sort(key.begin(), key.end());
+    for (uint64_t k : key) {
+      const uint32_t b = (uint32_t)k;
+      ctx->items.push_back(make_uint4(b, 0, (uint32_t)(ctx->bucket_start[b + 1] - ctx->bucket_start[b]), 0u));
+    }
+    return;
+  }
   struct It { double cost; uint4 v; };
   std::vector<It> its;
   its.reserve(nb);
   for (uint32_t b = 0; b < nb; ++b) {
-    double rw = 0;
-    for (uint32_t k = plan.ops_start[b]; k < plan.ops_start[b + 1]; ++k) rw += double(plan.ops[k].hi - plan.ops[k].lo);
     const double ev = b < bucket_events.size() ? bucket_events[b] : 0.0;
     const uint64_t span = ctx->bucket_start[b + 1] - ctx->bucket_start[b];
-    uint32_t np = 1;
-    if (rw > 2 * kPartWords && span >= 32) {
-      double by_range = rw / kPartWords, by_events = small ? by_range : rw / (ev * kWordsPerEvent + 1.0);
-      double x = std::min(by_range, by_events);
-      np = (uint32_t)std::max(1.0, std::min<double>(x, kMaxParts));
-      np = (uint32_t)std::min<uint64_t>(np, span / 16);
-    }
+    const uint32_t np = parts[b];
     const uint64_t step = ((span + np - 1) / np + 15) & ~15ull;
     for (uint32_t q = 0; q < np; ++q) {
       const uint64_t lo = std::min<uint64_t>(span, q * step), hi = std::min<uint64_t>(span, lo + step);
       if (lo >= hi && np > 1) continue;
-      const double cost = ev * kWordsPerEvent + rw * double(hi - lo) / double(std::max<uint64_t>(span, 1));
+      const double cost = ev * kWordsPerEvent + (np == 1 ? 0.0 : rws[b] * double(hi - lo) / double(span));
       its.push_back(It{cost, make_uint4(b, (uint32_t)lo, (uint32_t)hi, np > 1 ? 1u : 0u)});
     }
   }
-  std::stable_sort(its.begin(), its.end(), [](const It& a, const It& b) { return a.cost > b.cost; });
+  std::stable_sort(its.begin(), its.end(), [](const It& x, const It& y) { return x.cost > y.cost; });
   ctx->items.resize(its.size());
   for (size_t i = 0; i < its.size(); ++i) ctx->items[i] = its[i].v;
 }
@@ -490,12 +515,13 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     reset_batch(ctx);
     return fail(ctx, plan.rc, plan.err + " (batch position " + std::to_string(plan.err_pos) + ")");
   }
-  S.ms_host_control = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_host0).count();
   S.range_words = plan.range_words;
   S.range_ops = plan.range_ops.size();
   S.tasks = plan.tasks;
   S.ignored_words = hst.ignored_words + plan.ignored_words;
   build_items(ctx, plan, bucket_events);
+  S.work_items = ctx->items.size();
+  S.ms_host_control = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_host0).count();
   CK(upload_pinned(ctx->d_items, ctx->h_items, ctx->items, s), "upload work items");
   CK(upload_pinned(ctx->ops_start, ctx->h_ops_start, plan.ops_start, s), "upload ops_start");
   CK(upload_pinned(ctx->ops, ctx->h_ops, plan.ops, s), "upload ops");

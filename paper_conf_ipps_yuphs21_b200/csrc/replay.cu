@@ -200,11 +200,14 @@ __device__ __forceinline__ uint32_t hslot(uint32_t w) { return (w * 2654435761u)
 // not change the state, so a read's state-before is the state loaded
 // at the start of the step, or — if its word's single write precedes it — the
 // image of that write; the write event itself commits the word's final state.
+template <bool PARTIAL>
 __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
   uint32_t slot[RI], word[RI], pos[RI], op[RI], s_pre[RI];
   bool multi = false;
   const uint8_t* sh = p.shadow + S.bucket_base;
   uint2* hs = S.u.h.slot;
+  uint32_t plo = 0, pw = 0;
+  if (PARTIAL) { plo = S.part_lo; pw = S.part_hi - S.part_lo; }
 #pragma unroll
   for (int j = 0; j < RI; ++j) {   // shadow loads first: their latency overlaps the hashing
     const uint32_t i = threadIdx.x + j * RT;
@@ -212,7 +215,7 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
     if (i < m) {
       const uint2 e = ev[i];
       word[j] = e.x & kWordMask; op[j] = e.x >> 30; pos[j] = e.y;
-      if (word[j] - S.part_lo < S.part_hi - S.part_lo) s_pre[j] = __ldcg(sh + word[j]);
+      if (!PARTIAL || word[j] - plo < pw) s_pre[j] = __ldcg(sh + word[j]);
       else op[j] = 4;                                       // another work item's word
     }
   }
@@ -273,6 +276,11 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
   }
   // the caller's next barrier orders this reset before the next step's inserts
   return true;
+}
+
+// the fast step of a word-range part (rare: range-heavy buckets), out of line
+__device__ bool step_fast_partial(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
+  return step_fast<true>(S, p, ev, m);
 }
 
 // ---- sort step -------------------------------------------------------------------------
@@ -657,7 +665,7 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         for (uint32_t e = tid; e < m; e += RT) cnt += ev[e].y < S.next_op;
         cut = block_sum(cnt, S.red);
       }
-      const bool fast = step_fast(S, p, ev, cut);
+      const bool fast = S.partial ? step_fast_partial(S, p, ev, cut) : step_fast<false>(S, p, ev, cut);
       if (!fast) step_sort(S, p, ev, cut);
       if (tid == 0) atomicAdd(fast ? &p.st->steps_fast : &p.st->steps_sort, 1ull);
       e0 += cut;
