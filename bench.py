@@ -271,6 +271,7 @@ def main():
                   "ms_replay": 0.0, "ms_mir": 0.0, "ms_reports": 0.0, "ms_control": 0.0, "ms_total": 0.0,
                   "ms_sample": 0.0, "ms_segsort": 0.0, "ms_host_control": 0.0, "records": 0,
                   "steps_fast": 0, "steps_sort": 0, "max_bucket_events": 0, "work_items": 0,
+                  "hot_buckets": 0,
                   "by_kind": [0, 0, 0, 0]}
         for (a, b) in flushes:
             ctx.submit_events(recs[a:b], global_index=gidx[a:b], stream=stream)
@@ -278,7 +279,8 @@ def main():
             st = ctx.stats()
             for k in ("access_words", "range_words", "reports", "records", "ms_partition", "ms_replay",
                       "ms_mir", "ms_reports", "ms_control", "ms_total", "ms_sample", "ms_segsort",
-                      "ms_host_control", "steps_fast", "steps_sort", "work_items"):
+                      "ms_host_control", "steps_fast", "steps_sort", "work_items",
+                      "hot_buckets"):
                 st_acc[k] += st[k]
             st_acc["max_bucket_events"] = max(st_acc["max_bucket_events"], st["max_bucket_events"])
             st_acc["launches"] += st["kernel_launches"]
@@ -395,6 +397,7 @@ def main():
                            "replay_steps_fast_sort_rank0": [int(s0["steps_fast"]), int(s0["steps_sort"])],
                            "max_bucket_events_rank0": int(s0["max_bucket_events"]),
                            "replay_work_items_rank0": int(s0["work_items"]),
+                           "hot_buckets_rank0": int(s0["hot_buckets"]),
                            "l2": "inputs larger than L2 (>= 16 GB of records per step)",
                            "generation_s": round(t_gen, 2)},
                 "clocks": clk, "e2e": e2e, "gpu_launches": int(sum(s["launches"] for s in per_step)),

@@ -78,8 +78,10 @@ enum arb_status {
 #define ARB_F_DEDUP_FIRST 0x1u  /* keep only the first report per (word, kind) (Z3)      */
 #define ARB_F_TIMING      0x2u  /* record CUDA events around every kernel (arb_get_stats) */
 #define ARB_F_SMALL_PARTS 0x4u  /* test knob: split every bucket with >= 2048 range-op words
-                                   into word-range parts replayed by separate CTAs (the
-                                   mechanism normally used for range-heavy buckets only)  */
+                                   into word-range parts replayed by separate CTAs, and
+                                   replay every small bucket with >= 64 events as 3 time
+                                   slices (the mechanisms normally used for range-heavy
+                                   and hot buckets only)                                  */
 
 typedef struct {
   uint64_t addr_base;        /* tracked OV byte range [addr_base, addr_base+addr_bytes);   */
@@ -117,7 +119,8 @@ typedef struct {
   uint64_t steps_fast, steps_sort;  /* replay steps by kind                  */
   double   ms_segsort;       /* GPU: segment-entry sort (inside ms_control)                 */
   double   ms_host_control;  /* host wall time of the Table I / task resolution             */
-  uint64_t work_items;       /* replay work items (buckets, or word-range parts of buckets) */
+  uint64_t work_items;       /* replay work items (buckets, word-range parts, hot slices)   */
+  uint64_t hot_buckets;      /* buckets replayed as time slices (hot words, K5)             */
 } arb_stats;
 
 typedef struct arb_ctx_s* arb_ctx;

@@ -46,7 +46,7 @@ class arb_stats(ctypes.Structure):
                 ("kernel_launches", ctypes.c_uint64), ("ms_sample", ctypes.c_double),
                 ("steps_fast", ctypes.c_uint64), ("steps_sort", ctypes.c_uint64),
                 ("ms_segsort", ctypes.c_double), ("ms_host_control", ctypes.c_double),
-                ("work_items", ctypes.c_uint64)]
+                ("work_items", ctypes.c_uint64), ("hot_buckets", ctypes.c_uint64)]
 
     def as_dict(self):
         d = {}

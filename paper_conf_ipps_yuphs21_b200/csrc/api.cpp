@@ -6,6 +6,7 @@
 #include <dlfcn.h>
 #include <algorithm>
 #include <chrono>
+#include <cmath>
 #include <cstring>
 #include <new>
 #include <string>
@@ -98,6 +99,16 @@ struct arb_ctx_s {
   std::vector<uint32_t> bin_map, hist;
   std::vector<uint64_t> bucket_start;
   std::vector<uint4> items;                   // replay work items (see build_items)
+  std::vector<uint4> slice_items;             // K5 phase-3 items (second replay launch)
+  std::vector<uint4> hot;                     // K5 hot buckets {bucket, slices, span, 0}
+  std::vector<uint64_t> hot_off;              // per bucket scratch offset (hot buckets)
+  uint64_t hot_entries = 0;
+  DevBuf<uint4> d_slice_items, d_hot;
+  HostBuf<uint4> h_slice_items, h_hot;
+  DevBuf<uint64_t> d_hot_off;
+  HostBuf<uint64_t> h_hot_off;
+  DevBuf<uint16_t> hot_F;
+  DevBuf<uint8_t> hot_P;
   DevBuf<uint4> d_items;
   HostBuf<uint4> h_items;
   HostBuf<uint32_t> h_weight;
@@ -244,7 +255,9 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   ctx->m_rr_cum.release(); ctx->m_ins_inst.release(); ctx->m_qry_open_start.release(); ctx->m_open_list.release();
   ctx->m_own_start.release(); ctx->m_win_start.release(); ctx->m_own.release(); ctx->m_win.release();
   ctx->m_rr.release(); ctx->hkeys.release(); ctx->hvals.release(); ctx->counts.release();
-  ctx->d_bin_map.release(); ctx->d_items.release(); ctx->h_items.release(); ctx->h_weight.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_cut.release();
+  ctx->d_bin_map.release(); ctx->d_items.release(); ctx->h_items.release(); ctx->h_weight.release();
+  ctx->d_slice_items.release(); ctx->h_slice_items.release(); ctx->d_hot.release(); ctx->h_hot.release();
+  ctx->d_hot_off.release(); ctx->h_hot_off.release(); ctx->hot_F.release(); ctx->hot_P.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_cut.release();
   for (auto& e : ctx->ev) if (e) cudaEventDestroy(e);
   if (ctx->aux) cudaStreamDestroy(ctx->aux);
   ctx->h_stats.release(); ctx->h_nb.release(); ctx->h_ops_start.release(); ctx->h_bstart.release();
@@ -305,9 +318,18 @@ static void reset_batch(arb_ctx ctx) {
 // aligned): each part replays all of the bucket's events but acts only on its own
 // words, so the range-op streaming of one huge bucket spreads over many CTAs.
 // Cost model (per CTA): ~600 range-op words stream in the time of one event.
+//
+// Hot buckets (K5): a bucket of <= kHotSpan words whose estimated events exceed
+// 1.25x the per-CTA share of the flush (and 2^17) would be the replay's critical
+// path; it is cut into time slices of ~2^17 events: phase 1 (kItemSummary, in the
+// first replay launch) composes each slice's per-word transition functions,
+// k_carry (phase 2) carries the states across the slices and writes the final
+// shadow, and phase 3 (kItemSlice, second launch) replays each slice against its
+// carried-in states to classify its reads.
 static void build_items(arb_ctx ctx, const FlushPlan& plan, const std::vector<double>& bucket_events) {
   constexpr double kWordsPerEvent = 600.0;
-  constexpr uint32_t kMaxParts = 64;
+  constexpr uint32_t kMaxParts = 64, kMaxSlices = 64;
+  constexpr double kSliceEvents = double(1u << 17);
   const bool small = ctx->cfg.flags & ARB_F_SMALL_PARTS;
   const double kPartWords = small ? 1024.0 : double(1u << 24);
   const uint32_t nb = ctx->n_buckets;
@@ -328,8 +350,42 @@ static void build_items(arb_ctx ctx, const FlushPlan& plan, const std::vector<do
       any_split |= np > 1;
     }
   }
+  // hot buckets
+  ctx->hot.clear(); ctx->slice_items.clear(); ctx->hot_entries = 0;
+  double ev_tot = 0;
+  for (double e : bucket_events) ev_tot += e;
+  const double share = ev_tot / double(std::max(1, ctx->n_sms * kReplayCtasPerSm));
+  const bool force_hot = ctx->cfg.flags & ARB_F_SMALL_PARTS;     // test knob: slice every small busy bucket
+  std::vector<uint32_t> slices(nb, 0);
+  constexpr uint64_t kMaxHotEntries = 1ull << 29;      // K5 scratch: 3 B per entry
+  uint64_t hot_total = 0;
+  for (uint32_t b = 0; b < nb && b < bucket_events.size(); ++b) {
+    const uint64_t span = ctx->bucket_start[b + 1] - ctx->bucket_start[b];
+    const double ev = bucket_events[b];
+    if (parts[b] != 1 || span > kHotSpan) continue;
+    const bool hot = force_hot ? ev >= 64.0 : (ev > 1.25 * share && ev > kSliceEvents);
+    if (!hot) continue;
+    const double want = force_hot ? 3.0 : std::ceil(ev / kSliceEvents);
+    uint32_t ns = (uint32_t)std::max(2.0, std::min<double>(want, kMaxSlices));
+    const uint64_t span16 = (span + 15) & ~15ull;
+    ns = (uint32_t)std::min<uint64_t>(ns, kMaxHotEntries / 8 / span16);        // scratch per bucket
+    if (ns < 2 || hot_total + ns * span16 > kMaxHotEntries) continue;           // scratch per flush
+    hot_total += ns * span16;
+    slices[b] = ns;
+  }
+  bool any_hot = false;
+  ctx->hot_off.assign(nb, 0);
+  for (uint32_t b = 0; b < nb; ++b) {
+    if (!slices[b]) continue;
+    any_hot = true;
+    const uint32_t span = (uint32_t)(ctx->bucket_start[b + 1] - ctx->bucket_start[b]);
+    ctx->hot_off[b] = ctx->hot_entries;
+    ctx->hot_entries += (uint64_t)slices[b] * ((span + 15) & ~15u);
+    ctx->hot.push_back(make_uint4(b, slices[b], span, 0u));
+    for (uint32_t k = 0; k < slices[b]; ++k) ctx->slice_items.push_back(make_uint4(b, k, slices[b], kItemSlice));
+  }
   ctx->items.clear();
-  if (!any_split) {
+  if (!any_split && !any_hot) {
     // every bucket whole: order by sampled events, heaviest first (ties: bucket id)
     std::vector<uint64_t> key(nb);
     for (uint32_t b = 0; b < nb; ++b) {
@@ -350,13 +406,18 @@ static void build_items(arb_ctx ctx, const FlushPlan& plan, const std::vector<do
   for (uint32_t b = 0; b < nb; ++b) {
     const double ev = b < bucket_events.size() ? bucket_events[b] : 0.0;
     const uint64_t span = ctx->bucket_start[b + 1] - ctx->bucket_start[b];
+    if (slices[b]) {                   // phase-1 items of a hot bucket
+      for (uint32_t k = 0; k < slices[b]; ++k)
+        its.push_back(It{ev / slices[b] * kWordsPerEvent, make_uint4(b, k, slices[b], kItemSummary)});
+      continue;
+    }
     const uint32_t np = parts[b];
     const uint64_t step = ((span + np - 1) / np + 15) & ~15ull;
     for (uint32_t q = 0; q < np; ++q) {
       const uint64_t lo = std::min<uint64_t>(span, q * step), hi = std::min<uint64_t>(span, lo + step);
       if (lo >= hi && np > 1) continue;
       const double cost = ev * kWordsPerEvent + (np == 1 ? 0.0 : rws[b] * double(hi - lo) / double(span));
-      its.push_back(It{cost, make_uint4(b, (uint32_t)lo, (uint32_t)hi, np > 1 ? 1u : 0u)});
+      its.push_back(It{cost, make_uint4(b, (uint32_t)lo, (uint32_t)hi, np > 1 ? kItemPart : kItemWhole)});
     }
   }
   std::stable_sort(its.begin(), its.end(), [](const It& x, const It& y) { return x.cost > y.cost; });
@@ -520,9 +581,17 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   S.tasks = plan.tasks;
   S.ignored_words = hst.ignored_words + plan.ignored_words;
   build_items(ctx, plan, bucket_events);
-  S.work_items = ctx->items.size();
+  S.work_items = ctx->items.size() + ctx->slice_items.size();
+  S.hot_buckets = ctx->hot.size();
   S.ms_host_control = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_host0).count();
   CK(upload_pinned(ctx->d_items, ctx->h_items, ctx->items, s), "upload work items");
+  if (!ctx->hot.empty()) {
+    CK(upload_pinned(ctx->d_slice_items, ctx->h_slice_items, ctx->slice_items, s), "upload slice items");
+    CK(upload_pinned(ctx->d_hot, ctx->h_hot, ctx->hot, s), "upload hot buckets");
+    CK(upload_pinned(ctx->d_hot_off, ctx->h_hot_off, ctx->hot_off, s), "upload hot offsets");
+    CK(ctx->hot_F.ensure(ctx->hot_entries), "alloc hot F");
+    CK(ctx->hot_P.ensure(ctx->hot_entries), "alloc hot P");
+  }
   CK(upload_pinned(ctx->ops_start, ctx->h_ops_start, plan.ops_start, s), "upload ops_start");
   CK(upload_pinned(ctx->ops, ctx->h_ops, plan.ops, s), "upload ops");
   CK(ctx->cand.ensure(ctx->cand_cap), "alloc candidates");
@@ -536,8 +605,22 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   rp.items = ctx->d_items.p; rp.n_items = (uint32_t)ctx->items.size();
   rp.shadow = ctx->shadow; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
   rp.cand = ctx->cand.p; rp.cand_cap = ctx->cand_cap; rp.st = ctx->dstats.p;
+  rp.hot_off = ctx->d_hot_off.p; rp.hot_F = ctx->hot_F.p; rp.hot_P = ctx->hot_P.p;
   int n_ctas = std::max(1, std::min<int>((int)ctx->items.size(), ctx->n_sms * kReplayCtasPerSm));
   CK(launch_replay(rp, std::max(n_ctas, 1), s), "k_replay");
+  if (!ctx->hot.empty()) {
+    // K5 phases 2 and 3 (see build_items)
+    uint32_t max_span = 0;
+    for (const uint4& h : ctx->hot) max_span = std::max(max_span, h.z);
+    CK(launch_carry(ctx->d_hot.p, (uint32_t)ctx->hot.size(), max_span, ctx->d_bucket_start.p, ctx->d_hot_off.p,
+                    ctx->hot_F.p, ctx->hot_P.p, ctx->shadow, s), "k_carry");
+    CK(cudaMemsetAsync(&ctx->dstats.p->work, 0, sizeof(unsigned long long), s), "work reset");
+    ReplayParams r3 = rp;
+    r3.items = ctx->d_slice_items.p; r3.n_items = (uint32_t)ctx->slice_items.size();
+    const int n3 = std::max(1, std::min<int>((int)ctx->slice_items.size(), ctx->n_sms * kReplayCtasPerSm));
+    CK(launch_replay(r3, n3, s), "k_replay slices");
+    launches += 2;
+  }
   launches += 1;
   if (timing) cudaEventRecord(ctx->ev[3], s);
   CK(cudaMemcpyAsync(&hst, ctx->dstats.p, sizeof(hst), cudaMemcpyDeviceToHost, s), "stats d2h");

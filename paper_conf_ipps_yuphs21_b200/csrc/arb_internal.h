@@ -24,7 +24,7 @@ constexpr uint32_t kOVv = 1, kCVv = 2, kOVi = 4, kCVi = 8;
 // 5 = constant 1); 3 bits per output bit.  Every transition of P:255-261 is
 // a set-constant or copy-a-bit map, so the form is closed under composition.
 using Sel = uint32_t;
-constexpr Sel sel_make(uint32_t s0, uint32_t s1, uint32_t s2, uint32_t s3) {
+__host__ __device__ constexpr Sel sel_make(uint32_t s0, uint32_t s1, uint32_t s2, uint32_t s3) {
   return s0 | (s1 << 3) | (s2 << 6) | (s3 << 9);
 }
 constexpr Sel kSelId    = sel_make(0, 1, 2, 3);
@@ -54,6 +54,14 @@ constexpr int kReplayThreads = 256;
 constexpr int kReplayItems = 4;
 constexpr int kStep = kReplayThreads * kReplayItems;  // events per step
 constexpr int kReplayCtasPerSm = 4;
+
+// replay work items {bucket, y, z, kind}
+constexpr uint32_t kItemWhole = 0;      // the whole bucket
+constexpr uint32_t kItemPart = 1;       // words [y, z) of the bucket (range-heavy buckets)
+constexpr uint32_t kItemSlice = 2;      // hot bucket (K5), phase 3: events of time slice y of z,
+                                        //   replayed on a private copy of the carried-in states
+constexpr uint32_t kItemSummary = 3;    // hot bucket (K5), phase 1: transition functions of slice y of z
+constexpr uint32_t kHotSpan = 1u << 20; // hot buckets span at most this many words
 
 // device-side counters and error flags of one flush
 struct DevStats {
@@ -118,7 +126,11 @@ struct ReplayParams {
   uint32_t n_buckets, bucket_bits;
   const uint64_t* bucket_start;           // [n_buckets + 1] first relative word of each bucket
   const uint4* items; uint32_t n_items;   // work items in scheduling order (largest first):
-                                          // {bucket, word lo, word hi (bucket-relative), partial}
+                                          // {bucket, y, z, kItem*}
+  // hot buckets (K5): bucket b's scratch starts at entry hot_off[b] of hot_F
+  // (slice functions, u16 selector form) and hot_P (carried-in states, u8);
+  // slice k uses [hot_off[b] + k * span16, + span16), span16 = span rounded to 16
+  const uint64_t* hot_off; uint16_t* hot_F; uint8_t* hot_P;
   uint64_t n_words;
   uint8_t* shadow;                        // n_words bytes
   const uint32_t* ops_start;              // [n_buckets + 1]
@@ -161,6 +173,11 @@ cudaError_t launch_partition(const PartParams& p, cudaStream_t s);
 cudaError_t launch_sort_segments(uint2* a, uint2* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
                                  uint32_t* first, uint4* out, cudaStream_t s, int* launches);
 cudaError_t launch_replay(const ReplayParams& p, int n_ctas, cudaStream_t s);
+// K5 phase 2: for every hot bucket {bucket, slices, span, 0} carry the states
+// across its slices: P_0 = shadow, P_{k+1} = F_k(P_k); shadow = F_last(P_last)
+cudaError_t launch_carry(const uint4* hot, uint32_t n_hot, uint32_t max_span, const uint64_t* bucket_start,
+                         const uint64_t* hot_off, const uint16_t* hot_F, uint8_t* hot_P, uint8_t* shadow,
+                         cudaStream_t s);
 cudaError_t launch_mir(const MirParams& p, uint64_t n_ins_pos, uint64_t n_qry_pos, uint64_t n_rr_words,
                        cudaStream_t s, int* launches);
 // report compaction: sorts candidates, removes duplicates, optional dedup-first,

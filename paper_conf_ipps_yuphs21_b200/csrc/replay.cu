@@ -21,6 +21,7 @@
 // valid) and split UUM / USD with the init bits (Table II).  The shadow
 // (1 byte per word) carries each word's state across steps.
 #include "kcommon.cuh"
+#include <algorithm>
 
 namespace arb {
 
@@ -32,12 +33,15 @@ constexpr int kWin = 2 * RT;                 // segment descriptors staged per s
 constexpr int kHSlots = 4096;                // hash slots (load <= 1/2)
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
 constexpr uint32_t kWordMask = 0x3FFFFFFFu;
+constexpr int kZSlots = 2048;                // summary-step hash slots (<= 1024 writes per step)
+static_assert(kZSlots * 12 <= kHSlots * 8 && kZSlots >= 2 * STEP, "summary hash fits the hash area");
 
 struct ReplaySmem {
   uint2 ev[2][STEP];              // double-buffered step events {key, pos} (cp.async)
   union {
     struct { uint32_t keyA[STEP], posA[STEP], keyB[STEP], posB[STEP]; uint16_t hist[RT / 32][256]; } s;
     struct { uint2 slot[kHSlots]; } h;      // fast step: written words {word, pos << 2 | op}
+    struct { uint32_t key[kZSlots], lastw[kZSlots], anyw[kZSlots]; } z;  // hot-slice summary step (K5)
   } u;
   uint32_t wstart[kWin];          // staged segment list window: global event index
   uint32_t wcum[kWin + 1];        //   and bucket-relative first event of each segment
@@ -47,6 +51,10 @@ struct ReplaySmem {
   uint32_t bucket, op_cur, op_end, next_op;
   uint32_t part_lo, part_hi;      // the work item's word range inside the bucket
   bool partial;                   //   (partial: not the whole bucket)
+  uint32_t mode;                  // kItem* of the work item
+  uint8_t* shrel;                 // state of bucket-relative word w: shrel[w]
+  uint16_t* fsum;                 // summary slice: composed transition of word w: fsum[w]
+  uint32_t slice, n_slices;       // hot bucket slice (kItemSlice / kItemSummary)
   uint32_t seg0, cum0, n_segs, n_events, wsc, nwin;
   uint64_t bucket_base;
 };
@@ -80,14 +88,17 @@ __device__ __forceinline__ void block_minmax(uint32_t& lo, uint32_t& hi, uint32_
 }
 
 // ---- range ops ----------------------------------------------------------------
-// Apply transition `sel` to shadow bytes [lo, hi) (relative word indices).
-__device__ void stream_apply(uint8_t* shadow, uint64_t lo, uint64_t hi, Sel sel) {
+// Apply transition `sel` to the state bytes base[lo, hi).
+__device__ void stream_apply(uint8_t* base, uint64_t lo, uint64_t hi, Sel sel) {
   if (lo >= hi) return;
-  uint64_t a = (lo + 15) & ~15ull, b = hi & ~15ull;
-  if (a > b) { a = hi; b = hi; }
-  for (uint64_t j = lo + threadIdx.x; j < a; j += RT) __stcg(shadow + j, (uint8_t)sel_apply4(sel, __ldcg(shadow + j)));
-  for (uint64_t j = b + threadIdx.x; j < hi; j += RT) __stcg(shadow + j, (uint8_t)sel_apply4(sel, __ldcg(shadow + j)));
-  uint4* v = reinterpret_cast<uint4*>(shadow + a);
+  // 16-B aligned middle [a, b) of [lo, hi), by address
+  const uintptr_t p0 = reinterpret_cast<uintptr_t>(base + lo), p1 = reinterpret_cast<uintptr_t>(base + hi);
+  const uintptr_t pa = (p0 + 15) & ~(uintptr_t)15, pb = p1 & ~(uintptr_t)15;
+  uint64_t a = hi, b = hi;                       // no aligned middle: all bytes in the head loop
+  if (pa < pb) { a = lo + (pa - p0); b = hi - (p1 - pb); }
+  for (uint64_t j = lo + threadIdx.x; j < a; j += RT) __stcg(base + j, (uint8_t)sel_apply4(sel, __ldcg(base + j)));
+  for (uint64_t j = b + threadIdx.x; j < hi; j += RT) __stcg(base + j, (uint8_t)sel_apply4(sel, __ldcg(base + j)));
+  uint4* v = reinterpret_cast<uint4*>(base + a);
   const uint64_t nv = (b - a) >> 4;
   constexpr int U = 4;   // 4 x 16 B loads in flight per thread
   uint64_t j = threadIdx.x;
@@ -126,7 +137,15 @@ __device__ void apply_ops_before(ReplaySmem& S, const ReplayParams& p, uint32_t 
       ++k2;
     }
     const uint64_t lo = max(o.lo, S.bucket_base + S.part_lo), hi = min(o.hi, S.bucket_base + S.part_hi);
-    stream_apply(p.shadow, lo, hi, sel);
+    if (S.mode == kItemSummary) {
+      // hot slice, phase 1: compose the op into the words' slice functions
+      for (uint64_t j = lo + threadIdx.x; j < hi; j += RT) {
+        const uint32_t w = (uint32_t)(j - S.bucket_base);
+        S.fsum[w] = (uint16_t)sel_compose(sel, S.fsum[w]);
+      }
+    } else if (hi > lo) {
+      stream_apply(S.shrel, lo - S.bucket_base, hi - S.bucket_base, sel);
+    }
     __syncthreads();
     if (threadIdx.x == 0) {
       S.op_cur = k2;
@@ -204,7 +223,7 @@ template <bool PARTIAL>
 __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
   uint32_t slot[RI], word[RI], pos[RI], op[RI], s_pre[RI];
   bool multi = false;
-  const uint8_t* sh = p.shadow + S.bucket_base;
+  const uint8_t* sh = S.shrel;
   uint2* hs = S.u.h.slot;
   uint32_t plo = 0, pw = 0;
   if (PARTIAL) { plo = S.part_lo; pw = S.part_hi - S.part_lo; }
@@ -431,6 +450,7 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
   }
   // blocked arrangement: thread t owns sorted elements [RI*t, RI*t + RI)
   const uint64_t bb = S.bucket_base;
+  uint8_t* const sh = S.shrel;
   uint32_t val[RI], s0[RI], key[RI], wd[RI], ps[RI];
   bool head[RI];
   uint32_t agg = 0;
@@ -445,7 +465,7 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
       uint32_t v = acc_summary(k >> 30);
       uint32_t st = 0;
       if (h) {
-        st = __ldcg(p.shadow + bb + w) & 15u;
+        st = __ldcg(sh + w) & 15u;
         v = kHead | kConst | acc_apply(v, st);
       }
       key[j] = k; head[j] = h; s0[j] = st; val[j] = v; wd[j] = w; ps[j] = pin[i];
@@ -476,13 +496,112 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
       run = acc_combine(run, val[j]);
       fk[j] = classify(key[j] >> 30, before);
       const bool tail = (i + 1 == m) || ((kin[i + 1] & kWordMask) != wd[j]);
-      if (tail) __stcg(p.shadow + bb + wd[j], (uint8_t)(run & 15u));
+      if (tail) __stcg(sh + wd[j], (uint8_t)(run & 15u));
     }
   }
   emit_faults(p, fk, wd, ps, bb);
   __syncthreads();
   hash_clear(S);      // the sort arrays overlap the hash table
   __syncthreads();
+}
+
+// ---- hot bucket slices (K5) ---------------------------------------------------------
+// Phase 1: compose, for every word of the bucket, the transition function of the
+// slice (selector form; reads are identity).  Within a step a word's
+// writes compose to: valid bits of the last write, OVi set if any WH, CVi set if
+// any WT (Table II init bits); the last write of each word (by step
+// index) folds that function into fsum.
+__device__ void step_summary(ReplaySmem& S, const uint2* ev, uint32_t m) {
+  uint32_t* key = S.u.z.key;
+  uint32_t* lastw = S.u.z.lastw;
+  uint32_t* anyw = S.u.z.anyw;
+  uint32_t word[RI], op[RI], idx[RI], slot[RI];
+  bool last[RI];
+  uint32_t ab[RI];
+#pragma unroll
+  for (int j = 0; j < RI; ++j) {
+    const uint32_t i = threadIdx.x + j * RT;
+    op[j] = 4; word[j] = 0; idx[j] = i + 1; slot[j] = 0;
+    if (i < m) {
+      const uint2 e = ev[i];
+      word[j] = e.x & kWordMask; op[j] = e.x >> 30;
+      if (op[j] & 1u) {                // a write: find or insert the word's slot
+        uint32_t h = (word[j] * 2654435761u) >> 21;        // 11 bits
+        for (;;) {
+          const uint32_t old = atomicCAS(&key[h], kEmpty, word[j]);
+          if (old == kEmpty || old == word[j]) break;
+          h = (h + 1) & (kZSlots - 1);
+        }
+        slot[j] = h;
+        atomicMax(&lastw[h], (idx[j] << 2) | op[j]);
+        atomicOr(&anyw[h], op[j] == OP_WH ? 1u : 2u);
+      }
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < RI; ++j) {
+    last[j] = (op[j] & 1u) && (lastw[slot[j]] >> 2) == idx[j];
+    ab[j] = last[j] ? anyw[slot[j]] : 0u;
+  }
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < RI; ++j) {
+    if (last[j]) {
+      const Sel g = op[j] == OP_WH ? sel_make(5, 4, 5, (ab[j] & 2u) ? 5 : 3)     // OV latest; CVi kept unless a WT
+                                   : sel_make(4, 5, (ab[j] & 1u) ? 5 : 2, 5);    // CV latest; OVi kept unless a WH
+      S.fsum[word[j]] = (uint16_t)sel_compose(g, S.fsum[word[j]]);
+      key[slot[j]] = kEmpty;           // the word's only slot: reset by its last writer
+      lastw[slot[j]] = 0;
+      anyw[slot[j]] = 0;
+    }
+  }
+  __syncthreads();
+}
+
+// Position of event e of the bucket (one thread).
+__device__ uint32_t event_pos(const ReplaySmem& S, const ReplayParams& p, uint32_t e) {
+  uint32_t lo = 0, z = S.n_segs;
+  while (z - lo > 1) {
+    const uint32_t mid = (lo + z) >> 1;
+    if (p.segs[S.seg0 + mid].w - S.cum0 <= e) lo = mid; else z = mid;
+  }
+  const uint4 sg = p.segs[S.seg0 + lo];
+  return p.part_ev[(uint64_t)sg.x * kChunkCap + (sg.z & 0xFFFFu) + (e - (sg.w - S.cum0))].y;
+}
+// first op of the bucket (ops [a, z), trace order) at or after position q
+__device__ uint32_t ops_lower_bound(const ReplayParams& p, uint32_t a, uint32_t z, uint32_t q) {
+  while (a < z) {
+    const uint32_t mid = (a + z) >> 1;
+    if (p.ops[mid].pos < q) a = mid + 1; else z = mid;
+  }
+  return a;
+}
+
+// Phase 2: carry the word states across the slices (grid: words x hot buckets).
+__global__ void k_carry(const uint4* hot, const uint64_t* bucket_start, const uint64_t* hot_off,
+                        const uint16_t* hot_F, uint8_t* hot_P, uint8_t* shadow) {
+  const uint4 h = hot[blockIdx.y];
+  const uint32_t b = h.x, slices = h.y, span = h.z, span16 = (span + 15) & ~15u;
+  const uint64_t off = hot_off[b];
+  uint8_t* sh = shadow + bucket_start[b];
+  for (uint32_t w = blockIdx.x * blockDim.x + threadIdx.x; w < span; w += gridDim.x * blockDim.x) {
+    uint32_t st = sh[w];
+    for (uint32_t k = 0; k < slices; ++k) {
+      hot_P[off + (uint64_t)k * span16 + w] = (uint8_t)st;
+      st = sel_apply4(hot_F[off + (uint64_t)k * span16 + w], st) & 15u;
+    }
+    sh[w] = (uint8_t)st;
+  }
+}
+
+cudaError_t launch_carry(const uint4* hot, uint32_t n_hot, uint32_t max_span, const uint64_t* bucket_start,
+                         const uint64_t* hot_off, const uint16_t* hot_F, uint8_t* hot_P, uint8_t* shadow,
+                         cudaStream_t s) {
+  if (!n_hot) return cudaSuccess;
+  const uint32_t gx = std::min<uint32_t>((max_span + 255) / 256, 1024);
+  k_carry<<<dim3(gx, n_hot), 256, 0, s>>>(hot, bucket_start, hot_off, hot_F, hot_P, shadow);
+  return cudaGetLastError();
 }
 
 // ---- the bucket's segments -------------------------------------------------------------
@@ -623,8 +742,11 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       const unsigned long long w = atomicAdd(&p.st->work, 1ull);
       if (w < p.n_items) {
         const uint4 it = p.items[w];
-        S.bucket = it.x; S.part_lo = it.y; S.part_hi = it.z;
-        S.partial = it.w != 0;
+        S.bucket = it.x; S.mode = it.w;
+        S.part_lo = it.w == kItemPart ? it.y : 0;
+        S.part_hi = it.w == kItemPart ? it.z : 0xFFFFFFFFu;
+        S.partial = it.w == kItemPart;
+        S.slice = it.y; S.n_slices = it.z;
       } else {
         S.bucket = 0xFFFFFFFFu;
       }
@@ -632,18 +754,49 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
     __syncthreads();
     const uint32_t b = S.bucket;
     if (b >= p.n_buckets) return;
+    const uint32_t mode = S.mode;
     if (tid == 0) {
       S.op_cur = p.ops_start[b];
       S.op_end = p.ops_start[b + 1];
-      S.next_op = S.op_cur < S.op_end ? p.ops[S.op_cur].pos : 0xFFFFFFFFu;
       S.bucket_base = p.bucket_start[b];
+      S.shrel = p.shadow + S.bucket_base;
     }
     bucket_setup(S, p, b);
-    const uint32_t total = S.n_events;
-    uint32_t e0 = 0, cur = 0, m_cur = 0, hint = 0;
-    if (total) {
-      ensure_window(S, p, 0, hint);
-      m_cur = issue_gather(S, p, 0, total, S.ev[0], hint);
+    uint32_t first = 0, total = S.n_events;
+    if (mode >= kItemSlice) {
+      // hot bucket slice k of n: events [k E / n, (k+1) E / n) and the range ops
+      // from the slice's first event (slice 0: the bucket's first op) up to the
+      // next slice's first event (last slice: the bucket's last op)
+      const uint32_t k = S.slice, ns = S.n_slices, E = S.n_events;
+      const uint32_t span = (uint32_t)(p.bucket_start[b + 1] - p.bucket_start[b]), span16 = (span + 15) & ~15u;
+      first = (uint32_t)((uint64_t)k * E / ns);
+      total = (uint32_t)((uint64_t)(k + 1) * E / ns);
+      if (tid == 0) {
+        const uint32_t a0 = S.op_cur, a1 = S.op_end;
+        if (E == 0) {
+          if (k != 0) S.op_end = a0;
+        } else {
+          if (k > 0) S.op_cur = ops_lower_bound(p, a0, a1, event_pos(S, p, first));
+          if (k + 1 < ns) S.op_end = ops_lower_bound(p, a0, a1, event_pos(S, p, total));
+        }
+        const uint64_t off = p.hot_off[b] + (uint64_t)k * span16;
+        S.shrel = p.hot_P + off;
+        S.fsum = p.hot_F + off;
+        S.part_hi = span;
+      }
+      __syncthreads();
+      if (mode == kItemSummary) {
+        for (uint32_t w = tid; w < span; w += RT) S.fsum[w] = (uint16_t)kSelId;
+        for (uint32_t w = tid; w < kZSlots; w += RT) { S.u.z.key[w] = kEmpty; S.u.z.lastw[w] = 0; S.u.z.anyw[w] = 0; }
+        __syncthreads();
+      }
+    }
+    if (tid == 0) S.next_op = S.op_cur < S.op_end ? p.ops[S.op_cur].pos : 0xFFFFFFFFu;
+    __syncthreads();
+    uint32_t e0 = first, cur = 0, m_cur = 0, hint = 0;
+    if (e0 < total) {
+      ensure_window(S, p, e0, hint);
+      m_cur = issue_gather(S, p, e0, total, S.ev[0], hint);
     }
     while (e0 < total) {
       cp_async_wait_all();
@@ -665,9 +818,13 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         for (uint32_t e = tid; e < m; e += RT) cnt += ev[e].y < S.next_op;
         cut = block_sum(cnt, S.red);
       }
-      const bool fast = S.partial ? step_fast_partial(S, p, ev, cut) : step_fast<false>(S, p, ev, cut);
-      if (!fast) step_sort(S, p, ev, cut);
-      if (tid == 0) atomicAdd(fast ? &p.st->steps_fast : &p.st->steps_sort, 1ull);
+      if (mode == kItemSummary) {
+        step_summary(S, ev, cut);
+      } else {
+        const bool fast = S.partial ? step_fast_partial(S, p, ev, cut) : step_fast<false>(S, p, ev, cut);
+        if (!fast) step_sort(S, p, ev, cut);
+        if (tid == 0) atomicAdd(fast ? &p.st->steps_fast : &p.st->steps_sort, 1ull);
+      }
       e0 += cut;
       if (cut == m) {
         cur ^= 1;
@@ -681,9 +838,14 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         m_cur = issue_gather(S, p, e0, total, S.ev[cur], hint);
       }
     }
-    apply_ops_before(S, p, 0xFFFFFFFFu);
-    if (tid == 0 && total) atomicMax(&p.st->max_bucket_events, (unsigned long long)total);
+    // the ops after the last event (a slice replay's private states are not kept)
+    if (mode != kItemSlice) apply_ops_before(S, p, 0xFFFFFFFFu);
+    if (tid == 0 && total > first) atomicMax(&p.st->max_bucket_events, (unsigned long long)(total - first));
     __syncthreads();
+    if (mode == kItemSummary) {
+      hash_clear(S);                   // the summary arrays share the hash area
+      __syncthreads();
+    }
   }
 }
 

@@ -3,7 +3,8 @@
 // k_sample   sampled histogram of access addresses over coarse bins.
 // k_cut_*    contiguous, event-balanced address buckets: a bucket starts at
 //            bin 0, at every bin whose exclusive sample prefix enters a new
-//            quantile level (a heavy bin gets a bucket of its own) and at every
+//            quantile level or is at least 4 levels heavy (a heavy bin gets a
+//            bucket of its own) and at every
 //            2^30-word span boundary.  The histogram is rewritten in place as
 //            the bin map (bucket | offset-in-bins << kBucketBits, see arb_internal.h).
 //            Tiles of 1024 bins are handled by separate CTAs; two one-CTA
@@ -15,7 +16,14 @@ namespace arb {
 __global__ void k_sample(SampleParams p, uint64_t n_samples) {
   for (uint64_t k = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; k < n_samples;
        k += (uint64_t)gridDim.x * blockDim.x) {
-    const uint4 r = ld_stream(p.ev + k * p.stride);
+    // jittered sampling: record k * stride + (hash(k) mod stride) — a fixed stride
+    // aliases with periodic loop bodies (e.g. one of a stencil's 8 accesses)
+    uint64_t z = k * 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 29)) * 0xBF58476D1CE4E5B9ull;
+    z ^= z >> 32;
+    const uint64_t idx = k * p.stride + (p.stride > 1 ? z % p.stride : 0);
+    if (idx >= p.n) continue;
+    const uint4 r = ld_stream(p.ev + idx);
     const uint64_t w0 = (uint64_t)r.x | ((uint64_t)r.y << 32);
     if (((w0 >> 48) & 0xFFu) >= 4) continue;
     const uint64_t x = (w0 & kMask48) >> 3;
@@ -95,7 +103,8 @@ __global__ void __launch_bounds__(kT) k_cut_scan(uint32_t* v, uint32_t n, uint32
     if (first) {   // quantile target and span cap
       // leave room for the span cuts (n_words / 2^30 + 1 of them, <= 257)
       const uint32_t spans = (uint32_t)(a.n_words >> kMaxBucketSpanBits) + 1;
-      const uint32_t levels = max(1u, a.max_buckets - spans - 1);
+      // heavy-bin buckets (<= levels / 4 of them) need ids as well
+      const uint32_t levels = max(1u, (a.max_buckets - spans - 1) * 4 / 5);
       a.misc[1] = max(1u, (carry + levels - 1) / levels);
       const uint64_t span64 = (1ull << kMaxBucketSpanBits) >> a.coarse_bits;
       a.misc[2] = span64 == 0 ? 1u : (span64 > 0xFFFFFFFFull ? 0xFFFFFFFFu : (uint32_t)span64);
@@ -104,7 +113,7 @@ __global__ void __launch_bounds__(kT) k_cut_scan(uint32_t* v, uint32_t n, uint32
 }
 
 // flags of the bins of one tile (needs the tile's exclusive sample prefix)
-__device__ __forceinline__ bool cut_flag(const CutArgs& a, uint32_t i, uint32_t p, uint32_t h_prev_known,
+__device__ __forceinline__ bool cut_flag(const CutArgs& a, uint32_t i, uint32_t p, uint32_t h, uint32_t h_prev_known,
                                          uint32_t* levs) {
   const uint32_t target = a.misc[1], span = a.misc[2];
   const uint32_t lev = p / target;
@@ -114,7 +123,9 @@ __device__ __forceinline__ bool cut_flag(const CutArgs& a, uint32_t i, uint32_t 
   if (threadIdx.x > 0) prev = levs[threadIdx.x - 1];
   else prev = i == 0 ? 0xFFFFFFFFu : (p - h_prev_known) / target;   // level of the previous tile's last bin
   __syncthreads();
-  return i < a.n_bins && (i == 0 || i % span == 0 || lev != prev);
+  // a very heavy bin (>= 4 levels: a hot word's bin) also starts a bucket of its
+  // own, so the hot bucket spans one bin (the next bin is at a new level)
+  return i < a.n_bins && (i == 0 || i % span == 0 || lev != prev || h >= 4 * target);
 }
 
 __global__ void __launch_bounds__(kT) k_cut_flags(CutArgs a) {
@@ -125,7 +136,7 @@ __global__ void __launch_bounds__(kT) k_cut_flags(CutArgs a) {
   uint32_t tot;
   const uint32_t p = a.tile_a[blockIdx.x] + scan1024(h, ws, &tot);
   const uint32_t hprev = (i > 0 && threadIdx.x == 0) ? a.hist_map[i - 1] : 0;
-  const bool f = cut_flag(a, i, p, hprev, levs);
+  const bool f = cut_flag(a, i, p, h, hprev, levs);
   uint32_t nf;
   scan1024(f ? 1u : 0u, ws, &nf);
   if (threadIdx.x == 0) a.tile_b[blockIdx.x] = nf;
@@ -139,7 +150,7 @@ __global__ void __launch_bounds__(kT) k_cut_write(CutArgs a) {
   uint32_t tot;
   const uint32_t p = a.tile_a[blockIdx.x] + scan1024(h, ws, &tot);
   const uint32_t hprev = (i > 0 && threadIdx.x == 0) ? a.hist_map[i - 1] : 0;
-  const bool f = cut_flag(a, i, p, hprev, levs);
+  const bool f = cut_flag(a, i, p, h, hprev, levs);
   uint32_t nf;
   const uint32_t b = a.tile_b[blockIdx.x] + scan1024(f ? 1u : 0u, ws, &nf);
   if (f) { a.first_bin[b] = i; a.weight[b] = p; }

@@ -45,9 +45,11 @@ def _check_full(orc, prog, flags=0):
     return exp
 
 
-def test_config3_scaled(orc):
+@pytest.mark.parametrize("flags", [0, 4])
+def test_config3_scaled(orc, flags):
+    """flags=4 (ARB_F_SMALL_PARTS): busy small buckets replayed as time slices (K5)."""
     from gen import native
-    exp = _check_full(orc, native.config3(scale=0.01))
+    exp = _check_full(orc, native.config3(scale=0.01), flags=flags)
     kinds = {k for _, _, k in exp.triples()}
     assert kinds == {1, 2, 3}          # alloc-mapped row read, stale `stop`, the missing taskwait
 

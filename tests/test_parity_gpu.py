@@ -82,15 +82,18 @@ def test_config2_split_parts(orc):
     check(orc, rec, base, size, flags=4)
 
 
-def test_hot_word(orc):
-    """One word with ~10^5 events spanning many steps (the bfs `stop` flag shape)."""
+@pytest.mark.parametrize("n,flags", [(100000, 0), (100000, 4), (400000, 0)])
+def test_hot_word(orc, n, flags):
+    """One word with 10^5..4x10^5 events spanning many steps (the bfs `stop` flag
+    shape).  400000 events make the bucket hot (K5: replayed as time slices across
+    CTAs); flags=4 (ARB_F_SMALL_PARTS) forces 3 slices at 10^5."""
     from gen.trace import MAP, OP, TraceBuilder
     tb = TraceBuilder()
     A = 0x8000
     tb.wh(A)
     tb.enter(MAP.TO, A, 64)
     rs = np.random.default_rng(5)
-    ops = rs.choice([OP.RT, OP.WT, OP.RH, OP.WH], size=100000, p=[.4, .2, .3, .1])
+    ops = rs.choice([OP.RT, OP.WT, OP.RH, OP.WH], size=n, p=[.4, .2, .3, .1])
     for chunk in np.array_split(ops, 10):
         arr = np.zeros((chunk.size, 2), dtype=np.uint64)
         arr[:, 0] = np.uint64(A) | (chunk.astype(np.uint64) << np.uint64(48))
@@ -98,7 +101,9 @@ def test_hot_word(orc):
         tb.add_array(arr)
         tb.update(0, A, 64)
     tb.exit(MAP.TOFROM, A, 64)
-    check(orc, tb.array(), A, 64)
+    _, st = check(orc, tb.array(), A, 64, flags=flags)
+    if n > 300000 or flags:
+        assert st["hot_buckets"] >= 1
 
 
 def test_multi_flush_quiescent(orc):
