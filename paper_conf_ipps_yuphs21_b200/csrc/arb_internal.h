@@ -42,6 +42,7 @@ constexpr int kSegChunkBits = 21;                    // chunk id bits in the ent
 
 // ---- partition geometry ----------------------------------------------------
 constexpr int kPartThreads = 512;
+constexpr int kPartStages = 2;
 constexpr int kPartWarps = kPartThreads / 32;
 constexpr int kChunkRecords = 256;                  // records per chunk (one warp, independently)
 constexpr int kChunkCap = 2 * kChunkRecords;        // events per chunk (<= 2 words per access)

@@ -25,11 +25,12 @@ constexpr int PW = kPartWarps;              // 16 warps
 constexpr int WREC = kChunkRecords;         // 256 records per chunk
 constexpr int RPL = WREC / 32;              // 8 records per lane (two groups of 4 x 32)
 constexpr int kSegBuf = 64;                 // segment entries buffered per warp
+constexpr int NST = kPartStages;            // chunks staged per warp (prefetch distance NST - 1)
 
-// per-warp shared memory: stage[2][WREC] uint4, segbuf[kSegBuf] uint2,
+// per-warp shared memory: stage[NST][WREC] uint4, segbuf[kSegBuf] uint2,
 // tlist[2 * WREC] u16, row[NB] u16 (padded to 16 B)
 __host__ __device__ constexpr size_t warp_smem_bytes(uint32_t nb) {
-  return sizeof(uint4) * 2 * WREC + sizeof(uint2) * kSegBuf + 2 * (2 * WREC) + (((size_t)nb * 2 + 15) & ~(size_t)15);
+  return sizeof(uint4) * NST * WREC + sizeof(uint2) * kSegBuf + 2 * (2 * WREC) + (((size_t)nb * 2 + 15) & ~(size_t)15);
 }
 
 // Decoded record: info = cnt | b0 << 2 | b1 << kB1Shift (cnt = tracked words 0..2),
@@ -156,7 +157,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   const uint32_t lt = lanemask_lt();
   uint8_t* wbase = smem + warp * warp_smem_bytes(NB);
   uint4* stage = reinterpret_cast<uint4*>(wbase);                   // [2][WREC]
-  uint2* segbuf = reinterpret_cast<uint2*>(stage + 2 * WREC);       // [kSegBuf]
+  uint2* segbuf = reinterpret_cast<uint2*>(stage + NST * WREC);     // [kSegBuf]
   uint16_t* tlist = reinterpret_cast<uint16_t*>(segbuf + kSegBuf);   // [2 * WREC]
   uint16_t* row = tlist + 2 * WREC;                                  // [NB]
   for (uint32_t i = lane; i < NB; i += 32) row[i] = 0;
@@ -189,11 +190,12 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   const uint64_t nwarps = (uint64_t)gridDim.x * PW;
   uint32_t cur = 0;
   uint64_t chunk = (uint64_t)blockIdx.x * PW + warp;
-  fetch(chunk, stage);
+#pragma unroll
+  for (int k = 0; k < NST - 1; ++k) fetch(chunk + k * nwarps, stage + k * WREC);
   __syncwarp();
   for (; chunk < p.n_chunks; chunk += nwarps) {
-    fetch(chunk + nwarps, stage + (cur ^ 1) * WREC);
-    cp_async_wait_group<1>();
+    fetch(chunk + (NST - 1) * nwarps, stage + (cur == 0 ? NST - 1 : cur - 1) * WREC);
+    cp_async_wait_group<NST - 1>();
     __syncwarp();
     const uint4* st = stage + cur * WREC;
     const uint64_t rec0 = chunk * WREC;
@@ -206,7 +208,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     if (nvalid == WREC && fast_chunk(st, p, (uint32_t)rec0, (uint32_t)chunk, p.part_ev + chunk * kChunkCap,
                                      segbuf, nbuf, lane)) {
       n_acc += RPL;
-      cur ^= 1;
+      cur = cur + 1 == NST ? 0 : cur + 1;
       __syncwarp();                    // stage[cur] reads done before the next fetch overwrites it
       continue;
     }
@@ -361,7 +363,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     __syncwarp();
     for (uint32_t t = lane; t < nT; t += 32) row[tlist[t]] = 0;
     n_acc += e_lane;
-    cur ^= 1;
+    cur = cur + 1 == NST ? 0 : cur + 1;
     __syncwarp();                      // stage[cur] reads and row resets done before reuse
   }
   cp_async_wait_all();
