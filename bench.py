@@ -347,10 +347,20 @@ def main():
         traffic = tj["dram_bytes_per_launch"] / tj["records_in_launch"] * s0["records"] / len(flushes)
     except Exception:
         pass
+    kern = {}
+    for k in ("k_partition", "k_replay"):
+        ach = alg[k] / (phases[k] / 1e3) / 1e9 if phases[k] > 0 else 0.0
+        kern[k] = {"ms_per_step": phases[k], "alg_bytes_per_step": alg[k], "achieved": ach, "frac": ach / hbm_gbs}
+        try:
+            with open(os.path.join(ROOT, "profiles", "traffic.json")) as fh:
+                tk = json.load(fh)[k]
+            kern[k]["ncu_dram_bytes_per_record"] = tk["dram_bytes_per_launch"] / tk["records_in_launch"]
+        except Exception:
+            pass
     roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": hbm_gbs, "unit": "GB/s",
             "frac": achieved / hbm_gbs, "traffic": traffic, "traffic_unit": "bytes per launch (ncu)",
             "alg_bytes_per_launch": alg[dom] / len(flushes), "peak_source": peak_src,
-            "kernel_ms_per_step": phases[dom], "phase_ms_per_step": phases,
+            "kernel_ms_per_step": phases[dom], "phase_ms_per_step": phases, "kernels": kern,
             "path": {"b_alg_bytes_per_step": b_alg, "achieved": b_alg / (ms_per_step / 1e3) / 1e9,
                      "frac": b_alg / (ms_per_step / 1e3) / 1e9 / hbm_gbs}}
 
