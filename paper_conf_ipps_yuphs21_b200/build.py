@@ -27,7 +27,7 @@ def _stale(out, deps):
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
-    deps = sources() + glob.glob(os.path.join(CSRC, "*.h")) + [os.path.join(INCLUDE, "arbalest.h"), __file__]
+    deps = sources() + glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(CSRC, "*.cuh")) + [os.path.join(INCLUDE, "arbalest.h"), __file__]
     if not force and not _stale(LIB, deps):
         return LIB
     objdir = os.path.join(PKG, "build")

@@ -3,8 +3,8 @@
 // k_partition  persistent CTAs (one per SM, 16 warps).  Every warp works on its
 //              own 256-record chunks with no block-level synchronisation: the
 //              chunk's 16-B records are staged in the warp's shared memory by
-//              cp.async (double-buffered: the next chunk streams in while the
-//              current one is processed).  Lane L decodes records L, L+32, ...
+//              one TMA bulk copy completing on an mbarrier (double-buffered: the
+//              next chunk streams in while the current one is processed).  Lane L decodes records L, L+32, ...
 //              (access vs control; byte range -> its 1 or 2 8-byte words, P:267;
 //              word -> address bucket via the bin map) in two groups of 128, and
 //              each group is ranked stably into the warp's per-bucket counters —
@@ -28,9 +28,10 @@ constexpr int kSegBuf = 64;                 // segment entries buffered per warp
 constexpr int NST = kPartStages;            // chunks staged per warp (prefetch distance NST - 1)
 
 // per-warp shared memory: stage[NST][WREC] uint4, segbuf[kSegBuf] uint2,
-// tlist[2 * WREC] u16, row[NB] u16 (padded to 16 B)
+// tlist[2 * WREC] u16, row[NB] u16 (padded to 16 B), bar[NST] u64 (padded to 16 B)
 __host__ __device__ constexpr size_t warp_smem_bytes(uint32_t nb) {
-  return sizeof(uint4) * NST * WREC + sizeof(uint2) * kSegBuf + 2 * (2 * WREC) + (((size_t)nb * 2 + 15) & ~(size_t)15);
+  return sizeof(uint4) * NST * WREC + sizeof(uint2) * kSegBuf + 2 * (2 * WREC) + (((size_t)nb * 2 + 15) & ~(size_t)15) +
+         ((8 * NST + 15) & ~15);
 }
 
 // Decoded record: info = cnt | b0 << 2 | b1 << kB1Shift (cnt = tracked words 0..2),
@@ -117,32 +118,46 @@ __device__ __forceinline__ void rank_round(uint32_t info, uint16_t* row, uint16_
   r1 = r0 + 1;
 }
 
-// The fast chunk test and its output.  One check per record: an access (op < 4)
+// The fast chunk test and its output.  Every record must be an access (op < 4)
 // of 1..8 bytes inside one 8-byte word (such an access cannot leave the
-// 48-bit space) whose word is tracked; then every word must map to the bucket of
-// record 0.  Returns false (nothing written) when any record fails.
-__device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p, uint32_t rec0, uint32_t chunk,
-                                           uint2* out, uint2* segbuf, uint32_t& nbuf, uint32_t lane) {
-  const uint32_t cb = p.coarse_bits, cmask = (1u << cb) - 1u;
-  uint32_t key[RPL], b0 = 0;
-  bool ok = true;
+// 48-bit space), and all words must lie in one address bucket.  Buckets are
+// contiguous word ranges, so the test needs only the chunk's lowest and highest
+// word: each word is taken relative to record 0's word w0 (32-bit signed,
+// |d| < 2^30 as a bucket spans <= 2^30 words), the warp reduces min and max, and
+// two bin-map lookups decide.  A word's offset in the bucket is then
+// off(lowest) + d - dmin.  Returns false (nothing written) when the test fails.
+__device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p, uint32_t chunk, uint2* out,
+                                           uint2* segbuf, uint32_t& nbuf, uint32_t lane) {
+  const uint4 q0 = st[0];
+  const uint64_t w0 = ((uint64_t)((q0.y & 0xFFFFu) >> 3) << 32) | __funnelshift_r(q0.x, q0.y, 3);
+  uint32_t d[RPL], opk[RPL], bad = 0;
+  int32_t dmin = 0, dmax = 0;
 #pragma unroll
   for (int k = 0; k < RPL; ++k) {
     const uint4 q = st[k * 32 + lane];
-    const uint32_t bad = (q.y & 0x00FC0000u) | (q.w & 0xFFFFu) | ((q.z - 1u) & ~7u) | (((q.x & 7u) + q.z - 1u) & ~7u);
+    bad |= (q.y & 0x00FC0000u) | (q.w & 0xFFFFu) | ((q.z - 1u) & ~7u) | (((q.x & 7u) + q.z - 1u) & ~7u);
     const uint64_t word = ((uint64_t)((q.y & 0xFFFFu) >> 3) << 32) | __funnelshift_r(q.x, q.y, 3);
-    const uint64_t rel = word - p.base_word;
-    const bool okk = bad == 0 && rel < p.n_words;
-    const uint32_t m = okk ? __ldg(p.bin_map + (uint32_t)(rel >> cb)) : 0xFFFFFFFFu;
-    const uint32_t b = m & kBucketMask;
-    if (k == 0) b0 = b;
-    ok = ok && okk && b == b0;
-    key[k] = (((q.y >> 16) & 3u) << 30) | ((m >> kBucketBits) << cb) | ((uint32_t)rel & cmask);
+    const uint64_t diff = word - w0;
+    bad |= (uint32_t)((diff + (1ull << 30)) >> 31);      // d outside [-2^30, 2^30)
+    d[k] = (uint32_t)diff;
+    dmin = min(dmin, (int32_t)d[k]);
+    dmax = max(dmax, (int32_t)d[k]);
+    opk[k] = ((q.y >> 16) & 3u) << 30;
   }
-  const uint32_t bref = __shfl_sync(FULL, b0, 0);
-  if (!__all_sync(FULL, ok && b0 == bref)) return false;
+  if (!__all_sync(FULL, bad == 0)) return false;
+  dmin = __reduce_min_sync(FULL, dmin);
+  dmax = __reduce_max_sync(FULL, dmax);
+  const uint64_t rlo = w0 - p.base_word + (uint64_t)(int64_t)dmin;   // wraps below the range
+  const uint64_t rhi = w0 - p.base_word + (uint64_t)(int64_t)dmax;
+  if (rlo >= p.n_words || rhi >= p.n_words) return false;
+  const uint32_t cb = p.coarse_bits;
+  const uint32_t mlo = __ldg(p.bin_map + (uint32_t)(rlo >> cb)), mhi = __ldg(p.bin_map + (uint32_t)(rhi >> cb));
+  const uint32_t bref = mlo & kBucketMask;
+  if (bref != (mhi & kBucketMask)) return false;
+  const uint32_t c = (((mlo >> kBucketBits) << cb) | ((uint32_t)rlo & ((1u << cb) - 1u))) - (uint32_t)dmin;
+  const uint32_t rec0 = chunk * (uint32_t)WREC;
 #pragma unroll
-  for (int k = 0; k < RPL; ++k) out[k * 32 + lane] = make_uint2(key[k], rec0 + k * 32 + lane);
+  for (int k = 0; k < RPL; ++k) out[k * 32 + lane] = make_uint2(opk[k] | (d[k] + c), rec0 + k * 32 + lane);
   if (lane == 0)
     segbuf[nbuf] = make_uint2((bref << kSegChunkBits) | (chunk & ((1u << kSegChunkBits) - 1u)),
                               (uint32_t)WREC << 16 | ((chunk >> kSegChunkBits) << 31));
@@ -160,21 +175,22 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   uint2* segbuf = reinterpret_cast<uint2*>(stage + NST * WREC);     // [kSegBuf]
   uint16_t* tlist = reinterpret_cast<uint16_t*>(segbuf + kSegBuf);   // [2 * WREC]
   uint16_t* row = tlist + 2 * WREC;                                  // [NB]
+  uint64_t* bar = reinterpret_cast<uint64_t*>(row + ((NB + 7) & ~7u));   // [NST]
   for (uint32_t i = lane; i < NB; i += 32) row[i] = 0;
-  uint32_t n_acc = 0, n_ign = 0, nbuf = 0;
+  if (lane < NST) mbar_init(bar + lane, 1);
+  fence_mbar_init();
+  __syncwarp();
+  uint32_t n_acc = 0, n_ign = 0, nbuf = 0, phase = 0;   // phase: parity bit of each stage's barrier
 
-  auto fetch = [&](uint64_t c, uint4* dst) {
-    if (c < p.n_chunks) {
+  // the chunk's records arrive in stage k by one TMA bulk copy (lane 0) that
+  // completes on bar[k]
+  auto fetch = [&](uint64_t c, uint32_t k) {
+    if (c < p.n_chunks && lane == 0) {
       const uint64_t r0 = c * WREC;
       const uint32_t nv = p.n - r0 < (uint64_t)WREC ? (uint32_t)(p.n - r0) : (uint32_t)WREC;
-      const uint4* src = p.ev + r0;
-#pragma unroll
-      for (int k = 0; k < RPL; ++k) {
-        const uint32_t j = lane + k * 32;
-        if (j < nv) cp_async16(dst + j, src + j);
-      }
+      mbar_arrive_tx(bar + k, nv * 16u);
+      bulk_g2s(stage + k * WREC, p.ev + r0, nv * 16u, bar + k);
     }
-    cp_async_commit();                 // possibly empty: keeps the group count uniform
   };
   auto flush_segs = [&]() {
     __syncwarp();
@@ -191,12 +207,11 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   uint32_t cur = 0;
   uint64_t chunk = (uint64_t)blockIdx.x * PW + warp;
 #pragma unroll
-  for (int k = 0; k < NST - 1; ++k) fetch(chunk + k * nwarps, stage + k * WREC);
-  __syncwarp();
+  for (int k = 0; k < NST - 1; ++k) fetch(chunk + k * nwarps, k);
   for (; chunk < p.n_chunks; chunk += nwarps) {
-    fetch(chunk + (NST - 1) * nwarps, stage + (cur == 0 ? NST - 1 : cur - 1) * WREC);
-    cp_async_wait_group<NST - 1>();
-    __syncwarp();
+    fetch(chunk + (NST - 1) * nwarps, cur == 0 ? NST - 1 : cur - 1);
+    mbar_wait(bar + cur, (phase >> cur) & 1u);
+    phase ^= 1u << cur;
     const uint4* st = stage + cur * WREC;
     const uint64_t rec0 = chunk * WREC;
     const uint32_t nvalid = p.n - rec0 < (uint64_t)WREC ? (uint32_t)(p.n - rec0) : (uint32_t)WREC;
@@ -205,7 +220,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     // keep record order, so event j is record j: one coalesced store per record and
     // one segment entry for the chunk.  Anything else takes the general path below.
     if (nbuf == kSegBuf) flush_segs();
-    if (nvalid == WREC && fast_chunk(st, p, (uint32_t)rec0, (uint32_t)chunk, p.part_ev + chunk * kChunkCap,
+    if (nvalid == WREC && fast_chunk(st, p, (uint32_t)chunk, p.part_ev + chunk * kChunkCap,
                                      segbuf, nbuf, lane)) {
       n_acc += RPL;
       cur = cur + 1 == NST ? 0 : cur + 1;
@@ -366,7 +381,6 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     cur = cur + 1 == NST ? 0 : cur + 1;
     __syncwarp();                      // stage[cur] reads and row resets done before reuse
   }
-  cp_async_wait_all();
   flush_segs();
 
 #pragma unroll
