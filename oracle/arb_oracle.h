@@ -27,6 +27,9 @@
  *   MIR attribution to later event (Z11)  parity unpinned (definition only)
  *   dedup-first mode (Z3)                 parity unpinned (definition only)
  *   sub-word semantics (Z4)               parity unpinned (definition only)
+ *   buffer overflow, present-bit form (Z17) pinned (P:279 worked example + brute force vs the
+ *                                         value simulator's CV existence); the paper's base-interval
+ *                                         comparison (overflow into ANOTHER mapped CV) is not modelled
  */
 #ifndef ARB_ORACLE_H
 #define ARB_ORACLE_H
@@ -51,8 +54,8 @@ enum { ORC_TO = 0, ORC_FROM = 1, ORC_TOFROM = 2, ORC_ALLOC = 3,
 /* update direction */
 enum { ORC_UPD_TO = 0, ORC_UPD_FROM = 1 };
 #define ORC_SYNC_ALL 0xFFFFu
-/* report kinds */
-enum { ORC_UUM = 1, ORC_USD = 2, ORC_MIR = 3 };
+/* report kinds (BO: P:277-281) */
+enum { ORC_UUM = 1, ORC_USD = 2, ORC_MIR = 3, ORC_BO = 4 };
 /* status codes (same values as the library's, restated) */
 enum { ORC_OK = 0, ORC_EINVAL = -1, ORC_ENOMEM = -2, ORC_EMAP = -4,
        ORC_ETRACE = -5, ORC_EOPEN = -7 };
@@ -74,6 +77,12 @@ typedef struct {
    * (tracked_words == NULL) tracks every word of the range (Z12). */
   const uint64_t* tracked_words;
   uint64_t        n_tracked;
+  /* Buffer-overflow extension (reading Z17 of DESIGN.md): a 5th
+   * state bit CVp ("the word has a CV") is set by allocate and cleared by
+   * release; a target access (RT/WT) to a word without a CV is reported as
+   * ORC_BO and has no VSM effect (no UUM/USD check, no transition: the access
+   * did not touch this word's CV).  0 = off (the 4-bit VSM of P:255-263). */
+  int             detect_bo;
 } orc_config;
 
 typedef struct {
@@ -91,7 +100,8 @@ typedef struct {
  * order (word, record, kind ascending) that the caller frees with
  * orc_free(); shadow_out (dense: addr_bytes/8 bytes, sparse: n_tracked
  * bytes, may be NULL) receives the final states (bit0 OVv, bit1 CVv,
- * bit2 OVi, bit3 CVi — Table II).  Returns ORC_OK or an error. */
+ * bit2 OVi, bit3 CVi — Table II; bit4 CVp with detect_bo).
+ * Returns ORC_OK or an error. */
 int  orc_replay(const orc_config* cfg, const orc_record* rec, uint64_t n,
                 const uint64_t* global_index, orc_report** out, uint64_t* n_out,
                 uint8_t* shadow_out, orc_stats* stats);

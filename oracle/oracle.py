@@ -19,14 +19,14 @@ _SRC = os.path.join(_HERE, "arb_oracle.c")
 _HDR = os.path.join(_HERE, "arb_oracle.h")
 _LIB = os.path.join(_HERE, "liboracle.so")
 
-KIND_NAMES = {1: "UUM", 2: "USD", 3: "MIR"}
+KIND_NAMES = {1: "UUM", 2: "USD", 3: "MIR", 4: "BO"}
 
 
 class _Config(ctypes.Structure):
     _fields_ = [("addr_base", ctypes.c_uint64), ("addr_bytes", ctypes.c_uint64),
                 ("dedup_first", ctypes.c_int),
                 ("tracked_words", ctypes.POINTER(ctypes.c_uint64)),
-                ("n_tracked", ctypes.c_uint64)]
+                ("n_tracked", ctypes.c_uint64), ("detect_bo", ctypes.c_int)]
 
 
 class _Stats(ctypes.Structure):
@@ -80,8 +80,9 @@ class OracleResult:
 
 def replay(records: np.ndarray, addr_base: int, addr_bytes: int, *, dedup_first: bool = False,
            tracked_words: np.ndarray | None = None, global_index: np.ndarray | None = None,
-           want_shadow: bool = True) -> OracleResult:
-    """Replay ``records`` (uint64 array of shape (n, 2): w0, w1) through the oracle."""
+           want_shadow: bool = True, detect_bo: bool = False) -> OracleResult:
+    """Replay ``records`` (uint64 array of shape (n, 2): w0, w1) through the oracle.
+    ``detect_bo``: the buffer-overflow extension (reading Z17)."""
     lib = _load()
     rec = np.ascontiguousarray(records, dtype=np.uint64).reshape(-1, 2)
     n = rec.shape[0]
@@ -89,6 +90,7 @@ def replay(records: np.ndarray, addr_base: int, addr_bytes: int, *, dedup_first:
     cfg.addr_base = addr_base
     cfg.addr_bytes = addr_bytes
     cfg.dedup_first = 1 if dedup_first else 0
+    cfg.detect_bo = 1 if detect_bo else 0
     tw = None
     if tracked_words is not None:
         tw = np.ascontiguousarray(tracked_words, dtype=np.uint64)

@@ -45,14 +45,15 @@ def encode_seq(seq, base):
     return out
 
 
-def check_batch(orc, seqs, nwords):
-    """Concatenate the sequences on disjoint arrays, run the oracle once, compare per array."""
+def check_batch(orc, seqs, nwords, bo=False):
+    """Concatenate the sequences on disjoint arrays, run the oracle once, compare per array.
+    bo: the buffer-overflow extension on both sides (reading Z17)."""
     stride = 8 * nwords
     recs, expect, states, offsets = [], [], [], []
     for j, seq in enumerate(seqs):
         base = stride * j
         enc = encode_seq(seq, base)
-        vs = ValueSim()
+        vs = ValueSim(bo=bo)
         try:
             issues = vs.run(enc)
         except MapError:
@@ -64,7 +65,7 @@ def check_batch(orc, seqs, nwords):
         states.extend(vs.state_bits(base // 8 + w) for w in range(nwords))
     arr = np.array(recs, dtype=np.uint64).reshape(-1, 2)
     nseq = len(offsets)
-    res = orc.replay(arr, 0, stride * (len(seqs)))
+    res = orc.replay(arr, 0, stride * (len(seqs)), detect_bo=bo)
     assert res.rc == 0
     assert res.triples() == sorted(expect)
     # final states: only the arrays that were kept
@@ -136,3 +137,21 @@ def test_one_word_len6_reduced(orc):
     seqs = list(itertools.product(keep, repeat=6))
     for k in range(0, len(seqs), 250000):
         check_batch(orc, seqs[k:k + 250000], 1)
+
+
+@pytest.mark.parametrize("nwords,length", [(1, 4), (2, 3)])
+def test_bo_exhaustive(orc, nwords, length):
+    """Buffer-overflow extension (Z17): the oracle's CVp bit and BO
+    reports equal the value simulator's CV existence on every sequence (target
+    accesses before any map, after release/delete, outside a 1-word section of
+    a 2-word array), together with the UUM/USD reports and final states."""
+    sym = alphabet(nwords)
+    seqs = [s for L in range(1, length + 1) for s in itertools.product(sym, repeat=L)]
+    assert check_batch(orc, seqs, nwords, bo=True) > 50000
+
+
+def test_bo_random_long(orc):
+    sym = alphabet(2)
+    rs = np.random.default_rng(13)
+    seqs = [tuple(sym[i] for i in rs.integers(0, len(sym), rs.integers(4, 9))) for _ in range(40000)]
+    check_batch(orc, seqs, 2, bo=True)

@@ -268,3 +268,66 @@ def test_global_index(orc):
     gi = np.arange(rec.shape[0], dtype=np.uint64) * 10 + 7
     res = run(orc, rec, base, size, global_index=gi)
     assert res.triples() == [(w, r * 10 + 7, k) for w, r, k in expect]
+
+
+# ---- buffer-overflow extension (reading Z17) -----------------------
+BO = 4
+
+
+def _half_mapped(n, write):
+    """"the host program only maps the first half of an array to the
+    accelerator, while the compute kernel loops through the whole array"."""
+    A = 0x4000
+    tb = TraceBuilder()
+    tb.loop([(OP.WH, A)], n, 8)                       # host initialises a[0:n]
+    tb.enter(MAP.TOFROM, A, 8 * (n // 2))             # map(tofrom: a[0:n/2])
+    k0 = len(tb)
+    tb.loop([(OP.WT if write else OP.RT, A)], n, 8)   # kernel: for i < n: a[i] (= or read)
+    tb.exit(MAP.TOFROM, A, 8 * (n // 2))
+    return tb.array(), A, k0
+
+
+@pytest.mark.parametrize("write", [False, True])
+def test_bo_half_mapped_array(orc, write):
+    n = 64
+    rec, A, k0 = _half_mapped(n, write)
+    res = run(orc, rec, A, 8 * n, detect_bo=True)
+    # exactly the kernel accesses of the unmapped half, nothing else
+    assert res.triples() == [(A // 8 + i, k0 + i, BO) for i in range(n // 2, n)]
+    assert res.stats["transitions"] == res.stats["word_events"]
+    # the overflowing accesses had no effect: the unmapped half's OV still holds
+    # the host values (OVv, OVi) and it never had a CV; the mapped half was copied
+    # back at the tofrom exit and its CV released (CVp clear): OVv | OVi everywhere
+    assert set(res.shadow.tolist()) == {0b0101}
+    # without the extension the reads of the unmapped half are UUM (no CV value) and the
+    # writes are silent (P:263 only checks reads)
+    plain = run(orc, rec, A, 8 * n).triples()
+    assert plain == ([] if write else [(A // 8 + i, k0 + i, UUM) for i in range(n // 2, n)])
+
+
+def test_bo_fixed_mapping_is_clean(orc):
+    """The fixed program maps the whole array: no report with or without the extension."""
+    A, n = 0x4000, 64
+    tb = TraceBuilder()
+    tb.loop([(OP.WH, A)], n, 8)
+    tb.enter(MAP.TOFROM, A, 8 * n)
+    tb.loop([(OP.RT, A), (OP.WT, A)], n, 8)
+    tb.exit(MAP.TOFROM, A, 8 * n)
+    tb.loop([(OP.RH, A)], n, 8)
+    res = run(orc, tb.array(), A, 8 * n, detect_bo=True)
+    assert res.triples() == []
+
+
+def test_bo_after_release_and_host_unaffected(orc):
+    """A kernel access after the CV was deleted is BO; host accesses never are."""
+    A = 0x4000
+    tb = TraceBuilder()
+    tb.wh(A)
+    tb.enter(MAP.TO, A, 8)
+    i_ok = tb.rt(A)
+    tb.exit(MAP.DELETE, A, 8)
+    i_bo = tb.rt(A)
+    i_h = tb.rh(A)
+    res = run(orc, tb.array(), A, 8, detect_bo=True)
+    assert res.triples() == [(A // 8, i_bo, BO)]
+    assert i_ok < i_bo < i_h

@@ -24,7 +24,7 @@ BOT = 0  # undefined content
 RH, WH, RT, WT, MAP_ENTER, MAP_EXIT, UPDATE = 0, 1, 2, 3, 8, 9, 10
 TASK_BEGIN, TASK_END, SYNC = 12, 13, 14
 TO, FROM, TOFROM, ALLOC, RELEASE, DELETE = 0, 1, 2, 3, 4, 5
-UUM, USD = 1, 2
+UUM, USD, BO = 1, 2, 4
 
 
 class MapError(Exception):
@@ -32,7 +32,14 @@ class MapError(Exception):
 
 
 class ValueSim:
-    def __init__(self):
+    """bo=True: the buffer-overflow extension: a target access to a
+    word whose CV does not exist (no map entry created it, or it was deleted)
+    does not reach this word's CV at all; it is reported as BO and changes
+    nothing.  CV existence is tracked as a set of words here, not as a bit."""
+
+    def __init__(self, bo: bool = False):
+        self.bo = bo
+        self.alive: set[int] = set()      # words whose CV exists
         self.ov: dict[int, int] = {}
         self.cv: dict[int, int] = {}
         self.latest: dict[int, int] = {}
@@ -54,6 +61,9 @@ class ValueSim:
             self.issues.add((w, idx, UUM if got == BOT else USD))
 
     def word_op(self, name, w, idx):
+        if self.bo and name in ("RT", "WT") and w not in self.alive:
+            self.issues.add((w, idx, BO))
+            return
         if name == "RH":
             self._read(self.ov, w, idx)
         elif name == "RT":
@@ -68,6 +78,10 @@ class ValueSim:
             self.ov[w] = self.cv.get(w, BOT)
         elif name in ("NEW", "DEL"):  # fresh or deleted CV holds nothing
             self.cv[w] = BOT
+            if name == "NEW":
+                self.alive.add(w)
+            else:
+                self.alive.discard(w)
         else:
             raise ValueError(name)
 
@@ -137,7 +151,8 @@ class ValueSim:
         cv = self.cv.get(w, BOT)
         ovv = lat is not None and ov == lat
         cvv = lat is not None and cv == lat
-        return int(ovv) | (int(cvv) << 1) | (int(ov != BOT) << 2) | (int(cv != BOT) << 3)
+        bits = int(ovv) | (int(cvv) << 1) | (int(ov != BOT) << 2) | (int(cv != BOT) << 3)
+        return bits | (int(w in self.alive) << 4 if self.bo else 0)
 
 
 def schedule_issues(ops):
