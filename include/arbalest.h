@@ -52,7 +52,8 @@ enum arb_upd { ARB_UPD_TO = 0, ARB_UPD_FROM = 1 };
 #define ARB_SYNC_ALL 0xFFFFu
 
 /* ---- reports ---------------------------------------------------------------- */
-enum arb_kind { ARB_UUM = 1, ARB_USD = 2, ARB_MIR = 3 };
+enum arb_kind { ARB_UUM = 1, ARB_USD = 2, ARB_MIR = 3,
+                ARB_BO = 4  /* buffer overflow, with ARB_F_BO only (Z17) */ };
 /* w0: [0,48) absolute word index (= byte address / 8) | [48,56) kind
  * w1: global record index (0-based; see arb_submit_events)
  * Canonical order: word, then record, then kind, ascending; no duplicates. */
@@ -82,6 +83,11 @@ enum arb_status {
                                    replay every small bucket with >= 64 events as 3 time
                                    slices (the mechanisms normally used for range-heavy
                                    and hot buckets only)                                  */
+#define ARB_F_BO          0x8u  /* buffer-overflow extension (reading Z17): every
+                                   word carries a 5th state bit "has a CV" (set by allocate,
+                                   cleared by release); a target access (RT/WT) to a word
+                                   without a CV is reported as ARB_BO and has no VSM effect.
+                                   Hot buckets are then replayed whole (no time slices).  */
 
 typedef struct {
   uint64_t addr_base;        /* tracked OV byte range [addr_base, addr_base+addr_bytes);   */
@@ -121,6 +127,7 @@ typedef struct {
   double   ms_host_control;  /* host wall time of the Table I / task resolution             */
   uint64_t work_items;       /* replay work items (buckets, word-range parts, hot slices)   */
   uint64_t hot_buckets;      /* buckets replayed as time slices (hot words, K5)             */
+  uint64_t reports_bo;       /* reports of kind ARB_BO in the last flush (ARB_F_BO)         */
 } arb_stats;
 
 typedef struct arb_ctx_s* arb_ctx;

@@ -216,7 +216,7 @@ extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
   if (e != cudaSuccess) { delete ctx; return ARB_ENOMEM; }
   e = cudaMemset(ctx->shadow, 0, ctx->n_words);                 // all invalid
   if (e == cudaSuccess) e = ctx->dstats.ensure(1);
-  if (e == cudaSuccess) e = ctx->dcount.ensure(4);
+  if (e == cudaSuccess) e = ctx->dcount.ensure(8);
   if (e == cudaSuccess) e = ctx->ctl.ensure(ctx->ctl_cap);
   for (int i = 0; i < 10 && e == cudaSuccess; ++i) e = cudaEventCreate(&ctx->ev[i]);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->aux, cudaStreamNonBlocking);
@@ -363,6 +363,7 @@ static void build_items(arb_ctx ctx, const FlushPlan& plan, const std::vector<do
     const uint64_t span = ctx->bucket_start[b + 1] - ctx->bucket_start[b];
     const double ev = bucket_events[b];
     if (parts[b] != 1 || span > kHotSpan) continue;
+    if (ctx->cfg.flags & ARB_F_BO) continue;      // slice functions cannot express the BO condition (Z17)
     const bool hot = force_hot ? ev >= 64.0 : (ev > 1.25 * share && ev > kSliceEvents);
     if (!hot) continue;
     const double want = force_hot ? 3.0 : std::ceil(ev / kSliceEvents);
@@ -570,7 +571,8 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   }
   MapTable map = ctx->map;
   FlushPlan plan;
-  resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_start, map, plan);
+  resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_start, map, plan,
+                  (ctx->cfg.flags & ARB_F_BO) != 0);
   if (plan.rc != 0) {
     CK(cudaStreamSynchronize(s), "sync");
     reset_batch(ctx);
@@ -603,7 +605,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   rp.n_buckets = ctx->n_buckets; rp.bucket_bits = ctx->bucket_bits; rp.n_words = ctx->n_words;
   rp.bucket_start = ctx->d_bucket_start.p;
   rp.items = ctx->d_items.p; rp.n_items = (uint32_t)ctx->items.size();
-  rp.shadow = ctx->shadow; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
+  rp.shadow = ctx->shadow; rp.bo = (ctx->cfg.flags & ARB_F_BO) ? 1u : 0u; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
   rp.cand = ctx->cand.p; rp.cand_cap = ctx->cand_cap; rp.st = ctx->dstats.p;
   rp.hot_off = ctx->d_hot_off.p; rp.hot_F = ctx->hot_F.p; rp.hot_P = ctx->hot_P.p;
   int n_ctas = std::max(1, std::min<int>((int)ctx->items.size(), ctx->n_sms * kReplayCtasPerSm));
@@ -694,13 +696,14 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   cp.gidx = gidx; cp.index_base = index_base;
   cp.out = ctx->reports.p; cp.n_out = ctx->dcount.p;
   CK(launch_compact(cp, s, &launches), "compact");
-  unsigned long long cnt4[4] = {0, 0, 0, 0};
+  unsigned long long cnt4[8] = {0, 0, 0, 0, 0, 0, 0, 0};   // [0] total, [k] kind k
   CK(cudaMemcpyAsync(cnt4, ctx->dcount.p, sizeof(cnt4), cudaMemcpyDeviceToHost, s), "count d2h");
   if (timing) cudaEventRecord(ctx->ev[5], s);
   CK(cudaStreamSynchronize(s), "compact sync");
   const uint64_t n_out = cnt4[0];
   ctx->n_stored = n_out;
   for (int k = 1; k < 4; ++k) S.reports_by_kind[k] = cnt4[k];
+  S.reports_bo = cnt4[ARB_BO];
   // dropped VSM candidates are unique and distinct from every retained one
   ctx->n_reports = n_out + (n_vsm - kept_vsm);
   int rc = n_vsm > kept_vsm ? ARB_TRUNCATED : ARB_OK;

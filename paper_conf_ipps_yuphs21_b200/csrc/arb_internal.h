@@ -18,6 +18,8 @@ constexpr uint32_t kSyncAll = 0xFFFFu;
 
 // ---- VSM bits (Table II) ----------------------------------------
 constexpr uint32_t kOVv = 1, kCVv = 2, kOVi = 4, kCVi = 8;
+// buffer-overflow extension (ARB_F_BO, Z17): the word has a CV
+constexpr uint32_t kCVp = 16;
 
 // A transition function of the VSM in "selector" form: output bit j of the
 // 4-bit state is taken from source sel_j (0..3 = input bit, 4 = constant 0,
@@ -27,6 +29,9 @@ using Sel = uint32_t;
 __host__ __device__ constexpr Sel sel_make(uint32_t s0, uint32_t s1, uint32_t s2, uint32_t s3) {
   return s0 | (s1 << 3) | (s2 << 6) | (s3 << 9);
 }
+// Bits 12-13 act on the 5th state bit (kCVp, ARB_F_BO only): 0 keep, 2 clear,
+// 3 set; composition keeps the later non-keep action.
+constexpr Sel kPopClr = 2u << 12, kPopSet = 3u << 12;
 constexpr Sel kSelId    = sel_make(0, 1, 2, 3);
 constexpr Sel kSelUPT   = sel_make(0, 0, 2, 2);   // CV takes OV's validity and init (update_target)
 constexpr Sel kSelUPH   = sel_make(1, 1, 3, 3);   // OV takes CV's (update_host)
@@ -134,6 +139,7 @@ struct ReplayParams {
   const uint64_t* hot_off; uint16_t* hot_F; uint8_t* hot_P;
   uint64_t n_words;
   uint8_t* shadow;                        // n_words bytes
+  uint32_t bo;                            // ARB_F_BO: target accesses to words without kCVp are BO
   const uint32_t* ops_start;              // [n_buckets + 1]
   const BucketOp* ops;
   uint4* cand; uint64_t cand_cap;         // report candidates {word lo, word hi, pos, kind}

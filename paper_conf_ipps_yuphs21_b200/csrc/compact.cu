@@ -9,9 +9,11 @@ constexpr int kRsThreads = 512, kRsItems = 8, kRsTile = kRsThreads * kRsItems;
 struct RsPass { int field; int shift; int bits; };
 constexpr int kRsMaxBits = 11;                    // digits of up to 11 bits (2048 bins)
 constexpr int kRsBins = 1 << kRsMaxBits;
-// digit fields: uint4 {0: w, 1: z, 2: x, 3: y, 4: z << 2 | w}; uint2 {0: x, 1: y}
+// digit fields: uint4 {0: w, 1: z, 2: x, 3: y, 4: z << 3 | w}; uint2 {0: x, 1: y}
+// (w = report kind, 1..4: 3 bits)
+constexpr int kKindBits = 3;
 __device__ __forceinline__ uint32_t rs_field(uint4 c, int f) {
-  return f == 0 ? c.w : f == 1 ? c.z : f == 2 ? c.x : f == 3 ? c.y : (c.z << 2) | c.w;
+  return f == 0 ? c.w : f == 1 ? c.z : f == 2 ? c.x : f == 3 ? c.y : (c.z << kKindBits) | c.w;
 }
 __device__ __forceinline__ uint32_t rs_field(uint2 c, int f) { return f == 0 ? c.x : c.y; }
 template <class E>
@@ -201,7 +203,7 @@ __global__ void __launch_bounds__(kRsThreads) k_keep_write(const uint4* a, uint6
   uint32_t wpre = 0;
   for (uint32_t w = 0; w < warp; ++w) wpre += ws[w];
   uint64_t o = blk[blockIdx.x] + wpre + incl - c;
-  uint32_t kc[4] = {0, 0, 0, 0};
+  uint32_t kc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   for (int j = 0; j < kRsItems; ++j) {
     uint64_t i = base + (uint64_t)threadIdx.x * kRsItems + j;
     if (!kp[j]) continue;
@@ -211,7 +213,7 @@ __global__ void __launch_bounds__(kRsThreads) k_keep_write(const uint4* a, uint6
       uint64_t w0 = (word & kMask48) | ((uint64_t)x.w << 48);
       uint64_t w1 = gidx ? gidx[x.z] : index_base + x.z;
       out[o] = make_uint4((uint32_t)w0, (uint32_t)(w0 >> 32), (uint32_t)w1, (uint32_t)(w1 >> 32));
-      kc[x.w & 3u]++;                      // per-kind counts in n_out[1..3]
+      kc[x.w & 7u]++;                      // per-kind counts in n_out[1..4]
     } else {
       out[o] = x;
     }
@@ -219,7 +221,7 @@ __global__ void __launch_bounds__(kRsThreads) k_keep_write(const uint4* a, uint6
   }
   if (final_out) {
 #pragma unroll
-    for (int k = 1; k < 4; ++k) {
+    for (int k = 1; k < 5; ++k) {
       uint32_t v = kc[k];
       for (int d = 16; d; d >>= 1) v += __shfl_xor_sync(FULL, v, d);
       if (lane == 0 && v) atomicAdd(&n_out[k], (unsigned long long)v);
@@ -351,7 +353,7 @@ cudaError_t launch_sort_segments(uint2* a, uint2* b, uint64_t n, int chunk_bits,
 }
 
 cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches) {
-  cudaMemsetAsync(p.n_out, 0, 4 * sizeof(unsigned long long), s);
+  cudaMemsetAsync(p.n_out, 0, 8 * sizeof(unsigned long long), s);
   if (p.n_cand == 0) return cudaGetLastError();
   uint4* a = p.cand;
   uint4* b = p.tmp;
@@ -363,7 +365,7 @@ cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches
   if (p.dedup_first) {
     // (word, kind, pos): keep the first of each (word, kind)
     np = add_field_passes(ps, np, 1, p.pos_bits);
-    np = add_field_passes(ps, np, 0, 2);
+    np = add_field_passes(ps, np, 0, kKindBits);
     np = add_field_passes(ps, np, 2, wb_lo);
     np = add_field_passes(ps, np, 3, wb_hi);
     if ((e = radix_sort<uint4>(a, b, n, ps, np, p.blk, s, launches)) != cudaSuccess) return e;
@@ -380,10 +382,10 @@ cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches
     uint4* t = a; a = b; b = t;
     np = 0;
   }
-  if (p.pos_bits <= 30) {
-    np = add_field_passes(ps, np, 4, p.pos_bits + 2);         // record, then kind
+  if (p.pos_bits + kKindBits <= 32) {
+    np = add_field_passes(ps, np, 4, p.pos_bits + kKindBits); // record, then kind
   } else {
-    np = add_field_passes(ps, np, 0, 2);
+    np = add_field_passes(ps, np, 0, kKindBits);
     np = add_field_passes(ps, np, 1, p.pos_bits);
   }
   np = add_field_passes(ps, np, 2, wb_lo);
@@ -391,7 +393,7 @@ cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches
   if ((e = radix_sort<uint4>(a, b, n, ps, np, p.blk, s, launches)) != cudaSuccess) return e;
   uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
   if (n == 0) {
-    cudaMemsetAsync(p.n_out, 0, 4 * sizeof(unsigned long long), s);
+    cudaMemsetAsync(p.n_out, 0, 8 * sizeof(unsigned long long), s);
     return cudaGetLastError();
   }
   k_keep_count<<<nblk, kRsThreads, 0, s>>>(a, n, 0, p.blk);

@@ -40,7 +40,7 @@ struct Emitter {
 
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
-                     FlushPlan& out) {
+                     FlushPlan& out, bool bo) {
   const uint32_t n_buckets = (uint32_t)bucket_start.size() - 1;
   out = FlushPlan();
   Emitter em{base_word, n_words, &out};
@@ -89,7 +89,7 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
         if (f < 0) return fail(ARB_EMAP, c.pos, "map clause partially overlaps a present entry");
         if (f == 1) { it->second.rc += 1; break; }  // exist(CV): ref_count += 1
         map.emplace(addr, MapEntry{addr + len, 1});  // new CV, ref_count = 1
-        em.emit(pos, kSelALLOC, addr, addr + len, open);
+        em.emit(pos, kSelALLOC | (bo ? kPopSet : 0u), addr, addr + len, open);
         if (arg == MT_TO || arg == MT_TOFROM) em.emit(pos, kSelUPT, addr, addr + len, open);
         break;
       }
@@ -103,7 +103,7 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
         if (arg == MT_DELETE) it->second.rc = 0; else it->second.rc -= 1;
         if (it->second.rc == 0) {
           if (arg == MT_FROM || arg == MT_TOFROM) em.emit(pos, kSelUPH, addr, addr + len, open);
-          em.emit(pos, kSelREL, it->first, it->second.hi, open);
+          em.emit(pos, kSelREL | (bo ? kPopClr : 0u), it->first, it->second.hi, open);
           map.erase(it);
         }
         break;

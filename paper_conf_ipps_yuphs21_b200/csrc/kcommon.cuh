@@ -64,7 +64,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 }
 
 // ---- selector-form transition functions (see arb_internal.h) -------------
-// x holds 4 states, one per byte (low nibble); returns the 4 images.
+// x holds 4 states, one per byte (low nibble); returns the 4 images (bit 4 clear).
 __device__ __forceinline__ uint32_t sel_apply4(Sel s, uint32_t x) {
   uint32_t out = 0;
 #pragma unroll
@@ -75,8 +75,14 @@ __device__ __forceinline__ uint32_t sel_apply4(Sel s, uint32_t x) {
   }
   return out;
 }
+// ARB_F_BO contexts: bits 0-3 as sel_apply4, bit 4 (kCVp) kept, cleared or set
+// by the selector's bits 12-13.
+__device__ __forceinline__ uint32_t sel_apply5(Sel s, uint32_t x) {
+  const uint32_t pop = (s >> 12) & 3u;
+  return sel_apply4(s, x) | (pop == 0 ? (x & 0x10101010u) : (pop == 3 ? 0x10101010u : 0u));
+}
 __device__ __forceinline__ Sel sel_compose(Sel g, Sel f) {  // g after f
-  Sel r = 0;
+  Sel r = (g & (3u << 12)) ? (g & (3u << 12)) : (f & (3u << 12));
 #pragma unroll
   for (int j = 0; j < 4; ++j) {
     uint32_t gj = (g >> (3 * j)) & 7u;

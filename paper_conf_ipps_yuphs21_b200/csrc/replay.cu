@@ -88,7 +88,10 @@ __device__ __forceinline__ void block_minmax(uint32_t& lo, uint32_t& hi, uint32_
 }
 
 // ---- range ops ----------------------------------------------------------------
-// Apply transition `sel` to the state bytes base[lo, hi).
+// Apply transition `sel` to the state bytes base[lo, hi) (BO: 5-bit states, ARB_F_BO).
+template <bool BO>
+__device__ __forceinline__ uint32_t apply_sel(Sel s, uint32_t x) { return BO ? sel_apply5(s, x) : sel_apply4(s, x); }
+template <bool BO>
 __device__ void stream_apply(uint8_t* base, uint64_t lo, uint64_t hi, Sel sel) {
   if (lo >= hi) return;
   // 16-B aligned middle [a, b) of [lo, hi), by address
@@ -96,8 +99,8 @@ __device__ void stream_apply(uint8_t* base, uint64_t lo, uint64_t hi, Sel sel) {
   const uintptr_t pa = (p0 + 15) & ~(uintptr_t)15, pb = p1 & ~(uintptr_t)15;
   uint64_t a = hi, b = hi;                       // no aligned middle: all bytes in the head loop
   if (pa < pb) { a = lo + (pa - p0); b = hi - (p1 - pb); }
-  for (uint64_t j = lo + threadIdx.x; j < a; j += RT) __stcg(base + j, (uint8_t)sel_apply4(sel, __ldcg(base + j)));
-  for (uint64_t j = b + threadIdx.x; j < hi; j += RT) __stcg(base + j, (uint8_t)sel_apply4(sel, __ldcg(base + j)));
+  for (uint64_t j = lo + threadIdx.x; j < a; j += RT) __stcg(base + j, (uint8_t)apply_sel<BO>(sel, __ldcg(base + j)));
+  for (uint64_t j = b + threadIdx.x; j < hi; j += RT) __stcg(base + j, (uint8_t)apply_sel<BO>(sel, __ldcg(base + j)));
   uint4* v = reinterpret_cast<uint4*>(base + a);
   const uint64_t nv = (b - a) >> 4;
   constexpr int U = 4;   // 4 x 16 B loads in flight per thread
@@ -108,15 +111,15 @@ __device__ void stream_apply(uint8_t* base, uint64_t lo, uint64_t hi, Sel sel) {
     for (int u = 0; u < U; ++u) x[u] = __ldcg(v + j + u * RT);
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      x[u].x = sel_apply4(sel, x[u].x); x[u].y = sel_apply4(sel, x[u].y);
-      x[u].z = sel_apply4(sel, x[u].z); x[u].w = sel_apply4(sel, x[u].w);
+      x[u].x = apply_sel<BO>(sel, x[u].x); x[u].y = apply_sel<BO>(sel, x[u].y);
+      x[u].z = apply_sel<BO>(sel, x[u].z); x[u].w = apply_sel<BO>(sel, x[u].w);
       __stcg(v + j + u * RT, x[u]);
     }
   }
   for (; j < nv; j += RT) {
     uint4 x = __ldcg(v + j);
-    x.x = sel_apply4(sel, x.x); x.y = sel_apply4(sel, x.y);
-    x.z = sel_apply4(sel, x.z); x.w = sel_apply4(sel, x.w);
+    x.x = apply_sel<BO>(sel, x.x); x.y = apply_sel<BO>(sel, x.y);
+    x.z = apply_sel<BO>(sel, x.z); x.w = apply_sel<BO>(sel, x.w);
     __stcg(v + j, x);
   }
 }
@@ -124,6 +127,7 @@ __device__ void stream_apply(uint8_t* base, uint64_t lo, uint64_t hi, Sel sel) {
 // Apply every pending range op of the bucket with position < limit; runs of
 // ops on the identical range with no event in between are composed first.
 // S.next_op caches the position of the first pending op.
+template <bool BO>
 __device__ void apply_ops_before(ReplaySmem& S, const ReplayParams& p, uint32_t limit) {
   while (S.next_op < limit) {
     const uint32_t k = S.op_cur;
@@ -144,7 +148,7 @@ __device__ void apply_ops_before(ReplaySmem& S, const ReplayParams& p, uint32_t 
         S.fsum[w] = (uint16_t)sel_compose(sel, S.fsum[w]);
       }
     } else if (hi > lo) {
-      stream_apply(S.shrel, lo - S.bucket_base, hi - S.bucket_base, sel);
+      stream_apply<BO>(S.shrel, lo - S.bucket_base, hi - S.bucket_base, sel);
     }
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -219,9 +223,14 @@ __device__ __forceinline__ uint32_t hslot(uint32_t w) { return (w * 2654435761u)
 // not change the state, so a read's state-before is the state loaded
 // at the start of the step, or — if its word's single write precedes it — the
 // image of that write; the write event itself commits the word's final state.
-template <bool PARTIAL>
+//
+// BO (ARB_F_BO) is a template parameter: deciding that a target access is a
+// buffer overflow needs its word's state before the inserts, which would put
+// the shadow-load latency in front of the hashing for every replay.
+template <bool PARTIAL, bool BO>
 __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
   uint32_t slot[RI], word[RI], pos[RI], op[RI], s_pre[RI];
+  uint32_t bom = 0;                // bit j: event j is a buffer overflow (ARB_F_BO, Z17)
   bool multi = false;
   const uint8_t* sh = S.shrel;
   uint2* hs = S.u.h.slot;
@@ -236,6 +245,8 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
       word[j] = e.x & kWordMask; op[j] = e.x >> 30; pos[j] = e.y;
       if (!PARTIAL || word[j] - plo < pw) s_pre[j] = __ldcg(sh + word[j]);
       else op[j] = 4;                                       // another work item's word
+      // a target access (RT = 2, WT = 3) to a word without a CV: BO, no VSM effect
+      if (BO && (op[j] & 2u) && !(s_pre[j] & kCVp)) { bom |= 1u << j; op[j] = 4; }
     }
   }
   // writes (WH = 1, WT = 3: odd ops) enter the table: slot {word, pos << 2 | op}
@@ -282,9 +293,9 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
         }
       }
     } else if (op[j] & 1u) {
-      __stcg(const_cast<uint8_t*>(sh) + word[j], (uint8_t)vsm_write_op(op[j], s0));
+      __stcg(const_cast<uint8_t*>(sh) + word[j], (uint8_t)(vsm_write_op(op[j], s0) | (BO ? (s_pre[j] & kCVp) : 0u)));
     }
-    fk[j] = classify_bits(op[j], before);
+    fk[j] = ((bom >> j) & 1u) ? 4u : classify_bits(op[j], before);
   }
   emit_faults(p, fk, word, pos, S.bucket_base);
   if (any_w) {
@@ -298,8 +309,9 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
 }
 
 // the fast step of a word-range part (rare: range-heavy buckets), out of line
+template <bool BO>
 __device__ bool step_fast_partial(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
-  return step_fast<true>(S, p, ev, m);
+  return step_fast<true, BO>(S, p, ev, m);
 }
 
 // ---- sort step -------------------------------------------------------------------------
@@ -390,6 +402,7 @@ __device__ __forceinline__ uint32_t acc_summary(uint32_t op) {
   return op == OP_WH ? (1u | 4u) : (op == OP_WT ? (2u | 8u) : 0u);
 }
 
+template <bool BO>
 __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   uint32_t lo = 0xFFFFFFFFu, hi = 0;
@@ -451,24 +464,30 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
   // blocked arrangement: thread t owns sorted elements [RI*t, RI*t + RI)
   const uint64_t bb = S.bucket_base;
   uint8_t* const sh = S.shrel;
-  uint32_t val[RI], s0[RI], key[RI], wd[RI], ps[RI];
-  bool head[RI];
+  uint32_t val[RI], s0[RI], key[RI], wd[RI], ps[RI], pf[RI];
+  bool head[RI], isb[RI];
   uint32_t agg = 0;
+  constexpr bool bo = BO;
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
     const uint32_t i = tid * RI + j;
-    key[j] = 0; head[j] = false; s0[j] = 0; val[j] = 0; wd[j] = 0; ps[j] = 0;
+    key[j] = 0; head[j] = false; s0[j] = 0; val[j] = 0; wd[j] = 0; ps[j] = 0; pf[j] = 0; isb[j] = false;
     if (i < m) {
       const uint32_t k = kin[i];
       const uint32_t w = k & kWordMask;
       const bool h = (i == 0) || ((kin[i - 1] & kWordMask) != w);
-      uint32_t v = acc_summary(k >> 30);
+      // ARB_F_BO: kCVp is constant within a step (range ops cut steps); a target
+      // access to a word without a CV is BO and the identity (Z17)
+      const uint32_t full = (h || bo) ? __ldcg(sh + w) : 0u;
+      const bool b = bo && ((k >> 30) & 2u) && !(full & kCVp);
+      uint32_t v = b ? 0u : acc_summary(k >> 30);
       uint32_t st = 0;
       if (h) {
-        st = __ldcg(sh + w) & 15u;
+        st = full & 15u;
         v = kHead | kConst | acc_apply(v, st);
       }
       key[j] = k; head[j] = h; s0[j] = st; val[j] = v; wd[j] = w; ps[j] = pin[i];
+      pf[j] = full & kCVp; isb[j] = b;
     }
     agg = acc_combine(agg, val[j]);
   }
@@ -494,9 +513,9 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
     if (i < m) {
       const uint32_t before = head[j] ? s0[j] : (run & 15u);
       run = acc_combine(run, val[j]);
-      fk[j] = classify(key[j] >> 30, before);
+      fk[j] = isb[j] ? 4u : classify(key[j] >> 30, before);
       const bool tail = (i + 1 == m) || ((kin[i + 1] & kWordMask) != wd[j]);
-      if (tail) __stcg(sh + wd[j], (uint8_t)(run & 15u));
+      if (tail) __stcg(sh + wd[j], (uint8_t)((run & 15u) | pf[j]));
     }
   }
   emit_faults(p, fk, wd, ps, bb);
@@ -589,7 +608,7 @@ __global__ void k_carry(const uint4* hot, const uint64_t* bucket_start, const ui
     uint32_t st = sh[w];
     for (uint32_t k = 0; k < slices; ++k) {
       hot_P[off + (uint64_t)k * span16 + w] = (uint8_t)st;
-      st = sel_apply4(hot_F[off + (uint64_t)k * span16 + w], st) & 15u;
+      st = sel_apply4(hot_F[off + (uint64_t)k * span16 + w], st) & 15u;   // K5 never runs with ARB_F_BO
     }
     sh[w] = (uint8_t)st;
   }
@@ -732,6 +751,9 @@ __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t 
   return m;
 }
 
+// BO: ARB_F_BO contexts (the buffer-overflow extension, Z17) get their own
+// instance, so the default replay carries none of its checks.
+template <bool BO>
 __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   ReplaySmem& S = *reinterpret_cast<ReplaySmem*>(smem_raw);
@@ -811,7 +833,7 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         m_nxt = issue_gather(S, p, nxt, total, S.ev[cur ^ 1], hint);
       }
       // ---- range ops before the first event, then cut at the next one -------------
-      apply_ops_before(S, p, ev[0].y);
+      apply_ops_before<BO>(S, p, ev[0].y);
       uint32_t cut = m;
       if (S.next_op != 0xFFFFFFFFu && ev[m - 1].y > S.next_op) {
         uint32_t cnt = 0;
@@ -821,8 +843,8 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       if (mode == kItemSummary) {
         step_summary(S, ev, cut);
       } else {
-        const bool fast = S.partial ? step_fast_partial(S, p, ev, cut) : step_fast<false>(S, p, ev, cut);
-        if (!fast) step_sort(S, p, ev, cut);
+        const bool fast = S.partial ? step_fast_partial<BO>(S, p, ev, cut) : step_fast<false, BO>(S, p, ev, cut);
+        if (!fast) step_sort<BO>(S, p, ev, cut);
         if (tid == 0) atomicAdd(fast ? &p.st->steps_fast : &p.st->steps_sort, 1ull);
       }
       e0 += cut;
@@ -839,7 +861,7 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       }
     }
     // the ops after the last event (a slice replay's private states are not kept)
-    if (mode != kItemSlice) apply_ops_before(S, p, 0xFFFFFFFFu);
+    if (mode != kItemSlice) apply_ops_before<BO>(S, p, 0xFFFFFFFFu);
     if (tid == 0 && total > first) atomicMax(&p.st->max_bucket_events, (unsigned long long)(total - first));
     __syncthreads();
     if (mode == kItemSummary) {
@@ -851,9 +873,10 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
 
 cudaError_t launch_replay(const ReplayParams& p, int n_ctas, cudaStream_t s) {
   const size_t smem = sizeof(ReplaySmem);
-  cudaError_t e = cudaFuncSetAttribute(k_replay, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  auto kern = p.bo ? k_replay<true> : k_replay<false>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  k_replay<<<n_ctas, RT, smem, s>>>(p);
+  kern<<<n_ctas, RT, smem, s>>>(p);
   return cudaGetLastError();
 }
 

@@ -36,7 +36,7 @@ def _gpu_run(prog, lo, hi, flushes=None, recs=None, gidx=None, flags=0):
 def _check_full(orc, prog, flags=0):
     rec = prog.fill_host()
     lo, hi = prog.addr_base // 8, (prog.addr_base + prog.addr_bytes) // 8
-    exp = orc.replay(rec, prog.addr_base, prog.addr_bytes)
+    exp = orc.replay(rec, prog.addr_base, prog.addr_bytes, detect_bo=bool(flags & 8))
     assert exp.rc == 0
     ctx, got = _gpu_run(prog, lo, hi, flags=flags)
     assert sorted(got) == exp.triples()
@@ -45,9 +45,11 @@ def _check_full(orc, prog, flags=0):
     return exp
 
 
-@pytest.mark.parametrize("flags", [0, 4])
+@pytest.mark.parametrize("flags", [0, 4, 8])
 def test_config3_scaled(orc, flags):
-    """flags=4 (ARB_F_SMALL_PARTS): busy small buckets replayed as time slices (K5)."""
+    """flags=4 (ARB_F_SMALL_PARTS): busy small buckets replayed as time slices (K5);
+    flags=8 (ARB_F_BO): the buffer-overflow extension (every kernel access is inside a
+    mapped section here, so the report set is the same)."""
     from gen import native
     exp = _check_full(orc, native.config3(scale=0.01), flags=flags)
     kinds = {k for _, _, k in exp.triples()}

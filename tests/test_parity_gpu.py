@@ -14,8 +14,9 @@ pytestmark = pytest.mark.gpu
 
 def check(orc, rec, base, size, **kw):
     okw = {k: kw.pop(k) for k in ("dedup_first",) if k in kw}
-    exp = orc.replay(rec, base, size, **okw)
     flags = (1 if okw.get("dedup_first") else 0) | kw.pop("flags", 0)
+    okw["detect_bo"] = bool(flags & 8)                    # ARB_F_BO <-> the oracle's extension (Z17)
+    exp = orc.replay(rec, base, size, **okw)
     rc, got, shadow, st = run_gpu(rec, base, size, flags=flags, **kw)
     assert rc == exp.rc
     if rc == 0:
@@ -217,3 +218,63 @@ def test_untracked_words_ignored(orc):
     from gen.fuzz import random_program
     rec, base, span = random_program(91)
     check(orc, rec, base + 256, span // 2)
+
+
+# ---- buffer-overflow extension (ARB_F_BO = 8, Z17) ---------------
+@pytest.mark.parametrize("write", [False, True])
+def test_bo_half_mapped_array(orc, write):
+    """only the first half of the array is mapped, the kernel loops over all of it."""
+    from gen.trace import MAP, OP, TraceBuilder
+    A, n = 0x40000, 4096
+    tb = TraceBuilder()
+    tb.loop([(OP.WH, A)], n, 8)
+    tb.enter(MAP.TOFROM, A, 8 * (n // 2))
+    k0 = len(tb)
+    tb.loop([(OP.WT if write else OP.RT, A)], n, 8)
+    tb.exit(MAP.TOFROM, A, 8 * (n // 2))
+    exp, st = check(orc, tb.array(), A, 8 * n, flags=8)
+    assert exp.triples() == [(A // 8 + i, k0 + i, 4) for i in range(n // 2, n)]
+    assert st["reports_bo"] == n // 2
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_bo_fuzz_small(orc, seed):
+    from gen.fuzz import random_program
+    rec, base, span = random_program(3000 + seed)
+    for bb in (0, 2, 5):
+        check(orc, rec, base, span, bucket_bits=bb, flags=8)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_bo_fuzz_large_steps(orc, seed):
+    """Many steps per bucket, sort steps, range ops cutting steps; with parts (flags 4)."""
+    from gen.fuzz import random_program
+    rec, base, span = random_program(1000 + seed, n_arrays=6, array_words=8192, steps=500,
+                                     loop_max=20000)
+    for bb in (0, 11):
+        check(orc, rec, base, span, bucket_bits=bb, flags=8)
+    check(orc, rec, base, span, flags=8 | 4)
+
+
+def test_bo_config2_and_hot_word(orc):
+    """The DRACC-style suite and a hot word (no time slices under ARB_F_BO)."""
+    from gen.configs import config2
+    from gen.trace import MAP, OP, TraceBuilder
+    rec, base, size = config2()
+    check(orc, rec, base, size, flags=8)
+    tb = TraceBuilder()
+    A = 0x8000
+    tb.wh(A)
+    rs = np.random.default_rng(6)
+    ops = rs.choice([OP.RT, OP.WT, OP.RH, OP.WH], size=400000, p=[.4, .2, .3, .1])
+    for j, chunk in enumerate(np.array_split(ops, 10)):
+        if j % 2 == 0:
+            tb.enter(MAP.TO, A, 64)       # odd chunks run with the CV deleted: their target accesses are BO
+        arr = np.zeros((chunk.size, 2), dtype=np.uint64)
+        arr[:, 0] = np.uint64(A) | (chunk.astype(np.uint64) << np.uint64(48))
+        arr[:, 1] = 8
+        tb.add_array(arr)
+        if j % 2 == 0:
+            tb.exit(MAP.DELETE, A, 64)
+    exp, st = check(orc, tb.array(), A, 64, flags=8)
+    assert st["hot_buckets"] == 0 and st["reports_bo"] > 0
