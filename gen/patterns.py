@@ -290,3 +290,49 @@ PATTERNS = {
 }
 # bytes a pattern touches beyond ``n*esz`` from its base (P10 and P22 use two arrays)
 FOOTPRINT_ARRAYS = {"P10": 2, "P22": 2}
+
+
+# ---- buffer-overflow patterns (DRACC 23, 25, 28-31 analogues; Table III row BO,
+# P:376; detected with the extension of P:277-281, ARB_F_BO / detect_bo) ----------
+BO = 4
+
+
+def b23(tb, a, n, esz, buggy, task):   # map(tofrom: a[0:n/2]) but the kernel updates a[0:n]
+    _init(tb, a, n, esz)
+    sec = (n // 2 if buggy else n) * esz
+    tb.enter(MAP.TOFROM, a, sec); _kupdate(tb, a, n, esz); tb.exit(MAP.TOFROM, a, sec)
+    _hread(tb, a, n, esz)
+
+
+def b25(tb, a, n, esz, buggy, task):   # enter data map(to: a[0:n/2]), kernel reads a[0:n]
+    _init(tb, a, n, esz)
+    sec = (n // 2 if buggy else n) * esz
+    tb.enter(MAP.TO, a, sec); _kread(tb, a, n, esz); tb.exit(MAP.DELETE, a, sec)
+
+
+def b28(tb, a, n, esz, buggy, task):   # section one 8-B word short (P:267 granularity), kernel writes a[0:n]
+    _init(tb, a, n, esz)
+    sec = n * esz - (8 if buggy else 0)
+    tb.enter(MAP.FROM, a, sec); _kwrite(tb, a, n, esz); tb.exit(MAP.FROM, a, sec)
+    _hread(tb, a, sec // esz, esz)
+
+
+def b29(tb, a, n, esz, buggy, task):   # the kernel runs after `exit data delete`
+    _init(tb, a, n, esz)
+    tb.enter(MAP.TO, a, n * esz)
+    if buggy:
+        tb.exit(MAP.DELETE, a, n * esz); _kread(tb, a, n, esz)
+    else:
+        _kread(tb, a, n, esz); tb.exit(MAP.DELETE, a, n * esz)
+
+
+def b30(tb, a, n, esz, buggy, task):   # the kernel indexes past the mapped section's start
+    _init(tb, a, n, esz)
+    lo = n // 4 if buggy else 0
+    tb.enter(MAP.TOFROM, a + lo * esz, (n - lo) * esz)
+    _kupdate(tb, a, n, esz)
+    tb.exit(MAP.TOFROM, a + lo * esz, (n - lo) * esz)
+
+
+BO_PATTERNS = {"B23": (b23, {BO}), "B25": (b25, {BO}), "B28": (b28, {BO}), "B29": (b29, {BO}),
+               "B30": (b30, {BO})}

@@ -278,3 +278,19 @@ def test_bo_config2_and_hot_word(orc):
             tb.exit(MAP.DELETE, A, 64)
     exp, st = check(orc, tb.array(), A, 64, flags=8)
     assert st["hot_buckets"] == 0 and st["reports_bo"] > 0
+
+
+def test_bo_patterns(orc):
+    """The buffer-overflow patterns (DRACC 23/25/28-31 analogues), buggy and fixed,
+    concatenated on separate regions: GPU = oracle with the extension on."""
+    from gen.patterns import BO_PATTERNS
+    from gen.trace import TraceBuilder
+    tb = TraceBuilder()
+    region, base, k = 1 << 16, 0x100000, 0
+    for esz in (4, 8):
+        for name in sorted(BO_PATTERNS):
+            for buggy in (True, False):
+                BO_PATTERNS[name][0](tb, base + k * region, 2048, esz, buggy, 5)
+                k += 1
+    exp, st = check(orc, tb.array(), base, k * region, flags=8)
+    assert {t[2] for t in exp.triples()} == {4} and st["reports_bo"] == len(exp.triples())

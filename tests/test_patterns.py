@@ -43,3 +43,24 @@ def test_config2_suite(orc):
         per.setdefault(j, set()).add(k)
     for j, d in enumerate(inst):
         assert per.get(j, set()) == d["label"], (d["name"], d["buggy"])
+
+
+@pytest.mark.parametrize("name", sorted(__import__("gen.patterns", fromlist=["BO_PATTERNS"]).BO_PATTERNS))
+@pytest.mark.parametrize("esz", [4, 8])
+def test_bo_pattern(orc, name, esz):
+    """Buffer-overflow patterns (Table III row BO) with the extension of
+    P:277-281: buggy -> BO only, fixed -> clean; the value simulator (CV
+    existence as a set) agrees on every report."""
+    from gen.patterns import BO_PATTERNS
+    fn, label = BO_PATTERNS[name]
+    n = 64
+    for buggy in (True, False):
+        tb = TraceBuilder()
+        fn(tb, BASE, n, esz, buggy, 5)
+        rec = tb.array()
+        res = orc.replay(rec, BASE, 4 * n * esz, detect_bo=True)
+        assert res.rc == 0
+        kinds = {k for _, _, k in res.triples()}
+        assert kinds == (label if buggy else set()), (name, buggy, kinds)
+        vs = ValueSim(bo=True).run(rec)
+        assert sorted(vs) == [t for t in res.triples() if t[2] != 3]
