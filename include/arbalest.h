@@ -53,7 +53,7 @@ enum arb_upd { ARB_UPD_TO = 0, ARB_UPD_FROM = 1 };
 
 /* ---- reports ---------------------------------------------------------------- */
 enum arb_kind { ARB_UUM = 1, ARB_USD = 2, ARB_MIR = 3,
-                ARB_BO = 4  /* buffer overflow, with ARB_F_BO only (Z17) */ };
+                ARB_BO = 4  /* buffer overflow, with ARB_F_BO only (Z20) */ };
 /* w0: [0,48) absolute word index (= byte address / 8) | [48,56) kind
  * w1: global record index (0-based; see arb_submit_events)
  * Canonical order: word, then record, then kind, ascending; no duplicates. */
@@ -83,7 +83,7 @@ enum arb_status {
                                    replay every small bucket with >= 64 events as 3 time
                                    slices (the mechanisms normally used for range-heavy
                                    and hot buckets only)                                  */
-#define ARB_F_BO          0x8u  /* buffer-overflow extension (reading Z17): every
+#define ARB_F_BO          0x8u  /* buffer-overflow extension (reading Z20): every
                                    word carries a 5th state bit "has a CV" (set by allocate,
                                    cleared by release); a target access (RT/WT) to a word
                                    without a CV is reported as ARB_BO and has no VSM effect.

@@ -27,7 +27,7 @@
  *   MIR attribution to later event (Z11)  parity unpinned (definition only)
  *   dedup-first mode (Z3)                 parity unpinned (definition only)
  *   sub-word semantics (Z4)               parity unpinned (definition only)
- *   buffer overflow, present-bit form (Z17) pinned (P:279 worked example + brute force vs the
+ *   buffer overflow, present-bit form (Z20) pinned (P:279 worked example + brute force vs the
  *                                         value simulator's CV existence); the paper's base-interval
  *                                         comparison (overflow into ANOTHER mapped CV) is not modelled
  */
@@ -77,7 +77,7 @@ typedef struct {
    * (tracked_words == NULL) tracks every word of the range (Z12). */
   const uint64_t* tracked_words;
   uint64_t        n_tracked;
-  /* Buffer-overflow extension (reading Z17 of DESIGN.md): a 5th
+  /* Buffer-overflow extension (reading Z20 of DESIGN.md): a 5th
    * state bit CVp ("the word has a CV") is set by allocate and cleared by
    * release; a target access (RT/WT) to a word without a CV is reported as
    * ORC_BO and has no VSM effect (no UUM/USD check, no transition: the access

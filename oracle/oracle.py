@@ -82,7 +82,7 @@ def replay(records: np.ndarray, addr_base: int, addr_bytes: int, *, dedup_first:
            tracked_words: np.ndarray | None = None, global_index: np.ndarray | None = None,
            want_shadow: bool = True, detect_bo: bool = False) -> OracleResult:
     """Replay ``records`` (uint64 array of shape (n, 2): w0, w1) through the oracle.
-    ``detect_bo``: the buffer-overflow extension (reading Z17)."""
+    ``detect_bo``: the buffer-overflow extension (reading Z20)."""
     lib = _load()
     rec = np.ascontiguousarray(records, dtype=np.uint64).reshape(-1, 2)
     n = rec.shape[0]

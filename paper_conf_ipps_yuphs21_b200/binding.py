@@ -18,7 +18,7 @@ ARB_OK, ARB_TRUNCATED = 0, 1
 ARB_EINVAL, ARB_ENOMEM, ARB_ECUDA, ARB_EMAP, ARB_ETRACE, ARB_ESTATE, ARB_EOPEN = -1, -2, -3, -4, -5, -6, -7
 ARB_F_DEDUP_FIRST, ARB_F_TIMING = 0x1, 0x2
 ARB_F_SMALL_PARTS = 0x4
-ARB_F_BO = 0x8          # buffer-overflow extension (Z17)
+ARB_F_BO = 0x8          # buffer-overflow extension (Z20)
 ARB_BO = 4
 STATUS = {0: "ARB_OK", 1: "ARB_TRUNCATED", -1: "ARB_EINVAL", -2: "ARB_ENOMEM", -3: "ARB_ECUDA",
           -4: "ARB_EMAP", -5: "ARB_ETRACE", -6: "ARB_ESTATE", -7: "ARB_EOPEN"}

@@ -363,7 +363,7 @@ static void build_items(arb_ctx ctx, const FlushPlan& plan, const std::vector<do
     const uint64_t span = ctx->bucket_start[b + 1] - ctx->bucket_start[b];
     const double ev = bucket_events[b];
     if (parts[b] != 1 || span > kHotSpan) continue;
-    if (ctx->cfg.flags & ARB_F_BO) continue;      // slice functions cannot express the BO condition (Z17)
+    if (ctx->cfg.flags & ARB_F_BO) continue;      // slice functions cannot express the BO condition (Z20)
     const bool hot = force_hot ? ev >= 64.0 : (ev > 1.25 * share && ev > kSliceEvents);
     if (!hot) continue;
     const double want = force_hot ? 3.0 : std::ceil(ev / kSliceEvents);

@@ -18,7 +18,7 @@ constexpr uint32_t kSyncAll = 0xFFFFu;
 
 // ---- VSM bits (Table II) ----------------------------------------
 constexpr uint32_t kOVv = 1, kCVv = 2, kOVi = 4, kCVi = 8;
-// buffer-overflow extension (ARB_F_BO, Z17): the word has a CV
+// buffer-overflow extension (ARB_F_BO, Z20): the word has a CV
 constexpr uint32_t kCVp = 16;
 
 // A transition function of the VSM in "selector" form: output bit j of the

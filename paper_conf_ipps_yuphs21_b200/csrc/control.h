@@ -46,7 +46,7 @@ struct FlushPlan {
 // place only on success (the caller passes a copy and commits it).
 // `bucket_start` holds the first relative word of every address bucket plus
 // n_words at the end (ascending).
-// bo (ARB_F_BO): allocate / release also set / clear the kCVp bit (Z17).
+// bo (ARB_F_BO): allocate / release also set / clear the kCVp bit (Z20).
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
                      FlushPlan& out, bool bo = false);

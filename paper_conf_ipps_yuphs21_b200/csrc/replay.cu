@@ -230,7 +230,7 @@ __device__ __forceinline__ uint32_t hslot(uint32_t w) { return (w * 2654435761u)
 template <bool PARTIAL, bool BO>
 __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
   uint32_t slot[RI], word[RI], pos[RI], op[RI], s_pre[RI];
-  uint32_t bom = 0;                // bit j: event j is a buffer overflow (ARB_F_BO, Z17)
+  uint32_t bom = 0;                // bit j: event j is a buffer overflow (ARB_F_BO, Z20)
   bool multi = false;
   const uint8_t* sh = S.shrel;
   uint2* hs = S.u.h.slot;
@@ -477,7 +477,7 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
       const uint32_t w = k & kWordMask;
       const bool h = (i == 0) || ((kin[i - 1] & kWordMask) != w);
       // ARB_F_BO: kCVp is constant within a step (range ops cut steps); a target
-      // access to a word without a CV is BO and the identity (Z17)
+      // access to a word without a CV is BO and the identity (Z20)
       const uint32_t full = (h || bo) ? __ldcg(sh + w) : 0u;
       const bool b = bo && ((k >> 30) & 2u) && !(full & kCVp);
       uint32_t v = b ? 0u : acc_summary(k >> 30);
@@ -751,7 +751,7 @@ __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t 
   return m;
 }
 
-// BO: ARB_F_BO contexts (the buffer-overflow extension, Z17) get their own
+// BO: ARB_F_BO contexts (the buffer-overflow extension, Z20) get their own
 // instance, so the default replay carries none of its checks.
 template <bool BO>
 __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p) {

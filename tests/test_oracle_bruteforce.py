@@ -47,7 +47,7 @@ def encode_seq(seq, base):
 
 def check_batch(orc, seqs, nwords, bo=False):
     """Concatenate the sequences on disjoint arrays, run the oracle once, compare per array.
-    bo: the buffer-overflow extension on both sides (reading Z17)."""
+    bo: the buffer-overflow extension on both sides (reading Z20)."""
     stride = 8 * nwords
     recs, expect, states, offsets = [], [], [], []
     for j, seq in enumerate(seqs):
@@ -141,7 +141,7 @@ def test_one_word_len6_reduced(orc):
 
 @pytest.mark.parametrize("nwords,length", [(1, 4), (2, 3)])
 def test_bo_exhaustive(orc, nwords, length):
-    """Buffer-overflow extension (Z17): the oracle's CVp bit and BO
+    """Buffer-overflow extension (Z20): the oracle's CVp bit and BO
     reports equal the value simulator's CV existence on every sequence (target
     accesses before any map, after release/delete, outside a 1-word section of
     a 2-word array), together with the UUM/USD reports and final states."""

@@ -270,7 +270,7 @@ def test_global_index(orc):
     assert res.triples() == [(w, r * 10 + 7, k) for w, r, k in expect]
 
 
-# ---- buffer-overflow extension (reading Z17) -----------------------
+# ---- buffer-overflow extension (reading Z20) -----------------------
 BO = 4
 
 

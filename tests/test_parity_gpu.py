@@ -15,7 +15,7 @@ pytestmark = pytest.mark.gpu
 def check(orc, rec, base, size, **kw):
     okw = {k: kw.pop(k) for k in ("dedup_first",) if k in kw}
     flags = (1 if okw.get("dedup_first") else 0) | kw.pop("flags", 0)
-    okw["detect_bo"] = bool(flags & 8)                    # ARB_F_BO <-> the oracle's extension (Z17)
+    okw["detect_bo"] = bool(flags & 8)                    # ARB_F_BO <-> the oracle's extension (Z20)
     exp = orc.replay(rec, base, size, **okw)
     rc, got, shadow, st = run_gpu(rec, base, size, flags=flags, **kw)
     assert rc == exp.rc
@@ -220,7 +220,7 @@ def test_untracked_words_ignored(orc):
     check(orc, rec, base + 256, span // 2)
 
 
-# ---- buffer-overflow extension (ARB_F_BO = 8, Z17) ---------------
+# ---- buffer-overflow extension (ARB_F_BO = 8, Z20) ---------------
 @pytest.mark.parametrize("write", [False, True])
 def test_bo_half_mapped_array(orc, write):
     """only the first half of the array is mapped, the kernel loops over all of it."""

@@ -38,9 +38,11 @@ METRICS = [
 ]
 
 
-def short(name):
-    n = name.split("(")[0].strip()
-    return n.replace("void ", "")
+def short(name, keep_template=False):
+    n = name.split("(")[0].strip().replace("void ", "")
+    if not keep_template and ("k_replay" in n or "k_partition" in n):
+        n = n.split("<")[0]             # k_replay<BO>: one row per kernel
+    return n
 
 
 def launches(path):
