@@ -229,6 +229,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--bo", action="store_true", help="enable the buffer-overflow extension (ARB_F_BO, Z20)")
     ap.add_argument("--cpu-records", type=int, default=300_000_000)
     ap.add_argument("--ref-sample", type=int, default=15_000_000)
     args = ap.parse_args()
@@ -237,7 +238,7 @@ def main():
 
     import torch
     import torch.distributed as dist
-    from paper_conf_ipps_yuphs21_b200 import Context, ARB_F_TIMING, reports_to_triples
+    from paper_conf_ipps_yuphs21_b200 import Context, ARB_F_TIMING, ARB_F_BO, reports_to_triples
     from paper_conf_ipps_yuphs21_b200.shard import nccl_unique_id
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -263,7 +264,7 @@ def main():
         dist.broadcast(buf, 0)
         uid = bytes(buf.cpu().numpy().tobytes())
     ctx = Context(lo * 8, (hi - lo) * 8, device=local, rank=rank, world=world, nccl_unique_id=uid,
-                  flags=ARB_F_TIMING, report_capacity=1 << 25)
+                  flags=ARB_F_TIMING | (ARB_F_BO if args.bo else 0), report_capacity=1 << 25)
     stream = torch.cuda.Stream(device=dev)
 
     def one_step(collect=False):
@@ -404,7 +405,7 @@ def main():
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-                "config": {"workload": args.workload, "scale": args.scale,
+                "config": {"workload": args.workload, "scale": args.scale, "buffer_overflow_ext": bool(args.bo),
                            "records_per_step": int(records_all), "word_events_per_step": int(word_events_all),
                            "access_word_events_per_step_rank0": int(s0["access_words"]),
                            "range_word_events_per_step_rank0": int(s0["range_words"]),
