@@ -7,6 +7,8 @@
 #include <algorithm>
 #include <chrono>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -569,6 +571,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     std::memcpy(ctl.data(), ctx->h_ctl.p, hst.n_ctl * sizeof(CtlRec));
     std::sort(ctl.begin(), ctl.end(), [](const CtlRec& a, const CtlRec& b) { return a.pos < b.pos; });
   }
+  const auto t_host1 = std::chrono::steady_clock::now();
   MapTable map = ctx->map;
   FlushPlan plan;
   resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_start, map, plan,
@@ -582,7 +585,15 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   S.range_ops = plan.range_ops.size();
   S.tasks = plan.tasks;
   S.ignored_words = hst.ignored_words + plan.ignored_words;
+  const auto t_host2 = std::chrono::steady_clock::now();
   build_items(ctx, plan, bucket_events);
+  if (getenv("ARB_HOST_PROFILE")) {
+    const auto t3 = std::chrono::steady_clock::now();
+    auto ms = [](auto a, auto b) { return std::chrono::duration<double, std::milli>(b - a).count(); };
+    fprintf(stderr, "arb host: ctl d2h+sort %.3f ms (%llu ctl), resolve %.3f ms (%zu range ops, %zu bucket ops), "
+            "items %.3f ms\n", ms(t_host0, t_host1), (unsigned long long)hst.n_ctl, ms(t_host1, t_host2),
+            plan.range_ops.size(), plan.ops.size(), ms(t_host2, t3));
+  }
   S.work_items = ctx->items.size() + ctx->slice_items.size();
   S.hot_buckets = ctx->hot.size();
   S.ms_host_control = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_host0).count();
