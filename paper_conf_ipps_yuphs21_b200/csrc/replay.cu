@@ -30,9 +30,7 @@ constexpr int RI = kReplayItems;             // events per thread per step
 constexpr int STEP = RT * RI;                // 2048 events per step
 static_assert(RT >= 256 && STEP <= 4096, "sort_pass digit loop and u16 offsets");
 constexpr int kWin = 2 * RT;                 // segment descriptors staged per step
-constexpr int kHTab = 2048;                  // slots of one fast-step hash table (load <= 1/2)
-constexpr int kHSlots = 2 * kHTab;           // two tables, used by alternate fast steps
-static_assert((kHTab / 2) % kReplayThreads == 0, "table clear: whole uint4 rows per thread");
+constexpr int kHSlots = 4096;                // hash slots (load <= 1/2)
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
 constexpr uint32_t kWordMask = 0x3FFFFFFFu;
 constexpr int kZSlots = 2048;                // summary-step hash slots (<= 1024 writes per step)
@@ -42,7 +40,7 @@ struct ReplaySmem {
   uint2 ev[2][STEP];              // double-buffered step events {key, pos} (cp.async)
   union {
     struct { uint32_t keyA[STEP], posA[STEP], keyB[STEP], posB[STEP]; uint16_t hist[RT / 32][256]; } s;
-    struct { uint2 slot[kHSlots]; } h;      // fast steps: written words {word, pos << 2 | op}, 2 tables
+    struct { uint2 slot[kHSlots]; } h;      // fast step: written words {word, pos << 2 | op}
     struct { uint32_t key[kZSlots], lastw[kZSlots], anyw[kZSlots]; } z;  // hot-slice summary step (K5)
   } u;
   uint32_t wstart[kWin];          // staged segment list window: global event index
@@ -216,7 +214,7 @@ __device__ __forceinline__ uint32_t classify_bits(uint32_t op, uint32_t before) 
 
 // hash slot of a word (Fibonacci hashing: consecutive words land far apart, so
 // the linear probe chains of a run's words stay short)
-__device__ __forceinline__ uint32_t hslot(uint32_t w) { return (w * 2654435761u) >> 21; }
+__device__ __forceinline__ uint32_t hslot(uint32_t w) { return (w * 2654435761u) >> 20; }
 
 // ---- fast step: at most one write per word -------------------------------------------
 // Returns false (and leaves the shadow untouched) if some word has two writes.
@@ -226,33 +224,22 @@ __device__ __forceinline__ uint32_t hslot(uint32_t w) { return (w * 2654435761u)
 // at the start of the step, or — if its word's single write precedes it — the
 // image of that write; the write event itself commits the word's final state.
 //
-// Alternate fast steps use the two tables: step k inserts into table `tsel`
-// and clears the other one, which step k-1 used (its probes ended before the
-// barrier that opened step k), so no reset barrier is needed.  A failed fast
-// step is followed by the sort step, which clears both.
-//
 // BO (ARB_F_BO) is a template parameter: deciding that a target access is a
 // buffer overflow needs its word's state before the inserts, which would put
 // the shadow-load latency in front of the hashing for every replay.
 template <bool PARTIAL, bool BO>
-__device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m,
-                                          uint32_t tsel) {
-  uint32_t word[RI], pos[RI], op[RI], s_pre[RI];
+__device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
+  uint32_t slot[RI], word[RI], pos[RI], op[RI], s_pre[RI];
   uint32_t bom = 0;                // bit j: event j is a buffer overflow (ARB_F_BO, Z20)
   bool multi = false;
   const uint8_t* sh = S.shrel;
-  uint2* hs = S.u.h.slot + tsel * kHTab;
-  {
-    uint4* other = reinterpret_cast<uint4*>(S.u.h.slot + (tsel ^ 1u) * kHTab);
-#pragma unroll
-    for (int k = 0; k < kHTab / 2 / RT; ++k) other[threadIdx.x + k * RT] = make_uint4(kEmpty, kEmpty, kEmpty, kEmpty);
-  }
+  uint2* hs = S.u.h.slot;
   uint32_t plo = 0, pw = 0;
   if (PARTIAL) { plo = S.part_lo; pw = S.part_hi - S.part_lo; }
 #pragma unroll
   for (int j = 0; j < RI; ++j) {   // shadow loads first: their latency overlaps the hashing
     const uint32_t i = threadIdx.x + j * RT;
-    word[j] = 0; pos[j] = 0; op[j] = 4; s_pre[j] = 0;
+    slot[j] = 0; word[j] = 0; pos[j] = 0; op[j] = 4; s_pre[j] = 0;
     if (i < m) {
       const uint2 e = ev[i];
       word[j] = e.x & kWordMask; op[j] = e.x >> 30; pos[j] = e.y;
@@ -263,35 +250,47 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
     }
   }
   // writes (WH = 1, WT = 3: odd ops) enter the table: slot {word, pos << 2 | op}
+  bool any_w = false;
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
     if (op[j] & 1u) {
+      any_w = true;
       uint32_t h = hslot(word[j]);
       for (;;) {
         const uint32_t old = atomicCAS(&hs[h].x, kEmpty, word[j]);
         if (old == kEmpty) break;
         if (old == word[j]) { multi = true; break; }        // a second write of the word
-        h = (h + 1) & (kHTab - 1);
+        h = (h + 1) & (kHSlots - 1);
       }
+      slot[j] = h;
       hs[h].y = (pos[j] << 2) | op[j];
     }
   }
-  if (__syncthreads_or(multi)) return false;              // the sort step rebuilds the area
+  any_w = __syncthreads_or(any_w);
+  if (any_w && __syncthreads_or(multi)) {
+#pragma unroll
+    for (int j = 0; j < RI; ++j)
+      if (op[j] & 1u) hs[slot[j]] = make_uint2(kEmpty, kEmpty);
+    __syncthreads();
+    return false;
+  }
   uint32_t fk[RI];
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
     const uint32_t s0 = s_pre[j] & 15u;
     uint32_t before = s0;
     if (op[j] == OP_RH || op[j] == OP_RT) {
-      uint32_t h = hslot(word[j]);
-      for (;;) {                                            // probe for the word's write
-        const uint2 k = hs[h];
-        if (k.x == word[j]) {
-          if ((k.y >> 2) < pos[j]) before = vsm_write_op(k.y & 3u, s0);
-          break;
+      if (any_w) {
+        uint32_t h = hslot(word[j]);
+        for (;;) {                                          // probe for the word's write
+          const uint2 k = hs[h];
+          if (k.x == word[j]) {
+            if ((k.y >> 2) < pos[j]) before = vsm_write_op(k.y & 3u, s0);
+            break;
+          }
+          if (k.x == kEmpty) break;
+          h = (h + 1) & (kHSlots - 1);
         }
-        if (k.x == kEmpty) break;
-        h = (h + 1) & (kHTab - 1);
       }
     } else if (op[j] & 1u) {
       __stcg(const_cast<uint8_t*>(sh) + word[j], (uint8_t)(vsm_write_op(op[j], s0) | (BO ? (s_pre[j] & kCVp) : 0u)));
@@ -299,14 +298,20 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
     fk[j] = ((bom >> j) & 1u) ? 4u : classify_bits(op[j], before);
   }
   emit_faults(p, fk, word, pos, S.bucket_base);
-  // the caller's next barrier orders this step's probes before the next step's clear
+  if (any_w) {
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < RI; ++j)
+      if (op[j] & 1u) hs[slot[j]] = make_uint2(kEmpty, kEmpty);
+  }
+  // the caller's next barrier orders this reset before the next step's inserts
   return true;
 }
 
 // the fast step of a word-range part (rare: range-heavy buckets), out of line
 template <bool BO>
-__device__ bool step_fast_partial(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m, uint32_t tsel) {
-  return step_fast<true, BO>(S, p, ev, m, tsel);
+__device__ bool step_fast_partial(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
+  return step_fast<true, BO>(S, p, ev, m);
 }
 
 // ---- sort step -------------------------------------------------------------------------
@@ -754,7 +759,6 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
   ReplaySmem& S = *reinterpret_cast<ReplaySmem*>(smem_raw);
   const uint32_t tid = threadIdx.x;
   hash_clear(S);
-  uint32_t tsel = 0;                   // fast-step hash table of the next fast step (alternates across items too)
   for (;;) {
     if (tid == 0) {
       const unsigned long long w = atomicAdd(&p.st->work, 1ull);
@@ -839,10 +843,8 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       if (mode == kItemSummary) {
         step_summary(S, ev, cut);
       } else {
-        const bool fast = S.partial ? step_fast_partial<BO>(S, p, ev, cut, tsel)
-                                    : step_fast<false, BO>(S, p, ev, cut, tsel);
-        if (fast) tsel ^= 1u;
-        else step_sort<BO>(S, p, ev, cut);
+        const bool fast = S.partial ? step_fast_partial<BO>(S, p, ev, cut) : step_fast<false, BO>(S, p, ev, cut);
+        if (!fast) step_sort<BO>(S, p, ev, cut);
         if (tid == 0) atomicAdd(fast ? &p.st->steps_fast : &p.st->steps_sort, 1ull);
       }
       e0 += cut;
