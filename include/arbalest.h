@@ -155,6 +155,11 @@ int arb_submit_events(arb_ctx ctx, const arb_event* ev, uint64_t n,
 /* Replay the pending batch: decode + partition, control resolution (Table I),
  * per-address segmented scan + classification, MIR join, canonical report
  * compaction, and (world > 1) the allgather of per-rank report counts.
+ * Flush points may fall anywhere outside a TASK_BEGIN..TASK_END block: nowait
+ * instances that ended but are not joined yet are carried into the next flush
+ * (their access summary stays on the device) and keep racing until their SYNC
+ * (Z19), so the union of the flushes' reports equals the replay of
+ * the whole trace.  A block still open at the end of a flush is ARB_EOPEN.
  *  n_reports_local       this rank's report count (exact even if truncated)
  *  report_offset_global  exclusive prefix of the counts over ranks (0 if world 1)
  * Both may be NULL.  Synchronizes `stream`.  The batch is consumed.  Returns

@@ -141,6 +141,11 @@ struct arb_ctx_s {
   DevBuf<RangeRef> m_own, m_win, m_rr;
   DevBuf<unsigned long long> hkeys;
   DevBuf<uint32_t> hvals;
+  // N2: nowait instances unjoined at the end of the last flush (committed with the map table)
+  std::vector<CarriedInst> carried;
+  DevBuf<uint4> carry_ent, carry_next;        // their access summaries {word lo, word hi, carried idx, flag}
+  uint64_t n_carry = 0;
+  DevBuf<uint32_t> m_cmap, m_co_of;
   uint64_t ctl_cap = 1 << 16;
   uint64_t cand_cap = 1 << 24;
   MapTable map;
@@ -257,6 +262,7 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   ctx->m_rr_cum.release(); ctx->m_ins_inst.release(); ctx->m_qry_open_start.release(); ctx->m_open_list.release();
   ctx->m_own_start.release(); ctx->m_win_start.release(); ctx->m_own.release(); ctx->m_win.release();
   ctx->m_rr.release(); ctx->hkeys.release(); ctx->hvals.release(); ctx->counts.release();
+  ctx->carry_ent.release(); ctx->carry_next.release(); ctx->m_cmap.release(); ctx->m_co_of.release();
   ctx->d_bin_map.release(); ctx->d_items.release(); ctx->h_items.release(); ctx->h_weight.release();
   ctx->d_slice_items.release(); ctx->h_slice_items.release(); ctx->d_hot.release(); ctx->h_hot.release();
   ctx->d_hot_off.release(); ctx->h_hot_off.release(); ctx->hot_F.release(); ctx->hot_P.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_cut.release();
@@ -575,7 +581,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   MapTable map = ctx->map;
   FlushPlan plan;
   resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_start, map, plan,
-                  (ctx->cfg.flags & ARB_F_BO) != 0);
+                  (ctx->cfg.flags & ARB_F_BO) != 0, &ctx->carried);
   if (plan.rc != 0) {
     CK(cudaStreamSynchronize(s), "sync");
     reset_batch(ctx);
@@ -645,11 +651,13 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   S.steps_sort = hst.steps_sort;
 
   // ---- A6: MIR join ---------------------------------------------------------------
-  uint64_t n_mir = 0;
-  if (!plan.mir.empty()) {
+  uint64_t n_mir = 0, n_carry_next = 0;
+  const bool carry_in = ctx->n_carry && !plan.carry_in_dense.empty();
+  if (!plan.mir.empty() || carry_in || !plan.carry_out.empty()) {
     MirPlanH& M = plan.mir;
     uint64_t hcap = 1;
-    while (hcap < 2 * (2 * M.n_ins_pos + 1)) hcap <<= 1;
+    while (hcap < 2 * (2 * M.n_ins_pos + (carry_in ? ctx->n_carry : 0) + 1)) hcap <<= 1;
+    if (carry_in) CK(upload(ctx->m_cmap, plan.carry_in_dense, s), "mir carry map");
     CK(ctx->hkeys.ensure(hcap), "alloc hash");
     CK(ctx->hvals.ensure(hcap), "alloc hash");
     CK(upload(ctx->m_ins_lo, M.ins_lo, s), "mir"); CK(upload(ctx->m_ins_cum, M.ins_cum, s), "mir");
@@ -673,6 +681,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
       mp.win_start = ctx->m_win_start.p; mp.win_ops = ctx->m_win.p;
       mp.hkeys = ctx->hkeys.p; mp.hvals = ctx->hvals.p; mp.hmask = hcap - 1;
       mp.rr = ctx->m_rr.p; mp.rr_cum = ctx->m_rr_cum.p; mp.n_rr = (uint32_t)M.rr.size();
+      mp.carry = ctx->carry_ent.p; mp.n_carry = carry_in ? ctx->n_carry : 0; mp.cmap = ctx->m_cmap.p;
       mp.cand = ctx->cand.p + kept_vsm; mp.cand_cap = ctx->cand.cap - kept_vsm; mp.st = ctx->dstats.p;
       CK(launch_mir(mp, M.n_ins_pos, M.n_qry_pos, M.n_rr_words, s, &launches), "k_mir");
       unsigned long long c = 0;
@@ -687,6 +696,19 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
       CK(cudaStreamSynchronize(s), "copy sync");
       ctx->cand.release();
       ctx->cand = bigger;
+    }
+    if (!plan.carry_out.empty()) {
+      // N2: the access summaries of the instances still unjoined go to the next flush
+      CK(upload(ctx->m_co_of, plan.dense_carry_out, s), "carry map");
+      CK(ctx->carry_next.ensure(hcap), "alloc carry");
+      CK(cudaMemsetAsync(&ctx->dstats.p->n_carry_out, 0, sizeof(unsigned long long), s), "carry count");
+      CK(launch_carry_extract(ctx->hkeys.p, ctx->hvals.p, hcap, ctx->m_co_of.p, ctx->carry_next.p,
+                              &ctx->dstats.p->n_carry_out, s), "carry extract");
+      launches += 1;
+      unsigned long long c = 0;
+      CK(cudaMemcpyAsync(&c, &ctx->dstats.p->n_carry_out, sizeof(c), cudaMemcpyDeviceToHost, s), "carry d2h");
+      CK(cudaStreamSynchronize(s), "carry sync");
+      n_carry_next = c;
     }
   }
   if (timing) cudaEventRecord(ctx->ev[4], s);
@@ -747,6 +769,9 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     cudaEventElapsedTime(&ms, ctx->ev[0], ctx->ev[6]); S.ms_total = ms;
   }
   ctx->map.swap(map);
+  ctx->carried.swap(plan.carry_out);          // N2: committed with the map table
+  std::swap(ctx->carry_ent, ctx->carry_next);
+  ctx->n_carry = n_carry_next;
   ctx->next_index += n;
   ctx->flushed = true;
   S.reports = ctx->n_reports;

@@ -82,7 +82,8 @@ struct DevStats {
   unsigned long long n_mir_cand;
   unsigned long long steps_fast, steps_sort;
   unsigned long long n_segs;          // (chunk, bucket) segment entries written by k_partition
-  unsigned long long pad[4];
+  unsigned long long n_carry_out;     // N2: access summaries of instances carried into the next flush
+  unsigned long long pad[3];
 };
 
 // control record extracted by the partition kernel
@@ -161,6 +162,9 @@ struct MirParams {
   unsigned long long* hkeys; uint32_t* hvals; uint64_t hmask;
   // (ii) range-vs-range emission list
   const RangeRef* rr; const uint64_t* rr_cum; uint32_t n_rr;
+  // N2: access summaries of instances carried in from earlier flushes
+  // {word lo, word hi, carried index, write flag}; cmap: carried index -> dense index
+  const uint4* carry; uint64_t n_carry; const uint32_t* cmap;
   uint4* cand; uint64_t cand_cap;
   DevStats* st;
 };
@@ -187,6 +191,11 @@ cudaError_t launch_carry(const uint4* hot, uint32_t n_hot, uint32_t max_span, co
                          cudaStream_t s);
 cudaError_t launch_mir(const MirParams& p, uint64_t n_ins_pos, uint64_t n_qry_pos, uint64_t n_rr_words,
                        cudaStream_t s, int* launches);
+// N2: the hash entries of the instances still unjoined at the end of the flush
+// (dense index d with co_of[d] != 0xFFFFFFFF) -> out {word lo, word hi, co_of[d], flag};
+// *n_out counts them (out holds hcap entries)
+cudaError_t launch_carry_extract(const unsigned long long* hkeys, const uint32_t* hvals, uint64_t hcap,
+                                 const uint32_t* co_of, uint4* out, unsigned long long* n_out, cudaStream_t s);
 // report compaction: sorts candidates, removes duplicates, optional dedup-first,
 // maps positions to global indices and writes arb_report records.
 struct CompactParams {

@@ -40,14 +40,22 @@ struct Emitter {
 
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
-                     FlushPlan& out, bool bo) {
+                     FlushPlan& out, bool bo, const std::vector<CarriedInst>* carried_in) {
   const uint32_t n_buckets = (uint32_t)bucket_start.size() - 1;
   out = FlushPlan();
   Emitter em{base_word, n_words, &out};
-  // task instances (1-based; 0 = host)
+  // task instances (1-based; 0 = host); instances 1..nc are the carried-in ones,
+  // which ended before this flush (t_begin = t_end = kBefore)
+  constexpr uint64_t kBefore = UINT64_MAX - 1;
+  const uint32_t nc = carried_in ? (uint32_t)carried_in->size() : 0u;
   std::vector<uint64_t> t_begin{0}, t_end{0}, t_join{0};
   std::vector<uint32_t> t_id{0};
   std::vector<uint32_t> unjoined;
+  for (uint32_t c = 0; c < nc; ++c) {
+    t_begin.push_back(kBefore); t_end.push_back(kBefore); t_join.push_back(UINT64_MAX);
+    t_id.push_back((*carried_in)[c].task_id);
+    unjoined.push_back(c + 1);
+  }
   uint32_t open = 0;
   auto fail = [&](int rc, uint64_t pos, const char* why) {
     out.rc = rc; out.err_pos = pos; out.err = why;
@@ -124,9 +132,13 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   }
   if (open) return fail(ARB_EOPEN, n_records, "a task block is still open at the end of the flush");
   const uint32_t ninst = (uint32_t)t_begin.size() - 1;
-  out.tasks = ninst;
+  out.tasks = ninst - nc;
+  // instances not joined in this flush race with everything up to its end and
+  // are carried into the next flush (N2)
+  std::vector<uint8_t> carry(ninst + 1, 0);
   for (uint32_t q = 1; q <= ninst; ++q)
-    if (t_join[q] == UINT64_MAX) t_join[q] = n_records;   // never joined in this flush
+    if (t_join[q] == UINT64_MAX) { t_join[q] = n_records; carry[q] = 1; }
+  auto wstart = [&](uint32_t q) { return t_end[q] == kBefore ? 0 : t_end[q] + 1; };   // window [wstart, join)
 
   // ---- per-bucket CSR of range ops (trace order kept inside each bucket) ----
   auto first_bucket = [&](uint64_t w) {   // bucket holding relative word w
@@ -146,18 +158,23 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   }
 
   // ---- MIR join plan (Theorem 1) -------------------------------
-  // An instance q is racy if its window (end_q, join_q) holds at least one record.
+  // An instance q is racy if its window (end_q, join_q) holds at least one
+  // record; carried-out instances are listed too (their access summary is
+  // extracted from the join's hash after the MIR kernels).
   MirPlanH& M = out.mir;
   std::vector<uint32_t> dense(ninst + 1, 0xFFFFFFFFu);
   std::vector<uint32_t> racy;
   for (uint32_t q = 1; q <= ninst; ++q)
-    if (t_join[q] > t_end[q] + 1) { dense[q] = (uint32_t)racy.size(); racy.push_back(q); }
+    if (t_join[q] > wstart(q) || carry[q]) { dense[q] = (uint32_t)racy.size(); racy.push_back(q); }
   M.n_racy = (uint32_t)racy.size();
+  out.carry_in_dense.resize(nc);
+  for (uint32_t c = 0; c < nc; ++c) out.carry_in_dense[c] = dense[c + 1];
+  out.dense_carry_out.assign(racy.size(), 0xFFFFFFFFu);
   if (racy.empty()) return;
-  // insert ranges: records strictly inside each racy block
+  // insert ranges: records strictly inside each listed block of this flush
   M.ins_cum.push_back(0);
   for (uint32_t q : racy) {
-    if (t_end[q] > t_begin[q] + 1) {
+    if (t_end[q] != kBefore && t_end[q] > t_begin[q] + 1) {
       M.ins_lo.push_back(t_begin[q] + 1);
       M.ins_inst.push_back(dense[q]);
       M.ins_cum.push_back(M.ins_cum.back() + (t_end[q] - t_begin[q] - 1));
@@ -173,11 +190,21 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
     if (r.inst && dense[r.inst] != 0xFFFFFFFFu)
       own[dense[r.inst]].push_back(RangeRef{r.lo, r.hi, r.pos, r.inst});
   }
+  for (uint32_t c = 0; c < nc; ++c)          // a carried instance's range ops from earlier flushes
+    if (dense[c + 1] != 0xFFFFFFFFu)
+      own[dense[c + 1]].insert(own[dense[c + 1]].end(), (*carried_in)[c].own.begin(), (*carried_in)[c].own.end());
+  for (size_t d = 0; d < racy.size(); ++d) {
+    uint32_t q = racy[d];
+    if (!carry[q]) continue;
+    out.dense_carry_out[d] = (uint32_t)out.carry_out.size();
+    out.carry_out.push_back(CarriedInst{t_id[q], own[d]});
+  }
   for (size_t d = 0; d < racy.size(); ++d) {
     uint32_t q = racy[d];
     // range ops are in trace order: binary search the window
-    auto first = std::upper_bound(out.range_ops.begin(), out.range_ops.end(), (uint32_t)t_end[q],
-                                  [](uint32_t p, const RangeOpH& r) { return p < r.pos; });
+    auto first = t_end[q] == kBefore ? out.range_ops.begin()
+                 : std::upper_bound(out.range_ops.begin(), out.range_ops.end(), (uint32_t)t_end[q],
+                                    [](uint32_t p, const RangeOpH& r) { return p < r.pos; });
     for (auto it = first; it != out.range_ops.end() && it->pos < t_join[q]; ++it)
       win[d].push_back(RangeRef{it->lo, it->hi, it->pos, it->inst});
   }
@@ -201,7 +228,8 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   std::vector<std::pair<uint64_t, int64_t>> evs;   // (position, +/-(dense+1))
   for (size_t d = 0; d < racy.size(); ++d) {
     uint32_t q = racy[d];
-    evs.push_back({t_end[q] + 1, (int64_t)d + 1});
+    if (t_join[q] <= wstart(q)) continue;     // a carried-out instance with an empty window here
+    evs.push_back({wstart(q), (int64_t)d + 1});
     evs.push_back({t_join[q], -((int64_t)d + 1)});
   }
   std::sort(evs.begin(), evs.end());

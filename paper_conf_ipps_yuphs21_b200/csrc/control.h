@@ -32,11 +32,19 @@ struct MirPlanH {
   bool empty() const { return n_ins_pos == 0 && n_qry_pos == 0 && n_rr_words == 0; }
 };
 
+// A nowait task instance that ended in an earlier flush and is not joined yet
+// (SURVEY §8(f) N2): its own range ops (relative words; pos unused) travel on the
+// host, its (word, write-class) access summary on the device (ctx->carry_ent).
+struct CarriedInst { uint32_t task_id; std::vector<RangeRef> own; };
+
 struct FlushPlan {
   std::vector<RangeOpH> range_ops;       // in trace order
   std::vector<uint32_t> ops_start;       // per bucket CSR
   std::vector<BucketOp> ops;
   MirPlanH mir;
+  std::vector<uint32_t> carry_in_dense;  // per carried-in instance: its MIR dense index, or 0xFFFFFFFF
+  std::vector<uint32_t> dense_carry_out; // per MIR dense index: its carried-out index, or 0xFFFFFFFF
+  std::vector<CarriedInst> carry_out;    // instances still unjoined at the end of this flush
   uint64_t range_words = 0, ignored_words = 0, tasks = 0;
   int rc = 0; uint64_t err_pos = 0; std::string err;
 };
@@ -47,8 +55,11 @@ struct FlushPlan {
 // `bucket_start` holds the first relative word of every address bucket plus
 // n_words at the end (ascending).
 // bo (ARB_F_BO): allocate / release also set / clear the kCVp bit (Z20).
+// carried_in: instances unjoined at the end of the previous flush (their window
+// in this flush starts at position 0); instances unjoined at the end of this one
+// are returned in out.carry_out instead of being treated as joined (Z19).
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
-                     FlushPlan& out, bool bo = false);
+                     FlushPlan& out, bool bo = false, const std::vector<CarriedInst>* carried_in = nullptr);
 
 }  // namespace arb

@@ -57,6 +57,53 @@ __global__ void k_mir_insert(MirParams p, uint64_t n_pos) {
   }
 }
 
+// N2: the access summaries of instances carried in from earlier flushes enter
+// the hash like their records would, and (iii) window range ops covering them race.
+__global__ void k_mir_carry_insert(MirParams p) {
+  for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < p.n_carry;
+       g += (uint64_t)gridDim.x * blockDim.x) {
+    const uint4 e = p.carry[g];
+    const uint32_t qd = p.cmap[e.z];
+    if (qd == 0xFFFFFFFFu) continue;            // joined before this flush's first record
+    const uint64_t w = (uint64_t)e.x | ((uint64_t)e.y << 32);
+    unsigned long long key = ((unsigned long long)w << 20) | (qd + 1);
+    uint64_t h = hslot(key, p.hmask);
+    for (;;) {
+      unsigned long long old = atomicCAS(&p.hkeys[h], 0ull, key);
+      if (old == 0ull || old == key) break;
+      h = (h + 1) & p.hmask;
+    }
+    if (e.w) atomicOr(&p.hvals[h], 1u);
+    for (uint32_t j = p.win_start[qd]; j < p.win_start[qd + 1]; ++j) {
+      RangeRef rr = p.win_ops[j];
+      if (w >= rr.lo && w < rr.hi) emit_mir(p, w, rr.pos);
+    }
+  }
+}
+
+// N2: summaries of the instances carried out of this flush
+__global__ void k_mir_carry_extract(const unsigned long long* hkeys, const uint32_t* hvals, uint64_t hcap,
+                                    const uint32_t* co_of, uint4* out, unsigned long long* n_out) {
+  for (uint64_t h = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; h < hcap;
+       h += (uint64_t)gridDim.x * blockDim.x) {
+    const unsigned long long key = hkeys[h];
+    if (!key) continue;
+    const uint32_t co = co_of[(uint32_t)(key & 0xFFFFFu) - 1];
+    if (co == 0xFFFFFFFFu) continue;
+    const uint64_t w = key >> 20;
+    const unsigned long long slot = atomicAdd(n_out, 1ull);
+    out[slot] = make_uint4((uint32_t)w, (uint32_t)(w >> 32), co, hvals[h] & 1u);
+  }
+}
+
+cudaError_t launch_carry_extract(const unsigned long long* hkeys, const uint32_t* hvals, uint64_t hcap,
+                                 const uint32_t* co_of, uint4* out, unsigned long long* n_out, cudaStream_t s) {
+  const uint64_t g = (hcap + 255) / 256;
+  k_mir_carry_extract<<<(unsigned)(g > 148 * 64 ? 148 * 64 : (g ? g : 1)), 256, 0, s>>>(hkeys, hvals, hcap, co_of,
+                                                                                        out, n_out);
+  return cudaGetLastError();
+}
+
 // (iv) + (i): access ops inside race windows against the open instances'
 // access ops (hash) and range ops (lists).
 __global__ void k_mir_query(MirParams p, uint64_t n_pos) {
@@ -105,6 +152,7 @@ cudaError_t launch_mir(const MirParams& p, uint64_t n_ins_pos, uint64_t n_qry_po
                        cudaStream_t s, int* launches) {
   auto grid = [](uint64_t n) { uint64_t g = (n + 255) / 256; return (unsigned)(g > 148 * 64 ? 148 * 64 : (g ? g : 1)); };
   if (n_ins_pos) { k_mir_insert<<<grid(n_ins_pos), 256, 0, s>>>(p, n_ins_pos); ++*launches; }
+  if (p.n_carry) { k_mir_carry_insert<<<grid(p.n_carry), 256, 0, s>>>(p); ++*launches; }
   if (n_qry_pos) { k_mir_query<<<grid(n_qry_pos), 256, 0, s>>>(p, n_qry_pos); ++*launches; }
   if (n_rr_words) { k_mir_ranges<<<grid(n_rr_words), 256, 0, s>>>(p, n_rr_words); ++*launches; }
   return cudaGetLastError();

@@ -294,3 +294,74 @@ def test_bo_patterns(orc):
                 k += 1
     exp, st = check(orc, tb.array(), base, k * region, flags=8)
     assert {t[2] for t in exp.triples()} == {4} and st["reports_bo"] == len(exp.triples())
+
+
+# ---- N2: flushes between a nowait block's end and its join ------------
+def _cuts_outside_blocks(rec, k, seed):
+    """k random flush points that are not inside a TASK_BEGIN..TASK_END block
+    (an open block at a flush end is still ARB_EOPEN); they may fall between a
+    block's end and its taskwait, so unjoined instances cross flushes."""
+    op = (rec[:, 0] >> np.uint64(48)) & np.uint64(0xFF)
+    depth = np.cumsum((op == 12).astype(np.int64) - (op == 13).astype(np.int64))
+    ok = np.nonzero(depth == 0)[0] + 1                    # cut after record i: outside any block
+    ok = ok[ok < rec.shape[0]]
+    rs = np.random.default_rng(seed)
+    return sorted(set(int(x) for x in rs.choice(ok, size=min(k, ok.size), replace=False)))
+
+
+def _unjoined_across(rec, cuts):
+    """How many cuts separate a TASK_END from its join."""
+    op = (rec[:, 0] >> np.uint64(48)) & np.uint64(0xFF)
+    ends = np.nonzero(op == 13)[0]
+    syncs = np.nonzero(op == 14)[0]
+    n = 0
+    for e in ends:
+        j = syncs[syncs > e]
+        j = j[0] if j.size else rec.shape[0]
+        n += sum(1 for c in cuts if e < c <= j)
+    return n
+
+
+@pytest.mark.parametrize("seed", range(16))
+def test_flush_cuts_unjoined_tasks_fuzz(orc, seed):
+    """The union of the flushes' reports equals the whole-trace oracle for any
+    flush points outside task blocks (N2: unjoined instances are carried across)."""
+    from gen.fuzz import random_program
+    rec, base, span = random_program(4000 + seed, p_task=0.4)
+    exp = orc.replay(rec, base, span)
+    cuts = _cuts_outside_blocks(rec, 6, seed)
+    rc, got, shadow, st = run_gpu(rec, base, span, flush_points=cuts)
+    assert rc == exp.rc                          # a malformed program fails in the flush holding the error
+    if rc == 0:
+        assert sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+def test_flush_cuts_unjoined_tasks_config2(orc):
+    from gen.configs import config2
+    rec, base, size = config2(reps=2)
+    exp = orc.replay(rec, base, size)
+    cuts = _cuts_outside_blocks(rec, 40, 7)
+    assert _unjoined_across(rec, cuts) > 0
+    rc, got, shadow, st = run_gpu(rec, base, size, flush_points=cuts)
+    assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+def test_flush_between_end_and_join(orc):
+    """Fig. 2 shape across three flushes: the nowait write (flush 1), the racy host
+    read (flush 2), the taskwait (flush 3): the MIR at the host read is reported."""
+    from gen.trace import MAP, TraceBuilder
+    A = 0x4000
+    tb = TraceBuilder()
+    tb.wh(A); tb.enter(MAP.TOFROM, A, 64)
+    tb.task_begin(7); tb.wt(A); tb.task_end(7)
+    c1 = len(tb)
+    i_race = tb.rh(A + 0)
+    tb.wh(A + 8)
+    c2 = len(tb)
+    tb.sync(7)
+    tb.exit(MAP.TOFROM, A, 64)
+    rec = tb.array()
+    exp = orc.replay(rec, A, 64)
+    assert (A // 8, i_race, 3) in exp.triples()
+    rc, got, shadow, st = run_gpu(rec, A, 64, flush_points=[c1, c2])
+    assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
