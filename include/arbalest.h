@@ -69,7 +69,8 @@ enum arb_status {
   ARB_EMAP = -4,      /* map clause partially overlaps a present entry (Z6)          */
   ARB_ETRACE = -5,    /* malformed trace (Z18)                              */
   ARB_ESTATE = -6,    /* call out of order (e.g. get_reports before any flush)        */
-  ARB_EOPEN = -7      /* a TASK_BEGIN block is still open at the end of the flush     */
+  ARB_EOPEN = -7      /* reserved: open blocks are carried across flushes (Z19); the
+                         oracle returns it for a whole trace that ends inside a block */
 };
 /* After ARB_EMAP / ARB_ETRACE / ARB_EOPEN the pending batch is discarded, the
  * committed shadow is unchanged and the context stays usable.  After ARB_ECUDA
@@ -155,11 +156,11 @@ int arb_submit_events(arb_ctx ctx, const arb_event* ev, uint64_t n,
 /* Replay the pending batch: decode + partition, control resolution (Table I),
  * per-address segmented scan + classification, MIR join, canonical report
  * compaction, and (world > 1) the allgather of per-rank report counts.
- * Flush points may fall anywhere outside a TASK_BEGIN..TASK_END block: nowait
- * instances that ended but are not joined yet are carried into the next flush
- * (their access summary stays on the device) and keep racing until their SYNC
- * (Z19), so the union of the flushes' reports equals the replay of
- * the whole trace.  A block still open at the end of a flush is ARB_EOPEN.
+ * Flush points may fall anywhere, also inside a TASK_BEGIN..TASK_END block:
+ * nowait instances whose block is still open or that ended but are not joined
+ * yet are carried into the next flush (their access summary stays on the
+ * device) and keep racing until their SYNC (Z19), so the union of the
+ * flushes' reports equals the replay of the whole trace.
  *  n_reports_local       this rank's report count (exact even if truncated)
  *  report_offset_global  exclusive prefix of the counts over ranks (0 if world 1)
  * Both may be NULL.  Synchronizes `stream`.  The batch is consumed.  Returns

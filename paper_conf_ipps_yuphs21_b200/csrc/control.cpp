@@ -44,19 +44,21 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   const uint32_t n_buckets = (uint32_t)bucket_start.size() - 1;
   out = FlushPlan();
   Emitter em{base_word, n_words, &out};
-  // task instances (1-based; 0 = host); instances 1..nc are the carried-in ones,
-  // which ended before this flush (t_begin = t_end = kBefore)
-  constexpr uint64_t kBefore = UINT64_MAX - 1;
+  // task instances (1-based; 0 = host); instances 1..nc are the carried-in ones:
+  // they began before this flush (t_begin = kBefore) and either ended before it
+  // (t_end = kBefore) or are still open (t_end = kOpen until their TASK_END)
+  constexpr uint64_t kBefore = UINT64_MAX - 1, kOpen = UINT64_MAX - 2;
   const uint32_t nc = carried_in ? (uint32_t)carried_in->size() : 0u;
   std::vector<uint64_t> t_begin{0}, t_end{0}, t_join{0};
   std::vector<uint32_t> t_id{0};
   std::vector<uint32_t> unjoined;
-  for (uint32_t c = 0; c < nc; ++c) {
-    t_begin.push_back(kBefore); t_end.push_back(kBefore); t_join.push_back(UINT64_MAX);
-    t_id.push_back((*carried_in)[c].task_id);
-    unjoined.push_back(c + 1);
-  }
   uint32_t open = 0;
+  for (uint32_t c = 0; c < nc; ++c) {
+    const bool op_ = (*carried_in)[c].open;
+    t_begin.push_back(kBefore); t_end.push_back(op_ ? kOpen : kBefore); t_join.push_back(UINT64_MAX);
+    t_id.push_back((*carried_in)[c].task_id);
+    if (op_) open = c + 1; else unjoined.push_back(c + 1);
+  }
   auto fail = [&](int rc, uint64_t pos, const char* why) {
     out.rc = rc; out.err_pos = pos; out.err = why;
   };
@@ -69,7 +71,7 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
       case OP_TASK_BEGIN:
         if (open) return fail(ARB_ETRACE, c.pos, "TASK_BEGIN inside an open task block");
         if (tid == 0 || tid == kSyncAll) return fail(ARB_ETRACE, c.pos, "TASK_BEGIN with task id 0 or 0xFFFF");
-        t_begin.push_back(c.pos); t_end.push_back(0); t_join.push_back(UINT64_MAX); t_id.push_back(tid);
+        t_begin.push_back(c.pos); t_end.push_back(kOpen); t_join.push_back(UINT64_MAX); t_id.push_back(tid);
         open = (uint32_t)(t_begin.size() - 1);
         break;
       case OP_TASK_END:
@@ -130,7 +132,8 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
         return fail(ARB_ETRACE, c.pos, "unknown control op");
     }
   }
-  if (open) return fail(ARB_EOPEN, n_records, "a task block is still open at the end of the flush");
+  // a block still open at the end of the flush is carried (N2): its records so
+  // far are its own ops, its window starts after its TASK_END in a later flush
   const uint32_t ninst = (uint32_t)t_begin.size() - 1;
   out.tasks = ninst - nc;
   // instances not joined in this flush race with everything up to its end and
@@ -139,6 +142,7 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   for (uint32_t q = 1; q <= ninst; ++q)
     if (t_join[q] == UINT64_MAX) { t_join[q] = n_records; carry[q] = 1; }
   auto wstart = [&](uint32_t q) { return t_end[q] == kBefore ? 0 : t_end[q] + 1; };   // window [wstart, join)
+  auto has_window = [&](uint32_t q) { return t_end[q] != kOpen && t_join[q] > wstart(q); };
 
   // ---- per-bucket CSR of range ops (trace order kept inside each bucket) ----
   auto first_bucket = [&](uint64_t w) {   // bucket holding relative word w
@@ -165,19 +169,22 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   std::vector<uint32_t> dense(ninst + 1, 0xFFFFFFFFu);
   std::vector<uint32_t> racy;
   for (uint32_t q = 1; q <= ninst; ++q)
-    if (t_join[q] > wstart(q) || carry[q]) { dense[q] = (uint32_t)racy.size(); racy.push_back(q); }
+    if (has_window(q) || carry[q]) { dense[q] = (uint32_t)racy.size(); racy.push_back(q); }
   M.n_racy = (uint32_t)racy.size();
   out.carry_in_dense.resize(nc);
   for (uint32_t c = 0; c < nc; ++c) out.carry_in_dense[c] = dense[c + 1];
   out.dense_carry_out.assign(racy.size(), 0xFFFFFFFFu);
   if (racy.empty()) return;
-  // insert ranges: records strictly inside each listed block of this flush
+  // insert ranges: the records of each listed block that lie in this flush
   M.ins_cum.push_back(0);
   for (uint32_t q : racy) {
-    if (t_end[q] != kBefore && t_end[q] > t_begin[q] + 1) {
-      M.ins_lo.push_back(t_begin[q] + 1);
+    if (t_end[q] == kBefore) continue;                       // ended in an earlier flush
+    const uint64_t lo = t_begin[q] == kBefore ? 0 : t_begin[q] + 1;
+    const uint64_t hi = t_end[q] == kOpen ? n_records : t_end[q];
+    if (hi > lo) {
+      M.ins_lo.push_back(lo);
       M.ins_inst.push_back(dense[q]);
-      M.ins_cum.push_back(M.ins_cum.back() + (t_end[q] - t_begin[q] - 1));
+      M.ins_cum.push_back(M.ins_cum.back() + (hi - lo));
     }
   }
   M.n_ins_pos = M.ins_cum.back();
@@ -197,10 +204,11 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
     uint32_t q = racy[d];
     if (!carry[q]) continue;
     out.dense_carry_out[d] = (uint32_t)out.carry_out.size();
-    out.carry_out.push_back(CarriedInst{t_id[q], own[d]});
+    out.carry_out.push_back(CarriedInst{t_id[q], own[d], t_end[q] == kOpen});
   }
   for (size_t d = 0; d < racy.size(); ++d) {
     uint32_t q = racy[d];
+    if (!has_window(q)) continue;
     // range ops are in trace order: binary search the window
     auto first = t_end[q] == kBefore ? out.range_ops.begin()
                  : std::upper_bound(out.range_ops.begin(), out.range_ops.end(), (uint32_t)t_end[q],
@@ -228,7 +236,7 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   std::vector<std::pair<uint64_t, int64_t>> evs;   // (position, +/-(dense+1))
   for (size_t d = 0; d < racy.size(); ++d) {
     uint32_t q = racy[d];
-    if (t_join[q] <= wstart(q)) continue;     // a carried-out instance with an empty window here
+    if (!has_window(q)) continue;             // a carried-out instance with no window here
     evs.push_back({wstart(q), (int64_t)d + 1});
     evs.push_back({t_join[q], -((int64_t)d + 1)});
   }

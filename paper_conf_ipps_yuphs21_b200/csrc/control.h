@@ -35,7 +35,8 @@ struct MirPlanH {
 // A nowait task instance that ended in an earlier flush and is not joined yet
 // (SURVEY §8(f) N2): its own range ops (relative words; pos unused) travel on the
 // host, its (word, write-class) access summary on the device (ctx->carry_ent).
-struct CarriedInst { uint32_t task_id; std::vector<RangeRef> own; };
+// open: its TASK_BEGIN..TASK_END block is still open (its next records belong to it).
+struct CarriedInst { uint32_t task_id; std::vector<RangeRef> own; bool open; };
 
 struct FlushPlan {
   std::vector<RangeOpH> range_ops;       // in trace order
