@@ -9,6 +9,20 @@ build A
 patch -p1 < $PATCH > $OUT/patch.log || { echo "patch failed"; cat $OUT/patch.log; exit 1; }
 build B
 if [ -n "$PYTEST_B" ]; then timeout 900 python -m pytest tests -m gpu -x -q > $OUT/pytest_B.log 2>&1; echo "pytest B rc=$?"; tail -2 $OUT/pytest_B.log; fi
+if [ -n "$NCU_KERNEL" ]; then   # per-launch kernel durations under ncu (serialised, cold): less noisy than the bench
+  for v in A B; do
+    cp /tmp/lib_$v.so paper_conf_ipps_yuphs21_b200/libarbalest.so
+    timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"$NCU_KERNEL" --csv \
+      python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu "$@" > $OUT/ncu_$v.csv 2> $OUT/ncu_$v.err
+    python - $OUT/ncu_$v.csv $v <<'PY'
+import csv, io, sys
+t = open(sys.argv[1]).read(); t = t[t.find('"ID"'):]
+ms = [float(r["Metric Value"].replace(",", "")) / (1e6 if r["Metric Unit"] == "ns" else 1e3 if r["Metric Unit"] == "us" else 1)
+      for r in csv.DictReader(io.StringIO(t)) if r.get("Metric Name") == "gpu__time_duration.sum"]
+print(sys.argv[2], "ncu ms per launch:", [round(x, 4) for x in ms], "sum", round(sum(ms), 4))
+PY
+  done
+fi
 for v in A B A B; do
   cp /tmp/lib_$v.so paper_conf_ipps_yuphs21_b200/libarbalest.so
   timeout 300 python bench.py --no-e2e --no-cpu "$@" > $OUT/bench_$v.json 2> $OUT/bench_$v.err
