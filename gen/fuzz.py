@@ -14,7 +14,9 @@ from .trace import MAP, OP, UPD, SYNC_ALL, TraceBuilder, encode_np
 
 
 def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: int = 60,
-                   base: int = 0x10000, loop_max: int = 48, p_task: float = 0.15):
+                   base: int = 0x10000, loop_max: int = 48, p_task: float = 0.15, p_always: float = 0.0):
+    """p_always > 0: map clauses carry the `always` modifier with that probability
+    (the RNG stream of p_always = 0 programs is unchanged)."""
     rs = np.random.default_rng(seed)
     tb = TraceBuilder()
     arrays = [base + i * array_words * 8 * 2 for i in range(n_arrays)]   # gap between arrays
@@ -57,7 +59,10 @@ def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: i
             hi = lo + n
             ok = all(hi <= a or lo >= b or (a <= lo and hi <= b) for a, b in present[i])
             if ok:
-                tb.enter(int(rs.choice([MAP.TO, MAP.FROM, MAP.TOFROM, MAP.ALLOC])), lo, n)
+                mt = int(rs.choice([MAP.TO, MAP.FROM, MAP.TOFROM, MAP.ALLOC]))
+                if p_always and rs.random() < p_always:
+                    mt |= MAP.ALWAYS
+                tb.enter(mt, lo, n)
                 present[i].append((lo, hi))
         elif r < 0.65:
             i = int(rs.integers(n_arrays))
@@ -66,8 +71,10 @@ def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: i
                 lo, hi = present[i][k]
                 # exit only sections that contain no other present section
                 if all(not (lo <= a and b <= hi and (a, b) != (lo, hi)) for a, b in present[i]):
-                    tb.exit(int(rs.choice([MAP.TO, MAP.FROM, MAP.TOFROM, MAP.ALLOC,
-                                           MAP.RELEASE, MAP.DELETE])), lo, hi - lo)
+                    mt = int(rs.choice([MAP.TO, MAP.FROM, MAP.TOFROM, MAP.ALLOC, MAP.RELEASE, MAP.DELETE]))
+                    if p_always and rs.random() < p_always:
+                        mt |= MAP.ALWAYS
+                    tb.exit(mt, lo, hi - lo)
                     present[i].pop(k)
         elif r < 0.72:
             i = int(rs.integers(n_arrays))

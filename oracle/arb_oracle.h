@@ -51,6 +51,11 @@ enum { ORC_RH = 0, ORC_WH = 1, ORC_RT = 2, ORC_WT = 3,
 /* map-types (Table I) */
 enum { ORC_TO = 0, ORC_FROM = 1, ORC_TOFROM = 2, ORC_ALLOC = 3,
        ORC_RELEASE = 4, ORC_DELETE = 5 };
+/* map-type modifier bit in arg (OpenMP 5.1 `always`, reading Z21):
+ * on entry with to/tofrom the OV->CV copy happens even if the entry is present;
+ * on exit with from/tofrom the CV->OV copy happens even if the reference count
+ * stays above 0 */
+#define ORC_ALWAYS 0x10u
 /* update direction */
 enum { ORC_UPD_TO = 0, ORC_UPD_FROM = 1 };
 #define ORC_SYNC_ALL 0xFFFFu

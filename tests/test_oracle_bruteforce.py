@@ -155,3 +155,32 @@ def test_bo_random_long(orc):
     rs = np.random.default_rng(13)
     seqs = [tuple(sym[i] for i in rs.integers(0, len(sym), rs.integers(4, 9))) for _ in range(40000)]
     check_batch(orc, seqs, 2, bo=True)
+
+
+def alphabet_always(nwords):
+    """alphabet() plus the `always` map-type modifier on to/tofrom entries and
+    from/tofrom exits (OpenMP 5.1, reading Z21)."""
+    sym = alphabet(nwords)
+    sections = [(0, 1)] if nwords == 1 else [(0, 1), (1, 2), (0, 2)]
+    for lo, hi in sections:
+        for t in (MAP.TO, MAP.TOFROM):
+            sym.append(("ctl", OP.MAP_ENTER, lo * 8, (hi - lo) * 8, t | MAP.ALWAYS))
+        for t in (MAP.FROM, MAP.TOFROM):
+            sym.append(("ctl", OP.MAP_EXIT, lo * 8, (hi - lo) * 8, t | MAP.ALWAYS))
+    return sym
+
+
+@pytest.mark.parametrize("nwords,length", [(1, 4), (2, 3)])
+def test_always_exhaustive(orc, nwords, length):
+    """The `always` modifier: the oracle's reports and final states equal the value
+    simulator's (its own Table I + `always` reference-count model) on every sequence."""
+    sym = alphabet_always(nwords)
+    seqs = [s for L in range(1, length + 1) for s in itertools.product(sym, repeat=L)]
+    assert check_batch(orc, seqs, nwords) > 50000
+
+
+def test_always_random_long(orc):
+    sym = alphabet_always(2)
+    rs = np.random.default_rng(14)
+    seqs = [tuple(sym[i] for i in rs.integers(0, len(sym), rs.integers(4, 9))) for _ in range(40000)]
+    check_batch(orc, seqs, 2)

@@ -331,3 +331,28 @@ def test_bo_after_release_and_host_unaffected(orc):
     res = run(orc, tb.array(), A, 8, detect_bo=True)
     assert res.triples() == [(A // 8, i_bo, BO)]
     assert i_ok < i_bo < i_h
+
+
+def test_always_modifier_nested_region(orc):
+    """OpenMP 5.1 `always` (N4, Z21): inside an outer `target data map(tofrom)`, an
+    inner `map(always, tofrom)` refreshes the CV on entry and the OV on exit, so the
+    host read after the inner region is clean; without `always` it is stale (the
+    nested-refcount case of Table I)."""
+    A = 0x4000
+    for always, expect_usd in ((False, True), (True, False)):
+        tb = TraceBuilder()
+        tb.wh(A)
+        tb.enter(MAP.TOFROM, A, 8)                          # outer region: rc = 1
+        tb.wh(A)                                            # host update inside the outer region
+        mt = MAP.TOFROM | (MAP.ALWAYS if always else 0)
+        tb.enter(mt, A, 8)                                  # inner: rc = 2 (+ copy with always)
+        i_rt = tb.rt(A)
+        tb.wt(A)
+        tb.exit(mt, A, 8)                                   # rc = 1 (+ copy back with always)
+        i_rh = tb.rh(A)
+        tb.exit(MAP.TOFROM, A, 8)
+        res = run(orc, tb.array(), A, 8)
+        kinds = {(r, k) for _, r, k in res.triples()}
+        assert ((i_rt, USD) in kinds) == expect_usd          # the kernel read sees the old CV
+        assert ((i_rh, USD) in kinds) == expect_usd          # the host read misses the kernel write
+        assert sorted(ValueSim().run(tb.array())) == res.triples()

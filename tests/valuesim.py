@@ -24,6 +24,7 @@ BOT = 0  # undefined content
 RH, WH, RT, WT, MAP_ENTER, MAP_EXIT, UPDATE = 0, 1, 2, 3, 8, 9, 10
 TASK_BEGIN, TASK_END, SYNC = 12, 13, 14
 TO, FROM, TOFROM, ALLOC, RELEASE, DELETE = 0, 1, 2, 3, 4, 5
+ALWAYS = 0x10                       # map-type modifier bit (N4, reading Z21)
 UUM, USD, BO = 1, 2, 4
 
 
@@ -100,6 +101,8 @@ class ValueSim:
         return hit
 
     def record(self, op, addr, length, arg, idx):
+        always = bool(arg & ALWAYS)           # OpenMP 5.1 `always` map-type modifier (reading Z21)
+        arg &= ~ALWAYS
         if op in (RH, WH, RT, WT):
             name = {RH: "RH", WH: "WH", RT: "RT", WT: "WT"}[op]
             for w in self.words(addr, length):
@@ -108,6 +111,9 @@ class ValueSim:
             ent = self._lookup(addr, addr + length)
             if ent is not None:
                 ent[2] += 1
+                if always and arg in (TO, TOFROM):
+                    for w in self.words(addr, length):
+                        self.word_op("UPT", w, idx)
                 return
             self.present.append([addr, addr + length, 1])
             for w in self.words(addr, length):
@@ -120,6 +126,9 @@ class ValueSim:
             if ent is None:
                 return
             ent[2] = 0 if arg == DELETE else ent[2] - 1
+            if ent[2] != 0 and always and arg in (FROM, TOFROM):
+                for w in self.words(addr, length):
+                    self.word_op("UPH", w, idx)
             if ent[2] == 0:
                 if arg in (FROM, TOFROM):
                     for w in self.words(addr, length):
