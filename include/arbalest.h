@@ -47,6 +47,10 @@ enum arb_op {
 /* map-types (Table I) */
 enum arb_map { ARB_TO = 0, ARB_FROM = 1, ARB_TOFROM = 2, ARB_ALLOC = 3,
                ARB_RELEASE = 4, ARB_DELETE = 5 };
+/* map-type modifier, or-ed into the map-type (OpenMP 5.1 `always`; Z21):
+ * MAP_ENTER to/tofrom copies OV->CV even when the entry is present, MAP_EXIT
+ * from/tofrom copies CV->OV even when the reference count stays above 0 */
+#define ARB_MAP_ALWAYS 0x10u
 /* target update direction */
 enum arb_upd { ARB_UPD_TO = 0, ARB_UPD_FROM = 1 };
 #define ARB_SYNC_ALL 0xFFFFu

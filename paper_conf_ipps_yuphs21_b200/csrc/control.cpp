@@ -92,18 +92,26 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
         break;
       }
       case OP_MAP_ENTER: {                          // Table I, entry
+        const bool always = arg & kMapAlways;       // Z21
+        arg &= ~kMapAlways;
         if (arg > MT_ALLOC || len == 0 || addr + len > (1ull << 48))
           return fail(ARB_ETRACE, c.pos, "bad MAP_ENTER record");
         MapTable::iterator it;
         int f = map_find(map, addr, addr + len, it);
         if (f < 0) return fail(ARB_EMAP, c.pos, "map clause partially overlaps a present entry");
-        if (f == 1) { it->second.rc += 1; break; }  // exist(CV): ref_count += 1
+        if (f == 1) {                               // exist(CV): ref_count += 1, no transfer ...
+          it->second.rc += 1;
+          if (always && (arg == MT_TO || arg == MT_TOFROM)) em.emit(pos, kSelUPT, addr, addr + len, open);
+          break;                                    // ... unless `always`
+        }
         map.emplace(addr, MapEntry{addr + len, 1});  // new CV, ref_count = 1
         em.emit(pos, kSelALLOC | (bo ? kPopSet : 0u), addr, addr + len, open);
         if (arg == MT_TO || arg == MT_TOFROM) em.emit(pos, kSelUPT, addr, addr + len, open);
         break;
       }
       case OP_MAP_EXIT: {                           // Table I, exit (reading Z5)
+        const bool always = arg & kMapAlways;       // Z21
+        arg &= ~kMapAlways;
         if (arg > MT_DELETE || len == 0 || addr + len > (1ull << 48))
           return fail(ARB_ETRACE, c.pos, "bad MAP_EXIT record");
         MapTable::iterator it;
@@ -111,6 +119,8 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
         if (f < 0) return fail(ARB_EMAP, c.pos, "map clause partially overlaps a present entry");
         if (f == 0) break;                          // not present: no-op (Z7)
         if (arg == MT_DELETE) it->second.rc = 0; else it->second.rc -= 1;
+        if (it->second.rc != 0 && always && (arg == MT_FROM || arg == MT_TOFROM))
+          em.emit(pos, kSelUPH, addr, addr + len, open);   // `always`: copy back at rc > 0
         if (it->second.rc == 0) {
           if (arg == MT_FROM || arg == MT_TOFROM) em.emit(pos, kSelUPH, addr, addr + len, open);
           em.emit(pos, kSelREL | (bo ? kPopClr : 0u), it->first, it->second.hi, open);

@@ -370,3 +370,16 @@ def test_flush_between_end_and_join(orc):
     assert (A // 8, i_race, 3) in exp.triples()
     rc, got, shadow, st = run_gpu(rec, A, 64, flush_points=[c1, c2])
     assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+@pytest.mark.parametrize("seed", range(16))
+def test_always_modifier_fuzz(orc, seed):
+    """The `always` map-type modifier (N4, Z21) on random programs, with and
+    without flush cuts."""
+    from gen.fuzz import random_program
+    rec, base, span = random_program(5000 + seed, p_always=0.5, p_task=0.3)
+    check(orc, rec, base, span)
+    exp = orc.replay(rec, base, span)
+    if exp.rc == 0:
+        rc, got, shadow, _ = run_gpu(rec, base, span, flush_points=_cuts(rec, 4, seed))
+        assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
