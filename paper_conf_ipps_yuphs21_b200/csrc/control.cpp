@@ -181,6 +181,8 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   for (uint32_t q = 1; q <= ninst; ++q)
     if (has_window(q) || carry[q]) { dense[q] = (uint32_t)racy.size(); racy.push_back(q); }
   M.n_racy = (uint32_t)racy.size();
+  if (racy.size() >= (1u << 20) - 1)          // the MIR join keys hold the dense index in 20 bits
+    return fail(ARB_ENOMEM, n_records, "more than 2^20 - 2 racy or unjoined task instances in one flush");
   out.carry_in_dense.resize(nc);
   for (uint32_t c = 0; c < nc; ++c) out.carry_in_dense[c] = dense[c + 1];
   out.dense_carry_out.assign(racy.size(), 0xFFFFFFFFu);
