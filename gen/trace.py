@@ -13,6 +13,7 @@ class OP:
     RH, WH, RT, WT = 0, 1, 2, 3
     MAP_ENTER, MAP_EXIT, UPDATE = 8, 9, 10
     TASK_BEGIN, TASK_END, SYNC = 12, 13, 14
+    TASK_DEPEND = 15       # inside a block: depends on the last ended instance of task id k (Z22)
 
 
 class MAP:
@@ -127,6 +128,9 @@ class TraceBuilder:
 
     def sync(self, k=SYNC_ALL):
         return self._add(OP.SYNC, task=k)
+
+    def depend(self, k):
+        return self._add(OP.TASK_DEPEND, task=k)
 
     def extend(self, other: "TraceBuilder"):
         base = self._n

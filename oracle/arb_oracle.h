@@ -27,6 +27,7 @@
  *   MIR attribution to later event (Z11)  parity unpinned (definition only)
  *   dedup-first mode (Z3)                 parity unpinned (definition only)
  *   sub-word semantics (Z4)               parity unpinned (definition only)
+ *   depend (Z22)                          pinned (schedule enumeration with dependencies + witness search)
  *   buffer overflow, present-bit form (Z20) pinned (P:279 worked example + brute force vs the
  *                                         value simulator's CV existence); the paper's base-interval
  *                                         comparison (overflow into ANOTHER mapped CV) is not modelled
@@ -47,7 +48,9 @@ typedef struct { uint64_t w0, w1; } orc_record;
 /* ops (P:242-245 read/write host/target; P:106-123 device directives) */
 enum { ORC_RH = 0, ORC_WH = 1, ORC_RT = 2, ORC_WT = 3,
        ORC_MAP_ENTER = 8, ORC_MAP_EXIT = 9, ORC_UPDATE = 10,
-       ORC_TASK_BEGIN = 12, ORC_TASK_END = 13, ORC_SYNC = 14 };
+       ORC_TASK_BEGIN = 12, ORC_TASK_END = 13, ORC_SYNC = 14,
+       ORC_TASK_DEPEND = 15 /* inside a block: the task depends on the last ended
+                               instance of task id k (N4, reading Z22) */ };
 /* map-types (Table I) */
 enum { ORC_TO = 0, ORC_FROM = 1, ORC_TOFROM = 2, ORC_ALLOC = 3,
        ORC_RELEASE = 4, ORC_DELETE = 5 };

@@ -203,3 +203,161 @@ def test_mir_is_necessary_for_soundness(orc):
         if t and all(k == 3 for _, _, k in t):
             found += any(schedule_issues(to_word_ops(s)) for s in schedules(items))
     assert found > 50
+
+
+# ---- depend (reading Z22) --------------------------------------------
+def random_program_dep(rs, ntasks, read_bias=0.0):
+    """As random_program, but a launched task may depend on an earlier one:
+    ('t', k, ops, dep) with dep = an earlier task id or 0."""
+    items = []
+    launched = []
+    for it in random_program(rs, ntasks, read_bias):
+        if it[0] == "t":
+            dep = int(launched[rs.integers(len(launched))]) if launched and rs.random() < 0.7 else 0
+            items.append(("t", it[1], it[2], dep))
+            launched.append(it[1])
+        else:
+            items.append(it)
+    return items
+
+
+def serialize_dep(items):
+    recs = [encode(OP.WH, A, 8), encode(OP.MAP_ENTER, A, 8, arg=MAP.TOFROM)]
+    for it in items:
+        if it[0] == "h":
+            recs.append(rec_of(it[1]))
+        elif it[0] == "t":
+            recs.append(encode(OP.TASK_BEGIN, task=it[1]))
+            if it[3]:
+                recs.append(encode(OP.TASK_DEPEND, task=it[3]))
+            recs.extend(rec_of(o) for o in it[2])
+            recs.append(encode(OP.TASK_END, task=it[1]))
+        else:
+            recs.append(encode(OP.SYNC, task=it[1]))
+    recs.append(encode(OP.SYNC, task=0xFFFF))
+    recs.append(encode(OP.MAP_EXIT, A, 8, arg=MAP.TOFROM))
+    recs.append(encode(OP.RH, A, 8))
+    return recs
+
+
+def schedules_dep(items):
+    """Legal interleavings: a task runs its ops after launch and after its
+    dependency's ops have all run; a taskwait waits for the tasks it names."""
+    host, tasks, dep = [], {}, {}
+    for it in items:
+        if it[0] == "h":
+            host.append(("op", it[1]))
+        elif it[0] == "t":
+            host.append(("launch", it[1]))
+            tasks[it[1]] = it[2]
+            dep[it[1]] = it[3]
+        else:
+            host.append(("sync", it[1]))
+    host.append(("sync", 0xFFFF))
+    out = []
+
+    def done(state, k):
+        return state[k][0] and state[k][1] == len(tasks[k])
+
+    def rec(hi, state, acc):
+        for k, (launched, nxt) in state.items():
+            if launched and nxt < len(tasks[k]) and (not dep[k] or done(state, dep[k])):
+                st = dict(state); st[k] = (True, nxt + 1)
+                rec(hi, st, acc + [tasks[k][nxt]])
+        if hi == len(host):
+            if all(nxt == len(tasks[k]) for k, (_, nxt) in state.items()):
+                out.append(acc)
+            return
+        kind, v = host[hi]
+        if kind == "op":
+            rec(hi + 1, state, acc + [v])
+        elif kind == "launch":
+            st = dict(state); st[v] = (True, 0)
+            rec(hi + 1, st, acc)
+        else:
+            for k, (launched, nxt) in state.items():
+                if launched and (v == 0xFFFF or v == k) and nxt < len(tasks[k]):
+                    return
+            rec(hi + 1, state, acc)
+
+    rec(0, {k: (False, 0) for k in tasks}, [])
+    return out
+
+
+def witness_dep(recs, idx):
+    """Brute force with dependencies: an earlier conflicting op of another task that
+    is not an ancestor of the current one and not yet complete at idx (complete =
+    a SYNC naming it or one of its dependants after that dependant's end)."""
+    ops, dep, ends, cur = [], {}, {}, 0
+    for i, (w0, w1) in enumerate(recs):
+        op = (w0 >> 48) & 0xFF
+        if op == OP.TASK_BEGIN:
+            cur = int(w1 >> 48); dep[cur] = 0
+        elif op == OP.TASK_DEPEND:
+            dep[cur] = int(w1 >> 48)
+        elif op == OP.TASK_END:
+            ends[cur] = i; cur = 0
+        elif op in (OP.RH, OP.WH, OP.RT, OP.WT, OP.UPDATE, OP.MAP_ENTER, OP.MAP_EXIT):
+            ops.append((i, cur, op not in (OP.RH, OP.RT)))
+
+    def ancestors(t):
+        a = set()
+        while dep.get(t):
+            t = dep[t]; a.add(t)
+        return a
+
+    def complete_at(t):
+        js = [len(recs)]
+        for u in [t] + [u for u in dep if t in ancestors(u)]:
+            for j in range(ends[u], len(recs)):
+                if (recs[j][0] >> 48) & 0xFF == OP.SYNC and (recs[j][1] >> 48) in (u, 0xFFFF):
+                    js.append(j)
+                    break
+        return min(js)
+
+    me = [o for o in ops if o[0] == idx]
+    if not me:
+        return False
+    _, my_task, my_w = me[0]
+    anc = ancestors(my_task) if my_task else set()
+    for i, task, w in ops:
+        if i >= idx or task == 0 or task == my_task or task in anc or not (w or my_w):
+            continue
+        if complete_at(task) > idx:
+            return True
+    return False
+
+
+def _run_dep(orc, ntasks, nprog, seed, read_bias=0.0):
+    rs = np.random.default_rng(seed)
+    clean = racy = removed = 0
+    for _ in range(nprog):
+        items = random_program_dep(rs, ntasks, read_bias)
+        recs = serialize_dep(items)
+        res = orc.replay(np.array(recs, dtype=np.uint64).reshape(-1, 2), A, 8)
+        assert res.rc == 0
+        t = res.triples()
+        if not t:
+            clean += 1
+            for sched in schedules_dep(items):
+                assert not schedule_issues(to_word_ops(sched)), (items, sched)
+        for w, i, k in t:
+            if k == 3:
+                racy += 1
+                assert witness_dep(recs, i), (items, i)
+        # the same program without its depend records reports at least as many races
+        plain = [r for r in recs if (r[0] >> 48) & 0xFF != OP.TASK_DEPEND]
+        n_plain = sum(k == 3 for _, _, k in
+                      orc.replay(np.array(plain, dtype=np.uint64).reshape(-1, 2), A, 8).triples())
+        n_dep = sum(k == 3 for _, _, k in t)
+        assert n_plain >= n_dep
+        removed += n_plain > n_dep
+    return clean, racy, removed
+
+
+def test_theorem1_depend(orc):
+    """Z22 pinned by schedule enumeration: oracle-clean => every schedule that
+    respects the dependencies is clean; every MIR has a witness outside the
+    current task's ancestors; depend only ever removes races, and does."""
+    clean, racy, removed = _run_dep(orc, 3, 4000, 5)
+    assert clean > 50 and racy > 100 and removed > 100
