@@ -14,9 +14,11 @@ from .trace import MAP, OP, UPD, SYNC_ALL, TraceBuilder, encode_np
 
 
 def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: int = 60,
-                   base: int = 0x10000, loop_max: int = 48, p_task: float = 0.15, p_always: float = 0.0):
-    """p_always > 0: map clauses carry the `always` modifier with that probability
-    (the RNG stream of p_always = 0 programs is unchanged)."""
+                   base: int = 0x10000, loop_max: int = 48, p_task: float = 0.15, p_always: float = 0.0,
+                   p_depend: float = 0.0):
+    """p_always > 0: map clauses carry the `always` modifier with that probability;
+    p_depend > 0: a new nowait block depends on an earlier task with that
+    probability (the RNG streams of p_always = p_depend = 0 programs are unchanged)."""
     rs = np.random.default_rng(seed)
     tb = TraceBuilder()
     arrays = [base + i * array_words * 8 * 2 for i in range(n_arrays)]   # gap between arrays
@@ -24,6 +26,7 @@ def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: i
     in_task = 0
     next_task = 1
     unjoined = []
+    ended_ids = []
 
     def section(i):
         a = arrays[i]
@@ -88,9 +91,12 @@ def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: i
             next_task = next_task + 1 if next_task < 60000 else 1
             tb.task_begin(k)
             in_task = k
+            if p_depend and ended_ids and rs.random() < p_depend:
+                tb.depend(int(ended_ids[int(rs.integers(len(ended_ids)))]))
         elif in_task and r < 0.95:
             tb.task_end(in_task)
             unjoined.append(in_task)
+            ended_ids.append(in_task)
             in_task = 0
         elif not in_task and unjoined and r >= 0.95:
             if rs.random() < 0.5:

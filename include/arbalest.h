@@ -42,7 +42,10 @@ enum arb_op {
   ARB_MAP_ENTER = 8, ARB_MAP_EXIT = 9,                  /* map clause on region entry / exit   */
   ARB_UPDATE = 10,                                      /* target update to/from       */
   ARB_TASK_BEGIN = 12, ARB_TASK_END = 13,               /* nowait region block (Z8)     */
-  ARB_SYNC = 14                                         /* taskwait: joins task k, 0xFFFF = all */
+  ARB_SYNC = 14,                                        /* taskwait: joins task k, 0xFFFF = all */
+  ARB_TASK_DEPEND = 15  /* inside a block: the task depends on the last ended instance of task k
+                           (a `depend` clause; Z22): their ops are ordered, and
+                           joining the dependant joins the instance it depends on            */
 };
 /* map-types (Table I) */
 enum arb_map { ARB_TO = 0, ARB_FROM = 1, ARB_TOFROM = 2, ARB_ALLOC = 3,

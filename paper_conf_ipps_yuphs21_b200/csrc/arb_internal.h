@@ -11,7 +11,8 @@ namespace arb {
 constexpr uint64_t kMask48 = (1ull << 48) - 1;
 enum Op : uint32_t { OP_RH = 0, OP_WH = 1, OP_RT = 2, OP_WT = 3,
                      OP_MAP_ENTER = 8, OP_MAP_EXIT = 9, OP_UPDATE = 10,
-                     OP_TASK_BEGIN = 12, OP_TASK_END = 13, OP_SYNC = 14 };
+                     OP_TASK_BEGIN = 12, OP_TASK_END = 13, OP_SYNC = 14,
+                     OP_TASK_DEPEND = 15 };   // N4, Z22
 enum MapType : uint32_t { MT_TO = 0, MT_FROM = 1, MT_TOFROM = 2, MT_ALLOC = 3,
                           MT_RELEASE = 4, MT_DELETE = 5 };
 constexpr uint32_t kMapAlways = 0x10;   // `always` map-type modifier bit (N4, Z21)

@@ -53,11 +53,14 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   std::vector<uint32_t> t_id{0};
   std::vector<uint32_t> unjoined;
   uint32_t open = 0;
+  // depend edges {child, parent} in order of the child's creation (Z22)
+  std::vector<std::pair<uint32_t, uint32_t>> edges;
   for (uint32_t c = 0; c < nc; ++c) {
     const bool op_ = (*carried_in)[c].open;
     t_begin.push_back(kBefore); t_end.push_back(op_ ? kOpen : kBefore); t_join.push_back(UINT64_MAX);
     t_id.push_back((*carried_in)[c].task_id);
     if (op_) open = c + 1; else unjoined.push_back(c + 1);
+    for (uint32_t pc : (*carried_in)[c].deps) edges.push_back({c + 1, pc + 1});
   }
   auto fail = [&](int rc, uint64_t pos, const char* why) {
     out.rc = rc; out.err_pos = pos; out.err = why;
@@ -138,10 +141,29 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
         em.emit(pos, arg == 0 ? kSelUPT : kSelUPH, addr, addr + len, open);
         break;
       }
+      case OP_TASK_DEPEND: {                        // Z22: the open task runs after the last
+        if (!open || tid == 0 || tid == kSyncAll)   // ended instance of task `tid`
+          return fail(ARB_ETRACE, c.pos, "TASK_DEPEND outside a task block or with task id 0 / 0xFFFF");
+        for (uint32_t q = open - 1; q >= 1; --q)
+          if (t_id[q] == tid && t_end[q] != kOpen) { edges.push_back({open, q}); break; }
+        break;
+      }
       default:
         return fail(ARB_ETRACE, c.pos, "unknown control op");
     }
   }
+  // Z22: joining a dependant joins its ancestors (children come after parents)
+  for (size_t k = edges.size(); k-- > 0;)
+    t_join[edges[k].second] = std::min(t_join[edges[k].second], t_join[edges[k].first]);
+  auto is_anc = [&](uint32_t a, uint32_t c) {   // a is an ancestor of c through depend edges
+    std::vector<uint32_t> st{c};
+    while (!st.empty()) {
+      const uint32_t x = st.back(); st.pop_back();
+      for (const auto& e : edges)
+        if (e.first == x) { if (e.second == a) return true; st.push_back(e.second); }
+    }
+    return false;
+  };
   // a block still open at the end of the flush is carried (N2): its records so
   // far are its own ops, its window starts after its TASK_END in a later flush
   const uint32_t ninst = (uint32_t)t_begin.size() - 1;
@@ -216,7 +238,13 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
     uint32_t q = racy[d];
     if (!carry[q]) continue;
     out.dense_carry_out[d] = (uint32_t)out.carry_out.size();
-    out.carry_out.push_back(CarriedInst{t_id[q], own[d], t_end[q] == kOpen});
+    out.carry_out.push_back(CarriedInst{t_id[q], own[d], t_end[q] == kOpen, {}});
+  }
+  for (const auto& e : edges) {              // depend edges between carried-out instances (Z22)
+    const uint32_t dc = dense[e.first], dp = dense[e.second];
+    if (dc == 0xFFFFFFFFu || dp == 0xFFFFFFFFu) continue;
+    const uint32_t cc = out.dense_carry_out[dc], cp = out.dense_carry_out[dp];
+    if (cc != 0xFFFFFFFFu && cp != 0xFFFFFFFFu) out.carry_out[cc].deps.push_back(cp);
   }
   for (size_t d = 0; d < racy.size(); ++d) {
     uint32_t q = racy[d];
@@ -226,7 +254,8 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
                  : std::upper_bound(out.range_ops.begin(), out.range_ops.end(), (uint32_t)t_end[q],
                                     [](uint32_t p, const RangeOpH& r) { return p < r.pos; });
     for (auto it = first; it != out.range_ops.end() && it->pos < t_join[q]; ++it)
-      win[d].push_back(RangeRef{it->lo, it->hi, it->pos, it->inst});
+      if (edges.empty() || !it->inst || !is_anc(q, it->inst))   // a dependant's ops come after q's (Z22)
+        win[d].push_back(RangeRef{it->lo, it->hi, it->pos, it->inst});
   }
   for (size_t d = 0; d < racy.size(); ++d) {
     M.own_start[d + 1] = M.own_start[d] + (uint32_t)own[d].size();
@@ -252,22 +281,46 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
     evs.push_back({wstart(q), (int64_t)d + 1});
     evs.push_back({t_join[q], -((int64_t)d + 1)});
   }
+  // Z22: inside the block of an instance c, the windows of c's ancestors are not
+  // open (their ops precede c's): with depend edges, block boundaries split the
+  // query segments too (code 0; `blk` maps the position to the block's owner)
+  std::map<uint64_t, uint32_t> blk;          // position -> instance whose block starts (0: block ends)
+  if (!edges.empty()) {
+    for (uint32_t q = 1; q <= ninst; ++q) {
+      if (t_end[q] == kBefore) continue;
+      const uint64_t lo = t_begin[q] == kBefore ? 0 : t_begin[q] + 1;
+      const uint64_t hi = t_end[q] == kOpen ? n_records : t_end[q];
+      if (hi <= lo) continue;
+      blk[lo] = q;
+      if (!blk.count(hi)) blk[hi] = 0;
+      evs.push_back({lo, 0});
+      evs.push_back({hi, 0});
+    }
+  }
   std::sort(evs.begin(), evs.end());
   std::set<uint32_t> active;
+  uint32_t cur_blk = 0;
   M.qry_cum.push_back(0);
   M.qry_open_start.push_back(0);
   for (size_t k = 0; k < evs.size();) {
     uint64_t p = evs[k].first;
     while (k < evs.size() && evs[k].first == p) {
       if (evs[k].second > 0) active.insert((uint32_t)(evs[k].second - 1));
-      else active.erase((uint32_t)(-evs[k].second - 1));
+      else if (evs[k].second < 0) active.erase((uint32_t)(-evs[k].second - 1));
       ++k;
     }
+    if (!edges.empty()) {
+      auto b = blk.find(p);
+      if (b != blk.end()) cur_blk = b->second;
+    }
     if (k < evs.size() && !active.empty() && evs[k].first > p) {
+      const size_t before = M.open_list.size();
+      for (uint32_t d : active)
+        if (!cur_blk || !is_anc(racy[d], cur_blk)) M.open_list.push_back(d);
+      if (M.open_list.size() == before) continue;
       uint64_t len = evs[k].first - p;
       M.qry_lo.push_back(p);
       M.qry_cum.push_back(M.qry_cum.back() + len);
-      for (uint32_t d : active) M.open_list.push_back(d);
       M.qry_open_start.push_back((uint32_t)M.open_list.size());
     }
   }

@@ -36,7 +36,8 @@ struct MirPlanH {
 // (SURVEY §8(f) N2): its own range ops (relative words; pos unused) travel on the
 // host, its (word, write-class) access summary on the device (ctx->carry_ent).
 // open: its TASK_BEGIN..TASK_END block is still open (its next records belong to it).
-struct CarriedInst { uint32_t task_id; std::vector<RangeRef> own; bool open; };
+// deps: carried indices of the (unjoined) instances it depends on (Z22).
+struct CarriedInst { uint32_t task_id; std::vector<RangeRef> own; bool open; std::vector<uint32_t> deps; };
 
 struct FlushPlan {
   std::vector<RangeOpH> range_ops;       // in trace order

@@ -49,7 +49,7 @@ __device__ __forceinline__ Dec decode0(uint4 q, bool valid, const PartParams& p,
   const uint32_t len = q.z, hi = q.y & 0xFFFFu;
   // malformed access: len outside 1..8 or the byte range leaving the 48-bit space
   const bool bad_acc = (q.w & 0xFFFFu) != 0 || len - 1u > 7u || (hi == 0xFFFFu && q.x > 0u - len);
-  const bool ctl = op < 16 && ((0x7700u >> op) & 1u);            // ops 8, 9, 10, 12, 13, 14
+  const bool ctl = op < 16 && ((0xF700u >> op) & 1u);            // ops 8, 9, 10, 12, 13, 14, 15
   const bool acc = op < 4;
   flags = valid ? (acc ? (bad_acc ? 2u : 0u) : (ctl ? 1u : 2u)) : 0u;
   const bool ok = valid && acc && !bad_acc;

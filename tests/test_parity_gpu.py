@@ -383,3 +383,15 @@ def test_always_modifier_fuzz(orc, seed):
     if exp.rc == 0:
         rc, got, shadow, _ = run_gpu(rec, base, span, flush_points=_cuts(rec, 4, seed))
         assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+@pytest.mark.parametrize("seed", range(16))
+def test_depend_fuzz(orc, seed):
+    """Task dependencies (N4, Z22) on random programs, with and without flush cuts
+    (dependencies between instances carried across flushes)."""
+    from gen.fuzz import random_program
+    rec, base, span = random_program(6000 + seed, p_task=0.45, p_depend=0.6)
+    exp, _ = check(orc, rec, base, span)
+    if exp.rc == 0:
+        rc, got, shadow, _ = run_gpu(rec, base, span, flush_points=_cuts(rec, 5, seed))
+        assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
