@@ -19,6 +19,7 @@ class OP:
 class MAP:
     TO, FROM, TOFROM, ALLOC, RELEASE, DELETE = 0, 1, 2, 3, 4, 5
     ALWAYS = 0x10          # map-type modifier bit, or-ed into the map-type (N4, Z21)
+    PRESENT = 0x20         # map-type modifier bit: the section must already be mapped (Z21)
 
 
 class UPD:

@@ -59,6 +59,9 @@ enum { ORC_TO = 0, ORC_FROM = 1, ORC_TOFROM = 2, ORC_ALLOC = 3,
  * on exit with from/tofrom the CV->OV copy happens even if the reference count
  * stays above 0 */
 #define ORC_ALWAYS 0x10u
+/* `present` modifier (OpenMP 5.1; N4, reading Z21): a MAP_ENTER whose section is
+ * not present is a mapping error (ORC_EMAP) */
+#define ORC_PRESENT 0x20u
 /* update direction */
 enum { ORC_UPD_TO = 0, ORC_UPD_FROM = 1 };
 #define ORC_SYNC_ALL 0xFFFFu

@@ -109,9 +109,11 @@ def test_two_words_random_long(orc):
     check_batch(orc, seqs, 2)
 
 
-def test_emap_agrees(orc):
-    """Sequences the independent refcount model rejects are rejected by the oracle (ARB_EMAP)."""
-    sym = alphabet(2)
+@pytest.mark.parametrize("alpha", ["plain", "modifiers"])
+def test_emap_agrees(orc, alpha):
+    """Sequences the independent refcount model rejects (partial overlaps; with the
+    modifiers also `present` on an unmapped section) are rejected by the oracle (ARB_EMAP)."""
+    sym = alphabet(2) if alpha == "plain" else alphabet_always(2)
     n_bad = 0
     for seq in itertools.product(sym, repeat=2):
         enc = encode_seq(seq, 0)
@@ -167,6 +169,7 @@ def alphabet_always(nwords):
             sym.append(("ctl", OP.MAP_ENTER, lo * 8, (hi - lo) * 8, t | MAP.ALWAYS))
         for t in (MAP.FROM, MAP.TOFROM):
             sym.append(("ctl", OP.MAP_EXIT, lo * 8, (hi - lo) * 8, t | MAP.ALWAYS))
+        sym.append(("ctl", OP.MAP_ENTER, lo * 8, (hi - lo) * 8, MAP.TO | MAP.PRESENT))
     return sym
 
 

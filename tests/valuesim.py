@@ -25,6 +25,7 @@ RH, WH, RT, WT, MAP_ENTER, MAP_EXIT, UPDATE = 0, 1, 2, 3, 8, 9, 10
 TASK_BEGIN, TASK_END, SYNC = 12, 13, 14
 TO, FROM, TOFROM, ALLOC, RELEASE, DELETE = 0, 1, 2, 3, 4, 5
 ALWAYS = 0x10                       # map-type modifier bit (N4, reading Z21)
+PRESENT = 0x20                      # map-type modifier bit: the section must already be mapped
 UUM, USD, BO = 1, 2, 4
 
 
@@ -102,13 +103,16 @@ class ValueSim:
 
     def record(self, op, addr, length, arg, idx):
         always = bool(arg & ALWAYS)           # OpenMP 5.1 `always` map-type modifier (reading Z21)
-        arg &= ~ALWAYS
+        present = bool(arg & PRESENT)         # OpenMP 5.1 `present`: not mapped -> error
+        arg &= ~(ALWAYS | PRESENT)
         if op in (RH, WH, RT, WT):
             name = {RH: "RH", WH: "WH", RT: "RT", WT: "WT"}[op]
             for w in self.words(addr, length):
                 self.word_op(name, w, idx)
         elif op == MAP_ENTER:
             ent = self._lookup(addr, addr + length)
+            if ent is None and present:
+                raise MapError("present modifier on an unmapped section")
             if ent is not None:
                 ent[2] += 1
                 if always and arg in (TO, TOFROM):
