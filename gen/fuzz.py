@@ -65,6 +65,8 @@ def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: i
                 mt = int(rs.choice([MAP.TO, MAP.FROM, MAP.TOFROM, MAP.ALLOC]))
                 if p_always and rs.random() < p_always:
                     mt |= MAP.ALWAYS
+                if p_always and any(a <= lo and hi <= b for a, b in present[i]) and rs.random() < p_always:
+                    mt |= MAP.PRESENT            # a mapped section: `present` holds
                 tb.enter(mt, lo, n)
                 present[i].append((lo, hi))
         elif r < 0.65:

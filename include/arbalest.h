@@ -54,6 +54,9 @@ enum arb_map { ARB_TO = 0, ARB_FROM = 1, ARB_TOFROM = 2, ARB_ALLOC = 3,
  * MAP_ENTER to/tofrom copies OV->CV even when the entry is present, MAP_EXIT
  * from/tofrom copies CV->OV even when the reference count stays above 0 */
 #define ARB_MAP_ALWAYS 0x10u
+/* map-type modifier `present` (MAP_ENTER): the section must already be mapped,
+ * else the flush fails with ARB_EMAP (OpenMP 5.1 runtime error; Z21) */
+#define ARB_MAP_PRESENT 0x20u
 /* target update direction */
 enum arb_upd { ARB_UPD_TO = 0, ARB_UPD_FROM = 1 };
 #define ARB_SYNC_ALL 0xFFFFu

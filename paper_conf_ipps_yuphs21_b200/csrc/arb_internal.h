@@ -16,6 +16,7 @@ enum Op : uint32_t { OP_RH = 0, OP_WH = 1, OP_RT = 2, OP_WT = 3,
 enum MapType : uint32_t { MT_TO = 0, MT_FROM = 1, MT_TOFROM = 2, MT_ALLOC = 3,
                           MT_RELEASE = 4, MT_DELETE = 5 };
 constexpr uint32_t kMapAlways = 0x10;   // `always` map-type modifier bit (N4, Z21)
+constexpr uint32_t kMapPresent = 0x20;  // `present`: an unmapped section is a mapping error (Z21)
 constexpr uint32_t kSyncAll = 0xFFFFu;
 
 // ---- VSM bits (Table II) ----------------------------------------

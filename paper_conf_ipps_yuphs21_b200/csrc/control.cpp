@@ -96,12 +96,14 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
       }
       case OP_MAP_ENTER: {                          // Table I, entry
         const bool always = arg & kMapAlways;       // Z21
-        arg &= ~kMapAlways;
+        const bool present = arg & kMapPresent;
+        arg &= ~(kMapAlways | kMapPresent);
         if (arg > MT_ALLOC || len == 0 || addr + len > (1ull << 48))
           return fail(ARB_ETRACE, c.pos, "bad MAP_ENTER record");
         MapTable::iterator it;
         int f = map_find(map, addr, addr + len, it);
         if (f < 0) return fail(ARB_EMAP, c.pos, "map clause partially overlaps a present entry");
+        if (f == 0 && present) return fail(ARB_EMAP, c.pos, "map(present) of a section that is not mapped");
         if (f == 1) {                               // exist(CV): ref_count += 1, no transfer ...
           it->second.rc += 1;
           if (always && (arg == MT_TO || arg == MT_TOFROM)) em.emit(pos, kSelUPT, addr, addr + len, open);

@@ -155,7 +155,7 @@ def test_dedup_first(orc):
     check(orc, rec, base, size, dedup_first=True)
 
 
-@pytest.mark.parametrize("bad", ["op", "len", "emap", "nested"])
+@pytest.mark.parametrize("bad", ["op", "len", "emap", "present", "nested"])
 def test_errors_leave_state_unchanged(orc, bad):
     from gen.trace import MAP, TraceBuilder
     from paper_conf_ipps_yuphs21_b200 import Context, reports_to_triples
@@ -171,6 +171,8 @@ def test_errors_leave_state_unchanged(orc, bad):
         tb.rh(A, 0)
     elif bad == "emap":
         tb.enter(MAP.TO, A + 32, 64)
+    elif bad == "present":
+        tb.enter(MAP.TO | MAP.PRESENT, A + 128, 64)       # not mapped: ARB_EMAP (Z21)
     elif bad == "eopen":
         tb.task_begin(3); tb.wt(A)
     elif bad == "nested":
