@@ -27,6 +27,7 @@
  *   MIR attribution to later event (Z11)  parity unpinned (definition only)
  *   dedup-first mode (Z3)                 parity unpinned (definition only)
  *   sub-word semantics (Z4)               parity unpinned (definition only)
+ *   unified memory (Z23)                  pinned (brute force vs the value simulator with OV and CV aliased)
  *   depend (Z22)                          pinned (schedule enumeration with dependencies + witness search)
  *   buffer overflow, present-bit form (Z20) pinned (P:279 worked example + brute force vs the
  *                                         value simulator's CV existence); the paper's base-interval
@@ -94,6 +95,12 @@ typedef struct {
    * ORC_BO and has no VSM effect (no UUM/USD check, no transition: the access
    * did not touch this word's CV).  0 = off (the 4-bit VSM of P:255-263). */
   int             detect_bo;
+  /* Unified-memory mode (reading Z23): OV and CV are
+   * one storage, so map clauses and target update move no data (refcount
+   * bookkeeping and ORC_EMAP only, no word-ops), a write by either side is
+   * visible to both (all four bits set), reads fault only on never-written
+   * words (UUM), and races among the accesses remain (MIR).  Excludes detect_bo. */
+  int             unified;
 } orc_config;
 
 typedef struct {

@@ -45,7 +45,7 @@ def encode_seq(seq, base):
     return out
 
 
-def check_batch(orc, seqs, nwords, bo=False):
+def check_batch(orc, seqs, nwords, bo=False, unified=False):
     """Concatenate the sequences on disjoint arrays, run the oracle once, compare per array.
     bo: the buffer-overflow extension on both sides (reading Z20)."""
     stride = 8 * nwords
@@ -53,7 +53,7 @@ def check_batch(orc, seqs, nwords, bo=False):
     for j, seq in enumerate(seqs):
         base = stride * j
         enc = encode_seq(seq, base)
-        vs = ValueSim(bo=bo)
+        vs = ValueSim(bo=bo, unified=unified)
         try:
             issues = vs.run(enc)
         except MapError:
@@ -65,7 +65,7 @@ def check_batch(orc, seqs, nwords, bo=False):
         states.extend(vs.state_bits(base // 8 + w) for w in range(nwords))
     arr = np.array(recs, dtype=np.uint64).reshape(-1, 2)
     nseq = len(offsets)
-    res = orc.replay(arr, 0, stride * (len(seqs)), detect_bo=bo)
+    res = orc.replay(arr, 0, stride * (len(seqs)), detect_bo=bo, unified=unified)
     assert res.rc == 0
     assert res.triples() == sorted(expect)
     # final states: only the arrays that were kept
@@ -187,3 +187,13 @@ def test_always_random_long(orc):
     rs = np.random.default_rng(14)
     seqs = [tuple(sym[i] for i in rs.integers(0, len(sym), rs.integers(4, 9))) for _ in range(40000)]
     check_batch(orc, seqs, 2)
+
+
+@pytest.mark.parametrize("nwords,length", [(1, 4), (2, 3)])
+def test_unified_exhaustive(orc, nwords, length):
+    """Unified memory (reading Z23): the oracle's reports and final
+    states equal the value simulator's with OV and CV aliased (one storage; only
+    never-written words can be read wrongly — no stale copies exist)."""
+    sym = alphabet_always(nwords)
+    seqs = [s for L in range(1, length + 1) for s in itertools.product(sym, repeat=L)]
+    assert check_batch(orc, seqs, nwords, unified=True) > 50000

@@ -356,3 +356,18 @@ def test_always_modifier_nested_region(orc):
         assert ((i_rt, USD) in kinds) == expect_usd          # the kernel read sees the old CV
         assert ((i_rh, USD) in kinds) == expect_usd          # the host read misses the kernel write
         assert sorted(ValueSim().run(tb.array())) == res.triples()
+
+
+def test_unified_memory_paper(orc):
+    """Unified memory (reading Z23): "on-demand page migration helps
+    resolve data mapping issues in a data-race-free OpenMP application" — Fig. 1's
+    UUMs and Fig. 2's stale reads disappear, the synchronized Fig. 2 is clean — but
+    "data mapping issues may arise when updates on the host and reads on the GPU
+    occur concurrently without proper synchronization": the host accesses of lines
+    13 and 16 still race with the nowait region (the exit transfer of line 14 no
+    longer exists, so it no longer races)."""
+    for name, expect in (("fig1_n3.trace", set()), ("fig2_sync.trace", set()),
+                         ("fig2_no_sync.trace", {(10, MIR), (11, MIR), (13, MIR)})):
+        rec, base, size, _ = load(name)
+        res = run(orc, rec, base, size, unified=True)
+        assert {(r, k) for _, r, k in res.triples()} == expect, name

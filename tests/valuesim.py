@@ -39,11 +39,14 @@ class ValueSim:
     does not reach this word's CV at all; it is reported as BO and changes
     nothing.  CV existence is tracked as a set of words here, not as a bit."""
 
-    def __init__(self, bo: bool = False):
+    def __init__(self, bo: bool = False, unified: bool = False):
+        """unified=True: unified memory (reading Z23): OV and CV are the same
+        storage (one dict), so transfers, allocation and release change nothing."""
         self.bo = bo
+        self.unified = unified
         self.alive: set[int] = set()      # words whose CV exists
         self.ov: dict[int, int] = {}
-        self.cv: dict[int, int] = {}
+        self.cv: dict[int, int] = self.ov if unified else {}
         self.latest: dict[int, int] = {}
         self.next_id = 1
         self.present: list[list[int]] = []  # [lo, hi, refcount] byte intervals
@@ -74,6 +77,8 @@ class ValueSim:
             self._write(self.ov, w)
         elif name == "WT":
             self._write(self.cv, w)
+        elif self.unified and name in ("UPT", "UPH", "NEW", "DEL"):
+            return                        # one storage: nothing moves, nothing is (de)allocated
         elif name == "UPT":   # memcpy(CV, OV)
             self.cv[w] = self.ov.get(w, BOT)
         elif name == "UPH":   # memcpy(OV, CV)
