@@ -94,6 +94,12 @@ enum arb_status {
                                    replay every small bucket with >= 64 events as 3 time
                                    slices (the mechanisms normally used for range-heavy
                                    and hot buckets only)                                  */
+#define ARB_F_UNIFIED     0x10u /* unified memory (Z23): OV and CV are one
+                                   storage — map clauses and target update move no data
+                                   (reference counts and ARB_EMAP only), a write of either side
+                                   is visible to both, reads fault only on never-written words
+                                   (UUM), races among the accesses are still MIR.  Excludes
+                                   ARB_F_BO (ARB_EINVAL)                                   */
 #define ARB_F_BO          0x8u  /* buffer-overflow extension (reading Z20): every
                                    word carries a 5th state bit "has a CV" (set by allocate,
                                    cleared by release); a target access (RT/WT) to a word

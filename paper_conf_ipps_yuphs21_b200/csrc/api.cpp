@@ -188,7 +188,8 @@ extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
   *out = nullptr;
   if (!cfg || (cfg->addr_base & 7) || (cfg->addr_bytes & 7) || cfg->addr_bytes == 0 ||
       cfg->addr_base + cfg->addr_bytes > (1ull << 48) || cfg->world < 1 || cfg->rank < 0 ||
-      cfg->rank >= cfg->world || (cfg->world > 1 && !cfg->nccl_unique_id))
+      cfg->rank >= cfg->world || (cfg->world > 1 && !cfg->nccl_unique_id) ||
+      ((cfg->flags & ARB_F_BO) && (cfg->flags & ARB_F_UNIFIED)))
     return ARB_EINVAL;
   arb_ctx ctx = new (std::nothrow) arb_ctx_s();
   if (!ctx) return ARB_ENOMEM;
@@ -581,7 +582,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   MapTable map = ctx->map;
   FlushPlan plan;
   resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_start, map, plan,
-                  (ctx->cfg.flags & ARB_F_BO) != 0, &ctx->carried);
+                  (ctx->cfg.flags & ARB_F_BO) != 0, &ctx->carried, (ctx->cfg.flags & ARB_F_UNIFIED) != 0);
   if (plan.rc != 0) {
     CK(cudaStreamSynchronize(s), "sync");
     reset_batch(ctx);
@@ -622,7 +623,8 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   rp.n_buckets = ctx->n_buckets; rp.bucket_bits = ctx->bucket_bits; rp.n_words = ctx->n_words;
   rp.bucket_start = ctx->d_bucket_start.p;
   rp.items = ctx->d_items.p; rp.n_items = (uint32_t)ctx->items.size();
-  rp.shadow = ctx->shadow; rp.bo = (ctx->cfg.flags & ARB_F_BO) ? 1u : 0u; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
+  rp.shadow = ctx->shadow; rp.bo = (ctx->cfg.flags & ARB_F_BO) ? 1u : 0u;
+  rp.um = (ctx->cfg.flags & ARB_F_UNIFIED) ? 1u : 0u; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
   rp.cand = ctx->cand.p; rp.cand_cap = ctx->cand_cap; rp.st = ctx->dstats.p;
   rp.hot_off = ctx->d_hot_off.p; rp.hot_F = ctx->hot_F.p; rp.hot_P = ctx->hot_P.p;
   int n_ctas = std::max(1, std::min<int>((int)ctx->items.size(), ctx->n_sms * kReplayCtasPerSm));

@@ -144,6 +144,7 @@ struct ReplayParams {
   uint64_t n_words;
   uint8_t* shadow;                        // n_words bytes
   uint32_t bo;                            // ARB_F_BO: target accesses to words without kCVp are BO
+  uint32_t um;                            // ARB_F_UNIFIED: OV and CV are one storage (Z23)
   const uint32_t* ops_start;              // [n_buckets + 1]
   const BucketOp* ops;
   uint4* cand; uint64_t cand_cap;         // report candidates {word lo, word hi, pos, kind}

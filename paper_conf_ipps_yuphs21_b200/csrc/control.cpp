@@ -25,7 +25,9 @@ int map_find(MapTable& m, uint64_t lo, uint64_t hi, MapTable::iterator& it) {
 struct Emitter {
   uint64_t base_word, n_words;
   FlushPlan* out;
+  bool none;                              // unified memory: no data op exists (Z23)
   void emit(uint32_t pos, Sel sel, uint64_t byte_lo, uint64_t byte_hi, uint32_t inst) {
+    if (none) return;
     uint64_t w0 = byte_lo >> 3, w1 = ((byte_hi - 1) >> 3) + 1;    // [w0, w1) absolute
     uint64_t total = w1 - w0;
     uint64_t lo = std::max(w0, base_word), hi = std::min(w1, base_word + n_words);
@@ -40,10 +42,10 @@ struct Emitter {
 
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
-                     FlushPlan& out, bool bo, const std::vector<CarriedInst>* carried_in) {
+                     FlushPlan& out, bool bo, const std::vector<CarriedInst>* carried_in, bool unified) {
   const uint32_t n_buckets = (uint32_t)bucket_start.size() - 1;
   out = FlushPlan();
-  Emitter em{base_word, n_words, &out};
+  Emitter em{base_word, n_words, &out, unified};
   // task instances (1-based; 0 = host); instances 1..nc are the carried-in ones:
   // they began before this flush (t_begin = kBefore) and either ended before it
   // (t_end = kBefore) or are still open (t_end = kOpen until their TASK_END)

@@ -62,6 +62,9 @@ struct FlushPlan {
 // are returned in out.carry_out instead of being treated as joined (Z19).
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
-                     FlushPlan& out, bool bo = false, const std::vector<CarriedInst>* carried_in = nullptr);
+                     FlushPlan& out, bool bo = false, const std::vector<CarriedInst>* carried_in = nullptr,
+                     bool unified = false);
+// unified (ARB_F_UNIFIED, Z23): map clauses and target update keep the reference
+// counts (and their errors) but emit no range ops: nothing moves between OV and CV.
 
 }  // namespace arb

@@ -227,7 +227,9 @@ __device__ __forceinline__ uint32_t hslot(uint32_t w) { return (w * 2654435761u)
 // BO (ARB_F_BO) is a template parameter: deciding that a target access is a
 // buffer overflow needs its word's state before the inserts, which would put
 // the shadow-load latency in front of the hashing for every replay.
-template <bool PARTIAL, bool BO>
+// UM (ARB_F_UNIFIED, Z23): OV and CV are one storage — a write of either side
+// makes the word's state 0xF (both valid, both initialised).
+template <bool PARTIAL, bool BO, bool UM>
 __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
   uint32_t slot[RI], word[RI], pos[RI], op[RI], s_pre[RI];
   uint32_t bom = 0;                // bit j: event j is a buffer overflow (ARB_F_BO, Z20)
@@ -285,7 +287,7 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
         for (;;) {                                          // probe for the word's write
           const uint2 k = hs[h];
           if (k.x == word[j]) {
-            if ((k.y >> 2) < pos[j]) before = vsm_write_op(k.y & 3u, s0);
+            if ((k.y >> 2) < pos[j]) before = UM ? 15u : vsm_write_op(k.y & 3u, s0);
             break;
           }
           if (k.x == kEmpty) break;
@@ -293,7 +295,8 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
         }
       }
     } else if (op[j] & 1u) {
-      __stcg(const_cast<uint8_t*>(sh) + word[j], (uint8_t)(vsm_write_op(op[j], s0) | (BO ? (s_pre[j] & kCVp) : 0u)));
+      __stcg(const_cast<uint8_t*>(sh) + word[j],
+             (uint8_t)(UM ? 15u : vsm_write_op(op[j], s0) | (BO ? (s_pre[j] & kCVp) : 0u)));
     }
     fk[j] = ((bom >> j) & 1u) ? 4u : classify_bits(op[j], before);
   }
@@ -309,9 +312,9 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
 }
 
 // the fast step of a word-range part (rare: range-heavy buckets), out of line
-template <bool BO>
+template <bool BO, bool UM>
 __device__ bool step_fast_partial(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
-  return step_fast<true, BO>(S, p, ev, m);
+  return step_fast<true, BO, UM>(S, p, ev, m);
 }
 
 // ---- sort step -------------------------------------------------------------------------
@@ -402,7 +405,7 @@ __device__ __forceinline__ uint32_t acc_summary(uint32_t op) {
   return op == OP_WH ? (1u | 4u) : (op == OP_WT ? (2u | 8u) : 0u);
 }
 
-template <bool BO>
+template <bool BO, bool UM>
 __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   uint32_t lo = 0xFFFFFFFFu, hi = 0;
@@ -480,7 +483,8 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
       // access to a word without a CV is BO and the identity (Z20)
       const uint32_t full = (h || bo) ? __ldcg(sh + w) : 0u;
       const bool b = bo && ((k >> 30) & 2u) && !(full & kCVp);
-      uint32_t v = b ? 0u : acc_summary(k >> 30);
+      // UM: every write is {both valid, both initialised} (last write 3, any-WH and any-WT)
+      uint32_t v = b ? 0u : UM ? (((k >> 30) & 1u) ? 15u : 0u) : acc_summary(k >> 30);
       uint32_t st = 0;
       if (h) {
         st = full & 15u;
@@ -530,6 +534,7 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
 // writes compose to: valid bits of the last write, OVi set if any WH, CVi set if
 // any WT (Table II init bits); the last write of each word (by step
 // index) folds that function into fsum.
+template <bool UM>
 __device__ void step_summary(ReplaySmem& S, const uint2* ev, uint32_t m) {
   uint32_t* key = S.u.z.key;
   uint32_t* lastw = S.u.z.lastw;
@@ -567,7 +572,8 @@ __device__ void step_summary(ReplaySmem& S, const uint2* ev, uint32_t m) {
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
     if (last[j]) {
-      const Sel g = op[j] == OP_WH ? sel_make(5, 4, 5, (ab[j] & 2u) ? 5 : 3)     // OV latest; CVi kept unless a WT
+      const Sel g = UM ? sel_make(5, 5, 5, 5)                                      // Z23: one shared value
+                  : op[j] == OP_WH ? sel_make(5, 4, 5, (ab[j] & 2u) ? 5 : 3)     // OV latest; CVi kept unless a WT
                                    : sel_make(4, 5, (ab[j] & 1u) ? 5 : 2, 5);    // CV latest; OVi kept unless a WH
       S.fsum[word[j]] = (uint16_t)sel_compose(g, S.fsum[word[j]]);
       key[slot[j]] = kEmpty;           // the word's only slot: reset by its last writer
@@ -753,7 +759,7 @@ __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t 
 
 // BO: ARB_F_BO contexts (the buffer-overflow extension, Z20) get their own
 // instance, so the default replay carries none of its checks.
-template <bool BO>
+template <bool BO, bool UM>
 __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   ReplaySmem& S = *reinterpret_cast<ReplaySmem*>(smem_raw);
@@ -841,10 +847,10 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         cut = block_sum(cnt, S.red);
       }
       if (mode == kItemSummary) {
-        step_summary(S, ev, cut);
+        step_summary<UM>(S, ev, cut);
       } else {
-        const bool fast = S.partial ? step_fast_partial<BO>(S, p, ev, cut) : step_fast<false, BO>(S, p, ev, cut);
-        if (!fast) step_sort<BO>(S, p, ev, cut);
+        const bool fast = S.partial ? step_fast_partial<BO, UM>(S, p, ev, cut) : step_fast<false, BO, UM>(S, p, ev, cut);
+        if (!fast) step_sort<BO, UM>(S, p, ev, cut);
         if (tid == 0) atomicAdd(fast ? &p.st->steps_fast : &p.st->steps_sort, 1ull);
       }
       e0 += cut;
@@ -873,7 +879,8 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
 
 cudaError_t launch_replay(const ReplayParams& p, int n_ctas, cudaStream_t s) {
   const size_t smem = sizeof(ReplaySmem);
-  auto kern = p.bo ? k_replay<true> : k_replay<false>;
+  // ARB_F_BO and ARB_F_UNIFIED exclude each other (arb_init)
+  auto kern = p.um ? k_replay<false, true> : p.bo ? k_replay<true, false> : k_replay<false, false>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   kern<<<n_ctas, RT, smem, s>>>(p);

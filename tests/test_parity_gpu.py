@@ -16,6 +16,7 @@ def check(orc, rec, base, size, **kw):
     okw = {k: kw.pop(k) for k in ("dedup_first",) if k in kw}
     flags = (1 if okw.get("dedup_first") else 0) | kw.pop("flags", 0)
     okw["detect_bo"] = bool(flags & 8)                    # ARB_F_BO <-> the oracle's extension (Z20)
+    okw["unified"] = bool(flags & 16)                     # ARB_F_UNIFIED <-> unified memory (Z23)
     exp = orc.replay(rec, base, size, **okw)
     rc, got, shadow, st = run_gpu(rec, base, size, flags=flags, **kw)
     assert rc == exp.rc
@@ -397,3 +398,52 @@ def test_depend_fuzz(orc, seed):
     if exp.rc == 0:
         rc, got, shadow, _ = run_gpu(rec, base, span, flush_points=_cuts(rec, 5, seed))
         assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+# ---- unified memory (ARB_F_UNIFIED = 16, Z23) ---------------------
+@pytest.mark.parametrize("name", ["fig1_n3.trace", "fig2_no_sync.trace", "fig2_sync.trace"])
+def test_unified_golden(orc, name):
+    rec, base, size, _ = load(name)
+    check(orc, rec, base, size, flags=16)
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_unified_fuzz(orc, seed):
+    """Random programs (tasks, depend, modifiers) under unified memory, several bucket
+    sizes, forced parts / time slices (flags 4), and flush cuts."""
+    from gen.fuzz import random_program
+    rec, base, span = random_program(7000 + seed, p_task=0.3, p_always=0.3, p_depend=0.3, steps=120)
+    exp, _ = check(orc, rec, base, span, flags=16)
+    for bb in (2, 5):
+        check(orc, rec, base, span, bucket_bits=bb, flags=16)
+    check(orc, rec, base, span, flags=16 | 4)
+    if exp.rc == 0:
+        rc, got, shadow, _ = run_gpu(rec, base, span, flags=16, flush_points=_cuts(rec, 4, seed))
+        ex2 = orc.replay(rec, base, span, unified=True)
+        assert rc == 0 and sorted(got) == ex2.triples() and np.array_equal(shadow, ex2.shadow)
+
+
+def test_unified_config2_and_hot_word(orc):
+    from gen.configs import config2
+    from gen.trace import MAP, OP, TraceBuilder
+    rec, base, size = config2()
+    check(orc, rec, base, size, flags=16)
+    tb = TraceBuilder()
+    A = 0x8000
+    tb.wh(A)
+    tb.enter(MAP.TO, A, 64)
+    rs = np.random.default_rng(8)
+    ops = rs.choice([OP.RT, OP.WT, OP.RH, OP.WH], size=400000, p=[.4, .2, .3, .1])
+    arr = np.zeros((ops.size, 2), dtype=np.uint64)
+    arr[:, 0] = np.uint64(A) | (ops.astype(np.uint64) << np.uint64(48))
+    arr[:, 1] = 8
+    tb.add_array(arr)
+    tb.exit(MAP.TOFROM, A, 64)
+    _, st = check(orc, tb.array(), A, 64, flags=16)
+    assert st["hot_buckets"] >= 1                      # K5 time slices compose the shared-value writes
+
+
+def test_unified_excludes_bo():
+    from paper_conf_ipps_yuphs21_b200 import Context, ArbError
+    with pytest.raises(ArbError):
+        Context(0x1000, 4096, flags=8 | 16)
