@@ -18,7 +18,7 @@
  *   log the op if it runs inside a nowait task.  Output: the sorted unique
  *   (word, record, kind) triples and the final 4-bit state of every word.
  *
- * Parity status of each part (DESIGN.md §9):
+ * Parity status of each part (DESIGN.md §2, §4):
  *   VSM edges / fault condition          pinned (prose edges + Definition-1 brute force)
  *   UUM-vs-USD split (init bits, Z2)      pinned to Definition 1 (value simulator);
  *                                         parity unpinned BY THE PAPER (Fig.1/Fig.2 do not split readings)
@@ -27,6 +27,7 @@
  *   MIR attribution to later event (Z11)  parity unpinned (definition only)
  *   dedup-first mode (Z3)                 parity unpinned (definition only)
  *   sub-word semantics (Z4)               parity unpinned (definition only)
+ *   map modifiers always/present (Z21)    pinned (brute force vs the value simulator's own refcount model)
  *   unified memory (Z23)                  pinned (brute force vs the value simulator with OV and CV aliased)
  *   depend (Z22)                          pinned (schedule enumeration with dependencies + witness search)
  *   buffer overflow, present-bit form (Z20) pinned (P:279 worked example + brute force vs the
