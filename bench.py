@@ -253,6 +253,12 @@ def main():
     prog = make_program(args.workload, args.scale)
     t_gen = time.perf_counter()
     recs, gidx, flushes, (lo, hi) = rank_batches(prog, rank, world, dev)
+    if world > 1:
+        # every arb_flush exchanges the report counts (ncclAllGather), so all ranks
+        # must flush equally often: pad the shorter schedules with empty flushes
+        nf = torch.tensor([len(flushes)], dtype=torch.int64, device=dev)
+        dist.all_reduce(nf, op=dist.ReduceOp.MAX)
+        flushes = flushes + [(recs.shape[0], recs.shape[0])] * (int(nf.item()) - len(flushes))
     torch.cuda.synchronize()
     t_gen = time.perf_counter() - t_gen
 
@@ -325,8 +331,10 @@ def main():
     value = word_events_all * args.steps / (ms_max / 1e3)
     ms_per_step = ms_max / args.steps
 
+    n_busy = max(1, sum(1 for a, b in flushes if b > a))   # non-empty flushes (kernel launches)
     # ---- roofline: B_alg = 16 R + 2 W + 16 Rep -------------------------
-    W = sum(prog.distinct_words(lo, hi, [(int(gidx[a].item()), int(gidx[b - 1].item()) + 1) for a, b in flushes]))
+    W = sum(prog.distinct_words(lo, hi, [(int(gidx[a].item()), int(gidx[b - 1].item()) + 1)
+                                         for a, b in flushes if b > a]))
     b_alg = 16 * s0["records"] + 2 * W + 16 * s0["reports"]
     step_ms_lib = s0["ms_total"]
     phases = {"k_sample+balance": s0["ms_sample"], "k_partition": s0["ms_partition"] - s0["ms_sample"],
@@ -345,7 +353,7 @@ def main():
     try:
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as fh:
             tj = json.load(fh)[dom]
-        traffic = tj["dram_bytes_per_launch"] / tj["records_in_launch"] * s0["records"] / len(flushes)
+        traffic = tj["dram_bytes_per_launch"] / tj["records_in_launch"] * s0["records"] / n_busy
     except Exception:
         pass
     kern = {}
@@ -360,7 +368,7 @@ def main():
             pass
     roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": hbm_gbs, "unit": "GB/s",
             "frac": achieved / hbm_gbs, "traffic": traffic, "traffic_unit": "bytes per launch (ncu)",
-            "alg_bytes_per_launch": alg[dom] / len(flushes), "peak_source": peak_src,
+            "alg_bytes_per_launch": alg[dom] / n_busy, "peak_source": peak_src,
             "kernel_ms_per_step": phases[dom], "phase_ms_per_step": phases, "kernels": kern,
             "path": {"b_alg_bytes_per_step": b_alg, "achieved": b_alg / (ms_per_step / 1e3) / 1e9,
                      "frac": b_alg / (ms_per_step / 1e3) / 1e9 / hbm_gbs}}
@@ -410,7 +418,7 @@ def main():
                            "access_word_events_per_step_rank0": int(s0["access_words"]),
                            "range_word_events_per_step_rank0": int(s0["range_words"]),
                            "reports_per_step": int(reports_all), "reports_by_kind_rank0": s0["by_kind"][1:],
-                           "flushes_per_step_rank0": len(flushes), "shard_words": hi - lo,
+                           "flushes_per_step_rank0": n_busy, "shard_words": hi - lo,
                            "replay_steps_fast_sort_rank0": [int(s0["steps_fast"]), int(s0["steps_sort"])],
                            "max_bucket_events_rank0": int(s0["max_bucket_events"]),
                            "replay_work_items_rank0": int(s0["work_items"]),

@@ -447,3 +447,14 @@ def test_unified_excludes_bo():
     from paper_conf_ipps_yuphs21_b200 import Context, ArbError
     with pytest.raises(ArbError):
         Context(0x1000, 4096, flags=8 | 16)
+
+
+def test_empty_flushes(orc):
+    """An empty batch flushes cleanly (multi-GPU runs pad their flush schedules with
+    them so that every rank joins every count exchange) and changes nothing."""
+    from gen.configs import config1
+    rec, base, size = config1()
+    exp = orc.replay(rec, base, size)
+    rc, got, shadow, st = run_gpu(rec, base, size, flush_points=[0, 0, rec.shape[0], rec.shape[0]])
+    assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+    assert st["flushes"] == 5
