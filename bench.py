@@ -408,7 +408,7 @@ def main():
 
     if rank == 0:
         cpu = None
-        if not args.no_cpu:
+        if not args.no_cpu and world == 1:        # the oracle baseline is an N = 1 figure
             cpu = cpu_baseline(prog, recs, gidx, lo, hi, args.cpu_records)
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
