@@ -27,6 +27,7 @@
  *   MIR attribution to later event (Z11)  parity unpinned (definition only)
  *   dedup-first mode (Z3)                 parity unpinned (definition only)
  *   sub-word semantics (Z4)               parity unpinned (definition only)
+ *   several accelerators (Z24)            pinned (brute force vs the value simulator with one CV per device)
  *   map modifiers always/present (Z21)    pinned (brute force vs the value simulator's own refcount model)
  *   unified memory (Z23)                  pinned (brute force vs the value simulator with OV and CV aliased)
  *   depend (Z22)                          pinned (schedule enumeration with dependencies + witness search)
@@ -102,6 +103,13 @@ typedef struct {
    * visible to both (all four bits set), reads fault only on never-written
    * words (UUM), and races among the accesses remain (MIR).  Excludes detect_bo. */
   int             unified;
+  /* Several accelerators (reading Z24): n_devices > 1
+   * gives every word an (n+1)-tuple — OV plus one CV per device d < n_devices
+   * (n <= 3), each with its valid and initialised bit — and one mapping table
+   * per device.  The device is arg of RT/WT records and bits 6-7 of the arg of
+   * MAP_ENTER / MAP_EXIT / UPDATE.  Single-device traces are unchanged.
+   * Excludes detect_bo and unified.  (Oracle only: the CUDA path is single-device.) */
+  int             n_devices;
 } orc_config;
 
 typedef struct {
@@ -119,7 +127,8 @@ typedef struct {
  * order (word, record, kind ascending) that the caller frees with
  * orc_free(); shadow_out (dense: addr_bytes/8 bytes, sparse: n_tracked
  * bytes, may be NULL) receives the final states (bit0 OVv, bit1 CVv,
- * bit2 OVi, bit3 CVi — Table II; bit4 CVp with detect_bo).
+ * bit2 OVi, bit3 CVi — Table II; bit4 CVp with detect_bo; with
+ * n_devices > 1 bits 4/5 and 6/7 are CV valid/initialised of devices 1 and 2).
  * Returns ORC_OK or an error. */
 int  orc_replay(const orc_config* cfg, const orc_record* rec, uint64_t n,
                 const uint64_t* global_index, orc_report** out, uint64_t* n_out,

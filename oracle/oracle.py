@@ -26,7 +26,8 @@ class _Config(ctypes.Structure):
     _fields_ = [("addr_base", ctypes.c_uint64), ("addr_bytes", ctypes.c_uint64),
                 ("dedup_first", ctypes.c_int),
                 ("tracked_words", ctypes.POINTER(ctypes.c_uint64)),
-                ("n_tracked", ctypes.c_uint64), ("detect_bo", ctypes.c_int), ("unified", ctypes.c_int)]
+                ("n_tracked", ctypes.c_uint64), ("detect_bo", ctypes.c_int), ("unified", ctypes.c_int),
+                ("n_devices", ctypes.c_int)]
 
 
 class _Stats(ctypes.Structure):
@@ -80,7 +81,8 @@ class OracleResult:
 
 def replay(records: np.ndarray, addr_base: int, addr_bytes: int, *, dedup_first: bool = False,
            tracked_words: np.ndarray | None = None, global_index: np.ndarray | None = None,
-           want_shadow: bool = True, detect_bo: bool = False, unified: bool = False) -> OracleResult:
+           want_shadow: bool = True, detect_bo: bool = False, unified: bool = False,
+           n_devices: int = 1) -> OracleResult:
     """Replay ``records`` (uint64 array of shape (n, 2): w0, w1) through the oracle.
     ``detect_bo``: the buffer-overflow extension (reading Z20)."""
     lib = _load()
@@ -92,6 +94,7 @@ def replay(records: np.ndarray, addr_base: int, addr_bytes: int, *, dedup_first:
     cfg.dedup_first = 1 if dedup_first else 0
     cfg.detect_bo = 1 if detect_bo else 0
     cfg.unified = 1 if unified else 0
+    cfg.n_devices = n_devices
     tw = None
     if tracked_words is not None:
         tw = np.ascontiguousarray(tracked_words, dtype=np.uint64)

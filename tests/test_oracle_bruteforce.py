@@ -197,3 +197,63 @@ def test_unified_exhaustive(orc, nwords, length):
     sym = alphabet_always(nwords)
     seqs = [s for L in range(1, length + 1) for s in itertools.product(sym, repeat=L)]
     assert check_batch(orc, seqs, nwords, unified=True) > 50000
+
+
+def alphabet_devices(ndev):
+    """One word, several accelerators (reading Z24): host accesses, target
+    accesses and map / update clauses on every device (device in the access arg,
+    in bits 6-7 of a map / update arg)."""
+    sym = [("acc", OP.RH, 0, 8), ("acc", OP.WH, 0, 8)]
+    for d in range(ndev):
+        sym += [("accd", OP.RT, d), ("accd", OP.WT, d)]
+        for t in (MAP.TO, MAP.FROM, MAP.TOFROM, MAP.ALLOC):
+            sym.append(("ctl", OP.MAP_ENTER, 0, 8, t | (d << 6)))
+        for t in (MAP.FROM, MAP.TOFROM, MAP.RELEASE):
+            sym.append(("ctl", OP.MAP_EXIT, 0, 8, t | (d << 6)))
+        for u in (UPD.TO, UPD.FROM):
+            sym.append(("ctl", OP.UPDATE, 0, 8, u | (d << 6)))
+    return sym
+
+
+def _enc_dev(seq, base):
+    out = []
+    for s in seq:
+        if s[0] == "accd":
+            out.append(encode(s[1], base, 8, arg=s[2]))
+        elif s[0] == "acc":
+            out.append(encode(s[1], base + s[2], s[3]))
+        else:
+            out.append(encode(s[1], base + s[2], s[3], arg=s[4]))
+    return out
+
+
+@pytest.mark.parametrize("ndev,length", [(2, 4), (3, 3)])
+def test_devices_exhaustive(orc, ndev, length):
+    """Several accelerators: the oracle's (n+1)-tuple states and reports equal the
+    value simulator's with one CV and one mapping table per device."""
+    sym = alphabet_devices(ndev)
+    recs, expect, states, n = [], [], [], 0
+    for L in range(1, length + 1):
+        for j, seq in enumerate(itertools.product(sym, repeat=L)):
+            base = 8 * n
+            enc = _enc_dev(seq, base)
+            vs = ValueSim(devices=ndev)
+            try:
+                issues = vs.run(enc)
+            except MapError:
+                continue
+            off = len(recs)
+            recs.extend(enc)
+            expect.extend((w, i + off, k) for (w, i, k) in issues)
+            states.append(vs.state_bits(base // 8))
+            n += 1
+    res = orc.replay(np.array(recs, dtype=np.uint64).reshape(-1, 2), 0, 8 * n, n_devices=ndev)
+    assert res.rc == 0
+    assert res.triples() == sorted(expect)
+    assert res.shadow.tolist() == states
+    assert n > 20000
+    # a single-device run of device-0-only sequences is the plain oracle
+    one = [s for s in sym if not (s[0] == "accd" and s[2]) and not (s[0] == "ctl" and s[4] >> 6)]
+    enc = _enc_dev(one, 0)
+    assert orc.replay(np.array(enc, dtype=np.uint64).reshape(-1, 2), 0, 8, n_devices=ndev).triples() == \
+        orc.replay(np.array(enc, dtype=np.uint64).reshape(-1, 2), 0, 8).triples()

@@ -39,7 +39,7 @@ class ValueSim:
     does not reach this word's CV at all; it is reported as BO and changes
     nothing.  CV existence is tracked as a set of words here, not as a bit."""
 
-    def __init__(self, bo: bool = False, unified: bool = False):
+    def __init__(self, bo: bool = False, unified: bool = False, devices: int = 1):
         """unified=True: unified memory (reading Z23): OV and CV are the same
         storage (one dict), so transfers, allocation and release change nothing."""
         self.bo = bo
@@ -47,9 +47,14 @@ class ValueSim:
         self.alive: set[int] = set()      # words whose CV exists
         self.ov: dict[int, int] = {}
         self.cv: dict[int, int] = self.ov if unified else {}
+        # several accelerators (reading Z24): one CV and one present table per
+        # device; `self.cv` / `self.present` always name the current record's device
+        self.devices = devices
+        self.cvs = [self.cv] + [{} for _ in range(devices - 1)]
+        self.presents = [[] for _ in range(devices)]
         self.latest: dict[int, int] = {}
         self.next_id = 1
-        self.present: list[list[int]] = []  # [lo, hi, refcount] byte intervals
+        self.present: list[list[int]] = self.presents[0]  # [lo, hi, refcount] byte intervals
         self.issues: set[tuple[int, int, int]] = set()
 
     # -- per-word primitive operations ---------------------------------------
@@ -107,6 +112,10 @@ class ValueSim:
         return hit
 
     def record(self, op, addr, length, arg, idx):
+        if self.devices > 1:              # Z24: the device of the record
+            d = arg if op in (RT, WT) else (arg >> 6 if op in (MAP_ENTER, MAP_EXIT, UPDATE) else 0)
+            arg = arg & 0x3F if op in (MAP_ENTER, MAP_EXIT, UPDATE) else arg
+            self.cv, self.present = self.cvs[d], self.presents[d]
         always = bool(arg & ALWAYS)           # OpenMP 5.1 `always` map-type modifier (reading Z21)
         present = bool(arg & PRESENT)         # OpenMP 5.1 `present`: not mapped -> error
         arg &= ~(ALWAYS | PRESENT)
@@ -166,10 +175,13 @@ class ValueSim:
         """The 4 quantities of Table II as observed on values (for final-state pins)."""
         lat = self.latest.get(w)
         ov = self.ov.get(w, BOT)
-        cv = self.cv.get(w, BOT)
+        cv = self.cvs[0].get(w, BOT)
         ovv = lat is not None and ov == lat
         cvv = lat is not None and cv == lat
         bits = int(ovv) | (int(cvv) << 1) | (int(ov != BOT) << 2) | (int(cv != BOT) << 3)
+        for d in range(1, self.devices):  # Z24: device d's CV valid / initialised at bits 2d+2, 2d+3
+            c = self.cvs[d].get(w, BOT)
+            bits |= (int(lat is not None and c == lat) << (2 * d + 2)) | (int(c != BOT) << (2 * d + 3))
         return bits | (int(w in self.alive) << 4 if self.bo else 0)
 
 
