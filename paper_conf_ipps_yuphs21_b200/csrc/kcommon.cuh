@@ -19,11 +19,6 @@ __device__ __forceinline__ uint4 ld_stream(const uint4* p) {
                : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
   return r;
 }
-__device__ __forceinline__ uint2 ld_stream2(const uint2* p) {
-  uint2 r;
-  asm volatile("ld.global.cs.v2.u32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
-  return r;
-}
 
 // ---- cp.async staging -------------------------------------------------------
 __device__ __forceinline__ void cp_async16(void* smem_dst, const void* gsrc) {
@@ -36,8 +31,6 @@ __device__ __forceinline__ void cp_async8(void* smem_dst, const void* gsrc) {
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait_group() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
 // ---- TMA bulk copies completing on an mbarrier ------------------------------
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -90,13 +83,6 @@ __device__ __forceinline__ Sel sel_compose(Sel g, Sel f) {  // g after f
     r |= v << (3 * j);
   }
   return r;
-}
-
-// ---- the two access writes of the VSM on a 4-bit state --------
-__device__ __forceinline__ uint32_t vsm_write(uint32_t kind, uint32_t s) {
-  // kind 1 = write_host: OV holds the latest value, CV does not, OV initialised
-  // kind 2 = write_target: CV holds the latest value, OV does not, CV initialised
-  return kind == 1 ? ((s & kCVi) | kOVv | kOVi) : ((s & kOVi) | kCVv | kCVi);
 }
 
 }  // namespace arb
