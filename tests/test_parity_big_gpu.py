@@ -80,13 +80,17 @@ def test_config5_scaled_shard(orc):
     ctx.close()
 
 
-def _sampled_full_size(orc, prog, lo, hi, n_sample=3000, seed=0):
-    """Run the bench configuration on the device, then compare sampled words."""
+def _sampled_full_size(orc, prog, lo, hi, n_sample=3000, seed=0, one_flush=False, flags=0):
+    """Run the bench configuration on the device, then compare sampled words.
+    one_flush: the whole batch in a single flush (near the 2^30-record maximum)."""
     import torch
     import bench
     recs, gidx, flushes, (lo2, hi2) = bench.rank_batches(prog, 0, 1, torch.device("cuda", 0))
     assert (lo2, hi2) == (lo, hi)
-    ctx, got = _gpu_run(prog, lo, hi, flushes=flushes, recs=recs, gidx=gidx)
+    if one_flush:
+        assert 2 ** 29 < recs.shape[0] <= 2 ** 30
+        flushes = [(0, recs.shape[0])]
+    ctx, got = _gpu_run(prog, lo, hi, flushes=flushes, recs=recs, gidx=gidx, flags=flags)
     rs = np.random.default_rng(seed)
     # half of the sample from the words the trace touches most densely (mapped sections)
     secs = np.array([(a, b) for a, b, _ in prog.sections if b > lo and a < hi], dtype=np.int64)
@@ -136,3 +140,37 @@ def test_config4_full_size_sampled(orc):
     prog = native.config4()
     lo, hi = prog.addr_base // 8, (prog.addr_base + prog.addr_bytes) // 8
     _sampled_full_size(orc, prog, lo, hi)
+
+
+@pytest.mark.slow
+def test_config5_one_flush_near_max_batch(orc):
+    """Rank 0's whole config-5 batch (1.0e9 records, record positions up to 2^30)
+    in one flush: the largest batch the ABI accepts, sampled against the oracle."""
+    from gen import native
+    from paper_conf_ipps_yuphs21_b200.shard import shard_range
+    prog = native.config5()
+    lo, hi = shard_range(native.C5_BASE_WORD, native.C5_WORDS, 0, 8)
+    exp = _sampled_full_size(orc, prog, lo, hi, one_flush=True, seed=3)
+    assert len(exp.triples()) > 0
+
+
+def test_batch_limit():
+    """More than 2^30 records in one batch is ARB_EINVAL; the context stays usable."""
+    import torch
+    from paper_conf_ipps_yuphs21_b200 import Context, ArbError, reports_to_triples
+    from gen.configs import config1
+    ctx = Context(0x1000_0000, 1 << 16)
+    big = torch.empty(((1 << 30) + 1, 2), dtype=torch.int64, device="cuda")
+    with pytest.raises(ArbError):
+        ctx.submit_events(big)
+    del big
+    torch.cuda.empty_cache()
+    rec, base, size = config1()
+    ctx.close()
+    ctx = Context(base, size)
+    from gpu_util import to_device
+    d = to_device(rec)
+    ctx.submit_events(d)
+    rc, n, _ = ctx.flush()
+    assert rc == 0 and n == 1024
+    ctx.close()
