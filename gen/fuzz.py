@@ -15,14 +15,20 @@ from .trace import MAP, OP, UPD, SYNC_ALL, TraceBuilder, encode_np
 
 def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: int = 60,
                    base: int = 0x10000, loop_max: int = 48, p_task: float = 0.15, p_always: float = 0.0,
-                   p_depend: float = 0.0):
+                   p_depend: float = 0.0, n_devices: int = 1):
     """p_always > 0: map clauses carry the `always` modifier with that probability;
     p_depend > 0: a new nowait block depends on an earlier task with that
-    probability (the RNG streams of p_always = p_depend = 0 programs are unchanged)."""
+    probability; n_devices > 1: target accesses and map / update clauses on a
+    random accelerator (the device in the access arg and in bits 6-7 of a
+    map / update arg) (the RNG streams of the defaults are unchanged)."""
     rs = np.random.default_rng(seed)
     tb = TraceBuilder()
     arrays = [base + i * array_words * 8 * 2 for i in range(n_arrays)]   # gap between arrays
-    present = {i: [] for i in range(n_arrays)}   # list of (lo, hi) byte sections entered
+    # list of (lo, hi) byte sections entered, per array (and device with n_devices > 1)
+    present = {(i, d): [] for i in range(n_arrays) for d in range(n_devices)}
+
+    def pdev():
+        return int(rs.integers(n_devices)) if n_devices > 1 else 0
     in_task = 0
     next_task = 1
     unjoined = []
@@ -50,7 +56,8 @@ def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: i
         addr = arrays[i] + start + stride * np.arange(cnt, dtype=np.uint64)
         addr = addr[addr + size <= arrays[i] + array_words * 8 + 8]
         if addr.size:
-            tb.add_array(encode_np(op, addr, size))
+            arg = pdev() if op in (OP.RT, OP.WT) else 0
+            tb.add_array(encode_np(op, addr, size, arg=arg))
 
     for _ in range(steps):
         r = rs.random()
@@ -60,34 +67,40 @@ def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: i
             i = int(rs.integers(n_arrays))
             lo, n = section(i)
             hi = lo + n
-            ok = all(hi <= a or lo >= b or (a <= lo and hi <= b) for a, b in present[i])
+            dv = pdev()
+            pr = present[(i, dv)]
+            ok = all(hi <= a or lo >= b or (a <= lo and hi <= b) for a, b in pr)
             if ok:
                 mt = int(rs.choice([MAP.TO, MAP.FROM, MAP.TOFROM, MAP.ALLOC]))
                 if p_always and rs.random() < p_always:
                     mt |= MAP.ALWAYS
-                if p_always and any(a <= lo and hi <= b for a, b in present[i]) and rs.random() < p_always:
+                if p_always and any(a <= lo and hi <= b for a, b in pr) and rs.random() < p_always:
                     mt |= MAP.PRESENT            # a mapped section: `present` holds
-                tb.enter(mt, lo, n)
-                present[i].append((lo, hi))
+                tb.enter(mt | (dv << 6), lo, n)
+                pr.append((lo, hi))
         elif r < 0.65:
             i = int(rs.integers(n_arrays))
-            if present[i]:
-                k = int(rs.integers(len(present[i])))
-                lo, hi = present[i][k]
+            dv = pdev()
+            pr = present[(i, dv)]
+            if pr:
+                k = int(rs.integers(len(pr)))
+                lo, hi = pr[k]
                 # exit only sections that contain no other present section
-                if all(not (lo <= a and b <= hi and (a, b) != (lo, hi)) for a, b in present[i]):
+                if all(not (lo <= a and b <= hi and (a, b) != (lo, hi)) for a, b in pr):
                     mt = int(rs.choice([MAP.TO, MAP.FROM, MAP.TOFROM, MAP.ALLOC, MAP.RELEASE, MAP.DELETE]))
                     if p_always and rs.random() < p_always:
                         mt |= MAP.ALWAYS
-                    tb.exit(mt, lo, hi - lo)
-                    present[i].pop(k)
+                    tb.exit(mt | (dv << 6), lo, hi - lo)
+                    pr.pop(k)
         elif r < 0.72:
             i = int(rs.integers(n_arrays))
-            if present[i]:
-                lo, hi = present[i][int(rs.integers(len(present[i])))]
-                tb.update(int(rs.choice([UPD.TO, UPD.FROM])), lo, hi - lo)
+            dv = pdev()
+            pr = present[(i, dv)]
+            if pr:
+                lo, hi = pr[int(rs.integers(len(pr)))]
+                tb.update(int(rs.choice([UPD.TO, UPD.FROM])) | (dv << 6), lo, hi - lo)
             elif rs.random() < 0.3:
-                tb.update(int(rs.choice([UPD.TO, UPD.FROM])), arrays[i], array_words * 8)
+                tb.update(int(rs.choice([UPD.TO, UPD.FROM])) | (dv << 6), arrays[i], array_words * 8)
         elif r < 0.72 + p_task and not in_task:
             k = next_task
             next_task = next_task + 1 if next_task < 60000 else 1

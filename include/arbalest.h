@@ -94,6 +94,12 @@ enum arb_status {
                                    replay every small bucket with >= 64 events as 3 time
                                    slices (the mechanisms normally used for range-heavy
                                    and hot buckets only)                                  */
+/* several accelerators (Z24): n = 1 + ARB_F_DEVICES(flags) devices,
+ * n <= 3; the device of RT/WT is the record's arg, that of MAP_ENTER / MAP_EXIT /
+ * UPDATE bits 6-7 of its arg; batches of at most 2^29 records; excludes ARB_F_BO
+ * and ARB_F_UNIFIED */
+#define ARB_F_DEVICES_SHIFT 8
+#define ARB_F_DEVICES(n)  ((uint32_t)((n) - 1) << ARB_F_DEVICES_SHIFT)
 #define ARB_F_UNIFIED     0x10u /* unified memory (Z23): OV and CV are one
                                    storage — map clauses and target update move no data
                                    (reference counts and ARB_EMAP only), a write of either side

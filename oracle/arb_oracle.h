@@ -108,7 +108,7 @@ typedef struct {
    * (n <= 3), each with its valid and initialised bit — and one mapping table
    * per device.  The device is arg of RT/WT records and bits 6-7 of the arg of
    * MAP_ENTER / MAP_EXIT / UPDATE.  Single-device traces are unchanged.
-   * Excludes detect_bo and unified.  (Oracle only: the CUDA path is single-device.) */
+   * Excludes detect_bo and unified. */
   int             n_devices;
 } orc_config;
 

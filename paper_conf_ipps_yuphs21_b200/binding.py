@@ -21,6 +21,11 @@ ARB_F_SMALL_PARTS = 0x4
 ARB_F_BO = 0x8          # buffer-overflow extension (Z20)
 ARB_BO = 4
 ARB_F_UNIFIED = 0x10    # unified memory (Z23)
+
+
+def ARB_F_DEVICES(n):
+    """n accelerators (Z24), n <= 3."""
+    return (n - 1) << 8
 STATUS = {0: "ARB_OK", 1: "ARB_TRUNCATED", -1: "ARB_EINVAL", -2: "ARB_ENOMEM", -3: "ARB_ECUDA",
           -4: "ARB_EMAP", -5: "ARB_ETRACE", -6: "ARB_ESTATE", -7: "ARB_EOPEN"}
 EXPORTS = ("arb_init", "arb_submit_events", "arb_flush", "arb_get_reports", "arb_get_shadow",

@@ -189,7 +189,8 @@ extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
   if (!cfg || (cfg->addr_base & 7) || (cfg->addr_bytes & 7) || cfg->addr_bytes == 0 ||
       cfg->addr_base + cfg->addr_bytes > (1ull << 48) || cfg->world < 1 || cfg->rank < 0 ||
       cfg->rank >= cfg->world || (cfg->world > 1 && !cfg->nccl_unique_id) ||
-      ((cfg->flags & ARB_F_BO) && (cfg->flags & ARB_F_UNIFIED)))
+      ((cfg->flags & ARB_F_BO) && (cfg->flags & ARB_F_UNIFIED)) || ((cfg->flags >> ARB_F_DEVICES_SHIFT) & 3u) > 2u ||
+      (((cfg->flags >> ARB_F_DEVICES_SHIFT) & 3u) && (cfg->flags & (ARB_F_BO | ARB_F_UNIFIED))))
     return ARB_EINVAL;
   arb_ctx ctx = new (std::nothrow) arb_ctx_s();
   if (!ctx) return ARB_ENOMEM;
@@ -287,6 +288,8 @@ extern "C" int arb_submit_events(arb_ctx ctx, const arb_event* ev, uint64_t n, c
   if (n == 0) return ARB_OK;
   if (!ev) return fail(ctx, ARB_EINVAL, "null event pointer");
   if (ctx->pending + n > kMaxBatchRecords) return fail(ctx, ARB_EINVAL, "batch exceeds 2^30 records");
+  if (((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u) && ctx->pending + n > (kMaxBatchRecords >> 1))
+    return fail(ctx, ARB_EINVAL, "several accelerators: a batch holds at most 2^29 records");
   if ((global_index != nullptr && ctx->any_nogidx) || (global_index == nullptr && ctx->any_gidx))
     return fail(ctx, ARB_EINVAL, "global_index must be given for every submit of a batch or for none");
   cudaSetDevice(ctx->cfg.device);
@@ -373,6 +376,7 @@ static void build_items(arb_ctx ctx, const FlushPlan& plan, const std::vector<do
     const double ev = bucket_events[b];
     if (parts[b] != 1 || span > kHotSpan) continue;
     if (ctx->cfg.flags & ARB_F_BO) continue;      // slice functions cannot express the BO condition (Z20)
+    if ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u) continue;   // nor 8-bit states (Z24)
     const bool hot = force_hot ? ev >= 64.0 : (ev > 1.25 * share && ev > kSliceEvents);
     if (!hot) continue;
     const double want = force_hot ? 3.0 : std::ceil(ev / kSliceEvents);
@@ -521,6 +525,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     pp.coarse_bits = ctx->coarse_bits; pp.bin_map = balanced ? ctx->d_hist.p : ctx->d_bin_map.p;
     pp.bucket_bits = ctx->bucket_bits; pp.n_buckets = balanced ? (uint32_t)kMaxBuckets : ctx->n_buckets;
     pp.n_chunks = n_chunks;
+    pp.n_dev = 1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u);
     pp.part_ev = ctx->part_ev.p; pp.seg_out = ctx->seg_a.p; pp.seg_cap = ctx->seg_cap;
     pp.ctl = ctx->ctl.p; pp.ctl_cap = ctx->ctl_cap;
     pp.st = ctx->dstats.p;
@@ -582,7 +587,8 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   MapTable map = ctx->map;
   FlushPlan plan;
   resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_start, map, plan,
-                  (ctx->cfg.flags & ARB_F_BO) != 0, &ctx->carried, (ctx->cfg.flags & ARB_F_UNIFIED) != 0);
+                  (ctx->cfg.flags & ARB_F_BO) != 0, &ctx->carried, (ctx->cfg.flags & ARB_F_UNIFIED) != 0,
+                  1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u));
   if (plan.rc != 0) {
     CK(cudaStreamSynchronize(s), "sync");
     reset_batch(ctx);
@@ -624,7 +630,8 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   rp.bucket_start = ctx->d_bucket_start.p;
   rp.items = ctx->d_items.p; rp.n_items = (uint32_t)ctx->items.size();
   rp.shadow = ctx->shadow; rp.bo = (ctx->cfg.flags & ARB_F_BO) ? 1u : 0u;
-  rp.um = (ctx->cfg.flags & ARB_F_UNIFIED) ? 1u : 0u; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
+  rp.um = (ctx->cfg.flags & ARB_F_UNIFIED) ? 1u : 0u;
+  rp.md = ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u) ? 1u : 0u; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
   rp.cand = ctx->cand.p; rp.cand_cap = ctx->cand_cap; rp.st = ctx->dstats.p;
   rp.hot_off = ctx->d_hot_off.p; rp.hot_F = ctx->hot_F.p; rp.hot_P = ctx->hot_P.p;
   int n_ctas = std::max(1, std::min<int>((int)ctx->items.size(), ctx->n_sms * kReplayCtasPerSm));

@@ -41,6 +41,20 @@ constexpr Sel kSelUPH   = sel_make(1, 1, 3, 3);   // OV takes CV's (update_host)
 constexpr Sel kSelALLOC = sel_make(0, 4, 2, 4);   // fresh CV: not valid, not initialised
 constexpr Sel kSelREL   = sel_make(0, 4, 2, 4);   // released CV: same bits as allocate
 
+// ---- several accelerators (Z24) ---------------------------
+// 8-bit state: bit0 OVv, bit1 CV0v, bit2 OVi, bit3 CV0i, bits 4/5 CV1 valid /
+// initialised, bits 6/7 CV2.  Range ops use an 8-output selector ("Sel8"):
+// 4 bits per output bit j = its source (0-7 an input bit, 8 constant 0, 9 constant 1).
+__host__ __device__ constexpr uint32_t md_cvv(uint32_t d) { return d == 0 ? 1u : 4u + 2u * (d - 1u); }
+__host__ __device__ constexpr uint32_t md_cvi(uint32_t d) { return d == 0 ? 3u : 5u + 2u * (d - 1u); }
+constexpr uint32_t kSel8Id = 0x76543210u;
+__host__ __device__ constexpr uint32_t sel8_set(uint32_t s, uint32_t out_bit, uint32_t src) {
+  return (s & ~(15u << (4 * out_bit))) | (src << (4 * out_bit));
+}
+__host__ __device__ constexpr uint32_t sel8_upt(uint32_t d) { return sel8_set(sel8_set(kSel8Id, md_cvv(d), 0), md_cvi(d), 2); }
+__host__ __device__ constexpr uint32_t sel8_uph(uint32_t d) { return sel8_set(sel8_set(kSel8Id, 0, md_cvv(d)), 2, md_cvi(d)); }
+__host__ __device__ constexpr uint32_t sel8_clear(uint32_t d) { return sel8_set(sel8_set(kSel8Id, md_cvv(d), 8), md_cvi(d), 8); }
+
 // ---- compact event (partition output, 8 B) ---------------------------------
 // x: [0,30) word offset inside the address bucket | [30,32) access op (RH/WH/RT/WT)
 // y: record position inside the batch (< 2^30)
@@ -126,6 +140,7 @@ struct PartParams {
                                           // bit 21 << 31} per touched bucket of a chunk
   CtlRec* ctl; uint64_t ctl_cap;
   DevStats* st;
+  uint32_t n_dev;                         // accelerators (Z24): > 1 puts the device of RT/WT in pos bits 30-31
 };
 
 struct ReplayParams {
@@ -145,6 +160,7 @@ struct ReplayParams {
   uint8_t* shadow;                        // n_words bytes
   uint32_t bo;                            // ARB_F_BO: target accesses to words without kCVp are BO
   uint32_t um;                            // ARB_F_UNIFIED: OV and CV are one storage (Z23)
+  uint32_t md;                            // several accelerators (Z24): 8-bit states, device in pos bits 30-31
   const uint32_t* ops_start;              // [n_buckets + 1]
   const BucketOp* ops;
   uint4* cand; uint64_t cand_cap;         // report candidates {word lo, word hi, pos, kind}

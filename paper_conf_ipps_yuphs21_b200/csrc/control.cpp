@@ -42,7 +42,8 @@ struct Emitter {
 
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
-                     FlushPlan& out, bool bo, const std::vector<CarriedInst>* carried_in, bool unified) {
+                     FlushPlan& out, bool bo, const std::vector<CarriedInst>* carried_in, bool unified,
+                     uint32_t n_dev) {
   const uint32_t n_buckets = (uint32_t)bucket_start.size() - 1;
   out = FlushPlan();
   Emitter em{base_word, n_words, &out, unified};
@@ -67,8 +68,22 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   auto fail = [&](int rc, uint64_t pos, const char* why) {
     out.rc = rc; out.err_pos = pos; out.err = why;
   };
+  const bool md = n_dev > 1;
+  // selectors of the data ops on device d (Z24) — the 4-bit forms for one device
+  auto s_upt = [&](uint32_t d) { return md ? sel8_upt(d) : kSelUPT; };
+  auto s_uph = [&](uint32_t d) { return md ? sel8_uph(d) : kSelUPH; };
+  auto s_alloc = [&](uint32_t d) { return md ? sel8_clear(d) : (kSelALLOC | (bo ? kPopSet : 0u)); };
+  auto s_rel = [&](uint32_t d) { return md ? sel8_clear(d) : (kSelREL | (bo ? kPopClr : 0u)); };
+  constexpr uint64_t kAddrMask = (1ull << 56) - 1;
   for (const CtlRec& c : ctl) {
     uint32_t op = (uint32_t)(c.w0 >> 48) & 0xFFu, arg = (uint32_t)(c.w0 >> 56);
+    uint32_t dev = 0;                               // Z24: device of a MAP / UPDATE record
+    if (md && (op == OP_MAP_ENTER || op == OP_MAP_EXIT || op == OP_UPDATE)) {
+      dev = arg >> 6;
+      arg &= 0x3Fu;
+      if (dev >= n_dev) return fail(ARB_ETRACE, c.pos, "device id of a map / update record out of range");
+    }
+    const uint64_t dkey = (uint64_t)dev << 56;     // the device's entries: keys offset by dev << 56
     uint64_t addr = c.w0 & kMask48, len = c.w1 & kMask48;
     uint32_t tid = (uint32_t)(c.w1 >> 48);
     uint32_t pos = (uint32_t)c.pos;
@@ -103,17 +118,17 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
         if (arg > MT_ALLOC || len == 0 || addr + len > (1ull << 48))
           return fail(ARB_ETRACE, c.pos, "bad MAP_ENTER record");
         MapTable::iterator it;
-        int f = map_find(map, addr, addr + len, it);
+        int f = map_find(map, dkey | addr, dkey | (addr + len), it);
         if (f < 0) return fail(ARB_EMAP, c.pos, "map clause partially overlaps a present entry");
         if (f == 0 && present) return fail(ARB_EMAP, c.pos, "map(present) of a section that is not mapped");
         if (f == 1) {                               // exist(CV): ref_count += 1, no transfer ...
           it->second.rc += 1;
-          if (always && (arg == MT_TO || arg == MT_TOFROM)) em.emit(pos, kSelUPT, addr, addr + len, open);
+          if (always && (arg == MT_TO || arg == MT_TOFROM)) em.emit(pos, s_upt(dev), addr, addr + len, open);
           break;                                    // ... unless `always`
         }
-        map.emplace(addr, MapEntry{addr + len, 1});  // new CV, ref_count = 1
-        em.emit(pos, kSelALLOC | (bo ? kPopSet : 0u), addr, addr + len, open);
-        if (arg == MT_TO || arg == MT_TOFROM) em.emit(pos, kSelUPT, addr, addr + len, open);
+        map.emplace(dkey | addr, MapEntry{dkey | (addr + len), 1});  // new CV, ref_count = 1
+        em.emit(pos, s_alloc(dev), addr, addr + len, open);
+        if (arg == MT_TO || arg == MT_TOFROM) em.emit(pos, s_upt(dev), addr, addr + len, open);
         break;
       }
       case OP_MAP_EXIT: {                           // Table I, exit (reading Z5)
@@ -122,15 +137,15 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
         if (arg > MT_DELETE || len == 0 || addr + len > (1ull << 48))
           return fail(ARB_ETRACE, c.pos, "bad MAP_EXIT record");
         MapTable::iterator it;
-        int f = map_find(map, addr, addr + len, it);
+        int f = map_find(map, dkey | addr, dkey | (addr + len), it);
         if (f < 0) return fail(ARB_EMAP, c.pos, "map clause partially overlaps a present entry");
         if (f == 0) break;                          // not present: no-op (Z7)
         if (arg == MT_DELETE) it->second.rc = 0; else it->second.rc -= 1;
         if (it->second.rc != 0 && always && (arg == MT_FROM || arg == MT_TOFROM))
-          em.emit(pos, kSelUPH, addr, addr + len, open);   // `always`: copy back at rc > 0
+          em.emit(pos, s_uph(dev), addr, addr + len, open);   // `always`: copy back at rc > 0
         if (it->second.rc == 0) {
-          if (arg == MT_FROM || arg == MT_TOFROM) em.emit(pos, kSelUPH, addr, addr + len, open);
-          em.emit(pos, kSelREL | (bo ? kPopClr : 0u), it->first, it->second.hi, open);
+          if (arg == MT_FROM || arg == MT_TOFROM) em.emit(pos, s_uph(dev), addr, addr + len, open);
+          em.emit(pos, s_rel(dev), it->first & kAddrMask, it->second.hi & kAddrMask, open);
           map.erase(it);
         }
         break;
@@ -139,10 +154,10 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
         if (arg > 1 || len == 0 || addr + len > (1ull << 48))
           return fail(ARB_ETRACE, c.pos, "bad UPDATE record");
         MapTable::iterator it;
-        int f = map_find(map, addr, addr + len, it);
+        int f = map_find(map, dkey | addr, dkey | (addr + len), it);
         if (f < 0) return fail(ARB_EMAP, c.pos, "target update partially overlaps a present entry");
         if (f == 0) break;                          // not present: no-op (Z7)
-        em.emit(pos, arg == 0 ? kSelUPT : kSelUPH, addr, addr + len, open);
+        em.emit(pos, arg == 0 ? s_upt(dev) : s_uph(dev), addr, addr + len, open);
         break;
       }
       case OP_TASK_DEPEND: {                        // Z22: the open task runs after the last

@@ -63,7 +63,10 @@ struct FlushPlan {
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
                      FlushPlan& out, bool bo = false, const std::vector<CarriedInst>* carried_in = nullptr,
-                     bool unified = false);
+                     bool unified = false, uint32_t n_dev = 1);
+// n_dev > 1 (Z24): device bits 6-7 of MAP / UPDATE args select the device; its
+// entries live in the same table under keys offset by device << 56, and range
+// ops are 8-output selectors (Sel8).
 // unified (ARB_F_UNIFIED, Z23): map clauses and target update keep the reference
 // counts (and their errors) but emit no range ops: nothing moves between OV and CV.
 

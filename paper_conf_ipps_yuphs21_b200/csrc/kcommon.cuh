@@ -74,6 +74,26 @@ __device__ __forceinline__ uint32_t sel_apply5(Sel s, uint32_t x) {
   const uint32_t pop = (s >> 12) & 3u;
   return sel_apply4(s, x) | (pop == 0 ? (x & 0x10101010u) : (pop == 3 ? 0x10101010u : 0u));
 }
+// several accelerators (Z24): 8-output selectors on 8-bit states
+__device__ __forceinline__ uint32_t sel8_apply4(uint32_t s, uint32_t x) {
+  uint32_t out = 0;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    const uint32_t src = (s >> (4 * j)) & 15u;
+    const uint32_t v = src < 8 ? (x >> src) & 0x01010101u : (src == 9 ? 0x01010101u : 0u);
+    out |= v << j;
+  }
+  return out;
+}
+__device__ __forceinline__ uint32_t sel8_compose(uint32_t g, uint32_t f) {  // g after f
+  uint32_t r = 0;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    const uint32_t gj = (g >> (4 * j)) & 15u;
+    r |= (gj < 8 ? (f >> (4 * gj)) & 15u : gj) << (4 * j);
+  }
+  return r;
+}
 __device__ __forceinline__ Sel sel_compose(Sel g, Sel f) {  // g after f
   Sel r = (g & (3u << 12)) ? (g & (3u << 12)) : (f & (3u << 12));
 #pragma unroll

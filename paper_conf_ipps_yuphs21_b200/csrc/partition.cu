@@ -43,6 +43,7 @@ constexpr int kB1Shift = 2 + kBucketBits;
 // round interleave.  flags: bit0 control record, bit1 malformed.  valid =
 // record exists; two = an unaligned access that also touches the next word
 // (Z4, rare: handled by decode1).  b1 = b0 until decode1 says otherwise.
+template <bool MD>
 __device__ __forceinline__ Dec decode0(uint4 q, bool valid, const PartParams& p, uint32_t& ign, uint32_t& flags,
                                        bool& two) {
   const uint32_t op = (q.y >> 16) & 0xFFu;
@@ -52,7 +53,12 @@ __device__ __forceinline__ Dec decode0(uint4 q, bool valid, const PartParams& p,
   const bool ctl = op < 16 && ((0xF700u >> op) & 1u);            // ops 8, 9, 10, 12, 13, 14, 15
   const bool acc = op < 4;
   flags = valid ? (acc ? (bad_acc ? 2u : 0u) : (ctl ? 1u : 2u)) : 0u;
-  const bool ok = valid && acc && !bad_acc;
+  bool ok = valid && acc && !bad_acc;
+  uint32_t dev = 0;
+  if (MD) {                                  // several accelerators (Z24): the device of RT / WT is the arg
+    dev = (op & 2u) ? q.y >> 24 : 0u;
+    if (acc && dev >= p.n_dev) { flags = valid ? 2u : 0u; ok = false; }
+  }
   const uint64_t rel = ((((uint64_t)hi) << 29) | (q.x >> 3)) - p.base_word;   // wraps below the range
   const bool in0 = ok && rel < p.n_words;
   two = ok && (q.x & 7u) + len > 8u;
@@ -65,9 +71,11 @@ __device__ __forceinline__ Dec decode0(uint4 q, bool valid, const PartParams& p,
   d.k0 = (op << 30) | ((m0 >> kBucketBits) << cb) | ((uint32_t)rel & ((1u << cb) - 1u));
   d.k1 = 0;
   d.info = (uint32_t)in0 | (b0 << 2) | (b0 << kB1Shift);
+  if (MD) d.info |= (dev & 3u) << 24;
   return d;
 }
 // Second word of an unaligned access (the record is re-read from the stage).
+template <bool MD>
 __device__ __forceinline__ void decode1(Dec& d, uint4 q, const PartParams& p, uint32_t& ign) {
   const uint32_t op = (q.y >> 16) & 0xFFu;
   const uint64_t r1 = ((((uint64_t)(q.y & 0xFFFFu)) << 29) | (q.x >> 3)) - p.base_word + 1;
@@ -76,8 +84,9 @@ __device__ __forceinline__ void decode1(Dec& d, uint4 q, const PartParams& p, ui
   const uint32_t m = __ldg(p.bin_map + (uint32_t)(r1 >> cb));
   const uint32_t b = m & kBucketMask;
   const uint32_t k = (op << 30) | ((m >> kBucketBits) << cb) | ((uint32_t)r1 & ((1u << cb) - 1u));
-  if ((d.info & 3u) == 0) { d.k0 = k; d.info = 1u | (b << 2) | (b << kB1Shift); }
-  else { d.k1 = k; d.info = 2u | (d.info & (kBucketMask << 2)) | (b << kB1Shift); }
+  const uint32_t dv = MD ? d.info & (3u << 24) : 0u;   // the device bits (Z24)
+  if ((d.info & 3u) == 0) { d.k0 = k; d.info = 1u | (b << 2) | (b << kB1Shift) | dv; }
+  else { d.k1 = k; d.info = 2u | (d.info & (kBucketMask << 2)) | (b << kB1Shift) | dv; }
 }
 
 // append the buckets of lanes with `is_new` to the warp's touched list
@@ -126,16 +135,22 @@ __device__ __forceinline__ void rank_round(uint32_t info, uint16_t* row, uint16_
 // |d| < 2^30 as a bucket spans <= 2^30 words), the warp reduces min and max, and
 // two bin-map lookups decide.  A word's offset in the bucket is then
 // off(lowest) + d - dmin.  Returns false (nothing written) when the test fails.
+template <bool MD>
 __device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p, uint32_t chunk, uint2* out,
                                            uint2* segbuf, uint32_t& nbuf, uint32_t lane) {
   const uint4 q0 = st[0];
   const uint64_t w0 = ((uint64_t)((q0.y & 0xFFFFu) >> 3) << 32) | __funnelshift_r(q0.x, q0.y, 3);
-  uint32_t d[RPL], opk[RPL], bad = 0;
+  uint32_t d[RPL], opk[RPL], bad = 0, devs = 0;
   int32_t dmin = 0, dmax = 0;
 #pragma unroll
   for (int k = 0; k < RPL; ++k) {
     const uint4 q = st[k * 32 + lane];
     bad |= (q.y & 0x00FC0000u) | (q.w & 0xFFFFu) | ((q.z - 1u) & ~7u) | (((q.x & 7u) + q.z - 1u) & ~7u);
+    if (MD && (q.y & (1u << 17))) {                // RT / WT on device arg (Z24)
+      const uint32_t dv = q.y >> 24;
+      bad |= dv >= p.n_dev;
+      devs |= (dv & 3u) << (2 * k);
+    }
     const uint64_t word = ((uint64_t)((q.y & 0xFFFFu) >> 3) << 32) | __funnelshift_r(q.x, q.y, 3);
     const uint64_t diff = word - w0;
     bad |= (uint32_t)((diff + (1ull << 30)) >> 31);      // d outside [-2^30, 2^30)
@@ -157,7 +172,9 @@ __device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p,
   const uint32_t c = (((mlo >> kBucketBits) << cb) | ((uint32_t)rlo & ((1u << cb) - 1u))) - (uint32_t)dmin;
   const uint32_t rec0 = chunk * (uint32_t)WREC;
 #pragma unroll
-  for (int k = 0; k < RPL; ++k) out[k * 32 + lane] = make_uint2(opk[k] | (d[k] + c), rec0 + k * 32 + lane);
+  for (int k = 0; k < RPL; ++k)
+    out[k * 32 + lane] = make_uint2(opk[k] | (d[k] + c),
+                                    (rec0 + k * 32 + lane) | (MD ? ((devs >> (2 * k)) & 3u) << 30 : 0u));
   if (lane == 0)
     segbuf[nbuf] = make_uint2((bref << kSegChunkBits) | (chunk & ((1u << kSegChunkBits) - 1u)),
                               (uint32_t)WREC << 16 | ((chunk >> kSegChunkBits) << 31));
@@ -165,6 +182,9 @@ __device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p,
   return true;
 }
 
+// MD: several accelerators (Z24) — the device of RT / WT goes to bits 30-31 of the
+// event position; a separate instance so that the single-device kernel is unchanged
+template <bool MD>
 __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   extern __shared__ __align__(16) uint8_t smem[];
   const uint32_t NB = p.n_buckets;
@@ -220,7 +240,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     // keep record order, so event j is record j: one coalesced store per record and
     // one segment entry for the chunk.  Anything else takes the general path below.
     if (nbuf == kSegBuf) flush_segs();
-    if (nvalid == WREC && fast_chunk(st, p, (uint32_t)chunk, p.part_ev + chunk * kChunkCap,
+    if (nvalid == WREC && fast_chunk<MD>(st, p, (uint32_t)chunk, p.part_ev + chunk * kChunkCap,
                                      segbuf, nbuf, lane)) {
       n_acc += RPL;
       cur = cur + 1 == NST ? 0 : cur + 1;
@@ -240,7 +260,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
         const uint32_t j = g * 128 + k * 32 + lane;
         uint32_t flags;
         bool two;
-        dec[g * 4 + k] = decode0(st[j], j < nvalid, p, n_ign, flags, two);
+        dec[g * 4 + k] = decode0<MD>(st[j], j < nvalid, p, n_ign, flags, two);
         any_flag |= flags << (2 * k);
         twos |= (uint32_t)two << k;
       }
@@ -248,7 +268,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
         any2 = true;
 #pragma unroll
         for (int k = 0; k < 4; ++k)
-          if ((twos >> k) & 1u) decode1(dec[g * 4 + k], st[g * 128 + k * 32 + lane], p, n_ign);
+          if ((twos >> k) & 1u) decode1<MD>(dec[g * 4 + k], st[g * 128 + k * 32 + lane], p, n_ign);
       }
 #pragma unroll
       for (int k = 0; k < 4; ++k) e_lane += dec[g * 4 + k].info & 3u;
@@ -305,7 +325,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
         const uint32_t info = dec[g * 4 + k].info;
-        same &= (info & 3u) == 0 || (info & ~3u) == iref;
+        same &= (info & 3u) == 0 || (info & (MD ? 0xFFFFFCu : ~3u)) == iref;
       }
       if (__all_sync(FULL, same)) {
         const uint32_t base = row[bref];
@@ -364,14 +384,14 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
 #pragma unroll
     for (int r = 0; r < RPL; ++r) {
       const uint32_t info = dec[r].info;
-      const uint32_t pos = pos0 + (r >> 2) * 128 + (r & 3) * 32;
+      const uint32_t pos = (pos0 + (r >> 2) * 128 + (r & 3) * 32) | (MD ? (info >> 24) << 30 : 0u);   // | device
       if (info & 3u) out[row[(info >> 2) & kBucketMask] + (rk[r] & 0xFFFFu)] = make_uint2(dec[r].k0, pos);
     }
     if (any2) {
 #pragma unroll
       for (int r = 0; r < RPL; ++r) {
         const uint32_t info = dec[r].info;
-        const uint32_t pos = pos0 + (r >> 2) * 128 + (r & 3) * 32;
+        const uint32_t pos = (pos0 + (r >> 2) * 128 + (r & 3) * 32) | (MD ? (info >> 24) << 30 : 0u);
         if ((info & 3u) == 2u) out[row[(info >> kB1Shift) & kBucketMask] + (rk[r] >> 16)] = make_uint2(dec[r].k1, pos);
       }
     }
@@ -397,14 +417,15 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
 cudaError_t launch_partition(const PartParams& p, cudaStream_t s) {
   if (p.n_chunks == 0) return cudaSuccess;
   const size_t smem = PW * warp_smem_bytes(p.n_buckets);
-  cudaError_t e = cudaFuncSetAttribute(k_partition, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  auto kern = p.n_dev > 1 ? k_partition<true> : k_partition<false>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const uint64_t ctas = (p.n_chunks + PW - 1) / PW;
   const uint32_t grid = (uint32_t)std::min<uint64_t>(ctas, (uint64_t)sms);
-  k_partition<<<grid, PT, smem, s>>>(p);
+  kern<<<grid, PT, smem, s>>>(p);
   return cudaGetLastError();
 }
 

@@ -89,9 +89,11 @@ __device__ __forceinline__ void block_minmax(uint32_t& lo, uint32_t& hi, uint32_
 
 // ---- range ops ----------------------------------------------------------------
 // Apply transition `sel` to the state bytes base[lo, hi) (BO: 5-bit states, ARB_F_BO).
-template <bool BO>
-__device__ __forceinline__ uint32_t apply_sel(Sel s, uint32_t x) { return BO ? sel_apply5(s, x) : sel_apply4(s, x); }
-template <bool BO>
+template <bool BO, bool MD>
+__device__ __forceinline__ uint32_t apply_sel(Sel s, uint32_t x) {
+  return MD ? sel8_apply4(s, x) : BO ? sel_apply5(s, x) : sel_apply4(s, x);
+}
+template <bool BO, bool MD>
 __device__ void stream_apply(uint8_t* base, uint64_t lo, uint64_t hi, Sel sel) {
   if (lo >= hi) return;
   // 16-B aligned middle [a, b) of [lo, hi), by address
@@ -99,8 +101,8 @@ __device__ void stream_apply(uint8_t* base, uint64_t lo, uint64_t hi, Sel sel) {
   const uintptr_t pa = (p0 + 15) & ~(uintptr_t)15, pb = p1 & ~(uintptr_t)15;
   uint64_t a = hi, b = hi;                       // no aligned middle: all bytes in the head loop
   if (pa < pb) { a = lo + (pa - p0); b = hi - (p1 - pb); }
-  for (uint64_t j = lo + threadIdx.x; j < a; j += RT) __stcg(base + j, (uint8_t)apply_sel<BO>(sel, __ldcg(base + j)));
-  for (uint64_t j = b + threadIdx.x; j < hi; j += RT) __stcg(base + j, (uint8_t)apply_sel<BO>(sel, __ldcg(base + j)));
+  for (uint64_t j = lo + threadIdx.x; j < a; j += RT) __stcg(base + j, (uint8_t)apply_sel<BO, MD>(sel, __ldcg(base + j)));
+  for (uint64_t j = b + threadIdx.x; j < hi; j += RT) __stcg(base + j, (uint8_t)apply_sel<BO, MD>(sel, __ldcg(base + j)));
   uint4* v = reinterpret_cast<uint4*>(base + a);
   const uint64_t nv = (b - a) >> 4;
   constexpr int U = 4;   // 4 x 16 B loads in flight per thread
@@ -111,15 +113,15 @@ __device__ void stream_apply(uint8_t* base, uint64_t lo, uint64_t hi, Sel sel) {
     for (int u = 0; u < U; ++u) x[u] = __ldcg(v + j + u * RT);
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      x[u].x = apply_sel<BO>(sel, x[u].x); x[u].y = apply_sel<BO>(sel, x[u].y);
-      x[u].z = apply_sel<BO>(sel, x[u].z); x[u].w = apply_sel<BO>(sel, x[u].w);
+      x[u].x = apply_sel<BO, MD>(sel, x[u].x); x[u].y = apply_sel<BO, MD>(sel, x[u].y);
+      x[u].z = apply_sel<BO, MD>(sel, x[u].z); x[u].w = apply_sel<BO, MD>(sel, x[u].w);
       __stcg(v + j + u * RT, x[u]);
     }
   }
   for (; j < nv; j += RT) {
     uint4 x = __ldcg(v + j);
-    x.x = apply_sel<BO>(sel, x.x); x.y = apply_sel<BO>(sel, x.y);
-    x.z = apply_sel<BO>(sel, x.z); x.w = apply_sel<BO>(sel, x.w);
+    x.x = apply_sel<BO, MD>(sel, x.x); x.y = apply_sel<BO, MD>(sel, x.y);
+    x.z = apply_sel<BO, MD>(sel, x.z); x.w = apply_sel<BO, MD>(sel, x.w);
     __stcg(v + j, x);
   }
 }
@@ -127,7 +129,7 @@ __device__ void stream_apply(uint8_t* base, uint64_t lo, uint64_t hi, Sel sel) {
 // Apply every pending range op of the bucket with position < limit; runs of
 // ops on the identical range with no event in between are composed first.
 // S.next_op caches the position of the first pending op.
-template <bool BO>
+template <bool BO, bool MD>
 __device__ void apply_ops_before(ReplaySmem& S, const ReplayParams& p, uint32_t limit) {
   while (S.next_op < limit) {
     const uint32_t k = S.op_cur;
@@ -137,7 +139,7 @@ __device__ void apply_ops_before(ReplaySmem& S, const ReplayParams& p, uint32_t 
     while (k2 < S.op_end) {
       const BucketOp o2 = p.ops[k2];
       if (o2.pos >= limit || o2.lo != o.lo || o2.hi != o.hi) break;
-      sel = sel_compose(o2.sel, sel);
+      sel = MD ? sel8_compose(o2.sel, sel) : sel_compose(o2.sel, sel);
       ++k2;
     }
     const uint64_t lo = max(o.lo, S.bucket_base + S.part_lo), hi = min(o.hi, S.bucket_base + S.part_hi);
@@ -148,7 +150,7 @@ __device__ void apply_ops_before(ReplaySmem& S, const ReplayParams& p, uint32_t 
         S.fsum[w] = (uint16_t)sel_compose(sel, S.fsum[w]);
       }
     } else if (hi > lo) {
-      stream_apply<BO>(S.shrel, lo - S.bucket_base, hi - S.bucket_base, sel);
+      stream_apply<BO, MD>(S.shrel, lo - S.bucket_base, hi - S.bucket_base, sel);
     }
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -212,6 +214,21 @@ __device__ __forceinline__ uint32_t classify_bits(uint32_t op, uint32_t before) 
   return (op & 1u) || (v & 1u) || op > 3 ? 0u : 1u + ((v >> 2) & 1u);
 }
 
+// ---- several accelerators (Z24): 8-bit states ---------------------------------------------
+constexpr uint32_t kMdPos = 0x3FFFFFFFu;        // event position without the device bits
+constexpr uint32_t kMdAllCvv = 0x52u;           // CV0v | CV1v | CV2v
+// the state after a write: code bit 0 = target, bits 1-2 = its device
+__device__ __forceinline__ uint32_t md_write(uint32_t code, uint32_t s) {
+  if (!(code & 1u)) return (s & ~kMdAllCvv) | kOVv | kOVi;
+  const uint32_t d = code >> 1;
+  return (s & ~(kMdAllCvv | kOVv)) | (1u << md_cvv(d)) | (1u << md_cvi(d));
+}
+__device__ __forceinline__ uint32_t md_classify(uint32_t op, uint32_t dev, uint32_t s) {
+  if (op == OP_RH) return (s & kOVv) ? 0u : ((s & kOVi) ? 2u : 1u);
+  if (op == OP_RT) return ((s >> md_cvv(dev)) & 1u) ? 0u : (((s >> md_cvi(dev)) & 1u) ? 2u : 1u);
+  return 0u;
+}
+
 // hash slot of a word (Fibonacci hashing: consecutive words land far apart, so
 // the linear probe chains of a run's words stay short)
 __device__ __forceinline__ uint32_t hslot(uint32_t w) { return (w * 2654435761u) >> 20; }
@@ -229,10 +246,13 @@ __device__ __forceinline__ uint32_t hslot(uint32_t w) { return (w * 2654435761u)
 // the shadow-load latency in front of the hashing for every replay.
 // UM (ARB_F_UNIFIED, Z23): OV and CV are one storage — a write of either side
 // makes the word's state 0xF (both valid, both initialised).
-template <bool PARTIAL, bool BO, bool UM>
+// MD (several accelerators, Z24): 8-bit states; the device of a target access is in
+// bits 30-31 of its position, and a hash slot holds pos << 3 | device << 1 | target.
+template <bool PARTIAL, bool BO, bool UM, bool MD>
 __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
   uint32_t slot[RI], word[RI], pos[RI], op[RI], s_pre[RI];
   uint32_t bom = 0;                // bit j: event j is a buffer overflow (ARB_F_BO, Z20)
+  uint32_t devs = 0;               // MD: 2 bits per event
   bool multi = false;
   const uint8_t* sh = S.shrel;
   uint2* hs = S.u.h.slot;
@@ -244,7 +264,8 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
     slot[j] = 0; word[j] = 0; pos[j] = 0; op[j] = 4; s_pre[j] = 0;
     if (i < m) {
       const uint2 e = ev[i];
-      word[j] = e.x & kWordMask; op[j] = e.x >> 30; pos[j] = e.y;
+      word[j] = e.x & kWordMask; op[j] = e.x >> 30; pos[j] = MD ? (e.y & kMdPos) : e.y;
+      if (MD) devs |= (e.y >> 30) << (2 * j);
       if (!PARTIAL || word[j] - plo < pw) s_pre[j] = __ldcg(sh + word[j]);
       else op[j] = 4;                                       // another work item's word
       // a target access (RT = 2, WT = 3) to a word without a CV: BO, no VSM effect
@@ -265,7 +286,7 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
         h = (h + 1) & (kHSlots - 1);
       }
       slot[j] = h;
-      hs[h].y = (pos[j] << 2) | op[j];
+      hs[h].y = MD ? ((pos[j] << 3) | (((devs >> (2 * j)) & 3u) << 1) | (op[j] >> 1)) : ((pos[j] << 2) | op[j]);
     }
   }
   any_w = __syncthreads_or(any_w);
@@ -279,7 +300,7 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
   uint32_t fk[RI];
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
-    const uint32_t s0 = s_pre[j] & 15u;
+    const uint32_t s0 = s_pre[j] & (MD ? 255u : 15u);
     uint32_t before = s0;
     if (op[j] == OP_RH || op[j] == OP_RT) {
       if (any_w) {
@@ -287,7 +308,8 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
         for (;;) {                                          // probe for the word's write
           const uint2 k = hs[h];
           if (k.x == word[j]) {
-            if ((k.y >> 2) < pos[j]) before = UM ? 15u : vsm_write_op(k.y & 3u, s0);
+            if (MD) { if ((k.y >> 3) < pos[j]) before = md_write(k.y & 7u, s0); }
+            else if ((k.y >> 2) < pos[j]) before = UM ? 15u : vsm_write_op(k.y & 3u, s0);
             break;
           }
           if (k.x == kEmpty) break;
@@ -296,9 +318,11 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
       }
     } else if (op[j] & 1u) {
       __stcg(const_cast<uint8_t*>(sh) + word[j],
-             (uint8_t)(UM ? 15u : vsm_write_op(op[j], s0) | (BO ? (s_pre[j] & kCVp) : 0u)));
+             (uint8_t)(MD ? md_write((op[j] >> 1) | (((devs >> (2 * j)) & 3u) << 1), s0)
+                       : UM ? 15u : vsm_write_op(op[j], s0) | (BO ? (s_pre[j] & kCVp) : 0u)));
     }
-    fk[j] = ((bom >> j) & 1u) ? 4u : classify_bits(op[j], before);
+    fk[j] = ((bom >> j) & 1u) ? 4u : MD ? md_classify(op[j], (devs >> (2 * j)) & 3u, before)
+                                        : classify_bits(op[j], before);
   }
   emit_faults(p, fk, word, pos, S.bucket_base);
   if (any_w) {
@@ -312,9 +336,9 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
 }
 
 // the fast step of a word-range part (rare: range-heavy buckets), out of line
-template <bool BO, bool UM>
+template <bool BO, bool UM, bool MD>
 __device__ bool step_fast_partial(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
-  return step_fast<true, BO, UM>(S, p, ev, m);
+  return step_fast<true, BO, UM, MD>(S, p, ev, m);
 }
 
 // ---- sort step -------------------------------------------------------------------------
@@ -404,8 +428,33 @@ __device__ __forceinline__ uint32_t acc_combine(uint32_t a, uint32_t b) {  // a 
 __device__ __forceinline__ uint32_t acc_summary(uint32_t op) {
   return op == OP_WH ? (1u | 4u) : (op == OP_WT ? (2u | 8u) : 0u);
 }
+// MD (Z24): bit 31 HEAD, bit 30 CONST; const: bits 0-7 = state; summary: bits 0-2
+// last write (1 host, 2 + d target on device d), bits 3-6 "some write initialised"
+// OV, CV0, CV1, CV2.
+constexpr uint32_t kHeadMd = 1u << 31, kConstMd = 1u << 30;
+__device__ __forceinline__ uint32_t acc_apply_md(uint32_t v, uint32_t s) {
+  const uint32_t lw = v & 7u;
+  if (lw == 1u) s = (s & ~kMdAllCvv) | kOVv;
+  else if (lw >= 2u) s = (s & ~(kMdAllCvv | kOVv)) | (1u << md_cvv(lw - 2u));
+  if (v & 8u) s |= kOVi;
+#pragma unroll
+  for (uint32_t d = 0; d < 3; ++d)
+    if (v & (16u << d)) s |= 1u << md_cvi(d);
+  return s;
+}
+__device__ __forceinline__ uint32_t acc_combine_md(uint32_t a, uint32_t b) {  // a before b
+  if (b & kHeadMd) return b;
+  if (a & kConstMd) return (a & kHeadMd) | kConstMd | acc_apply_md(b, a & 255u);
+  const uint32_t lw = (b & 7u) ? (b & 7u) : (a & 7u);
+  return (a & kHeadMd) | lw | ((a | b) & 0x78u);
+}
+__device__ __forceinline__ uint32_t acc_summary_md(uint32_t op, uint32_t dev) {
+  return op == OP_WH ? (1u | 8u) : (op == OP_WT ? ((2u + dev) | (16u << dev)) : 0u);
+}
+template <bool MD>
+__device__ __forceinline__ uint32_t acc_comb(uint32_t a, uint32_t b) { return MD ? acc_combine_md(a, b) : acc_combine(a, b); }
 
-template <bool BO, bool UM>
+template <bool BO, bool UM, bool MD>
 __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m) {
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   uint32_t lo = 0xFFFFFFFFu, hi = 0;
@@ -484,22 +533,26 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
       const uint32_t full = (h || bo) ? __ldcg(sh + w) : 0u;
       const bool b = bo && ((k >> 30) & 2u) && !(full & kCVp);
       // UM: every write is {both valid, both initialised} (last write 3, any-WH and any-WT)
-      uint32_t v = b ? 0u : UM ? (((k >> 30) & 1u) ? 15u : 0u) : acc_summary(k >> 30);
+      const uint32_t dev = MD ? pin[i] >> 30 : 0u;
+      uint32_t v = b ? 0u : MD ? acc_summary_md(k >> 30, dev) : UM ? (((k >> 30) & 1u) ? 15u : 0u)
+                                                                  : acc_summary(k >> 30);
       uint32_t st = 0;
       if (h) {
-        st = full & 15u;
-        v = kHead | kConst | acc_apply(v, st);
+        st = full & (MD ? 255u : 15u);
+        v = MD ? (kHeadMd | kConstMd | acc_apply_md(v, st)) : (kHead | kConst | acc_apply(v, st));
       }
-      key[j] = k; head[j] = h; s0[j] = st; val[j] = v; wd[j] = w; ps[j] = pin[i];
-      pf[j] = full & kCVp; isb[j] = b;
+      key[j] = k; head[j] = h; s0[j] = st; val[j] = v; wd[j] = w;
+      ps[j] = MD ? (pin[i] & kMdPos) : pin[i];
+      pf[j] = MD ? dev : (full & kCVp);          // MD: the event's device (no kCVp bit then)
+      isb[j] = b;
     }
-    agg = acc_combine(agg, val[j]);
+    agg = acc_comb<MD>(agg, val[j]);
   }
   uint32_t incl = agg;
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {
     const uint32_t o = __shfl_up_sync(FULL, incl, d);
-    if (lane >= (uint32_t)d) incl = acc_combine(o, incl);
+    if (lane >= (uint32_t)d) incl = acc_comb<MD>(o, incl);
   }
   uint32_t excl_lane = __shfl_up_sync(FULL, incl, 1);
   if (lane == 0) excl_lane = 0;
@@ -507,19 +560,19 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
   if (lane == 31) S.wscan[warp] = incl;
   __syncthreads();
   uint32_t wpre = 0;
-  for (uint32_t w = 0; w < warp; ++w) wpre = acc_combine(wpre, S.wscan[w]);
-  uint32_t run = acc_combine(wpre, excl_lane);
+  for (uint32_t w = 0; w < warp; ++w) wpre = acc_comb<MD>(wpre, S.wscan[w]);
+  uint32_t run = acc_comb<MD>(wpre, excl_lane);
   uint32_t fk[RI];
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
     const uint32_t i = tid * RI + j;
     fk[j] = 0;
     if (i < m) {
-      const uint32_t before = head[j] ? s0[j] : (run & 15u);
-      run = acc_combine(run, val[j]);
-      fk[j] = isb[j] ? 4u : classify(key[j] >> 30, before);
+      const uint32_t before = head[j] ? s0[j] : (run & (MD ? 255u : 15u));
+      run = acc_comb<MD>(run, val[j]);
+      fk[j] = isb[j] ? 4u : MD ? md_classify(key[j] >> 30, pf[j], before) : classify(key[j] >> 30, before);
       const bool tail = (i + 1 == m) || ((kin[i + 1] & kWordMask) != wd[j]);
-      if (tail) __stcg(sh + wd[j], (uint8_t)((run & 15u) | pf[j]));
+      if (tail) __stcg(sh + wd[j], (uint8_t)(MD ? (run & 255u) : ((run & 15u) | pf[j])));
     }
   }
   emit_faults(p, fk, wd, ps, bb);
@@ -759,7 +812,7 @@ __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t 
 
 // BO: ARB_F_BO contexts (the buffer-overflow extension, Z20) get their own
 // instance, so the default replay carries none of its checks.
-template <bool BO, bool UM>
+template <bool BO, bool UM, bool MD>
 __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   ReplaySmem& S = *reinterpret_cast<ReplaySmem*>(smem_raw);
@@ -839,18 +892,20 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         m_nxt = issue_gather(S, p, nxt, total, S.ev[cur ^ 1], hint);
       }
       // ---- range ops before the first event, then cut at the next one -------------
-      apply_ops_before<BO>(S, p, ev[0].y);
+      constexpr uint32_t pm = MD ? kMdPos : 0xFFFFFFFFu;   // MD: strip the device bits (Z24)
+      apply_ops_before<BO, MD>(S, p, ev[0].y & pm);
       uint32_t cut = m;
-      if (S.next_op != 0xFFFFFFFFu && ev[m - 1].y > S.next_op) {
+      if (S.next_op != 0xFFFFFFFFu && (ev[m - 1].y & pm) > S.next_op) {
         uint32_t cnt = 0;
-        for (uint32_t e = tid; e < m; e += RT) cnt += ev[e].y < S.next_op;
+        for (uint32_t e = tid; e < m; e += RT) cnt += (ev[e].y & pm) < S.next_op;
         cut = block_sum(cnt, S.red);
       }
       if (mode == kItemSummary) {
         step_summary<UM>(S, ev, cut);
       } else {
-        const bool fast = S.partial ? step_fast_partial<BO, UM>(S, p, ev, cut) : step_fast<false, BO, UM>(S, p, ev, cut);
-        if (!fast) step_sort<BO, UM>(S, p, ev, cut);
+        const bool fast = S.partial ? step_fast_partial<BO, UM, MD>(S, p, ev, cut)
+                                    : step_fast<false, BO, UM, MD>(S, p, ev, cut);
+        if (!fast) step_sort<BO, UM, MD>(S, p, ev, cut);
         if (tid == 0) atomicAdd(fast ? &p.st->steps_fast : &p.st->steps_sort, 1ull);
       }
       e0 += cut;
@@ -867,7 +922,7 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       }
     }
     // the ops after the last event (a slice replay's private states are not kept)
-    if (mode != kItemSlice) apply_ops_before<BO>(S, p, 0xFFFFFFFFu);
+    if (mode != kItemSlice) apply_ops_before<BO, MD>(S, p, 0xFFFFFFFFu);
     if (tid == 0 && total > first) atomicMax(&p.st->max_bucket_events, (unsigned long long)(total - first));
     __syncthreads();
     if (mode == kItemSummary) {
@@ -880,7 +935,8 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
 cudaError_t launch_replay(const ReplayParams& p, int n_ctas, cudaStream_t s) {
   const size_t smem = sizeof(ReplaySmem);
   // ARB_F_BO and ARB_F_UNIFIED exclude each other (arb_init)
-  auto kern = p.um ? k_replay<false, true> : p.bo ? k_replay<true, false> : k_replay<false, false>;
+  auto kern = p.md ? k_replay<false, false, true> : p.um ? k_replay<false, true, false>
+            : p.bo ? k_replay<true, false, false> : k_replay<false, false, false>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   kern<<<n_ctas, RT, smem, s>>>(p);

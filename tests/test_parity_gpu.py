@@ -17,6 +17,7 @@ def check(orc, rec, base, size, **kw):
     flags = (1 if okw.get("dedup_first") else 0) | kw.pop("flags", 0)
     okw["detect_bo"] = bool(flags & 8)                    # ARB_F_BO <-> the oracle's extension (Z20)
     okw["unified"] = bool(flags & 16)                     # ARB_F_UNIFIED <-> unified memory (Z23)
+    okw["n_devices"] = 1 + ((flags >> 8) & 3)             # ARB_F_DEVICES(n) <-> accelerators (Z24)
     exp = orc.replay(rec, base, size, **okw)
     rc, got, shadow, st = run_gpu(rec, base, size, flags=flags, **kw)
     assert rc == exp.rc
@@ -458,3 +459,42 @@ def test_empty_flushes(orc):
     rc, got, shadow, st = run_gpu(rec, base, size, flush_points=[0, 0, rec.shape[0], rec.shape[0]])
     assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
     assert st["flushes"] == 5
+
+
+
+# ---- several accelerators (ARB_F_DEVICES(n), Z24) ----------------------
+def test_devices_example(orc):
+    from gen.trace import encode, OP, MAP
+    A = 0x1000
+    recs = [encode(OP.WH, A, 8), encode(OP.MAP_ENTER, A, 8, arg=MAP.TO | (1 << 6)),
+            encode(OP.RT, A, 8, arg=0), encode(OP.RT, A, 8, arg=1), encode(OP.WT, A, 8, arg=1),
+            encode(OP.RH, A, 8), encode(OP.MAP_EXIT, A, 8, arg=MAP.FROM | (1 << 6)), encode(OP.RH, A, 8)]
+    exp, _ = check(orc, np.array(recs, dtype=np.uint64).reshape(-1, 2), A, 64, flags=1 << 8)
+    assert exp.triples() == [(A // 8, 2, 1), (A // 8, 5, 2)]   # RT on device 0: no CV there; stale host read
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_devices_fuzz(orc, seed):
+    """Random programs on 2 and 3 accelerators: several bucket sizes, word-range
+    parts (flags 4) and flush cuts."""
+    from gen.fuzz import random_program
+    nd = 2 + seed % 2
+    fl = (nd - 1) << 8
+    rec, base, span = random_program(8000 + seed, n_devices=nd, p_task=0.3, p_always=0.2, steps=120)
+    exp, _ = check(orc, rec, base, span, flags=fl)
+    for bb in (2, 5):
+        check(orc, rec, base, span, bucket_bits=bb, flags=fl)
+    check(orc, rec, base, span, flags=fl | 4)
+    if exp.rc == 0:
+        rc, got, shadow, _ = run_gpu(rec, base, span, flags=fl, flush_points=_cuts(rec, 4, seed))
+        assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_devices_large_steps(orc, seed):
+    """Many steps per bucket with sort steps and range ops cutting steps, 3 devices."""
+    from gen.fuzz import random_program
+    rec, base, span = random_program(8100 + seed, n_arrays=6, array_words=8192, steps=500,
+                                     loop_max=20000, n_devices=3)
+    for bb in (0, 11):
+        check(orc, rec, base, span, bucket_bits=bb, flags=2 << 8)
