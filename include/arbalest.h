@@ -188,8 +188,9 @@ int arb_submit_events(arb_ctx ctx, const arb_event* ev, uint64_t n,
  * Both may be NULL.  Synchronizes `stream`.  The batch is consumed.  Returns
  * ARB_OK, ARB_TRUNCATED (more candidates than report_capacity; the count is
  * exact, the stored set is the canonical order of the retained candidates),
- * ARB_EMAP / ARB_ETRACE / ARB_EOPEN (batch discarded, shadow unchanged) or
- * ARB_ECUDA / ARB_ENOMEM. */
+ * ARB_EMAP / ARB_ETRACE (batch discarded, shadow, mapping tables and carried
+ * tasks unchanged), ARB_ENOMEM (also: more than 2^20 - 2 racy or carried task
+ * instances in one flush) or ARB_ECUDA. */
 int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local,
               uint64_t* report_offset_global);
 
