@@ -5,7 +5,10 @@
 // by k_partition.  Output: resolved range ops (Table I),
 // task instances with their joins (Theorem 1, reading Z8),
 // the per-bucket range-op lists consumed by k_replay and the MIR join plan
-// consumed by k_mir_*.  O(C log C) for C control records.
+// consumed by k_mir_*.  O(C log C) for C control records.  Also: TASK_DEPEND
+// edges (Z22), the `always` / `present` modifiers (Z21), unified memory (Z23),
+// one mapping table per accelerator (Z24) and the instances carried across
+// flushes (N2, Z19).
 #pragma once
 #include <cstdint>
 #include <map>

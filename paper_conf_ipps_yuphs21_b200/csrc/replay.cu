@@ -6,7 +6,7 @@
 // staged window of entries (cp.async, double-buffered), applies the resolved range ops
 // (Table I transfers / allocate / release; target update P:121) to
 // the bucket's shadow at their trace positions, and processes the events in
-// steps of <= 2048 that never straddle a range op:
+// steps of <= 1024 that never straddle a range op:
 //
 //   fast step  (every word has at most one write in the step): a shared-memory
 //              hash of the written words, word -> write position.  A read's
@@ -20,6 +20,10 @@
 // Both classify reads as in P:263 (read_host needs OV valid, read_target CV
 // valid) and split UUM / USD with the init bits (Table II).  The shadow
 // (1 byte per word) carries each word's state across steps.
+//
+// k_replay<BO, UM, MD> instances: the default one, the buffer-overflow extension
+// (ARB_F_BO, Z20), unified memory (ARB_F_UNIFIED, Z23) and several accelerators
+// (ARB_F_DEVICES, 8-bit states, Z24); the mode checks compile away in the others.
 #include "kcommon.cuh"
 #include <algorithm>
 
