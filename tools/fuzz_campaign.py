@@ -27,7 +27,7 @@ for k in range(n):
         flags |= 4                               # word-range parts / time slices
     if rs.random() < 0.2:
         flags |= 1                               # dedup-first
-    big = rs.random() < 0.2
+    big = rs.random() < float(os.environ.get("BIG_FRACTION", "0.2"))
     rec, base, span = random_program(seed, n_arrays=int(rs.integers(1, 6)),
                                      array_words=int(rs.choice([16, 64, 512, 4096])) if not big else 8192,
                                      steps=int(rs.integers(20, 200)) if not big else 400,
