@@ -116,16 +116,22 @@ class Program:
             self.quiescent.append(self.n)
         return self
 
-    def distinct_words(self, lo, hi, ranges):
+    def distinct_words(self, lo, hi, ranges, sector_words=1):
         """W of B_alg for each global record range: the union of the mapped sections
         entered in the range, clipped to the tracked words [lo, hi).  Every access
-        of these programs lies inside a section of its own region."""
+        of these programs lies inside a section of its own region.  sector_words > 1:
+        whole shadow sectors of that many words (1 B of shadow per word) counted as
+        touched words (the sector-granular variant of SURVEY §8(d))."""
         secs = np.array(self.sections, dtype=np.uint64).reshape(-1, 3)
         out = []
+        g = np.int64(sector_words)
         for g0, g1 in ranges:
             m = (secs[:, 2] >= g0) & (secs[:, 2] < g1)
             a = np.maximum(secs[m, 0], np.uint64(lo)).astype(np.int64)
             b = np.minimum(secs[m, 1], np.uint64(hi)).astype(np.int64)
+            if sector_words > 1:
+                keep = a < b
+                a, b = (a[keep] // g) * g, ((b[keep] + g - 1) // g) * g
             keep = a < b
             a, b = a[keep], b[keep]
             order = np.argsort(a)

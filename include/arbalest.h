@@ -79,15 +79,33 @@ enum arb_status {
   ARB_EMAP = -4,      /* map clause partially overlaps a present entry (Z6)          */
   ARB_ETRACE = -5,    /* malformed trace (Z18)                              */
   ARB_ESTATE = -6,    /* call out of order (e.g. get_reports before any flush)        */
-  ARB_EOPEN = -7      /* reserved: open blocks are carried across flushes (Z19); the
+  ARB_EOPEN = -7,     /* reserved: open blocks are carried across flushes (Z19); the
                          oracle returns it for a whole trace that ends inside a block */
+  ARB_EPEER = -8      /* communicator only: another rank's arb_flush failed (see below) */
 };
 /* After ARB_EMAP / ARB_ETRACE / ARB_EOPEN the pending batch is discarded, the
  * committed shadow is unchanged and the context stays usable.  After ARB_ECUDA
- * the context must be destroyed. */
+ * the context must be destroyed.
+ * With a communicator (world > 1, or world == 1 with an NCCL id) arb_flush is a
+ * collective: every rank calls it equally often, and the ranks exchange their
+ * status twice per flush (ncclAllGather):
+ *  - after validation (decode, Table I resolution): if any rank's batch is
+ *    rejected, every rank discards its batch — the failing rank returns its own
+ *    error, the others ARB_EPEER — and every context stays usable (shadow,
+ *    mapping tables and carried tasks unchanged);
+ *  - with the report counts at the end: a rank that failed after validation
+ *    (ARB_ENOMEM / ARB_ECUDA) still takes part, and the others return ARB_EPEER;
+ *    then every rank's context must be destroyed (their shadows differ in state).
+ * So one malformed record on one shard fails every rank's flush, and none waits
+ * in a collective a peer skipped. */
 
 /* ---- configuration ------------------------------------------------------------- */
-#define ARB_F_DEDUP_FIRST 0x1u  /* keep only the first report per (word, kind) (Z3)      */
+#define ARB_F_DEDUP_FIRST 0x1u  /* keep only the first report per (word, kind) (Z3) over the
+                                   whole trace: a pair reported by an earlier flush is not
+                                   reported again (a device set of the reported pairs
+                                   persists across flushes).  With
+                                   ARB_TRUNCATED the count is an upper bound and the stored
+                                   set may miss firsts that were dropped                    */
 #define ARB_F_TIMING      0x2u  /* record CUDA events around every kernel (arb_get_stats) */
 #define ARB_F_SMALL_PARTS 0x4u  /* test knob: split every bucket with >= 2048 range-op words
                                    into word-range parts replayed by separate CTAs, and
@@ -119,7 +137,9 @@ typedef struct {
                              /*   mode the range is this rank's shard.                     */
   int      device;           /* CUDA ordinal                                               */
   int      rank, world;      /* address shard of this process; world == 1: single GPU      */
-  const void* nccl_unique_id;/* ncclUniqueId* (128 B) when world > 1, else NULL            */
+  const void* nccl_unique_id;/* ncclUniqueId* (128 B): required when world > 1; with
+                                world == 1 an id makes a 1-rank communicator (the count
+                                exchange then runs on one GPU); NULL: no communicator      */
   uint64_t report_capacity;  /* device report-candidate capacity, 0 = default (2^24)       */
   uint32_t flags;            /* ARB_F_*                                                    */
   uint32_t bucket_bits;      /* log2 words per address bucket, 0 = automatic               */
@@ -151,13 +171,17 @@ typedef struct {
   uint64_t work_items;       /* replay work items (buckets, word-range parts, hot slices)   */
   uint64_t hot_buckets;      /* buckets replayed as time slices (hot words, K5)             */
   uint64_t reports_bo;       /* reports of kind ARB_BO in the last flush (ARB_F_BO)         */
+  uint64_t nccl_ranks;       /* ranks of the context's NCCL communicator (ncclCommCount), 0 =
+                                no communicator                                              */
+  uint64_t exchanges;        /* collectives (status / count ncclAllGather) of the last flush */
 } arb_stats;
 
 typedef struct arb_ctx_s* arb_ctx;
 
 /* Create a context on cfg->device: allocates and zeroes the shadow (all words
- * start invalid), workspaces, and (world > 1) the NCCL communicator from
- * cfg->nccl_unique_id.  Returns ARB_OK and *out, or an error (*out = NULL).
+ * start invalid), workspaces, and (if cfg->nccl_unique_id) the NCCL
+ * communicator of cfg->world ranks.  Returns ARB_OK and *out, or an error
+ * (*out = NULL): ARB_EINVAL for a bad range, rank, or an unknown flag bit.
  * Ownership: the context owns the shadow, workspaces and report buffer. */
 int arb_init(const arb_config* cfg, arb_ctx* out);
 
@@ -202,7 +226,9 @@ int arb_get_reports(arb_ctx ctx, arb_report* out, uint64_t cap, uint64_t* n_writ
 
 /* Copy the final shadow byte of words [word_lo, word_lo + n) (absolute word
  * indices inside the tracked range) to out (host or device).  Bits: 0 OVv,
- * 1 CVv, 2 OVi, 3 CVi (Table II).  Synchronous. */
+ * 1 CVv, 2 OVi, 3 CVi (Table II); with ARB_F_BO bit 4 = CVp (the word
+ * has a CV, Z20); with ARB_F_DEVICES(n) bits 1/3 are device 0's CV valid /
+ * initialised and bits 4/5, 6/7 those of devices 1 and 2 (Z24).  Synchronous. */
 int arb_get_shadow(arb_ctx ctx, uint64_t word_lo, uint64_t n, uint8_t* out, int out_on_device);
 
 /* Statistics of the last flush and totals. */

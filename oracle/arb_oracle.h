@@ -110,6 +110,12 @@ typedef struct {
    * MAP_ENTER / MAP_EXIT / UPDATE.  Single-device traces are unchanged.
    * Excludes detect_bo and unified. */
   int             n_devices;
+  /* Continuation: if non-NULL, the state of every tracked word before the first
+   * record (one byte per slot, as shadow_out) — the final shadow of a replay of
+   * the records that precede this trace, cut where no task is open or unjoined
+   * and no section is mapped (a quiescent point).  NULL: every word starts
+   * invalid. */
+  const uint8_t*  shadow_in;
 } orc_config;
 
 typedef struct {
@@ -133,6 +139,14 @@ typedef struct {
 int  orc_replay(const orc_config* cfg, const orc_record* rec, uint64_t n,
                 const uint64_t* global_index, orc_report** out, uint64_t* n_out,
                 uint8_t* shadow_out, orc_stats* stats);
+/* Address-sharded mode (the oracle "on all host cores"): the
+ * same sequential replay run by `threads` POSIX threads, each over a contiguous
+ * range of the tracked words (each thread walks every record and resolves the
+ * replicated control stream itself; the task pre-pass is shared).  Results —
+ * reports, shadow, stats — are identical to orc_replay's. */
+int  orc_replay_sharded(const orc_config* cfg, const orc_record* rec, uint64_t n,
+                        const uint64_t* global_index, int threads, orc_report** out, uint64_t* n_out,
+                        uint8_t* shadow_out, orc_stats* stats);
 void orc_free(void* p);
 
 #ifdef __cplusplus

@@ -27,7 +27,7 @@ class _Config(ctypes.Structure):
                 ("dedup_first", ctypes.c_int),
                 ("tracked_words", ctypes.POINTER(ctypes.c_uint64)),
                 ("n_tracked", ctypes.c_uint64), ("detect_bo", ctypes.c_int), ("unified", ctypes.c_int),
-                ("n_devices", ctypes.c_int)]
+                ("n_devices", ctypes.c_int), ("shadow_in", ctypes.c_void_p)]
 
 
 class _Stats(ctypes.Structure):
@@ -45,7 +45,7 @@ def build(force: bool = False) -> str:
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < newest:
         tmp = _LIB + f".tmp{os.getpid()}"
         subprocess.check_call(["gcc", "-O2", "-std=c99", "-Wall", "-shared", "-fPIC",
-                               "-o", tmp, _SRC])
+                               "-o", tmp, _SRC, "-lpthread"])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -62,6 +62,11 @@ def _load():
                                    ctypes.c_void_p, ctypes.POINTER(ctypes.c_void_p),
                                    ctypes.POINTER(ctypes.c_uint64), ctypes.c_void_p,
                                    ctypes.POINTER(_Stats)]
+        lib.orc_replay_sharded.restype = ctypes.c_int
+        lib.orc_replay_sharded.argtypes = [ctypes.POINTER(_Config), ctypes.c_void_p, ctypes.c_uint64,
+                                           ctypes.c_void_p, ctypes.c_int, ctypes.POINTER(ctypes.c_void_p),
+                                           ctypes.POINTER(ctypes.c_uint64), ctypes.c_void_p,
+                                           ctypes.POINTER(_Stats)]
         lib.orc_free.argtypes = [ctypes.c_void_p]
         lib.orc_free.restype = None
         _lib = lib
@@ -82,9 +87,13 @@ class OracleResult:
 def replay(records: np.ndarray, addr_base: int, addr_bytes: int, *, dedup_first: bool = False,
            tracked_words: np.ndarray | None = None, global_index: np.ndarray | None = None,
            want_shadow: bool = True, detect_bo: bool = False, unified: bool = False,
-           n_devices: int = 1) -> OracleResult:
+           n_devices: int = 1, threads: int = 1, shadow_in: np.ndarray | None = None) -> OracleResult:
     """Replay ``records`` (uint64 array of shape (n, 2): w0, w1) through the oracle.
-    ``detect_bo``: the buffer-overflow extension (reading Z20)."""
+    ``detect_bo``: the buffer-overflow extension (reading Z20).
+    ``threads`` > 1: the address-sharded mode (``orc_replay_sharded``: the same
+    sequential replay, one thread per contiguous range of tracked words).
+    ``shadow_in``: continuation state (the final shadow of a replay of the preceding
+    records, cut at a quiescent point); None = every word starts invalid."""
     lib = _load()
     rec = np.ascontiguousarray(records, dtype=np.uint64).reshape(-1, 2)
     n = rec.shape[0]
@@ -103,6 +112,11 @@ def replay(records: np.ndarray, addr_base: int, addr_bytes: int, *, dedup_first:
         nslots = tw.size
     else:
         nslots = addr_bytes // 8
+    sin = None
+    if shadow_in is not None:
+        sin = np.ascontiguousarray(shadow_in, dtype=np.uint8)
+        assert sin.size >= nslots
+        cfg.shadow_in = sin.ctypes.data
     gi = None
     if global_index is not None:
         gi = np.ascontiguousarray(global_index, dtype=np.uint64)
@@ -111,14 +125,17 @@ def replay(records: np.ndarray, addr_base: int, addr_bytes: int, *, dedup_first:
     out = ctypes.c_void_p()
     nout = ctypes.c_uint64()
     st = _Stats()
-    rc = lib.orc_replay(ctypes.byref(cfg), rec.ctypes.data if n else None, n,
-                        gi.ctypes.data if gi is not None else None, ctypes.byref(out),
-                        ctypes.byref(nout), shadow.ctypes.data if shadow is not None else None,
-                        ctypes.byref(st))
+    args = (ctypes.byref(cfg), rec.ctypes.data if n else None, n, gi.ctypes.data if gi is not None else None)
+    tail = (ctypes.byref(out), ctypes.byref(nout), shadow.ctypes.data if shadow is not None else None,
+            ctypes.byref(st))
+    if threads > 1:
+        rc = lib.orc_replay_sharded(*args, threads, *tail)
+    else:
+        rc = lib.orc_replay(*args, *tail)
     reps = np.zeros(0, dtype=REPORT_DTYPE)
     if rc == 0 and nout.value:
         buf = (ctypes.c_char * (nout.value * REPORT_DTYPE.itemsize)).from_address(out.value)
-        reps = np.frombuffer(bytes(buf), dtype=REPORT_DTYPE).copy()
+        reps = np.frombuffer(buf, dtype=REPORT_DTYPE).copy()
     if out.value:
         lib.orc_free(out)
     stats = {name: int(getattr(st, name)) for name, _ in _Stats._fields_}

@@ -6,5 +6,5 @@ and ``shard.py`` (host-side address sharding of traces for multi-GPU runs).
 """
 from .binding import (Context, ArbError, load, reports_to_triples, EXPORTS,  # noqa: F401
                       ARB_OK, ARB_TRUNCATED, ARB_EINVAL, ARB_ENOMEM, ARB_ECUDA, ARB_EMAP,
-                      ARB_ETRACE, ARB_ESTATE, ARB_EOPEN, ARB_F_DEDUP_FIRST, ARB_F_TIMING,
+                      ARB_ETRACE, ARB_ESTATE, ARB_EOPEN, ARB_EPEER, ARB_F_DEDUP_FIRST, ARB_F_TIMING,
                       ARB_F_SMALL_PARTS, ARB_F_BO, ARB_BO, ARB_F_UNIFIED, ARB_F_DEVICES)

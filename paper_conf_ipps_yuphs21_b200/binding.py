@@ -16,6 +16,7 @@ LIB_PATH = os.path.join(PKG, "libarbalest.so")
 
 ARB_OK, ARB_TRUNCATED = 0, 1
 ARB_EINVAL, ARB_ENOMEM, ARB_ECUDA, ARB_EMAP, ARB_ETRACE, ARB_ESTATE, ARB_EOPEN = -1, -2, -3, -4, -5, -6, -7
+ARB_EPEER = -8
 ARB_F_DEDUP_FIRST, ARB_F_TIMING = 0x1, 0x2
 ARB_F_SMALL_PARTS = 0x4
 ARB_F_BO = 0x8          # buffer-overflow extension (Z20)
@@ -27,7 +28,7 @@ def ARB_F_DEVICES(n):
     """n accelerators (Z24), n <= 3."""
     return (n - 1) << 8
 STATUS = {0: "ARB_OK", 1: "ARB_TRUNCATED", -1: "ARB_EINVAL", -2: "ARB_ENOMEM", -3: "ARB_ECUDA",
-          -4: "ARB_EMAP", -5: "ARB_ETRACE", -6: "ARB_ESTATE", -7: "ARB_EOPEN"}
+          -4: "ARB_EMAP", -5: "ARB_ETRACE", -6: "ARB_ESTATE", -7: "ARB_EOPEN", -8: "ARB_EPEER"}
 EXPORTS = ("arb_init", "arb_submit_events", "arb_flush", "arb_get_reports", "arb_get_shadow",
            "arb_get_stats", "arb_last_error", "arb_destroy")
 
@@ -55,7 +56,8 @@ class arb_stats(ctypes.Structure):
                 ("steps_fast", ctypes.c_uint64), ("steps_sort", ctypes.c_uint64),
                 ("ms_segsort", ctypes.c_double), ("ms_host_control", ctypes.c_double),
                 ("work_items", ctypes.c_uint64), ("hot_buckets", ctypes.c_uint64),
-                ("reports_bo", ctypes.c_uint64)]
+                ("reports_bo", ctypes.c_uint64), ("nccl_ranks", ctypes.c_uint64),
+                ("exchanges", ctypes.c_uint64)]
 
     def as_dict(self):
         d = {}

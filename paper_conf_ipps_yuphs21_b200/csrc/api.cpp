@@ -24,7 +24,8 @@ struct NcclId { char internal[128]; };
 typedef int (*nccl_init_fn)(void** comm, int nranks, NcclId id, int rank);
 typedef int (*nccl_allgather_fn)(const void* send, void* recv, size_t count, int dtype, void* comm, cudaStream_t s);
 typedef int (*nccl_destroy_fn)(void* comm);
-constexpr int kNcclUint64 = 5;  // ncclUint64
+typedef int (*nccl_count_fn)(const void* comm, int* count);
+constexpr int kNcclInt64 = 4;   // ncclInt64
 
 template <class T>
 struct DevBuf {
@@ -143,6 +144,10 @@ struct arb_ctx_s {
   DevBuf<uint32_t> hvals;
   // N2: nowait instances unjoined at the end of the last flush (committed with the map table)
   std::vector<CarriedInst> carried;
+  LastEnded last_ended;                       // Z22 across flushes (committed with `carried`)
+  // ARB_F_DEDUP_FIRST across flushes: (word, kind) keys reported so far (open addressing)
+  DevBuf<unsigned long long> dset, dset_cnt;
+  uint64_t dset_slots = 0, dset_n = 0;
   DevBuf<uint4> carry_ent, carry_next;        // their access summaries {word lo, word hi, carried idx, flag}
   uint64_t n_carry = 0;
   DevBuf<uint32_t> m_cmap, m_co_of;
@@ -167,8 +172,13 @@ struct arb_ctx_s {
   void* comm = nullptr;
   nccl_allgather_fn nccl_allgather = nullptr;
   nccl_destroy_fn nccl_destroy = nullptr;
-  DevBuf<uint64_t> counts;
+  DevBuf<int64_t> counts;                     // [world] x {status, report count} + own pair
+  int comm_ranks = 0;
 };
+
+// every ARB_F_* bit arb_init accepts (the two ARB_F_DEVICES bits included)
+constexpr uint32_t kKnownFlags = ARB_F_DEDUP_FIRST | ARB_F_TIMING | ARB_F_SMALL_PARTS | ARB_F_BO | ARB_F_UNIFIED |
+                                 (3u << ARB_F_DEVICES_SHIFT);
 
 static int fail(arb_ctx c, int rc, const std::string& msg) {
   if (c) c->err = msg;
@@ -183,12 +193,29 @@ static int cuda_fail(arb_ctx c, cudaError_t e, const char* where) {
     if (_e != cudaSuccess) return cuda_fail(ctx, _e, where); \
   } while (0)
 
+// ncclAllGather of one {a, b} pair per rank (stream-ordered, then synchronised);
+// all = world pairs in rank order.  ARB_ECUDA if NCCL or CUDA fails.
+static int nccl_exchange(arb_ctx ctx, cudaStream_t s, int64_t a, int64_t b, std::vector<int64_t>& all) {
+  const int w = ctx->cfg.world;
+  int64_t mine[2] = {a, b};
+  all.assign(2 * (size_t)w, 0);
+  int64_t* own = ctx->counts.p + 2 * w;
+  if (cudaMemcpyAsync(own, mine, sizeof(mine), cudaMemcpyHostToDevice, s) != cudaSuccess)
+    return fail(ctx, ARB_ECUDA, "count exchange: copy");
+  if (ctx->nccl_allgather(own, ctx->counts.p, 2, kNcclInt64, ctx->comm, s) != 0)
+    return fail(ctx, ARB_ECUDA, "ncclAllGather failed");
+  if (cudaMemcpyAsync(all.data(), ctx->counts.p, 16 * (size_t)w, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess)
+    return fail(ctx, ARB_ECUDA, "count exchange: read-back");
+  return ARB_OK;
+}
+
 extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
   if (!out) return ARB_EINVAL;
   *out = nullptr;
   if (!cfg || (cfg->addr_base & 7) || (cfg->addr_bytes & 7) || cfg->addr_bytes == 0 ||
       cfg->addr_base + cfg->addr_bytes > (1ull << 48) || cfg->world < 1 || cfg->rank < 0 ||
-      cfg->rank >= cfg->world || (cfg->world > 1 && !cfg->nccl_unique_id) ||
+      cfg->rank >= cfg->world || (cfg->world > 1 && !cfg->nccl_unique_id) || (cfg->flags & ~kKnownFlags) ||
       ((cfg->flags & ARB_F_BO) && (cfg->flags & ARB_F_UNIFIED)) || ((cfg->flags >> ARB_F_DEVICES_SHIFT) & 3u) > 2u ||
       (((cfg->flags >> ARB_F_DEVICES_SHIFT) & 3u) && (cfg->flags & (ARB_F_BO | ARB_F_UNIFIED))))
     return ARB_EINVAL;
@@ -235,19 +262,24 @@ extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
   if (e == cudaSuccess) e = ctx->h_weight.ensure(kMaxBuckets);
   if (e == cudaSuccess) e = cudaDeviceSynchronize();
   if (e != cudaSuccess) { arb_destroy(ctx); return ARB_ENOMEM; }
-  if (cfg->world > 1) {
+  if (cfg->nccl_unique_id) {
+    // world > 1: the address-sharded job's communicator; world == 1 with an id: a
+    // 1-rank communicator, so that the exchange path runs on a single GPU too
     ctx->nccl_lib = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
     if (!ctx->nccl_lib) { arb_destroy(ctx); return ARB_ECUDA; }
     auto init = (nccl_init_fn)dlsym(ctx->nccl_lib, "ncclCommInitRank");
+    auto count = (nccl_count_fn)dlsym(ctx->nccl_lib, "ncclCommCount");
     ctx->nccl_allgather = (nccl_allgather_fn)dlsym(ctx->nccl_lib, "ncclAllGather");
     ctx->nccl_destroy = (nccl_destroy_fn)dlsym(ctx->nccl_lib, "ncclCommDestroy");
-    if (!init || !ctx->nccl_allgather || !ctx->nccl_destroy) { arb_destroy(ctx); return ARB_ECUDA; }
+    if (!init || !count || !ctx->nccl_allgather || !ctx->nccl_destroy) { arb_destroy(ctx); return ARB_ECUDA; }
     NcclId id;
     std::memcpy(id.internal, cfg->nccl_unique_id, sizeof(id.internal));
-    if (init(&ctx->comm, cfg->world, id, cfg->rank) != 0 || ctx->counts.ensure(cfg->world + 1) != cudaSuccess) {
+    if (init(&ctx->comm, cfg->world, id, cfg->rank) != 0 || ctx->counts.ensure(2 * cfg->world + 2) != cudaSuccess ||
+        count(ctx->comm, &ctx->comm_ranks) != 0 || ctx->comm_ranks != cfg->world) {
       arb_destroy(ctx);
       return ARB_ECUDA;
     }
+    ctx->stats.nccl_ranks = (uint64_t)ctx->comm_ranks;
   }
   *out = ctx;
   return ARB_OK;
@@ -264,7 +296,7 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   ctx->m_rr_cum.release(); ctx->m_ins_inst.release(); ctx->m_qry_open_start.release(); ctx->m_open_list.release();
   ctx->m_own_start.release(); ctx->m_win_start.release(); ctx->m_own.release(); ctx->m_win.release();
   ctx->m_rr.release(); ctx->hkeys.release(); ctx->hvals.release(); ctx->counts.release();
-  ctx->carry_ent.release(); ctx->carry_next.release(); ctx->m_cmap.release(); ctx->m_co_of.release();
+  ctx->carry_ent.release(); ctx->carry_next.release(); ctx->dset.release(); ctx->dset_cnt.release(); ctx->m_cmap.release(); ctx->m_co_of.release();
   ctx->d_bin_map.release(); ctx->d_items.release(); ctx->h_items.release(); ctx->h_weight.release();
   ctx->d_slice_items.release(); ctx->h_slice_items.release(); ctx->d_hot.release(); ctx->h_hot.release();
   ctx->d_hot_off.release(); ctx->h_hot_off.release(); ctx->hot_F.release(); ctx->hot_P.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_cut.release();
@@ -447,15 +479,29 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   int launches = 0;
   const uint64_t n = ctx->pending;
   arb_stats& S = ctx->stats;
+  S.exchanges = 0;
   S.records = n; S.access_words = S.range_words = S.control_records = S.range_ops = S.tasks = 0;
   S.reports = 0; std::memset(S.reports_by_kind, 0, sizeof(S.reports_by_kind)); S.ignored_words = 0;
   S.ms_partition = S.ms_control = S.ms_replay = S.ms_mir = S.ms_reports = S.ms_total = 0;
   S.ms_segsort = S.ms_host_control = 0;
   S.buckets = ctx->n_buckets; S.bucket_bits = ctx->bucket_bits; S.max_bucket_events = 0;
 
-  // ---- resolve the batch into one device array ---------------------------
+  // Phase A (validation): decode + partition and control resolution.  Nothing
+  // committed changes here, so an error discards the batch and leaves the context
+  // usable.  With a communicator every rank then exchanges its phase-A status, and
+  // a batch any rank rejects is discarded by all of them (ARB_EPEER on the others):
+  // the ranks stay in lockstep and nobody waits in a collective a peer skipped.
   const uint4* ev = nullptr;
   const uint64_t* gidx = nullptr;
+  const uint64_t index_base = ctx->next_index;
+  const bool balanced = ctx->bucket_bits == 0;
+  DevStats& hst = *ctx->h_stats.p;
+  std::vector<double> bucket_events;      // estimated events per bucket (sampled)
+  MapTable map;
+  FlushPlan plan;
+  std::chrono::steady_clock::time_point t_host0, t_host1;
+  int rc = [&]() -> int {
+  // ---- resolve the batch into one device array ---------------------------
   if (n) {
     bool single_dev = ctx->subs.size() == 1 && ctx->subs[0].on_device;
     if (single_dev) {
@@ -478,10 +524,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
       gidx = ctx->any_gidx ? ctx->gidx_staging.p : nullptr;
     }
   }
-  const uint64_t index_base = ctx->next_index;
-
   if (timing) cudaEventRecord(ctx->ev[0], s);
-  const bool balanced = ctx->bucket_bits == 0;
   // ---- bucket balancing on a sampled address histogram (all on the device) ----
   if (balanced) {
     CK(ctx->d_hist.ensure(ctx->n_bins), "alloc hist");
@@ -516,7 +559,6 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   CK(ctx->part_ev.ensure((size_t)std::max<uint32_t>(n_chunks, 1) * kChunkCap), "alloc part_ev");
   if (ctx->seg_cap < (uint64_t)n_chunks * 2 + 4096) ctx->seg_cap = (uint64_t)n_chunks * 2 + 4096;
   CK(ctx->seg_a.ensure(std::max<uint64_t>(ctx->seg_cap, 1)), "alloc segments");
-  DevStats& hst = *ctx->h_stats.p;
   PartParams pp{};
   for (int attempt = 0; attempt < 2; ++attempt) {
     CK(cudaMemsetAsync(ctx->dstats.p, 0, sizeof(DevStats), s), "stats init");
@@ -540,11 +582,8 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     CK(ctx->seg_a.ensure(ctx->seg_cap), "grow segments");
   }
   if (timing) cudaEventRecord(ctx->ev[1], s);
-  if (hst.err_pos != ~0ull) {
-    reset_batch(ctx);
+  if (hst.err_pos != ~0ull)
     return fail(ctx, ARB_ETRACE, "malformed record at batch position " + std::to_string(hst.err_pos));
-  }
-  std::vector<double> bucket_events;      // estimated events per bucket (sampled)
   if (balanced) {
     const uint32_t nb = *ctx->h_nb.p;
     ctx->bucket_start.assign(ctx->h_bstart.p, ctx->h_bstart.p + nb + 1);
@@ -571,7 +610,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
                             ctx->segs.p, s, &launches), "sort segments");
     if (timing) cudaEventRecord(ctx->ev[8], s);
   }
-  const auto t_host0 = std::chrono::steady_clock::now();
+  t_host0 = std::chrono::steady_clock::now();
 
   // ---- A2: control resolution on the host -------------------------------------
   std::vector<CtlRec> ctl(hst.n_ctl);
@@ -583,21 +622,41 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     std::memcpy(ctl.data(), ctx->h_ctl.p, hst.n_ctl * sizeof(CtlRec));
     std::sort(ctl.begin(), ctl.end(), [](const CtlRec& a, const CtlRec& b) { return a.pos < b.pos; });
   }
-  const auto t_host1 = std::chrono::steady_clock::now();
-  MapTable map = ctx->map;
-  FlushPlan plan;
+  t_host1 = std::chrono::steady_clock::now();
+  map = ctx->map;
   resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_start, map, plan,
                   (ctx->cfg.flags & ARB_F_BO) != 0, &ctx->carried, (ctx->cfg.flags & ARB_F_UNIFIED) != 0,
-                  1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u));
-  if (plan.rc != 0) {
-    CK(cudaStreamSynchronize(s), "sync");
-    reset_batch(ctx);
+                  1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u), &ctx->last_ended);
+  if (plan.rc != 0)
     return fail(ctx, plan.rc, plan.err + " (batch position " + std::to_string(plan.err_pos) + ")");
+  return ARB_OK;
+  }();
+  {   // every rank learns whether every rank's batch is valid
+    int64_t peer = 0;
+    if (ctx->comm) {
+      std::vector<int64_t> all;
+      if (nccl_exchange(ctx, s, rc, 0, all) != ARB_OK) { reset_batch(ctx); return ARB_ECUDA; }
+      for (int r = 0; r < (int)all.size() / 2; ++r)
+        if (r != ctx->cfg.rank && all[2 * r] < 0) peer = all[2 * r];
+      S.exchanges += 1;
+    }
+    if (rc == ARB_OK && peer < 0) rc = fail(ctx, ARB_EPEER, "another rank rejected its part of the batch (" +
+                                                                   std::to_string(peer) + "); batch discarded");
+  }
+  if (rc != ARB_OK) {
+    cudaStreamSynchronize(s);
+    reset_batch(ctx);
+    return rc;
   }
   S.range_words = plan.range_words;
   S.range_ops = plan.range_ops.size();
   S.tasks = plan.tasks;
   S.ignored_words = hst.ignored_words + plan.ignored_words;
+  // Phase B: replay (commits the shadow), MIR join, report compaction.  A failure
+  // here is ARB_ENOMEM / ARB_ECUDA: the context must be destroyed (on every rank);
+  // the count exchange still runs so that no peer waits for this rank.
+  uint64_t n_vsm = 0, kept_vsm = 0, n_carry_next = 0;
+  int rcb = [&]() -> int {
   const auto t_host2 = std::chrono::steady_clock::now();
   build_items(ctx, plan, bucket_events);
   if (getenv("ARB_HOST_PROFILE")) {
@@ -653,14 +712,14 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   if (timing) cudaEventRecord(ctx->ev[3], s);
   CK(cudaMemcpyAsync(&hst, ctx->dstats.p, sizeof(hst), cudaMemcpyDeviceToHost, s), "stats d2h");
   CK(cudaStreamSynchronize(s), "replay sync");
-  const uint64_t n_vsm = hst.n_cand;                 // exact: VSM candidates are unique
-  uint64_t kept_vsm = std::min(n_vsm, ctx->cand_cap);
+  n_vsm = hst.n_cand;                                // exact: VSM candidates are unique
+  kept_vsm = std::min(n_vsm, ctx->cand_cap);
   S.max_bucket_events = hst.max_bucket_events;
   S.steps_fast = hst.steps_fast;
   S.steps_sort = hst.steps_sort;
 
   // ---- A6: MIR join ---------------------------------------------------------------
-  uint64_t n_mir = 0, n_carry_next = 0;
+  uint64_t n_mir = 0;
   const bool carry_in = ctx->n_carry && !plan.carry_in_dense.empty();
   if (!plan.mir.empty() || carry_in || !plan.carry_out.empty()) {
     MirPlanH& M = plan.mir;
@@ -737,7 +796,28 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   cp.dedup_first = (ctx->cfg.flags & ARB_F_DEDUP_FIRST) ? 1 : 0;
   cp.gidx = gidx; cp.index_base = index_base;
   cp.out = ctx->reports.p; cp.n_out = ctx->dcount.p;
+  if (cp.dedup_first) {
+    // the persistent (word, kind) set of earlier flushes: keep its load <= 1/2
+    const uint64_t need = 2 * (ctx->dset_n + n_cand);
+    if (ctx->dset_slots < need) {
+      uint64_t slots = 1ull << 16;
+      while (slots < need) slots <<= 1;
+      DevBuf<unsigned long long> nb;
+      CK(nb.ensure(slots), "alloc dedup set");
+      CK(cudaMemsetAsync(nb.p, 0, slots * 8, s), "clear dedup set");
+      if (ctx->dset_slots) CK(launch_dedup_rehash(ctx->dset.p, ctx->dset_slots, nb.p, slots - 1, s), "rehash");
+      CK(cudaStreamSynchronize(s), "rehash sync");
+      ctx->dset.release();
+      ctx->dset = nb;
+      ctx->dset_slots = slots;
+    }
+    CK(ctx->dset_cnt.ensure(1), "alloc dedup count");
+    CK(cudaMemsetAsync(ctx->dset_cnt.p, 0, 8, s), "dedup count");
+    cp.dset = ctx->dset.p; cp.dset_mask = ctx->dset_slots - 1; cp.dset_count = ctx->dset_cnt.p;
+  }
   CK(launch_compact(cp, s, &launches), "compact");
+  unsigned long long dset_new = 0;
+  if (cp.dedup_first) CK(cudaMemcpyAsync(&dset_new, ctx->dset_cnt.p, 8, cudaMemcpyDeviceToHost, s), "dedup count d2h");
   unsigned long long cnt4[8] = {0, 0, 0, 0, 0, 0, 0, 0};   // [0] total, [k] kind k
   CK(cudaMemcpyAsync(cnt4, ctx->dcount.p, sizeof(cnt4), cudaMemcpyDeviceToHost, s), "count d2h");
   if (timing) cudaEventRecord(ctx->ev[5], s);
@@ -746,24 +826,37 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   ctx->n_stored = n_out;
   for (int k = 1; k < 4; ++k) S.reports_by_kind[k] = cnt4[k];
   S.reports_bo = cnt4[ARB_BO];
-  // dropped VSM candidates are unique and distinct from every retained one
+  ctx->dset_n += dset_new;
+  // dropped VSM candidates are unique and distinct from every retained one (raw
+  // mode; with ARB_F_DEDUP_FIRST an upper bound, see arbalest.h)
   ctx->n_reports = n_out + (n_vsm - kept_vsm);
-  int rc = n_vsm > kept_vsm ? ARB_TRUNCATED : ARB_OK;
-  if (rc == ARB_TRUNCATED) ctx->err = "report candidates exceeded report_capacity";
+  return ARB_OK;
+  }();
 
-  // ---- A7: multi-GPU count exchange ----------------------------------------------
+  // ---- A7: multi-GPU count exchange --------------------------------
+  // One ncclAllGather of {status, report count} per rank; the exclusive prefix of
+  // the counts in rank order is this rank's offset in the global report list.
   uint64_t offset = 0;
-  if (ctx->cfg.world > 1) {
-    uint64_t mine = ctx->n_reports;
-    CK(cudaMemcpyAsync(ctx->counts.p + ctx->cfg.world, &mine, 8, cudaMemcpyHostToDevice, s), "counts");
-    if (ctx->nccl_allgather(ctx->counts.p + ctx->cfg.world, ctx->counts.p, 1, kNcclUint64, ctx->comm, s) != 0)
-      return fail(ctx, ARB_ECUDA, "ncclAllGather failed");
-    std::vector<uint64_t> all(ctx->cfg.world);
-    CK(cudaMemcpyAsync(all.data(), ctx->counts.p, 8 * ctx->cfg.world, cudaMemcpyDeviceToHost, s), "counts d2h");
-    CK(cudaStreamSynchronize(s), "counts sync");
-    for (int r = 0; r < ctx->cfg.rank; ++r) offset += all[r];
+  if (ctx->comm) {
+    std::vector<int64_t> all;
+    const int e = nccl_exchange(ctx, s, rcb, rcb < 0 ? 0 : (int64_t)ctx->n_reports, all);
+    if (e != ARB_OK) { reset_batch(ctx); return ARB_ECUDA; }
+    S.exchanges += 1;
     launches += 1;
+    int64_t peer = 0;
+    for (int r = 0; r < (int)all.size() / 2; ++r) {
+      if (r < ctx->cfg.rank) offset += (uint64_t)all[2 * r + 1];
+      if (r != ctx->cfg.rank && all[2 * r] < 0) peer = all[2 * r];
+    }
+    if (rcb == ARB_OK && peer < 0)
+      rcb = fail(ctx, ARB_EPEER, "another rank failed while replaying its part of the batch; destroy the context");
   }
+  if (rcb != ARB_OK) {
+    reset_batch(ctx);
+    return rcb;
+  }
+  rc = n_vsm > kept_vsm ? ARB_TRUNCATED : ARB_OK;
+  if (rc == ARB_TRUNCATED) ctx->err = "report candidates exceeded report_capacity";
   if (timing) {
     cudaEventRecord(ctx->ev[6], s);
     cudaEventSynchronize(ctx->ev[6]);
@@ -779,6 +872,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   }
   ctx->map.swap(map);
   ctx->carried.swap(plan.carry_out);          // N2: committed with the map table
+  ctx->last_ended.swap(plan.last_ended_out);
   std::swap(ctx->carry_ent, ctx->carry_next);
   ctx->n_carry = n_carry_next;
   ctx->next_index += n;

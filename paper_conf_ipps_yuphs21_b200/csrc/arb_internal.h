@@ -229,7 +229,12 @@ struct CompactParams {
   uint64_t index_base;                    // used when gidx is null
   uint4* out;                             // arb_report output (w0 lo/hi, w1 lo/hi)
   unsigned long long* n_out;              // device count
+  // dedup_first across flushes: persistent set of reported (word, kind) keys, or null
+  unsigned long long* dset; uint64_t dset_mask; unsigned long long* dset_count;
 };
 cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches);
+// grow the cross-flush dedup set: reinsert the n_old slots of `old` into `set` (mask + 1 slots, zeroed)
+cudaError_t launch_dedup_rehash(const unsigned long long* old, uint64_t n_old, unsigned long long* set, uint64_t mask,
+                                cudaStream_t s);
 
 }  // namespace arb

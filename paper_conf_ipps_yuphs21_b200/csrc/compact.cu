@@ -156,6 +156,7 @@ __global__ void __launch_bounds__(kRsThreads) k_rs_scatter(const E* in, E* out, 
 // keep flags: unique (all fields differ from the predecessor), or dedup-first
 // (word, kind differ from the predecessor) for the (word, kind, pos) order.
 __device__ __forceinline__ bool keep_elem(const uint4* a, uint64_t i, int mode) {
+  if (mode == 2) return a[i].w != 0;           // cross-flush dedup: kind 0 marks a dropped element
   if (i == 0) return true;
   uint4 x = a[i], y = a[i - 1];
   if (mode == 0) return x.x != y.x || x.y != y.y || x.z != y.z || x.w != y.w;
@@ -228,6 +229,48 @@ __global__ void __launch_bounds__(kRsThreads) k_keep_write(const uint4* a, uint6
     }
   }
   if (blockIdx.x == nblk - 1 && threadIdx.x == kRsThreads - 1) *n_out = o;
+}
+
+// ARB_F_DEDUP_FIRST across flushes (Z3 over the whole trace, N2): the (word, kind)
+// pairs reported so far live in a persistent open-addressing set of keys
+// (word << 3 | kind) + 1 (0 = empty slot).  Each candidate that is the first of its
+// (word, kind) in this flush is inserted; if the key was already there an earlier
+// flush reported the pair, and the candidate is dropped (kind := 0).
+__global__ void k_dedup_set(uint4* a, uint64_t n, unsigned long long* set, uint64_t mask,
+                            unsigned long long* inserted) {
+  uint32_t ins = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    uint4 x = a[i];
+    const unsigned long long key = ((((unsigned long long)x.y << 32) | x.x) << 3 | (x.w & 7u)) + 1ull;
+    uint64_t h = (key * 0x9E3779B97F4A7C15ull) >> 20;
+    for (;;) {
+      h &= mask;
+      const unsigned long long old = atomicCAS(&set[h], 0ull, key);
+      if (old == 0ull) { ++ins; break; }
+      if (old == key) { a[i].w = 0; break; }
+      ++h;
+    }
+  }
+  for (int d = 16; d; d >>= 1) ins += __shfl_xor_sync(FULL, ins, d);
+  if ((threadIdx.x & 31) == 0 && ins) atomicAdd(inserted, (unsigned long long)ins);
+}
+// rehash the set into a larger table
+__global__ void k_dedup_rehash(const unsigned long long* old, uint64_t n_old, unsigned long long* set, uint64_t mask) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n_old; i += (uint64_t)gridDim.x * blockDim.x) {
+    const unsigned long long key = old[i];
+    if (!key) continue;
+    uint64_t h = (key * 0x9E3779B97F4A7C15ull) >> 20;
+    for (;;) {
+      h &= mask;
+      if (atomicCAS(&set[h], 0ull, key) == 0ull) break;
+      ++h;
+    }
+  }
+}
+cudaError_t launch_dedup_rehash(const unsigned long long* old, uint64_t n_old, unsigned long long* set, uint64_t mask,
+                                cudaStream_t s) {
+  if (n_old) k_dedup_rehash<<<(unsigned)std::min<uint64_t>((n_old + 255) / 256, 4096), 256, 0, s>>>(old, n_old, set, mask);
+  return cudaGetLastError();
 }
 
 template <class E>
@@ -381,6 +424,19 @@ cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches
     n = kept;
     uint4* t = a; a = b; b = t;
     np = 0;
+    if (p.dset && n) {               // drop the (word, kind) pairs earlier flushes reported
+      k_dedup_set<<<(unsigned)std::min<uint64_t>((n + 255) / 256, 4096), 256, 0, s>>>(a, n, p.dset, p.dset_mask,
+                                                                                   p.dset_count);
+      nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
+      k_keep_count<<<nblk, kRsThreads, 0, s>>>(a, n, 2, p.blk);
+      scan_u32(p.blk, nblk, p.blk + nblk, s, launches);
+      k_keep_write<<<nblk, kRsThreads, 0, s>>>(a, n, 2, p.blk, b, 0, 0, nullptr, 0, p.n_out, nblk);
+      *launches += 3;
+      cudaMemcpyAsync(&kept, p.n_out, sizeof(kept), cudaMemcpyDeviceToHost, s);
+      cudaStreamSynchronize(s);
+      n = kept;
+      t = a; a = b; b = t;
+    }
   }
   if (p.pos_bits + kKindBits <= 32) {
     np = add_field_passes(ps, np, 4, p.pos_bits + kKindBits); // record, then kind

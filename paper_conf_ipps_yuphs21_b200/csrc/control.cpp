@@ -43,7 +43,7 @@ struct Emitter {
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
                      FlushPlan& out, bool bo, const std::vector<CarriedInst>* carried_in, bool unified,
-                     uint32_t n_dev) {
+                     uint32_t n_dev, const LastEnded* last_ended_in) {
   const uint32_t n_buckets = (uint32_t)bucket_start.size() - 1;
   out = FlushPlan();
   Emitter em{base_word, n_words, &out, unified};
@@ -163,8 +163,18 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
       case OP_TASK_DEPEND: {                        // Z22: the open task runs after the last
         if (!open || tid == 0 || tid == kSyncAll)   // ended instance of task `tid`
           return fail(ARB_ETRACE, c.pos, "TASK_DEPEND outside a task block or with task id 0 / 0xFFFF");
-        for (uint32_t q = open - 1; q >= 1; --q)
-          if (t_id[q] == tid && t_end[q] != kOpen) { edges.push_back({open, q}); break; }
+        // instances of this flush (and a carried block that ended in it), latest first;
+        // blocks do not nest, so creation order is end order
+        bool found = false;
+        for (uint32_t q = open - 1; q >= 1 && !found; --q) {
+          if (t_end[q] == kBefore) break;              // carried, ended in an earlier flush
+          if (t_id[q] == tid && t_end[q] != kOpen) { edges.push_back({open, q}); found = true; }
+        }
+        if (!found && last_ended_in) {                 // ended in an earlier flush: joined or carried
+          auto it = last_ended_in->find(tid);
+          if (it != last_ended_in->end() && it->second >= 0 && (uint32_t)it->second < nc)
+            edges.push_back({open, (uint32_t)it->second + 1});
+        }
         break;
       }
       default:
@@ -192,6 +202,21 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   std::vector<uint8_t> carry(ninst + 1, 0);
   for (uint32_t q = 1; q <= ninst; ++q)
     if (t_join[q] == UINT64_MAX) { t_join[q] = n_records; carry[q] = 1; }
+  // LastEnded after this flush; carried indices are filled in once carry_out is built
+  // (set_last_ended below), joined instances map to -1
+  std::vector<uint32_t> last_q;                  // instances that ended in this flush, in end order
+  for (uint32_t q = 1; q <= ninst; ++q)
+    if (t_end[q] != kBefore && t_end[q] != kOpen) last_q.push_back(q);
+  auto set_last_ended = [&](const std::vector<uint32_t>& carry_idx) {   // carry_idx[q]: carried-out index or ~0
+    out.last_ended_out.clear();
+    if (last_ended_in)
+      for (const auto& kv : *last_ended_in) {
+        int32_t v = -1;
+        if (kv.second >= 0 && (uint32_t)kv.second < nc && carry_idx[kv.second + 1] != ~0u) v = (int32_t)carry_idx[kv.second + 1];
+        out.last_ended_out[kv.first] = v;
+      }
+    for (uint32_t q : last_q) out.last_ended_out[t_id[q]] = carry_idx[q] != ~0u ? (int32_t)carry_idx[q] : -1;
+  };
   auto wstart = [&](uint32_t q) { return t_end[q] == kBefore ? 0 : t_end[q] + 1; };   // window [wstart, join)
   auto has_window = [&](uint32_t q) { return t_end[q] != kOpen && t_join[q] > wstart(q); };
 
@@ -227,7 +252,10 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   out.carry_in_dense.resize(nc);
   for (uint32_t c = 0; c < nc; ++c) out.carry_in_dense[c] = dense[c + 1];
   out.dense_carry_out.assign(racy.size(), 0xFFFFFFFFu);
-  if (racy.empty()) return;
+  if (racy.empty()) {                         // nothing is carried
+    set_last_ended(std::vector<uint32_t>(ninst + 1, ~0u));
+    return;
+  }
   // insert ranges: the records of each listed block that lie in this flush
   M.ins_cum.push_back(0);
   for (uint32_t q : racy) {
@@ -258,6 +286,11 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
     if (!carry[q]) continue;
     out.dense_carry_out[d] = (uint32_t)out.carry_out.size();
     out.carry_out.push_back(CarriedInst{t_id[q], own[d], t_end[q] == kOpen, {}});
+  }
+  {
+    std::vector<uint32_t> carry_idx(ninst + 1, ~0u);
+    for (size_t d = 0; d < racy.size(); ++d) carry_idx[racy[d]] = out.dense_carry_out[d];
+    set_last_ended(carry_idx);
   }
   for (const auto& e : edges) {              // depend edges between carried-out instances (Z22)
     const uint32_t dc = dense[e.first], dp = dense[e.second];

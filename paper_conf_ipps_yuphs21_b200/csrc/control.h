@@ -13,6 +13,7 @@
 #include <cstdint>
 #include <map>
 #include <string>
+#include <unordered_map>
 #include <vector>
 #include "arb_internal.h"
 #include "arbalest.h"
@@ -42,6 +43,12 @@ struct MirPlanH {
 // deps: carried indices of the (unjoined) instances it depends on (Z22).
 struct CarriedInst { uint32_t task_id; std::vector<RangeRef> own; bool open; std::vector<uint32_t> deps; };
 
+// For every task id, the last instance that ended in an earlier flush (Z22: a
+// TASK_DEPEND(k) binds to the last ended instance of task id k, joined or not):
+// its carried index if that instance is still carried, else -1 (it is joined, so a
+// dependency on it adds no constraint).  Ids that never ended have no entry.
+using LastEnded = std::unordered_map<uint32_t, int32_t>;
+
 struct FlushPlan {
   std::vector<RangeOpH> range_ops;       // in trace order
   std::vector<uint32_t> ops_start;       // per bucket CSR
@@ -50,6 +57,7 @@ struct FlushPlan {
   std::vector<uint32_t> carry_in_dense;  // per carried-in instance: its MIR dense index, or 0xFFFFFFFF
   std::vector<uint32_t> dense_carry_out; // per MIR dense index: its carried-out index, or 0xFFFFFFFF
   std::vector<CarriedInst> carry_out;    // instances still unjoined at the end of this flush
+  LastEnded last_ended_out;              // LastEnded after this flush (committed with carry_out)
   uint64_t range_words = 0, ignored_words = 0, tasks = 0;
   int rc = 0; uint64_t err_pos = 0; std::string err;
 };
@@ -63,10 +71,12 @@ struct FlushPlan {
 // carried_in: instances unjoined at the end of the previous flush (their window
 // in this flush starts at position 0); instances unjoined at the end of this one
 // are returned in out.carry_out instead of being treated as joined (Z19).
+// last_ended_in: the LastEnded table after the previous flush (indices into
+// carried_in); the updated table is returned in out.last_ended_out.
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
                      FlushPlan& out, bool bo = false, const std::vector<CarriedInst>* carried_in = nullptr,
-                     bool unified = false, uint32_t n_dev = 1);
+                     bool unified = false, uint32_t n_dev = 1, const LastEnded* last_ended_in = nullptr);
 // n_dev > 1 (Z24): device bits 6-7 of MAP / UPDATE args select the device; its
 // entries live in the same table under keys offset by device << 56, and range
 // ops are 8-output selectors (Sel8).

@@ -2,11 +2,8 @@
 
 * scaled: the same generator programs at sizes the oracle replays in seconds,
   compared element by element (every report, every shadow byte);
-* full size (BASELINE.json sizes, in the launch configuration bench.py times:
-  device-generated trace, rank-0 shard, quiescent flushes): compared on a random
-  sample of words, for which the oracle replays the filtered trace (control
-  records + the accesses touching the sampled words) in sparse mode.  Word
-  states are independent, so the sampled comparison is exact for those words.
+* full size: the whole traces of configs 3-5 exactly in test_parity_full_gpu.py;
+  here rank 0's config-5 batch (1.0e9 records) in a single flush, exactly.
 """
 import numpy as np
 import pytest
@@ -80,78 +77,33 @@ def test_config5_scaled_shard(orc):
     ctx.close()
 
 
-def _sampled_full_size(orc, prog, lo, hi, n_sample=3000, seed=0, one_flush=False, flags=0):
-    """Run the bench configuration on the device, then compare sampled words.
-    one_flush: the whole batch in a single flush (near the 2^30-record maximum)."""
-    import torch
-    import bench
-    recs, gidx, flushes, (lo2, hi2) = bench.rank_batches(prog, 0, 1, torch.device("cuda", 0))
-    assert (lo2, hi2) == (lo, hi)
-    if one_flush:
-        assert 2 ** 29 < recs.shape[0] <= 2 ** 30
-        flushes = [(0, recs.shape[0])]
-    ctx, got = _gpu_run(prog, lo, hi, flushes=flushes, recs=recs, gidx=gidx, flags=flags)
-    rs = np.random.default_rng(seed)
-    # half of the sample from the words the trace touches most densely (mapped sections)
-    secs = np.array([(a, b) for a, b, _ in prog.sections if b > lo and a < hi], dtype=np.int64)
-    words = set(rs.integers(lo, hi, n_sample // 2).tolist())
-    for _ in range(n_sample // 2):
-        a, b = secs[rs.integers(len(secs))]
-        a, b = max(a, lo), min(b, hi)
-        words.add(int(rs.integers(a, b)))
-    # plus every word the GPU reported on (sampled to keep the filter small)
-    rep_words = sorted({w for w, _, _ in got})
-    words.update(rs.choice(rep_words, min(500, len(rep_words)), replace=False).tolist() if rep_words else [])
-    words = np.array(sorted(words), dtype=np.uint64)
-    del recs, gidx
-    torch.cuda.empty_cache()
-    frec, fgi = prog.filter_host(words=words, cap=30_000_000)
-    exp = orc.replay(frec, lo * 8, (hi - lo) * 8, tracked_words=words, global_index=fgi)
-    assert exp.rc == 0
-    wset = set(words.tolist())
-    assert sorted(t for t in got if t[0] in wset) == exp.triples()
-    gpu_shadow = np.array([ctx.get_shadow(int(w), 1)[0] for w in words], dtype=np.uint8)
-    assert np.array_equal(gpu_shadow, exp.shadow)
-    ctx.close()
-    return exp
-
-
-@pytest.mark.slow
-def test_config5_full_size_sampled(orc):
-    from gen import native
-    from paper_conf_ipps_yuphs21_b200.shard import shard_range
-    prog = native.config5()
-    lo, hi = shard_range(native.C5_BASE_WORD, native.C5_WORDS, 0, 8)
-    exp = _sampled_full_size(orc, prog, lo, hi)
-    assert len(exp.triples()) > 0
-
-
-@pytest.mark.slow
-def test_config3_full_size_sampled(orc):
-    from gen import native
-    prog = native.config3()
-    lo, hi = prog.addr_base // 8, (prog.addr_base + prog.addr_bytes) // 8
-    _sampled_full_size(orc, prog, lo, hi)
-
-
-@pytest.mark.slow
-def test_config4_full_size_sampled(orc):
-    from gen import native
-    prog = native.config4()
-    lo, hi = prog.addr_base // 8, (prog.addr_base + prog.addr_bytes) // 8
-    _sampled_full_size(orc, prog, lo, hi)
-
-
 @pytest.mark.slow
 def test_config5_one_flush_near_max_batch(orc):
-    """Rank 0's whole config-5 batch (1.0e9 records, record positions up to 2^30)
-    in one flush: the largest batch the ABI accepts, sampled against the oracle."""
+    """Rank 0 of 8 of the full config-5 trace (1.0e9 records, record positions up to
+    2^30) in ONE flush -- the largest batch the ABI accepts -- every report and every
+    shadow byte against the address-sharded oracle."""
+    import os
+    import torch
+    import bench
     from gen import native
+    from paper_conf_ipps_yuphs21_b200 import Context, ARB_F_TIMING
     from paper_conf_ipps_yuphs21_b200.shard import shard_range
+    from test_parity_full_gpu import _gpu_batch, _compare_shadow
     prog = native.config5()
     lo, hi = shard_range(native.C5_BASE_WORD, native.C5_WORDS, 0, 8)
-    exp = _sampled_full_size(orc, prog, lo, hi, one_flush=True, seed=3)
-    assert len(exp.triples()) > 0
+    src = bench.BatchSource(prog, lo, hi, torch.device("cuda", 0))
+    recs, gidx, _ = src.make(0, prog.n)
+    assert 2 ** 29 < recs.shape[0] <= 2 ** 30
+    ctx = Context(lo * 8, (hi - lo) * 8, flags=ARB_F_TIMING, report_capacity=1 << 25)
+    got = _gpu_batch(ctx, recs, gidx, [(0, recs.shape[0])])
+    host, gi = recs.cpu().numpy().view(np.uint64), gidx.cpu().numpy().view(np.uint64)
+    del recs, gidx, src
+    torch.cuda.empty_cache()
+    exp = orc.replay(host, lo * 8, (hi - lo) * 8, global_index=gi, threads=os.cpu_count() or 8)
+    assert exp.rc == 0 and exp.reports.size > 0
+    assert np.array_equal(got, exp.reports)
+    _compare_shadow(ctx, lo, hi - lo, exp.shadow)
+    ctx.close()
 
 
 def test_batch_limit():

@@ -498,3 +498,60 @@ def test_devices_large_steps(orc, seed):
                                      loop_max=20000, n_devices=3)
     for bb in (0, 11):
         check(orc, rec, base, span, bucket_bits=bb, flags=2 << 8)
+
+
+def test_depend_binds_to_joined_instance_across_flush(orc):
+    """a TASK_DEPEND(k) after a flush cut binds to the last ended
+    instance of task id k even when that instance was joined in the earlier flush
+    (Z22).  X(1) and Y(1) end, Z(2) depends on Y, SYNC(2) joins Z and, through the
+    dependency, Y; X stays unjoined and is carried.  After the cut W(3) depends on
+    task 1 = Y (joined: no constraint), so W's read of the word X wrote races with X."""
+    from gen.trace import TraceBuilder, MAP
+    base = 0x1000_0000
+    tb = TraceBuilder()
+    tb.wh(base)
+    tb.enter(MAP.TOFROM, base, 64)
+    tb.task_begin(1); tb.wt(base); tb.task_end(1)          # X
+    tb.task_begin(1); tb.wt(base + 8); tb.task_end(1)      # Y
+    tb.task_begin(2); tb.depend(1); tb.rt(base + 8); tb.task_end(2)   # Z after Y
+    tb.sync(2)                                              # joins Z and Y
+    cut = len(tb)
+    tb.task_begin(3); tb.depend(1); tb.rt(base); tb.task_end(3)        # W
+    w_read = len(tb) - 2
+    tb.sync()
+    tb.exit(MAP.TOFROM, base, 64)
+    rec = tb.array()
+    exp = orc.replay(rec, base, 64)
+    assert exp.rc == 0
+    assert (base // 8, w_read, 3) in exp.triples()           # W races with X
+    for cuts in ([], [cut]):
+        rc, got, shadow, _ = run_gpu(rec, base, 64, flush_points=cuts)
+        assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_dedup_first_across_flush_cuts(orc, seed):
+    """ARB_F_DEDUP_FIRST with random flush cuts (also inside task blocks) equals the
+    whole-trace oracle in dedup-first mode (Z3 over the whole trace)."""
+    from gen.fuzz import random_program
+    rec, base, span = random_program(8100 + seed, p_task=0.35, p_depend=0.2, steps=90)
+    exp = orc.replay(rec, base, span, dedup_first=True)
+    if exp.rc != 0:
+        pytest.skip("program rejected by the oracle")
+    for k in (3, 9):
+        rc, got, shadow, _ = run_gpu(rec, base, span, flags=1, flush_points=_cuts(rec, k, seed))
+        assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+def test_dedup_first_set_grows(orc):
+    """Many flushes, many distinct (word, kind) pairs: the persistent set is rehashed."""
+    from gen.configs import config2
+    rec, base, size = config2()
+    exp = orc.replay(rec, base, size, dedup_first=True)
+    assert exp.rc == 0 and len(exp.triples()) > 1000
+    op = (rec[:, 0] >> np.uint64(48)) & np.uint64(0xFF)
+    depth = np.cumsum((op == 12).astype(np.int64) - (op == 13).astype(np.int64))
+    ok = np.nonzero(depth == 0)[0] + 1
+    cuts = sorted(set(ok[np.linspace(0, ok.size - 1, 40).astype(int)].tolist()) - {rec.shape[0]})
+    rc, got, shadow, _ = run_gpu(rec, base, size, flags=1, flush_points=cuts)
+    assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
