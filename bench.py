@@ -428,6 +428,7 @@ def main():
     ap.add_argument("--workload", default="config5")
     ap.add_argument("--scale", type=float, default=1.0)
     ap.add_argument("--batches", type=int, default=8, help="time batches of the trace (quiescent cuts)")
+    ap.add_argument("--max-batches", type=int, default=0, help="profiling: replay only the first K batches")
     ap.add_argument("--e2e-steps", type=int, default=1)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
@@ -460,6 +461,8 @@ def main():
     prog = make_program(args.workload, args.scale)
     lo, hi = rank_range(prog, rank, world)
     batches = time_batches(prog, args.batches if prog.name == "config5" else 1)
+    if args.max_batches:
+        batches = batches[:args.max_batches]
     src = BatchSource(prog, lo, hi, dev)
 
     uid = None

@@ -166,7 +166,7 @@ typedef struct {
   uint64_t kernel_launches;  /* kernels launched by the last flush                         */
   double   ms_sample;        /* address sampling + bucket balancing (inside ms_partition)  */
   uint64_t steps_fast, steps_sort;  /* replay steps by kind                  */
-  double   ms_segsort;       /* GPU: segment-entry sort (inside ms_control)                 */
+  double   ms_segsort;       /* unused (0): the one-sweep partition has no segment sort     */
   double   ms_host_control;  /* host wall time of the Table I / task resolution             */
   uint64_t work_items;       /* replay work items (buckets, word-range parts, hot slices)   */
   uint64_t hot_buckets;      /* buckets replayed as time slices (hot words, K5)             */
@@ -174,6 +174,8 @@ typedef struct {
   uint64_t nccl_ranks;       /* ranks of the context's NCCL communicator (ncclCommCount), 0 =
                                 no communicator                                              */
   uint64_t exchanges;        /* collectives (status / count ncclAllGather) of the last flush */
+  uint64_t partition_retries;/* partition re-runs with exact bucket sizes (a sampled region
+                                overflowed) in the last flush                                */
 } arb_stats;
 
 typedef struct arb_ctx_s* arb_ctx;
@@ -192,7 +194,12 @@ int arb_init(const arb_config* cfg, arb_ctx* out);
  *  global_index NULL: record i of the batch gets the index (records submitted
  *               since arb_init) + i; else an array of n u64 global indices in the
  *               same memory space as ev (sharded mode: the rank sees a subset of
- *               the global trace, in order).  Read only on the report path.
+ *               the global trace, in order).  Read only on the report path: a
+ *               device array is read by the compaction kernel, a host array is
+ *               NOT copied — it is read on the host for the reports only and must
+ *               stay valid until arb_flush returns.  One batch's arrays are all
+ *               host (host submits) or all device (a device submit with an index
+ *               array after a host one is ARB_EINVAL).
  *  stream       cudaStream_t (NULL = legacy default stream).
  * Records of one batch keep their relative order; a batch holds at most 2^30
  * records.  Errors: ARB_EINVAL, ARB_ENOMEM, ARB_ECUDA. */

@@ -32,8 +32,9 @@
  *   unified memory (Z23)                  pinned (brute force vs the value simulator with OV and CV aliased)
  *   depend (Z22)                          pinned (schedule enumeration with dependencies + witness search)
  *   buffer overflow, present-bit form (Z20) pinned (P:279 worked example + brute force vs the
- *                                         value simulator's CV existence); the paper's base-interval
- *                                         comparison (overflow into ANOTHER mapped CV) is not modelled
+ *                                         value simulator's CV existence)
+ *   buffer overflow, base-interval form (Z25) pinned (the P:279 adjacent-CV example + brute force vs
+ *                                         the value simulator's per-entry CV identities)
  */
 #ifndef ARB_ORACLE_H
 #define ARB_ORACLE_H
@@ -53,7 +54,10 @@ enum { ORC_RH = 0, ORC_WH = 1, ORC_RT = 2, ORC_WT = 3,
        ORC_MAP_ENTER = 8, ORC_MAP_EXIT = 9, ORC_UPDATE = 10,
        ORC_TASK_BEGIN = 12, ORC_TASK_END = 13, ORC_SYNC = 14,
        ORC_TASK_DEPEND = 15 /* inside a block: the task depends on the last ended
-                               instance of task id k (N4, reading Z22) */ };
+                               instance of task id k (N4, reading Z22) */,
+       ORC_BASE = 11        /* pointer tag k (task-id field, 1..0xFFFF) now has the base
+                               byte address of this record (LLVM IR base; N1,
+                               reading Z25); no word-ops */ };
 /* map-types (Table I) */
 enum { ORC_TO = 0, ORC_FROM = 1, ORC_TOFROM = 2, ORC_ALLOC = 3,
        ORC_RELEASE = 4, ORC_DELETE = 5 };
@@ -97,6 +101,11 @@ typedef struct {
    * ORC_BO and has no VSM effect (no UUM/USD check, no transition: the access
    * did not touch this word's CV).  0 = off (the 4-bit VSM of P:255-263). */
   int             detect_bo;
+  /* ... and (reading Z25) a target access whose record carries a pointer
+   * tag t != 0 in w1[48,64) with a base defined by an ORC_BASE record is also
+   * reported as ORC_BO when its word and the base lie in different mapping
+   * entries (or the base in none) -- an overflow into ANOTHER variable's CV; the
+   * access then still acts on the CV it reached (VSM effect as usual). */
   /* Unified-memory mode (reading Z23): OV and CV are
    * one storage, so map clauses and target update move no data (refcount
    * bookkeeping and ORC_EMAP only, no word-ops), a write by either side is

@@ -63,6 +63,7 @@ cudaError_t upload(DevBuf<T>& b, const std::vector<T>& v, cudaStream_t s) {
   return cudaMemcpyAsync(b.p, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice, s);
 }
 
+// gidx: device global indices (on_device), or host ones read on the report path only
 struct Submit { const void* ev; uint64_t n; const uint64_t* gidx; int on_device; };
 
 // pinned host buffer (async copies, no staging through pageable memory)
@@ -114,7 +115,6 @@ struct arb_ctx_s {
   DevBuf<uint8_t> hot_P;
   DevBuf<uint4> d_items;
   HostBuf<uint4> h_items;
-  HostBuf<uint32_t> h_weight;
   DevBuf<uint32_t> d_bin_map, d_hist, d_cut, d_cutscr;
   DevBuf<uint64_t> d_bucket_start;
   int n_sms = 148;
@@ -122,13 +122,14 @@ struct arb_ctx_s {
   std::vector<Submit> subs;
   uint64_t pending = 0;
   bool any_gidx = false, any_nogidx = false;
+  bool host_gidx = false, dev_gidx = false;   // where this batch's global indices live
   DevBuf<uint4> staging;
   DevBuf<uint64_t> gidx_staging;
-  DevBuf<uint2> part_ev;
-  DevBuf<uint2> seg_a, seg_b;                 // partition entries, sort ping-pong
-  DevBuf<uint4> segs;                         // replay form
-  DevBuf<uint32_t> seg_first;
-  uint64_t seg_cap = 0;
+  DevBuf<uint2> part_ev;                      // bucket regions of the partition output
+  DevBuf<uint64_t> d_reg_start, d_btotal;     // region start, exact events per bucket
+  DevBuf<uint32_t> d_reg_cap;                 // region capacity
+  HostBuf<uint64_t> h_btotal;
+  DevBuf<unsigned long long> ring;            // look-back status ring
   DevBuf<CtlRec> ctl;
   DevBuf<uint4> cand, cand_tmp, reports;
   DevBuf<uint32_t> blk;
@@ -156,7 +157,9 @@ struct arb_ctx_s {
   MapTable map;
   uint64_t next_index = 0;
   uint64_t n_reports = 0;      // exact count of the last flush
-  uint64_t n_stored = 0;       // reports held in `reports`
+  uint64_t n_stored = 0;       // reports held in `reports` (or h_reports)
+  bool reports_on_host = false;             // host global indices: translated reports in h_reports
+  HostBuf<uint4> h_reports;
   bool flushed = false;
   std::string err;
   arb_stats stats{};
@@ -259,7 +262,7 @@ extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
   if (e == cudaSuccess) e = ctx->h_stats.ensure(1);
   if (e == cudaSuccess) e = ctx->h_nb.ensure(1);
   if (e == cudaSuccess) e = ctx->h_bstart.ensure(kMaxBuckets + 1);
-  if (e == cudaSuccess) e = ctx->h_weight.ensure(kMaxBuckets);
+  if (e == cudaSuccess) e = ctx->h_btotal.ensure(kMaxBuckets);
   if (e == cudaSuccess) e = cudaDeviceSynchronize();
   if (e != cudaSuccess) { arb_destroy(ctx); return ARB_ENOMEM; }
   if (cfg->nccl_unique_id) {
@@ -289,7 +292,8 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   if (!ctx) return ARB_OK;
   if (ctx->comm && ctx->nccl_destroy) ctx->nccl_destroy(ctx->comm);
   if (ctx->shadow) cudaFree(ctx->shadow);
-  ctx->staging.release(); ctx->gidx_staging.release(); ctx->part_ev.release(); ctx->seg_a.release(); ctx->seg_b.release(); ctx->segs.release(); ctx->seg_first.release();
+  ctx->staging.release(); ctx->gidx_staging.release(); ctx->part_ev.release(); ctx->d_reg_start.release();
+  ctx->d_btotal.release(); ctx->d_reg_cap.release(); ctx->h_btotal.release(); ctx->ring.release();
   ctx->ctl.release(); ctx->cand.release(); ctx->cand_tmp.release(); ctx->reports.release(); ctx->blk.release();
   ctx->ops_start.release(); ctx->ops.release(); ctx->dstats.release(); ctx->dcount.release();
   ctx->m_ins_lo.release(); ctx->m_ins_cum.release(); ctx->m_qry_lo.release(); ctx->m_qry_cum.release();
@@ -297,13 +301,13 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   ctx->m_own_start.release(); ctx->m_win_start.release(); ctx->m_own.release(); ctx->m_win.release();
   ctx->m_rr.release(); ctx->hkeys.release(); ctx->hvals.release(); ctx->counts.release();
   ctx->carry_ent.release(); ctx->carry_next.release(); ctx->dset.release(); ctx->dset_cnt.release(); ctx->m_cmap.release(); ctx->m_co_of.release();
-  ctx->d_bin_map.release(); ctx->d_items.release(); ctx->h_items.release(); ctx->h_weight.release();
+  ctx->d_bin_map.release(); ctx->d_items.release(); ctx->h_items.release();
   ctx->d_slice_items.release(); ctx->h_slice_items.release(); ctx->d_hot.release(); ctx->h_hot.release();
   ctx->d_hot_off.release(); ctx->h_hot_off.release(); ctx->hot_F.release(); ctx->hot_P.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_cut.release();
   for (auto& e : ctx->ev) if (e) cudaEventDestroy(e);
   if (ctx->aux) cudaStreamDestroy(ctx->aux);
   ctx->h_stats.release(); ctx->h_nb.release(); ctx->h_ops_start.release(); ctx->h_bstart.release();
-  ctx->h_ctl.release(); ctx->h_ops.release();
+  ctx->h_ctl.release(); ctx->h_ops.release(); ctx->h_reports.release();
   if (ctx->nccl_lib) dlclose(ctx->nccl_lib);
   delete ctx;
   return ARB_OK;
@@ -335,15 +339,23 @@ extern "C" int arb_submit_events(arb_ctx ctx, const arb_event* ev, uint64_t n, c
     if (e != cudaSuccess) return fail(ctx, ARB_ENOMEM, "staging buffer");
     e = cudaMemcpyAsync(ctx->staging.p + off, ev, n * sizeof(arb_event), cudaMemcpyHostToDevice, s);
     if (e != cudaSuccess) return cuda_fail(ctx, e, "copy host records");
-    if (global_index) {
+    const uint64_t* host_gi = nullptr;
+    if (global_index && ctx->dev_gidx) {
+      // the batch's other indices are on the device: copy these next to them
       if ((e = ctx->gidx_staging.ensure_keep(off + n, off)) != cudaSuccess) return fail(ctx, ARB_ENOMEM, "gidx staging");
       e = cudaMemcpyAsync(ctx->gidx_staging.p + off, global_index, n * 8, cudaMemcpyHostToDevice, s);
       if (e != cudaSuccess) return cuda_fail(ctx, e, "copy host global_index");
+    } else if (global_index) {
+      host_gi = global_index;      // read on the report path only (no H2D copy, §8(b))
+      ctx->host_gidx = true;
     }
-    e = cudaStreamSynchronize(s);  // the caller may free the host buffer on return
+    e = cudaStreamSynchronize(s);  // the caller may free the host records on return
     if (e != cudaSuccess) return cuda_fail(ctx, e, "submit sync");
-    ctx->subs.push_back(Submit{nullptr, n, nullptr, 0});
+    ctx->subs.push_back(Submit{nullptr, n, host_gi, 0});
   } else {
+    if (global_index && ctx->host_gidx)
+      return fail(ctx, ARB_EINVAL, "global_index of one batch: host arrays (host submits) or device arrays, not both");
+    if (global_index) ctx->dev_gidx = true;
     ctx->subs.push_back(Submit{ev, n, global_index, 1});
   }
   if (global_index) ctx->any_gidx = true; else ctx->any_nogidx = true;
@@ -355,6 +367,7 @@ static void reset_batch(arb_ctx ctx) {
   ctx->subs.clear();
   ctx->pending = 0;
   ctx->any_gidx = ctx->any_nogidx = false;
+  ctx->host_gidx = ctx->dev_gidx = false;
 }
 
 // Replay work items, heaviest first.  A bucket whose range ops cover many words
@@ -484,6 +497,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   S.reports = 0; std::memset(S.reports_by_kind, 0, sizeof(S.reports_by_kind)); S.ignored_words = 0;
   S.ms_partition = S.ms_control = S.ms_replay = S.ms_mir = S.ms_reports = S.ms_total = 0;
   S.ms_segsort = S.ms_host_control = 0;
+  S.partition_retries = 0;
   S.buckets = ctx->n_buckets; S.bucket_bits = ctx->bucket_bits; S.max_bucket_events = 0;
 
   // Phase A (validation): decode + partition and control resolution.  Nothing
@@ -496,7 +510,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   const uint64_t index_base = ctx->next_index;
   const bool balanced = ctx->bucket_bits == 0;
   DevStats& hst = *ctx->h_stats.p;
-  std::vector<double> bucket_events;      // estimated events per bucket (sampled)
+  std::vector<double> bucket_events;      // events per bucket (exact, from the partition)
   MapTable map;
   FlushPlan plan;
   std::chrono::steady_clock::time_point t_host0, t_host1;
@@ -512,104 +526,128 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
       uint64_t off = 0;
       CK(cudaStreamSynchronize(s), "staging sync");
       CK(ctx->staging.ensure_keep(n, n), "staging");
-      if (ctx->any_gidx) CK(ctx->gidx_staging.ensure_keep(n, n), "gidx staging");
+      if (ctx->any_gidx && !ctx->host_gidx) CK(ctx->gidx_staging.ensure_keep(n, n), "gidx staging");
       for (const Submit& sb : ctx->subs) {
         if (sb.on_device) {
           CK(cudaMemcpyAsync(ctx->staging.p + off, sb.ev, sb.n * 16, cudaMemcpyDeviceToDevice, s), "gather");
-          if (sb.gidx) CK(cudaMemcpyAsync(ctx->gidx_staging.p + off, sb.gidx, sb.n * 8, cudaMemcpyDeviceToDevice, s), "gather gidx");
+          if (sb.gidx && !ctx->host_gidx)
+            CK(cudaMemcpyAsync(ctx->gidx_staging.p + off, sb.gidx, sb.n * 8, cudaMemcpyDeviceToDevice, s), "gather gidx");
         }
         off += sb.n;
       }
       ev = ctx->staging.p;
-      gidx = ctx->any_gidx ? ctx->gidx_staging.p : nullptr;
+      gidx = ctx->any_gidx && !ctx->host_gidx ? ctx->gidx_staging.p : nullptr;
     }
   }
   if (timing) cudaEventRecord(ctx->ev[0], s);
-  // ---- bucket balancing on a sampled address histogram (all on the device) ----
-  if (balanced) {
+  // ---- sampled address histogram: bucket balancing and region sizes (on the device) ----
+  const uint32_t n_chunks = (uint32_t)((n + kChunkRecords - 1) / kChunkRecords);
+  const uint32_t n_tiles = (n_chunks + kPartWarps - 1) / kPartWarps;
+  const uint64_t ev_cap = 2 * n + 2 * (uint64_t)kMaxBuckets + 64;    // events: <= 2 per record
+  const uint64_t sample_stride = std::max<uint64_t>(1, n / kSampleCap);
+  {
     CK(ctx->d_hist.ensure(ctx->n_bins), "alloc hist");
     CK(cudaMemsetAsync(ctx->d_hist.p, 0, ctx->n_bins * sizeof(uint32_t), s), "hist clear");
     SampleParams sp{};
-    sp.ev = ev; sp.n = n; sp.stride = std::max<uint64_t>(1, n / kSampleCap);
+    sp.ev = ev; sp.n = n; sp.stride = sample_stride;
     sp.base_word = ctx->base_word; sp.n_words = ctx->n_words; sp.coarse_bits = ctx->coarse_bits;
     sp.hist = ctx->d_hist.p;
     const uint64_t n_samples = n ? (n + sp.stride - 1) / sp.stride : 0;
     CK(launch_sample(sp, n_samples, s), "k_sample");
     launches += n_samples ? 1 : 0;
-    // cut balanced buckets; the histogram becomes the bin map in place
+  }
+  if (ctx->d_bucket_start.cap == 0) {       // the read-back below copies every slot
     CK(ctx->d_bucket_start.ensure(kMaxBuckets + 1), "alloc buckets");
+    CK(cudaMemsetAsync(ctx->d_bucket_start.p, 0, (kMaxBuckets + 1) * 8, s), "clear buckets");
+  }
+  if (ctx->d_cut.cap == 0) {
     CK(ctx->d_cut.ensure(2 * kMaxBuckets + 2), "alloc cut scratch");
+    CK(cudaMemsetAsync(ctx->d_cut.p, 0, (2 * kMaxBuckets + 2) * 4, s), "clear cut scratch");
+  }
+  CK(ctx->d_reg_start.ensure(kMaxBuckets), "alloc regions");
+  CK(ctx->d_reg_cap.ensure(kMaxBuckets), "alloc regions");
+  CK(ctx->d_btotal.ensure(kMaxBuckets), "alloc bucket totals");
+  if (balanced) {
+    // cut balanced buckets; the histogram becomes the bin map in place
     CK(ctx->d_cutscr.ensure(2 * ((ctx->n_bins + 1023) / 1024) + 4 + ctx->n_bins), "alloc cut scratch");
     CK(launch_cut(ctx->d_hist.p, ctx->n_bins, ctx->coarse_bits, ctx->n_words, kMaxBuckets, ctx->d_bucket_start.p,
                   ctx->d_cut.p, ctx->d_cut.p + kMaxBuckets, ctx->d_cut.p + 2 * kMaxBuckets, ctx->d_cutscr.p,
                   s, &launches), "k_cut");
+    CK(launch_regions(ctx->d_cut.p, ctx->d_cut.p + 2 * kMaxBuckets, 0, (double)sample_stride, ev_cap,
+                      ctx->d_reg_start.p, ctx->d_reg_cap.p, s), "k_regions");
     // the bucket count and starts come back with the partition's counters (one sync)
     CK(cudaMemcpyAsync(ctx->h_nb.p, ctx->d_cut.p + 2 * kMaxBuckets, 4, cudaMemcpyDeviceToHost, s), "nb d2h");
     CK(cudaMemcpyAsync(ctx->h_bstart.p, ctx->d_bucket_start.p, (kMaxBuckets + 1) * 8, cudaMemcpyDeviceToHost, s),
        "buckets d2h");
-    CK(cudaMemcpyAsync(ctx->h_weight.p, ctx->d_cut.p, kMaxBuckets * 4, cudaMemcpyDeviceToHost, s), "weights d2h");
-  } else if (ctx->d_bin_map.cap == 0) {
-    CK(upload(ctx->d_bin_map, ctx->bin_map, s), "upload bin map");
-    CK(upload(ctx->d_bucket_start, ctx->bucket_start, s), "upload bucket starts");
+  } else {
+    if (ctx->d_bin_map.cap == 0) {
+      CK(upload(ctx->d_bin_map, ctx->bin_map, s), "upload bin map");
+      CK(upload(ctx->d_bucket_start, ctx->bucket_start, s), "upload bucket starts");
+    }
+    // fixed buckets: coarse bins are the buckets, so the histogram is the weights
+    CK(launch_regions(ctx->d_hist.p, nullptr, (uint32_t)ctx->bin_map.size(), (double)sample_stride, ev_cap,
+                      ctx->d_reg_start.p, ctx->d_reg_cap.p, s), "k_regions");
   }
+  launches += 1;
   if (!balanced) ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;   // fixed buckets
   if (timing) cudaEventRecord(ctx->ev[7], s);
-  // ---- A1/A3a: decode + partition ------------------------------------------
-  const uint32_t n_chunks = (uint32_t)((n + kChunkRecords - 1) / kChunkRecords);
-  CK(ctx->part_ev.ensure((size_t)std::max<uint32_t>(n_chunks, 1) * kChunkCap), "alloc part_ev");
-  if (ctx->seg_cap < (uint64_t)n_chunks * 2 + 4096) ctx->seg_cap = (uint64_t)n_chunks * 2 + 4096;
-  CK(ctx->seg_a.ensure(std::max<uint64_t>(ctx->seg_cap, 1)), "alloc segments");
+  // ---- A1 + A3: decode + one-sweep partition into contiguous bucket regions ---------
+  CK(ctx->part_ev.ensure(ev_cap), "alloc part_ev");
+  CK(ctx->ring.ensure((size_t)kRingTiles * kMaxBuckets), "alloc look-back ring");
   PartParams pp{};
-  for (int attempt = 0; attempt < 2; ++attempt) {
+  for (int attempt = 0; attempt < 3; ++attempt) {
     CK(cudaMemsetAsync(ctx->dstats.p, 0, sizeof(DevStats), s), "stats init");
     CK(cudaMemsetAsync(&ctx->dstats.p->err_pos, 0xFF, sizeof(unsigned long long), s), "stats init");
+    CK(cudaMemsetAsync(ctx->ring.p, 0, (size_t)kRingTiles * kMaxBuckets * 8, s), "ring clear");
+    CK(cudaMemsetAsync(ctx->d_btotal.p, 0, kMaxBuckets * 8, s), "totals clear");
     pp.ev = ev; pp.n = n; pp.base_word = ctx->base_word; pp.n_words = ctx->n_words;
     pp.coarse_bits = ctx->coarse_bits; pp.bin_map = balanced ? ctx->d_hist.p : ctx->d_bin_map.p;
     pp.bucket_bits = ctx->bucket_bits; pp.n_buckets = balanced ? (uint32_t)kMaxBuckets : ctx->n_buckets;
-    pp.n_chunks = n_chunks;
+    pp.n_chunks = n_chunks; pp.n_tiles = n_tiles;
     pp.n_dev = 1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u);
-    pp.part_ev = ctx->part_ev.p; pp.seg_out = ctx->seg_a.p; pp.seg_cap = ctx->seg_cap;
+    pp.part_ev = ctx->part_ev.p; pp.reg_start = ctx->d_reg_start.p; pp.reg_cap = ctx->d_reg_cap.p;
+    pp.ring = ctx->ring.p; pp.bucket_total = ctx->d_btotal.p;
     pp.ctl = ctx->ctl.p; pp.ctl_cap = ctx->ctl_cap;
     pp.st = ctx->dstats.p;
     CK(launch_partition(pp, s), "k_partition");
     launches += n_chunks ? 1 : 0;
     CK(cudaMemcpyAsync(&hst, ctx->dstats.p, sizeof(hst), cudaMemcpyDeviceToHost, s), "stats d2h");
+    CK(cudaMemcpyAsync(ctx->h_btotal.p, ctx->d_btotal.p, kMaxBuckets * 8, cudaMemcpyDeviceToHost, s), "totals d2h");
     CK(cudaStreamSynchronize(s), "partition sync");
-    if (hst.n_ctl <= ctx->ctl_cap && hst.n_segs <= ctx->seg_cap) break;
-    if (hst.n_ctl > ctx->ctl_cap) ctx->ctl_cap = hst.n_ctl + hst.n_ctl / 2;
-    if (hst.n_segs > ctx->seg_cap) ctx->seg_cap = hst.n_segs + hst.n_segs / 4;
-    CK(ctx->ctl.ensure(ctx->ctl_cap), "grow ctl");
-    CK(ctx->seg_a.ensure(ctx->seg_cap), "grow segments");
+    if (hst.n_ctl <= ctx->ctl_cap && !hst.overflow) break;
+    if (hst.n_ctl > ctx->ctl_cap) {
+      ctx->ctl_cap = hst.n_ctl + hst.n_ctl / 2;
+      CK(ctx->ctl.ensure(ctx->ctl_cap), "grow ctl");
+    }
+    if (hst.overflow) {
+      // a bucket outgrew its sampled region: size every region by the exact counts
+      std::vector<uint64_t> rs(kMaxBuckets);
+      std::vector<uint32_t> rc(kMaxBuckets);
+      uint64_t at = 0;
+      for (int b = 0; b < kMaxBuckets; ++b) {
+        rs[b] = at;
+        rc[b] = (uint32_t)((ctx->h_btotal.p[b] + 1) & ~1ull);
+        at += rc[b];
+      }
+      CK(cudaMemcpyAsync(ctx->d_reg_start.p, rs.data(), kMaxBuckets * 8, cudaMemcpyHostToDevice, s), "regions");
+      CK(cudaMemcpyAsync(ctx->d_reg_cap.p, rc.data(), kMaxBuckets * 4, cudaMemcpyHostToDevice, s), "regions");
+      S.partition_retries += 1;
+    }
   }
   if (timing) cudaEventRecord(ctx->ev[1], s);
   if (hst.err_pos != ~0ull)
     return fail(ctx, ARB_ETRACE, "malformed record at batch position " + std::to_string(hst.err_pos));
+  if (hst.overflow) return fail(ctx, ARB_ENOMEM, "partition regions overflowed twice");
   if (balanced) {
     const uint32_t nb = *ctx->h_nb.p;
     ctx->bucket_start.assign(ctx->h_bstart.p, ctx->h_bstart.p + nb + 1);
-    const double stride = (double)std::max<uint64_t>(1, n / kSampleCap);
-    bucket_events.resize(nb);
-    for (uint32_t b = 0; b < nb; ++b) bucket_events[b] = ctx->h_weight.p[b] * stride;
   }
   ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;
+  bucket_events.assign(ctx->h_btotal.p, ctx->h_btotal.p + ctx->n_buckets);   // exact, from the look-back
   S.buckets = ctx->n_buckets;
   S.access_words = hst.access_words;
   S.control_records = hst.n_ctl;
-
-  // ---- A3b: segment entries sorted by (bucket, chunk) — on the GPU while the
-  // host resolves the control records ------------------------------------------------
-  {
-    const uint64_t ns = hst.n_segs;
-    CK(ctx->seg_b.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
-    CK(ctx->segs.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
-    CK(ctx->seg_first.ensure(ctx->n_buckets + 1), "alloc seg_first");
-    CK(ctx->blk.ensure((ns + 4095) / 4096 * 2049 + 4096), "alloc blk");   // 2048-bin digit counters + scan scratch
-    int cb = 1;
-    while (cb < 22 && ((uint64_t)n_chunks >> cb)) ++cb;
-    CK(launch_sort_segments(ctx->seg_a.p, ctx->seg_b.p, ns, cb, ctx->n_buckets, ctx->blk.p, ctx->seg_first.p,
-                            ctx->segs.p, s, &launches), "sort segments");
-    if (timing) cudaEventRecord(ctx->ev[8], s);
-  }
+  if (timing) cudaEventRecord(ctx->ev[8], s);
   t_host0 = std::chrono::steady_clock::now();
 
   // ---- A2: control resolution on the host -------------------------------------
@@ -684,7 +722,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
 
   // ---- A3b/A4/A5: replay ---------------------------------------------------------
   ReplayParams rp{};
-  rp.part_ev = ctx->part_ev.p; rp.segs = ctx->segs.p; rp.seg_first = ctx->seg_first.p;
+  rp.part_ev = ctx->part_ev.p; rp.reg_start = ctx->d_reg_start.p; rp.bucket_count = ctx->d_btotal.p;
   rp.n_buckets = ctx->n_buckets; rp.bucket_bits = ctx->bucket_bits; rp.n_words = ctx->n_words;
   rp.bucket_start = ctx->d_bucket_start.p;
   rp.items = ctx->d_items.p; rp.n_items = (uint32_t)ctx->items.size();
@@ -794,7 +832,8 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   int pb = 1; while (pb < 32 && (n ? (n - 1) >> pb : 0)) ++pb;
   cp.word_bits = wb; cp.pos_bits = pb;
   cp.dedup_first = (ctx->cfg.flags & ARB_F_DEDUP_FIRST) ? 1 : 0;
-  cp.gidx = gidx; cp.index_base = index_base;
+  // host global indices: positions now, translated on the host below
+  cp.gidx = ctx->host_gidx ? nullptr : gidx; cp.index_base = ctx->host_gidx ? 0 : index_base;
   cp.out = ctx->reports.p; cp.n_out = ctx->dcount.p;
   if (cp.dedup_first) {
     // the persistent (word, kind) set of earlier flushes: keep its load <= 1/2
@@ -824,6 +863,22 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   CK(cudaStreamSynchronize(s), "compact sync");
   const uint64_t n_out = cnt4[0];
   ctx->n_stored = n_out;
+  ctx->reports_on_host = ctx->host_gidx;
+  if (ctx->host_gidx && n_out) {
+    // the report path reads the host global indices: position -> global_index[position]
+    CK(ctx->h_reports.ensure(n_out), "pinned reports");
+    CK(cudaMemcpyAsync(ctx->h_reports.p, ctx->reports.p, n_out * 16, cudaMemcpyDeviceToHost, s), "reports d2h");
+    CK(cudaStreamSynchronize(s), "reports sync");
+    std::vector<uint64_t> off(ctx->subs.size() + 1, 0);
+    for (size_t k = 0; k < ctx->subs.size(); ++k) off[k + 1] = off[k] + ctx->subs[k].n;
+    for (uint64_t i = 0; i < n_out; ++i) {
+      uint4& r = ctx->h_reports.p[i];
+      const uint64_t pos = (uint64_t)r.z | ((uint64_t)r.w << 32);
+      const size_t k = (size_t)(std::upper_bound(off.begin(), off.end(), pos) - off.begin()) - 1;
+      const uint64_t g = ctx->subs[k].gidx ? ctx->subs[k].gidx[pos - off[k]] : ctx->next_index + pos;
+      r.z = (uint32_t)g; r.w = (uint32_t)(g >> 32);
+    }
+  }
   for (int k = 1; k < 4; ++k) S.reports_by_kind[k] = cnt4[k];
   S.reports_bo = cnt4[ARB_BO];
   ctx->dset_n += dset_new;
@@ -895,8 +950,14 @@ extern "C" int arb_get_reports(arb_ctx ctx, arb_report* out, uint64_t cap, uint6
   uint64_t k = std::min(cap, ctx->n_stored);
   if (k) {
     if (!out) return fail(ctx, ARB_EINVAL, "null output");
-    cudaError_t e = cudaMemcpy(out, ctx->reports.p, k * sizeof(arb_report),
-                               out_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost);
+    cudaError_t e;
+    if (ctx->reports_on_host) {
+      if (out_on_device) e = cudaMemcpy(out, ctx->h_reports.p, k * sizeof(arb_report), cudaMemcpyHostToDevice);
+      else { std::memcpy(out, ctx->h_reports.p, k * sizeof(arb_report)); e = cudaSuccess; }
+    } else {
+      e = cudaMemcpy(out, ctx->reports.p, k * sizeof(arb_report),
+                     out_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost);
+    }
     if (e != cudaSuccess) return cuda_fail(ctx, e, "get_reports");
   }
   if (n_written) *n_written = k;

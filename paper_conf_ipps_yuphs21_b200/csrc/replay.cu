@@ -1,9 +1,10 @@
 // replay.cu — A3b + A4 + A5: per-address replay of each bucket.
 //
 // One CTA per address bucket at a time (persistent; buckets in largest-first
-// order).  The bucket's events are the segments of its sorted segment entries
-// (chunk order = trace order); the CTA gathers them step by step through a
-// staged window of entries (cp.async, double-buffered), applies the resolved range ops
+// order).  The bucket's events are one contiguous array in trace order (the
+// partition's bucket region); the CTA streams it step by step into shared memory
+// with one TMA bulk copy per step (cp.async.bulk, double-buffered on two
+// mbarriers: the next step arrives while this one runs), applies the resolved range ops
 // (Table I transfers / allocate / release; target update P:121) to
 // the bucket's shadow at their trace positions, and processes the events in
 // steps of <= 1024 that never straddle a range op:
@@ -33,22 +34,23 @@ constexpr int RT = kReplayThreads;           // threads per CTA (>= 256)
 constexpr int RI = kReplayItems;             // events per thread per step
 constexpr int STEP = RT * RI;                // 2048 events per step
 static_assert(RT >= 256 && STEP <= 4096, "sort_pass digit loop and u16 offsets");
-constexpr int kWin = 2 * RT;                 // segment descriptors staged per step
 constexpr int kHSlots = 4096;                // hash slots (load <= 1/2)
+constexpr int kDSlots = 2 * kHSlots;         // direct-step window (words), same bytes as the hash
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
 constexpr uint32_t kWordMask = 0x3FFFFFFFu;
 constexpr int kZSlots = 2048;                // summary-step hash slots (<= 1024 writes per step)
 static_assert(kZSlots * 12 <= kHSlots * 8 && kZSlots >= 2 * STEP, "summary hash fits the hash area");
 
 struct ReplaySmem {
-  uint2 ev[2][STEP];              // double-buffered step events {key, pos} (cp.async)
+  uint2 ev[2][STEP + 2];          // double-buffered step events {key, pos} (bulk copies; an odd
+                                  //   first event lands at index 1 so the source stays 16-B aligned)
+  uint64_t bar[2];                // their mbarriers
   union {
     struct { uint32_t keyA[STEP], posA[STEP], keyB[STEP], posB[STEP]; uint16_t hist[RT / 32][256]; } s;
     struct { uint2 slot[kHSlots]; } h;      // fast step: written words {word, pos << 2 | op}
+    struct { uint32_t w[kDSlots]; } d;      // direct step: word - anchor -> {step index << 4 | write code}
     struct { uint32_t key[kZSlots], lastw[kZSlots], anyw[kZSlots]; } z;  // hot-slice summary step (K5)
   } u;
-  uint32_t wstart[kWin];          // staged segment list window: global event index
-  uint32_t wcum[kWin + 1];        //   and bucket-relative first event of each segment
   uint32_t pref[256];             // radix digit scratch
   uint32_t red[RT / 32], red2[RT / 32], wscan[RT / 32];
   uint32_t wcnt[RT / 32], wev[RT / 32];
@@ -56,11 +58,12 @@ struct ReplaySmem {
   uint32_t part_lo, part_hi;      // the work item's word range inside the bucket
   bool partial;                   //   (partial: not the whole bucket)
   uint32_t mode;                  // kItem* of the work item
+  uint32_t skip_direct;           // steps left before the direct step is tried again
   uint8_t* shrel;                 // state of bucket-relative word w: shrel[w]
   uint16_t* fsum;                 // summary slice: composed transition of word w: fsum[w]
   uint32_t slice, n_slices;       // hot bucket slice (kItemSlice / kItemSummary)
-  uint32_t seg0, cum0, n_segs, n_events, wsc, nwin;
-  uint64_t bucket_base;
+  uint32_t n_events, evoff[2];
+  uint64_t bucket_base, ev_base;
 };
 
 // ---- block-level helpers ----------------------------------------------------
@@ -283,14 +286,16 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
     if (op[j] & 1u) {
       any_w = true;
       uint32_t h = hslot(word[j]);
+      bool won = false;
       for (;;) {
         const uint32_t old = atomicCAS(&hs[h].x, kEmpty, word[j]);
-        if (old == kEmpty) break;
+        if (old == kEmpty) { won = true; break; }
         if (old == word[j]) { multi = true; break; }        // a second write of the word
         h = (h + 1) & (kHSlots - 1);
       }
       slot[j] = h;
-      hs[h].y = MD ? ((pos[j] << 3) | (((devs >> (2 * j)) & 3u) << 1) | (op[j] >> 1)) : ((pos[j] << 2) | op[j]);
+      if (won)   // the slot's owner; a second writer only flags the fallback
+        hs[h].y = MD ? ((pos[j] << 3) | (((devs >> (2 * j)) & 3u) << 1) | (op[j] >> 1)) : ((pos[j] << 2) | op[j]);
     }
   }
   any_w = __syncthreads_or(any_w);
@@ -335,6 +340,91 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
     for (int j = 0; j < RI; ++j)
       if (op[j] & 1u) hs[slot[j]] = make_uint2(kEmpty, kEmpty);
   }
+  // the caller's next barrier orders this reset before the next step's inserts
+  return true;
+}
+
+// ---- direct step: at most one write per word, every word near the step's first ------------
+// Same computation as step_fast, with the hash replaced by a window of kDSlots
+// words centred on the step's first word: slot = word - anchor, no hashing and
+// no probing.  A write claims its slot with one CAS ({step index << 4 | code});
+// a read's state-before is the initial state, or the image of the slot's write
+// when that write comes earlier in the step.  Returns false (nothing written,
+// table clean) if a word has two writes or an event lies outside the window;
+// *oow reports the latter (the caller then prefers the hash step for a while).
+template <bool PARTIAL, bool BO, bool UM, bool MD>
+__device__ __forceinline__ bool step_direct(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m,
+                                            bool* oow_out) {
+  uint32_t idx[RI], word[RI], pos[RI], op[RI], s_pre[RI];
+  uint32_t bom = 0, devs = 0;
+  bool bad = false, oow = false;
+  const uint8_t* sh = S.shrel;
+  uint32_t* tab = S.u.d.w;
+  const uint32_t anchor = (ev[0].x & kWordMask) - (uint32_t)(kDSlots / 2);
+  uint32_t plo = 0, pw = 0;
+  if (PARTIAL) { plo = S.part_lo; pw = S.part_hi - S.part_lo; }
+#pragma unroll
+  for (int j = 0; j < RI; ++j) {   // shadow loads first: their latency overlaps the table work
+    const uint32_t i = threadIdx.x + j * RT;
+    word[j] = 0; pos[j] = 0; op[j] = 4; s_pre[j] = 0; idx[j] = 0;
+    if (i < m) {
+      const uint2 e = ev[i];
+      word[j] = e.x & kWordMask; op[j] = e.x >> 30; pos[j] = MD ? (e.y & kMdPos) : e.y;
+      if (MD) devs |= (e.y >> 30) << (2 * j);
+      if (!PARTIAL || word[j] - plo < pw) s_pre[j] = __ldcg(sh + word[j]);
+      else op[j] = 4;                                       // another work item's word
+      if (BO && (op[j] & 2u) && !(s_pre[j] & kCVp)) { bom |= 1u << j; op[j] = 4; }
+      idx[j] = word[j] - anchor;
+      if (op[j] < 4 && idx[j] >= (uint32_t)kDSlots) { oow = true; op[j] |= 8u; }   // outside the window
+    }
+  }
+  bool any_w = false;
+  uint32_t won = 0;
+#pragma unroll
+  for (int j = 0; j < RI; ++j) {
+    if ((op[j] & 9u) == 1u) {      // an in-window write (WH = 1, WT = 3)
+      any_w = true;
+      const uint32_t i = threadIdx.x + j * RT;
+      const uint32_t code = MD ? ((((devs >> (2 * j)) & 3u) << 1) | (op[j] >> 1)) : op[j];
+      if (atomicCAS(&tab[idx[j]], kEmpty, (i << 4) | code) == kEmpty) won |= 1u << j;
+      else bad = true;                                      // a second write of the word
+    }
+  }
+  any_w = __syncthreads_or(any_w);
+  if (any_w && __syncthreads_or(bad || oow)) {
+#pragma unroll
+    for (int j = 0; j < RI; ++j)
+      if ((won >> j) & 1u) tab[idx[j]] = kEmpty;
+    *oow_out = __syncthreads_or(oow);
+    return false;
+  }
+  uint32_t fk[RI];
+#pragma unroll
+  for (int j = 0; j < RI; ++j) {
+    const uint32_t o = op[j] & 7u;
+    const uint32_t s0 = s_pre[j] & (MD ? 255u : 15u);
+    uint32_t before = s0;
+    if (o == OP_RH || o == OP_RT) {
+      if (any_w) {
+        const uint32_t t = tab[idx[j]];
+        if (t != kEmpty && (t >> 4) < threadIdx.x + j * RT)
+          before = MD ? md_write(t & 7u, s0) : UM ? 15u : vsm_write_op(t & 3u, s0);
+      }
+    } else if (o & 1u) {
+      __stcg(const_cast<uint8_t*>(sh) + word[j],
+             (uint8_t)(MD ? md_write((o >> 1) | (((devs >> (2 * j)) & 3u) << 1), s0)
+                       : UM ? 15u : vsm_write_op(o, s0) | (BO ? (s_pre[j] & kCVp) : 0u)));
+    }
+    fk[j] = ((bom >> j) & 1u) ? 4u : MD ? md_classify(o, (devs >> (2 * j)) & 3u, before) : classify_bits(o, before);
+  }
+  emit_faults(p, fk, word, pos, S.bucket_base);
+  if (any_w) {
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < RI; ++j)
+      if ((won >> j) & 1u) tab[idx[j]] = kEmpty;
+  }
+  *oow_out = false;
   // the caller's next barrier orders this reset before the next step's inserts
   return true;
 }
@@ -641,15 +731,9 @@ __device__ void step_summary(ReplaySmem& S, const uint2* ev, uint32_t m) {
   __syncthreads();
 }
 
-// Position of event e of the bucket (one thread).
-__device__ uint32_t event_pos(const ReplaySmem& S, const ReplayParams& p, uint32_t e) {
-  uint32_t lo = 0, z = S.n_segs;
-  while (z - lo > 1) {
-    const uint32_t mid = (lo + z) >> 1;
-    if (p.segs[S.seg0 + mid].w - S.cum0 <= e) lo = mid; else z = mid;
-  }
-  const uint4 sg = p.segs[S.seg0 + lo];
-  return p.part_ev[(uint64_t)sg.x * kChunkCap + (sg.z & 0xFFFFu) + (e - (sg.w - S.cum0))].y;
+// Position of event e of the bucket.
+__device__ __forceinline__ uint32_t event_pos(const ReplaySmem& S, const ReplayParams& p, uint32_t e) {
+  return p.part_ev[S.ev_base + e].y;
 }
 // first op of the bucket (ops [a, z), trace order) at or after position q
 __device__ uint32_t ops_lower_bound(const ReplayParams& p, uint32_t a, uint32_t z, uint32_t q) {
@@ -686,131 +770,20 @@ cudaError_t launch_carry(const uint4* hot, uint32_t n_hot, uint32_t max_span, co
   return cudaGetLastError();
 }
 
-// ---- the bucket's segments -------------------------------------------------------------
-// The sorted entries of bucket b are p.segs[f0, f1) in chunk order (= trace
-// order); entry i covers bucket-relative events [segs[i].w - segs[f0].w, + len)
-// stored at part_ev[chunk * kChunkCap + start].
-__device__ void bucket_setup(ReplaySmem& S, const ReplayParams& p, uint32_t b) {
+// ---- the bucket's events: stream [e0, e0 + m) into buffer k ------------------------------
+// One thread issues the bulk copy; the events sit at S.ev[k] + S.evoff[k].  Regions
+// start at even slots, so the source is 16-B aligned when rounded down to an even
+// event; the copy may read one event past the step (inside the allocation).
+__device__ __forceinline__ uint32_t issue_step(ReplaySmem& S, const ReplayParams& p, uint32_t e0, uint32_t total,
+                                               uint32_t k) {
+  const uint32_t m = min((uint32_t)STEP, total - e0);
   if (threadIdx.x == 0) {
-    const uint32_t f0 = p.seg_first[b], f1 = p.seg_first[b + 1];
-    S.seg0 = f0; S.n_segs = f1 - f0;
-    S.cum0 = 0; S.n_events = 0;
-    if (f1 > f0) {
-      const uint4 first = p.segs[f0], last = p.segs[f1 - 1];
-      S.cum0 = first.w;
-      S.n_events = last.w + (last.z >> 16) - first.w;
-    }
-    S.wsc = 0; S.nwin = 0; S.wcum[0] = 1;      // empty window: forces a load
+    const uint32_t odd = e0 & 1u;
+    const uint32_t bytes = ((m + odd + 1u) & ~1u) * 8u;
+    S.evoff[k] = odd;
+    mbar_arrive_tx(&S.bar[k], bytes);
+    bulk_g2s(S.ev[k], p.part_ev + S.ev_base + (e0 - odd), bytes, &S.bar[k]);
   }
-  __syncthreads();
-}
-
-// Make the staged window of segment descriptors contain event e0 (reloads
-// about every kWin segments; sequential progress needs no search).
-__device__ void ensure_window(ReplaySmem& S, const ReplayParams& p, uint32_t e0, uint32_t& hint) {
-  if (e0 >= S.wcum[0] && e0 < S.wcum[S.nwin]) return;
-  hint = 0;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    uint32_t a;
-    if (S.nwin && e0 == S.wcum[S.nwin]) {
-      a = S.wsc + S.nwin;                       // the window's successor
-    } else {                                    // last segment starting at or before e0
-      uint32_t lo = 0, z = S.n_segs;
-      while (z - lo > 1) {
-        const uint32_t mid = (lo + z) >> 1;
-        if (p.segs[S.seg0 + mid].w - S.cum0 <= e0) lo = mid; else z = mid;
-      }
-      a = lo;
-    }
-    S.wsc = a;
-    S.nwin = min((uint32_t)kWin, S.n_segs - a);
-  }
-  __syncthreads();
-  const uint32_t sc = S.wsc, nwin = S.nwin;
-  const uint4* segs = p.segs + S.seg0 + sc;
-  for (uint32_t k = threadIdx.x; k < nwin; k += RT) {
-    const uint4 e = segs[k];
-    S.wstart[k] = e.x * (uint32_t)kChunkCap + (e.z & 0xFFFFu);
-    S.wcum[k] = e.w - S.cum0;
-  }
-  if (threadIdx.x == 0) S.wcum[nwin] = sc + nwin < S.n_segs ? segs[nwin].w - S.cum0 : S.n_events;
-  __syncthreads();
-}
-
-// Issue cp.async copies of events [e0, e0 + m) of the bucket into dst; the
-// window must contain e0.  Returns m (<= STEP, clipped to the window).
-// `hint` (per thread, block-uniform) is a window segment index with
-// wcum[hint] <= e0; it is advanced to the last segment gathered.
-__device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t e0, uint32_t total, uint2* dst,
-                                 uint32_t& hint) {
-  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const uint32_t nwin = S.nwin;
-  const uint32_t m = min(min((uint32_t)STEP, total - e0), S.wcum[nwin] - e0);
-  // Warp w gathers the slice [e0 + 32*RI*w, +32*RI) of the step.  Segment j holds
-  // event e iff wcum[j] <= e < wcum[j+1]; every warp counts, from the hint, the
-  // segments starting at or before its slice start and before the step's last
-  // event (ballots, no barrier), then each lane walks forward to the segment of
-  // each of its events (segments are usually longer than the slice).
-  const uint32_t s0 = e0 + warp * (32 * RI), last = e0 + m - 1;
-  const uint32_t base0 = hint & ~31u;
-  uint32_t c0 = 0, c1 = 0;
-  for (uint32_t base = base0; base < nwin; base += 32) {
-    const uint32_t j = base + lane;
-    const uint32_t w = j < nwin ? S.wcum[j] : 0xFFFFFFFFu;
-    c0 += __popc(__ballot_sync(FULL, w <= s0));
-    const uint32_t b1 = __ballot_sync(FULL, w <= last);
-    c1 += __popc(b1);
-    if (b1 != FULL) break;
-  }
-  hint = base0 + c1 - 1;                 // segment of the step's last event
-  if (s0 < e0 + m) {
-    uint32_t seg = base0 + c0 - 1, seg_end = S.wcum[seg + 1];
-    // event e of segment seg sits at part_ev[wstart[seg] + e - wcum[seg]] = bp[e]
-    int64_t bp = (int64_t)S.wstart[seg] - (int64_t)S.wcum[seg];
-    const uint32_t s_end = min(s0 + 32 * RI, e0 + m);
-    if (s_end <= seg_end) {
-      // the whole slice lies in one segment (warp-uniform; the common case):
-      // a contiguous copy, 16 B per lane when both sides are 16-B aligned
-      const uint2* src = p.part_ev + (bp + s0);
-      uint2* d = dst + (s0 - e0);
-      const uint32_t cnt = s_end - s0;
-      if (cnt == 32 * RI && ((reinterpret_cast<uintptr_t>(src) & 15u) == 0)) {
-#pragma unroll
-        for (int k = 0; k < RI / 2; ++k) cp_async16(d + 2 * (lane + 32 * k), src + 2 * (lane + 32 * k));
-      } else {
-#pragma unroll
-        for (int k = 0; k < RI; ++k)
-          if (lane + 32 * k < cnt) cp_async8(d + lane + 32 * k, src + lane + 32 * k);
-      }
-      cp_async_commit();
-      return m;
-    }
-    uint2* d = dst + (s0 - e0) + lane;
-    if (seg + 2 <= nwin && s_end <= S.wcum[seg + 2]) {
-      // two segments: select the base per event
-      const int64_t bp1 = (int64_t)S.wstart[seg + 1] - (int64_t)seg_end;
-#pragma unroll
-      for (int k = 0; k < RI; ++k) {
-        const uint32_t e = s0 + k * 32 + lane;
-        if (e < s_end) cp_async8(d + k * 32, p.part_ev + ((e < seg_end ? bp : bp1) + e));
-      }
-      cp_async_commit();
-      return m;
-    }
-#pragma unroll
-    for (int k = 0; k < RI; ++k) {
-      const uint32_t e = s0 + k * 32 + lane;
-      if (e < e0 + m) {
-        if (e >= seg_end) {
-          do { ++seg; seg_end = S.wcum[seg + 1]; } while (e >= seg_end);
-          bp = (int64_t)S.wstart[seg] - (int64_t)S.wcum[seg];
-        }
-        cp_async8(d + k * 32, p.part_ev + (bp + e));
-      }
-    }
-  }
-  cp_async_commit();
   return m;
 }
 
@@ -822,6 +795,9 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
   ReplaySmem& S = *reinterpret_cast<ReplaySmem*>(smem_raw);
   const uint32_t tid = threadIdx.x;
   hash_clear(S);
+  if (tid == 0) { mbar_init(&S.bar[0], 1); mbar_init(&S.bar[1], 1); }
+  fence_mbar_init();
+  uint32_t bph = 0;                    // parity of each buffer's mbarrier (bit k)
   for (;;) {
     if (tid == 0) {
       const unsigned long long w = atomicAdd(&p.st->work, 1ull);
@@ -845,8 +821,11 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       S.op_end = p.ops_start[b + 1];
       S.bucket_base = p.bucket_start[b];
       S.shrel = p.shadow + S.bucket_base;
+      S.ev_base = p.reg_start[b];
+      S.n_events = (uint32_t)p.bucket_count[b];
+      S.skip_direct = 0;
     }
-    bucket_setup(S, p, b);
+    __syncthreads();
     uint32_t first = 0, total = S.n_events;
     if (mode >= kItemSlice) {
       // hot bucket slice k of n: events [k E / n, (k+1) E / n) and the range ops
@@ -878,23 +857,14 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
     }
     if (tid == 0) S.next_op = S.op_cur < S.op_end ? p.ops[S.op_cur].pos : 0xFFFFFFFFu;
     __syncthreads();
-    uint32_t e0 = first, cur = 0, m_cur = 0, hint = 0;
-    if (e0 < total) {
-      ensure_window(S, p, e0, hint);
-      m_cur = issue_gather(S, p, e0, total, S.ev[0], hint);
-    }
+    uint32_t e0 = first, cur = 0, m_cur = 0;
+    if (e0 < total) m_cur = issue_step(S, p, e0, total, 0);
     while (e0 < total) {
-      cp_async_wait_all();
-      __syncthreads();
-      const uint2* ev = S.ev[cur];
+      mbar_wait(&S.bar[cur], (bph >> cur) & 1u);
+      bph ^= 1u << cur;
+      __syncthreads();                 // the other buffer's readers are done: it may be refilled
+      const uint2* ev = S.ev[cur] + S.evoff[cur];
       const uint32_t m = m_cur;
-      // ---- prefetch the next step's events (assumes the step is not cut) ---------
-      const uint32_t nxt = e0 + m;
-      uint32_t m_nxt = 0;
-      if (nxt < total) {
-        ensure_window(S, p, nxt, hint);
-        m_nxt = issue_gather(S, p, nxt, total, S.ev[cur ^ 1], hint);
-      }
       // ---- range ops before the first event, then cut at the next one -------------
       constexpr uint32_t pm = MD ? kMdPos : 0xFFFFFFFFu;   // MD: strip the device bits (Z24)
       apply_ops_before<BO, MD>(S, p, ev[0].y & pm);
@@ -904,26 +874,35 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         for (uint32_t e = tid; e < m; e += RT) cnt += (ev[e].y & pm) < S.next_op;
         cut = block_sum(cnt, S.red);
       }
+      // ---- prefetch the next step (from the cut) ---------------------------------------
+      const uint32_t nxt = e0 + cut;
+      const uint32_t m_nxt = nxt < total ? issue_step(S, p, nxt, total, cur ^ 1u) : 0u;
       if (mode == kItemSummary) {
         step_summary<UM>(S, ev, cut);
       } else {
-        const bool fast = S.partial ? step_fast_partial<BO, UM, MD>(S, p, ev, cut)
-                                    : step_fast<false, BO, UM, MD>(S, p, ev, cut);
-        if (!fast) step_sort<BO, UM, MD>(S, p, ev, cut);
-        if (tid == 0) atomicAdd(fast ? &p.st->steps_fast : &p.st->steps_sort, 1ull);
+        bool fast = false, oow = false;
+        const uint32_t skip = S.skip_direct;
+        if (!skip) {
+          fast = S.partial ? step_direct<true, BO, UM, MD>(S, p, ev, cut, &oow)
+                           : step_direct<false, BO, UM, MD>(S, p, ev, cut, &oow);
+        }
+        if (!fast) {
+          if (!skip && !oow) {           // two writes of a word: straight to the sort step
+            step_sort<BO, UM, MD>(S, p, ev, cut);
+          } else {
+            fast = S.partial ? step_fast_partial<BO, UM, MD>(S, p, ev, cut)
+                             : step_fast<false, BO, UM, MD>(S, p, ev, cut);
+            if (!fast) step_sort<BO, UM, MD>(S, p, ev, cut);
+          }
+        }
+        if (tid == 0) {
+          S.skip_direct = oow ? 8u : (skip ? skip - 1u : 0u);
+          atomicAdd(fast ? &p.st->steps_fast : &p.st->steps_sort, 1ull);
+        }
       }
       e0 += cut;
-      if (cut == m) {
-        cur ^= 1;
-        m_cur = m_nxt;
-      } else {
-        // the prefetch started at e0_old + m: drain it and gather from e0
-        cp_async_wait_all();
-        __syncthreads();
-        hint = 0;
-        ensure_window(S, p, e0, hint);
-        m_cur = issue_gather(S, p, e0, total, S.ev[cur], hint);
-      }
+      cur ^= 1u;
+      m_cur = m_nxt;
     }
     // the ops after the last event (a slice replay's private states are not kept)
     if (mode != kItemSlice) apply_ops_before<BO, MD>(S, p, 0xFFFFFFFFu);

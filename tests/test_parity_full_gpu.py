@@ -56,7 +56,9 @@ def _gpu_batch(ctx, recs, gidx, flushes):
         rc, n, _ = ctx.flush()
         assert rc == 0, ctx.last_error()
         out.append(_reports_np(ctx.get_reports(n)))
-    return np.concatenate(out) if out else _reports_np(np.zeros((0, 2), np.uint64))
+    got = np.concatenate(out) if out else _reports_np(np.zeros((0, 2), np.uint64))
+    # each flush's list is canonical; the batch's is the canonical order of their union
+    return got[np.lexsort((got["kind"], got["record"], got["word"]))]
 
 
 def _compare_shadow(ctx, lo, n, expected, chunk=1 << 30):

@@ -555,3 +555,29 @@ def test_dedup_first_set_grows(orc):
     cuts = sorted(set(ok[np.linspace(0, ok.size - 1, 40).astype(int)].tolist()) - {rec.shape[0]})
     rc, got, shadow, _ = run_gpu(rec, base, size, flags=1, flush_points=cuts)
     assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+@pytest.mark.parametrize("split", [1, 3])
+def test_host_submit_host_global_index(orc, split):
+    """Host records with host global indices (a shard of config 5): the indices are not
+    copied to the device; the report path translates positions on the host (§8(b))."""
+    from gen import native
+    from paper_conf_ipps_yuphs21_b200 import Context, reports_to_triples
+    from paper_conf_ipps_yuphs21_b200.shard import shard_range
+    prog = native.config5(total_records=2_000_000, groups=24, stale_rate=10)
+    lo, hi = shard_range(native.C5_BASE_WORD, native.C5_WORDS, 2, 8)
+    rec, gi = prog.filter_host(word_lo=lo, word_hi=hi)
+    exp = orc.replay(rec, lo * 8, (hi - lo) * 8, global_index=gi)
+    assert exp.rc == 0 and len(exp.triples()) > 0
+    ctx = Context(lo * 8, (hi - lo) * 8)
+    cuts = np.linspace(0, rec.shape[0], split + 1).astype(int)
+    for a, b in zip(cuts[:-1], cuts[1:]):          # several host submits, one flush
+        ctx.submit_events(np.ascontiguousarray(rec[a:b]), global_index=np.ascontiguousarray(gi[a:b]))
+    rc, n, _ = ctx.flush()
+    assert rc == 0
+    assert reports_to_triples(ctx.get_reports(n)) == exp.triples()
+    import torch
+    dev_out = torch.zeros((max(n, 1), 2), dtype=torch.int64, device="cuda")
+    ctx.get_reports(n, out=dev_out)                 # device output of host-translated reports
+    assert reports_to_triples(dev_out[:n].cpu().numpy().view(np.uint64)) == exp.triples()
+    ctx.close()

@@ -22,6 +22,7 @@ from __future__ import annotations
 BOT = 0  # undefined content
 
 RH, WH, RT, WT, MAP_ENTER, MAP_EXIT, UPDATE = 0, 1, 2, 3, 8, 9, 10
+BASE = 11                           # pointer tag -> base address (reading Z25)
 TASK_BEGIN, TASK_END, SYNC = 12, 13, 14
 TO, FROM, TOFROM, ALLOC, RELEASE, DELETE = 0, 1, 2, 3, 4, 5
 ALWAYS = 0x10                       # map-type modifier bit (N4, reading Z21)
@@ -56,6 +57,8 @@ class ValueSim:
         self.next_id = 1
         self.present: list[list[int]] = self.presents[0]  # [lo, hi, refcount] byte intervals
         self.issues: set[tuple[int, int, int]] = set()
+        self.base: dict[int, int] = {}    # pointer tag -> base byte address (Z25)
+        self.tag = 0                      # tag of the current target access
 
     # -- per-word primitive operations ---------------------------------------
     def _write(self, side, w):
@@ -70,10 +73,22 @@ class ValueSim:
         if lat is None or got != lat:
             self.issues.add((w, idx, UUM if got == BOT else USD))
 
+    def _entry_of(self, byte):
+        for ent in self.present:
+            if ent[0] <= byte < ent[1]:
+                return ent
+        return None
+
     def word_op(self, name, w, idx):
         if self.bo and name in ("RT", "WT") and w not in self.alive:
             self.issues.add((w, idx, BO))
             return
+        if self.bo and name in ("RT", "WT") and self.tag in self.base:
+            # the access must land in the CV allocated for its pointer's
+            # base; reaching another variable's CV is an overflow (the access still
+            # reads / writes the CV it reached)
+            if self._entry_of(self.base[self.tag]) is not self._entry_of(8 * w):
+                self.issues.add((w, idx, BO))
         if name == "RH":
             self._read(self.ov, w, idx)
         elif name == "RT":
@@ -111,7 +126,7 @@ class ValueSim:
                 raise MapError("partial overlap")
         return hit
 
-    def record(self, op, addr, length, arg, idx):
+    def record(self, op, addr, length, arg, idx, tag=0):
         if self.devices > 1:              # Z24: the device of the record
             d = arg if op in (RT, WT) else (arg >> 6 if op in (MAP_ENTER, MAP_EXIT, UPDATE) else 0)
             arg = arg & 0x3F if op in (MAP_ENTER, MAP_EXIT, UPDATE) else arg
@@ -121,8 +136,12 @@ class ValueSim:
         arg &= ~(ALWAYS | PRESENT)
         if op in (RH, WH, RT, WT):
             name = {RH: "RH", WH: "WH", RT: "RT", WT: "WT"}[op]
+            self.tag = tag if op in (RT, WT) else 0
             for w in self.words(addr, length):
                 self.word_op(name, w, idx)
+            self.tag = 0
+        elif op == BASE:
+            self.base[tag] = addr
         elif op == MAP_ENTER:
             ent = self._lookup(addr, addr + length)
             if ent is None and present:
@@ -168,7 +187,7 @@ class ValueSim:
             w0 = int(w0)
             w1 = int(w1)
             self.record((w0 >> 48) & 0xFF, w0 & ((1 << 48) - 1), w1 & ((1 << 48) - 1),
-                        w0 >> 56, idx)
+                        w0 >> 56, idx, w1 >> 48)
         return self.issues
 
     def state_bits(self, w):

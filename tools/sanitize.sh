@@ -8,7 +8,9 @@ for tool in memcheck racecheck synccheck initcheck; do
   mode=""
   [ "$tool" = "racecheck" ] && mode="quick"
   [ "$tool" = "initcheck" ] && mode="quick"
-  timeout 1500 compute-sanitizer --tool $tool --print-limit 50 --error-exitcode 9 \
+  extra=""
+  [ "$tool" = "synccheck" ] && extra="--num-cuda-barriers 65536"
+  timeout 1500 compute-sanitizer --tool $tool $extra --print-limit 50 --error-exitcode 9 \
       --kernel-name kns=3arb python tools/sanitize_run.py $mode > "$out/$tool.log" 2>&1
   echo "$tool rc=$?" | tee -a "$out/summary.txt"
   tail -3 "$out/$tool.log" >> "$out/summary.txt"
