@@ -15,12 +15,15 @@ from .trace import MAP, OP, UPD, SYNC_ALL, TraceBuilder, encode_np
 
 def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: int = 60,
                    base: int = 0x10000, loop_max: int = 48, p_task: float = 0.15, p_always: float = 0.0,
-                   p_depend: float = 0.0, n_devices: int = 1):
+                   p_depend: float = 0.0, n_devices: int = 1, p_tag: float = 0.0):
     """p_always > 0: map clauses carry the `always` modifier with that probability;
     p_depend > 0: a new nowait block depends on an earlier task with that
     probability; n_devices > 1: target accesses and map / update clauses on a
     random accelerator (the device in the access arg and in bits 6-7 of a
-    map / update arg) (the RNG streams of the defaults are unchanged)."""
+    map / update arg); p_tag > 0: pointer tags (ARB_BASE records, reading Z25): tag
+    i + 1 has array i's base, target accesses carry a tag with that probability
+    (mostly their own array's, sometimes another's), and tags are sometimes
+    redefined (the RNG streams of the defaults are unchanged)."""
     rs = np.random.default_rng(seed)
     tb = TraceBuilder()
     arrays = [base + i * array_words * 8 * 2 for i in range(n_arrays)]   # gap between arrays
@@ -29,6 +32,9 @@ def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: i
 
     def pdev():
         return int(rs.integers(n_devices)) if n_devices > 1 else 0
+    if p_tag:
+        for i in range(n_arrays):
+            tb._add(OP.BASE, arrays[i], 0, task=i + 1)
     in_task = 0
     next_task = 1
     unjoined = []
@@ -57,9 +63,15 @@ def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: i
         addr = addr[addr + size <= arrays[i] + array_words * 8 + 8]
         if addr.size:
             arg = pdev() if op in (OP.RT, OP.WT) else 0
-            tb.add_array(encode_np(op, addr, size, arg=arg))
+            tag = 0
+            if p_tag and op in (OP.RT, OP.WT) and rs.random() < p_tag:
+                tag = i + 1 if rs.random() < 0.7 else int(rs.integers(1, n_arrays + 2))
+            tb.add_array(encode_np(op, addr, size, arg=arg, task=tag))
 
     for _ in range(steps):
+        if p_tag and rs.random() < 0.04:         # a pointer re-based into some array
+            j = int(rs.integers(n_arrays))
+            tb._add(OP.BASE, arrays[j] + 8 * int(rs.integers(array_words)), 0, task=int(rs.integers(1, n_arrays + 2)))
         r = rs.random()
         if r < 0.35:
             loop(int(rs.choice([OP.RH, OP.WH, OP.RT, OP.WT])))

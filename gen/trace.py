@@ -14,6 +14,7 @@ class OP:
     MAP_ENTER, MAP_EXIT, UPDATE = 8, 9, 10
     TASK_BEGIN, TASK_END, SYNC = 12, 13, 14
     TASK_DEPEND = 15       # inside a block: depends on the last ended instance of task id k (Z22)
+    BASE = 11              # pointer tag k (task field) -> base address (N1, Z25)
 
 
 class MAP:

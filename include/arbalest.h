@@ -43,9 +43,14 @@ enum arb_op {
   ARB_UPDATE = 10,                                      /* target update to/from       */
   ARB_TASK_BEGIN = 12, ARB_TASK_END = 13,               /* nowait region block (Z8)     */
   ARB_SYNC = 14,                                        /* taskwait: joins task k, 0xFFFF = all */
-  ARB_TASK_DEPEND = 15  /* inside a block: the task depends on the last ended instance of task k
+  ARB_TASK_DEPEND = 15, /* inside a block: the task depends on the last ended instance of task k
                            (a `depend` clause; Z22): their ops are ordered, and
                            joining the dependant joins the instance it depends on            */
+  ARB_BASE = 11         /* pointer tag k (w1 [48,64), 1..0xFFFF) now has the base byte address
+                           w0 [0,48) -- the base LLVM IR gives a pointer (Z25).  With
+                           ARB_F_BO a target access whose w1 [48,64) holds tag k is also BO
+                           when its word lies in another mapping entry than that base (an
+                           overflow into another variable's CV); no word-ops          */
 };
 /* map-types (Table I) */
 enum arb_map { ARB_TO = 0, ARB_FROM = 1, ARB_TOFROM = 2, ARB_ALLOC = 3,
@@ -128,7 +133,10 @@ enum arb_status {
                                    word carries a 5th state bit "has a CV" (set by allocate,
                                    cleared by release); a target access (RT/WT) to a word
                                    without a CV is reported as ARB_BO and has no VSM effect.
-                                   Hot buckets are then replayed whole (no time slices).  */
+                                   Hot buckets are then replayed whole (no time slices).
+                                   Target accesses may carry a pointer tag (ARB_BASE, Z25):
+                                   an access outside its base's entry is BO as well, and
+                                   still acts on the CV it reached                         */
 
 typedef struct {
   uint64_t addr_base;        /* tracked OV byte range [addr_base, addr_base+addr_bytes);   */

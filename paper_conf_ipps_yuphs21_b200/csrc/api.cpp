@@ -126,6 +126,9 @@ struct arb_ctx_s {
   DevBuf<uint4> staging;
   DevBuf<uint64_t> gidx_staging;
   DevBuf<uint2> part_ev;                      // bucket regions of the partition output
+  TagBases tags;                              // N1 (Z25): pointer tag bases (committed per flush)
+  DevBuf<uint32_t> d_tag_first;
+  DevBuf<TagSeg> d_tag_segs;
   DevBuf<uint64_t> d_reg_start, d_btotal;     // region start, exact events per bucket
   DevBuf<uint32_t> d_reg_cap;                 // region capacity
   HostBuf<uint64_t> h_btotal;
@@ -294,6 +297,7 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   if (ctx->shadow) cudaFree(ctx->shadow);
   ctx->staging.release(); ctx->gidx_staging.release(); ctx->part_ev.release(); ctx->d_reg_start.release();
   ctx->d_btotal.release(); ctx->d_reg_cap.release(); ctx->h_btotal.release(); ctx->ring.release();
+  ctx->d_tag_first.release(); ctx->d_tag_segs.release();
   ctx->ctl.release(); ctx->cand.release(); ctx->cand_tmp.release(); ctx->reports.release(); ctx->blk.release();
   ctx->ops_start.release(); ctx->ops.release(); ctx->dstats.release(); ctx->dcount.release();
   ctx->m_ins_lo.release(); ctx->m_ins_cum.release(); ctx->m_qry_lo.release(); ctx->m_qry_cum.release();
@@ -629,6 +633,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
         rc[b] = (uint32_t)((ctx->h_btotal.p[b] + 1) & ~1ull);
         at += rc[b];
       }
+      if (at > ctx->part_ev.cap) CK(ctx->part_ev.ensure(at + 64), "grow part_ev");
       CK(cudaMemcpyAsync(ctx->d_reg_start.p, rs.data(), kMaxBuckets * 8, cudaMemcpyHostToDevice, s), "regions");
       CK(cudaMemcpyAsync(ctx->d_reg_cap.p, rc.data(), kMaxBuckets * 4, cudaMemcpyHostToDevice, s), "regions");
       S.partition_retries += 1;
@@ -664,7 +669,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   map = ctx->map;
   resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_start, map, plan,
                   (ctx->cfg.flags & ARB_F_BO) != 0, &ctx->carried, (ctx->cfg.flags & ARB_F_UNIFIED) != 0,
-                  1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u), &ctx->last_ended);
+                  1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u), &ctx->last_ended, &ctx->tags);
   if (plan.rc != 0)
     return fail(ctx, plan.rc, plan.err + " (batch position " + std::to_string(plan.err_pos) + ")");
   return ARB_OK;
@@ -817,6 +822,28 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
       n_carry_next = c;
     }
   }
+  // ---- N1 (Z25): accesses through a tagged pointer outside its base's entry ------------
+  if (!plan.tag_first.empty() && n) {
+    CK(upload(ctx->d_tag_first, plan.tag_first, s), "tag table");
+    CK(upload(ctx->d_tag_segs, plan.tag_segs, s), "tag segments");
+    for (int attempt = 0; attempt < 2; ++attempt) {
+      const uint64_t used = kept_vsm + n_mir;
+      CK(cudaMemsetAsync(&ctx->dstats.p->n_bo_cand, 0, sizeof(unsigned long long), s), "bo count");
+      CK(launch_bo_tags(ev, n, ctx->base_word, ctx->n_words, ctx->d_tag_first.p, ctx->d_tag_segs.p,
+                        ctx->cand.p + used, ctx->cand.cap - used, &ctx->dstats.p->n_bo_cand, s), "k_bo_tags");
+      launches += 1;
+      unsigned long long c = 0;
+      CK(cudaMemcpyAsync(&c, &ctx->dstats.p->n_bo_cand, sizeof(c), cudaMemcpyDeviceToHost, s), "bo d2h");
+      CK(cudaStreamSynchronize(s), "bo sync");
+      if (used + c <= ctx->cand.cap) { n_mir += c; break; }
+      DevBuf<uint4> bigger;                    // read-only kernel: grow and run it again
+      CK(bigger.ensure(used + c), "grow candidates");
+      if (used) CK(cudaMemcpyAsync(bigger.p, ctx->cand.p, used * 16, cudaMemcpyDeviceToDevice, s), "copy cand");
+      CK(cudaStreamSynchronize(s), "copy sync");
+      ctx->cand.release();
+      ctx->cand = bigger;
+    }
+  }
   if (timing) cudaEventRecord(ctx->ev[4], s);
 
   // ---- canonical order + unique ---------------------------------------------------
@@ -928,6 +955,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   ctx->map.swap(map);
   ctx->carried.swap(plan.carry_out);          // N2: committed with the map table
   ctx->last_ended.swap(plan.last_ended_out);
+  ctx->tags.swap(plan.tags_out);
   std::swap(ctx->carry_ent, ctx->carry_next);
   ctx->n_carry = n_carry_next;
   ctx->next_index += n;

@@ -12,7 +12,8 @@ constexpr uint64_t kMask48 = (1ull << 48) - 1;
 enum Op : uint32_t { OP_RH = 0, OP_WH = 1, OP_RT = 2, OP_WT = 3,
                      OP_MAP_ENTER = 8, OP_MAP_EXIT = 9, OP_UPDATE = 10,
                      OP_TASK_BEGIN = 12, OP_TASK_END = 13, OP_SYNC = 14,
-                     OP_TASK_DEPEND = 15 };   // N4, Z22
+                     OP_TASK_DEPEND = 15,     // N4, Z22
+                     OP_BASE = 11 };          // pointer tag -> base address (N1, Z25)
 enum MapType : uint32_t { MT_TO = 0, MT_FROM = 1, MT_TOFROM = 2, MT_ALLOC = 3,
                           MT_RELEASE = 4, MT_DELETE = 5 };
 constexpr uint32_t kMapAlways = 0x10;   // `always` map-type modifier bit (N4, Z21)
@@ -104,7 +105,8 @@ struct DevStats {
   unsigned long long steps_fast, steps_sort;
   unsigned long long overflow;        // a bucket received more events than its region holds
   unsigned long long n_carry_out;     // N2: access summaries of instances carried into the next flush
-  unsigned long long pad[3];
+  unsigned long long n_bo_cand;       // N1 (Z25): base-tag overflow candidates
+  unsigned long long pad[2];
 };
 
 // control record extracted by the partition kernel
@@ -116,6 +118,10 @@ struct BucketOp {
   uint32_t sel;      // transition function (selector form)
   uint64_t lo, hi;   // word range [lo, hi) relative to the tracked base
 };
+
+// N1 (Z25): from batch position `pos` on, the mapping entry holding pointer tag t's
+// base spans the absolute words [lo, hi) (lo == hi: the base is not mapped)
+struct TagSeg { uint32_t pos; uint32_t pad; uint64_t lo, hi; };
 
 // a range op for the MIR join (absolute relative words, instance of its block)
 struct RangeRef { uint64_t lo, hi; uint32_t pos; uint32_t inst; };
@@ -216,6 +222,12 @@ cudaError_t launch_carry(const uint4* hot, uint32_t n_hot, uint32_t max_span, co
                          cudaStream_t s);
 cudaError_t launch_mir(const MirParams& p, uint64_t n_ins_pos, uint64_t n_qry_pos, uint64_t n_rr_words,
                        cudaStream_t s, int* launches);
+// N1 (Z25): target accesses through pointer tag t (w1[48,64)) whose word lies outside
+// the entry of t's base at that position -> BO candidates {word lo, word hi, pos, 4}
+// (tag_first: [65537] CSR into segs, by tag; words relative to base_word in the output)
+cudaError_t launch_bo_tags(const uint4* ev, uint64_t n, uint64_t base_word, uint64_t n_words,
+                           const uint32_t* tag_first, const TagSeg* segs, uint4* cand, uint64_t cand_cap,
+                           unsigned long long* count, cudaStream_t s);
 // N2: the hash entries of the instances still unjoined at the end of the flush
 // (dense index d with co_of[d] != 0xFFFFFFFF) -> out {word lo, word hi, co_of[d], flag};
 // *n_out counts them (out holds hcap entries)

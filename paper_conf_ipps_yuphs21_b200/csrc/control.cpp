@@ -43,7 +43,7 @@ struct Emitter {
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
                      FlushPlan& out, bool bo, const std::vector<CarriedInst>* carried_in, bool unified,
-                     uint32_t n_dev, const LastEnded* last_ended_in) {
+                     uint32_t n_dev, const LastEnded* last_ended_in, const TagBases* tags_in) {
   const uint32_t n_buckets = (uint32_t)bucket_start.size() - 1;
   out = FlushPlan();
   Emitter em{base_word, n_words, &out, unified};
@@ -75,6 +75,32 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   auto s_alloc = [&](uint32_t d) { return md ? sel8_clear(d) : (kSelALLOC | (bo ? kPopSet : 0u)); };
   auto s_rel = [&](uint32_t d) { return md ? sel8_clear(d) : (kSelREL | (bo ? kPopClr : 0u)); };
   constexpr uint64_t kAddrMask = (1ull << 56) - 1;
+  // N1 (Z25): pointer tags and the entry holding each tag's base, as a timeline
+  if (tags_in) out.tags_out = *tags_in;
+  std::vector<std::vector<TagSeg>> tseg;        // per tag (index into tag_ids)
+  std::map<uint32_t, uint32_t> tag_ix;          // tag -> index
+  auto entry_words = [&](uint64_t byte, uint64_t& lo, uint64_t& hi) {   // the entry holding `byte`
+    lo = hi = 0;
+    auto nx = map.upper_bound(byte);
+    if (nx == map.begin()) return;
+    auto pv = std::prev(nx);
+    // the words whose first byte lies in the entry (the oracle's containment test)
+    if (byte < pv->second.hi) { lo = ((pv->first & kAddrMask) + 7) >> 3; hi = ((pv->second.hi & kAddrMask) + 7) >> 3; }
+  };
+  auto tag_note = [&](uint32_t t, uint32_t pos) {   // tag t's base entry from pos on
+    auto it = tag_ix.find(t);
+    if (it == tag_ix.end()) { it = tag_ix.emplace(t, (uint32_t)tseg.size()).first; tseg.emplace_back(); }
+    TagSeg g{pos, 0, 0, 0};
+    entry_words(out.tags_out[t], g.lo, g.hi);
+    auto& v = tseg[it->second];
+    if (!v.empty() && v.back().pos == pos) v.back() = g; else v.push_back(g);
+  };
+  auto tags_in_range = [&](uint64_t lo, uint64_t hi, uint32_t pos) {   // an entry [lo, hi) changed
+    for (const auto& kv : out.tags_out)
+      if (kv.second >= lo && kv.second < hi) tag_note(kv.first, pos);
+  };
+  if (bo && n_dev == 1)
+    for (const auto& kv : out.tags_out) tag_note(kv.first, 0);
   for (const CtlRec& c : ctl) {
     uint32_t op = (uint32_t)(c.w0 >> 48) & 0xFFu, arg = (uint32_t)(c.w0 >> 56);
     uint32_t dev = 0;                               // Z24: device of a MAP / UPDATE record
@@ -127,6 +153,7 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
           break;                                    // ... unless `always`
         }
         map.emplace(dkey | addr, MapEntry{dkey | (addr + len), 1});  // new CV, ref_count = 1
+        if (bo && n_dev == 1 && !out.tags_out.empty()) tags_in_range(addr, addr + len, pos);
         em.emit(pos, s_alloc(dev), addr, addr + len, open);
         if (arg == MT_TO || arg == MT_TOFROM) em.emit(pos, s_upt(dev), addr, addr + len, open);
         break;
@@ -146,7 +173,9 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
         if (it->second.rc == 0) {
           if (arg == MT_FROM || arg == MT_TOFROM) em.emit(pos, s_uph(dev), addr, addr + len, open);
           em.emit(pos, s_rel(dev), it->first & kAddrMask, it->second.hi & kAddrMask, open);
+          const uint64_t elo = it->first & kAddrMask, ehi = it->second.hi & kAddrMask;
           map.erase(it);
+          if (bo && n_dev == 1 && !out.tags_out.empty()) tags_in_range(elo, ehi, pos);
         }
         break;
       }
@@ -158,6 +187,12 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
         if (f < 0) return fail(ARB_EMAP, c.pos, "target update partially overlaps a present entry");
         if (f == 0) break;                          // not present: no-op (Z7)
         em.emit(pos, arg == 0 ? s_upt(dev) : s_uph(dev), addr, addr + len, open);
+        break;
+      }
+      case OP_BASE: {                               // Z25: pointer tag -> base address
+        if (tid == 0) return fail(ARB_ETRACE, c.pos, "ARB_BASE with pointer tag 0");
+        out.tags_out[tid] = addr;
+        if (bo && n_dev == 1) tag_note(tid, pos);
         break;
       }
       case OP_TASK_DEPEND: {                        // Z22: the open task runs after the last
@@ -180,6 +215,14 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
       default:
         return fail(ARB_ETRACE, c.pos, "unknown control op");
     }
+  }
+  if (!tseg.empty()) {                          // N1: CSR by tag id for k_bo_tags
+    out.tag_first.assign(65537, 0);
+    for (const auto& kv : tag_ix) out.tag_first[kv.first + 1] = (uint32_t)tseg[kv.second].size();
+    for (uint32_t t = 0; t < 65536; ++t) out.tag_first[t + 1] += out.tag_first[t];
+    out.tag_segs.resize(out.tag_first[65536]);
+    for (const auto& kv : tag_ix)
+      std::copy(tseg[kv.second].begin(), tseg[kv.second].end(), out.tag_segs.begin() + out.tag_first[kv.first]);
   }
   // Z22: joining a dependant joins its ancestors (children come after parents)
   for (size_t k = edges.size(); k-- > 0;)

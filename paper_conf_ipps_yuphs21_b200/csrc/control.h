@@ -49,6 +49,9 @@ struct CarriedInst { uint32_t task_id; std::vector<RangeRef> own; bool open; std
 // dependency on it adds no constraint).  Ids that never ended have no entry.
 using LastEnded = std::unordered_map<uint32_t, int32_t>;
 
+// N1 (Z25): the base byte address of every pointer tag defined so far (ARB_BASE records)
+using TagBases = std::map<uint32_t, uint64_t>;
+
 struct FlushPlan {
   std::vector<RangeOpH> range_ops;       // in trace order
   std::vector<uint32_t> ops_start;       // per bucket CSR
@@ -58,6 +61,9 @@ struct FlushPlan {
   std::vector<uint32_t> dense_carry_out; // per MIR dense index: its carried-out index, or 0xFFFFFFFF
   std::vector<CarriedInst> carry_out;    // instances still unjoined at the end of this flush
   LastEnded last_ended_out;              // LastEnded after this flush (committed with carry_out)
+  TagBases tags_out;                     // tag bases after this flush (committed likewise)
+  std::vector<uint32_t> tag_first;       // N1 with bo: [65537] CSR of tag_segs by tag (empty: no tag)
+  std::vector<TagSeg> tag_segs;
   uint64_t range_words = 0, ignored_words = 0, tasks = 0;
   int rc = 0; uint64_t err_pos = 0; std::string err;
 };
@@ -73,10 +79,14 @@ struct FlushPlan {
 // are returned in out.carry_out instead of being treated as joined (Z19).
 // last_ended_in: the LastEnded table after the previous flush (indices into
 // carried_in); the updated table is returned in out.last_ended_out.
+// tags_in: pointer tag bases defined by earlier flushes (ARB_BASE, Z25); the updated
+// set is returned in out.tags_out; with bo, out.tag_first / tag_segs give every
+// defined tag's base entry over the batch (the k_bo_tags timeline).
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
                      FlushPlan& out, bool bo = false, const std::vector<CarriedInst>* carried_in = nullptr,
-                     bool unified = false, uint32_t n_dev = 1, const LastEnded* last_ended_in = nullptr);
+                     bool unified = false, uint32_t n_dev = 1, const LastEnded* last_ended_in = nullptr,
+                     const TagBases* tags_in = nullptr);
 // n_dev > 1 (Z24): device bits 6-7 of MAP / UPDATE args select the device; its
 // entries live in the same table under keys offset by device << 56, and range
 // ops are 8-output selectors (Sel8).

@@ -158,4 +158,42 @@ cudaError_t launch_mir(const MirParams& p, uint64_t n_ins_pos, uint64_t n_qry_po
   return cudaGetLastError();
 }
 
+// ---- N1 (Z25): accesses through a tagged pointer outside its base's entry ----
+__global__ void k_bo_tags(const uint4* ev, uint64_t n, uint64_t base_word, uint64_t n_words,
+                          const uint32_t* tag_first, const TagSeg* segs, uint4* cand, uint64_t cand_cap,
+                          unsigned long long* count) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint4 q = ld_stream(ev + i);
+    const uint32_t op = (q.y >> 16) & 0xFFu, tag = q.w >> 16;
+    if ((op != OP_RT && op != OP_WT) || tag == 0) continue;
+    uint32_t a = __ldg(tag_first + tag), z = __ldg(tag_first + tag + 1);
+    if (a == z || segs[a].pos > (uint32_t)i) continue;        // no base defined yet
+    while (z - a > 1) {                                        // last segment starting at or before i
+      const uint32_t mid = (a + z) >> 1;
+      if (segs[mid].pos <= (uint32_t)i) a = mid; else z = mid;
+    }
+    const uint64_t lo = segs[a].lo, hi = segs[a].hi;
+    const uint64_t addr = (uint64_t)q.x | ((uint64_t)(q.y & 0xFFFFu) << 32), len = q.z;
+    const uint64_t w0 = addr >> 3, w1 = (addr + len - 1) >> 3;
+    for (uint64_t x = w0; x <= w1; ++x) {
+      if (x < base_word || x - base_word >= n_words || (x >= lo && x < hi)) continue;
+      const unsigned long long slot = atomicAdd(count, 1ull);
+      if (slot < cand_cap) {
+        const uint64_t r = x - base_word;
+        cand[slot] = make_uint4((uint32_t)r, (uint32_t)(r >> 32), (uint32_t)i, 4u);   // ARB_BO
+      }
+    }
+  }
+}
+
+cudaError_t launch_bo_tags(const uint4* ev, uint64_t n, uint64_t base_word, uint64_t n_words,
+                           const uint32_t* tag_first, const TagSeg* segs, uint4* cand, uint64_t cand_cap,
+                           unsigned long long* count, cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  const uint64_t g = (n + 255) / 256;
+  k_bo_tags<<<(unsigned)std::min<uint64_t>(g, 148 * 16), 256, 0, s>>>(ev, n, base_word, n_words, tag_first, segs,
+                                                                     cand, cand_cap, count);
+  return cudaGetLastError();
+}
+
 }  // namespace arb

@@ -60,7 +60,7 @@ __device__ __forceinline__ Dec decode0(uint4 q, bool valid, const PartParams& p,
   const uint32_t len = q.z, hi = q.y & 0xFFFFu;
   // malformed access: len outside 1..8 or the byte range leaving the 48-bit space
   const bool bad_acc = (q.w & 0xFFFFu) != 0 || len - 1u > 7u || (hi == 0xFFFFu && q.x > 0u - len);
-  const bool ctl = op < 16 && ((0xF700u >> op) & 1u);            // ops 8, 9, 10, 12, 13, 14, 15
+  const bool ctl = op < 16 && ((0xFF00u >> op) & 1u);            // ops 8-15 (11: ARB_BASE, Z25)
   const bool acc = op < 4;
   flags = valid ? (acc ? (bad_acc ? 2u : 0u) : (ctl ? 1u : 2u)) : 0u;
   bool ok = valid && acc && !bad_acc;
@@ -382,7 +382,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
       for (uint32_t w = 0; w < PW; ++w) {
         uint16_t* r = reinterpret_cast<uint16_t*>(smem + kCtaSmem + w * kWarpSmem + sizeof(uint4) * WREC + 4 * WREC) + b;
         const uint32_t c = *r;
-        *r = (uint16_t)run;
+        if (c) *r = (uint16_t)run;     // rows of warps that did not touch b stay 0
         run += c;
       }
       tbase[b] = run;

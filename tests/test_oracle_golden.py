@@ -371,3 +371,42 @@ def test_unified_memory_paper(orc):
         rec, base, size, _ = load(name)
         res = run(orc, rec, base, size, unified=True)
         assert {(r, k) for _, r, k in res.triples()} == expect, name
+
+
+def test_bo_overflow_into_adjacent_cv(orc):
+    """"the host program only maps the first half of an array ... the compute
+    kernel loops through the whole array ... It may retrieve a valid value from an
+    adjacent memory location which happens to be another variable's CV."  Here the
+    adjacent location IS mapped (variable B right after A's first half), so the
+    present-bit form (Z20) sees nothing; through the kernel's pointer to A (tag 1,
+    base A) every access to B's words is BO (Z25), and the accesses still
+    read B's CV."""
+    from gen.trace import encode
+    A, n = 0x4000, 64
+    B = A + 8 * (n // 2)                 # B occupies the second half of A's extent
+    tb = TraceBuilder()
+    tb.loop([(OP.WH, A)], n, 8)          # host initialises A's first half and B
+    tb.enter(MAP.TO, A, 8 * (n // 2))    # map(to: a[0:n/2])
+    tb.enter(MAP.TO, B, 8 * (n // 2))    # map(to: b[0:n/2]) -- B's CV, adjacent
+    tb.add_array(np.array([encode(11, A, 0, task=1)], dtype=np.uint64))   # pointer tag 1 -> base A
+    k0 = len(tb)
+    for i in range(n):
+        tb.add_array(np.array([encode(OP.RT, A + 8 * i, 8, task=1)], dtype=np.uint64))
+    tb.exit(MAP.TO, B, 8 * (n // 2))
+    tb.exit(MAP.TO, A, 8 * (n // 2))
+    rec = tb.array()
+    res = run(orc, rec, A, 8 * n, detect_bo=True)
+    assert res.triples() == [(A // 8 + i, k0 + i, BO) for i in range(n // 2, n)]
+    # the present-bit form alone (no tag) reports nothing: B's words have a CV
+    untagged = rec.copy()
+    untagged[k0:k0 + n, 1] &= np.uint64((1 << 48) - 1)
+    assert run(orc, untagged, A, 8 * n, detect_bo=True).triples() == []
+    # a correctly mapped array (one section for the whole extent) is clean
+    tb2 = TraceBuilder()
+    tb2.loop([(OP.WH, A)], n, 8)
+    tb2.enter(MAP.TO, A, 8 * n)
+    tb2.add_array(np.array([encode(11, A, 0, task=1)], dtype=np.uint64))
+    for i in range(n):
+        tb2.add_array(np.array([encode(OP.RT, A + 8 * i, 8, task=1)], dtype=np.uint64))
+    tb2.exit(MAP.TO, A, 8 * n)
+    assert run(orc, tb2.array(), A, 8 * n, detect_bo=True).triples() == []

@@ -581,3 +581,38 @@ def test_host_submit_host_global_index(orc, split):
     ctx.get_reports(n, out=dev_out)                 # device output of host-translated reports
     assert reports_to_triples(dev_out[:n].cpu().numpy().view(np.uint64)) == exp.triples()
     ctx.close()
+
+
+# ---- N1: buffer overflow through a tagged pointer (ARB_BASE, Z25) -------------
+def test_bo_overflow_into_adjacent_cv_gpu(orc):
+    """The P:279 case the present-bit form misses: the kernel's pointer to A runs into
+    B's (mapped) CV; every such access is BO and still reads B's CV."""
+    from gen.trace import TraceBuilder, MAP, OP, encode
+    A, n = 0x4000, 64
+    B = A + 8 * (n // 2)
+    tb = TraceBuilder()
+    tb.loop([(OP.WH, A)], n, 8)
+    tb.enter(MAP.TO, A, 8 * (n // 2))
+    tb.enter(MAP.TO, B, 8 * (n // 2))
+    tb.add_array(np.array([encode(OP.BASE, A, 0, task=1)], dtype=np.uint64))
+    for i in range(n):
+        tb.add_array(np.array([encode(OP.RT, A + 8 * i, 8, task=1)], dtype=np.uint64))
+    tb.exit(MAP.TO, B, 8 * (n // 2))
+    tb.exit(MAP.TO, A, 8 * (n // 2))
+    rec = tb.array()
+    exp, st = check(orc, rec, A, 8 * n, flags=8)
+    assert len(exp.triples()) == n // 2 and {t[2] for t in exp.triples()} == {4}
+    assert st["reports_bo"] == n // 2
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_bo_tags_fuzz(orc, seed):
+    """Random programs with pointer tags, re-based tags, tasks and flush cuts (the tag
+    bases and entries carried across flushes), several bucket sizes."""
+    from gen.fuzz import random_program
+    rec, base, span = random_program(9100 + seed, p_tag=0.6, p_task=0.3, steps=120)
+    exp, _ = check(orc, rec, base, span, flags=8)
+    check(orc, rec, base, span, flags=8, bucket_bits=4)
+    if exp.rc == 0:
+        rc, got, shadow, _ = run_gpu(rec, base, span, flags=8, flush_points=_cuts(rec, 5, seed))
+        assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
