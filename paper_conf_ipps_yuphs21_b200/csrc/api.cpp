@@ -488,6 +488,45 @@ static void build_items(arb_ctx ctx, const FlushPlan& plan, const std::vector<do
   for (size_t i = 0; i < its.size(); ++i) ctx->items[i] = its[i].v;
 }
 
+// Debug aid (ARB_CHECK_PARTITION=1): every bucket region must hold, in trace order,
+// exactly the events of the records whose words the bucket owns.  Prints the first
+// violations to stderr.
+static void check_partition(arb_ctx ctx, const uint4* ev, uint64_t n, cudaStream_t s) {
+  cudaStreamSynchronize(s);
+  std::vector<uint4> rec(n);
+  std::vector<uint64_t> rs(kMaxBuckets);
+  if (n) cudaMemcpy(rec.data(), ev, n * 16, cudaMemcpyDeviceToHost);
+  cudaMemcpy(rs.data(), ctx->d_reg_start.p, kMaxBuckets * 8, cudaMemcpyDeviceToHost);
+  uint64_t tot = 0;
+  for (uint32_t b = 0; b < ctx->n_buckets; ++b) tot = std::max(tot, rs[b] + ctx->h_btotal.p[b]);
+  std::vector<uint2> pe(tot + 1);
+  if (tot) cudaMemcpy(pe.data(), ctx->part_ev.p, tot * 8, cudaMemcpyDeviceToHost);
+  uint64_t bad = 0, events = 0;
+  for (uint32_t b = 0; b < ctx->n_buckets; ++b) {
+    const uint64_t c = ctx->h_btotal.p[b];
+    events += c;
+    int64_t last = -1;
+    for (uint64_t i = 0; i < c; ++i) {
+      const uint2 e = pe[rs[b] + i];
+      const uint32_t pos = e.y & (((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u) ? 0x3FFFFFFFu : 0xFFFFFFFFu);
+      bool ok = pos < n && (int64_t)pos >= last;
+      if (ok) {
+        const uint4 q = rec[pos];
+        const uint64_t addr = (uint64_t)q.x | ((uint64_t)(q.y & 0xFFFFu) << 32);
+        const uint64_t w = ctx->base_word + ctx->bucket_start[b] + (e.x & 0x3FFFFFFFu);
+        ok = ((q.y >> 16) & 0xFFu) == (e.x >> 30) && w >= (addr >> 3) && w <= ((addr + q.z - 1) >> 3);
+      }
+      if (!ok && bad++ < 8)
+        fprintf(stderr, "arb check_partition: bucket %u event %llu/%llu pos %u (last %lld) key %08x\n", b,
+                (unsigned long long)i, (unsigned long long)c, pos, (long long)last, e.x);
+      last = pos;
+    }
+  }
+  fprintf(stderr, "arb check_partition: %llu records, %llu events in %u buckets, %llu bad (access words %llu)\n",
+          (unsigned long long)n, (unsigned long long)events, ctx->n_buckets, (unsigned long long)bad,
+          (unsigned long long)ctx->h_stats.p->access_words);
+}
+
 extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, uint64_t* report_offset_global) {
   if (!ctx) return ARB_EINVAL;
   cudaSetDevice(ctx->cfg.device);
@@ -649,6 +688,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   }
   ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;
   bucket_events.assign(ctx->h_btotal.p, ctx->h_btotal.p + ctx->n_buckets);   // exact, from the look-back
+  if (getenv("ARB_CHECK_PARTITION")) check_partition(ctx, ev, n, s);
   S.buckets = ctx->n_buckets;
   S.access_words = hst.access_words;
   S.control_records = hst.n_ctl;
@@ -734,6 +774,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   rp.shadow = ctx->shadow; rp.bo = (ctx->cfg.flags & ARB_F_BO) ? 1u : 0u;
   rp.um = (ctx->cfg.flags & ARB_F_UNIFIED) ? 1u : 0u;
   rp.md = ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u) ? 1u : 0u; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
+  rp.no_direct = getenv("ARB_NO_DIRECT") ? 1u : 0u;
   rp.cand = ctx->cand.p; rp.cand_cap = ctx->cand_cap; rp.st = ctx->dstats.p;
   rp.hot_off = ctx->d_hot_off.p; rp.hot_F = ctx->hot_F.p; rp.hot_P = ctx->hot_P.p;
   int n_ctas = std::max(1, std::min<int>((int)ctx->items.size(), ctx->n_sms * kReplayCtasPerSm));

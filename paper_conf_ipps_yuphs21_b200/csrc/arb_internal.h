@@ -106,7 +106,8 @@ struct DevStats {
   unsigned long long overflow;        // a bucket received more events than its region holds
   unsigned long long n_carry_out;     // N2: access summaries of instances carried into the next flush
   unsigned long long n_bo_cand;       // N1 (Z25): base-tag overflow candidates
-  unsigned long long pad[2];
+  unsigned long long tile_ticket;     // k_partition: next CTA tile to take (in order)
+  unsigned long long pad[1];
 };
 
 // control record extracted by the partition kernel
@@ -172,6 +173,7 @@ struct ReplayParams {
   uint32_t bo;                            // ARB_F_BO: target accesses to words without kCVp are BO
   uint32_t um;                            // ARB_F_UNIFIED: OV and CV are one storage (Z23)
   uint32_t md;                            // several accelerators (Z24): 8-bit states, device in pos bits 30-31
+  uint32_t no_direct;                     // debug: never use the direct step
   const uint32_t* ops_start;              // [n_buckets + 1]
   const BucketOp* ops;
   uint4* cand; uint64_t cand_cap;         // report candidates {word lo, word hi, pos, kind}

@@ -2,8 +2,12 @@
 // in one sweep over the batch, with a decoupled look-back across CTA tiles.
 //
 // k_partition  persistent CTAs (one per SM, 16 warps).  A CTA tile is 16 chunks of
-//              256 records (4096 records), one chunk per warp; tile t of the batch
-//              is processed by CTA t mod grid.  Per tile:
+//              256 records (4096 records), one chunk per warp; CTAs take tiles in
+//              order from a ticket counter (one tile ahead, so the next tile's
+//              records stream in during this one) — tickets let the CTAs drift
+//              apart, so a tile's predecessors have mostly published inclusive
+//              prefixes by the time it looks back (a lockstep grid would make every
+//              tile of a wave walk back to the previous wave).  Per tile:
 //   1. every warp decodes its chunk (staged in its shared memory by one TMA bulk
 //      copy, cp.async.bulk, completing on an mbarrier; the warp's chunk of the
 //      next tile is fetched as soon as this one is decoded): access vs control
@@ -221,6 +225,11 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     sreg[i] = p.reg_start[i]; scap[i] = p.reg_cap[i]; ttag[i] = 0;
   }
   if (tid < 2) nU[tid] = 0;
+  __shared__ uint32_t s_tick[2];
+  if (tid == 0) {
+    s_tick[0] = (uint32_t)atomicAdd(&p.st->tile_ticket, 1ull);
+    s_tick[1] = (uint32_t)atomicAdd(&p.st->tile_ticket, 1ull);
+  }
   for (uint32_t i = lane; i < NBK; i += 32) row[i] = 0;
   if (lane == 0) mbar_init(bar, 1);
   fence_mbar_init();
@@ -236,10 +245,10 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
       bulk_g2s(stage, p.ev + r0, nv * 16u, bar);
     }
   };
-  const uint32_t G = gridDim.x;
-  fetch((uint64_t)blockIdx.x * PW + warp);
+  uint32_t tile = s_tick[0], nxt = s_tick[1];
+  fetch((uint64_t)tile * PW + warp);
   uint32_t tag = 0, par = 0;
-  for (uint32_t tile = blockIdx.x; tile < p.n_tiles; tile += G, par ^= 1u) {
+  while (tile < p.n_tiles) {
     tag = tag + 1 == 0 ? 1 : tag + 1;
     const uint64_t chunk = (uint64_t)tile * PW + warp;
     const uint64_t rec0 = chunk * WREC;
@@ -366,7 +375,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
       for (int k = 0; k < RPL; ++k) { dec[k].info = 0; rk[k] = 0; }
     }
     __syncwarp();                      // stage reads done
-    fetch(chunk + (uint64_t)G * PW);   // this warp's chunk of its next tile streams in meanwhile
+    fetch((uint64_t)nxt * PW + warp);  // this warp's chunk of the CTA's next tile streams in meanwhile
     // ---- 2. the buckets the tile touches ------------------------------------------------
     for (uint32_t t = lane; t < nT; t += 32) {
       const uint32_t b = tlist[t];
@@ -387,7 +396,10 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
       }
       tbase[b] = run;
     }
-    if (tid == 0) nU[par ^ 1u] = 0;
+    if (tid == 0) {
+      nU[par ^ 1u] = 0;
+      s_tick[par] = (uint32_t)atomicAdd(&p.st->tile_ticket, 1ull);   // the tile after next
+    }
     __syncthreads();
     // ---- 3. decoupled look-back over the tiles (buckets 4 tid .. 4 tid + 3) -------------
     {
@@ -471,6 +483,9 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     __syncwarp();
     for (uint32_t t = lane; t < nT; t += 32) row[tlist[t]] = 0;
     __syncwarp();
+    tile = nxt;
+    nxt = s_tick[par];                 // written before the look-back barrier
+    par ^= 1u;
   }
 
 #pragma unroll

@@ -382,8 +382,10 @@ __device__ __forceinline__ bool step_direct(ReplaySmem& S, const ReplayParams& p
   uint32_t won = 0;
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
-    if ((op[j] & 9u) == 1u) {      // an in-window write (WH = 1, WT = 3)
-      any_w = true;
+    // every write counts (one outside the window forces the fallback below, or a
+    // later read of its word would miss it); in-window writes claim their slot
+    if ((op[j] & 5u) == 1u) any_w = true;      // WH = 1, WT = 3 (| 8 outside the window)
+    if ((op[j] & 13u) == 1u) {                 // an in-window write
       const uint32_t i = threadIdx.x + j * RT;
       const uint32_t code = MD ? ((((devs >> (2 * j)) & 3u) << 1) | (op[j] >> 1)) : op[j];
       if (atomicCAS(&tab[idx[j]], kEmpty, (i << 4) | code) == kEmpty) won |= 1u << j;
@@ -881,7 +883,7 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         step_summary<UM>(S, ev, cut);
       } else {
         bool fast = false, oow = false;
-        const uint32_t skip = S.skip_direct;
+        const uint32_t skip = p.no_direct ? 1u : S.skip_direct;
         if (!skip) {
           fast = S.partial ? step_direct<true, BO, UM, MD>(S, p, ev, cut, &oow)
                            : step_direct<false, BO, UM, MD>(S, p, ev, cut, &oow);
