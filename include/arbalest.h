@@ -174,7 +174,7 @@ typedef struct {
   uint64_t kernel_launches;  /* kernels launched by the last flush                         */
   double   ms_sample;        /* address sampling + bucket balancing (inside ms_partition)  */
   uint64_t steps_fast, steps_sort;  /* replay steps by kind                  */
-  double   ms_segsort;       /* unused (0): the one-sweep partition has no segment sort     */
+  double   ms_segsort;       /* GPU: segment-entry sort (inside ms_control)                 */
   double   ms_host_control;  /* host wall time of the Table I / task resolution             */
   uint64_t work_items;       /* replay work items (buckets, word-range parts, hot slices)   */
   uint64_t hot_buckets;      /* buckets replayed as time slices (hot words, K5)             */
@@ -182,8 +182,6 @@ typedef struct {
   uint64_t nccl_ranks;       /* ranks of the context's NCCL communicator (ncclCommCount), 0 =
                                 no communicator                                              */
   uint64_t exchanges;        /* collectives (status / count ncclAllGather) of the last flush */
-  uint64_t partition_retries;/* partition re-runs with exact bucket sizes (a sampled region
-                                overflowed) in the last flush                                */
 } arb_stats;
 
 typedef struct arb_ctx_s* arb_ctx;

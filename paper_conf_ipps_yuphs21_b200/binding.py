@@ -57,7 +57,7 @@ class arb_stats(ctypes.Structure):
                 ("ms_segsort", ctypes.c_double), ("ms_host_control", ctypes.c_double),
                 ("work_items", ctypes.c_uint64), ("hot_buckets", ctypes.c_uint64),
                 ("reports_bo", ctypes.c_uint64), ("nccl_ranks", ctypes.c_uint64),
-                ("exchanges", ctypes.c_uint64), ("partition_retries", ctypes.c_uint64)]
+                ("exchanges", ctypes.c_uint64)]
 
     def as_dict(self):
         d = {}

@@ -125,14 +125,15 @@ struct arb_ctx_s {
   bool host_gidx = false, dev_gidx = false;   // where this batch's global indices live
   DevBuf<uint4> staging;
   DevBuf<uint64_t> gidx_staging;
-  DevBuf<uint2> part_ev;                      // bucket regions of the partition output
+  DevBuf<uint2> part_ev;
+  DevBuf<uint2> seg_a, seg_b;                 // partition entries, sort ping-pong
+  DevBuf<uint4> segs;                         // replay form
+  DevBuf<uint32_t> seg_first;
+  uint64_t seg_cap = 0;
+  HostBuf<uint32_t> h_weight;
   TagBases tags;                              // N1 (Z25): pointer tag bases (committed per flush)
   DevBuf<uint32_t> d_tag_first;
   DevBuf<TagSeg> d_tag_segs;
-  DevBuf<uint64_t> d_reg_start, d_btotal;     // region start, exact events per bucket
-  DevBuf<uint32_t> d_reg_cap;                 // region capacity
-  HostBuf<uint64_t> h_btotal;
-  DevBuf<unsigned long long> ring;            // look-back status ring
   DevBuf<CtlRec> ctl;
   DevBuf<uint4> cand, cand_tmp, reports;
   DevBuf<uint32_t> blk;
@@ -265,7 +266,7 @@ extern "C" int arb_init(const arb_config* cfg, arb_ctx* out) {
   if (e == cudaSuccess) e = ctx->h_stats.ensure(1);
   if (e == cudaSuccess) e = ctx->h_nb.ensure(1);
   if (e == cudaSuccess) e = ctx->h_bstart.ensure(kMaxBuckets + 1);
-  if (e == cudaSuccess) e = ctx->h_btotal.ensure(kMaxBuckets);
+  if (e == cudaSuccess) e = ctx->h_weight.ensure(kMaxBuckets);
   if (e == cudaSuccess) e = cudaDeviceSynchronize();
   if (e != cudaSuccess) { arb_destroy(ctx); return ARB_ENOMEM; }
   if (cfg->nccl_unique_id) {
@@ -295,8 +296,8 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   if (!ctx) return ARB_OK;
   if (ctx->comm && ctx->nccl_destroy) ctx->nccl_destroy(ctx->comm);
   if (ctx->shadow) cudaFree(ctx->shadow);
-  ctx->staging.release(); ctx->gidx_staging.release(); ctx->part_ev.release(); ctx->d_reg_start.release();
-  ctx->d_btotal.release(); ctx->d_reg_cap.release(); ctx->h_btotal.release(); ctx->ring.release();
+  ctx->staging.release(); ctx->gidx_staging.release(); ctx->part_ev.release(); ctx->seg_a.release(); ctx->seg_b.release(); ctx->segs.release(); ctx->seg_first.release();
+  ctx->h_weight.release();
   ctx->d_tag_first.release(); ctx->d_tag_segs.release();
   ctx->ctl.release(); ctx->cand.release(); ctx->cand_tmp.release(); ctx->reports.release(); ctx->blk.release();
   ctx->ops_start.release(); ctx->ops.release(); ctx->dstats.release(); ctx->dcount.release();
@@ -488,45 +489,6 @@ static void build_items(arb_ctx ctx, const FlushPlan& plan, const std::vector<do
   for (size_t i = 0; i < its.size(); ++i) ctx->items[i] = its[i].v;
 }
 
-// Debug aid (ARB_CHECK_PARTITION=1): every bucket region must hold, in trace order,
-// exactly the events of the records whose words the bucket owns.  Prints the first
-// violations to stderr.
-static void check_partition(arb_ctx ctx, const uint4* ev, uint64_t n, cudaStream_t s) {
-  cudaStreamSynchronize(s);
-  std::vector<uint4> rec(n);
-  std::vector<uint64_t> rs(kMaxBuckets);
-  if (n) cudaMemcpy(rec.data(), ev, n * 16, cudaMemcpyDeviceToHost);
-  cudaMemcpy(rs.data(), ctx->d_reg_start.p, kMaxBuckets * 8, cudaMemcpyDeviceToHost);
-  uint64_t tot = 0;
-  for (uint32_t b = 0; b < ctx->n_buckets; ++b) tot = std::max(tot, rs[b] + ctx->h_btotal.p[b]);
-  std::vector<uint2> pe(tot + 1);
-  if (tot) cudaMemcpy(pe.data(), ctx->part_ev.p, tot * 8, cudaMemcpyDeviceToHost);
-  uint64_t bad = 0, events = 0;
-  for (uint32_t b = 0; b < ctx->n_buckets; ++b) {
-    const uint64_t c = ctx->h_btotal.p[b];
-    events += c;
-    int64_t last = -1;
-    for (uint64_t i = 0; i < c; ++i) {
-      const uint2 e = pe[rs[b] + i];
-      const uint32_t pos = e.y & (((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u) ? 0x3FFFFFFFu : 0xFFFFFFFFu);
-      bool ok = pos < n && (int64_t)pos >= last;
-      if (ok) {
-        const uint4 q = rec[pos];
-        const uint64_t addr = (uint64_t)q.x | ((uint64_t)(q.y & 0xFFFFu) << 32);
-        const uint64_t w = ctx->base_word + ctx->bucket_start[b] + (e.x & 0x3FFFFFFFu);
-        ok = ((q.y >> 16) & 0xFFu) == (e.x >> 30) && w >= (addr >> 3) && w <= ((addr + q.z - 1) >> 3);
-      }
-      if (!ok && bad++ < 8)
-        fprintf(stderr, "arb check_partition: bucket %u event %llu/%llu pos %u (last %lld) key %08x\n", b,
-                (unsigned long long)i, (unsigned long long)c, pos, (long long)last, e.x);
-      last = pos;
-    }
-  }
-  fprintf(stderr, "arb check_partition: %llu records, %llu events in %u buckets, %llu bad (access words %llu)\n",
-          (unsigned long long)n, (unsigned long long)events, ctx->n_buckets, (unsigned long long)bad,
-          (unsigned long long)ctx->h_stats.p->access_words);
-}
-
 extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, uint64_t* report_offset_global) {
   if (!ctx) return ARB_EINVAL;
   cudaSetDevice(ctx->cfg.device);
@@ -540,7 +502,6 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   S.reports = 0; std::memset(S.reports_by_kind, 0, sizeof(S.reports_by_kind)); S.ignored_words = 0;
   S.ms_partition = S.ms_control = S.ms_replay = S.ms_mir = S.ms_reports = S.ms_total = 0;
   S.ms_segsort = S.ms_host_control = 0;
-  S.partition_retries = 0;
   S.buckets = ctx->n_buckets; S.bucket_bits = ctx->bucket_bits; S.max_bucket_events = 0;
 
   // Phase A (validation): decode + partition and control resolution.  Nothing
@@ -553,7 +514,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   const uint64_t index_base = ctx->next_index;
   const bool balanced = ctx->bucket_bits == 0;
   DevStats& hst = *ctx->h_stats.p;
-  std::vector<double> bucket_events;      // events per bucket (exact, from the partition)
+  std::vector<double> bucket_events;      // estimated events per bucket (sampled)
   MapTable map;
   FlushPlan plan;
   std::chrono::steady_clock::time_point t_host0, t_host1;
@@ -583,116 +544,97 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     }
   }
   if (timing) cudaEventRecord(ctx->ev[0], s);
-  // ---- sampled address histogram: bucket balancing and region sizes (on the device) ----
-  const uint32_t n_chunks = (uint32_t)((n + kChunkRecords - 1) / kChunkRecords);
-  const uint32_t n_tiles = (n_chunks + kPartWarps - 1) / kPartWarps;
-  const uint64_t ev_cap = 2 * n + 2 * (uint64_t)kMaxBuckets + 64;    // events: <= 2 per record
-  const uint64_t sample_stride = std::max<uint64_t>(1, n / kSampleCap);
-  {
+  // ---- bucket balancing on a sampled address histogram (all on the device) ----
+  if (balanced) {
     CK(ctx->d_hist.ensure(ctx->n_bins), "alloc hist");
     CK(cudaMemsetAsync(ctx->d_hist.p, 0, ctx->n_bins * sizeof(uint32_t), s), "hist clear");
     SampleParams sp{};
-    sp.ev = ev; sp.n = n; sp.stride = sample_stride;
+    sp.ev = ev; sp.n = n; sp.stride = std::max<uint64_t>(1, n / kSampleCap);
     sp.base_word = ctx->base_word; sp.n_words = ctx->n_words; sp.coarse_bits = ctx->coarse_bits;
     sp.hist = ctx->d_hist.p;
     const uint64_t n_samples = n ? (n + sp.stride - 1) / sp.stride : 0;
     CK(launch_sample(sp, n_samples, s), "k_sample");
     launches += n_samples ? 1 : 0;
-  }
-  if (ctx->d_bucket_start.cap == 0) {       // the read-back below copies every slot
-    CK(ctx->d_bucket_start.ensure(kMaxBuckets + 1), "alloc buckets");
-    CK(cudaMemsetAsync(ctx->d_bucket_start.p, 0, (kMaxBuckets + 1) * 8, s), "clear buckets");
-  }
-  if (ctx->d_cut.cap == 0) {
-    CK(ctx->d_cut.ensure(2 * kMaxBuckets + 2), "alloc cut scratch");
-    CK(cudaMemsetAsync(ctx->d_cut.p, 0, (2 * kMaxBuckets + 2) * 4, s), "clear cut scratch");
-  }
-  CK(ctx->d_reg_start.ensure(kMaxBuckets), "alloc regions");
-  CK(ctx->d_reg_cap.ensure(kMaxBuckets), "alloc regions");
-  CK(ctx->d_btotal.ensure(kMaxBuckets), "alloc bucket totals");
-  if (balanced) {
     // cut balanced buckets; the histogram becomes the bin map in place
+    if (ctx->d_bucket_start.cap == 0) {       // the read-back below copies every slot
+      CK(ctx->d_bucket_start.ensure(kMaxBuckets + 1), "alloc buckets");
+      CK(cudaMemsetAsync(ctx->d_bucket_start.p, 0, (kMaxBuckets + 1) * 8, s), "clear buckets");
+    }
+    if (ctx->d_cut.cap == 0) {
+      CK(ctx->d_cut.ensure(2 * kMaxBuckets + 2), "alloc cut scratch");
+      CK(cudaMemsetAsync(ctx->d_cut.p, 0, (2 * kMaxBuckets + 2) * 4, s), "clear cut scratch");
+    }
     CK(ctx->d_cutscr.ensure(2 * ((ctx->n_bins + 1023) / 1024) + 4 + ctx->n_bins), "alloc cut scratch");
     CK(launch_cut(ctx->d_hist.p, ctx->n_bins, ctx->coarse_bits, ctx->n_words, kMaxBuckets, ctx->d_bucket_start.p,
                   ctx->d_cut.p, ctx->d_cut.p + kMaxBuckets, ctx->d_cut.p + 2 * kMaxBuckets, ctx->d_cutscr.p,
                   s, &launches), "k_cut");
-    CK(launch_regions(ctx->d_cut.p, ctx->d_cut.p + 2 * kMaxBuckets, 0, (double)sample_stride, ev_cap,
-                      ctx->d_reg_start.p, ctx->d_reg_cap.p, s), "k_regions");
     // the bucket count and starts come back with the partition's counters (one sync)
     CK(cudaMemcpyAsync(ctx->h_nb.p, ctx->d_cut.p + 2 * kMaxBuckets, 4, cudaMemcpyDeviceToHost, s), "nb d2h");
     CK(cudaMemcpyAsync(ctx->h_bstart.p, ctx->d_bucket_start.p, (kMaxBuckets + 1) * 8, cudaMemcpyDeviceToHost, s),
        "buckets d2h");
-  } else {
-    if (ctx->d_bin_map.cap == 0) {
-      CK(upload(ctx->d_bin_map, ctx->bin_map, s), "upload bin map");
-      CK(upload(ctx->d_bucket_start, ctx->bucket_start, s), "upload bucket starts");
-    }
-    // fixed buckets: coarse bins are the buckets, so the histogram is the weights
-    CK(launch_regions(ctx->d_hist.p, nullptr, (uint32_t)ctx->bin_map.size(), (double)sample_stride, ev_cap,
-                      ctx->d_reg_start.p, ctx->d_reg_cap.p, s), "k_regions");
+    CK(cudaMemcpyAsync(ctx->h_weight.p, ctx->d_cut.p, kMaxBuckets * 4, cudaMemcpyDeviceToHost, s), "weights d2h");
+  } else if (ctx->d_bin_map.cap == 0) {
+    CK(upload(ctx->d_bin_map, ctx->bin_map, s), "upload bin map");
+    CK(upload(ctx->d_bucket_start, ctx->bucket_start, s), "upload bucket starts");
   }
-  launches += 1;
   if (!balanced) ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;   // fixed buckets
   if (timing) cudaEventRecord(ctx->ev[7], s);
-  // ---- A1 + A3: decode + one-sweep partition into contiguous bucket regions ---------
-  CK(ctx->part_ev.ensure(ev_cap), "alloc part_ev");
-  CK(ctx->ring.ensure((size_t)kRingTiles * kMaxBuckets), "alloc look-back ring");
+  // ---- A1/A3a: decode + partition ------------------------------------------
+  const uint32_t n_chunks = (uint32_t)((n + kChunkRecords - 1) / kChunkRecords);
+  CK(ctx->part_ev.ensure((size_t)std::max<uint32_t>(n_chunks, 1) * kChunkCap), "alloc part_ev");
+  if (ctx->seg_cap < (uint64_t)n_chunks * 2 + 4096) ctx->seg_cap = (uint64_t)n_chunks * 2 + 4096;
+  CK(ctx->seg_a.ensure(std::max<uint64_t>(ctx->seg_cap, 1)), "alloc segments");
   PartParams pp{};
-  for (int attempt = 0; attempt < 3; ++attempt) {
+  for (int attempt = 0; attempt < 2; ++attempt) {
     CK(cudaMemsetAsync(ctx->dstats.p, 0, sizeof(DevStats), s), "stats init");
     CK(cudaMemsetAsync(&ctx->dstats.p->err_pos, 0xFF, sizeof(unsigned long long), s), "stats init");
-    CK(cudaMemsetAsync(ctx->ring.p, 0, (size_t)kRingTiles * kMaxBuckets * 8, s), "ring clear");
-    CK(cudaMemsetAsync(ctx->d_btotal.p, 0, kMaxBuckets * 8, s), "totals clear");
     pp.ev = ev; pp.n = n; pp.base_word = ctx->base_word; pp.n_words = ctx->n_words;
     pp.coarse_bits = ctx->coarse_bits; pp.bin_map = balanced ? ctx->d_hist.p : ctx->d_bin_map.p;
     pp.bucket_bits = ctx->bucket_bits; pp.n_buckets = balanced ? (uint32_t)kMaxBuckets : ctx->n_buckets;
-    pp.n_chunks = n_chunks; pp.n_tiles = n_tiles;
+    pp.n_chunks = n_chunks;
     pp.n_dev = 1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u);
-    pp.part_ev = ctx->part_ev.p; pp.reg_start = ctx->d_reg_start.p; pp.reg_cap = ctx->d_reg_cap.p;
-    pp.ring = ctx->ring.p; pp.bucket_total = ctx->d_btotal.p;
+    pp.part_ev = ctx->part_ev.p; pp.seg_out = ctx->seg_a.p; pp.seg_cap = ctx->seg_cap;
     pp.ctl = ctx->ctl.p; pp.ctl_cap = ctx->ctl_cap;
     pp.st = ctx->dstats.p;
     CK(launch_partition(pp, s), "k_partition");
     launches += n_chunks ? 1 : 0;
     CK(cudaMemcpyAsync(&hst, ctx->dstats.p, sizeof(hst), cudaMemcpyDeviceToHost, s), "stats d2h");
-    CK(cudaMemcpyAsync(ctx->h_btotal.p, ctx->d_btotal.p, kMaxBuckets * 8, cudaMemcpyDeviceToHost, s), "totals d2h");
     CK(cudaStreamSynchronize(s), "partition sync");
-    if (hst.n_ctl <= ctx->ctl_cap && !hst.overflow) break;
-    if (hst.n_ctl > ctx->ctl_cap) {
-      ctx->ctl_cap = hst.n_ctl + hst.n_ctl / 2;
-      CK(ctx->ctl.ensure(ctx->ctl_cap), "grow ctl");
-    }
-    if (hst.overflow) {
-      // a bucket outgrew its sampled region: size every region by the exact counts
-      std::vector<uint64_t> rs(kMaxBuckets);
-      std::vector<uint32_t> rc(kMaxBuckets);
-      uint64_t at = 0;
-      for (int b = 0; b < kMaxBuckets; ++b) {
-        rs[b] = at;
-        rc[b] = (uint32_t)((ctx->h_btotal.p[b] + 1) & ~1ull);
-        at += rc[b];
-      }
-      if (at > ctx->part_ev.cap) CK(ctx->part_ev.ensure(at + 64), "grow part_ev");
-      CK(cudaMemcpyAsync(ctx->d_reg_start.p, rs.data(), kMaxBuckets * 8, cudaMemcpyHostToDevice, s), "regions");
-      CK(cudaMemcpyAsync(ctx->d_reg_cap.p, rc.data(), kMaxBuckets * 4, cudaMemcpyHostToDevice, s), "regions");
-      S.partition_retries += 1;
-    }
+    if (hst.n_ctl <= ctx->ctl_cap && hst.n_segs <= ctx->seg_cap) break;
+    if (hst.n_ctl > ctx->ctl_cap) ctx->ctl_cap = hst.n_ctl + hst.n_ctl / 2;
+    if (hst.n_segs > ctx->seg_cap) ctx->seg_cap = hst.n_segs + hst.n_segs / 4;
+    CK(ctx->ctl.ensure(ctx->ctl_cap), "grow ctl");
+    CK(ctx->seg_a.ensure(ctx->seg_cap), "grow segments");
   }
   if (timing) cudaEventRecord(ctx->ev[1], s);
   if (hst.err_pos != ~0ull)
     return fail(ctx, ARB_ETRACE, "malformed record at batch position " + std::to_string(hst.err_pos));
-  if (hst.overflow) return fail(ctx, ARB_ENOMEM, "partition regions overflowed twice");
   if (balanced) {
     const uint32_t nb = *ctx->h_nb.p;
     ctx->bucket_start.assign(ctx->h_bstart.p, ctx->h_bstart.p + nb + 1);
+    const double stride = (double)std::max<uint64_t>(1, n / kSampleCap);
+    bucket_events.resize(nb);
+    for (uint32_t b = 0; b < nb; ++b) bucket_events[b] = ctx->h_weight.p[b] * stride;
   }
   ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;
-  bucket_events.assign(ctx->h_btotal.p, ctx->h_btotal.p + ctx->n_buckets);   // exact, from the look-back
-  if (getenv("ARB_CHECK_PARTITION")) check_partition(ctx, ev, n, s);
   S.buckets = ctx->n_buckets;
   S.access_words = hst.access_words;
   S.control_records = hst.n_ctl;
-  if (timing) cudaEventRecord(ctx->ev[8], s);
+
+  // ---- A3b: segment entries sorted by (bucket, chunk) — on the GPU while the
+  // host resolves the control records ------------------------------------------------
+  {
+    const uint64_t ns = hst.n_segs;
+    CK(ctx->seg_b.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
+    CK(ctx->segs.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
+    CK(ctx->seg_first.ensure(ctx->n_buckets + 1), "alloc seg_first");
+    CK(ctx->blk.ensure((ns + 4095) / 4096 * 2049 + 4096), "alloc blk");   // 2048-bin digit counters + scan scratch
+    int cb = 1;
+    while (cb < 22 && ((uint64_t)n_chunks >> cb)) ++cb;
+    CK(launch_sort_segments(ctx->seg_a.p, ctx->seg_b.p, ns, cb, ctx->n_buckets, ctx->blk.p, ctx->seg_first.p,
+                            ctx->segs.p, s, &launches), "sort segments");
+    if (timing) cudaEventRecord(ctx->ev[8], s);
+  }
   t_host0 = std::chrono::steady_clock::now();
 
   // ---- A2: control resolution on the host -------------------------------------
@@ -767,7 +709,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
 
   // ---- A3b/A4/A5: replay ---------------------------------------------------------
   ReplayParams rp{};
-  rp.part_ev = ctx->part_ev.p; rp.reg_start = ctx->d_reg_start.p; rp.bucket_count = ctx->d_btotal.p;
+  rp.part_ev = ctx->part_ev.p; rp.segs = ctx->segs.p; rp.seg_first = ctx->seg_first.p;
   rp.n_buckets = ctx->n_buckets; rp.bucket_bits = ctx->bucket_bits; rp.n_words = ctx->n_words;
   rp.bucket_start = ctx->d_bucket_start.p;
   rp.items = ctx->d_items.p; rp.n_items = (uint32_t)ctx->items.size();

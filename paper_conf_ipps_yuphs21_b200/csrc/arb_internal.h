@@ -59,23 +59,19 @@ __host__ __device__ constexpr uint32_t sel8_clear(uint32_t d) { return sel8_set(
 // ---- compact event (partition output, 8 B) ---------------------------------
 // x: [0,30) word offset inside the address bucket | [30,32) access op (RH/WH/RT/WT)
 // y: record position inside the batch (< 2^30)
-// The partition writes every bucket's events contiguously, in trace order, into
-// the bucket's region [reg_start[b], reg_start[b] + reg_cap[b]) of part_ev.
 constexpr int kMaxBucketSpanBits = 30;               // buckets span <= 2^30 words
 constexpr uint32_t kMaxBatchRecords = 1u << 30;
+constexpr int kSegChunkBits = 21;                    // chunk id bits in the entry key (bit 21 in y)
 
 // ---- partition geometry ----------------------------------------------------
 constexpr int kPartThreads = 512;
+constexpr int kPartStages = 2;
 constexpr int kPartWarps = kPartThreads / 32;
-constexpr int kChunkRecords = 256;                  // records per chunk (one warp)
-constexpr int kTileRecords = kPartWarps * kChunkRecords;   // records per CTA tile (look-back unit)
+constexpr int kChunkRecords = 256;                  // records per chunk (one warp, independently)
+constexpr int kChunkCap = 2 * kChunkRecords;        // events per chunk (<= 2 words per access)
 constexpr int kBucketBits = 11;                    // bucket ids are 11-bit
 constexpr int kMaxBuckets = 1 << kBucketBits;
 constexpr uint32_t kBucketMask = kMaxBuckets - 1;
-// decoupled look-back status ring: kRingTiles slots of kMaxBuckets u64 entries
-// {tile + 1 : 24 | flag : 2 (1 aggregate, 2 inclusive prefix) | count : 38}; the
-// ring is cleared at the start of every partition launch
-constexpr uint32_t kRingTiles = 512;
 
 // ---- replay geometry -------------------------------------------------------
 constexpr int kReplayThreads = 256;
@@ -103,11 +99,10 @@ struct DevStats {
   unsigned long long range_words_applied;
   unsigned long long n_mir_cand;
   unsigned long long steps_fast, steps_sort;
-  unsigned long long overflow;        // a bucket received more events than its region holds
+  unsigned long long n_segs;          // (chunk, bucket) segment entries written by k_partition
   unsigned long long n_carry_out;     // N2: access summaries of instances carried into the next flush
   unsigned long long n_bo_cand;       // N1 (Z25): base-tag overflow candidates
-  unsigned long long tile_ticket;     // k_partition: next CTA tile to take (in order)
-  unsigned long long pad[1];
+  unsigned long long pad[2];
 };
 
 // control record extracted by the partition kernel
@@ -145,21 +140,20 @@ struct PartParams {
   uint64_t base_word, n_words;            // tracked words [base_word, base_word + n_words)
   uint32_t coarse_bits; const uint32_t* bin_map;
   uint32_t bucket_bits, n_buckets;
-  uint32_t n_chunks, n_tiles;
-  uint2* part_ev;                         // bucket regions (events)
-  const uint64_t* reg_start;              // [kMaxBuckets] first event slot of each bucket's region
-  const uint32_t* reg_cap;                // [kMaxBuckets] region capacity (events)
-  unsigned long long* ring;               // [kRingTiles][kMaxBuckets] look-back status (zeroed)
-  uint64_t* bucket_total;                 // [kMaxBuckets] events per bucket (written by the last tile)
+  uint32_t n_chunks;
+  uint2* part_ev;                         // [n_chunks][kChunkCap]
+  uint2* seg_out; uint64_t seg_cap;       // {bucket << 21 | chunk bits 0-20, start | len << 16 | chunk
+                                          // bit 21 << 31} per touched bucket of a chunk
   CtlRec* ctl; uint64_t ctl_cap;
   DevStats* st;
   uint32_t n_dev;                         // accelerators (Z24): > 1 puts the device of RT/WT in pos bits 30-31
 };
 
 struct ReplayParams {
-  const uint2* part_ev;                   // bucket regions (trace order inside each)
-  const uint64_t* reg_start;              // [n_buckets] first event of each bucket
-  const uint64_t* bucket_count;           // [n_buckets] events of each bucket
+  const uint2* part_ev;
+  const uint4* segs;                      // segment entries sorted by (bucket, chunk); .w = exclusive
+                                          // prefix of the event counts over the sorted array
+  const uint32_t* seg_first;              // [n_buckets + 1] first entry of each bucket
   uint32_t n_buckets, bucket_bits;
   const uint64_t* bucket_start;           // [n_buckets + 1] first relative word of each bucket
   const uint4* items; uint32_t n_items;   // work items in scheduling order (largest first):
@@ -210,12 +204,12 @@ cudaError_t launch_cut(uint32_t* hist_map, uint32_t n_bins, uint32_t coarse_bits
                        uint32_t max_buckets, uint64_t* bucket_start, uint32_t* weight, uint32_t* first_bin,
                        uint32_t* nb_out, uint32_t* scratch, cudaStream_t s, int* launches);
 cudaError_t launch_partition(const PartParams& p, cudaStream_t s);
-// Bucket regions from sampled weights: cap[b] covers the estimate weight[b] * stride
-// with a margin (even), reg_start = exclusive prefix (even), total <= capacity
-// events (else the caps are scaled down: the partition then overflows and the
-// host retries with exact counts).  nb: device bucket count (or nullptr: n_fixed).
-cudaError_t launch_regions(const uint32_t* weight, const uint32_t* nb, uint32_t n_fixed, double stride,
-                           uint64_t capacity, uint64_t* reg_start, uint32_t* reg_cap, cudaStream_t s);
+// Sorts the 8-B segment entries {bucket << 21 | chunk, start | len << 16 | chunk bit 21 << 31}
+// by (bucket, chunk) (a, b: ping-pong buffers), writes the replay form
+// {chunk, bucket, start | len << 16, exclusive event prefix} to out and each
+// bucket's first entry; cnt: (n / 4096 + 1) * 256 + 4096 u32
+cudaError_t launch_sort_segments(uint2* a, uint2* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
+                                 uint32_t* first, uint4* out, cudaStream_t s, int* launches);
 cudaError_t launch_replay(const ReplayParams& p, int n_ctas, cudaStream_t s);
 // K5 phase 2: for every hot bucket {bucket, slices, span, 0} carry the states
 // across its slices: P_0 = shadow, P_{k+1} = F_k(P_k); shadow = F_last(P_last)

@@ -304,6 +304,97 @@ static int add_field_passes(RsPass* ps, int np, int field, int bits) {
   return np;
 }
 
+// Segment entries as written by k_partition (8 B): x = bucket << 21 | chunk bits
+// 0-20, y = start | len << 16 | chunk bit 21 << 31 (start, len <= 512).
+__device__ __forceinline__ uint32_t seg_bucket(uint2 e) { return e.x >> kSegChunkBits; }
+__device__ __forceinline__ uint32_t seg_len(uint2 e) { return (e.y >> 16) & 0x3FFu; }
+__device__ __forceinline__ uint32_t seg_chunk(uint2 e) {
+  return (e.x & ((1u << kSegChunkBits) - 1u)) | ((e.y >> 31) << kSegChunkBits);
+}
+
+// first entry of every bucket in the sorted entries
+__global__ void k_seg_first(const uint2* segs, uint64_t n, uint32_t n_buckets, uint32_t* first) {
+  for (uint32_t b = blockIdx.x * blockDim.x + threadIdx.x; b <= n_buckets; b += gridDim.x * blockDim.x) {
+    uint64_t a = 0, z = n;                 // first entry with bucket >= b
+    while (a < z) { const uint64_t mid = (a + z) >> 1; if (seg_bucket(segs[mid]) < b) a = mid + 1; else z = mid; }
+    first[b] = (uint32_t)a;
+  }
+}
+
+// event count of each tile of sorted entries (blocked: thread t owns 8 entries)
+__global__ void __launch_bounds__(kRsThreads) k_seg_tile_sum(const uint2* segs, uint64_t n, uint32_t* blk) {
+  __shared__ uint32_t red[kRsThreads / 32];
+  const uint64_t base = (uint64_t)blockIdx.x * kRsTile + (uint64_t)threadIdx.x * kRsItems;
+  uint32_t c = 0;
+#pragma unroll
+  for (int j = 0; j < kRsItems; ++j)
+    if (base + j < n) c += seg_len(segs[base + j]);
+  for (int d = 16; d; d >>= 1) c += __shfl_xor_sync(FULL, c, d);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = c;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t t = 0;
+    for (int w = 0; w < kRsThreads / 32; ++w) t += red[w];
+    blk[blockIdx.x] = t;
+  }
+}
+// replay form {chunk, bucket, start | len << 16, exclusive event prefix over the array}
+__global__ void __launch_bounds__(kRsThreads) k_seg_cum(const uint2* segs, uint64_t n, const uint32_t* blk,
+                                                        uint4* out) {
+  __shared__ uint32_t ws[kRsThreads / 32];
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint64_t base = (uint64_t)blockIdx.x * kRsTile + (uint64_t)threadIdx.x * kRsItems;
+  uint2 e[kRsItems];
+  uint32_t c = 0;
+#pragma unroll
+  for (int j = 0; j < kRsItems; ++j) {
+    e[j] = base + j < n ? segs[base + j] : make_uint2(0, 0);
+    c += seg_len(e[j]);
+  }
+  uint32_t incl = c;
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint32_t o = __shfl_up_sync(FULL, incl, d);
+    if (lane >= (uint32_t)d) incl += o;
+  }
+  if (lane == 31) ws[warp] = incl;
+  __syncthreads();
+  uint32_t run = blk[blockIdx.x] + incl - c;
+  for (uint32_t w = 0; w < warp; ++w) run += ws[w];
+#pragma unroll
+  for (int j = 0; j < kRsItems; ++j) {
+    if (base + j < n)
+      out[base + j] = make_uint4(seg_chunk(e[j]), seg_bucket(e[j]), e[j].y & 0x3FFFFFFu, run);
+    run += seg_len(e[j]);
+  }
+}
+
+cudaError_t launch_sort_segments(uint2* a, uint2* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
+                                 uint32_t* first, uint4* out, cudaStream_t s, int* launches) {
+  RsPass ps[8];
+  int np = 0;
+  const int lo_bits = chunk_bits < kSegChunkBits ? chunk_bits : kSegChunkBits;
+  np = add_field_passes(ps, np, 0, lo_bits);
+  if (chunk_bits > kSegChunkBits) ps[np++] = RsPass{1, 31, 1};    // chunk bit 21 (batches > 2^29 records)
+  {
+    int nbb = 1;
+    while ((1u << nbb) < n_buckets) ++nbb;                      // bucket bits actually used
+    for (int sh = kSegChunkBits, k = 0; k < 1; ++k) ps[np++] = RsPass{0, sh, nbb};
+  }
+  cudaError_t e = cudaSuccess;
+  if (n) e = radix_sort(a, b, n, ps, np, cnt, s, launches);
+  if (e != cudaSuccess) return e;
+  if (n) {
+    const uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
+    k_seg_tile_sum<<<nblk, kRsThreads, 0, s>>>(a, n, cnt);
+    scan_u32(cnt, nblk, cnt + nblk, s, launches);
+    k_seg_cum<<<nblk, kRsThreads, 0, s>>>(a, n, cnt, out);
+    *launches += 2;
+  }
+  k_seg_first<<<(n_buckets + 256) / 256, 256, 0, s>>>(a, n, n_buckets, first);
+  *launches += 1;
+  return cudaGetLastError();
+}
+
 cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches) {
   cudaMemsetAsync(p.n_out, 0, 8 * sizeof(unsigned long long), s);
   if (p.n_cand == 0) return cudaGetLastError();

@@ -1,14 +1,16 @@
 // replay.cu — A3b + A4 + A5: per-address replay of each bucket.
 //
 // One CTA per address bucket at a time (persistent; buckets in largest-first
-// order).  The bucket's events are one contiguous array in trace order (the
-// partition's bucket region); the CTA streams it step by step into shared memory
-// with one TMA bulk copy per step (cp.async.bulk, double-buffered on two
-// mbarriers: the next step arrives while this one runs), applies the resolved range ops
+// order).  The bucket's events are the segments of its sorted segment entries
+// (chunk order = trace order); the CTA gathers them step by step through a
+// staged window of entries (cp.async, double-buffered), applies the resolved range ops
 // (Table I transfers / allocate / release; target update P:121) to
 // the bucket's shadow at their trace positions, and processes the events in
 // steps of <= 1024 that never straddle a range op:
 //
+//   direct step (at most one write per word, every word within +-4096 of the
+//              step's first word): a direct-mapped table word - anchor -> the
+//              word's write, no hashing or probing; else
 //   fast step  (every word has at most one write in the step): a shared-memory
 //              hash of the written words, word -> write position.  A read's
 //              state-before is the initial state, or the image of the one
@@ -34,6 +36,7 @@ constexpr int RT = kReplayThreads;           // threads per CTA (>= 256)
 constexpr int RI = kReplayItems;             // events per thread per step
 constexpr int STEP = RT * RI;                // 2048 events per step
 static_assert(RT >= 256 && STEP <= 4096, "sort_pass digit loop and u16 offsets");
+constexpr int kWin = 2 * RT;                 // segment descriptors staged per step
 constexpr int kHSlots = 4096;                // hash slots (load <= 1/2)
 constexpr int kDSlots = 2 * kHSlots;         // direct-step window (words), same bytes as the hash
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
@@ -42,15 +45,15 @@ constexpr int kZSlots = 2048;                // summary-step hash slots (<= 1024
 static_assert(kZSlots * 12 <= kHSlots * 8 && kZSlots >= 2 * STEP, "summary hash fits the hash area");
 
 struct ReplaySmem {
-  uint2 ev[2][STEP + 2];          // double-buffered step events {key, pos} (bulk copies; an odd
-                                  //   first event lands at index 1 so the source stays 16-B aligned)
-  uint64_t bar[2];                // their mbarriers
+  uint2 ev[2][STEP];              // double-buffered step events {key, pos} (cp.async)
   union {
     struct { uint32_t keyA[STEP], posA[STEP], keyB[STEP], posB[STEP]; uint16_t hist[RT / 32][256]; } s;
     struct { uint2 slot[kHSlots]; } h;      // fast step: written words {word, pos << 2 | op}
     struct { uint32_t w[kDSlots]; } d;      // direct step: word - anchor -> {step index << 4 | write code}
     struct { uint32_t key[kZSlots], lastw[kZSlots], anyw[kZSlots]; } z;  // hot-slice summary step (K5)
   } u;
+  uint32_t wstart[kWin];          // staged segment list window: global event index
+  uint32_t wcum[kWin + 1];        //   and bucket-relative first event of each segment
   uint32_t pref[256];             // radix digit scratch
   uint32_t red[RT / 32], red2[RT / 32], wscan[RT / 32];
   uint32_t wcnt[RT / 32], wev[RT / 32];
@@ -62,8 +65,8 @@ struct ReplaySmem {
   uint8_t* shrel;                 // state of bucket-relative word w: shrel[w]
   uint16_t* fsum;                 // summary slice: composed transition of word w: fsum[w]
   uint32_t slice, n_slices;       // hot bucket slice (kItemSlice / kItemSummary)
-  uint32_t n_events, evoff[2];
-  uint64_t bucket_base, ev_base;
+  uint32_t seg0, cum0, n_segs, n_events, wsc, nwin;
+  uint64_t bucket_base;
 };
 
 // ---- block-level helpers ----------------------------------------------------
@@ -733,9 +736,15 @@ __device__ void step_summary(ReplaySmem& S, const uint2* ev, uint32_t m) {
   __syncthreads();
 }
 
-// Position of event e of the bucket.
-__device__ __forceinline__ uint32_t event_pos(const ReplaySmem& S, const ReplayParams& p, uint32_t e) {
-  return p.part_ev[S.ev_base + e].y;
+// Position of event e of the bucket (one thread).
+__device__ uint32_t event_pos(const ReplaySmem& S, const ReplayParams& p, uint32_t e) {
+  uint32_t lo = 0, z = S.n_segs;
+  while (z - lo > 1) {
+    const uint32_t mid = (lo + z) >> 1;
+    if (p.segs[S.seg0 + mid].w - S.cum0 <= e) lo = mid; else z = mid;
+  }
+  const uint4 sg = p.segs[S.seg0 + lo];
+  return p.part_ev[(uint64_t)sg.x * kChunkCap + (sg.z & 0xFFFFu) + (e - (sg.w - S.cum0))].y;
 }
 // first op of the bucket (ops [a, z), trace order) at or after position q
 __device__ uint32_t ops_lower_bound(const ReplayParams& p, uint32_t a, uint32_t z, uint32_t q) {
@@ -772,20 +781,131 @@ cudaError_t launch_carry(const uint4* hot, uint32_t n_hot, uint32_t max_span, co
   return cudaGetLastError();
 }
 
-// ---- the bucket's events: stream [e0, e0 + m) into buffer k ------------------------------
-// One thread issues the bulk copy; the events sit at S.ev[k] + S.evoff[k].  Regions
-// start at even slots, so the source is 16-B aligned when rounded down to an even
-// event; the copy may read one event past the step (inside the allocation).
-__device__ __forceinline__ uint32_t issue_step(ReplaySmem& S, const ReplayParams& p, uint32_t e0, uint32_t total,
-                                               uint32_t k) {
-  const uint32_t m = min((uint32_t)STEP, total - e0);
+// ---- the bucket's segments -------------------------------------------------------------
+// The sorted entries of bucket b are p.segs[f0, f1) in chunk order (= trace
+// order); entry i covers bucket-relative events [segs[i].w - segs[f0].w, + len)
+// stored at part_ev[chunk * kChunkCap + start].
+__device__ void bucket_setup(ReplaySmem& S, const ReplayParams& p, uint32_t b) {
   if (threadIdx.x == 0) {
-    const uint32_t odd = e0 & 1u;
-    const uint32_t bytes = ((m + odd + 1u) & ~1u) * 8u;
-    S.evoff[k] = odd;
-    mbar_arrive_tx(&S.bar[k], bytes);
-    bulk_g2s(S.ev[k], p.part_ev + S.ev_base + (e0 - odd), bytes, &S.bar[k]);
+    const uint32_t f0 = p.seg_first[b], f1 = p.seg_first[b + 1];
+    S.seg0 = f0; S.n_segs = f1 - f0;
+    S.cum0 = 0; S.n_events = 0;
+    if (f1 > f0) {
+      const uint4 first = p.segs[f0], last = p.segs[f1 - 1];
+      S.cum0 = first.w;
+      S.n_events = last.w + (last.z >> 16) - first.w;
+    }
+    S.wsc = 0; S.nwin = 0; S.wcum[0] = 1;      // empty window: forces a load
   }
+  __syncthreads();
+}
+
+// Make the staged window of segment descriptors contain event e0 (reloads
+// about every kWin segments; sequential progress needs no search).
+__device__ void ensure_window(ReplaySmem& S, const ReplayParams& p, uint32_t e0, uint32_t& hint) {
+  if (e0 >= S.wcum[0] && e0 < S.wcum[S.nwin]) return;
+  hint = 0;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t a;
+    if (S.nwin && e0 == S.wcum[S.nwin]) {
+      a = S.wsc + S.nwin;                       // the window's successor
+    } else {                                    // last segment starting at or before e0
+      uint32_t lo = 0, z = S.n_segs;
+      while (z - lo > 1) {
+        const uint32_t mid = (lo + z) >> 1;
+        if (p.segs[S.seg0 + mid].w - S.cum0 <= e0) lo = mid; else z = mid;
+      }
+      a = lo;
+    }
+    S.wsc = a;
+    S.nwin = min((uint32_t)kWin, S.n_segs - a);
+  }
+  __syncthreads();
+  const uint32_t sc = S.wsc, nwin = S.nwin;
+  const uint4* segs = p.segs + S.seg0 + sc;
+  for (uint32_t k = threadIdx.x; k < nwin; k += RT) {
+    const uint4 e = segs[k];
+    S.wstart[k] = e.x * (uint32_t)kChunkCap + (e.z & 0xFFFFu);
+    S.wcum[k] = e.w - S.cum0;
+  }
+  if (threadIdx.x == 0) S.wcum[nwin] = sc + nwin < S.n_segs ? segs[nwin].w - S.cum0 : S.n_events;
+  __syncthreads();
+}
+
+// Issue cp.async copies of events [e0, e0 + m) of the bucket into dst; the
+// window must contain e0.  Returns m (<= STEP, clipped to the window).
+// `hint` (per thread, block-uniform) is a window segment index with
+// wcum[hint] <= e0; it is advanced to the last segment gathered.
+__device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t e0, uint32_t total, uint2* dst,
+                                 uint32_t& hint) {
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t nwin = S.nwin;
+  const uint32_t m = min(min((uint32_t)STEP, total - e0), S.wcum[nwin] - e0);
+  // Warp w gathers the slice [e0 + 32*RI*w, +32*RI) of the step.  Segment j holds
+  // event e iff wcum[j] <= e < wcum[j+1]; every warp counts, from the hint, the
+  // segments starting at or before its slice start and before the step's last
+  // event (ballots, no barrier), then each lane walks forward to the segment of
+  // each of its events (segments are usually longer than the slice).
+  const uint32_t s0 = e0 + warp * (32 * RI), last = e0 + m - 1;
+  const uint32_t base0 = hint & ~31u;
+  uint32_t c0 = 0, c1 = 0;
+  for (uint32_t base = base0; base < nwin; base += 32) {
+    const uint32_t j = base + lane;
+    const uint32_t w = j < nwin ? S.wcum[j] : 0xFFFFFFFFu;
+    c0 += __popc(__ballot_sync(FULL, w <= s0));
+    const uint32_t b1 = __ballot_sync(FULL, w <= last);
+    c1 += __popc(b1);
+    if (b1 != FULL) break;
+  }
+  hint = base0 + c1 - 1;                 // segment of the step's last event
+  if (s0 < e0 + m) {
+    uint32_t seg = base0 + c0 - 1, seg_end = S.wcum[seg + 1];
+    // event e of segment seg sits at part_ev[wstart[seg] + e - wcum[seg]] = bp[e]
+    int64_t bp = (int64_t)S.wstart[seg] - (int64_t)S.wcum[seg];
+    const uint32_t s_end = min(s0 + 32 * RI, e0 + m);
+    if (s_end <= seg_end) {
+      // the whole slice lies in one segment (warp-uniform; the common case):
+      // a contiguous copy, 16 B per lane when both sides are 16-B aligned
+      const uint2* src = p.part_ev + (bp + s0);
+      uint2* d = dst + (s0 - e0);
+      const uint32_t cnt = s_end - s0;
+      if (cnt == 32 * RI && ((reinterpret_cast<uintptr_t>(src) & 15u) == 0)) {
+#pragma unroll
+        for (int k = 0; k < RI / 2; ++k) cp_async16(d + 2 * (lane + 32 * k), src + 2 * (lane + 32 * k));
+      } else {
+#pragma unroll
+        for (int k = 0; k < RI; ++k)
+          if (lane + 32 * k < cnt) cp_async8(d + lane + 32 * k, src + lane + 32 * k);
+      }
+      cp_async_commit();
+      return m;
+    }
+    uint2* d = dst + (s0 - e0) + lane;
+    if (seg + 2 <= nwin && s_end <= S.wcum[seg + 2]) {
+      // two segments: select the base per event
+      const int64_t bp1 = (int64_t)S.wstart[seg + 1] - (int64_t)seg_end;
+#pragma unroll
+      for (int k = 0; k < RI; ++k) {
+        const uint32_t e = s0 + k * 32 + lane;
+        if (e < s_end) cp_async8(d + k * 32, p.part_ev + ((e < seg_end ? bp : bp1) + e));
+      }
+      cp_async_commit();
+      return m;
+    }
+#pragma unroll
+    for (int k = 0; k < RI; ++k) {
+      const uint32_t e = s0 + k * 32 + lane;
+      if (e < e0 + m) {
+        if (e >= seg_end) {
+          do { ++seg; seg_end = S.wcum[seg + 1]; } while (e >= seg_end);
+          bp = (int64_t)S.wstart[seg] - (int64_t)S.wcum[seg];
+        }
+        cp_async8(d + k * 32, p.part_ev + (bp + e));
+      }
+    }
+  }
+  cp_async_commit();
   return m;
 }
 
@@ -797,9 +917,6 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
   ReplaySmem& S = *reinterpret_cast<ReplaySmem*>(smem_raw);
   const uint32_t tid = threadIdx.x;
   hash_clear(S);
-  if (tid == 0) { mbar_init(&S.bar[0], 1); mbar_init(&S.bar[1], 1); }
-  fence_mbar_init();
-  uint32_t bph = 0;                    // parity of each buffer's mbarrier (bit k)
   for (;;) {
     if (tid == 0) {
       const unsigned long long w = atomicAdd(&p.st->work, 1ull);
@@ -823,11 +940,9 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       S.op_end = p.ops_start[b + 1];
       S.bucket_base = p.bucket_start[b];
       S.shrel = p.shadow + S.bucket_base;
-      S.ev_base = p.reg_start[b];
-      S.n_events = (uint32_t)p.bucket_count[b];
       S.skip_direct = 0;
     }
-    __syncthreads();
+    bucket_setup(S, p, b);
     uint32_t first = 0, total = S.n_events;
     if (mode >= kItemSlice) {
       // hot bucket slice k of n: events [k E / n, (k+1) E / n) and the range ops
@@ -859,14 +974,23 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
     }
     if (tid == 0) S.next_op = S.op_cur < S.op_end ? p.ops[S.op_cur].pos : 0xFFFFFFFFu;
     __syncthreads();
-    uint32_t e0 = first, cur = 0, m_cur = 0;
-    if (e0 < total) m_cur = issue_step(S, p, e0, total, 0);
+    uint32_t e0 = first, cur = 0, m_cur = 0, hint = 0;
+    if (e0 < total) {
+      ensure_window(S, p, e0, hint);
+      m_cur = issue_gather(S, p, e0, total, S.ev[0], hint);
+    }
     while (e0 < total) {
-      mbar_wait(&S.bar[cur], (bph >> cur) & 1u);
-      bph ^= 1u << cur;
-      __syncthreads();                 // the other buffer's readers are done: it may be refilled
-      const uint2* ev = S.ev[cur] + S.evoff[cur];
+      cp_async_wait_all();
+      __syncthreads();
+      const uint2* ev = S.ev[cur];
       const uint32_t m = m_cur;
+      // ---- prefetch the next step's events (assumes the step is not cut) ---------
+      const uint32_t nxt = e0 + m;
+      uint32_t m_nxt = 0;
+      if (nxt < total) {
+        ensure_window(S, p, nxt, hint);
+        m_nxt = issue_gather(S, p, nxt, total, S.ev[cur ^ 1], hint);
+      }
       // ---- range ops before the first event, then cut at the next one -------------
       constexpr uint32_t pm = MD ? kMdPos : 0xFFFFFFFFu;   // MD: strip the device bits (Z24)
       apply_ops_before<BO, MD>(S, p, ev[0].y & pm);
@@ -876,9 +1000,6 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         for (uint32_t e = tid; e < m; e += RT) cnt += (ev[e].y & pm) < S.next_op;
         cut = block_sum(cnt, S.red);
       }
-      // ---- prefetch the next step (from the cut) ---------------------------------------
-      const uint32_t nxt = e0 + cut;
-      const uint32_t m_nxt = nxt < total ? issue_step(S, p, nxt, total, cur ^ 1u) : 0u;
       if (mode == kItemSummary) {
         step_summary<UM>(S, ev, cut);
       } else {
@@ -903,8 +1024,17 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         }
       }
       e0 += cut;
-      cur ^= 1u;
-      m_cur = m_nxt;
+      if (cut == m) {
+        cur ^= 1;
+        m_cur = m_nxt;
+      } else {
+        // the prefetch started at e0_old + m: drain it and gather from e0
+        cp_async_wait_all();
+        __syncthreads();
+        hint = 0;
+        ensure_window(S, p, e0, hint);
+        m_cur = issue_gather(S, p, e0, total, S.ev[cur], hint);
+      }
     }
     // the ops after the last event (a slice replay's private states are not kept)
     if (mode != kItemSlice) apply_ops_before<BO, MD>(S, p, 0xFFFFFFFFu);
