@@ -11,9 +11,10 @@ resolution, replay + classification, MIR join, report compaction, count
 exchange) over the whole named workload.  Default: config 5, the 9.0e9-record
 trace over 2^33 words (64 GiB of locations) -- strong scaling: rank r of N owns
 the words [r * 2^33 / N, (r + 1) * 2^33 / N) and replays every record touching
-them (all control records replicated).  The trace is cut into 8
+them (all control records replicated).  The trace is cut into 9
 time batches at quiescent points ("1-GPU = the same total trace,
-in 8 quiescent batches"); each batch is generated on the device (untimed) and its
+in quiescent batches"; 9 so that each batch is one flush of <= 2^30 records,
+the ABI's maximum); each batch is generated on the device (untimed) and its
 flushes are timed with CUDA events on the replay stream between a barrier + a
 synchronize; a step's time is the sum over batches of the max over ranks.
 Events = word-events: one per (tracked word, data op).
@@ -34,7 +35,8 @@ sys.path.insert(0, ROOT)
 
 METRIC = "events/sec replayed (1/2/4/8 B200) and % of HBM roofline; vs CPU oracle"
 UNIT = "word-events/s"
-MAX_FLUSH = 1 << 29          # records per flush (cut at the last quiescent point below it)
+MAX_FLUSH = 1 << 30          # records per flush: the ABI's maximum batch (arb_submit_events)
+DEFAULT_BATCHES = 9          # config 5: 9 quiescent time batches of ~1.0e9 records -> one flush each
 
 
 def peaks():
@@ -198,14 +200,18 @@ class BatchSource:
             local_q = (q - g0).tolist()
         else:
             local_q = torch.searchsorted(gidx, torch.tensor(q, device=self.device)).cpu().numpy().tolist()
+        # as few flushes as the 2^30-record limit allows, cut near equal sizes
+        nf = max(1, -(-k // MAX_FLUSH))
         cuts = [0]
-        last = 0
-        for a in local_q + [k]:
-            if a - cuts[-1] > MAX_FLUSH and last > cuts[-1]:
-                cuts.append(last)
-            last = a
+        qa = np.asarray(local_q, dtype=np.int64)
+        for j in range(1, nf):
+            want = k * j // nf
+            ok = qa[(qa > cuts[-1]) & (qa - cuts[-1] <= MAX_FLUSH)]
+            if ok.size:
+                cuts.append(int(ok[np.argmin(np.abs(ok - want))]))
         if cuts[-1] != k:
             cuts.append(k)
+        assert all(b - a <= MAX_FLUSH for a, b in zip(cuts[:-1], cuts[1:])), "no quiescent cut below 2^30 records"
         flushes = [(a, b) for a, b in zip(cuts[:-1], cuts[1:]) if b > a] or [(0, 0)]
         return recs, gidx, flushes
 
@@ -427,7 +433,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="config5")
     ap.add_argument("--scale", type=float, default=1.0)
-    ap.add_argument("--batches", type=int, default=8, help="time batches of the trace (quiescent cuts)")
+    ap.add_argument("--batches", type=int, default=DEFAULT_BATCHES, help="time batches of the trace (quiescent cuts)")
     ap.add_argument("--max-batches", type=int, default=0, help="profiling: replay only the first K batches")
     ap.add_argument("--e2e-steps", type=int, default=1)
     ap.add_argument("--no-e2e", action="store_true")

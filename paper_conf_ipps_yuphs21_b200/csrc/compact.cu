@@ -273,6 +273,40 @@ cudaError_t launch_dedup_rehash(const unsigned long long* old, uint64_t n_old, u
   return cudaGetLastError();
 }
 
+// dedup-first (Z3): the kept candidates are sorted by (word, kind, pos) and hold at
+// most one element per (word, kind), so a word's group has <= 8 elements; the
+// canonical order (word, pos, kind) is a rank inside the group.  Writes the
+// arb_report records (as k_keep_write with final_out) and the per-kind counts.
+__global__ void k_dedup_canonical(const uint4* a, uint64_t n, uint4* out, uint64_t base_word, const uint64_t* gidx,
+                                  uint64_t index_base, unsigned long long* n_out) {
+  uint32_t kc[5] = {0, 0, 0, 0, 0};
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint4 x = a[i];
+    uint64_t g0 = i, g1 = i + 1;
+    while (g0 > 0 && i - g0 < 8 && a[g0 - 1].x == x.x && a[g0 - 1].y == x.y) --g0;
+    while (g1 < n && g1 - i < 8 && a[g1].x == x.x && a[g1].y == x.y) ++g1;
+    uint32_t rank = 0;
+    for (uint64_t j = g0; j < g1; ++j) {
+      const uint4 y = a[j];
+      rank += (y.z < x.z) || (y.z == x.z && y.w < x.w);
+    }
+    const uint64_t word = ((uint64_t)x.x | ((uint64_t)x.y << 32)) + base_word;
+    const uint64_t w0 = (word & kMask48) | ((uint64_t)x.w << 48);
+    const uint64_t w1 = gidx ? gidx[x.z] : index_base + x.z;
+    out[g0 + rank] = make_uint4((uint32_t)w0, (uint32_t)(w0 >> 32), (uint32_t)w1, (uint32_t)(w1 >> 32));
+    const uint32_t kd = x.w & 7u;
+    kc[kd < 5 ? kd : 0]++;
+  }
+  const uint32_t lane = threadIdx.x & 31;
+#pragma unroll
+  for (int k = 1; k < 5; ++k) {
+    uint32_t v = kc[k];
+    for (int d = 16; d; d >>= 1) v += __shfl_xor_sync(FULL, v, d);
+    if (lane == 0 && v) atomicAdd(&n_out[k], (unsigned long long)v);
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) n_out[0] = n;
+}
+
 template <class E>
 static cudaError_t radix_sort(E*& a, E*& b, uint64_t n, const RsPass* passes, int np, uint32_t* cnt,
                               cudaStream_t s, int* launches) {
@@ -438,6 +472,11 @@ cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches
       t = a; a = b; b = t;
     }
     if (n == 0) return cudaGetLastError();     // every pair was reported by an earlier flush
+    // canonical order inside each word's group of <= 8 (one per kind): no second sort
+    k_dedup_canonical<<<(unsigned)std::min<uint64_t>((n + 255) / 256, 148 * 8), 256, 0, s>>>(
+        a, n, p.out, p.base_word, p.gidx, p.index_base, p.n_out);
+    *launches += 1;
+    return cudaGetLastError();
   }
   if (p.pos_bits + kKindBits <= 32) {
     np = add_field_passes(ps, np, 4, p.pos_bits + kKindBits); // record, then kind

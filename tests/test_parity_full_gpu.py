@@ -3,9 +3,9 @@ configuration bench.py times (north_star: "GPU reports must match the oracle
 bit-exactly, as the same report set ... on all configs").
 
 * config 5: the whole 9.0e9-record trace over 2^33 words (64 GiB of locations),
-  replayed exactly as the N = 1 bench line replays it -- 8 time batches cut at
-  quiescent points, each generated on the device and cut into flushes of at most
-  2^29 records -- compared batch by batch with the oracle (address-sharded over
+  replayed exactly as the N = 1 bench line replays it -- 9 time batches cut at
+  quiescent points, each generated on the device and replayed as one flush of at
+  most 2^30 records -- compared batch by batch with the oracle (address-sharded over
   the host cores, continuing from the previous batch's final shadow), then the
   whole 8 GiB final shadow byte for byte;
 * configs 3 and 4: the whole trace of each (1.0e9 / 0.89e9 records; config 4 with
@@ -75,7 +75,7 @@ def test_config5_whole_trace_exact(orc):
     from paper_conf_ipps_yuphs21_b200 import Context, ARB_F_TIMING
     prog = bench.make_program("config5")
     lo, hi = bench.rank_range(prog, 0, 1)
-    batches = bench.time_batches(prog, 8)
+    batches = bench.time_batches(prog, bench.DEFAULT_BATCHES)
     src = bench.BatchSource(prog, lo, hi, torch.device("cuda", 0))
     ctx = Context(lo * 8, (hi - lo) * 8, flags=ARB_F_TIMING, report_capacity=1 << 25)
     shadow = None
@@ -105,7 +105,7 @@ def test_config5_whole_trace_dedup_first(orc):
     from paper_conf_ipps_yuphs21_b200 import Context, ARB_F_TIMING, ARB_F_DEDUP_FIRST
     prog = bench.make_program("config5")
     lo, hi = bench.rank_range(prog, 0, 1)
-    batches = bench.time_batches(prog, 8)[:3]          # the first three batches (the state carries)
+    batches = bench.time_batches(prog, bench.DEFAULT_BATCHES)[:3]   # the first three batches (the state carries)
     src = bench.BatchSource(prog, lo, hi, torch.device("cuda", 0))
     ctx = Context(lo * 8, (hi - lo) * 8, flags=ARB_F_TIMING | ARB_F_DEDUP_FIRST, report_capacity=1 << 25)
     shadow = None
