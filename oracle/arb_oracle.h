@@ -45,6 +45,8 @@ extern "C" {
 #endif
 
 /* Trace record: two little-endian 64-bit words.
+ * (CV translation, Z26: parity pinned by brute force vs the value simulator's own
+ * CV-address table, tests/test_oracle_bruteforce.py.)
  * w0: [0,48) byte address | [48,56) op | [56,64) arg (map-type or update dir)
  * w1: [0,48) length in bytes          | [48,64) task id (TASK_BEGIN/END, SYNC) */
 typedef struct { uint64_t w0, w1; } orc_record;
@@ -55,9 +57,16 @@ enum { ORC_RH = 0, ORC_WH = 1, ORC_RT = 2, ORC_WT = 3,
        ORC_TASK_BEGIN = 12, ORC_TASK_END = 13, ORC_SYNC = 14,
        ORC_TASK_DEPEND = 15 /* inside a block: the task depends on the last ended
                                instance of task id k (N4, reading Z22) */,
-       ORC_BASE = 11        /* pointer tag k (task-id field, 1..0xFFFF) now has the base
+       ORC_BASE = 11,       /* pointer tag k (task-id field, 1..0xFFFF) now has the base
                                byte address of this record (LLVM IR base; N1,
-                               reading Z25); no word-ops */ };
+                               reading Z25); no word-ops */
+       ORC_CV_BASE = 16     /* the mapping entry holding OV byte address w0[0,48) has its CV
+                               at device address w1[0,48) for that byte (N1, reading Z26);
+                               no word-ops */ };
+/* arg bit of RT / WT (reading Z26): the record's address is a CV (device) address,
+ * translated to the OV address through the mapping entries' CV intervals (the
+ * interval tree of P:269); a CV address in no entry's CV is not tracked */
+#define ORC_CV_ADDR 0x80u
 /* map-types (Table I) */
 enum { ORC_TO = 0, ORC_FROM = 1, ORC_TOFROM = 2, ORC_ALLOC = 3,
        ORC_RELEASE = 4, ORC_DELETE = 5 };

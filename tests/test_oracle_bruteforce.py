@@ -367,3 +367,122 @@ def test_bo_base_tags_fuzz_programs(orc, seed):
     res = orc.replay(rec, base, span, detect_bo=True)
     assert res.rc == 0
     assert [t for t in res.triples() if t[2] != 3] == expect
+
+
+# ---- CV -> OV translation (P:269 interval tree, reading Z26) --------------------------------
+CV_BASE_OP, CV_ADDR = 16, 0x80
+
+
+def alphabet_cv():
+    """Two words A (0) and B (1): target accesses by OV address or by CV address
+    (the CV of the entry holding the word, or a stray one), host accesses, entering
+    / exiting A, B or both, and the runtime's CV placement records (CV_BASE) --
+    including a wrong one (B's CV placed where A's is)."""
+    sym = []
+    for op in (OP.RT, OP.WT):
+        for w in (0, 1):
+            sym.append(("acc", op, w * 8, 8, 0))
+        for c in (0, 8, 16):                              # CV byte offsets (16: past both)
+            sym.append(("cva", op, c, 8, CV_ADDR))
+    for op in (OP.RH, OP.WH):
+        for w in (0, 1):
+            sym.append(("acc", op, w * 8, 8, 0))
+    for lo, hi in ((0, 1), (1, 2), (0, 2)):
+        for t in (MAP.TO, MAP.ALLOC):
+            sym.append(("ctl", OP.MAP_ENTER, lo * 8, (hi - lo) * 8, t))
+        for t in (MAP.FROM, MAP.RELEASE):
+            sym.append(("ctl", OP.MAP_EXIT, lo * 8, (hi - lo) * 8, t))
+    sym += [("cvb", 0, 0), ("cvb", 8, 8), ("cvb", 8, 0)]  # OV byte -> CV offset
+    return sym
+
+
+def encode_cv(seq, base, cvbase):
+    out = []
+    for s in seq:
+        if s[0] == "acc":
+            out.append(encode(s[1], base + s[2], s[3]))
+        elif s[0] == "cva":
+            out.append(encode(s[1], cvbase + s[2], s[3], arg=s[4]))
+        elif s[0] == "cvb":
+            out.append(encode(CV_BASE_OP, base + s[1], cvbase + s[2]))
+        else:
+            out.append(encode(s[1], base + s[2], s[3], arg=s[4]))
+    return out
+
+
+def check_cv(orc, seqs, bo):
+    recs, expect, states = [], [], []
+    for j, seq in enumerate(seqs):
+        base, cvbase = 16 * j, (1 << 40) + 64 * j
+        enc = encode_cv(seq, base, cvbase)
+        vs = ValueSim(bo=bo)
+        try:
+            issues = vs.run(enc)
+        except MapError:
+            continue
+        off = len(recs)
+        recs.extend(enc)
+        expect.extend((w, i + off, k) for (w, i, k) in issues)
+        states.extend(vs.state_bits(base // 8 + w) for w in range(2))
+    arr = np.array(recs, dtype=np.uint64).reshape(-1, 2)
+    res = orc.replay(arr, 0, 16 * len(seqs), detect_bo=bo)
+    assert res.rc == 0
+    assert res.triples() == sorted(expect)
+    return len(states) // 2
+
+
+@pytest.mark.parametrize("bo", [False, True])
+def test_cv_translation_exhaustive(orc, bo):
+    """Z26 against the value simulator, which keeps its own CV-address table per entry
+    and translates a device address through it: every sequence of length <= 3."""
+    sym = alphabet_cv()
+    seqs = [s for L in range(1, 4) for s in itertools.product(sym, repeat=L)]
+    n = 0
+    for k in range(0, len(seqs), 40000):
+        n += check_cv(orc, seqs[k:k + 40000], bo)
+    assert n > 20000
+
+
+@pytest.mark.parametrize("bo", [False, True])
+def test_cv_translation_random_long(orc, bo):
+    sym = alphabet_cv()
+    rs = np.random.default_rng(16 + bo)
+    seqs = [tuple(sym[i] for i in rs.integers(0, len(sym), rs.integers(4, 10))) for _ in range(30000)]
+    check_cv(orc, seqs, bo)
+
+
+def test_cv_translation_equals_ov_addressing(orc):
+    """A trace whose target accesses to mapped words use CV addresses, with every CV
+    placed by a CV_BASE record, replays exactly like the same trace with OV
+    addresses (a target access to an unmapped word keeps its OV address: its CV
+    address would be in no CV, Z26)."""
+    from gen.fuzz import random_program
+    for seed in range(6):
+        rec, base, span = random_program(9300 + seed, p_task=0.3)
+        op = (rec[:, 0] >> np.uint64(48)) & np.uint64(0xFF)
+        addr = rec[:, 0] & np.uint64((1 << 48) - 1)
+        cv_off = np.uint64(1 << 44)                      # every CV at OV + 2^44
+        tracker = ValueSim()                             # which words are mapped, record by record
+        out = []
+        for i in range(rec.shape[0]):
+            w0, w1 = int(rec[i, 0]), int(rec[i, 1])
+            mapped = op[i] in (OP.RT, OP.WT) and tracker._entry_of(int(addr[i])) is not None
+            try:
+                tracker.record(int(op[i]), int(addr[i]), w1 & ((1 << 48) - 1), w0 >> 56, i)
+            except MapError:
+                pass
+            if mapped:
+                w0 = (w0 & ~((1 << 48) - 1) & ~(0xFF << 56)) | int(addr[i] + cv_off) | ((CV_ADDR | (w0 >> 56)) << 56)
+            out.append((w0, w1))
+            if op[i] == OP.MAP_ENTER:                    # the runtime reports where the CV went
+                out.append(encode(CV_BASE_OP, int(addr[i]), int(addr[i] + cv_off)))
+        cv = np.array(out, dtype=np.uint64)
+        a = orc.replay(rec, base, span)
+        b = orc.replay(cv, base, span)
+        assert a.rc == b.rc
+        if a.rc != 0:
+            continue
+        # same reports, record indices shifted by the inserted CV_BASE records
+        keep = [j for j, (w0, _) in enumerate(out) if ((w0 >> 48) & 0xFF) != CV_BASE_OP]
+        assert [(w, keep[r], k) for w, r, k in a.triples()] == b.triples()
+        assert np.array_equal(a.shadow, b.shadow)

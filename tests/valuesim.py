@@ -23,6 +23,8 @@ BOT = 0  # undefined content
 
 RH, WH, RT, WT, MAP_ENTER, MAP_EXIT, UPDATE = 0, 1, 2, 3, 8, 9, 10
 BASE = 11                           # pointer tag -> base address (reading Z25)
+CV_BASE = 16                        # the CV address of a mapped OV address (reading Z26)
+CV_ADDR = 0x80                      # RT / WT arg bit: the address is a CV address (Z26)
 TASK_BEGIN, TASK_END, SYNC = 12, 13, 14
 TO, FROM, TOFROM, ALLOC, RELEASE, DELETE = 0, 1, 2, 3, 4, 5
 ALWAYS = 0x10                       # map-type modifier bit (N4, reading Z21)
@@ -55,7 +57,8 @@ class ValueSim:
         self.presents = [[] for _ in range(devices)]
         self.latest: dict[int, int] = {}
         self.next_id = 1
-        self.present: list[list[int]] = self.presents[0]  # [lo, hi, refcount] byte intervals
+        self.present: list[list[int]] = self.presents[0]  # [lo, hi, refcount, cv] byte intervals
+        self.ignored = 0                  # word-ops of CV addresses no CV holds (Z26)
         self.issues: set[tuple[int, int, int]] = set()
         self.base: dict[int, int] = {}    # pointer tag -> base byte address (Z25)
         self.tag = 0                      # tag of the current target access
@@ -127,13 +130,32 @@ class ValueSim:
         return hit
 
     def record(self, op, addr, length, arg, idx, tag=0):
+        cv_addr = op in (RT, WT) and bool(arg & CV_ADDR)    # Z26: a device address
+        if op in (RT, WT):
+            arg &= ~CV_ADDR
         if self.devices > 1:              # Z24: the device of the record
-            d = arg if op in (RT, WT) else (arg >> 6 if op in (MAP_ENTER, MAP_EXIT, UPDATE) else 0)
-            arg = arg & 0x3F if op in (MAP_ENTER, MAP_EXIT, UPDATE) else arg
+            d = arg if op in (RT, WT) else (arg >> 6 if op in (MAP_ENTER, MAP_EXIT, UPDATE, CV_BASE) else 0)
+            arg = arg & 0x3F if op in (MAP_ENTER, MAP_EXIT, UPDATE, CV_BASE) else arg
             self.cv, self.present = self.cvs[d], self.presents[d]
         always = bool(arg & ALWAYS)           # OpenMP 5.1 `always` map-type modifier (reading Z21)
         present = bool(arg & PRESENT)         # OpenMP 5.1 `present`: not mapped -> error
         arg &= ~(ALWAYS | PRESENT)
+        if cv_addr:
+            # the interval tree of P:269: which entry's CV holds this device address
+            hit = [e for e in self.present if len(e) > 3 and e[3] is not None and e[3] <= addr < e[3] + e[1] - e[0]]
+            if not hit:
+                self.ignored += (addr + length - 1) // 8 - addr // 8 + 1
+                return
+            addr = hit[0][0] + (addr - hit[0][3])
+        if op == CV_BASE:
+            ent = self._entry_of(addr)
+            if ent is not None:
+                c = length - (addr - ent[0])            # w1 [0,48) carries the CV address
+                for f in self.present:                  # one CV per device address: older
+                    if f is not ent and f[3] is not None and f[3] < c + ent[1] - ent[0] and c < f[3] + f[1] - f[0]:
+                        f[3] = None                     # overlapping placements are gone
+                ent[3] = c
+            return
         if op in (RH, WH, RT, WT):
             name = {RH: "RH", WH: "WH", RT: "RT", WT: "WT"}[op]
             self.tag = tag if op in (RT, WT) else 0
@@ -152,7 +174,7 @@ class ValueSim:
                     for w in self.words(addr, length):
                         self.word_op("UPT", w, idx)
                 return
-            self.present.append([addr, addr + length, 1])
+            self.present.append([addr, addr + length, 1, None])
             for w in self.words(addr, length):
                 self.word_op("NEW", w, idx)
             if arg in (TO, TOFROM):
