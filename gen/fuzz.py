@@ -136,3 +136,39 @@ def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: i
         tb.task_end(in_task)
     span = n_arrays * array_words * 8 * 2
     return tb.array(), base, span
+
+
+def to_cv_addressing(rec, cv_off=1 << 44, frac=1.0, seed=0):
+    """The same program with its target accesses to mapped words addressed by CV
+    (device) address (arg bit 0x80, reading Z26): every entry's CV sits at its OV
+    address + cv_off, reported by an ARB_CV_BASE record (op 16) after each map entry.
+    frac < 1: only that fraction of the eligible accesses is rewritten.  Mapped-ness
+    is tracked with a plain interval list (structure only, no replay)."""
+    rs = np.random.default_rng(seed)
+    op = ((rec[:, 0] >> np.uint64(48)) & np.uint64(0xFF)).astype(np.int64)
+    addr = (rec[:, 0] & np.uint64((1 << 48) - 1)).astype(np.int64)
+    ln = (rec[:, 1] & np.uint64((1 << 48) - 1)).astype(np.int64)
+    arg = (rec[:, 0] >> np.uint64(56)).astype(np.int64)
+    entries = []                                  # [lo, hi, rc]
+    out = []
+    for i in range(rec.shape[0]):
+        w0, w1 = int(rec[i, 0]), int(rec[i, 1])
+        o, a, n = int(op[i]), int(addr[i]), int(ln[i])
+        if o in (OP.RT, OP.WT) and any(e[0] <= a < e[1] for e in entries) and rs.random() < frac:
+            w0 = (w0 & ~((1 << 48) - 1) & ~(0xFF << 56)) | (a + cv_off) | ((0x80 | int(arg[i])) << 56)
+        out.append((w0, w1))
+        if o == OP.MAP_ENTER:
+            hit = [e for e in entries if e[0] <= a and a + n <= e[1]]
+            if hit:
+                hit[0][2] += 1
+            elif not any(a < e[1] and e[0] < a + n for e in entries):
+                entries.append([a, a + n, 1])
+                out.append(tuple(int(x) for x in encode_np(16, [a], [a + cv_off])[0]))
+        elif o == OP.MAP_EXIT:
+            hit = [e for e in entries if e[0] <= a and a + n <= e[1]]
+            if hit:
+                e = hit[0]
+                e[2] = 0 if (int(arg[i]) & 0xF) == MAP.DELETE else e[2] - 1
+                if e[2] == 0:
+                    entries.remove(e)
+    return np.array(out, dtype=np.uint64).reshape(-1, 2)

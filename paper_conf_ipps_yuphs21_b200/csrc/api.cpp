@@ -132,6 +132,9 @@ struct arb_ctx_s {
   uint64_t seg_cap = 0;
   HostBuf<uint32_t> h_weight;
   TagBases tags;                              // N1 (Z25): pointer tag bases (committed per flush)
+  DevBuf<uint4> cv_buf;                       // N1 (Z26): the batch with CV addresses translated
+  DevBuf<uint32_t> d_cv_epoch_pos, d_cv_epoch_first;
+  DevBuf<CvPlace> d_cv_place;
   DevBuf<uint32_t> d_tag_first;
   DevBuf<TagSeg> d_tag_segs;
   DevBuf<CtlRec> ctl;
@@ -298,7 +301,8 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   if (ctx->shadow) cudaFree(ctx->shadow);
   ctx->staging.release(); ctx->gidx_staging.release(); ctx->part_ev.release(); ctx->seg_a.release(); ctx->seg_b.release(); ctx->segs.release(); ctx->seg_first.release();
   ctx->h_weight.release();
-  ctx->d_tag_first.release(); ctx->d_tag_segs.release();
+  ctx->d_tag_first.release(); ctx->d_tag_segs.release(); ctx->cv_buf.release(); ctx->d_cv_epoch_pos.release();
+  ctx->d_cv_epoch_first.release(); ctx->d_cv_place.release();
   ctx->ctl.release(); ctx->cand.release(); ctx->cand_tmp.release(); ctx->reports.release(); ctx->blk.release();
   ctx->ops_start.release(); ctx->ops.release(); ctx->dstats.release(); ctx->dcount.release();
   ctx->m_ins_lo.release(); ctx->m_ins_cum.release(); ctx->m_qry_lo.release(); ctx->m_qry_cum.release();
@@ -544,116 +548,137 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     }
   }
   if (timing) cudaEventRecord(ctx->ev[0], s);
-  // ---- bucket balancing on a sampled address histogram (all on the device) ----
-  if (balanced) {
-    CK(ctx->d_hist.ensure(ctx->n_bins), "alloc hist");
-    CK(cudaMemsetAsync(ctx->d_hist.p, 0, ctx->n_bins * sizeof(uint32_t), s), "hist clear");
-    SampleParams sp{};
-    sp.ev = ev; sp.n = n; sp.stride = std::max<uint64_t>(1, n / kSampleCap);
-    sp.base_word = ctx->base_word; sp.n_words = ctx->n_words; sp.coarse_bits = ctx->coarse_bits;
-    sp.hist = ctx->d_hist.p;
-    const uint64_t n_samples = n ? (n + sp.stride - 1) / sp.stride : 0;
-    CK(launch_sample(sp, n_samples, s), "k_sample");
-    launches += n_samples ? 1 : 0;
-    // cut balanced buckets; the histogram becomes the bin map in place
-    if (ctx->d_bucket_start.cap == 0) {       // the read-back below copies every slot
-      CK(ctx->d_bucket_start.ensure(kMaxBuckets + 1), "alloc buckets");
-      CK(cudaMemsetAsync(ctx->d_bucket_start.p, 0, (kMaxBuckets + 1) * 8, s), "clear buckets");
+  // N1 (Z26): a batch with CV-addressed target accesses runs this part twice: the
+  // first pass finds them (left untracked) and resolves the CV placements, the
+  // second partitions a copy with those accesses translated to OV addresses
+  for (bool translated = false;;) {
+    // ---- bucket balancing on a sampled address histogram (all on the device) ----
+    if (balanced) {
+      CK(ctx->d_hist.ensure(ctx->n_bins), "alloc hist");
+      CK(cudaMemsetAsync(ctx->d_hist.p, 0, ctx->n_bins * sizeof(uint32_t), s), "hist clear");
+      SampleParams sp{};
+      sp.ev = ev; sp.n = n; sp.stride = std::max<uint64_t>(1, n / kSampleCap);
+      sp.base_word = ctx->base_word; sp.n_words = ctx->n_words; sp.coarse_bits = ctx->coarse_bits;
+      sp.hist = ctx->d_hist.p;
+      const uint64_t n_samples = n ? (n + sp.stride - 1) / sp.stride : 0;
+      CK(launch_sample(sp, n_samples, s), "k_sample");
+      launches += n_samples ? 1 : 0;
+      // cut balanced buckets; the histogram becomes the bin map in place
+      if (ctx->d_bucket_start.cap == 0) {       // the read-back below copies every slot
+        CK(ctx->d_bucket_start.ensure(kMaxBuckets + 1), "alloc buckets");
+        CK(cudaMemsetAsync(ctx->d_bucket_start.p, 0, (kMaxBuckets + 1) * 8, s), "clear buckets");
+      }
+      if (ctx->d_cut.cap == 0) {
+        CK(ctx->d_cut.ensure(2 * kMaxBuckets + 2), "alloc cut scratch");
+        CK(cudaMemsetAsync(ctx->d_cut.p, 0, (2 * kMaxBuckets + 2) * 4, s), "clear cut scratch");
+      }
+      CK(ctx->d_cutscr.ensure(2 * ((ctx->n_bins + 1023) / 1024) + 4 + ctx->n_bins), "alloc cut scratch");
+      CK(launch_cut(ctx->d_hist.p, ctx->n_bins, ctx->coarse_bits, ctx->n_words, kMaxBuckets, ctx->d_bucket_start.p,
+                    ctx->d_cut.p, ctx->d_cut.p + kMaxBuckets, ctx->d_cut.p + 2 * kMaxBuckets, ctx->d_cutscr.p,
+                    s, &launches), "k_cut");
+      // the bucket count and starts come back with the partition's counters (one sync)
+      CK(cudaMemcpyAsync(ctx->h_nb.p, ctx->d_cut.p + 2 * kMaxBuckets, 4, cudaMemcpyDeviceToHost, s), "nb d2h");
+      CK(cudaMemcpyAsync(ctx->h_bstart.p, ctx->d_bucket_start.p, (kMaxBuckets + 1) * 8, cudaMemcpyDeviceToHost, s),
+         "buckets d2h");
+      CK(cudaMemcpyAsync(ctx->h_weight.p, ctx->d_cut.p, kMaxBuckets * 4, cudaMemcpyDeviceToHost, s), "weights d2h");
+    } else if (ctx->d_bin_map.cap == 0) {
+      CK(upload(ctx->d_bin_map, ctx->bin_map, s), "upload bin map");
+      CK(upload(ctx->d_bucket_start, ctx->bucket_start, s), "upload bucket starts");
     }
-    if (ctx->d_cut.cap == 0) {
-      CK(ctx->d_cut.ensure(2 * kMaxBuckets + 2), "alloc cut scratch");
-      CK(cudaMemsetAsync(ctx->d_cut.p, 0, (2 * kMaxBuckets + 2) * 4, s), "clear cut scratch");
+    if (!balanced) ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;   // fixed buckets
+    if (timing) cudaEventRecord(ctx->ev[7], s);
+    // ---- A1/A3a: decode + partition ------------------------------------------
+    const uint32_t n_chunks = (uint32_t)((n + kChunkRecords - 1) / kChunkRecords);
+    CK(ctx->part_ev.ensure((size_t)std::max<uint32_t>(n_chunks, 1) * kChunkCap), "alloc part_ev");
+    if (ctx->seg_cap < (uint64_t)n_chunks * 2 + 4096) ctx->seg_cap = (uint64_t)n_chunks * 2 + 4096;
+    CK(ctx->seg_a.ensure(std::max<uint64_t>(ctx->seg_cap, 1)), "alloc segments");
+    PartParams pp{};
+    for (int attempt = 0; attempt < 2; ++attempt) {
+      CK(cudaMemsetAsync(ctx->dstats.p, 0, sizeof(DevStats), s), "stats init");
+      CK(cudaMemsetAsync(&ctx->dstats.p->err_pos, 0xFF, sizeof(unsigned long long), s), "stats init");
+      pp.ev = ev; pp.n = n; pp.base_word = ctx->base_word; pp.n_words = ctx->n_words;
+      pp.coarse_bits = ctx->coarse_bits; pp.bin_map = balanced ? ctx->d_hist.p : ctx->d_bin_map.p;
+      pp.bucket_bits = ctx->bucket_bits; pp.n_buckets = balanced ? (uint32_t)kMaxBuckets : ctx->n_buckets;
+      pp.n_chunks = n_chunks;
+      pp.n_dev = 1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u);
+      pp.part_ev = ctx->part_ev.p; pp.seg_out = ctx->seg_a.p; pp.seg_cap = ctx->seg_cap;
+      pp.ctl = ctx->ctl.p; pp.ctl_cap = ctx->ctl_cap;
+      pp.st = ctx->dstats.p;
+      CK(launch_partition(pp, s), "k_partition");
+      launches += n_chunks ? 1 : 0;
+      CK(cudaMemcpyAsync(&hst, ctx->dstats.p, sizeof(hst), cudaMemcpyDeviceToHost, s), "stats d2h");
+      CK(cudaStreamSynchronize(s), "partition sync");
+      if (hst.n_ctl <= ctx->ctl_cap && hst.n_segs <= ctx->seg_cap) break;
+      if (hst.n_ctl > ctx->ctl_cap) ctx->ctl_cap = hst.n_ctl + hst.n_ctl / 2;
+      if (hst.n_segs > ctx->seg_cap) ctx->seg_cap = hst.n_segs + hst.n_segs / 4;
+      CK(ctx->ctl.ensure(ctx->ctl_cap), "grow ctl");
+      CK(ctx->seg_a.ensure(ctx->seg_cap), "grow segments");
     }
-    CK(ctx->d_cutscr.ensure(2 * ((ctx->n_bins + 1023) / 1024) + 4 + ctx->n_bins), "alloc cut scratch");
-    CK(launch_cut(ctx->d_hist.p, ctx->n_bins, ctx->coarse_bits, ctx->n_words, kMaxBuckets, ctx->d_bucket_start.p,
-                  ctx->d_cut.p, ctx->d_cut.p + kMaxBuckets, ctx->d_cut.p + 2 * kMaxBuckets, ctx->d_cutscr.p,
-                  s, &launches), "k_cut");
-    // the bucket count and starts come back with the partition's counters (one sync)
-    CK(cudaMemcpyAsync(ctx->h_nb.p, ctx->d_cut.p + 2 * kMaxBuckets, 4, cudaMemcpyDeviceToHost, s), "nb d2h");
-    CK(cudaMemcpyAsync(ctx->h_bstart.p, ctx->d_bucket_start.p, (kMaxBuckets + 1) * 8, cudaMemcpyDeviceToHost, s),
-       "buckets d2h");
-    CK(cudaMemcpyAsync(ctx->h_weight.p, ctx->d_cut.p, kMaxBuckets * 4, cudaMemcpyDeviceToHost, s), "weights d2h");
-  } else if (ctx->d_bin_map.cap == 0) {
-    CK(upload(ctx->d_bin_map, ctx->bin_map, s), "upload bin map");
-    CK(upload(ctx->d_bucket_start, ctx->bucket_start, s), "upload bucket starts");
-  }
-  if (!balanced) ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;   // fixed buckets
-  if (timing) cudaEventRecord(ctx->ev[7], s);
-  // ---- A1/A3a: decode + partition ------------------------------------------
-  const uint32_t n_chunks = (uint32_t)((n + kChunkRecords - 1) / kChunkRecords);
-  CK(ctx->part_ev.ensure((size_t)std::max<uint32_t>(n_chunks, 1) * kChunkCap), "alloc part_ev");
-  if (ctx->seg_cap < (uint64_t)n_chunks * 2 + 4096) ctx->seg_cap = (uint64_t)n_chunks * 2 + 4096;
-  CK(ctx->seg_a.ensure(std::max<uint64_t>(ctx->seg_cap, 1)), "alloc segments");
-  PartParams pp{};
-  for (int attempt = 0; attempt < 2; ++attempt) {
-    CK(cudaMemsetAsync(ctx->dstats.p, 0, sizeof(DevStats), s), "stats init");
-    CK(cudaMemsetAsync(&ctx->dstats.p->err_pos, 0xFF, sizeof(unsigned long long), s), "stats init");
-    pp.ev = ev; pp.n = n; pp.base_word = ctx->base_word; pp.n_words = ctx->n_words;
-    pp.coarse_bits = ctx->coarse_bits; pp.bin_map = balanced ? ctx->d_hist.p : ctx->d_bin_map.p;
-    pp.bucket_bits = ctx->bucket_bits; pp.n_buckets = balanced ? (uint32_t)kMaxBuckets : ctx->n_buckets;
-    pp.n_chunks = n_chunks;
-    pp.n_dev = 1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u);
-    pp.part_ev = ctx->part_ev.p; pp.seg_out = ctx->seg_a.p; pp.seg_cap = ctx->seg_cap;
-    pp.ctl = ctx->ctl.p; pp.ctl_cap = ctx->ctl_cap;
-    pp.st = ctx->dstats.p;
-    CK(launch_partition(pp, s), "k_partition");
-    launches += n_chunks ? 1 : 0;
-    CK(cudaMemcpyAsync(&hst, ctx->dstats.p, sizeof(hst), cudaMemcpyDeviceToHost, s), "stats d2h");
-    CK(cudaStreamSynchronize(s), "partition sync");
-    if (hst.n_ctl <= ctx->ctl_cap && hst.n_segs <= ctx->seg_cap) break;
-    if (hst.n_ctl > ctx->ctl_cap) ctx->ctl_cap = hst.n_ctl + hst.n_ctl / 2;
-    if (hst.n_segs > ctx->seg_cap) ctx->seg_cap = hst.n_segs + hst.n_segs / 4;
-    CK(ctx->ctl.ensure(ctx->ctl_cap), "grow ctl");
-    CK(ctx->seg_a.ensure(ctx->seg_cap), "grow segments");
-  }
-  if (timing) cudaEventRecord(ctx->ev[1], s);
-  if (hst.err_pos != ~0ull)
-    return fail(ctx, ARB_ETRACE, "malformed record at batch position " + std::to_string(hst.err_pos));
-  if (balanced) {
-    const uint32_t nb = *ctx->h_nb.p;
-    ctx->bucket_start.assign(ctx->h_bstart.p, ctx->h_bstart.p + nb + 1);
-    const double stride = (double)std::max<uint64_t>(1, n / kSampleCap);
-    bucket_events.resize(nb);
-    for (uint32_t b = 0; b < nb; ++b) bucket_events[b] = ctx->h_weight.p[b] * stride;
-  }
-  ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;
-  S.buckets = ctx->n_buckets;
-  S.access_words = hst.access_words;
-  S.control_records = hst.n_ctl;
+    if (timing) cudaEventRecord(ctx->ev[1], s);
+    if (hst.err_pos != ~0ull)
+      return fail(ctx, ARB_ETRACE, "malformed record at batch position " + std::to_string(hst.err_pos));
+    if (balanced) {
+      const uint32_t nb = *ctx->h_nb.p;
+      ctx->bucket_start.assign(ctx->h_bstart.p, ctx->h_bstart.p + nb + 1);
+      const double stride = (double)std::max<uint64_t>(1, n / kSampleCap);
+      bucket_events.resize(nb);
+      for (uint32_t b = 0; b < nb; ++b) bucket_events[b] = ctx->h_weight.p[b] * stride;
+    }
+    ctx->n_buckets = (uint32_t)ctx->bucket_start.size() - 1;
+    S.buckets = ctx->n_buckets;
+    S.access_words = hst.access_words;
+    S.control_records = hst.n_ctl;
 
-  // ---- A3b: segment entries sorted by (bucket, chunk) — on the GPU while the
-  // host resolves the control records ------------------------------------------------
-  {
-    const uint64_t ns = hst.n_segs;
-    CK(ctx->seg_b.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
-    CK(ctx->segs.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
-    CK(ctx->seg_first.ensure(ctx->n_buckets + 1), "alloc seg_first");
-    CK(ctx->blk.ensure((ns + 4095) / 4096 * 2049 + 4096), "alloc blk");   // 2048-bin digit counters + scan scratch
-    int cb = 1;
-    while (cb < 22 && ((uint64_t)n_chunks >> cb)) ++cb;
-    CK(launch_sort_segments(ctx->seg_a.p, ctx->seg_b.p, ns, cb, ctx->n_buckets, ctx->blk.p, ctx->seg_first.p,
-                            ctx->segs.p, s, &launches), "sort segments");
-    if (timing) cudaEventRecord(ctx->ev[8], s);
-  }
-  t_host0 = std::chrono::steady_clock::now();
+    // ---- A3b: segment entries sorted by (bucket, chunk) — on the GPU while the
+    // host resolves the control records ------------------------------------------------
+    {
+      const uint64_t ns = hst.n_segs;
+      CK(ctx->seg_b.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
+      CK(ctx->segs.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
+      CK(ctx->seg_first.ensure(ctx->n_buckets + 1), "alloc seg_first");
+      CK(ctx->blk.ensure((ns + 4095) / 4096 * 2049 + 4096), "alloc blk");   // 2048-bin digit counters + scan scratch
+      int cb = 1;
+      while (cb < 22 && ((uint64_t)n_chunks >> cb)) ++cb;
+      CK(launch_sort_segments(ctx->seg_a.p, ctx->seg_b.p, ns, cb, ctx->n_buckets, ctx->blk.p, ctx->seg_first.p,
+                              ctx->segs.p, s, &launches), "sort segments");
+      if (timing) cudaEventRecord(ctx->ev[8], s);
+    }
+    t_host0 = std::chrono::steady_clock::now();
 
-  // ---- A2: control resolution on the host -------------------------------------
-  std::vector<CtlRec> ctl(hst.n_ctl);
-  if (hst.n_ctl) {
-    CK(ctx->h_ctl.ensure(hst.n_ctl), "pinned ctl");
-    CK(cudaMemcpyAsync(ctx->h_ctl.p, ctx->ctl.p, hst.n_ctl * sizeof(CtlRec), cudaMemcpyDeviceToHost, ctx->aux),
-       "ctl d2h");
-    CK(cudaStreamSynchronize(ctx->aux), "ctl sync");
-    std::memcpy(ctl.data(), ctx->h_ctl.p, hst.n_ctl * sizeof(CtlRec));
-    std::sort(ctl.begin(), ctl.end(), [](const CtlRec& a, const CtlRec& b) { return a.pos < b.pos; });
+    // ---- A2: control resolution on the host -------------------------------------
+    std::vector<CtlRec> ctl(hst.n_ctl);
+    if (hst.n_ctl) {
+      CK(ctx->h_ctl.ensure(hst.n_ctl), "pinned ctl");
+      CK(cudaMemcpyAsync(ctx->h_ctl.p, ctx->ctl.p, hst.n_ctl * sizeof(CtlRec), cudaMemcpyDeviceToHost, ctx->aux),
+         "ctl d2h");
+      CK(cudaStreamSynchronize(ctx->aux), "ctl sync");
+      std::memcpy(ctl.data(), ctx->h_ctl.p, hst.n_ctl * sizeof(CtlRec));
+      std::sort(ctl.begin(), ctl.end(), [](const CtlRec& a, const CtlRec& b) { return a.pos < b.pos; });
+    }
+    t_host1 = std::chrono::steady_clock::now();
+    map = ctx->map;
+    resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_start, map, plan,
+                    (ctx->cfg.flags & ARB_F_BO) != 0, &ctx->carried, (ctx->cfg.flags & ARB_F_UNIFIED) != 0,
+                    1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u), &ctx->last_ended, &ctx->tags,
+                  hst.n_cv_acc != 0);
+    if (plan.rc != 0)
+      return fail(ctx, plan.rc, plan.err + " (batch position " + std::to_string(plan.err_pos) + ")");
+  if (hst.n_cv_acc && !translated) {
+    if ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u)
+      return fail(ctx, ARB_ETRACE, "CV-addressed accesses (Z26) with several accelerators are oracle-only");
+    CK(upload(ctx->d_cv_epoch_pos, plan.cv_epoch_pos, s), "cv epochs");
+    CK(upload(ctx->d_cv_epoch_first, plan.cv_epoch_first, s), "cv epochs");
+    CK(upload(ctx->d_cv_place, plan.cv_place, s), "cv placements");
+    CK(ctx->cv_buf.ensure(n), "cv copy");
+    CK(launch_cv_translate(ev, ctx->cv_buf.p, n, ctx->d_cv_epoch_pos.p, ctx->d_cv_epoch_first.p,
+                           (uint32_t)plan.cv_epoch_pos.size(), ctx->d_cv_place.p, s), "k_cv_translate");
+    launches += 1;
+    ev = ctx->cv_buf.p;
+    translated = true;
+    continue;
   }
-  t_host1 = std::chrono::steady_clock::now();
-  map = ctx->map;
-  resolve_control(ctl, n, ctx->base_word, ctx->n_words, ctx->bucket_start, map, plan,
-                  (ctx->cfg.flags & ARB_F_BO) != 0, &ctx->carried, (ctx->cfg.flags & ARB_F_UNIFIED) != 0,
-                  1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u), &ctx->last_ended, &ctx->tags);
-  if (plan.rc != 0)
-    return fail(ctx, plan.rc, plan.err + " (batch position " + std::to_string(plan.err_pos) + ")");
+  break;
+  }
   return ARB_OK;
   }();
   {   // every rank learns whether every rank's batch is valid

@@ -13,7 +13,9 @@ enum Op : uint32_t { OP_RH = 0, OP_WH = 1, OP_RT = 2, OP_WT = 3,
                      OP_MAP_ENTER = 8, OP_MAP_EXIT = 9, OP_UPDATE = 10,
                      OP_TASK_BEGIN = 12, OP_TASK_END = 13, OP_SYNC = 14,
                      OP_TASK_DEPEND = 15,     // N4, Z22
-                     OP_BASE = 11 };          // pointer tag -> base address (N1, Z25)
+                     OP_BASE = 11,            // pointer tag -> base address (N1, Z25)
+                     OP_CV_BASE = 16 };       // an entry's CV placement (N1, Z26)
+constexpr uint32_t kCvAddrBit = 1u << 31;     // q.y bit 31 = arg bit 7 of RT / WT: a CV address (Z26)
 enum MapType : uint32_t { MT_TO = 0, MT_FROM = 1, MT_TOFROM = 2, MT_ALLOC = 3,
                           MT_RELEASE = 4, MT_DELETE = 5 };
 constexpr uint32_t kMapAlways = 0x10;   // `always` map-type modifier bit (N4, Z21)
@@ -102,7 +104,8 @@ struct DevStats {
   unsigned long long n_segs;          // (chunk, bucket) segment entries written by k_partition
   unsigned long long n_carry_out;     // N2: access summaries of instances carried into the next flush
   unsigned long long n_bo_cand;       // N1 (Z25): base-tag overflow candidates
-  unsigned long long pad[2];
+  unsigned long long n_cv_acc;        // N1 (Z26): target accesses by CV address (left untracked)
+  unsigned long long pad[1];
 };
 
 // control record extracted by the partition kernel
@@ -118,6 +121,9 @@ struct BucketOp {
 // N1 (Z25): from batch position `pos` on, the mapping entry holding pointer tag t's
 // base spans the absolute words [lo, hi) (lo == hi: the base is not mapped)
 struct TagSeg { uint32_t pos; uint32_t pad; uint64_t lo, hi; };
+
+// N1 (Z26): a live CV placement: device bytes [cv_lo, cv_hi) hold OV bytes from ov_lo on
+struct CvPlace { uint64_t cv_lo, cv_hi, ov_lo; };
 
 // a range op for the MIR join (absolute relative words, instance of its block)
 struct RangeRef { uint64_t lo, hi; uint32_t pos; uint32_t inst; };
@@ -218,6 +224,13 @@ cudaError_t launch_carry(const uint4* hot, uint32_t n_hot, uint32_t max_span, co
                          cudaStream_t s);
 cudaError_t launch_mir(const MirParams& p, uint64_t n_ins_pos, uint64_t n_qry_pos, uint64_t n_rr_words,
                        cudaStream_t s, int* launches);
+// N1 (Z26): copy the batch, translating CV-addressed target accesses to OV addresses
+// through the placements live at their position (epoch e covers positions from
+// epoch_pos[e], its placements are place[epoch_first[e], epoch_first[e+1]), sorted
+// by cv_lo and disjoint); an access in no placement keeps its CV flag (untracked)
+cudaError_t launch_cv_translate(const uint4* in, uint4* out, uint64_t n, const uint32_t* epoch_pos,
+                                const uint32_t* epoch_first, uint32_t n_epochs, const CvPlace* place,
+                                cudaStream_t s);
 // N1 (Z25): target accesses through pointer tag t (w1[48,64)) whose word lies outside
 // the entry of t's base at that position -> BO candidates {word lo, word hi, pos, 4}
 // (tag_first: [65537] CSR into segs, by tag; words relative to base_word in the output)

@@ -43,7 +43,7 @@ struct Emitter {
 void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_t base_word,
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
                      FlushPlan& out, bool bo, const std::vector<CarriedInst>* carried_in, bool unified,
-                     uint32_t n_dev, const LastEnded* last_ended_in, const TagBases* tags_in) {
+                     uint32_t n_dev, const LastEnded* last_ended_in, const TagBases* tags_in, bool want_cv) {
   const uint32_t n_buckets = (uint32_t)bucket_start.size() - 1;
   out = FlushPlan();
   Emitter em{base_word, n_words, &out, unified};
@@ -101,10 +101,26 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
   };
   if (bo && n_dev == 1)
     for (const auto& kv : out.tags_out) tag_note(kv.first, 0);
+  // N1 (Z26): snapshot of the live CV placements from position pos on
+  auto cv_epoch = [&](uint32_t pos) {
+    if (!want_cv) return;
+    if (!out.cv_epoch_pos.empty() && out.cv_epoch_pos.back() == pos) {   // replace the same position's
+      out.cv_place.resize(out.cv_epoch_first.back());
+      out.cv_epoch_pos.pop_back(); out.cv_epoch_first.pop_back();
+    }
+    out.cv_epoch_pos.push_back(pos);
+    out.cv_epoch_first.push_back((uint32_t)out.cv_place.size());
+    const size_t a = out.cv_place.size();
+    for (const auto& kv : map)
+      if (kv.second.cv != UINT64_MAX && (kv.first >> 56) == 0)       // device 0 (single device)
+        out.cv_place.push_back(CvPlace{kv.second.cv, kv.second.cv + (kv.second.hi - kv.first), kv.first});
+    std::sort(out.cv_place.begin() + a, out.cv_place.end(), [](const CvPlace& x, const CvPlace& y) { return x.cv_lo < y.cv_lo; });
+  };
+  cv_epoch(0);
   for (const CtlRec& c : ctl) {
     uint32_t op = (uint32_t)(c.w0 >> 48) & 0xFFu, arg = (uint32_t)(c.w0 >> 56);
     uint32_t dev = 0;                               // Z24: device of a MAP / UPDATE record
-    if (md && (op == OP_MAP_ENTER || op == OP_MAP_EXIT || op == OP_UPDATE)) {
+    if (md && (op == OP_MAP_ENTER || op == OP_MAP_EXIT || op == OP_UPDATE || op == OP_CV_BASE)) {
       dev = arg >> 6;
       arg &= 0x3Fu;
       if (dev >= n_dev) return fail(ARB_ETRACE, c.pos, "device id of a map / update record out of range");
@@ -174,8 +190,10 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
           if (arg == MT_FROM || arg == MT_TOFROM) em.emit(pos, s_uph(dev), addr, addr + len, open);
           em.emit(pos, s_rel(dev), it->first & kAddrMask, it->second.hi & kAddrMask, open);
           const uint64_t elo = it->first & kAddrMask, ehi = it->second.hi & kAddrMask;
+          const bool had_cv = it->second.cv != UINT64_MAX;
           map.erase(it);
           if (bo && n_dev == 1 && !out.tags_out.empty()) tags_in_range(elo, ehi, pos);
+          if (had_cv) cv_epoch(pos);
         }
         break;
       }
@@ -187,6 +205,19 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
         if (f < 0) return fail(ARB_EMAP, c.pos, "target update partially overlaps a present entry");
         if (f == 0) break;                          // not present: no-op (Z7)
         em.emit(pos, arg == 0 ? s_upt(dev) : s_uph(dev), addr, addr + len, open);
+        break;
+      }
+      case OP_CV_BASE: {                            // Z26: the runtime placed an entry's CV
+        MapTable::iterator it;
+        if (map_find(map, dkey | addr, dkey | (addr + 1), it) == 1) {
+          const uint64_t c = len - (addr - (it->first & kAddrMask)), sz = it->second.hi - it->first;
+          for (auto& kv : map)                      // one CV per device address: older overlaps go
+            if (&kv.second != &it->second && (kv.first >> 56) == (dkey >> 56) && kv.second.cv != UINT64_MAX &&
+                kv.second.cv < c + sz && c < kv.second.cv + (kv.second.hi - kv.first))
+              kv.second.cv = UINT64_MAX;
+          it->second.cv = c;
+          cv_epoch(pos);
+        }
         break;
       }
       case OP_BASE: {                               // Z25: pointer tag -> base address
@@ -216,6 +247,7 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
         return fail(ARB_ETRACE, c.pos, "unknown control op");
     }
   }
+  if (want_cv) out.cv_epoch_first.push_back((uint32_t)out.cv_place.size());
   if (!tseg.empty()) {                          // N1: CSR by tag id for k_bo_tags
     out.tag_first.assign(65537, 0);
     for (const auto& kv : tag_ix) out.tag_first[kv.first + 1] = (uint32_t)tseg[kv.second].size();

@@ -20,7 +20,8 @@
 
 namespace arb {
 
-struct MapEntry { uint64_t hi; uint64_t rc; };        // keyed by lo (bytes), [lo, hi)
+struct MapEntry { uint64_t hi; uint64_t rc; uint64_t cv = UINT64_MAX; };   // keyed by lo (bytes), [lo, hi);
+                                                      // cv: CV address of byte lo (Z26), MAX unknown
 using MapTable = std::map<uint64_t, MapEntry>;
 
 struct RangeOpH { uint32_t pos; uint32_t sel; uint64_t lo, hi; uint32_t inst; };  // rel words [lo, hi)
@@ -64,6 +65,10 @@ struct FlushPlan {
   TagBases tags_out;                     // tag bases after this flush (committed likewise)
   std::vector<uint32_t> tag_first;       // N1 with bo: [65537] CSR of tag_segs by tag (empty: no tag)
   std::vector<TagSeg> tag_segs;
+  // N1 (Z26, with want_cv): CV placements by epoch: epoch e starts at batch position
+  // cv_epoch_pos[e]; its live placements are cv_place[cv_epoch_first[e], [e + 1]), sorted
+  std::vector<uint32_t> cv_epoch_pos, cv_epoch_first;
+  std::vector<CvPlace> cv_place;
   uint64_t range_words = 0, ignored_words = 0, tasks = 0;
   int rc = 0; uint64_t err_pos = 0; std::string err;
 };
@@ -86,7 +91,7 @@ void resolve_control(const std::vector<CtlRec>& ctl, uint64_t n_records, uint64_
                      uint64_t n_words, const std::vector<uint64_t>& bucket_start, MapTable& map,
                      FlushPlan& out, bool bo = false, const std::vector<CarriedInst>* carried_in = nullptr,
                      bool unified = false, uint32_t n_dev = 1, const LastEnded* last_ended_in = nullptr,
-                     const TagBases* tags_in = nullptr);
+                     const TagBases* tags_in = nullptr, bool want_cv = false);
 // n_dev > 1 (Z24): device bits 6-7 of MAP / UPDATE args select the device; its
 // entries live in the same table under keys offset by device << 56, and range
 // ops are 8-output selectors (Sel8).

@@ -196,4 +196,41 @@ cudaError_t launch_bo_tags(const uint4* ev, uint64_t n, uint64_t base_word, uint
   return cudaGetLastError();
 }
 
+// ---- N1 (Z26): CV -> OV translation of device-addressed target accesses ----------
+__global__ void k_cv_translate(const uint4* in, uint4* out, uint64_t n, const uint32_t* epoch_pos,
+                               const uint32_t* epoch_first, uint32_t n_epochs, const CvPlace* place) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    uint4 q = ld_stream(in + i);
+    const uint32_t op = (q.y >> 16) & 0xFFu;
+    if ((op == OP_RT || op == OP_WT) && (q.y & kCvAddrBit)) {
+      uint32_t a = 0, z = n_epochs;                       // the epoch holding position i
+      while (z - a > 1) {
+        const uint32_t mid = (a + z) >> 1;
+        if (epoch_pos[mid] <= (uint32_t)i) a = mid; else z = mid;
+      }
+      uint32_t lo = epoch_first[a], hi = epoch_first[a + 1];
+      const uint64_t y = (uint64_t)q.x | ((uint64_t)(q.y & 0xFFFFu) << 32);
+      while (hi - lo > 1) {                                // the last placement starting at or before y
+        const uint32_t mid = (lo + hi) >> 1;
+        if (place[mid].cv_lo <= y) lo = mid; else hi = mid;
+      }
+      if (lo < epoch_first[a + 1] && place[lo].cv_lo <= y && y < place[lo].cv_hi) {
+        const uint64_t x = place[lo].ov_lo + (y - place[lo].cv_lo);
+        q.x = (uint32_t)x;
+        q.y = (q.y & 0x7FFF0000u) | (uint32_t)((x >> 32) & 0xFFFFu);   // OV address, CV flag cleared
+      }
+    }
+    out[i] = q;
+  }
+}
+
+cudaError_t launch_cv_translate(const uint4* in, uint4* out, uint64_t n, const uint32_t* epoch_pos,
+                                const uint32_t* epoch_first, uint32_t n_epochs, const CvPlace* place,
+                                cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  k_cv_translate<<<(unsigned)std::min<uint64_t>((n + 255) / 256, 148 * 16), 256, 0, s>>>(in, out, n, epoch_pos,
+                                                                                        epoch_first, n_epochs, place);
+  return cudaGetLastError();
+}
+
 }  // namespace arb

@@ -45,18 +45,21 @@ constexpr int kB1Shift = 2 + kBucketBits;
 // (Z4, rare: handled by decode1).  b1 = b0 until decode1 says otherwise.
 template <bool MD>
 __device__ __forceinline__ Dec decode0(uint4 q, bool valid, const PartParams& p, uint32_t& ign, uint32_t& flags,
-                                       bool& two) {
+                                       bool& two, uint32_t& cvn) {
   const uint32_t op = (q.y >> 16) & 0xFFu;
   const uint32_t len = q.z, hi = q.y & 0xFFFFu;
   // malformed access: len outside 1..8 or the byte range leaving the 48-bit space
-  const bool bad_acc = (q.w & 0xFFFFu) != 0 || len - 1u > 7u || (hi == 0xFFFFu && q.x > 0u - len);
-  const bool ctl = op < 16 && ((0xFF00u >> op) & 1u);            // ops 8-15 (11: ARB_BASE, Z25)
+  const bool cv = (op & 2u) && (q.y & kCvAddrBit);                // Z26: a CV address (translated first)
+  const bool bad_acc = (q.w & 0xFFFFu) != 0 || len - 1u > 7u || (hi == 0xFFFFu && q.x > 0u - len) ||
+                       (!(op & 2u) && (q.y & kCvAddrBit));         // host accesses use OV addresses
+  const bool ctl = op <= 16 && ((0x1FF00u >> op) & 1u);          // ops 8-16 (11 ARB_BASE, 16 ARB_CV_BASE)
   const bool acc = op < 4;
   flags = valid ? (acc ? (bad_acc ? 2u : 0u) : (ctl ? 1u : 2u)) : 0u;
-  bool ok = valid && acc && !bad_acc;
+  bool ok = valid && acc && !bad_acc && !cv;
+  if (valid && acc && cv && !bad_acc) ++cvn;
   uint32_t dev = 0;
   if (MD) {                                  // several accelerators (Z24): the device of RT / WT is the arg
-    dev = (op & 2u) ? q.y >> 24 : 0u;
+    dev = (op & 2u) ? (q.y >> 24) & 0x7Fu : 0u;
     if (acc && dev >= p.n_dev) { flags = valid ? 2u : 0u; ok = false; }
   }
   const uint64_t rel = ((((uint64_t)hi) << 29) | (q.x >> 3)) - p.base_word;   // wraps below the range
@@ -145,7 +148,7 @@ __device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p,
 #pragma unroll
   for (int k = 0; k < RPL; ++k) {
     const uint4 q = st[k * 32 + lane];
-    bad |= (q.y & 0x00FC0000u) | (q.w & 0xFFFFu) | ((q.z - 1u) & ~7u) | (((q.x & 7u) + q.z - 1u) & ~7u);
+    bad |= (q.y & (0x00FC0000u | kCvAddrBit)) | (q.w & 0xFFFFu) | ((q.z - 1u) & ~7u) | (((q.x & 7u) + q.z - 1u) & ~7u);
     if (MD && (q.y & (1u << 17))) {                // RT / WT on device arg (Z24)
       const uint32_t dv = q.y >> 24;
       bad |= dv >= p.n_dev;
@@ -200,7 +203,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   if (lane < NST) mbar_init(bar + lane, 1);
   fence_mbar_init();
   __syncwarp();
-  uint32_t n_acc = 0, n_ign = 0, nbuf = 0, phase = 0;   // phase: parity bit of each stage's barrier
+  uint32_t n_acc = 0, n_ign = 0, n_cv = 0, nbuf = 0, phase = 0;   // phase: parity bit of each stage's barrier
 
   // the chunk's records arrive in stage k by one TMA bulk copy (lane 0) that
   // completes on bar[k]
@@ -260,7 +263,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
         const uint32_t j = g * 128 + k * 32 + lane;
         uint32_t flags;
         bool two;
-        dec[g * 4 + k] = decode0<MD>(st[j], j < nvalid, p, n_ign, flags, two);
+        dec[g * 4 + k] = decode0<MD>(st[j], j < nvalid, p, n_ign, flags, two, n_cv);
         any_flag |= flags << (2 * k);
         twos |= (uint32_t)two << k;
       }
@@ -407,10 +410,12 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   for (int d = 16; d; d >>= 1) {
     n_acc += __shfl_xor_sync(FULL, n_acc, d);
     n_ign += __shfl_xor_sync(FULL, n_ign, d);
+    n_cv += __shfl_xor_sync(FULL, n_cv, d);
   }
   if (lane == 0) {
     if (n_acc) atomicAdd(&p.st->access_words, (unsigned long long)n_acc);
     if (n_ign) atomicAdd(&p.st->ignored_words, (unsigned long long)n_ign);
+    if (n_cv) atomicAdd(&p.st->n_cv_acc, (unsigned long long)n_cv);
   }
 }
 

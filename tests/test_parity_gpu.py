@@ -616,3 +616,20 @@ def test_bo_tags_fuzz(orc, seed):
     if exp.rc == 0:
         rc, got, shadow, _ = run_gpu(rec, base, span, flags=8, flush_points=_cuts(rec, 5, seed))
         assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+# ---- N1: CV -> OV translation (ARB_CV_BASE, CV-addressed target accesses, Z26) -----
+@pytest.mark.parametrize("seed", range(8))
+def test_cv_addressed_fuzz(orc, seed):
+    """Random programs whose target accesses to mapped words use CV (device) addresses:
+    the batch is partitioned, the CV placements resolved, the accesses translated and
+    the batch partitioned again; with flush cuts (placements carried across flushes),
+    with the buffer-overflow extension, and with only half of the accesses rewritten."""
+    from gen.fuzz import random_program, to_cv_addressing
+    rec, base, span = random_program(9400 + seed, p_task=0.3, steps=100)
+    cv = to_cv_addressing(rec, frac=1.0 if seed % 2 else 0.5, seed=seed)
+    exp, _ = check(orc, cv, base, span)
+    check(orc, cv, base, span, flags=8)
+    if exp.rc == 0:
+        rc, got, shadow, _ = run_gpu(cv, base, span, flush_points=_cuts(cv, 4, seed))
+        assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
