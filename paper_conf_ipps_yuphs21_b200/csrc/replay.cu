@@ -348,9 +348,9 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
 }
 
 // ---- direct step: at most one write per word, every word near the step's first ------------
-// Same computation as step_fast, with the hash replaced by a window of kDSlots
-// words centred on the step's first word: slot = word - anchor, no hashing and
-// no probing.  A write claims its slot with one CAS ({step index << 4 | code});
+// Same computation as step_fast, with the hash replaced by two windows of
+// kDSlots / 2 words anchored at the step's first and last events: slot = word -
+// anchor, no hashing and no probing.  A write claims its slot with one CAS ({step index << 4 | code});
 // a read's state-before is the initial state, or the image of the slot's write
 // when that write comes earlier in the step.  Returns false (nothing written,
 // table clean) if a word has two writes or an event lies outside the window;
@@ -363,7 +363,11 @@ __device__ __forceinline__ bool step_direct(ReplaySmem& S, const ReplayParams& p
   bool bad = false, oow = false;
   const uint8_t* sh = S.shrel;
   uint32_t* tab = S.u.d.w;
-  const uint32_t anchor = (ev[0].x & kWordMask) - (uint32_t)(kDSlots / 2);
+  // two windows of kDSlots / 2 words, from 1/8 below the step's first and its last
+  // word (a step usually spans at most two runs of an access stream); a word in
+  // both maps to the first
+  constexpr uint32_t kW = kDSlots / 2, kBelow = kW / 8;
+  const uint32_t anchor_a = (ev[0].x & kWordMask) - kBelow, anchor_b = (ev[m - 1].x & kWordMask) - kBelow;
   uint32_t plo = 0, pw = 0;
   if (PARTIAL) { plo = S.part_lo; pw = S.part_hi - S.part_lo; }
 #pragma unroll
@@ -377,8 +381,9 @@ __device__ __forceinline__ bool step_direct(ReplaySmem& S, const ReplayParams& p
       if (!PARTIAL || word[j] - plo < pw) s_pre[j] = __ldcg(sh + word[j]);
       else op[j] = 4;                                       // another work item's word
       if (BO && (op[j] & 2u) && !(s_pre[j] & kCVp)) { bom |= 1u << j; op[j] = 4; }
-      idx[j] = word[j] - anchor;
-      if (op[j] < 4 && idx[j] >= (uint32_t)kDSlots) { oow = true; op[j] |= 8u; }   // outside the window
+      const uint32_t da = word[j] - anchor_a, db = word[j] - anchor_b;
+      idx[j] = da < kW ? da : kW + db;
+      if (op[j] < 4 && da >= kW && db >= kW) { oow = true; op[j] |= 8u; }   // outside both windows
     }
   }
   bool any_w = false;
@@ -1019,7 +1024,7 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
           }
         }
         if (tid == 0) {
-          S.skip_direct = oow ? 8u : (skip ? skip - 1u : 0u);
+          S.skip_direct = oow ? 4u : (skip ? skip - 1u : 0u);
           atomicAdd(fast ? &p.st->steps_fast : &p.st->steps_sort, 1ull);
         }
       }
