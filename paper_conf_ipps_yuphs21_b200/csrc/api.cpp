@@ -111,7 +111,7 @@ struct arb_ctx_s {
   HostBuf<uint4> h_slice_items, h_hot;
   DevBuf<uint64_t> d_hot_off;
   HostBuf<uint64_t> h_hot_off;
-  DevBuf<uint16_t> hot_F;
+  DevBuf<uint32_t> hot_F;
   DevBuf<uint8_t> hot_P;
   DevBuf<uint4> d_items;
   HostBuf<uint4> h_items;
@@ -423,14 +423,12 @@ static void build_items(arb_ctx ctx, const FlushPlan& plan, const std::vector<do
   const double share = ev_tot / double(std::max(1, ctx->n_sms * kReplayCtasPerSm));
   const bool force_hot = ctx->cfg.flags & ARB_F_SMALL_PARTS;     // test knob: slice every small busy bucket
   std::vector<uint32_t> slices(nb, 0);
-  constexpr uint64_t kMaxHotEntries = 1ull << 29;      // K5 scratch: 3 B per entry
+  constexpr uint64_t kMaxHotEntries = 1ull << 29;      // K5 scratch: 5 B per entry
   uint64_t hot_total = 0;
   for (uint32_t b = 0; b < nb && b < bucket_events.size(); ++b) {
     const uint64_t span = ctx->bucket_start[b + 1] - ctx->bucket_start[b];
     const double ev = bucket_events[b];
     if (parts[b] != 1 || span > kHotSpan) continue;
-    if (ctx->cfg.flags & ARB_F_BO) continue;      // slice functions cannot express the BO condition (Z20)
-    if ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u) continue;   // nor 8-bit states (Z24)
     const bool hot = force_hot ? ev >= 64.0 : (ev > 1.25 * share && ev > kSliceEvents);
     if (!hot) continue;
     const double want = force_hot ? 3.0 : std::ceil(ev / kSliceEvents);
@@ -741,7 +739,6 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   rp.shadow = ctx->shadow; rp.bo = (ctx->cfg.flags & ARB_F_BO) ? 1u : 0u;
   rp.um = (ctx->cfg.flags & ARB_F_UNIFIED) ? 1u : 0u;
   rp.md = ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u) ? 1u : 0u; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
-  rp.no_direct = getenv("ARB_NO_DIRECT") ? 1u : 0u;
   rp.cand = ctx->cand.p; rp.cand_cap = ctx->cand_cap; rp.st = ctx->dstats.p;
   rp.hot_off = ctx->d_hot_off.p; rp.hot_F = ctx->hot_F.p; rp.hot_P = ctx->hot_P.p;
   int n_ctas = std::max(1, std::min<int>((int)ctx->items.size(), ctx->n_sms * kReplayCtasPerSm));
@@ -751,7 +748,8 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     uint32_t max_span = 0;
     for (const uint4& h : ctx->hot) max_span = std::max(max_span, h.z);
     CK(launch_carry(ctx->d_hot.p, (uint32_t)ctx->hot.size(), max_span, ctx->d_bucket_start.p, ctx->d_hot_off.p,
-                    ctx->hot_F.p, ctx->hot_P.p, ctx->shadow, s), "k_carry");
+                    ctx->hot_F.p, ctx->hot_P.p, ctx->shadow, (ctx->cfg.flags & ARB_F_BO) ? 1 : 0,
+                    ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u) ? 1 : 0, s), "k_carry");
     CK(cudaMemsetAsync(&ctx->dstats.p->work, 0, sizeof(unsigned long long), s), "work reset");
     ReplayParams r3 = rp;
     r3.items = ctx->d_slice_items.p; r3.n_items = (uint32_t)ctx->slice_items.size();

@@ -165,15 +165,14 @@ struct ReplayParams {
   const uint4* items; uint32_t n_items;   // work items in scheduling order (largest first):
                                           // {bucket, y, z, kItem*}
   // hot buckets (K5): bucket b's scratch starts at entry hot_off[b] of hot_F
-  // (slice functions, u16 selector form) and hot_P (carried-in states, u8);
+  // (slice functions, 32 bits: see kfun_* in replay.cu) and hot_P (carried-in states, u8);
   // slice k uses [hot_off[b] + k * span16, + span16), span16 = span rounded to 16
-  const uint64_t* hot_off; uint16_t* hot_F; uint8_t* hot_P;
+  const uint64_t* hot_off; uint32_t* hot_F; uint8_t* hot_P;
   uint64_t n_words;
   uint8_t* shadow;                        // n_words bytes
   uint32_t bo;                            // ARB_F_BO: target accesses to words without kCVp are BO
   uint32_t um;                            // ARB_F_UNIFIED: OV and CV are one storage (Z23)
   uint32_t md;                            // several accelerators (Z24): 8-bit states, device in pos bits 30-31
-  uint32_t no_direct;                     // debug: never use the direct step
   const uint32_t* ops_start;              // [n_buckets + 1]
   const BucketOp* ops;
   uint4* cand; uint64_t cand_cap;         // report candidates {word lo, word hi, pos, kind}
@@ -220,8 +219,8 @@ cudaError_t launch_replay(const ReplayParams& p, int n_ctas, cudaStream_t s);
 // K5 phase 2: for every hot bucket {bucket, slices, span, 0} carry the states
 // across its slices: P_0 = shadow, P_{k+1} = F_k(P_k); shadow = F_last(P_last)
 cudaError_t launch_carry(const uint4* hot, uint32_t n_hot, uint32_t max_span, const uint64_t* bucket_start,
-                         const uint64_t* hot_off, const uint16_t* hot_F, uint8_t* hot_P, uint8_t* shadow,
-                         cudaStream_t s);
+                         const uint64_t* hot_off, const uint32_t* hot_F, uint8_t* hot_P, uint8_t* shadow,
+                         int bo, int md, cudaStream_t s);
 cudaError_t launch_mir(const MirParams& p, uint64_t n_ins_pos, uint64_t n_qry_pos, uint64_t n_rr_words,
                        cudaStream_t s, int* launches);
 // N1 (Z26): copy the batch, translating CV-addressed target accesses to OV addresses

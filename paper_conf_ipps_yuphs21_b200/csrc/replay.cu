@@ -8,9 +8,6 @@
 // the bucket's shadow at their trace positions, and processes the events in
 // steps of <= 1024 that never straddle a range op:
 //
-//   direct step (at most one write per word, every word within +-4096 of the
-//              step's first word): a direct-mapped table word - anchor -> the
-//              word's write, no hashing or probing; else
 //   fast step  (every word has at most one write in the step): a shared-memory
 //              hash of the written words, word -> write position.  A read's
 //              state-before is the initial state, or the image of the one
@@ -38,7 +35,6 @@ constexpr int STEP = RT * RI;                // 2048 events per step
 static_assert(RT >= 256 && STEP <= 4096, "sort_pass digit loop and u16 offsets");
 constexpr int kWin = 2 * RT;                 // segment descriptors staged per step
 constexpr int kHSlots = 4096;                // hash slots (load <= 1/2)
-constexpr int kDSlots = 2 * kHSlots;         // direct-step window (words), same bytes as the hash
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
 constexpr uint32_t kWordMask = 0x3FFFFFFFu;
 constexpr int kZSlots = 2048;                // summary-step hash slots (<= 1024 writes per step)
@@ -49,7 +45,6 @@ struct ReplaySmem {
   union {
     struct { uint32_t keyA[STEP], posA[STEP], keyB[STEP], posB[STEP]; uint16_t hist[RT / 32][256]; } s;
     struct { uint2 slot[kHSlots]; } h;      // fast step: written words {word, pos << 2 | op}
-    struct { uint32_t w[kDSlots]; } d;      // direct step: word - anchor -> {step index << 4 | write code}
     struct { uint32_t key[kZSlots], lastw[kZSlots], anyw[kZSlots]; } z;  // hot-slice summary step (K5)
   } u;
   uint32_t wstart[kWin];          // staged segment list window: global event index
@@ -61,9 +56,8 @@ struct ReplaySmem {
   uint32_t part_lo, part_hi;      // the work item's word range inside the bucket
   bool partial;                   //   (partial: not the whole bucket)
   uint32_t mode;                  // kItem* of the work item
-  uint32_t skip_direct;           // steps left before the direct step is tried again
   uint8_t* shrel;                 // state of bucket-relative word w: shrel[w]
-  uint16_t* fsum;                 // summary slice: composed transition of word w: fsum[w]
+  uint32_t* fsum;                 // summary slice: composed transition of word w: fsum[w] (kfun_*)
   uint32_t slice, n_slices;       // hot bucket slice (kItemSlice / kItemSummary)
   uint32_t seg0, cum0, n_segs, n_events, wsc, nwin;
   uint64_t bucket_base;
@@ -95,6 +89,32 @@ __device__ __forceinline__ void block_minmax(uint32_t& lo, uint32_t& hi, uint32_
   lo = 0xFFFFFFFFu; hi = 0;
 #pragma unroll
   for (int w = 0; w < RT / 32; ++w) { lo = min(lo, r1[w]); hi = max(hi, r2[w]); }
+}
+
+// ---- K5 slice functions (32 bits per word) -------------------------------------------------
+// default / UM: a 4-bit selector (low 16 bits); ARB_F_BO (Z20): a pair of selectors
+// with CVp actions, the low half for a word entering the slice without a CV, the
+// high half with one (a target write is the identity on a word without a CV, so
+// the function depends on CVp); several accelerators (Z24): an 8-output selector.
+template <bool BO, bool MD>
+__device__ __forceinline__ uint32_t kfun_id() { return MD ? kSel8Id : BO ? (kSelId | (kSelId << 16)) : kSelId; }
+// an unconditional transition g (range op) after f
+template <bool BO, bool MD>
+__device__ __forceinline__ uint32_t kfun_then(uint32_t g, uint32_t f) {
+  if (MD) return sel8_compose(g, f);
+  if (BO) return sel_compose(g, f & 0xFFFFu) | (sel_compose(g, f >> 16) << 16);
+  return sel_compose(g, f);
+}
+// CVp after selector half h for a word entering with CVp = c (bits 12-13: 0 keep, 2 clear, 3 set)
+__device__ __forceinline__ uint32_t half_cvp(uint32_t h, uint32_t c) {
+  const uint32_t pop = (h >> 12) & 3u;
+  return pop == 0 ? c : (pop == 3 ? 1u : 0u);
+}
+template <bool BO, bool MD>
+__device__ __forceinline__ uint32_t kfun_apply(uint32_t f, uint32_t s) {
+  if (MD) return sel8_apply4(f, s) & 255u;
+  if (BO) return sel_apply5((s & kCVp) ? f >> 16 : f & 0xFFFFu, s) & 31u;
+  return sel_apply4(f, s) & 15u;
 }
 
 // ---- range ops ----------------------------------------------------------------
@@ -157,7 +177,7 @@ __device__ void apply_ops_before(ReplaySmem& S, const ReplayParams& p, uint32_t 
       // hot slice, phase 1: compose the op into the words' slice functions
       for (uint64_t j = lo + threadIdx.x; j < hi; j += RT) {
         const uint32_t w = (uint32_t)(j - S.bucket_base);
-        S.fsum[w] = (uint16_t)sel_compose(sel, S.fsum[w]);
+        S.fsum[w] = kfun_then<BO, MD>(sel, S.fsum[w]);
       }
     } else if (hi > lo) {
       stream_apply<BO, MD>(S.shrel, lo - S.bucket_base, hi - S.bucket_base, sel);
@@ -343,98 +363,6 @@ __device__ __forceinline__ bool step_fast(ReplaySmem& S, const ReplayParams& p, 
     for (int j = 0; j < RI; ++j)
       if (op[j] & 1u) hs[slot[j]] = make_uint2(kEmpty, kEmpty);
   }
-  // the caller's next barrier orders this reset before the next step's inserts
-  return true;
-}
-
-// ---- direct step: at most one write per word, every word near the step's first ------------
-// Same computation as step_fast, with the hash replaced by two windows of
-// kDSlots / 2 words anchored at the step's first and last events: slot = word -
-// anchor, no hashing and no probing.  A write claims its slot with one CAS ({step index << 4 | code});
-// a read's state-before is the initial state, or the image of the slot's write
-// when that write comes earlier in the step.  Returns false (nothing written,
-// table clean) if a word has two writes or an event lies outside the window;
-// *oow reports the latter (the caller then prefers the hash step for a while).
-template <bool PARTIAL, bool BO, bool UM, bool MD>
-__device__ __forceinline__ bool step_direct(ReplaySmem& S, const ReplayParams& p, const uint2* ev, uint32_t m,
-                                            bool* oow_out) {
-  uint32_t idx[RI], word[RI], pos[RI], op[RI], s_pre[RI];
-  uint32_t bom = 0, devs = 0;
-  bool bad = false, oow = false;
-  const uint8_t* sh = S.shrel;
-  uint32_t* tab = S.u.d.w;
-  // two windows of kDSlots / 2 words, from 1/8 below the step's first and its last
-  // word (a step usually spans at most two runs of an access stream); a word in
-  // both maps to the first
-  constexpr uint32_t kW = kDSlots / 2, kBelow = kW / 8;
-  const uint32_t anchor_a = (ev[0].x & kWordMask) - kBelow, anchor_b = (ev[m - 1].x & kWordMask) - kBelow;
-  uint32_t plo = 0, pw = 0;
-  if (PARTIAL) { plo = S.part_lo; pw = S.part_hi - S.part_lo; }
-#pragma unroll
-  for (int j = 0; j < RI; ++j) {   // shadow loads first: their latency overlaps the table work
-    const uint32_t i = threadIdx.x + j * RT;
-    word[j] = 0; pos[j] = 0; op[j] = 4; s_pre[j] = 0; idx[j] = 0;
-    if (i < m) {
-      const uint2 e = ev[i];
-      word[j] = e.x & kWordMask; op[j] = e.x >> 30; pos[j] = MD ? (e.y & kMdPos) : e.y;
-      if (MD) devs |= (e.y >> 30) << (2 * j);
-      if (!PARTIAL || word[j] - plo < pw) s_pre[j] = __ldcg(sh + word[j]);
-      else op[j] = 4;                                       // another work item's word
-      if (BO && (op[j] & 2u) && !(s_pre[j] & kCVp)) { bom |= 1u << j; op[j] = 4; }
-      const uint32_t da = word[j] - anchor_a, db = word[j] - anchor_b;
-      idx[j] = da < kW ? da : kW + db;
-      if (op[j] < 4 && da >= kW && db >= kW) { oow = true; op[j] |= 8u; }   // outside both windows
-    }
-  }
-  bool any_w = false;
-  uint32_t won = 0;
-#pragma unroll
-  for (int j = 0; j < RI; ++j) {
-    // every write counts (one outside the window forces the fallback below, or a
-    // later read of its word would miss it); in-window writes claim their slot
-    if ((op[j] & 5u) == 1u) any_w = true;      // WH = 1, WT = 3 (| 8 outside the window)
-    if ((op[j] & 13u) == 1u) {                 // an in-window write
-      const uint32_t i = threadIdx.x + j * RT;
-      const uint32_t code = MD ? ((((devs >> (2 * j)) & 3u) << 1) | (op[j] >> 1)) : op[j];
-      if (atomicCAS(&tab[idx[j]], kEmpty, (i << 4) | code) == kEmpty) won |= 1u << j;
-      else bad = true;                                      // a second write of the word
-    }
-  }
-  any_w = __syncthreads_or(any_w);
-  if (any_w && __syncthreads_or(bad || oow)) {
-#pragma unroll
-    for (int j = 0; j < RI; ++j)
-      if ((won >> j) & 1u) tab[idx[j]] = kEmpty;
-    *oow_out = __syncthreads_or(oow);
-    return false;
-  }
-  uint32_t fk[RI];
-#pragma unroll
-  for (int j = 0; j < RI; ++j) {
-    const uint32_t o = op[j] & 7u;
-    const uint32_t s0 = s_pre[j] & (MD ? 255u : 15u);
-    uint32_t before = s0;
-    if (o == OP_RH || o == OP_RT) {
-      if (any_w) {
-        const uint32_t t = tab[idx[j]];
-        if (t != kEmpty && (t >> 4) < threadIdx.x + j * RT)
-          before = MD ? md_write(t & 7u, s0) : UM ? 15u : vsm_write_op(t & 3u, s0);
-      }
-    } else if (o & 1u) {
-      __stcg(const_cast<uint8_t*>(sh) + word[j],
-             (uint8_t)(MD ? md_write((o >> 1) | (((devs >> (2 * j)) & 3u) << 1), s0)
-                       : UM ? 15u : vsm_write_op(o, s0) | (BO ? (s_pre[j] & kCVp) : 0u)));
-    }
-    fk[j] = ((bom >> j) & 1u) ? 4u : MD ? md_classify(o, (devs >> (2 * j)) & 3u, before) : classify_bits(o, before);
-  }
-  emit_faults(p, fk, word, pos, S.bucket_base);
-  if (any_w) {
-    __syncthreads();
-#pragma unroll
-    for (int j = 0; j < RI; ++j)
-      if ((won >> j) & 1u) tab[idx[j]] = kEmpty;
-  }
-  *oow_out = false;
   // the caller's next barrier orders this reset before the next step's inserts
   return true;
 }
@@ -690,15 +618,18 @@ __device__ void step_sort(ReplaySmem& S, const ReplayParams& p, const uint2* ev,
 // slice (selector form; reads are identity).  Within a step a word's
 // writes compose to: valid bits of the last write, OVi set if any WH, CVi set if
 // any WT (Table II init bits); the last write of each word (by step
-// index) folds that function into fsum.
-template <bool UM>
+// index) folds that function into fsum.  ARB_F_BO: CVp is constant inside a step
+// (range ops cut steps), so for each half of the pair the word's CVp after the
+// slice so far decides whether its target writes count (Z20).  Several
+// accelerators: the last write's device and the devices any WT initialised (Z24).
+template <bool BO, bool UM, bool MD>
 __device__ void step_summary(ReplaySmem& S, const uint2* ev, uint32_t m) {
   uint32_t* key = S.u.z.key;
   uint32_t* lastw = S.u.z.lastw;
   uint32_t* anyw = S.u.z.anyw;
   uint32_t word[RI], op[RI], idx[RI], slot[RI];
   bool last[RI];
-  uint32_t ab[RI];
+  uint32_t ab[RI], lw[RI];
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
     const uint32_t i = threadIdx.x + j * RT;
@@ -706,6 +637,7 @@ __device__ void step_summary(ReplaySmem& S, const uint2* ev, uint32_t m) {
     if (i < m) {
       const uint2 e = ev[i];
       word[j] = e.x & kWordMask; op[j] = e.x >> 30;
+      const uint32_t dev = MD ? e.y >> 30 : 0u;
       if (op[j] & 1u) {                // a write: find or insert the word's slot
         uint32_t h = (word[j] * 2654435761u) >> 21;        // 11 bits
         for (;;) {
@@ -714,25 +646,50 @@ __device__ void step_summary(ReplaySmem& S, const uint2* ev, uint32_t m) {
           h = (h + 1) & (kZSlots - 1);
         }
         slot[j] = h;
-        atomicMax(&lastw[h], (idx[j] << 2) | op[j]);
-        atomicOr(&anyw[h], op[j] == OP_WH ? 1u : 2u);
+        atomicMax(&lastw[h], (idx[j] << 4) | (dev << 2) | op[j]);
+        atomicOr(&anyw[h], op[j] == OP_WH ? 1u : (2u << dev));   // bit 0 WH, bit 1 + d WT on device d
       }
     }
   }
   __syncthreads();
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
-    last[j] = (op[j] & 1u) && (lastw[slot[j]] >> 2) == idx[j];
+    const uint32_t l = (op[j] & 1u) ? lastw[slot[j]] : 0u;
+    last[j] = (op[j] & 1u) && (l >> 4) == idx[j];
     ab[j] = last[j] ? anyw[slot[j]] : 0u;
+    lw[j] = l & 15u;
   }
   __syncthreads();
 #pragma unroll
   for (int j = 0; j < RI; ++j) {
     if (last[j]) {
-      const Sel g = UM ? sel_make(5, 5, 5, 5)                                      // Z23: one shared value
-                  : op[j] == OP_WH ? sel_make(5, 4, 5, (ab[j] & 2u) ? 5 : 3)     // OV latest; CVi kept unless a WT
-                                   : sel_make(4, 5, (ab[j] & 1u) ? 5 : 2, 5);    // CV latest; OVi kept unless a WH
-      S.fsum[word[j]] = (uint16_t)sel_compose(g, S.fsum[word[j]]);
+      const uint32_t f = S.fsum[word[j]];
+      uint32_t nf;
+      if (MD) {
+        const uint32_t ldev = (lw[j] >> 2) & 3u;
+        const bool host = (lw[j] & 3u) == OP_WH;
+        uint32_t g = kSel8Id;
+        g = sel8_set(g, 0, host ? 9u : 8u);                             // OVv: the last write was the host's
+        for (uint32_t d = 0; d < 3; ++d) {
+          g = sel8_set(g, md_cvv(d), (!host && ldev == d) ? 9u : 8u);   // only the writing device's CV valid
+          if (ab[j] & (2u << d)) g = sel8_set(g, md_cvi(d), 9u);       // initialised by a WT on d
+        }
+        if (ab[j] & 1u) g = sel8_set(g, 2, 9u);                        // OVi: some WH
+        nf = sel8_compose(g, f);
+      } else {
+        const Sel g = UM ? sel_make(5, 5, 5, 5)                                      // Z23: one shared value
+                    : op[j] == OP_WH ? sel_make(5, 4, 5, (ab[j] & 2u) ? 5 : 3)     // OV latest; CVi kept unless a WT
+                                     : sel_make(4, 5, (ab[j] & 1u) ? 5 : 2, 5);    // CV latest; OVi kept unless a WH
+        if (BO) {
+          // without a CV the step's target writes do nothing: only its host writes count
+          const Sel gh = (ab[j] & 1u) ? sel_make(5, 4, 5, 3) : kSelId;
+          const uint32_t lo = f & 0xFFFFu, hi = f >> 16;
+          nf = sel_compose(half_cvp(lo, 0u) ? g : gh, lo) | (sel_compose(half_cvp(hi, 1u) ? g : gh, hi) << 16);
+        } else {
+          nf = sel_compose(g, f);
+        }
+      }
+      S.fsum[word[j]] = nf;
       key[slot[j]] = kEmpty;           // the word's only slot: reset by its last writer
       lastw[slot[j]] = 0;
       anyw[slot[j]] = 0;
@@ -741,7 +698,7 @@ __device__ void step_summary(ReplaySmem& S, const uint2* ev, uint32_t m) {
   __syncthreads();
 }
 
-// Position of event e of the bucket (one thread).
+// Position of event e of the bucket (one thread; several accelerators: device bits stripped).
 __device__ uint32_t event_pos(const ReplaySmem& S, const ReplayParams& p, uint32_t e) {
   uint32_t lo = 0, z = S.n_segs;
   while (z - lo > 1) {
@@ -749,7 +706,8 @@ __device__ uint32_t event_pos(const ReplaySmem& S, const ReplayParams& p, uint32
     if (p.segs[S.seg0 + mid].w - S.cum0 <= e) lo = mid; else z = mid;
   }
   const uint4 sg = p.segs[S.seg0 + lo];
-  return p.part_ev[(uint64_t)sg.x * kChunkCap + (sg.z & 0xFFFFu) + (e - (sg.w - S.cum0))].y;
+  const uint32_t pos = p.part_ev[(uint64_t)sg.x * kChunkCap + (sg.z & 0xFFFFu) + (e - (sg.w - S.cum0))].y;
+  return p.md ? (pos & kMdPos) : pos;
 }
 // first op of the bucket (ops [a, z), trace order) at or after position q
 __device__ uint32_t ops_lower_bound(const ReplayParams& p, uint32_t a, uint32_t z, uint32_t q) {
@@ -761,8 +719,9 @@ __device__ uint32_t ops_lower_bound(const ReplayParams& p, uint32_t a, uint32_t 
 }
 
 // Phase 2: carry the word states across the slices (grid: words x hot buckets).
+template <bool BO, bool MD>
 __global__ void k_carry(const uint4* hot, const uint64_t* bucket_start, const uint64_t* hot_off,
-                        const uint16_t* hot_F, uint8_t* hot_P, uint8_t* shadow) {
+                        const uint32_t* hot_F, uint8_t* hot_P, uint8_t* shadow) {
   const uint4 h = hot[blockIdx.y];
   const uint32_t b = h.x, slices = h.y, span = h.z, span16 = (span + 15) & ~15u;
   const uint64_t off = hot_off[b];
@@ -771,18 +730,19 @@ __global__ void k_carry(const uint4* hot, const uint64_t* bucket_start, const ui
     uint32_t st = sh[w];
     for (uint32_t k = 0; k < slices; ++k) {
       hot_P[off + (uint64_t)k * span16 + w] = (uint8_t)st;
-      st = sel_apply4(hot_F[off + (uint64_t)k * span16 + w], st) & 15u;   // K5 never runs with ARB_F_BO
+      st = kfun_apply<BO, MD>(hot_F[off + (uint64_t)k * span16 + w], st);
     }
     sh[w] = (uint8_t)st;
   }
 }
 
 cudaError_t launch_carry(const uint4* hot, uint32_t n_hot, uint32_t max_span, const uint64_t* bucket_start,
-                         const uint64_t* hot_off, const uint16_t* hot_F, uint8_t* hot_P, uint8_t* shadow,
-                         cudaStream_t s) {
+                         const uint64_t* hot_off, const uint32_t* hot_F, uint8_t* hot_P, uint8_t* shadow,
+                         int bo, int md, cudaStream_t s) {
   if (!n_hot) return cudaSuccess;
   const uint32_t gx = std::min<uint32_t>((max_span + 255) / 256, 1024);
-  k_carry<<<dim3(gx, n_hot), 256, 0, s>>>(hot, bucket_start, hot_off, hot_F, hot_P, shadow);
+  auto kern = md ? k_carry<false, true> : bo ? k_carry<true, false> : k_carry<false, false>;
+  kern<<<dim3(gx, n_hot), 256, 0, s>>>(hot, bucket_start, hot_off, hot_F, hot_P, shadow);
   return cudaGetLastError();
 }
 
@@ -945,7 +905,6 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       S.op_end = p.ops_start[b + 1];
       S.bucket_base = p.bucket_start[b];
       S.shrel = p.shadow + S.bucket_base;
-      S.skip_direct = 0;
     }
     bucket_setup(S, p, b);
     uint32_t first = 0, total = S.n_events;
@@ -972,7 +931,7 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       }
       __syncthreads();
       if (mode == kItemSummary) {
-        for (uint32_t w = tid; w < span; w += RT) S.fsum[w] = (uint16_t)kSelId;
+        for (uint32_t w = tid; w < span; w += RT) S.fsum[w] = kfun_id<BO, MD>();
         for (uint32_t w = tid; w < kZSlots; w += RT) { S.u.z.key[w] = kEmpty; S.u.z.lastw[w] = 0; S.u.z.anyw[w] = 0; }
         __syncthreads();
       }
@@ -1006,27 +965,12 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         cut = block_sum(cnt, S.red);
       }
       if (mode == kItemSummary) {
-        step_summary<UM>(S, ev, cut);
+        step_summary<BO, UM, MD>(S, ev, cut);
       } else {
-        bool fast = false, oow = false;
-        const uint32_t skip = p.no_direct ? 1u : S.skip_direct;
-        if (!skip) {
-          fast = S.partial ? step_direct<true, BO, UM, MD>(S, p, ev, cut, &oow)
-                           : step_direct<false, BO, UM, MD>(S, p, ev, cut, &oow);
-        }
-        if (!fast) {
-          if (!skip && !oow) {           // two writes of a word: straight to the sort step
-            step_sort<BO, UM, MD>(S, p, ev, cut);
-          } else {
-            fast = S.partial ? step_fast_partial<BO, UM, MD>(S, p, ev, cut)
-                             : step_fast<false, BO, UM, MD>(S, p, ev, cut);
-            if (!fast) step_sort<BO, UM, MD>(S, p, ev, cut);
-          }
-        }
-        if (tid == 0) {
-          S.skip_direct = oow ? 4u : (skip ? skip - 1u : 0u);
-          atomicAdd(fast ? &p.st->steps_fast : &p.st->steps_sort, 1ull);
-        }
+        const bool fast = S.partial ? step_fast_partial<BO, UM, MD>(S, p, ev, cut)
+                                    : step_fast<false, BO, UM, MD>(S, p, ev, cut);
+        if (!fast) step_sort<BO, UM, MD>(S, p, ev, cut);
+        if (tid == 0) atomicAdd(fast ? &p.st->steps_fast : &p.st->steps_sort, 1ull);
       }
       e0 += cut;
       if (cut == m) {

@@ -261,7 +261,9 @@ def test_bo_fuzz_large_steps(orc, seed):
 
 
 def test_bo_config2_and_hot_word(orc):
-    """The DRACC-style suite and a hot word (no time slices under ARB_F_BO)."""
+    """The DRACC-style suite and a hot word under ARB_F_BO: the hot bucket is replayed
+    as K5 time slices whose per-word functions are selector pairs keyed by the CV
+    present bit (the CV is deleted and re-created between the slices' events)."""
     from gen.configs import config2
     from gen.trace import MAP, OP, TraceBuilder
     rec, base, size = config2()
@@ -281,7 +283,8 @@ def test_bo_config2_and_hot_word(orc):
         if j % 2 == 0:
             tb.exit(MAP.DELETE, A, 64)
     exp, st = check(orc, tb.array(), A, 64, flags=8)
-    assert st["hot_buckets"] == 0 and st["reports_bo"] > 0
+    assert st["hot_buckets"] >= 1 and st["reports_bo"] > 0
+    check(orc, tb.array(), A, 64, flags=8 | 4)         # forced slices of every busy bucket
 
 
 def test_bo_patterns(orc):
@@ -633,3 +636,26 @@ def test_cv_addressed_fuzz(orc, seed):
     if exp.rc == 0:
         rc, got, shadow, _ = run_gpu(cv, base, span, flush_points=_cuts(cv, 4, seed))
         assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+def test_devices_hot_word(orc):
+    """A hot word on 3 accelerators: K5 time slices with 8-output selector functions
+    (writes on different devices, transfers to and from each device between them)."""
+    from gen.trace import MAP, OP, TraceBuilder, encode_np
+    A = 0x8000
+    tb = TraceBuilder()
+    tb.wh(A)
+    rs = np.random.default_rng(8)
+    for j in range(12):
+        d = j % 3
+        tb.enter(MAP.TO | (d << 6), A, 64)
+        ops = rs.choice([OP.RT, OP.WT, OP.RH, OP.WH], size=40000, p=[.4, .2, .3, .1])
+        dev = np.where((ops == OP.RT) | (ops == OP.WT), rs.integers(0, 3, ops.size), 0)
+        tb.add_array(encode_np(0, np.full(ops.size, A, dtype=np.uint64), 8) |
+                     np.stack([(ops.astype(np.uint64) << np.uint64(48)) | (dev.astype(np.uint64) << np.uint64(56)),
+                               np.zeros(ops.size, np.uint64)], axis=1))
+        tb.exit(MAP.FROM | (d << 6), A, 64)
+    rec = tb.array()
+    exp, st = check(orc, rec, A, 64, flags=2 << 8)
+    assert st["hot_buckets"] >= 1
+    check(orc, rec, A, 64, flags=(2 << 8) | 4)
