@@ -410,3 +410,19 @@ def test_bo_overflow_into_adjacent_cv(orc):
         tb2.add_array(np.array([encode(OP.RT, A + 8 * i, 8, task=1)], dtype=np.uint64))
     tb2.exit(MAP.TO, A, 8 * n)
     assert run(orc, tb2.array(), A, 8 * n, detect_bo=True).triples() == []
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_dedup_first_is_first_per_word_kind(orc, seed):
+    """Z3: dedup-first mode returns exactly the earliest raw report of every
+    (word, kind) pair -- checked against the raw report list on random programs
+    with tasks (MIR), unaligned accesses and map errors avoided by the generator."""
+    from gen.fuzz import random_program
+    rec, base, span = random_program(7700 + seed, p_task=0.4, p_depend=0.2)
+    raw = run(orc, rec, base, span)
+    if raw.rc != 0:
+        pytest.skip("program rejected")
+    first = {}
+    for w, r, k in raw.triples():                    # canonical order: word, record, kind
+        first.setdefault((w, k), (w, r, k))
+    assert run(orc, rec, base, span, dedup_first=True).triples() == sorted(first.values())

@@ -175,8 +175,6 @@ def test_errors_leave_state_unchanged(orc, bad):
         tb.enter(MAP.TO, A + 32, 64)
     elif bad == "present":
         tb.enter(MAP.TO | MAP.PRESENT, A + 128, 64)       # not mapped: ARB_EMAP (Z21)
-    elif bad == "eopen":
-        tb.task_begin(3); tb.wt(A)
     elif bad == "nested":
         tb.task_begin(3); tb.task_begin(4)
     ctx = Context(A, 256)
