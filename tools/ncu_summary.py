@@ -89,9 +89,10 @@ def main():
         agg[k][0] += 1
         agg[k][1] += ms
     tot = sum(v[1] for v in agg.values()) or 1.0
-    lines = [f"# {name} — launch list of one bench step (config 5, rank 0)", "",
-             "`ncu --metrics gpu__time_duration.sum --clock-control none` over "
-             "`python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu` (cold-cache, serialised; "
+    what = os.environ.get("WHAT", "the first batch (one flush, ~1.0e9 records) of the whole config-5 trace, N = 1")
+    cmd = os.environ.get("CMD", "python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu --no-side --max-batches 1")
+    lines = [f"# {name} — launch list: {what}", "",
+             f"`ncu --metrics gpu__time_duration.sum --clock-control none` over `{cmd}` (cold-cache, serialised; "
              "compare shares, not absolutes).  Generator kernels run before the timed region "
              "and are excluded.", "",
              "| kernel | launches | total ms | share of library time |", "|---|---|---|---|"]
@@ -104,9 +105,9 @@ def main():
     if os.path.exists(rep):
         ks = full(rep)
         cols = [k for k, _, _ in ks]
-        lines = [f"# {name} — ncu --set full of the hot kernels (first flush of config 5, rank 0)", "",
-                 "`ncu --set full --clock-control none --import-source on -k regex:\"k_partition|k_replay\" -c 2 "
-                 "python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu`", "",
+        lines = [f"# {name} — ncu --set full of the hot kernels: {what}", "",
+                 f"`ncu --set full --clock-control none --import-source on -k regex:\"k_partition|k_replay\" -c 2 {cmd}`",
+                 "",
                  "| metric | " + " | ".join(cols) + " |", "|---|" + "---|" * len(cols)]
         for m in METRICS:
             vals = [d.get(m, "") for _, d, _ in ks]
@@ -129,7 +130,7 @@ def main():
             recs = old.get("records_in_launch")
             tj[kk] = {"dram_bytes_per_launch": rd + wr, "read": rd, "write": wr,
                       "records_in_launch": int(sys.argv[3]) if len(sys.argv) > 3 else recs,
-                      "source": f"profiles/{name}_ncu_full.md (first flush of config 5, rank 0)"}
+                      "source": f"profiles/{name}_ncu_full.md ({what})"}
         with open(tj_path, "w") as fh:
             json.dump(tj, fh, indent=1)
     print("\n".join(lines))
