@@ -80,6 +80,7 @@ constexpr int kReplayThreads = 256;
 constexpr int kReplayItems = 4;
 constexpr int kStep = kReplayThreads * kReplayItems;  // events per step
 constexpr int kReplayCtasPerSm = 4;
+constexpr int kReplayHashBits = 12;                  // fast-step hash: 2^12 slots
 
 // replay work items {bucket, y, z, kind}
 constexpr uint32_t kItemWhole = 0;      // the whole bucket

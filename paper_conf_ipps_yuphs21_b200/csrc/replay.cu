@@ -31,13 +31,15 @@ namespace arb {
 
 constexpr int RT = kReplayThreads;           // threads per CTA (>= 256)
 constexpr int RI = kReplayItems;             // events per thread per step
-constexpr int STEP = RT * RI;                // 2048 events per step
+constexpr int STEP = RT * RI;                // events per step (1024)
 static_assert(RT >= 256 && STEP <= 4096, "sort_pass digit loop and u16 offsets");
 constexpr int kWin = 2 * RT;                 // segment descriptors staged per step
-constexpr int kHSlots = 4096;                // hash slots (load <= 1/2)
+constexpr int kHBits = kReplayHashBits;
+constexpr int kHSlots = 1 << kHBits;         // hash slots (load <= 1/2)
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
 constexpr uint32_t kWordMask = 0x3FFFFFFFu;
-constexpr int kZSlots = 2048;                // summary-step hash slots (<= 1024 writes per step)
+constexpr int kZBits = kHBits - 1;
+constexpr int kZSlots = 1 << kZBits;         // summary-step hash slots (>= 2 x the writes of a step)
 static_assert(kZSlots * 12 <= kHSlots * 8 && kZSlots >= 2 * STEP, "summary hash fits the hash area");
 
 struct ReplaySmem {
@@ -261,7 +263,7 @@ __device__ __forceinline__ uint32_t md_classify(uint32_t op, uint32_t dev, uint3
 
 // hash slot of a word (Fibonacci hashing: consecutive words land far apart, so
 // the linear probe chains of a run's words stay short)
-__device__ __forceinline__ uint32_t hslot(uint32_t w) { return (w * 2654435761u) >> 20; }
+__device__ __forceinline__ uint32_t hslot(uint32_t w) { return (w * 2654435761u) >> (32 - kHBits); }
 
 // ---- fast step: at most one write per word -------------------------------------------
 // Returns false (and leaves the shadow untouched) if some word has two writes.
@@ -639,7 +641,7 @@ __device__ void step_summary(ReplaySmem& S, const uint2* ev, uint32_t m) {
       word[j] = e.x & kWordMask; op[j] = e.x >> 30;
       const uint32_t dev = MD ? e.y >> 30 : 0u;
       if (op[j] & 1u) {                // a write: find or insert the word's slot
-        uint32_t h = (word[j] * 2654435761u) >> 21;        // 11 bits
+        uint32_t h = (word[j] * 2654435761u) >> (32 - kZBits);
         for (;;) {
           const uint32_t old = atomicCAS(&key[h], kEmpty, word[j]);
           if (old == kEmpty || old == word[j]) break;
