@@ -15,7 +15,10 @@ constexpr int kKindBits = 3;
 __device__ __forceinline__ uint32_t rs_field(uint4 c, int f) {
   return f == 0 ? c.w : f == 1 ? c.z : f == 2 ? c.x : f == 3 ? c.y : (c.z << kKindBits) | c.w;
 }
-__device__ __forceinline__ uint32_t rs_field(uint2 c, int f) { return f == 0 ? c.x : c.y; }
+// uint2 {0: x, 1: y, 2: segment entry chunk (x bits 0-20 | y bit 31 << 21)}
+__device__ __forceinline__ uint32_t rs_field(uint2 c, int f) {
+  return f == 0 ? c.x : f == 1 ? c.y : (c.x & ((1u << kSegChunkBits) - 1u)) | ((c.y >> 31) << kSegChunkBits);
+}
 template <class E>
 __device__ __forceinline__ uint32_t rs_digit(E c, RsPass ps) {
   return (rs_field(c, ps.field) >> ps.shift) & ((1u << ps.bits) - 1u);
@@ -406,9 +409,7 @@ cudaError_t launch_sort_segments(uint2* a, uint2* b, uint64_t n, int chunk_bits,
                                  uint32_t* first, uint4* out, cudaStream_t s, int* launches) {
   RsPass ps[8];
   int np = 0;
-  const int lo_bits = chunk_bits < kSegChunkBits ? chunk_bits : kSegChunkBits;
-  np = add_field_passes(ps, np, 0, lo_bits);
-  if (chunk_bits > kSegChunkBits) ps[np++] = RsPass{1, 31, 1};    // chunk bit 21 (batches > 2^29 records)
+  np = add_field_passes(ps, np, 2, chunk_bits);                // the whole chunk id (<= 22 bits: 2 passes)
   {
     int nbb = 1;
     while ((1u << nbb) < n_buckets) ++nbb;                      // bucket bits actually used
