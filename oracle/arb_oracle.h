@@ -26,7 +26,8 @@
  *   MIR predicate (Theorem 1, Z10)        pinned (schedule enumeration)
  *   MIR attribution to later event (Z11)  parity unpinned (definition only)
  *   dedup-first mode (Z3)                 parity unpinned (definition only)
- *   sub-word semantics (Z4)               parity unpinned (definition only)
+ *   sub-word semantics (Z4)               pinned (metamorphic: sub-word invariance and straddling
+ *                                         access = two word accesses, tests/test_oracle_metamorphic.py)
  *   several accelerators (Z24)            pinned (brute force vs the value simulator with one CV per device)
  *   map modifiers always/present (Z21)    pinned (brute force vs the value simulator's own refcount model)
  *   unified memory (Z23)                  pinned (brute force vs the value simulator with OV and CV aliased)
