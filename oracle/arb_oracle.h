@@ -24,7 +24,8 @@
  *                                         parity unpinned BY THE PAPER (Fig.1/Fig.2 do not split readings)
  *   Table I refcount resolution (Z5-Z7)   pinned (hand scenarios + brute force vs independent model)
  *   MIR predicate (Theorem 1, Z10)        pinned (schedule enumeration)
- *   MIR attribution to later event (Z11)  parity unpinned (definition only)
+ *   MIR attribution to later event (Z11)  pinned (brute-force pair search: a record is reported
+ *                                         iff it is the later op of a race, tests/test_theorem1.py)
  *   dedup-first mode (Z3)                 parity unpinned (definition only)
  *   sub-word semantics (Z4)               pinned (metamorphic: sub-word invariance and straddling
  *                                         access = two word accesses, tests/test_oracle_metamorphic.py)

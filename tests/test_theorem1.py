@@ -11,7 +11,9 @@ Pins:
     legal schedule is clean under Definition 1 (value simulator, P:79);
   * every reported MIR has a witness: an op of some nowait task instance on
     the same word, conflicting, whose join comes after the reported record,
-    found by a brute-force pair search independent of the oracle's log.
+    found by a brute-force pair search independent of the oracle's log; and
+    conversely every record with a witness is reported (reading Z11: one MIR
+    triple at the later op of each racing pair's word).
 """
 import numpy as np
 
@@ -169,6 +171,11 @@ def _run(orc, ntasks, nprog, seed, read_bias=0.0):
             if k == 3:
                 racy += 1
                 assert witness(recs, i), (items, i)
+        # Z11 attribution, both ways: a record is reported as MIR exactly when the
+        # brute-force pair search finds it the later op of a race
+        mir_at = {i for _, i, k in t if k == 3}
+        for idx in range(len(recs)):
+            assert witness(recs, idx) == (idx in mir_at), (items, idx)
         if t and all(k == 3 for _, _, k in t):
             # negative control: a MIR-only program usually has an unclean schedule
             pass
