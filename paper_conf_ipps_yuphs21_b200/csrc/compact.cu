@@ -9,30 +9,34 @@ constexpr int kRsThreads = 512, kRsItems = 8, kRsTile = kRsThreads * kRsItems;
 struct RsPass { int field; int shift; int bits; };
 constexpr int kRsMaxBits = 11;                    // digits of up to 11 bits (2048 bins)
 constexpr int kRsBins = 1 << kRsMaxBits;
-// digit fields: uint4 {0: w, 1: z, 2: x, 3: y, 4: z << 3 | w}; uint2 {0: x, 1: y}
-// (w = report kind, 1..4: 3 bits)
+// digit fields (64-bit): uint4 report candidates {x, y = word, z = record, w = kind}:
+// 0: kind, 1: record, 5: record << 3 | kind, 6: word, 7: kind << 30 | record (records < 2^30);
+// uint2 {0: x, 1: y} (w = report kind, 1..4: 3 bits)
 constexpr int kKindBits = 3;
-__device__ __forceinline__ uint32_t rs_field(uint4 c, int f) {
-  return f == 0 ? c.w : f == 1 ? c.z : f == 2 ? c.x : f == 3 ? c.y : (c.z << kKindBits) | c.w;
+__device__ __forceinline__ uint64_t rs_field(uint4 c, int f) {
+  return f == 0 ? c.w : f == 1 ? c.z : f == 5 ? ((uint64_t)c.z << kKindBits) | c.w
+       : f == 6 ? ((uint64_t)c.y << 32) | c.x : ((uint64_t)c.w << 30) | c.z;
 }
 // uint2 {0: x, 1: y, 2: segment entry chunk (x bits 0-20 | y bit 31 << 21)}
-__device__ __forceinline__ uint32_t rs_field(uint2 c, int f) {
+__device__ __forceinline__ uint64_t rs_field(uint2 c, int f) {
   return f == 0 ? c.x : f == 1 ? c.y : (c.x & ((1u << kSegChunkBits) - 1u)) | ((c.y >> 31) << kSegChunkBits);
 }
 template <class E>
 __device__ __forceinline__ uint32_t rs_digit(E c, RsPass ps) {
-  return (rs_field(c, ps.field) >> ps.shift) & ((1u << ps.bits) - 1u);
+  return (uint32_t)(rs_field(c, ps.field) >> ps.shift) & ((1u << ps.bits) - 1u);
 }
 
+// A block owns `sub` consecutive tiles of kRsTile elements (fewer, larger blocks
+// for large arrays: the digit-count matrix and its scan shrink by `sub`).
 template <class E>
 __global__ void __launch_bounds__(kRsThreads) k_rs_hist(const E* in, uint64_t n, RsPass ps, uint32_t* cnt,
-                                                        uint32_t nblk) {
+                                                        uint32_t nblk, uint32_t sub) {
   __shared__ uint32_t h[kRsBins];
   const int nd = 1 << ps.bits;
   for (int i = threadIdx.x; i < nd; i += kRsThreads) h[i] = 0;
   __syncthreads();
-  uint64_t base = (uint64_t)blockIdx.x * kRsTile;
-  for (int j = 0; j < kRsItems; ++j) {
+  const uint64_t base = (uint64_t)blockIdx.x * kRsTile * sub;
+  for (uint32_t j = 0; j < kRsItems * sub; ++j) {
     uint64_t i = base + (uint64_t)j * kRsThreads + threadIdx.x;
     if (i < n) atomicAdd(&h[rs_digit(in[i], ps)], 1u);
   }
@@ -118,19 +122,25 @@ static void scan_u32(uint32_t* a, uint64_t n, uint32_t* scratch, cudaStream_t s,
 // dynamic shared memory: hist[kRsThreads / 32][2^bits] u16 + dbase[2^bits] u32
 template <class E>
 __global__ void __launch_bounds__(kRsThreads) k_rs_scatter(const E* in, E* out, uint64_t n, RsPass ps,
-                                                           const uint32_t* cnt, uint32_t nblk) {
+                                                           const uint32_t* cnt, uint32_t nblk, uint32_t sub) {
   extern __shared__ __align__(16) uint8_t rs_smem[];
   const int nd = 1 << ps.bits;
   uint16_t* hist = reinterpret_cast<uint16_t*>(rs_smem);                     // [warp][nd]
   uint32_t* dbase = reinterpret_cast<uint32_t*>(rs_smem + (kRsThreads / 32) * nd * 2);
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   uint32_t* h32 = reinterpret_cast<uint32_t*>(hist);
+  for (int d = tid; d < nd; d += kRsThreads) dbase[d] = cnt[(uint64_t)d * nblk + blockIdx.x];
+  uint16_t* row = hist + warp * nd;
+  const uint32_t lt = lanemask_lt();
+  constexpr int kDig = kRsBins / kRsThreads;       // digits per thread in the offset pass
+  // the block's tiles in order; within a tile a stable rank per warp (kRsItems
+  // rounds of 32), then per-digit offsets across the warps
+  for (uint32_t t = 0; t < sub; ++t) {
+  const uint64_t base = ((uint64_t)blockIdx.x * sub + t) * kRsTile;
+  if (base >= n) break;
   for (uint32_t i = tid; i < (uint32_t)((kRsThreads / 32) * nd / 2); i += kRsThreads) h32[i] = 0;
   __syncthreads();
-  uint16_t* row = hist + warp * nd;
-  uint64_t base = (uint64_t)blockIdx.x * kRsTile;
   E c[kRsItems]; uint32_t rk[kRsItems], dg[kRsItems];
-  const uint32_t lt = lanemask_lt();
   for (int r = 0; r < kRsItems; ++r) {
     uint64_t i = base + warp * (32 * kRsItems) + r * 32 + lane;
     bool valid = i < n;
@@ -144,15 +154,24 @@ __global__ void __launch_bounds__(kRsThreads) k_rs_scatter(const E* in, E* out, 
     dg[r] = d; rk[r] = b + __popc(grp & lt);
   }
   __syncthreads();
-  for (int d = tid; d < nd; d += kRsThreads) {
+  uint32_t tot[kDig];
+#pragma unroll
+  for (int k = 0; k < kDig; ++k) {
+    const int d = tid + k * kRsThreads;
     uint32_t s = 0;
-    for (int w = 0; w < kRsThreads / 32; ++w) { uint32_t x = hist[w * nd + d]; hist[w * nd + d] = (uint16_t)s; s += x; }
-    dbase[d] = cnt[(uint64_t)d * nblk + blockIdx.x];
+    if (d < nd)
+      for (int w = 0; w < kRsThreads / 32; ++w) { uint32_t x = hist[w * nd + d]; hist[w * nd + d] = (uint16_t)s; s += x; }
+    tot[k] = s;
   }
   __syncthreads();
   for (int r = 0; r < kRsItems; ++r) {
     uint64_t i = base + warp * (32 * kRsItems) + r * 32 + lane;
     if (i < n) out[dbase[dg[r]] + row[dg[r]] + rk[r]] = c[r];
+  }
+  __syncthreads();
+#pragma unroll
+  for (int k = 0; k < kDig; ++k)
+    if (tid + k * kRsThreads < nd) dbase[tid + k * kRsThreads] += tot[k];
   }
 }
 
@@ -313,15 +332,19 @@ __global__ void k_dedup_canonical(const uint4* a, uint64_t n, uint4* out, uint64
 template <class E>
 static cudaError_t radix_sort(E*& a, E*& b, uint64_t n, const RsPass* passes, int np, uint32_t* cnt,
                               cudaStream_t s, int* launches) {
-  uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
+  // tiles per block: the largest power of two <= 8 that still gives >= 4 blocks per SM
+  // (the scatter walks its tiles one after the other)
+  uint32_t sub = 1;
+  while (sub < 8 && n / ((uint64_t)kRsTile * sub * 2) >= 4 * 148) sub *= 2;
+  const uint32_t nblk = (uint32_t)((n + (uint64_t)kRsTile * sub - 1) / ((uint64_t)kRsTile * sub));
   const size_t smem_max = (kRsThreads / 32) * kRsBins * 2 + kRsBins * 4;
   cudaError_t e = cudaFuncSetAttribute(k_rs_scatter<E>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_max);
   if (e != cudaSuccess) return e;
   for (int k = 0; k < np; ++k) {
     const uint64_t nd = 1ull << passes[k].bits;
-    k_rs_hist<E><<<nblk, kRsThreads, 0, s>>>(a, n, passes[k], cnt, nblk);
+    k_rs_hist<E><<<nblk, kRsThreads, 0, s>>>(a, n, passes[k], cnt, nblk, sub);
     scan_u32(cnt, (uint64_t)nblk * nd, cnt + (uint64_t)nblk * nd, s, launches);
-    k_rs_scatter<E><<<nblk, kRsThreads, (kRsThreads / 32) * nd * 2 + nd * 4, s>>>(a, b, n, passes[k], cnt, nblk);
+    k_rs_scatter<E><<<nblk, kRsThreads, (kRsThreads / 32) * nd * 2 + nd * 4, s>>>(a, b, n, passes[k], cnt, nblk, sub);
     *launches += 2;
     E* t = a; a = b; b = t;
   }
@@ -438,14 +461,11 @@ cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches
   uint64_t n = p.n_cand;
   RsPass ps[24];
   int np = 0;
-  int wb_lo = p.word_bits > 32 ? 32 : p.word_bits, wb_hi = p.word_bits > 32 ? p.word_bits - 32 : 0;
   cudaError_t e;
   if (p.dedup_first) {
     // (word, kind, pos): keep the first of each (word, kind)
-    np = add_field_passes(ps, np, 1, p.pos_bits);
-    np = add_field_passes(ps, np, 0, kKindBits);
-    np = add_field_passes(ps, np, 2, wb_lo);
-    np = add_field_passes(ps, np, 3, wb_hi);
+    np = add_field_passes(ps, np, 7, 30 + kKindBits);            // record, then kind (one field)
+    np = add_field_passes(ps, np, 6, p.word_bits);
     if ((e = radix_sort<uint4>(a, b, n, ps, np, p.blk, s, launches)) != cudaSuccess) return e;
     uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
     k_keep_count<<<nblk, kRsThreads, 0, s>>>(a, n, 1, p.blk);
@@ -479,14 +499,8 @@ cudaError_t launch_compact(const CompactParams& p, cudaStream_t s, int* launches
     *launches += 1;
     return cudaGetLastError();
   }
-  if (p.pos_bits + kKindBits <= 32) {
-    np = add_field_passes(ps, np, 4, p.pos_bits + kKindBits); // record, then kind
-  } else {
-    np = add_field_passes(ps, np, 0, kKindBits);
-    np = add_field_passes(ps, np, 1, p.pos_bits);
-  }
-  np = add_field_passes(ps, np, 2, wb_lo);
-  np = add_field_passes(ps, np, 3, wb_hi);
+  np = add_field_passes(ps, np, 5, p.pos_bits + kKindBits);   // record, then kind (one field)
+  np = add_field_passes(ps, np, 6, p.word_bits);
   if ((e = radix_sort<uint4>(a, b, n, ps, np, p.blk, s, launches)) != cudaSuccess) return e;
   uint32_t nblk = (uint32_t)((n + kRsTile - 1) / kRsTile);
   if (n == 0) {
