@@ -132,7 +132,8 @@ __device__ __forceinline__ void rank_round(uint32_t info, uint16_t* row, uint16_
 
 // The fast chunk test and its output.  Every record must be an access (op < 4)
 // of 1..8 bytes inside one 8-byte word (such an access cannot leave the
-// 48-bit space), and all words must lie in one address bucket.  Buckets are
+// 48-bit space), and all words must lie in one address bucket or in two
+// adjacent ones (a stable two-way split by the bucket boundary).  Buckets are
 // contiguous word ranges, so the test needs only the chunk's lowest and highest
 // word: each word is taken relative to record 0's word w0 (32-bit signed,
 // |d| < 2^30 as a bucket spans <= 2^30 words), the warp reduces min and max, and
@@ -170,18 +171,53 @@ __device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p,
   if (rlo >= p.n_words || rhi >= p.n_words) return false;
   const uint32_t cb = p.coarse_bits;
   const uint32_t mlo = __ldg(p.bin_map + (uint32_t)(rlo >> cb)), mhi = __ldg(p.bin_map + (uint32_t)(rhi >> cb));
-  const uint32_t bref = mlo & kBucketMask;
-  if (bref != (mhi & kBucketMask)) return false;
+  const uint32_t bref = mlo & kBucketMask, bhi = mhi & kBucketMask;
+  if (bhi != bref && bhi != bref + 1) return false;
   const uint32_t c = (((mlo >> kBucketBits) << cb) | ((uint32_t)rlo & ((1u << cb) - 1u))) - (uint32_t)dmin;
   const uint32_t rec0 = chunk * (uint32_t)WREC;
+  const uint32_t ck = (bref << kSegChunkBits) | (chunk & ((1u << kSegChunkBits) - 1u));
+  const uint32_t chi = (chunk >> kSegChunkBits) << 31;
+  if (bhi == bref) {
 #pragma unroll
-  for (int k = 0; k < RPL; ++k)
-    out[k * 32 + lane] = make_uint2(opk[k] | (d[k] + c),
-                                    (rec0 + k * 32 + lane) | (MD ? ((devs >> (2 * k)) & 3u) << 30 : 0u));
-  if (lane == 0)
-    segbuf[nbuf] = make_uint2((bref << kSegChunkBits) | (chunk & ((1u << kSegChunkBits) - 1u)),
-                              (uint32_t)WREC << 16 | ((chunk >> kSegChunkBits) << 31));
-  ++nbuf;
+    for (int k = 0; k < RPL; ++k)
+      out[k * 32 + lane] = make_uint2(opk[k] | (d[k] + c),
+                                      (rec0 + k * 32 + lane) | (MD ? ((devs >> (2 * k)) & 3u) << 30 : 0u));
+    if (lane == 0) segbuf[nbuf] = make_uint2(ck, (uint32_t)WREC << 16 | chi);
+    ++nbuf;
+    return true;
+  }
+  // Two adjacent buckets (a run crossing a bucket boundary, or two runs on either
+  // side of it: the usual non-uniform chunk).  Bucket bhi starts at the first
+  // coarse bin of bhi, boundary = (bin(rhi) - bin offset of rhi in bhi) << cb
+  // (relative word); a record is in bhi iff d >= tb.  Stable two-way split: the
+  // bref events first, then the bhi events, each in record order; offsets in
+  // bhi are d + cB.
+  const uint64_t boundary = ((rhi >> cb) - (uint64_t)(mhi >> kBucketBits)) << cb;
+  const uint64_t r0w = w0 - p.base_word;
+  const int32_t tb = (int32_t)(uint32_t)(boundary - r0w);
+  const uint32_t cB = (uint32_t)(r0w - boundary);
+  uint32_t bm[RPL], nB = 0;
+#pragma unroll
+  for (int k = 0; k < RPL; ++k) {
+    bm[k] = __ballot_sync(FULL, (int32_t)d[k] >= tb);
+    nB += __popc(bm[k]);
+  }
+  const uint32_t nA = WREC - nB, lt = lanemask_lt();
+  uint32_t runA = 0, runB = nA;
+#pragma unroll
+  for (int k = 0; k < RPL; ++k) {
+    const bool isB = (bm[k] >> lane) & 1u;
+    const uint32_t o = isB ? runB + __popc(bm[k] & lt) : runA + __popc(~bm[k] & lt);
+    out[o] = make_uint2(opk[k] | (d[k] + (isB ? cB : c)),
+                        (rec0 + k * 32 + lane) | (MD ? ((devs >> (2 * k)) & 3u) << 30 : 0u));
+    runB += __popc(bm[k]);
+    runA += 32 - __popc(bm[k]);
+  }
+  if (lane == 0) {
+    segbuf[nbuf] = make_uint2(ck, nA << 16 | chi);
+    segbuf[nbuf + 1] = make_uint2(ck + (1u << kSegChunkBits), nA | (nB << 16) | chi);
+  }
+  nbuf += 2;
   return true;
 }
 
@@ -238,11 +274,11 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     const uint4* st = stage + cur * WREC;
     const uint64_t rec0 = chunk * WREC;
     const uint32_t nvalid = p.n - rec0 < (uint64_t)WREC ? (uint32_t)(p.n - rec0) : (uint32_t)WREC;
-    // ---- fast chunk: 256 single-word tracked accesses of one bucket ----------------------
-    // (the common case of real access streams: a run over one array).  The events
-    // keep record order, so event j is record j: one coalesced store per record and
-    // one segment entry for the chunk.  Anything else takes the general path below.
-    if (nbuf == kSegBuf) flush_segs();
+    // ---- fast chunk: 256 single-word tracked accesses of one bucket or two adjacent
+    // ones (the common case of real access streams: runs over one array).  One bucket:
+    // event j is record j, one coalesced store per record, one segment entry; two:
+    // a stable two-way split and two entries.  Anything else takes the general path.
+    if (nbuf + 2 > kSegBuf) flush_segs();
     if (nvalid == WREC && fast_chunk<MD>(st, p, (uint32_t)chunk, p.part_ev + chunk * kChunkCap,
                                      segbuf, nbuf, lane)) {
       n_acc += RPL;
