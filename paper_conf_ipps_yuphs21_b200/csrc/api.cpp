@@ -94,6 +94,31 @@ cudaError_t upload_pinned(DevBuf<T>& b, HostBuf<T>& h, const std::vector<T>& v, 
   return cudaMemcpyAsync(b.p, h.p, v.size() * sizeof(T), cudaMemcpyHostToDevice, s);
 }
 
+// Several host vectors in one pinned staging buffer and one H2D copy into one device
+// buffer (16-B aligned parts); `at` gives a part's device address.
+struct PackUpload {
+  struct Part { const void* src; size_t bytes, off; };
+  std::vector<Part> parts;
+  size_t total = 0;
+  template <class T>
+  size_t add(const std::vector<T>& v) {
+    const size_t o = total, b = v.size() * sizeof(T);
+    parts.push_back({v.data(), b, o});
+    total += (std::max<size_t>(b, 1) + 15) & ~(size_t)15;
+    return o;
+  }
+  cudaError_t run(DevBuf<uint8_t>& d, HostBuf<uint8_t>& h, cudaStream_t s) {
+    cudaError_t e = d.ensure(std::max<size_t>(total, 16));
+    if (e == cudaSuccess) e = h.ensure(std::max<size_t>(total, 16));
+    if (e != cudaSuccess) return e;
+    for (const Part& q : parts)
+      if (q.bytes) std::memcpy(h.p + q.off, q.src, q.bytes);
+    return total ? cudaMemcpyAsync(d.p, h.p, total, cudaMemcpyHostToDevice, s) : cudaSuccess;
+  }
+  template <class P>
+  static P at(const DevBuf<uint8_t>& d, size_t off) { return reinterpret_cast<P>(d.p + off); }
+};
+
 }  // namespace
 
 struct arb_ctx_s {
@@ -144,10 +169,9 @@ struct arb_ctx_s {
   DevBuf<BucketOp> ops;
   DevBuf<DevStats> dstats;
   DevBuf<unsigned long long> dcount;
-  // MIR
-  DevBuf<uint64_t> m_ins_lo, m_ins_cum, m_qry_lo, m_qry_cum, m_rr_cum;
-  DevBuf<uint32_t> m_ins_inst, m_qry_open_start, m_open_list, m_own_start, m_win_start;
-  DevBuf<RangeRef> m_own, m_win, m_rr;
+  // MIR: the join plan's arrays, packed (one pinned staging buffer, one copy)
+  DevBuf<uint8_t> m_pack;
+  HostBuf<uint8_t> h_m_pack;
   DevBuf<unsigned long long> hkeys;
   DevBuf<uint32_t> hvals;
   // N2: nowait instances unjoined at the end of the last flush (committed with the map table)
@@ -158,7 +182,7 @@ struct arb_ctx_s {
   uint64_t dset_slots = 0, dset_n = 0;
   DevBuf<uint4> carry_ent, carry_next;        // their access summaries {word lo, word hi, carried idx, flag}
   uint64_t n_carry = 0;
-  DevBuf<uint32_t> m_cmap, m_co_of;
+  DevBuf<uint32_t> m_co_of;
   uint64_t ctl_cap = 1 << 16;
   uint64_t cand_cap = 1 << 24;
   MapTable map;
@@ -305,11 +329,8 @@ extern "C" int arb_destroy(arb_ctx ctx) {
   ctx->d_cv_epoch_first.release(); ctx->d_cv_place.release();
   ctx->ctl.release(); ctx->cand.release(); ctx->cand_tmp.release(); ctx->reports.release(); ctx->blk.release();
   ctx->ops_start.release(); ctx->ops.release(); ctx->dstats.release(); ctx->dcount.release();
-  ctx->m_ins_lo.release(); ctx->m_ins_cum.release(); ctx->m_qry_lo.release(); ctx->m_qry_cum.release();
-  ctx->m_rr_cum.release(); ctx->m_ins_inst.release(); ctx->m_qry_open_start.release(); ctx->m_open_list.release();
-  ctx->m_own_start.release(); ctx->m_win_start.release(); ctx->m_own.release(); ctx->m_win.release();
-  ctx->m_rr.release(); ctx->hkeys.release(); ctx->hvals.release(); ctx->counts.release();
-  ctx->carry_ent.release(); ctx->carry_next.release(); ctx->dset.release(); ctx->dset_cnt.release(); ctx->m_cmap.release(); ctx->m_co_of.release();
+  ctx->m_pack.release(); ctx->h_m_pack.release(); ctx->hkeys.release(); ctx->hvals.release(); ctx->counts.release();
+  ctx->carry_ent.release(); ctx->carry_next.release(); ctx->dset.release(); ctx->dset_cnt.release(); ctx->m_co_of.release();
   ctx->d_bin_map.release(); ctx->d_items.release(); ctx->h_items.release();
   ctx->d_slice_items.release(); ctx->h_slice_items.release(); ctx->d_hot.release(); ctx->h_hot.release();
   ctx->d_hot_off.release(); ctx->h_hot_off.release(); ctx->hot_F.release(); ctx->hot_P.release(); ctx->d_hist.release(); ctx->d_bucket_start.release(); ctx->d_cut.release();
@@ -774,31 +795,41 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
     MirPlanH& M = plan.mir;
     uint64_t hcap = 1;
     while (hcap < 2 * (2 * M.n_ins_pos + (carry_in ? ctx->n_carry : 0) + 1)) hcap <<= 1;
-    if (carry_in) CK(upload(ctx->m_cmap, plan.carry_in_dense, s), "mir carry map");
     CK(ctx->hkeys.ensure(hcap), "alloc hash");
     CK(ctx->hvals.ensure(hcap), "alloc hash");
-    CK(upload(ctx->m_ins_lo, M.ins_lo, s), "mir"); CK(upload(ctx->m_ins_cum, M.ins_cum, s), "mir");
-    CK(upload(ctx->m_ins_inst, M.ins_inst, s), "mir"); CK(upload(ctx->m_qry_lo, M.qry_lo, s), "mir");
-    CK(upload(ctx->m_qry_cum, M.qry_cum, s), "mir"); CK(upload(ctx->m_qry_open_start, M.qry_open_start, s), "mir");
-    CK(upload(ctx->m_open_list, M.open_list, s), "mir"); CK(upload(ctx->m_own_start, M.own_start, s), "mir");
-    CK(upload(ctx->m_win_start, M.win_start, s), "mir"); CK(upload(ctx->m_own, M.own_ops, s), "mir");
-    CK(upload(ctx->m_win, M.win_ops, s), "mir"); CK(upload(ctx->m_rr, M.rr, s), "mir");
-    CK(upload(ctx->m_rr_cum, M.rr_cum, s), "mir");
+    PackUpload pk;
+    const size_t o_cmap = pk.add(plan.carry_in_dense);
+    const size_t o_ins_lo = pk.add(M.ins_lo), o_ins_cum = pk.add(M.ins_cum), o_ins_inst = pk.add(M.ins_inst);
+    const size_t o_qry_lo = pk.add(M.qry_lo), o_qry_cum = pk.add(M.qry_cum), o_qos = pk.add(M.qry_open_start);
+    const size_t o_open = pk.add(M.open_list), o_own_start = pk.add(M.own_start), o_win_start = pk.add(M.win_start);
+    const size_t o_own = pk.add(M.own_ops), o_win = pk.add(M.win_ops), o_rr = pk.add(M.rr), o_rr_cum = pk.add(M.rr_cum);
+    CK(pk.run(ctx->m_pack, ctx->h_m_pack, s), "upload mir plan");
+    const DevBuf<uint8_t>& D = ctx->m_pack;
     for (int attempt = 0; attempt < 2; ++attempt) {
       CK(cudaMemsetAsync(ctx->hkeys.p, 0, hcap * sizeof(unsigned long long), s), "hash clear");
       CK(cudaMemsetAsync(ctx->hvals.p, 0, hcap * sizeof(uint32_t), s), "hash clear");
       CK(cudaMemsetAsync(&ctx->dstats.p->n_mir_cand, 0, sizeof(unsigned long long), s), "mir count");
       MirParams mp{};
       mp.ev = ev; mp.base_word = ctx->base_word; mp.n_words = ctx->n_words;
-      mp.ins_lo = ctx->m_ins_lo.p; mp.ins_cum = ctx->m_ins_cum.p; mp.ins_inst = ctx->m_ins_inst.p;
+      mp.ins_lo = PackUpload::at<decltype(mp.ins_lo)>(D, o_ins_lo);
+      mp.ins_cum = PackUpload::at<decltype(mp.ins_cum)>(D, o_ins_cum);
+      mp.ins_inst = PackUpload::at<decltype(mp.ins_inst)>(D, o_ins_inst);
       mp.n_ins = (uint32_t)M.ins_lo.size();
-      mp.qry_lo = ctx->m_qry_lo.p; mp.qry_cum = ctx->m_qry_cum.p; mp.qry_open_start = ctx->m_qry_open_start.p;
-      mp.n_qry = (uint32_t)M.qry_lo.size(); mp.open_list = ctx->m_open_list.p;
-      mp.own_start = ctx->m_own_start.p; mp.own_ops = ctx->m_own.p;
-      mp.win_start = ctx->m_win_start.p; mp.win_ops = ctx->m_win.p;
+      mp.qry_lo = PackUpload::at<decltype(mp.qry_lo)>(D, o_qry_lo);
+      mp.qry_cum = PackUpload::at<decltype(mp.qry_cum)>(D, o_qry_cum);
+      mp.qry_open_start = PackUpload::at<decltype(mp.qry_open_start)>(D, o_qos);
+      mp.n_qry = (uint32_t)M.qry_lo.size();
+      mp.open_list = PackUpload::at<decltype(mp.open_list)>(D, o_open);
+      mp.own_start = PackUpload::at<decltype(mp.own_start)>(D, o_own_start);
+      mp.own_ops = PackUpload::at<decltype(mp.own_ops)>(D, o_own);
+      mp.win_start = PackUpload::at<decltype(mp.win_start)>(D, o_win_start);
+      mp.win_ops = PackUpload::at<decltype(mp.win_ops)>(D, o_win);
       mp.hkeys = ctx->hkeys.p; mp.hvals = ctx->hvals.p; mp.hmask = hcap - 1;
-      mp.rr = ctx->m_rr.p; mp.rr_cum = ctx->m_rr_cum.p; mp.n_rr = (uint32_t)M.rr.size();
-      mp.carry = ctx->carry_ent.p; mp.n_carry = carry_in ? ctx->n_carry : 0; mp.cmap = ctx->m_cmap.p;
+      mp.rr = PackUpload::at<decltype(mp.rr)>(D, o_rr);
+      mp.rr_cum = PackUpload::at<decltype(mp.rr_cum)>(D, o_rr_cum);
+      mp.n_rr = (uint32_t)M.rr.size();
+      mp.carry = ctx->carry_ent.p; mp.n_carry = carry_in ? ctx->n_carry : 0;
+      mp.cmap = carry_in ? PackUpload::at<decltype(mp.cmap)>(D, o_cmap) : nullptr;
       mp.cand = ctx->cand.p + kept_vsm; mp.cand_cap = ctx->cand.cap - kept_vsm; mp.st = ctx->dstats.p;
       CK(launch_mir(mp, M.n_ins_pos, M.n_qry_pos, M.n_rr_words, s, &launches), "k_mir");
       unsigned long long c = 0;

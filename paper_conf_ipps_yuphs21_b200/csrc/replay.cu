@@ -38,16 +38,18 @@ constexpr int kHBits = kReplayHashBits;
 constexpr int kHSlots = 1 << kHBits;         // hash slots (load <= 1/2)
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
 constexpr uint32_t kWordMask = 0x3FFFFFFFu;
-constexpr int kZBits = kHBits - 1;
-constexpr int kZSlots = 1 << kZBits;         // summary-step hash slots (>= 2 x the writes of a step)
-static_assert(kZSlots * 12 <= kHSlots * 8 && kZSlots >= 2 * STEP, "summary hash fits the hash area");
+constexpr int ilog2c(int x) { return x <= 1 ? 0 : 1 + ilog2c(x >> 1); }
+constexpr int kZBits = ilog2c(2 * STEP);
+constexpr int kZSlots = 1 << kZBits;         // summary-step hash slots (2 x the events of a step)
+static_assert(kZSlots == 2 * STEP, "summary hash: twice the step");
 
 struct ReplaySmem {
   uint2 ev[2][STEP];              // double-buffered step events {key, pos} (cp.async)
   union {
     struct { uint32_t keyA[STEP], posA[STEP], keyB[STEP], posB[STEP]; uint16_t hist[RT / 32][256]; } s;
     struct { uint2 slot[kHSlots]; } h;      // fast step: written words {word, pos << 2 | op}
-    struct { uint32_t key[kZSlots], lastw[kZSlots], anyw[kZSlots]; } z;  // hot-slice summary step (K5)
+    struct { uint32_t key[kZSlots], lastw[kZSlots], anyw[kZSlots / 4]; } z;  // hot-slice summary step (K5);
+                                                                            // anyw: one byte per slot
   } u;
   uint32_t wstart[kWin];          // staged segment list window: global event index
   uint32_t wcum[kWin + 1];        //   and bucket-relative first event of each segment
@@ -649,7 +651,7 @@ __device__ void step_summary(ReplaySmem& S, const uint2* ev, uint32_t m) {
         }
         slot[j] = h;
         atomicMax(&lastw[h], (idx[j] << 4) | (dev << 2) | op[j]);
-        atomicOr(&anyw[h], op[j] == OP_WH ? 1u : (2u << dev));   // bit 0 WH, bit 1 + d WT on device d
+        atomicOr(&anyw[h >> 2], (op[j] == OP_WH ? 1u : (2u << dev)) << (8 * (h & 3)));   // bit 0 WH, bit 1 + d WT on d
       }
     }
   }
@@ -658,7 +660,7 @@ __device__ void step_summary(ReplaySmem& S, const uint2* ev, uint32_t m) {
   for (int j = 0; j < RI; ++j) {
     const uint32_t l = (op[j] & 1u) ? lastw[slot[j]] : 0u;
     last[j] = (op[j] & 1u) && (l >> 4) == idx[j];
-    ab[j] = last[j] ? anyw[slot[j]] : 0u;
+    ab[j] = last[j] ? (anyw[slot[j] >> 2] >> (8 * (slot[j] & 3))) & 0xFFu : 0u;
     lw[j] = l & 15u;
   }
   __syncthreads();
@@ -694,7 +696,7 @@ __device__ void step_summary(ReplaySmem& S, const uint2* ev, uint32_t m) {
       S.fsum[word[j]] = nf;
       key[slot[j]] = kEmpty;           // the word's only slot: reset by its last writer
       lastw[slot[j]] = 0;
-      anyw[slot[j]] = 0;
+      atomicAnd(&anyw[slot[j] >> 2], ~(0xFFu << (8 * (slot[j] & 3))));
     }
   }
   __syncthreads();
@@ -934,7 +936,8 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       __syncthreads();
       if (mode == kItemSummary) {
         for (uint32_t w = tid; w < span; w += RT) S.fsum[w] = kfun_id<BO, MD>();
-        for (uint32_t w = tid; w < kZSlots; w += RT) { S.u.z.key[w] = kEmpty; S.u.z.lastw[w] = 0; S.u.z.anyw[w] = 0; }
+        for (uint32_t w = tid; w < kZSlots; w += RT) { S.u.z.key[w] = kEmpty; S.u.z.lastw[w] = 0; }
+        for (uint32_t w = tid; w < kZSlots / 4; w += RT) S.u.z.anyw[w] = 0;
         __syncthreads();
       }
     }
