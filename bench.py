@@ -218,7 +218,7 @@ class BatchSource:
 
 STAT_KEYS = ("access_words", "range_words", "reports", "records", "ms_partition", "ms_replay", "ms_mir",
              "ms_reports", "ms_control", "ms_total", "ms_sample", "ms_segsort", "ms_host_control", "steps_fast",
-             "steps_sort", "work_items", "hot_buckets", "kernel_launches", "exchanges")
+             "steps_sort", "steps_run", "segments", "work_items", "hot_buckets", "kernel_launches", "exchanges")
 
 
 def run_workload(prog, ctx, src, batches, steps, warmup, stream, world, dev, on_batch=None, clocks=None):
@@ -580,7 +580,9 @@ def main():
                            "reports_per_step": int(reports_all), "reports_by_kind_rank0": s0["by_kind"][1:],
                            "time_batches": len(batches), "flushes_per_step_rank0": int(s0["flushes"]),
                            "rank_words": hi - lo, "batches_rank0": binfo,
-                           "replay_steps_fast_sort_rank0": [int(s0["steps_fast"]), int(s0["steps_sort"])],
+                           "replay_steps_fast_sort_run_rank0": [int(s0["steps_fast"]), int(s0["steps_sort"]),
+                                                                int(s0["steps_run"])],
+                           "segments_rank0": int(s0["segments"]),
                            "max_bucket_events_rank0": int(s0["max_bucket_events"]),
                            "replay_work_items_rank0": int(s0["work_items"]),
                            "hot_buckets_rank0": int(s0["hot_buckets"]),

@@ -15,7 +15,8 @@ from .trace import MAP, OP, UPD, SYNC_ALL, TraceBuilder, encode_np
 
 def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: int = 60,
                    base: int = 0x10000, loop_max: int = 48, p_task: float = 0.15, p_always: float = 0.0,
-                   p_depend: float = 0.0, n_devices: int = 1, p_tag: float = 0.0):
+                   p_depend: float = 0.0, n_devices: int = 1, p_tag: float = 0.0,
+                   strides=(1, 4, 8, 8, 8, 12), sizes=(1, 2, 4, 8, 8, 8)):
     """p_always > 0: map clauses carry the `always` modifier with that probability;
     p_depend > 0: a new nowait block depends on an earlier task with that
     probability; n_devices > 1: target accesses and map / update clauses on a
@@ -23,7 +24,9 @@ def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: i
     map / update arg); p_tag > 0: pointer tags (ARB_BASE records, reading Z25): tag
     i + 1 has array i's base, target accesses carry a tag with that probability
     (mostly their own array's, sometimes another's), and tags are sometimes
-    redefined (the RNG streams of the defaults are unchanged)."""
+    redefined (the RNG streams of the defaults are unchanged).  strides / sizes: the
+    loop access strides and sizes are drawn from them (8 / 8: runs over consecutive
+    words)."""
     rs = np.random.default_rng(seed)
     tb = TraceBuilder()
     arrays = [base + i * array_words * 8 * 2 for i in range(n_arrays)]   # gap between arrays
@@ -57,8 +60,8 @@ def random_program(seed: int, n_arrays: int = 4, array_words: int = 64, steps: i
         i = int(rs.integers(n_arrays))
         cnt = int(rs.integers(1, loop_max))
         start = int(rs.integers(0, array_words * 8 - 8))
-        stride = int(rs.choice([1, 4, 8, 8, 8, 12]))
-        size = int(rs.choice([1, 2, 4, 8, 8, 8]))
+        stride = int(rs.choice(list(strides)))
+        size = int(rs.choice(list(sizes)))
         addr = arrays[i] + start + stride * np.arange(cnt, dtype=np.uint64)
         addr = addr[addr + size <= arrays[i] + array_words * 8 + 8]
         if addr.size:
@@ -172,3 +175,11 @@ def to_cv_addressing(rec, cv_off=1 << 44, frac=1.0, seed=0):
                 if e[2] == 0:
                     entries.remove(e)
     return np.array(out, dtype=np.uint64).reshape(-1, 2)
+
+
+def run_program(seed: int, n_arrays: int = 6, array_words: int = 4096, steps: int = 400, loop_max: int = 1500):
+    """Programs whose loops are mostly runs (stride 8, size 8: consecutive records
+    on consecutive words with one op), so that most chunks take the partition's run
+    form, with some stride-4 / stride-16 loops mixed in."""
+    return random_program(seed, n_arrays=n_arrays, array_words=array_words, steps=steps, loop_max=loop_max,
+                          strides=(8, 8, 8, 8, 8, 8, 8, 4, 16), sizes=(8, 8, 8, 8, 8, 8, 8, 4, 8))

@@ -182,6 +182,9 @@ typedef struct {
   uint64_t nccl_ranks;       /* ranks of the context's NCCL communicator (ncclCommCount), 0 =
                                 no communicator                                              */
   uint64_t exchanges;        /* collectives (status / count ncclAllGather) of the last flush */
+  uint64_t steps_run;        /* replay steps made only of run segments       */
+  uint64_t segments;         /* (chunk, bucket) segment entries of the last flush (runs and
+                                stored-event segments)                                        */
 } arb_stats;
 
 typedef struct arb_ctx_s* arb_ctx;

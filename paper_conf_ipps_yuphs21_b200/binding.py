@@ -57,7 +57,8 @@ class arb_stats(ctypes.Structure):
                 ("ms_segsort", ctypes.c_double), ("ms_host_control", ctypes.c_double),
                 ("work_items", ctypes.c_uint64), ("hot_buckets", ctypes.c_uint64),
                 ("reports_bo", ctypes.c_uint64), ("nccl_ranks", ctypes.c_uint64),
-                ("exchanges", ctypes.c_uint64)]
+                ("exchanges", ctypes.c_uint64), ("steps_run", ctypes.c_uint64),
+                ("segments", ctypes.c_uint64)]
 
     def as_dict(self):
         d = {}

@@ -525,6 +525,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   S.reports = 0; std::memset(S.reports_by_kind, 0, sizeof(S.reports_by_kind)); S.ignored_words = 0;
   S.ms_partition = S.ms_control = S.ms_replay = S.ms_mir = S.ms_reports = S.ms_total = 0;
   S.ms_segsort = S.ms_host_control = 0;
+  S.steps_run = S.segments = 0;
   S.buckets = ctx->n_buckets; S.bucket_bits = ctx->bucket_bits; S.max_bucket_events = 0;
 
   // Phase A (validation): decode + partition and control resolution.  Nothing
@@ -621,6 +622,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
       pp.n_chunks = n_chunks;
       pp.n_dev = 1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u);
       pp.part_ev = ctx->part_ev.p; pp.seg_out = ctx->seg_a.p; pp.seg_cap = ctx->seg_cap;
+      pp.no_runs = getenv("ARB_NO_RUNS") != nullptr;
       pp.ctl = ctx->ctl.p; pp.ctl_cap = ctx->ctl_cap;
       pp.st = ctx->dstats.p;
       CK(launch_partition(pp, s), "k_partition");
@@ -761,6 +763,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   rp.um = (ctx->cfg.flags & ARB_F_UNIFIED) ? 1u : 0u;
   rp.md = ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u) ? 1u : 0u; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
   rp.cand = ctx->cand.p; rp.cand_cap = ctx->cand_cap; rp.st = ctx->dstats.p;
+  rp.no_run_steps = getenv("ARB_NO_RUN_STEPS") != nullptr;
   rp.hot_off = ctx->d_hot_off.p; rp.hot_F = ctx->hot_F.p; rp.hot_P = ctx->hot_P.p;
   int n_ctas = std::max(1, std::min<int>((int)ctx->items.size(), ctx->n_sms * kReplayCtasPerSm));
   CK(launch_replay(rp, std::max(n_ctas, 1), s), "k_replay");
@@ -787,6 +790,8 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   S.max_bucket_events = hst.max_bucket_events;
   S.steps_fast = hst.steps_fast;
   S.steps_sort = hst.steps_sort;
+  S.steps_run = hst.steps_run;
+  S.segments = hst.n_segs;
 
   // ---- A6: MIR join ---------------------------------------------------------------
   uint64_t n_mir = 0;

@@ -64,6 +64,12 @@ __host__ __device__ constexpr uint32_t sel8_clear(uint32_t d) { return sel8_set(
 constexpr int kMaxBucketSpanBits = 30;               // buckets span <= 2^30 words
 constexpr uint32_t kMaxBatchRecords = 1u << 30;
 constexpr int kSegChunkBits = 21;                    // chunk id bits in the entry key (bit 21 in y)
+// Run segments: a segment entry whose start has kRunFlag holds a run —
+// event j of the segment is {key + j, position + j}, where {key, position} is the
+// run's descriptor stored at the start slot of the chunk's output (no other events
+// are written).  A fast chunk of at most kMaxChunkRuns runs is written in this form.
+constexpr uint32_t kRunFlag = 0x8000u;
+constexpr int kMaxChunkRuns = 16;
 
 // ---- partition geometry ----------------------------------------------------
 constexpr int kPartThreads = 512;
@@ -106,7 +112,7 @@ struct DevStats {
   unsigned long long n_carry_out;     // N2: access summaries of instances carried into the next flush
   unsigned long long n_bo_cand;       // N1 (Z25): base-tag overflow candidates
   unsigned long long n_cv_acc;        // N1 (Z26): target accesses by CV address (left untracked)
-  unsigned long long pad[1];
+  unsigned long long steps_run;      // replay steps made only of run segments
 };
 
 // control record extracted by the partition kernel
@@ -154,6 +160,7 @@ struct PartParams {
   CtlRec* ctl; uint64_t ctl_cap;
   DevStats* st;
   uint32_t n_dev;                         // accelerators (Z24): > 1 puts the device of RT/WT in pos bits 30-31
+  uint32_t no_runs;                       // debug (ARB_NO_RUNS): never write the run form
 };
 
 struct ReplayParams {
@@ -174,6 +181,7 @@ struct ReplayParams {
   uint32_t bo;                            // ARB_F_BO: target accesses to words without kCVp are BO
   uint32_t um;                            // ARB_F_UNIFIED: OV and CV are one storage (Z23)
   uint32_t md;                            // several accelerators (Z24): 8-bit states, device in pos bits 30-31
+  uint32_t no_run_steps;                  // debug (ARB_NO_RUN_STEPS): run segments only as synthesised events
   const uint32_t* ops_start;              // [n_buckets + 1]
   const BucketOp* ops;
   uint4* cand; uint64_t cand_cap;         // report candidates {word lo, word hi, pos, kind}

@@ -132,8 +132,9 @@ __device__ __forceinline__ void rank_round(uint32_t info, uint16_t* row, uint16_
 
 // The fast chunk test and its output.  Every record must be an access (op < 4)
 // of 1..8 bytes inside one 8-byte word (such an access cannot leave the
-// 48-bit space), and all words must lie in one address bucket or in two
-// adjacent ones (a stable two-way split by the bucket boundary).  Buckets are
+// 48-bit space).  A chunk of few runs (below) is written in run form; otherwise
+// all words must lie in one address bucket or in two adjacent ones (a stable
+// two-way split by the bucket boundary).  Buckets are
 // contiguous word ranges, so the test needs only the chunk's lowest and highest
 // word: each word is taken relative to record 0's word w0 (32-bit signed,
 // |d| < 2^30 as a bucket spans <= 2^30 words), the warp reduces min and max, and
@@ -141,7 +142,7 @@ __device__ __forceinline__ void rank_round(uint32_t info, uint16_t* row, uint16_
 // off(lowest) + d - dmin.  Returns false (nothing written) when the test fails.
 template <bool MD>
 __device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p, uint32_t chunk, uint2* out,
-                                           uint2* segbuf, uint32_t& nbuf, uint32_t lane) {
+                                           uint2* segbuf, uint32_t& nbuf, uint32_t lane, uint16_t* scratch) {
   const uint4 q0 = st[0];
   const uint64_t w0 = ((uint64_t)((q0.y & 0xFFFFu) >> 3) << 32) | __funnelshift_r(q0.x, q0.y, 3);
   uint32_t d[RPL], opk[RPL], bad = 0, devs = 0;
@@ -170,13 +171,97 @@ __device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p,
   const uint64_t rhi = w0 - p.base_word + (uint64_t)(int64_t)dmax;
   if (rlo >= p.n_words || rhi >= p.n_words) return false;
   const uint32_t cb = p.coarse_bits;
+  const uint32_t rec0 = chunk * (uint32_t)WREC;
+  const uint32_t chi = (chunk >> kSegChunkBits) << 31;
+  if (!MD && !p.no_runs && (uint32_t)(dmax - dmin) < (1u << 28)) {
+    // ---- run form: a run = consecutive records with the same op on
+    // consecutive words (event j of the run: word + j, position + j).  Record i's
+    // key (d_i - i) << 3 | op << 1 is constant along a run (exact: |d| spans < 2^28);
+    // a run starts where the key changes.  A chunk of <= kMaxChunkRuns runs, each
+    // inside one bucket (any buckets) or split at the boundary of two adjacent ones,
+    // writes one 8-B descriptor (the piece's first event, at the slot of its first
+    // record) and one segment entry (start flagged kRunFlag) per piece instead of 8 B
+    // per record.
+    uint32_t sm[RPL], nR = 0, rprev = 0;
+#pragma unroll
+    for (int k = 0; k < RPL; ++k) {
+      const uint32_t key = ((d[k] - (uint32_t)(k * 32) - lane) << 3) | (opk[k] >> 29);
+      const uint32_t r = __shfl_sync(FULL, key, (lane + 31) & 31);    // lane L: key of lane L - 1
+      const uint32_t prev = lane ? r : rprev;                          // lane 0: lane 31 of round k - 1
+      rprev = __shfl_sync(FULL, r, 0);
+      sm[k] = __ballot_sync(FULL, (k == 0 && lane == 0) || key != prev);
+      nR += __popc(sm[k]);
+    }
+    if (nR <= (uint32_t)kMaxChunkRuns) {
+      uint32_t* kb = reinterpret_cast<uint32_t*>(scratch);             // [0, 16): record index, [16, 32): key
+      const uint32_t lt = lanemask_lt();
+      uint32_t before = 0;
+#pragma unroll
+      for (int k = 0; k < RPL; ++k) {
+        if (sm[k]) {
+          if ((sm[k] >> lane) & 1u) {
+            const uint32_t rk = before + __popc(sm[k] & lt);
+            kb[rk] = k * 32 + lane;
+            kb[kMaxChunkRuns + rk] = ((d[k] - (uint32_t)(k * 32) - lane) << 2) | (opk[k] >> 30);
+          }
+          before += __popc(sm[k]);
+        }
+      }
+      __syncwarp();
+      // lane r: run r, inside one bucket or split at the boundary of two adjacent ones
+      bool ok = true, split = false;
+      uint32_t i = 0, len = 0, len1 = 0, bkt = 0, off = 0, opr = 0;
+      if (lane < nR) {
+        i = kb[lane];
+        len = (lane + 1 < nR ? kb[lane + 1] : (uint32_t)WREC) - i;
+        const uint32_t kv = kb[kMaxChunkRuns + lane];
+        opr = kv & 3u;
+        const uint64_t first = w0 - p.base_word + (uint64_t)(int64_t)((int32_t)kv >> 2) + i;   // d_i = v + i
+        const uint64_t last = first + len - 1;
+        const uint32_t m1 = __ldg(p.bin_map + (uint32_t)(first >> cb)), m2 = __ldg(p.bin_map + (uint32_t)(last >> cb));
+        bkt = m1 & kBucketMask;
+        const uint32_t b2 = m2 & kBucketMask;
+        split = b2 == bkt + 1;
+        ok = b2 == bkt || split;
+        len1 = len;
+        if (split) len1 = (uint32_t)((((last >> cb) - (uint64_t)(m2 >> kBucketBits)) << cb) - first);
+        off = ((m1 >> kBucketBits) << cb) | ((uint32_t)first & ((1u << cb) - 1u));
+      }
+      __syncwarp();
+      if (__all_sync(FULL, ok)) {
+        const uint32_t sp = __ballot_sync(FULL, split);
+        if (lane < nR) {
+          const uint32_t ck = chunk & ((1u << kSegChunkBits) - 1u);
+          const uint32_t e = nbuf + lane + __popc(sp & lanemask_lt());
+          out[i] = make_uint2((opr << 30) | off, rec0 + i);
+          segbuf[e] = make_uint2((bkt << kSegChunkBits) | ck, i | kRunFlag | (len1 << 16) | chi);
+          if (split) {                     // the rest starts at the first word of bucket bkt + 1
+            out[i + len1] = make_uint2(opr << 30, rec0 + i + len1);
+            segbuf[e + 1] = make_uint2(((bkt + 1) << kSegChunkBits) | ck, (i + len1) | kRunFlag | ((len - len1) << 16) | chi);
+          }
+        }
+        nbuf += nR + __popc(sp);
+        return true;
+      }
+    }
+  }
   const uint32_t mlo = __ldg(p.bin_map + (uint32_t)(rlo >> cb)), mhi = __ldg(p.bin_map + (uint32_t)(rhi >> cb));
   const uint32_t bref = mlo & kBucketMask, bhi = mhi & kBucketMask;
   if (bhi != bref && bhi != bref + 1) return false;
   const uint32_t c = (((mlo >> kBucketBits) << cb) | ((uint32_t)rlo & ((1u << cb) - 1u))) - (uint32_t)dmin;
-  const uint32_t rec0 = chunk * (uint32_t)WREC;
   const uint32_t ck = (bref << kSegChunkBits) | (chunk & ((1u << kSegChunkBits) - 1u));
-  const uint32_t chi = (chunk >> kSegChunkBits) << 31;
+  // Two adjacent buckets (a run crossing a bucket boundary, or two runs on either
+  // side of it).  Bucket bhi starts at the first coarse bin of bhi, boundary =
+  // (bin(rhi) - bin offset of rhi in bhi) << cb (relative word); a record is in bhi
+  // iff d >= tb; its offset in bhi is d + cB.
+  int32_t tb = 0x7FFFFFFF;
+  uint32_t cB = 0;
+  if (bhi != bref) {
+    const uint64_t boundary = ((rhi >> cb) - (uint64_t)(mhi >> kBucketBits)) << cb;
+    const uint64_t r0w = w0 - p.base_word;
+    tb = (int32_t)(uint32_t)(boundary - r0w);
+    cB = (uint32_t)(r0w - boundary);
+  }
   if (bhi == bref) {
 #pragma unroll
     for (int k = 0; k < RPL; ++k)
@@ -186,16 +271,8 @@ __device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p,
     ++nbuf;
     return true;
   }
-  // Two adjacent buckets (a run crossing a bucket boundary, or two runs on either
-  // side of it: the usual non-uniform chunk).  Bucket bhi starts at the first
-  // coarse bin of bhi, boundary = (bin(rhi) - bin offset of rhi in bhi) << cb
-  // (relative word); a record is in bhi iff d >= tb.  Stable two-way split: the
-  // bref events first, then the bhi events, each in record order; offsets in
-  // bhi are d + cB.
-  const uint64_t boundary = ((rhi >> cb) - (uint64_t)(mhi >> kBucketBits)) << cb;
-  const uint64_t r0w = w0 - p.base_word;
-  const int32_t tb = (int32_t)(uint32_t)(boundary - r0w);
-  const uint32_t cB = (uint32_t)(r0w - boundary);
+  // Two adjacent buckets: stable two-way split, the bref events first, then the
+  // bhi events, each in record order.
   uint32_t bm[RPL], nB = 0;
 #pragma unroll
   for (int k = 0; k < RPL; ++k) {
@@ -278,9 +355,9 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     // ones (the common case of real access streams: runs over one array).  One bucket:
     // event j is record j, one coalesced store per record, one segment entry; two:
     // a stable two-way split and two entries.  Anything else takes the general path.
-    if (nbuf + 2 > kSegBuf) flush_segs();
+    if (nbuf + 2 * kMaxChunkRuns > kSegBuf) flush_segs();
     if (nvalid == WREC && fast_chunk<MD>(st, p, (uint32_t)chunk, p.part_ev + chunk * kChunkCap,
-                                     segbuf, nbuf, lane)) {
+                                     segbuf, nbuf, lane, tlist)) {
       n_acc += RPL;
       cur = cur + 1 == NST ? 0 : cur + 1;
       __syncwarp();                    // stage[cur] reads done before the next fetch overwrites it

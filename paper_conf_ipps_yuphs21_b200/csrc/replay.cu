@@ -43,8 +43,23 @@ constexpr int kZBits = ilog2c(2 * STEP);
 constexpr int kZSlots = 1 << kZBits;         // summary-step hash slots (2 x the events of a step)
 static_assert(kZSlots == 2 * STEP, "summary hash: twice the step");
 
+// Run steps: a step made only of run segments never materialises
+// its events; the gather stages the runs' descriptors in the step's event buffer.
+constexpr int kMaxStepRuns = 32;             // run segments per run step
+constexpr uint32_t kRunStepMax = 8192;       // events per run step
+struct RunStage {
+  uint4 info[kMaxStepRuns];                  // {first event's offset in the run, events, step-relative start, 0}
+  uint2 desc[kMaxStepRuns];                  // the runs' descriptors {key, position} (cp.async)
+  uint4 run[kMaxStepRuns];                   // {A, B, op, position of word A} (A, B: words from the
+                                             //   4-aligned word below the bucket's first word)
+  uint2 mi[kMaxStepRuns];                    // merged 4-word-group intervals {first group, first unit}
+  uint32_t mm[kMaxStepRuns];                 // the runs overlapping merged interval j
+  uint32_t nm, G;                            // merged intervals, groups
+};
+static_assert(sizeof(RunStage) <= sizeof(uint2) * STEP, "a run stage fits in one step buffer");
+
 struct ReplaySmem {
-  uint2 ev[2][STEP];              // double-buffered step events {key, pos} (cp.async)
+  uint2 ev[2][STEP];              // double-buffered step events {key, pos} (cp.async), or a RunStage
   union {
     struct { uint32_t keyA[STEP], posA[STEP], keyB[STEP], posB[STEP]; uint16_t hist[RT / 32][256]; } s;
     struct { uint2 slot[kHSlots]; } h;      // fast step: written words {word, pos << 2 | op}
@@ -64,6 +79,8 @@ struct ReplaySmem {
   uint32_t* fsum;                 // summary slice: composed transition of word w: fsum[w] (kfun_*)
   uint32_t slice, n_slices;       // hot bucket slice (kItemSlice / kItemSummary)
   uint32_t seg0, cum0, n_segs, n_events, wsc, nwin;
+  uint32_t runk[2];               // run segments staged in buffer b (0: an event step)
+  uint32_t span;                  // words of the bucket
   uint64_t bucket_base;
 };
 
@@ -710,7 +727,9 @@ __device__ uint32_t event_pos(const ReplaySmem& S, const ReplayParams& p, uint32
     if (p.segs[S.seg0 + mid].w - S.cum0 <= e) lo = mid; else z = mid;
   }
   const uint4 sg = p.segs[S.seg0 + lo];
-  const uint32_t pos = p.part_ev[(uint64_t)sg.x * kChunkCap + (sg.z & 0xFFFFu) + (e - (sg.w - S.cum0))].y;
+  const uint32_t st = sg.z & 0xFFFFu, off = e - (sg.w - S.cum0);
+  const uint32_t pos = (st & kRunFlag) ? p.part_ev[(uint64_t)sg.x * kChunkCap + (st & ~kRunFlag)].y + off
+                                       : p.part_ev[(uint64_t)sg.x * kChunkCap + st + off].y;
   return p.md ? (pos & kMdPos) : pos;
 }
 // first op of the bucket (ops [a, z), trace order) at or after position q
@@ -795,21 +814,78 @@ __device__ void ensure_window(ReplaySmem& S, const ReplayParams& p, uint32_t e0,
   const uint4* segs = p.segs + S.seg0 + sc;
   for (uint32_t k = threadIdx.x; k < nwin; k += RT) {
     const uint4 e = segs[k];
-    S.wstart[k] = e.x * (uint32_t)kChunkCap + (e.z & 0xFFFFu);
+    const uint32_t st = e.z & 0xFFFFu;         // bit 31 of wstart: a run segment
+    S.wstart[k] = (e.x * (uint32_t)kChunkCap + (st & ~kRunFlag)) | ((st & kRunFlag) << 16);
     S.wcum[k] = e.w - S.cum0;
   }
   if (threadIdx.x == 0) S.wcum[nwin] = sc + nwin < S.n_segs ? segs[nwin].w - S.cum0 : S.n_events;
   __syncthreads();
 }
 
-// Issue cp.async copies of events [e0, e0 + m) of the bucket into dst; the
-// window must contain e0.  Returns m (<= STEP, clipped to the window).
+// Event j of window segment `seg` into shared memory: a cp.async of the stored
+// event, or (a run segment, bit 31 of wstart) the run's descriptor + j.
+__device__ __forceinline__ void gather_ev(uint2* d, const ReplayParams& p, uint32_t ws, uint32_t j) {
+  if (ws >> 31) {
+    const uint2 r = p.part_ev[ws & 0x7FFFFFFFu];
+    *d = make_uint2(r.x + j, r.y + j);
+  } else {
+    cp_async8(d, p.part_ev + (ws + j));
+  }
+}
+
+// Stage the step that starts at event e0 of the bucket into buffer buf; the
+// window must contain e0.  Returns the step's event count m.
 // `hint` (per thread, block-uniform) is a window segment index with
 // wcum[hint] <= e0; it is advanced to the last segment gathered.
-__device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t e0, uint32_t total, uint2* dst,
-                                 uint32_t& hint) {
+//
+// Run step (runs_ok: a whole-bucket item of a single-device context): when the
+// segment holding e0 is a run segment, the step is the following run segments (at
+// most kMaxStepRuns, kRunStepMax events, the window's end): warp 0 stages one
+// {offset, count, start} entry per segment and cp.async-copies its descriptor;
+// S.runk[buf] = the number of segments.  Otherwise an event step of <= STEP events
+// (S.runk[buf] = 0): cp.async copies of the stored events, runs synthesised.
+__device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t e0, uint32_t total, uint32_t buf,
+                                 uint32_t& hint, bool runs_ok) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t nwin = S.nwin;
+  uint2* dst = S.ev[buf];
+  const uint32_t base0 = hint & ~31u;
+  if (runs_ok) {
+    // the segment holding e0: usually the hint or the next one (steps end at segment ends)
+    uint32_t sa = hint;
+    if (sa + 1 < nwin && S.wcum[sa + 1] <= e0) {
+      ++sa;
+      if (sa + 1 < nwin && S.wcum[sa + 1] <= e0) {
+        uint32_t c0 = 0;                   // segments of the window starting at or before e0
+        for (uint32_t base = base0; base < nwin; base += 32) {
+          const uint32_t j = base + lane;
+          const uint32_t bl = __ballot_sync(FULL, (j < nwin ? S.wcum[j] : 0xFFFFFFFFu) <= e0);
+          c0 += __popc(bl);
+          if (bl != FULL) break;
+        }
+        sa = base0 + c0 - 1;
+      }
+    }
+    if (S.wstart[sa] >> 31) {
+      const uint32_t j = sa + lane;
+      const uint32_t msk = __ballot_sync(FULL, j < nwin && (S.wstart[j] >> 31));
+      const uint32_t nr = msk == FULL ? 32u : (uint32_t)__ffs(~msk) - 1u;   // consecutive run segments
+      const uint32_t e_end = min(min(total, S.wcum[sa + nr]), e0 + kRunStepMax);
+      const bool in = lane < nr && S.wcum[j] < e_end;
+      const uint32_t nseg = __popc(__ballot_sync(FULL, in));
+      if (warp == 0 && in) {
+        RunStage& R = *reinterpret_cast<RunStage*>(dst);
+        const uint32_t a = max(S.wcum[j], e0), z = min(S.wcum[j + 1], e_end);
+        R.info[lane] = make_uint4(a - S.wcum[j], z - a, a - e0, 0u);
+        cp_async8(&R.desc[lane], p.part_ev + (S.wstart[j] & 0x7FFFFFFFu));
+      }
+      cp_async_commit();
+      if (threadIdx.x == 0) S.runk[buf] = nseg;
+      hint = sa + nseg - 1;
+      return e_end - e0;
+    }
+  }
+  if (threadIdx.x == 0) S.runk[buf] = 0;
   const uint32_t m = min(min((uint32_t)STEP, total - e0), S.wcum[nwin] - e0);
   // Warp w gathers the slice [e0 + 32*RI*w, +32*RI) of the step.  Segment j holds
   // event e iff wcum[j] <= e < wcum[j+1]; every warp counts, from the hint, the
@@ -817,7 +893,6 @@ __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t 
   // event (ballots, no barrier), then each lane walks forward to the segment of
   // each of its events (segments are usually longer than the slice).
   const uint32_t s0 = e0 + warp * (32 * RI), last = e0 + m - 1;
-  const uint32_t base0 = hint & ~31u;
   uint32_t c0 = 0, c1 = 0;
   for (uint32_t base = base0; base < nwin; base += 32) {
     const uint32_t j = base + lane;
@@ -830,34 +905,42 @@ __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t 
   hint = base0 + c1 - 1;                 // segment of the step's last event
   if (s0 < e0 + m) {
     uint32_t seg = base0 + c0 - 1, seg_end = S.wcum[seg + 1];
-    // event e of segment seg sits at part_ev[wstart[seg] + e - wcum[seg]] = bp[e]
-    int64_t bp = (int64_t)S.wstart[seg] - (int64_t)S.wcum[seg];
     const uint32_t s_end = min(s0 + 32 * RI, e0 + m);
+    uint2* d = dst + (s0 - e0);
     if (s_end <= seg_end) {
       // the whole slice lies in one segment (warp-uniform; the common case):
       // a contiguous copy, 16 B per lane when both sides are 16-B aligned
-      const uint2* src = p.part_ev + (bp + s0);
-      uint2* d = dst + (s0 - e0);
+      const uint32_t ws = S.wstart[seg], c = S.wcum[seg];
       const uint32_t cnt = s_end - s0;
-      if (cnt == 32 * RI && ((reinterpret_cast<uintptr_t>(src) & 15u) == 0)) {
-#pragma unroll
-        for (int k = 0; k < RI / 2; ++k) cp_async16(d + 2 * (lane + 32 * k), src + 2 * (lane + 32 * k));
-      } else {
+      if (ws >> 31) {
+        const uint2 r = p.part_ev[ws & 0x7FFFFFFFu];
 #pragma unroll
         for (int k = 0; k < RI; ++k)
-          if (lane + 32 * k < cnt) cp_async8(d + lane + 32 * k, src + lane + 32 * k);
+          if (lane + 32 * k < cnt) d[lane + 32 * k] = make_uint2(r.x + (s0 - c) + lane + 32 * k, r.y + (s0 - c) + lane + 32 * k);
+      } else {
+        const uint2* src = p.part_ev + (ws + (s0 - c));
+        if (cnt == 32 * RI && ((reinterpret_cast<uintptr_t>(src) & 15u) == 0)) {
+#pragma unroll
+          for (int k = 0; k < RI / 2; ++k) cp_async16(d + 2 * (lane + 32 * k), src + 2 * (lane + 32 * k));
+        } else {
+#pragma unroll
+          for (int k = 0; k < RI; ++k)
+            if (lane + 32 * k < cnt) cp_async8(d + lane + 32 * k, src + lane + 32 * k);
+        }
       }
       cp_async_commit();
       return m;
     }
-    uint2* d = dst + (s0 - e0) + lane;
+    d += lane;
     if (seg + 2 <= nwin && s_end <= S.wcum[seg + 2]) {
-      // two segments: select the base per event
-      const int64_t bp1 = (int64_t)S.wstart[seg + 1] - (int64_t)seg_end;
+      // two segments: select the segment per event
 #pragma unroll
       for (int k = 0; k < RI; ++k) {
         const uint32_t e = s0 + k * 32 + lane;
-        if (e < s_end) cp_async8(d + k * 32, p.part_ev + ((e < seg_end ? bp : bp1) + e));
+        if (e < s_end) {
+          const uint32_t sg = e < seg_end ? seg : seg + 1;
+          gather_ev(d + k * 32, p, S.wstart[sg], e - S.wcum[sg]);
+        }
       }
       cp_async_commit();
       return m;
@@ -868,14 +951,210 @@ __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t 
       if (e < e0 + m) {
         if (e >= seg_end) {
           do { ++seg; seg_end = S.wcum[seg + 1]; } while (e >= seg_end);
-          bp = (int64_t)S.wstart[seg] - (int64_t)S.wcum[seg];
         }
-        cp_async8(d + k * 32, p.part_ev + (bp + e));
+        gather_ev(d + k * 32, p, S.wstart[seg], e - S.wcum[seg]);
       }
     }
   }
   cp_async_commit();
   return m;
+}
+
+// ---- run step -------------------------------------------------------------------------
+// Byte mask of bytes [a, a + n) of a 32-bit group (n = 1..4)
+__device__ __forceinline__ uint32_t byte_mask(uint32_t a, uint32_t n) {
+  return (0xFFFFFFFFu >> (32 - 8 * n)) << (8 * a);
+}
+
+// A step made only of runs (each: word A + j, op, position + j for j < count).  No
+// event is materialised: the shadow is processed in aligned groups of 4 words (one
+// 32-bit load per group, 4 states in SWAR form), and each group applies, in trace
+// order, every run that overlaps it — reads classify the covered bytes (P:263:
+// read_host needs OVv, read_target CVv; UUM / USD by the init bits), writes
+// take the VSM write image (WH: OVv, OVi set, CVv clear; WT: CVv, CVi set, OVv
+// clear).  Groups are the union of the runs' group intervals, merged so
+// that each group has one owner thread.  Every warp derives the run table and the
+// merged intervals itself (no block barrier).  BO (Z20): a target access to a word
+// without kCVp is a BO report and no transition; UM (Z23): a write makes 0xF.
+template <bool BO, bool UM>
+__device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uint32_t nseg, uint32_t cut) {
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint64_t bb = S.bucket_base;
+  const uint32_t a3 = (uint32_t)bb & 3u;
+  uint32_t* const gbase = reinterpret_cast<uint32_t*>(p.shadow + (bb - a3));
+  const uint32_t wlo = a3, whi = a3 + S.span;      // the bucket's words in A-coordinates
+  if (warp == 0) {                                  // the run table and the merged group intervals
+    constexpr uint32_t kNone = 0xFFFFFFFFu;
+    uint32_t A = 0, B = 0, ga = kNone, gb = 0, op = 0, pos = 0;
+    uint32_t len = 0;
+    if (lane < nseg) {
+      const uint4 inf = R.info[lane];
+      const uint2 ds = R.desc[lane];
+      len = inf.z >= cut ? 0u : min(inf.y, cut - inf.z);
+      const uint32_t key = ds.x + inf.x;
+      op = key >> 30; pos = ds.y + inf.x;
+      A = a3 + (key & kWordMask); B = A + len;
+    }
+    // a segment that continues the previous one (a run cut at a chunk boundary: same
+    // op, next word, next position) joins it: runs = chains of segments
+    const uint32_t pA = __shfl_up_sync(FULL, B, 1), pop = __shfl_up_sync(FULL, op, 1);
+    const uint32_t ppe = __shfl_up_sync(FULL, pos + (B - A), 1);
+    const uint32_t lens = __ballot_sync(FULL, len != 0);
+    const bool cont = lane > 0 && len && ((lens >> (lane - 1)) & 1u) && pA == A && pop == op && ppe == pos;
+    const uint32_t heads = __ballot_sync(FULL, len && !cont);
+    // chain end: the lane before the next head or the next empty segment
+    const uint32_t after = (heads | ~lens) & (lane == 31 ? 0u : 0xFFFFFFFEu << lane);
+    const uint32_t endl = after ? __ffs(after) - 2 : 31u;
+    const uint32_t Bc = __shfl_sync(FULL, B, endl);
+    const uint32_t nr = __popc(heads);
+    if ((heads >> lane) & 1u) R.run[__popc(heads & lanemask_lt())] = make_uint4(A, Bc, op, pos);
+    R.mm[lane] = 0;
+    __syncwarp();
+    if (lane < nr) {
+      const uint4 r = R.run[lane];
+      ga = r.x >> 2; gb = (r.y + 3) >> 2;
+    }
+    // sort the group intervals by first group (bitonic over the lanes; empty ones last)
+    uint32_t sga = ga, sgb = gb, sr = lane;
+    const uint32_t kmax = nr <= 1 ? 1u : 1u << (32 - __clz(nr - 1));       // sorting network width
+#pragma unroll
+    for (uint32_t k = 2; k <= 32; k <<= 1) {
+      if (k > kmax) break;
+#pragma unroll
+      for (uint32_t j = k >> 1; j > 0; j >>= 1) {
+        const uint32_t oga = __shfl_xor_sync(FULL, sga, j), ogb = __shfl_xor_sync(FULL, sgb, j);
+        const uint32_t orr = __shfl_xor_sync(FULL, sr, j);
+        const bool keep_min = ((lane & j) == 0) == ((lane & k) == 0 || k == kmax);
+        if (keep_min ? oga < sga : oga > sga) { sga = oga; sgb = ogb; sr = orr; }
+      }
+    }
+    const bool valid = sga != kNone;
+    uint32_t incl = valid ? sgb : 0u;                // inclusive prefix max of the interval ends
+#pragma unroll
+    for (uint32_t d = 1; d < 32; d <<= 1) {
+      const uint32_t o = __shfl_up_sync(FULL, incl, d);
+      if (lane >= d) incl = max(incl, o);
+    }
+    uint32_t excl = __shfl_up_sync(FULL, incl, 1);
+    if (lane == 0) excl = 0;
+    const bool start = valid && (lane == 0 || sga >= excl);
+    const uint32_t smask = __ballot_sync(FULL, start), vmask = __ballot_sync(FULL, valid);
+    const uint32_t nm = __popc(smask);
+    const uint32_t idx = __popc(smask & (0xFFFFFFFFu >> (31 - lane))) - 1u;   // merged interval of this lane
+    const bool lastl = valid && (lane == 31 || !((vmask >> (lane + 1)) & 1u) || ((smask >> (lane + 1)) & 1u));
+    __syncwarp();
+    if (valid) atomicOr(&R.mm[idx], 1u << sr);
+    if (start) R.mi[idx].x = sga;
+    if (lastl) R.mi[idx].y = incl;                   // the interval's end (exclusive group)
+    __syncwarp();
+    uint32_t n = 0, gs = 0;
+    if (lane < nm) { const uint2 v = R.mi[lane]; gs = v.x; n = v.y - v.x; }
+    uint32_t sc = n;
+#pragma unroll
+    for (uint32_t d = 1; d < 32; d <<= 1) {
+      const uint32_t o = __shfl_up_sync(FULL, sc, d);
+      if (lane >= d) sc += o;
+    }
+    __syncwarp();
+    if (lane < nm) R.mi[lane] = make_uint2(gs, sc - n);
+    if (lane == 31) { R.nm = nm; R.G = sc; }
+  }
+  __syncthreads();
+  const uint32_t nm = R.nm, G = R.G;
+  const uint64_t wbase = bb - a3;                    // relative word of A = 0
+  // a run's reports in one group, packed: run index (bits 0-4), faulting bytes
+  // (bits 5-8), 2 bits of kind per byte from bit 9 (0 UUM, 1 USD, 2 BO)
+  auto emit_one = [&](uint32_t slot, uint32_t w0, unsigned long long base) {
+    const uint4 r = R.run[slot & 31u];
+#pragma unroll
+    for (uint32_t b = 0; b < 4; ++b) {
+      if (!((slot >> (5 + b)) & 1u)) continue;
+      const uint32_t kc = (slot >> (9 + 2 * b)) & 3u;
+      if (base < p.cand_cap) {
+        const uint64_t wd = wbase + w0 + b;
+        p.cand[base] = make_uint4((uint32_t)wd, (uint32_t)(wd >> 32), r.w + (w0 + b - r.x), kc == 2 ? 4u : kc + 1u);
+      }
+      ++base;
+    }
+  };
+  for (uint32_t u0 = 0; u0 < G; u0 += RT) {
+    const uint32_t u = u0 + threadIdx.x;
+    uint32_t ns = 0, fs0 = 0, fs1 = 0;
+    uint32_t w0 = 0;
+    if (u < G) {
+      uint32_t j = 0;                                 // merged interval: the last with first unit <= u
+#pragma unroll
+      for (uint32_t st = 16; st; st >>= 1)
+        if (j + st < nm && R.mi[j + st].y <= u) j += st;
+      const uint2 mv = R.mi[j];
+      const uint32_t g = mv.x + (u - mv.y);
+      w0 = 4 * g;
+      uint32_t s = __ldcg(gbase + g);
+      uint32_t wr = 0;
+      for (uint32_t mm = R.mm[j]; mm; mm &= mm - 1) {
+        const uint32_t ri = __ffs(mm) - 1;
+        const uint4 r = R.run[ri];
+        const uint32_t lo = max(r.x, w0), hi = min(r.y, w0 + 4);
+        if (lo >= hi) continue;
+        const uint32_t M = byte_mask(lo - w0, hi - lo);
+        const uint32_t o = r.z;
+        uint32_t Me = M, bof = 0;
+        if (BO && (o & 2u)) {                         // no CV: buffer overflow, no transition (Z20)
+          bof = (~s >> 4) & 0x01010101u & M;
+          Me = M & ~(bof * 0xFFu);
+        }
+        uint32_t fv = 0;
+        if (!(o & 1u)) {
+          fv = (~s >> (o >> 1)) & 0x01010101u & Me;   // RH: OVv (bit 0), RT: CVv (bit 1)
+        } else {
+          const uint32_t img = UM ? 0x0F0F0F0Fu
+                             : o == OP_WH ? ((s & (BO ? 0x18181818u : 0x08080808u)) | 0x05050505u)
+                                          : ((s & (BO ? 0x14141414u : 0x04040404u)) | 0x0A0A0A0Au);
+          s = (s & ~Me) | (img & Me);
+          wr |= Me;
+        }
+        if (fv | bof) {                               // reports (rare)
+          const uint32_t usd = (s >> (2 + (o >> 1))) & 0x01010101u;   // the read side's init bit
+          uint32_t slot = ri;
+#pragma unroll
+          for (uint32_t b = 0; b < 4; ++b) {
+            if (!(((fv | bof) >> (8 * b)) & 1u)) continue;
+            const uint32_t kc = ((bof >> (8 * b)) & 1u) ? 2u : (usd >> (8 * b)) & 1u;
+            slot |= (1u << (5 + b)) | (kc << (9 + 2 * b));
+          }
+          if (ns == 0) fs0 = slot;
+          else if (ns == 1) fs1 = slot;
+          else emit_one(slot, w0, atomicAdd(&p.st->n_cand, (unsigned long long)__popc((slot >> 5) & 15u)));
+          ++ns;
+        }
+      }
+      if (wr) {
+        if (w0 >= wlo && w0 + 4 <= whi) {
+          __stcg(gbase + g, s);
+        } else {                                      // a group shared with a neighbouring bucket
+          uint8_t* gb8 = reinterpret_cast<uint8_t*>(gbase + g);
+#pragma unroll
+          for (uint32_t b = 0; b < 4; ++b)
+            if ((wr >> (8 * b)) & 0xFFu) __stcg(gb8 + b, (uint8_t)(s >> (8 * b)));
+        }
+      }
+    }
+    // the reports of each lane's first two faulting runs: one warp-aggregated append
+    const uint32_t k = (ns > 0 ? __popc((fs0 >> 5) & 15u) : 0u) + (ns > 1 ? __popc((fs1 >> 5) & 15u) : 0u);
+    if (__any_sync(FULL, k != 0)) {
+      uint32_t sk = k;
+#pragma unroll
+      for (uint32_t d = 1; d < 32; d <<= 1) {
+        const uint32_t o = __shfl_up_sync(FULL, sk, d);
+        if (lane >= d) sk += o;
+      }
+      unsigned long long base = 0;
+      if (lane == 31) base = atomicAdd(&p.st->n_cand, (unsigned long long)sk);
+      base = __shfl_sync(FULL, base, 31) + (sk - k);
+      if (ns > 0) emit_one(fs0, w0, base);
+      if (ns > 1) emit_one(fs1, w0, base + __popc((fs0 >> 5) & 15u));
+    }
+  }
 }
 
 // BO: ARB_F_BO contexts (the buffer-overflow extension, Z20) get their own
@@ -908,6 +1187,7 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       S.op_cur = p.ops_start[b];
       S.op_end = p.ops_start[b + 1];
       S.bucket_base = p.bucket_start[b];
+      S.span = (uint32_t)(p.bucket_start[b + 1] - S.bucket_base);
       S.shrel = p.shadow + S.bucket_base;
     }
     bucket_setup(S, p, b);
@@ -944,9 +1224,10 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
     if (tid == 0) S.next_op = S.op_cur < S.op_end ? p.ops[S.op_cur].pos : 0xFFFFFFFFu;
     __syncthreads();
     uint32_t e0 = first, cur = 0, m_cur = 0, hint = 0;
+    const bool runs_ok = !MD && mode == kItemWhole && !p.no_run_steps;   // run steps: whole buckets, one device
     if (e0 < total) {
       ensure_window(S, p, e0, hint);
-      m_cur = issue_gather(S, p, e0, total, S.ev[0], hint);
+      m_cur = issue_gather(S, p, e0, total, 0, hint, runs_ok);
     }
     while (e0 < total) {
       cp_async_wait_all();
@@ -958,18 +1239,39 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       uint32_t m_nxt = 0;
       if (nxt < total) {
         ensure_window(S, p, nxt, hint);
-        m_nxt = issue_gather(S, p, nxt, total, S.ev[cur ^ 1], hint);
+        m_nxt = issue_gather(S, p, nxt, total, cur ^ 1, hint, runs_ok);
       }
       // ---- range ops before the first event, then cut at the next one -------------
       constexpr uint32_t pm = MD ? kMdPos : 0xFFFFFFFFu;   // MD: strip the device bits (Z24)
-      apply_ops_before<BO, MD>(S, p, ev[0].y & pm);
+      const uint32_t nrs = MD ? 0u : S.runk[cur];
+      RunStage& R = *reinterpret_cast<RunStage*>(S.ev[cur]);
       uint32_t cut = m;
-      if (S.next_op != 0xFFFFFFFFu && (ev[m - 1].y & pm) > S.next_op) {
-        uint32_t cnt = 0;
-        for (uint32_t e = tid; e < m; e += RT) cnt += (ev[e].y & pm) < S.next_op;
-        cut = block_sum(cnt, S.red);
+      if (nrs) {                                   // run step: positions from the descriptors
+        apply_ops_before<BO, MD>(S, p, R.desc[0].y + R.info[0].x);
+        const uint4 li = R.info[nrs - 1];
+        const uint32_t nx = S.next_op;
+        if (nx != 0xFFFFFFFFu && R.desc[nrs - 1].y + li.x + li.y - 1 > nx) {
+          const uint32_t lane = tid & 31;
+          uint32_t c = 0;
+          if (lane < nrs) {
+            const uint4 in = R.info[lane];
+            const uint32_t p0 = R.desc[lane].y + in.x;
+            c = p0 + in.y <= nx ? in.y : (p0 < nx ? nx - p0 : 0u);
+          }
+          cut = __reduce_add_sync(FULL, c);
+        }
+      } else {
+        apply_ops_before<BO, MD>(S, p, ev[0].y & pm);
+        if (S.next_op != 0xFFFFFFFFu && (ev[m - 1].y & pm) > S.next_op) {
+          uint32_t cnt = 0;
+          for (uint32_t e = tid; e < m; e += RT) cnt += (ev[e].y & pm) < S.next_op;
+          cut = block_sum(cnt, S.red);
+        }
       }
-      if (mode == kItemSummary) {
+      if (nrs) {
+        if (cut) step_runs<BO, UM>(S, p, R, nrs, cut);
+        if (tid == 0) atomicAdd(&p.st->steps_run, 1ull);
+      } else if (mode == kItemSummary) {
         step_summary<BO, UM, MD>(S, ev, cut);
       } else {
         const bool fast = S.partial ? step_fast_partial<BO, UM, MD>(S, p, ev, cut)
@@ -987,10 +1289,12 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         __syncthreads();
         hint = 0;
         ensure_window(S, p, e0, hint);
-        m_cur = issue_gather(S, p, e0, total, S.ev[cur], hint);
+        m_cur = issue_gather(S, p, e0, total, cur, hint, runs_ok);
       }
     }
-    // the ops after the last event (a slice replay's private states are not kept)
+    // the ops after the last event (a slice replay's private states are not kept);
+    // the last step's shadow stores (a run step ends without a barrier) come first
+    __syncthreads();
     if (mode != kItemSlice) apply_ops_before<BO, MD>(S, p, 0xFFFFFFFFu);
     if (tid == 0 && total > first) atomicMax(&p.st->max_bucket_events, (unsigned long long)(total - first));
     __syncthreads();

@@ -657,3 +657,20 @@ def test_devices_hot_word(orc):
     exp, st = check(orc, rec, A, 64, flags=2 << 8)
     assert st["hot_buckets"] >= 1
     check(orc, rec, A, 64, flags=(2 << 8) | 4)
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_runs_fuzz(orc, seed):
+    """Run-form chunks and run steps: loops mostly over consecutive
+    words, bucket sizes that put bucket boundaries inside runs, the BO and UM
+    instances, flush cuts (tasks included)."""
+    from gen.fuzz import run_program
+    rec, base, span = run_program(2000 + seed)
+    flags = [0, 8, 16][seed % 3]
+    runs = 0
+    for bb in (0, 9, 12):
+        _, st = check(orc, rec, base, span, bucket_bits=bb, flags=flags)
+        runs += st["steps_run"]
+    assert runs > 0
+    cuts = sorted(int(x) for x in np.random.default_rng(seed).choice(rec.shape[0], 3, replace=False))
+    check(orc, rec, base, span, flags=flags, flush_points=cuts)
