@@ -185,6 +185,8 @@ typedef struct {
   uint64_t steps_run;        /* replay steps made only of run segments       */
   uint64_t segments;         /* (chunk, bucket) segment entries of the last flush (runs and
                                 stored-event segments)                                        */
+  uint64_t chunks, chunks_fast, chunks_run;  /* partition chunks (256 records) of the last flush:
+                                all, on the fast path, written in run form                     */
 } arb_stats;
 
 typedef struct arb_ctx_s* arb_ctx;

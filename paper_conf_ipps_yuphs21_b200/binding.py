@@ -58,7 +58,8 @@ class arb_stats(ctypes.Structure):
                 ("work_items", ctypes.c_uint64), ("hot_buckets", ctypes.c_uint64),
                 ("reports_bo", ctypes.c_uint64), ("nccl_ranks", ctypes.c_uint64),
                 ("exchanges", ctypes.c_uint64), ("steps_run", ctypes.c_uint64),
-                ("segments", ctypes.c_uint64)]
+                ("segments", ctypes.c_uint64), ("chunks", ctypes.c_uint64),
+                ("chunks_fast", ctypes.c_uint64), ("chunks_run", ctypes.c_uint64)]
 
     def as_dict(self):
         d = {}

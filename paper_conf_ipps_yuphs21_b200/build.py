@@ -35,7 +35,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     objs = []
     for src in sources():
         obj = os.path.join(objdir, os.path.basename(src) + ".o")
-        cmd = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC,-O3,-Wall",
+        cmd = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", *os.environ.get("ARB_NVCC_FLAGS", "").split(),
+               "-Xcompiler", "-fPIC,-O3,-Wall",
                "-I", INCLUDE, "-I", CSRC, "-c", src, "-o", obj]
         if src.endswith(".cu"):
             cmd += ["-Xptxas", "-v"] if verbose else []

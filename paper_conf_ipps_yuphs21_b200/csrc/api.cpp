@@ -525,7 +525,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   S.reports = 0; std::memset(S.reports_by_kind, 0, sizeof(S.reports_by_kind)); S.ignored_words = 0;
   S.ms_partition = S.ms_control = S.ms_replay = S.ms_mir = S.ms_reports = S.ms_total = 0;
   S.ms_segsort = S.ms_host_control = 0;
-  S.steps_run = S.segments = 0;
+  S.steps_run = S.segments = S.chunks = S.chunks_fast = S.chunks_run = 0;
   S.buckets = ctx->n_buckets; S.bucket_bits = ctx->bucket_bits; S.max_bucket_events = 0;
 
   // Phase A (validation): decode + partition and control resolution.  Nothing
@@ -764,6 +764,8 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   rp.md = ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u) ? 1u : 0u; rp.ops_start = ctx->ops_start.p; rp.ops = ctx->ops.p;
   rp.cand = ctx->cand.p; rp.cand_cap = ctx->cand_cap; rp.st = ctx->dstats.p;
   rp.no_run_steps = getenv("ARB_NO_RUN_STEPS") != nullptr;
+  rp.no_run_prep = getenv("ARB_NO_RUN_PREP") != nullptr;
+  rp.run_step_max = getenv("ARB_RUN_STEP_MAX") ? (uint32_t)std::max(256, atoi(getenv("ARB_RUN_STEP_MAX"))) : 16384u;
   rp.hot_off = ctx->d_hot_off.p; rp.hot_F = ctx->hot_F.p; rp.hot_P = ctx->hot_P.p;
   int n_ctas = std::max(1, std::min<int>((int)ctx->items.size(), ctx->n_sms * kReplayCtasPerSm));
   CK(launch_replay(rp, std::max(n_ctas, 1), s), "k_replay");
@@ -792,6 +794,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   S.steps_sort = hst.steps_sort;
   S.steps_run = hst.steps_run;
   S.segments = hst.n_segs;
+  S.chunks = (n + kChunkRecords - 1) / kChunkRecords; S.chunks_fast = hst.chunks_fast; S.chunks_run = hst.chunks_run;
 
   // ---- A6: MIR join ---------------------------------------------------------------
   uint64_t n_mir = 0;

@@ -67,7 +67,8 @@ constexpr int kSegChunkBits = 21;                    // chunk id bits in the ent
 // Run segments: a segment entry whose start has kRunFlag holds a run —
 // event j of the segment is {key + j, position + j}, where {key, position} is the
 // run's descriptor stored at the start slot of the chunk's output (no other events
-// are written).  A fast chunk of at most kMaxChunkRuns runs is written in this form.
+// are written).  A fast chunk of at most kMaxChunkRuns runs is written in this form;
+// a run that continues into the warp's next chunk extends its entry (len < 2^15).
 constexpr uint32_t kRunFlag = 0x8000u;
 constexpr int kMaxChunkRuns = 16;
 
@@ -113,6 +114,7 @@ struct DevStats {
   unsigned long long n_bo_cand;       // N1 (Z25): base-tag overflow candidates
   unsigned long long n_cv_acc;        // N1 (Z26): target accesses by CV address (left untracked)
   unsigned long long steps_run;      // replay steps made only of run segments
+  unsigned long long chunks_run, chunks_fast;   // partition chunks written in run form / fast event form
 };
 
 // control record extracted by the partition kernel
@@ -182,6 +184,8 @@ struct ReplayParams {
   uint32_t um;                            // ARB_F_UNIFIED: OV and CV are one storage (Z23)
   uint32_t md;                            // several accelerators (Z24): 8-bit states, device in pos bits 30-31
   uint32_t no_run_steps;                  // debug (ARB_NO_RUN_STEPS): run segments only as synthesised events
+  uint32_t no_run_prep;                   // debug (ARB_NO_RUN_PREP): no run-step table built during the previous step
+  uint32_t run_step_max;                  // events per run step (ARB_RUN_STEP_MAX, default 16384)
   const uint32_t* ops_start;              // [n_buckets + 1]
   const BucketOp* ops;
   uint4* cand; uint64_t cand_cap;         // report candidates {word lo, word hi, pos, kind}

@@ -365,9 +365,10 @@ static int add_field_passes(RsPass* ps, int np, int field, int bits) {
 }
 
 // Segment entries as written by k_partition (8 B): x = bucket << 21 | chunk bits
-// 0-20, y = start | len << 16 | chunk bit 21 << 31 (start, len <= 512).
+// 0-20, y = start | len << 16 | chunk bit 21 << 31 (start < 512 with kRunFlag for a
+// run; len <= 512 for stored events, < 2^15 for a run continued over chunks).
 __device__ __forceinline__ uint32_t seg_bucket(uint2 e) { return e.x >> kSegChunkBits; }
-__device__ __forceinline__ uint32_t seg_len(uint2 e) { return (e.y >> 16) & 0x3FFu; }
+__device__ __forceinline__ uint32_t seg_len(uint2 e) { return (e.y >> 16) & 0x7FFFu; }
 __device__ __forceinline__ uint32_t seg_chunk(uint2 e) {
   return (e.x & ((1u << kSegChunkBits) - 1u)) | ((e.y >> 31) << kSegChunkBits);
 }
@@ -423,7 +424,7 @@ __global__ void __launch_bounds__(kRsThreads) k_seg_cum(const uint2* segs, uint6
 #pragma unroll
   for (int j = 0; j < kRsItems; ++j) {
     if (base + j < n)
-      out[base + j] = make_uint4(seg_chunk(e[j]), seg_bucket(e[j]), e[j].y & 0x3FFFFFFu, run);
+      out[base + j] = make_uint4(seg_chunk(e[j]), seg_bucket(e[j]), e[j].y & 0x7FFFFFFFu, run);
     run += seg_len(e[j]);
   }
 }

@@ -130,40 +130,54 @@ __device__ __forceinline__ void rank_round(uint32_t info, uint16_t* row, uint16_
   r1 = r0 + 1;
 }
 
+// The run that ended the warp's previous chunk (warp-uniform): its segment entry is
+// still in the warp's buffer (segbuf[idx]), so a run of the next chunk (the warp's
+// chunks are consecutive) that continues it — same op, the next word, same bucket —
+// extends that entry instead of opening a new one.
+struct OpenRun { uint32_t idx, op, bkt, len; uint64_t next_word; };
+constexpr uint32_t kNoOpen = 0xFFFFFFFFu;
+constexpr uint32_t kMaxRunLen = 0x7FFFu;      // events of a run entry (15-bit length field)
+
 // The fast chunk test and its output.  Every record must be an access (op < 4)
 // of 1..8 bytes inside one 8-byte word (such an access cannot leave the
-// 48-bit space).  A chunk of few runs (below) is written in run form; otherwise
-// all words must lie in one address bucket or in two adjacent ones (a stable
-// two-way split by the bucket boundary).  Buckets are
-// contiguous word ranges, so the test needs only the chunk's lowest and highest
-// word: each word is taken relative to record 0's word w0 (32-bit signed,
-// |d| < 2^30 as a bucket spans <= 2^30 words), the warp reduces min and max, and
-// two bin-map lookups decide.  A word's offset in the bucket is then
+// 48-bit space) in record 0's 2^32-byte block or a neighbouring one (so word
+// differences are 32-bit).  A chunk of few runs (below) is written in run form; otherwise all
+// words must lie in one address bucket or in two adjacent ones (a stable two-way
+// split by the bucket boundary).  Buckets are contiguous word ranges, so the test
+// needs only the chunk's lowest and highest word: each word is taken relative to
+// record 0's word w0 (32-bit signed, |d| < 2^30), the warp reduces min and max,
+// and two bin-map lookups decide.  A word's offset in the bucket is then
 // off(lowest) + d - dmin.  Returns false (nothing written) when the test fails.
 template <bool MD>
 __device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p, uint32_t chunk, uint2* out,
-                                           uint2* segbuf, uint32_t& nbuf, uint32_t lane, uint16_t* scratch) {
+                                           uint2* segbuf, uint32_t& nbuf, uint32_t lane, uint16_t* scratch,
+                                           OpenRun& orun) {
   const uint4 q0 = st[0];
   const uint64_t w0 = ((uint64_t)((q0.y & 0xFFFFu) >> 3) << 32) | __funnelshift_r(q0.x, q0.y, 3);
+  const uint32_t x0w = __funnelshift_r(q0.x, q0.y, 3);        // record 0's word, low 32 bits
+  const uint32_t h0 = (q0.y & 0xFFFFu) - 1u;                   // record 0's address bits 32-47, minus 1
   uint32_t d[RPL], opk[RPL], bad = 0, devs = 0;
   int32_t dmin = 0, dmax = 0;
 #pragma unroll
   for (int k = 0; k < RPL; ++k) {
     const uint4 q = st[k * 32 + lane];
-    bad |= (q.y & (0x00FC0000u | kCvAddrBit)) | (q.w & 0xFFFFu) | ((q.z - 1u) & ~7u) | (((q.x & 7u) + q.z - 1u) & ~7u);
+    // an access (op < 4, OV address) of 1..8 bytes inside one word, whose address
+    // bits 32-47 are record 0's, or one more or less: its word is then record 0's
+    // word + d with |d| < 2^30, d = the difference of the words' low 32 bits
+    bad |= (q.y & (0x00FC0000u | kCvAddrBit)) | (q.w & 0xFFFFu) | ((q.y & 0xFFFFu) - h0 > 2u) |
+           (((q.z - 1u) | ((q.x & 7u) + q.z - 1u)) & ~7u);
     if (MD && (q.y & (1u << 17))) {                // RT / WT on device arg (Z24)
       const uint32_t dv = q.y >> 24;
       bad |= dv >= p.n_dev;
       devs |= (dv & 3u) << (2 * k);
     }
-    const uint64_t word = ((uint64_t)((q.y & 0xFFFFu) >> 3) << 32) | __funnelshift_r(q.x, q.y, 3);
-    const uint64_t diff = word - w0;
-    bad |= (uint32_t)((diff + (1ull << 30)) >> 31);      // d outside [-2^30, 2^30)
-    d[k] = (uint32_t)diff;
+    d[k] = __funnelshift_r(q.x, q.y, 3) - x0w;
     dmin = min(dmin, (int32_t)d[k]);
     dmax = max(dmax, (int32_t)d[k]);
     opk[k] = ((q.y >> 16) & 3u) << 30;
   }
+  const OpenRun prev = orun;
+  orun.idx = kNoOpen;                        // reset unless the chunk ends in a run
   if (!__all_sync(FULL, bad == 0)) return false;
   dmin = __reduce_min_sync(FULL, dmin);
   dmax = __reduce_max_sync(FULL, dmax);
@@ -211,12 +225,13 @@ __device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p,
       // lane r: run r, inside one bucket or split at the boundary of two adjacent ones
       bool ok = true, split = false;
       uint32_t i = 0, len = 0, len1 = 0, bkt = 0, off = 0, opr = 0;
+      uint64_t first = 0;
       if (lane < nR) {
         i = kb[lane];
         len = (lane + 1 < nR ? kb[lane + 1] : (uint32_t)WREC) - i;
         const uint32_t kv = kb[kMaxChunkRuns + lane];
         opr = kv & 3u;
-        const uint64_t first = w0 - p.base_word + (uint64_t)(int64_t)((int32_t)kv >> 2) + i;   // d_i = v + i
+        first = w0 - p.base_word + (uint64_t)(int64_t)((int32_t)kv >> 2) + i;   // d_i = v + i
         const uint64_t last = first + len - 1;
         const uint32_t m1 = __ldg(p.bin_map + (uint32_t)(first >> cb)), m2 = __ldg(p.bin_map + (uint32_t)(last >> cb));
         bkt = m1 & kBucketMask;
@@ -230,17 +245,34 @@ __device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p,
       __syncwarp();
       if (__all_sync(FULL, ok)) {
         const uint32_t sp = __ballot_sync(FULL, split);
+        // run 0 continues the previous chunk's open run?
+        const uint32_t mg = __shfl_sync(FULL, (uint32_t)(lane == 0 && prev.idx != kNoOpen && opr == prev.op &&
+                                                         first == prev.next_word && bkt == prev.bkt &&
+                                                         prev.len + len1 <= kMaxRunLen), 0);
+        const uint32_t e = nbuf + lane + __popc(sp & lanemask_lt()) - mg;   // entry of this run's first piece
         if (lane < nR) {
           const uint32_t ck = chunk & ((1u << kSegChunkBits) - 1u);
-          const uint32_t e = nbuf + lane + __popc(sp & lanemask_lt());
-          out[i] = make_uint2((opr << 30) | off, rec0 + i);
-          segbuf[e] = make_uint2((bkt << kSegChunkBits) | ck, i | kRunFlag | (len1 << 16) | chi);
+          if (lane == 0 && mg) {
+            segbuf[prev.idx].y += len1 << 16;
+          } else {
+            out[i] = make_uint2((opr << 30) | off, rec0 + i);
+            segbuf[e] = make_uint2((bkt << kSegChunkBits) | ck, i | kRunFlag | (len1 << 16) | chi);
+          }
           if (split) {                     // the rest starts at the first word of bucket bkt + 1
             out[i + len1] = make_uint2(opr << 30, rec0 + i + len1);
             segbuf[e + 1] = make_uint2(((bkt + 1) << kSegChunkBits) | ck, (i + len1) | kRunFlag | ((len - len1) << 16) | chi);
           }
         }
-        nbuf += nR + __popc(sp);
+        // the chunk's last piece stays open for the next chunk
+        const uint32_t L = nR - 1;
+        const uint32_t oi = (L == 0 && mg && !split) ? prev.idx : e + (split ? 1u : 0u);
+        const uint32_t ol = (L == 0 && mg && !split) ? prev.len + len1 : (split ? len - len1 : len1);
+        orun.idx = __shfl_sync(FULL, oi, L);
+        orun.len = __shfl_sync(FULL, ol, L);
+        orun.op = __shfl_sync(FULL, opr, L);
+        orun.bkt = __shfl_sync(FULL, split ? bkt + 1 : bkt, L);
+        orun.next_word = __shfl_sync(FULL, first + len, L);
+        nbuf += nR + __popc(sp) - mg;
         return true;
       }
     }
@@ -317,11 +349,18 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   fence_mbar_init();
   __syncwarp();
   uint32_t n_acc = 0, n_ign = 0, n_cv = 0, nbuf = 0, phase = 0;   // phase: parity bit of each stage's barrier
+  uint32_t n_fast = 0, n_runc = 0;                                 // chunks: fast path / ending in an open run
 
   // the chunk's records arrive in stage k by one TMA bulk copy (lane 0) that
   // completes on bar[k]
+  // the warp's chunks: a contiguous range (consecutive chunks let runs continue
+  // from one chunk into the next, OpenRun)
+  const uint64_t nwarps = (uint64_t)gridDim.x * PW;
+  const uint64_t cpw = (p.n_chunks + nwarps - 1) / nwarps;
+  const uint64_t c_begin = ((uint64_t)blockIdx.x * PW + warp) * cpw;
+  const uint64_t c_end = c_begin + cpw < p.n_chunks ? c_begin + cpw : p.n_chunks;
   auto fetch = [&](uint64_t c, uint32_t k) {
-    if (c < p.n_chunks && lane == 0) {
+    if (c < c_end && lane == 0) {
       const uint64_t r0 = c * WREC;
       const uint32_t nv = p.n - r0 < (uint64_t)WREC ? (uint32_t)(p.n - r0) : (uint32_t)WREC;
       mbar_arrive_tx(bar + k, nv * 16u);
@@ -338,14 +377,15 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     __syncwarp();
     nbuf = 0;
   };
+  OpenRun orun;
+  orun.idx = kNoOpen; orun.op = orun.bkt = orun.len = 0; orun.next_word = 0;
 
-  const uint64_t nwarps = (uint64_t)gridDim.x * PW;
   uint32_t cur = 0;
-  uint64_t chunk = (uint64_t)blockIdx.x * PW + warp;
+  uint64_t chunk = c_begin;
 #pragma unroll
-  for (int k = 0; k < NST - 1; ++k) fetch(chunk + k * nwarps, k);
-  for (; chunk < p.n_chunks; chunk += nwarps) {
-    fetch(chunk + (NST - 1) * nwarps, cur == 0 ? NST - 1 : cur - 1);
+  for (int k = 0; k < NST - 1; ++k) fetch(chunk + k, k);
+  for (; chunk < c_end; ++chunk) {
+    fetch(chunk + (NST - 1), cur == 0 ? NST - 1 : cur - 1);
     mbar_wait(bar + cur, (phase >> cur) & 1u);
     phase ^= 1u << cur;
     const uint4* st = stage + cur * WREC;
@@ -355,9 +395,23 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     // ones (the common case of real access streams: runs over one array).  One bucket:
     // event j is record j, one coalesced store per record, one segment entry; two:
     // a stable two-way split and two entries.  Anything else takes the general path.
-    if (nbuf + 2 * kMaxChunkRuns > kSegBuf) flush_segs();
+    if (nbuf + 2 * kMaxChunkRuns > kSegBuf) {
+      if (orun.idx != kNoOpen) {         // keep the open run's entry (the last one) in the buffer
+        const uint2 keep = segbuf[nbuf - 1];
+        --nbuf;
+        flush_segs();
+        if (lane == 0) segbuf[0] = keep;
+        __syncwarp();
+        nbuf = 1; orun.idx = 0;
+      } else {
+        flush_segs();
+      }
+    }
+    if (nvalid < WREC) orun.idx = kNoOpen;
     if (nvalid == WREC && fast_chunk<MD>(st, p, (uint32_t)chunk, p.part_ev + chunk * kChunkCap,
-                                     segbuf, nbuf, lane, tlist)) {
+                                     segbuf, nbuf, lane, tlist, orun)) {
+      n_fast += 1u;
+      n_runc += orun.idx != kNoOpen;
       n_acc += RPL;
       cur = cur + 1 == NST ? 0 : cur + 1;
       __syncwarp();                    // stage[cur] reads done before the next fetch overwrites it
@@ -529,6 +583,8 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     if (n_acc) atomicAdd(&p.st->access_words, (unsigned long long)n_acc);
     if (n_ign) atomicAdd(&p.st->ignored_words, (unsigned long long)n_ign);
     if (n_cv) atomicAdd(&p.st->n_cv_acc, (unsigned long long)n_cv);
+    if (n_fast) atomicAdd(&p.st->chunks_fast, (unsigned long long)n_fast);
+    if (n_runc) atomicAdd(&p.st->chunks_run, (unsigned long long)n_runc);
   }
 }
 

@@ -46,7 +46,6 @@ static_assert(kZSlots == 2 * STEP, "summary hash: twice the step");
 // Run steps: a step made only of run segments never materialises
 // its events; the gather stages the runs' descriptors in the step's event buffer.
 constexpr int kMaxStepRuns = 32;             // run segments per run step
-constexpr uint32_t kRunStepMax = 8192;       // events per run step
 struct RunStage {
   uint4 info[kMaxStepRuns];                  // {first event's offset in the run, events, step-relative start, 0}
   uint2 desc[kMaxStepRuns];                  // the runs' descriptors {key, position} (cp.async)
@@ -79,7 +78,6 @@ struct ReplaySmem {
   uint32_t* fsum;                 // summary slice: composed transition of word w: fsum[w] (kfun_*)
   uint32_t slice, n_slices;       // hot bucket slice (kItemSlice / kItemSummary)
   uint32_t seg0, cum0, n_segs, n_events, wsc, nwin;
-  uint32_t runk[2];               // run segments staged in buffer b (0: an event step)
   uint32_t span;                  // words of the bucket
   uint64_t bucket_base;
 };
@@ -144,6 +142,25 @@ template <bool BO, bool MD>
 __device__ __forceinline__ uint32_t apply_sel(Sel s, uint32_t x) {
   return MD ? sel8_apply4(s, x) : BO ? sel_apply5(s, x) : sel_apply4(s, x);
 }
+// A 4-bit selector as SWAR masks over 4 states: out = (x & K) | C | ((x << 1) & U) |
+// ((x >> 1) & D) — every output bit kept, constant, or copied from the other bit of
+// its pair (OV/CV valid bits 0-1, init bits 2-3), which covers the transitions of
+// Table I and their compositions.  Returns false for any other selector.
+__device__ __forceinline__ bool sel_swar(Sel s, uint32_t& K, uint32_t& C, uint32_t& U, uint32_t& D) {
+  K = C = U = D = 0;
+#pragma unroll
+  for (uint32_t j = 0; j < 4; ++j) {
+    const uint32_t src = (s >> (3 * j)) & 7u, b = 0x01010101u << j;
+    if (src == j) K |= b;
+    else if (src == 5) C |= b;
+    else if (src == 4) {}
+    else if ((j & 1u) && src == j - 1) U |= b;
+    else if (!(j & 1u) && src == j + 1) D |= b;
+    else return false;
+  }
+  return true;
+}
+
 template <bool BO, bool MD>
 __device__ void stream_apply(uint8_t* base, uint64_t lo, uint64_t hi, Sel sel) {
   if (lo >= hi) return;
@@ -158,6 +175,26 @@ __device__ void stream_apply(uint8_t* base, uint64_t lo, uint64_t hi, Sel sel) {
   const uint64_t nv = (b - a) >> 4;
   constexpr int U = 4;   // 4 x 16 B loads in flight per thread
   uint64_t j = threadIdx.x;
+  uint32_t mK, mC, mU, mD;
+  if (!BO && !MD && sel_swar(sel, mK, mC, mU, mD)) {
+    auto f = [&](uint32_t x) { return (x & mK) | mC | ((x << 1) & mU) | ((x >> 1) & mD); };
+    for (; j + (U - 1) * RT < nv; j += U * RT) {
+      uint4 x[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) x[u] = __ldcg(v + j + u * RT);
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        x[u].x = f(x[u].x); x[u].y = f(x[u].y); x[u].z = f(x[u].z); x[u].w = f(x[u].w);
+        __stcg(v + j + u * RT, x[u]);
+      }
+    }
+    for (; j < nv; j += RT) {
+      uint4 x = __ldcg(v + j);
+      x.x = f(x.x); x.y = f(x.y); x.z = f(x.z); x.w = f(x.w);
+      __stcg(v + j, x);
+    }
+    return;
+  }
   for (; j + (U - 1) * RT < nv; j += U * RT) {
     uint4 x[U];
 #pragma unroll
@@ -840,12 +877,13 @@ __device__ __forceinline__ void gather_ev(uint2* d, const ReplayParams& p, uint3
 //
 // Run step (runs_ok: a whole-bucket item of a single-device context): when the
 // segment holding e0 is a run segment, the step is the following run segments (at
-// most kMaxStepRuns, kRunStepMax events, the window's end): warp 0 stages one
+// most kMaxStepRuns, p.run_step_max events, the window's end): warp 0 stages one
 // {offset, count, start} entry per segment and cp.async-copies its descriptor;
-// S.runk[buf] = the number of segments.  Otherwise an event step of <= STEP events
-// (S.runk[buf] = 0): cp.async copies of the stored events, runs synthesised.
+// nrun = the number of segments.  Otherwise an event step of <= STEP events
+// (nrun = 0): cp.async copies of the stored events, runs synthesised.
 __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t e0, uint32_t total, uint32_t buf,
-                                 uint32_t& hint, bool runs_ok) {
+                                 uint32_t& hint, bool runs_ok, uint32_t& nrun) {
+  nrun = 0;
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t nwin = S.nwin;
   uint2* dst = S.ev[buf];
@@ -870,7 +908,7 @@ __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t 
       const uint32_t j = sa + lane;
       const uint32_t msk = __ballot_sync(FULL, j < nwin && (S.wstart[j] >> 31));
       const uint32_t nr = msk == FULL ? 32u : (uint32_t)__ffs(~msk) - 1u;   // consecutive run segments
-      const uint32_t e_end = min(min(total, S.wcum[sa + nr]), e0 + kRunStepMax);
+      const uint32_t e_end = min(min(total, S.wcum[sa + nr]), e0 + p.run_step_max);
       const bool in = lane < nr && S.wcum[j] < e_end;
       const uint32_t nseg = __popc(__ballot_sync(FULL, in));
       if (warp == 0 && in) {
@@ -880,12 +918,11 @@ __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t 
         cp_async8(&R.desc[lane], p.part_ev + (S.wstart[j] & 0x7FFFFFFFu));
       }
       cp_async_commit();
-      if (threadIdx.x == 0) S.runk[buf] = nseg;
+      nrun = nseg;
       hint = sa + nseg - 1;
       return e_end - e0;
     }
   }
-  if (threadIdx.x == 0) S.runk[buf] = 0;
   const uint32_t m = min(min((uint32_t)STEP, total - e0), S.wcum[nwin] - e0);
   // Warp w gathers the slice [e0 + 32*RI*w, +32*RI) of the step.  Segment j holds
   // event e iff wcum[j] <= e < wcum[j+1]; every warp counts, from the hint, the
@@ -976,90 +1013,125 @@ __device__ __forceinline__ uint32_t byte_mask(uint32_t a, uint32_t n) {
 // that each group has one owner thread.  Every warp derives the run table and the
 // merged intervals itself (no block barrier).  BO (Z20): a target access to a word
 // without kCVp is a BO report and no transition; UM (Z23): a write makes 0xF.
+// One warp: the step's run table (segments that continue one another joined) and
+// the merged 4-word-group intervals, for the step's first `cut` events.
+__device__ void run_setup(RunStage& R, uint32_t nseg, uint32_t cut, uint32_t a3, uint32_t plo, uint32_t phi) {
+  const uint32_t lane = threadIdx.x & 31;
+  constexpr uint32_t kNone = 0xFFFFFFFFu;
+  uint32_t A = 0, B = 0, ga = kNone, gb = 0, op = 0, pos = 0;
+  uint32_t len = 0;
+  if (lane < nseg) {
+    const uint4 inf = R.info[lane];
+    const uint2 ds = R.desc[lane];
+    len = inf.z >= cut ? 0u : min(inf.y, cut - inf.z);
+    const uint32_t key = ds.x + inf.x;
+    op = key >> 30; pos = ds.y + inf.x;
+    A = a3 + (key & kWordMask); B = A + len;
+  }
+  // a segment that continues the previous one (a run cut at a chunk boundary: same
+  // op, next word, next position) joins it: runs = chains of segments
+  const uint32_t pA = __shfl_up_sync(FULL, B, 1), pop = __shfl_up_sync(FULL, op, 1);
+  const uint32_t ppe = __shfl_up_sync(FULL, pos + (B - A), 1);
+  const uint32_t lens = __ballot_sync(FULL, len != 0);
+  const bool cont = lane > 0 && len && ((lens >> (lane - 1)) & 1u) && pA == A && pop == op && ppe == pos;
+  const uint32_t heads = __ballot_sync(FULL, len && !cont);
+  // chain end: the lane before the next head or the next empty segment
+  const uint32_t after = (heads | ~lens) & (lane == 31 ? 0u : 0xFFFFFFFEu << lane);
+  const uint32_t endl = after ? __ffs(after) - 2 : 31u;
+  const uint32_t Bc = __shfl_sync(FULL, B, endl);
+  const uint32_t nr = __popc(heads);
+  if ((heads >> lane) & 1u) {                        // clipped to the work item's words [plo, phi)
+    const uint32_t Ac = max(A, plo), Be = min(Bc, phi);
+    R.run[__popc(heads & lanemask_lt())] = Ac < Be ? make_uint4(Ac, Be, op, pos + (Ac - A)) : make_uint4(0, 0, 0, 0);
+  }
+  R.mm[lane] = 0;
+  __syncwarp();
+  if (lane < nr) {
+    const uint4 r = R.run[lane];
+    if (r.y > r.x) { ga = r.x >> 2; gb = (r.y + 3) >> 2; }
+  }
+  // sort the group intervals by first group (bitonic over the lanes; empty ones last)
+  uint32_t sga = ga, sgb = gb, sr = lane;
+  const uint32_t kmax = nr <= 1 ? 1u : 1u << (32 - __clz(nr - 1));       // sorting network width
+#pragma unroll
+  for (uint32_t k = 2; k <= 32; k <<= 1) {
+    if (k > kmax) break;
+#pragma unroll
+    for (uint32_t j = k >> 1; j > 0; j >>= 1) {
+      const uint32_t oga = __shfl_xor_sync(FULL, sga, j), ogb = __shfl_xor_sync(FULL, sgb, j);
+      const uint32_t orr = __shfl_xor_sync(FULL, sr, j);
+      const bool keep_min = ((lane & j) == 0) == ((lane & k) == 0 || k == kmax);
+      if (keep_min ? oga < sga : oga > sga) { sga = oga; sgb = ogb; sr = orr; }
+    }
+  }
+  const bool valid = sga != kNone;
+  uint32_t incl = valid ? sgb : 0u;                  // inclusive prefix max of the interval ends
+#pragma unroll
+  for (uint32_t d = 1; d < 32; d <<= 1) {
+    const uint32_t o = __shfl_up_sync(FULL, incl, d);
+    if (lane >= d) incl = max(incl, o);
+  }
+  uint32_t excl = __shfl_up_sync(FULL, incl, 1);
+  if (lane == 0) excl = 0;
+  const bool start = valid && (lane == 0 || sga >= excl);
+  const uint32_t smask = __ballot_sync(FULL, start), vmask = __ballot_sync(FULL, valid);
+  const uint32_t nm = __popc(smask);
+  const uint32_t idx = __popc(smask & (0xFFFFFFFFu >> (31 - lane))) - 1u;   // merged interval of this lane
+  const bool lastl = valid && (lane == 31 || !((vmask >> (lane + 1)) & 1u) || ((smask >> (lane + 1)) & 1u));
+  __syncwarp();
+  if (valid) atomicOr(&R.mm[idx], 1u << sr);
+  if (start) R.mi[idx].x = sga;
+  if (lastl) R.mi[idx].y = incl;                     // the interval's end (exclusive group)
+  __syncwarp();
+  uint32_t n = 0, gs = 0;
+  if (lane < nm) { const uint2 v = R.mi[lane]; gs = v.x; n = v.y - v.x; }
+  uint32_t sc = n;
+#pragma unroll
+  for (uint32_t d = 1; d < 32; d <<= 1) {
+    const uint32_t o = __shfl_up_sync(FULL, sc, d);
+    if (lane >= d) sc += o;
+  }
+  __syncwarp();
+  if (lane < nm) R.mi[lane] = make_uint2(gs, sc - n);
+  if (lane == 31) { R.nm = nm; R.G = sc; }
+  __syncwarp();
+}
+
+// A step made only of runs (each: word A + j, op, position + j for j < count).  No
+// event is materialised: the shadow is processed in aligned groups of 4 words (one
+// 32-bit load per group, 4 states in SWAR form), and each group applies, in trace
+// order, every run that overlaps it — reads classify the covered bytes (P:263:
+// read_host needs OVv, read_target CVv; UUM / USD by the init bits), writes
+// take the VSM write image (WH: OVv, OVi set, CVv clear; WT: CVv, CVi set, OVv
+// clear).  Groups are the union of the runs' group intervals, merged so
+// that each group has one owner thread.  BO (Z20): a target access to a word
+// without kCVp is a BO report and no transition; UM (Z23): a write makes 0xF.
+// The table is built by run_setup (warp 0, usually during the previous step:
+// `prepared`, a block-uniform register — not a shared flag, which warp 0 would set
+// while other warps still test it); warps 1.. process the groups while warp 0
+// builds the next run step's table (Rn, nsn segments of mn events; nsn = 0: the
+// next step is not a run step).
 template <bool BO, bool UM>
-__device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uint32_t nseg, uint32_t cut) {
+__device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uint32_t nseg, uint32_t cut,
+                          bool prepared, RunStage& Rn, uint32_t nsn, uint32_t mn) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint64_t bb = S.bucket_base;
   const uint32_t a3 = (uint32_t)bb & 3u;
   uint32_t* const gbase = reinterpret_cast<uint32_t*>(p.shadow + (bb - a3));
-  const uint32_t wlo = a3, whi = a3 + S.span;      // the bucket's words in A-coordinates
-  if (warp == 0) {                                  // the run table and the merged group intervals
-    constexpr uint32_t kNone = 0xFFFFFFFFu;
-    uint32_t A = 0, B = 0, ga = kNone, gb = 0, op = 0, pos = 0;
-    uint32_t len = 0;
-    if (lane < nseg) {
-      const uint4 inf = R.info[lane];
-      const uint2 ds = R.desc[lane];
-      len = inf.z >= cut ? 0u : min(inf.y, cut - inf.z);
-      const uint32_t key = ds.x + inf.x;
-      op = key >> 30; pos = ds.y + inf.x;
-      A = a3 + (key & kWordMask); B = A + len;
-    }
-    // a segment that continues the previous one (a run cut at a chunk boundary: same
-    // op, next word, next position) joins it: runs = chains of segments
-    const uint32_t pA = __shfl_up_sync(FULL, B, 1), pop = __shfl_up_sync(FULL, op, 1);
-    const uint32_t ppe = __shfl_up_sync(FULL, pos + (B - A), 1);
-    const uint32_t lens = __ballot_sync(FULL, len != 0);
-    const bool cont = lane > 0 && len && ((lens >> (lane - 1)) & 1u) && pA == A && pop == op && ppe == pos;
-    const uint32_t heads = __ballot_sync(FULL, len && !cont);
-    // chain end: the lane before the next head or the next empty segment
-    const uint32_t after = (heads | ~lens) & (lane == 31 ? 0u : 0xFFFFFFFEu << lane);
-    const uint32_t endl = after ? __ffs(after) - 2 : 31u;
-    const uint32_t Bc = __shfl_sync(FULL, B, endl);
-    const uint32_t nr = __popc(heads);
-    if ((heads >> lane) & 1u) R.run[__popc(heads & lanemask_lt())] = make_uint4(A, Bc, op, pos);
-    R.mm[lane] = 0;
-    __syncwarp();
-    if (lane < nr) {
-      const uint4 r = R.run[lane];
-      ga = r.x >> 2; gb = (r.y + 3) >> 2;
-    }
-    // sort the group intervals by first group (bitonic over the lanes; empty ones last)
-    uint32_t sga = ga, sgb = gb, sr = lane;
-    const uint32_t kmax = nr <= 1 ? 1u : 1u << (32 - __clz(nr - 1));       // sorting network width
-#pragma unroll
-    for (uint32_t k = 2; k <= 32; k <<= 1) {
-      if (k > kmax) break;
-#pragma unroll
-      for (uint32_t j = k >> 1; j > 0; j >>= 1) {
-        const uint32_t oga = __shfl_xor_sync(FULL, sga, j), ogb = __shfl_xor_sync(FULL, sgb, j);
-        const uint32_t orr = __shfl_xor_sync(FULL, sr, j);
-        const bool keep_min = ((lane & j) == 0) == ((lane & k) == 0 || k == kmax);
-        if (keep_min ? oga < sga : oga > sga) { sga = oga; sgb = ogb; sr = orr; }
-      }
-    }
-    const bool valid = sga != kNone;
-    uint32_t incl = valid ? sgb : 0u;                // inclusive prefix max of the interval ends
-#pragma unroll
-    for (uint32_t d = 1; d < 32; d <<= 1) {
-      const uint32_t o = __shfl_up_sync(FULL, incl, d);
-      if (lane >= d) incl = max(incl, o);
-    }
-    uint32_t excl = __shfl_up_sync(FULL, incl, 1);
-    if (lane == 0) excl = 0;
-    const bool start = valid && (lane == 0 || sga >= excl);
-    const uint32_t smask = __ballot_sync(FULL, start), vmask = __ballot_sync(FULL, valid);
-    const uint32_t nm = __popc(smask);
-    const uint32_t idx = __popc(smask & (0xFFFFFFFFu >> (31 - lane))) - 1u;   // merged interval of this lane
-    const bool lastl = valid && (lane == 31 || !((vmask >> (lane + 1)) & 1u) || ((smask >> (lane + 1)) & 1u));
-    __syncwarp();
-    if (valid) atomicOr(&R.mm[idx], 1u << sr);
-    if (start) R.mi[idx].x = sga;
-    if (lastl) R.mi[idx].y = incl;                   // the interval's end (exclusive group)
-    __syncwarp();
-    uint32_t n = 0, gs = 0;
-    if (lane < nm) { const uint2 v = R.mi[lane]; gs = v.x; n = v.y - v.x; }
-    uint32_t sc = n;
-#pragma unroll
-    for (uint32_t d = 1; d < 32; d <<= 1) {
-      const uint32_t o = __shfl_up_sync(FULL, sc, d);
-      if (lane >= d) sc += o;
-    }
-    __syncwarp();
-    if (lane < nm) R.mi[lane] = make_uint2(gs, sc - n);
-    if (lane == 31) { R.nm = nm; R.G = sc; }
+  // the work item's words in A-coordinates: the bucket, or a part of it (kItemPart)
+  const uint32_t wlo = a3 + (S.partial ? S.part_lo : 0u), whi = a3 + (S.partial ? S.part_hi : S.span);
+  if (!prepared) {                                  // first run step of a stretch, or cut by a range op
+    if (warp == 0) run_setup(R, nseg, cut, a3, wlo, whi);
+    __syncthreads();
   }
-  __syncthreads();
+  if (warp == 0) {
+    if (nsn) {                                      // the next step's table, overlapped with this step
+      cp_async_wait_all();                          // its descriptors (copied by warp 0)
+      __syncwarp();
+      run_setup(Rn, nsn, mn, a3, wlo, whi);
+    }
+    return;
+  }
   const uint32_t nm = R.nm, G = R.G;
   const uint64_t wbase = bb - a3;                    // relative word of A = 0
   // a run's reports in one group, packed: run index (bits 0-4), faulting bytes
@@ -1077,14 +1149,14 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
       ++base;
     }
   };
-  for (uint32_t u0 = 0; u0 < G; u0 += RT) {
-    const uint32_t u = u0 + threadIdx.x;
+  const uint32_t st0 = nm <= 1 ? 0u : 1u << (31 - __clz(nm - 1));   // search span (nm is uniform)
+  for (uint32_t u0 = 0; u0 < G; u0 += RT - 32) {
+    const uint32_t u = u0 + threadIdx.x - 32;
     uint32_t ns = 0, fs0 = 0, fs1 = 0;
     uint32_t w0 = 0;
     if (u < G) {
       uint32_t j = 0;                                 // merged interval: the last with first unit <= u
-#pragma unroll
-      for (uint32_t st = 16; st; st >>= 1)
+      for (uint32_t st = st0; st; st >>= 1)
         if (j + st < nm && R.mi[j + st].y <= u) j += st;
       const uint2 mv = R.mi[j];
       const uint32_t g = mv.x + (u - mv.y);
@@ -1223,11 +1295,13 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
     }
     if (tid == 0) S.next_op = S.op_cur < S.op_end ? p.ops[S.op_cur].pos : 0xFFFFFFFFu;
     __syncthreads();
-    uint32_t e0 = first, cur = 0, m_cur = 0, hint = 0;
-    const bool runs_ok = !MD && mode == kItemWhole && !p.no_run_steps;   // run steps: whole buckets, one device
+    uint32_t e0 = first, cur = 0, m_cur = 0, hint = 0, nr_cur = 0;
+    bool prep_cur = false;                   // the current run step's table was built during the last step
+    // run steps: whole buckets or word-range parts, one device
+    const bool runs_ok = !MD && (mode == kItemWhole || mode == kItemPart) && !p.no_run_steps;
     if (e0 < total) {
       ensure_window(S, p, e0, hint);
-      m_cur = issue_gather(S, p, e0, total, 0, hint, runs_ok);
+      m_cur = issue_gather(S, p, e0, total, 0, hint, runs_ok, nr_cur);
     }
     while (e0 < total) {
       cp_async_wait_all();
@@ -1236,14 +1310,14 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       const uint32_t m = m_cur;
       // ---- prefetch the next step's events (assumes the step is not cut) ---------
       const uint32_t nxt = e0 + m;
-      uint32_t m_nxt = 0;
+      uint32_t m_nxt = 0, nr_nxt = 0;
       if (nxt < total) {
         ensure_window(S, p, nxt, hint);
-        m_nxt = issue_gather(S, p, nxt, total, cur ^ 1, hint, runs_ok);
+        m_nxt = issue_gather(S, p, nxt, total, cur ^ 1, hint, runs_ok, nr_nxt);
       }
       // ---- range ops before the first event, then cut at the next one -------------
       constexpr uint32_t pm = MD ? kMdPos : 0xFFFFFFFFu;   // MD: strip the device bits (Z24)
-      const uint32_t nrs = MD ? 0u : S.runk[cur];
+      const uint32_t nrs = MD ? 0u : nr_cur;
       RunStage& R = *reinterpret_cast<RunStage*>(S.ev[cur]);
       uint32_t cut = m;
       if (nrs) {                                   // run step: positions from the descriptors
@@ -1269,11 +1343,16 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         }
       }
       if (nrs) {
-        if (cut) step_runs<BO, UM>(S, p, R, nrs, cut);
+        const bool nx_run = nr_nxt != 0 && cut == m && !p.no_run_prep;
+        step_runs<BO, UM>(S, p, R, nrs, cut, prep_cur && cut == m, *reinterpret_cast<RunStage*>(S.ev[cur ^ 1]),
+                          nx_run ? nr_nxt : 0u, m_nxt);
+        prep_cur = nx_run;
         if (tid == 0) atomicAdd(&p.st->steps_run, 1ull);
       } else if (mode == kItemSummary) {
+        prep_cur = false;
         step_summary<BO, UM, MD>(S, ev, cut);
       } else {
+        prep_cur = false;
         const bool fast = S.partial ? step_fast_partial<BO, UM, MD>(S, p, ev, cut)
                                     : step_fast<false, BO, UM, MD>(S, p, ev, cut);
         if (!fast) step_sort<BO, UM, MD>(S, p, ev, cut);
@@ -1283,13 +1362,15 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
       if (cut == m) {
         cur ^= 1;
         m_cur = m_nxt;
+        nr_cur = nr_nxt;
       } else {
         // the prefetch started at e0_old + m: drain it and gather from e0
         cp_async_wait_all();
         __syncthreads();
         hint = 0;
+        prep_cur = false;
         ensure_window(S, p, e0, hint);
-        m_cur = issue_gather(S, p, e0, total, cur, hint, runs_ok);
+        m_cur = issue_gather(S, p, e0, total, cur, hint, runs_ok, nr_cur);
       }
     }
     // the ops after the last event (a slice replay's private states are not kept);

@@ -669,8 +669,28 @@ def test_runs_fuzz(orc, seed):
     flags = [0, 8, 16][seed % 3]
     runs = 0
     for bb in (0, 9, 12):
-        _, st = check(orc, rec, base, span, bucket_bits=bb, flags=flags)
+        exp, st = check(orc, rec, base, span, bucket_bits=bb, flags=flags)
         runs += st["steps_run"]
     assert runs > 0
     cuts = sorted(int(x) for x in np.random.default_rng(seed).choice(rec.shape[0], 3, replace=False))
-    check(orc, rec, base, span, flags=flags, flush_points=cuts)
+    rc, got, shadow, st = run_gpu(rec, base, span, flags=flags, bucket_bits=9, flush_points=cuts)
+    assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+@pytest.mark.parametrize("seed", [3000, 3001, 3002, 3004, 3005, 3006])   # well-formed programs (rc 0)
+def test_runs_fuzz_large(orc, seed):
+    """Traces of more chunks than the partition has warps, so that runs continue
+    from a warp's chunk into its next one (one entry per run), with
+    range ops, tasks and flush cuts; the BO and UM instances."""
+    from gen.fuzz import run_program
+    rec, base, span = run_program(seed, n_arrays=8, array_words=1 << 16, steps=500, loop_max=40000)
+    assert rec.shape[0] > 2 * 148 * 16 * 256 and orc.replay(rec, base, span).rc == 0
+    flags = [0, 8, 16][seed % 3]
+    for bb in (0, 12, 15):
+        exp, st = check(orc, rec, base, span, bucket_bits=bb, flags=flags)
+        # automatic buckets are narrower than the runs here; 2^15-word buckets are few
+        # and heavy, so they are replayed as K5 time slices (event steps)
+        assert st["steps_run"] > 0 or bb != 12
+    cuts = sorted(int(x) for x in np.random.default_rng(seed).choice(rec.shape[0], 4, replace=False))
+    rc, got, shadow, st = run_gpu(rec, base, span, flags=flags, flush_points=cuts)
+    assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
