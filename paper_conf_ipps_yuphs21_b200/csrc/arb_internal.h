@@ -88,6 +88,10 @@ constexpr int kReplayItems = 4;
 constexpr int kStep = kReplayThreads * kReplayItems;  // events per step
 constexpr int kReplayCtasPerSm = 4;
 constexpr int kReplayHashBits = 12;                  // fast-step hash: 2^12 slots
+#ifndef ARB_RUN_GROUPS_IN_FLIGHT
+#define ARB_RUN_GROUPS_IN_FLIGHT 1
+#endif
+constexpr uint32_t kRunGroupsInFlight = ARB_RUN_GROUPS_IN_FLIGHT;   // run step: shadow loads per thread issued together
 
 // replay work items {bucket, y, z, kind}
 constexpr uint32_t kItemWhole = 0;      // the whole bucket

@@ -1150,18 +1150,33 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
     }
   };
   const uint32_t st0 = nm <= 1 ? 0u : 1u << (31 - __clz(nm - 1));   // search span (nm is uniform)
-  for (uint32_t u0 = 0; u0 < G; u0 += RT - 32) {
-    const uint32_t u = u0 + threadIdx.x - 32;
-    uint32_t ns = 0, fs0 = 0, fs1 = 0;
-    uint32_t w0 = 0;
+  constexpr uint32_t GU = kRunGroupsInFlight;      // groups per thread whose loads are issued together
+  constexpr uint32_t GT = RT - 32;                  // group threads (warps 1..)
+  for (uint32_t u00 = 0; u00 < G; u00 += GU * GT) {
+  uint32_t gq[GU], jq[GU], sq[GU];
+#pragma unroll
+  for (uint32_t q = 0; q < GU; ++q) {
+    const uint32_t u = u00 + q * GT + threadIdx.x - 32;
+    gq[q] = 0; jq[q] = 0; sq[q] = 0;
     if (u < G) {
       uint32_t j = 0;                                 // merged interval: the last with first unit <= u
       for (uint32_t st = st0; st; st >>= 1)
         if (j + st < nm && R.mi[j + st].y <= u) j += st;
       const uint2 mv = R.mi[j];
-      const uint32_t g = mv.x + (u - mv.y);
+      gq[q] = mv.x + (u - mv.y);
+      jq[q] = j;
+      sq[q] = __ldcg(gbase + gq[q]);
+    }
+  }
+#pragma unroll
+  for (uint32_t q = 0; q < GU; ++q) {
+    const uint32_t u = u00 + q * GT + threadIdx.x - 32;
+    uint32_t ns = 0, fs0 = 0, fs1 = 0;
+    uint32_t w0 = 0;
+    if (u < G) {
+      const uint32_t j = jq[q], g = gq[q];
       w0 = 4 * g;
-      uint32_t s = __ldcg(gbase + g);
+      uint32_t s = sq[q];
       uint32_t wr = 0;
       for (uint32_t mm = R.mm[j]; mm; mm &= mm - 1) {
         const uint32_t ri = __ffs(mm) - 1;
@@ -1226,6 +1241,7 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
       if (ns > 0) emit_one(fs0, w0, base);
       if (ns > 1) emit_one(fs1, w0, base + __popc((fs0 >> 5) & 15u));
     }
+  }
   }
 }
 
