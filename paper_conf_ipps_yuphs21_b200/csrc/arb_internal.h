@@ -146,7 +146,7 @@ struct RangeRef { uint64_t lo, hi; uint32_t pos; uint32_t inst; };
 // so one lookup gives both the bucket and the word offset inside it.  The map
 // is balanced on a sampled histogram of the batch's access addresses.
 #ifndef ARB_COARSE_BINS_LOG2
-#define ARB_COARSE_BINS_LOG2 18
+#define ARB_COARSE_BINS_LOG2 19
 #endif
 constexpr int kMaxCoarseBins = 1 << ARB_COARSE_BINS_LOG2;
 constexpr uint32_t kSampleCap = 1u << 20;

@@ -1343,7 +1343,7 @@ __global__ void __launch_bounds__(RT, kReplayCtasPerSm) k_replay(ReplayParams p)
         if (nx != 0xFFFFFFFFu && R.desc[nrs - 1].y + li.x + li.y - 1 > nx) {
           const uint32_t lane = tid & 31;
           uint32_t c = 0;
-          if (lane < nrs) {
+          if (!MD && lane < nrs) {
             const uint4 in = R.info[lane];
             const uint32_t p0 = R.desc[lane].y + in.x;
             c = p0 + in.y <= nx ? in.y : (p0 < nx ? nx - p0 : 0u);
