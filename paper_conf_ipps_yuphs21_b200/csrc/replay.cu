@@ -51,6 +51,8 @@ struct RunStage {
   uint2 desc[kMaxStepRuns];                  // the runs' descriptors {key, position} (cp.async)
   uint4 run[kMaxStepRuns];                   // {A, B, op, position of word A} (A, B: words from the
                                              //   4-aligned word below the bucket's first word)
+  uint4 cmp[kMaxStepRuns];                   // compounds: adjacent runs on identical words {A, B, first
+                                             //   run | runs << 5, their ops (2 bits each, trace order)}
   uint2 mi[kMaxStepRuns];                    // merged 4-word-group intervals {first group, first unit}
   uint32_t mm[kMaxStepRuns];                 // the runs overlapping merged interval j
   uint32_t nm, G;                            // merged intervals, groups
@@ -1046,13 +1048,37 @@ __device__ void run_setup(RunStage& R, uint32_t nseg, uint32_t cut, uint32_t a3,
   }
   R.mm[lane] = 0;
   __syncwarp();
-  if (lane < nr) {
-    const uint4 r = R.run[lane];
-    if (r.y > r.x) { ga = r.x >> 2; gb = (r.y + 3) >> 2; }
+  // compounds: adjacent runs on identical words (config 5's WT, RT, RT of one run of
+  // words) — the group pass computes their overlap once and applies their ops in order
+  uint4 r = make_uint4(0, 0, 0, 0);
+  if (lane < nr) r = R.run[lane];
+  const bool ne = lane < nr && r.y > r.x;
+  const uint32_t pX = __shfl_up_sync(FULL, r.x, 1), pY = __shfl_up_sync(FULL, r.y, 1);
+  const bool same = lane > 0 && ne && pX == r.x && pY == r.y;
+  const uint32_t le = 0xFFFFFFFFu >> (31 - lane);
+  uint32_t cst = __ballot_sync(FULL, ne && !same);
+  uint32_t t = ne ? lane - (31 - __clz(cst & le)) : 0u;
+  cst |= __ballot_sync(FULL, ne && t >= 16 && (t & 15u) == 0);        // at most 16 ops per compound
+  const uint32_t cs = ne ? 31 - __clz(cst & le) : lane;
+  t = lane - cs;
+  uint32_t opsv = ne ? r.z << (2 * t) : 0u;                            // OR over the compound's members so far
+#pragma unroll
+  for (uint32_t d = 1; d < 32; d <<= 1) {
+    const uint32_t o = __shfl_up_sync(FULL, opsv, d);
+    if (lane >= d && lane - d >= cs) opsv |= o;
+  }
+  const uint32_t nxs = __shfl_down_sync(FULL, (uint32_t)same, 1);      // does the next lane continue the compound?
+  const bool tail = ne && (lane == 31 || !nxs || ((cst >> (lane + 1)) & 1u));
+  const uint32_t nc = __popc(cst);
+  if (tail) R.cmp[__popc(cst & le) - 1] = make_uint4(r.x, r.y, cs | ((t + 1) << 5), opsv);
+  __syncwarp();
+  if (lane < nc) {
+    const uint4 c = R.cmp[lane];
+    ga = c.x >> 2; gb = (c.y + 3) >> 2;
   }
   // sort the group intervals by first group (bitonic over the lanes; empty ones last)
   uint32_t sga = ga, sgb = gb, sr = lane;
-  const uint32_t kmax = nr <= 1 ? 1u : 1u << (32 - __clz(nr - 1));       // sorting network width
+  const uint32_t kmax = nc <= 1 ? 1u : 1u << (32 - __clz(nc - 1));       // sorting network width
 #pragma unroll
   for (uint32_t k = 2; k <= 32; k <<= 1) {
     if (k > kmax) break;
@@ -1179,12 +1205,14 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
       uint32_t s = sq[q];
       uint32_t wr = 0;
       for (uint32_t mm = R.mm[j]; mm; mm &= mm - 1) {
-        const uint32_t ri = __ffs(mm) - 1;
-        const uint4 r = R.run[ri];
-        const uint32_t lo = max(r.x, w0), hi = min(r.y, w0 + 4);
+        const uint4 cp = R.cmp[__ffs(mm) - 1];
+        const uint32_t lo = max(cp.x, w0), hi = min(cp.y, w0 + 4);
         if (lo >= hi) continue;
         const uint32_t M = byte_mask(lo - w0, hi - lo);
-        const uint32_t o = r.z;
+        const uint32_t r0 = cp.z & 31u, kn = cp.z >> 5;
+        for (uint32_t t = 0; t < kn; ++t) {
+        const uint32_t ri = r0 + t;
+        const uint32_t o = (cp.w >> (2 * t)) & 3u;
         uint32_t Me = M, bof = 0;
         if (BO && (o & 2u)) {                         // no CV: buffer overflow, no transition (Z20)
           bof = (~s >> 4) & 0x01010101u & M;
@@ -1213,6 +1241,7 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
           else if (ns == 1) fs1 = slot;
           else emit_one(slot, w0, atomicAdd(&p.st->n_cand, (unsigned long long)__popc((slot >> 5) & 15u)));
           ++ns;
+        }
         }
       }
       if (wr) {
