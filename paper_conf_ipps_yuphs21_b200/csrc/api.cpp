@@ -623,6 +623,8 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
       pp.n_dev = 1u + ((ctx->cfg.flags >> ARB_F_DEVICES_SHIFT) & 3u);
       pp.part_ev = ctx->part_ev.p; pp.seg_out = ctx->seg_a.p; pp.seg_cap = ctx->seg_cap;
       pp.no_runs = getenv("ARB_NO_RUNS") != nullptr;
+      pp.grid = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>((n_chunks + kPartWarps - 1) / kPartWarps,
+                                                                   (uint64_t)ctx->n_sms));
       pp.ctl = ctx->ctl.p; pp.ctl_cap = ctx->ctl_cap;
       pp.st = ctx->dstats.p;
       CK(launch_partition(pp, s), "k_partition");
@@ -658,9 +660,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
       CK(ctx->segs.ensure(std::max<uint64_t>(ns, 1)), "alloc segments");
       CK(ctx->seg_first.ensure(ctx->n_buckets + 1), "alloc seg_first");
       CK(ctx->blk.ensure((ns + 4095) / 4096 * 2049 + 4096), "alloc blk");   // 2048-bin digit counters + scan scratch
-      int cb = 1;
-      while (cb < 22 && ((uint64_t)n_chunks >> cb)) ++cb;
-      CK(launch_sort_segments(ctx->seg_a.p, ctx->seg_b.p, ns, cb, ctx->n_buckets, ctx->blk.p, ctx->seg_first.p,
+      CK(launch_sort_segments(ctx->seg_a.p, ctx->seg_b.p, ns, n_chunks, ctx->n_buckets, ctx->blk.p, ctx->seg_first.p,
                               ctx->segs.p, s, &launches), "sort segments");
       if (timing) cudaEventRecord(ctx->ev[8], s);
     }

@@ -71,6 +71,7 @@ constexpr int kSegChunkBits = 21;                    // chunk id bits in the ent
 // a run that continues into the warp's next chunk extends its entry (len < 2^15).
 constexpr uint32_t kRunFlag = 0x8000u;
 constexpr int kMaxChunkRuns = 16;
+constexpr uint32_t kChunkBlock = 16;          // partition work unit: consecutive chunks per ticket
 
 // ---- partition geometry ----------------------------------------------------
 constexpr int kPartThreads = 512;
@@ -119,6 +120,7 @@ struct DevStats {
   unsigned long long n_cv_acc;        // N1 (Z26): target accesses by CV address (left untracked)
   unsigned long long steps_run;      // replay steps made only of run segments
   unsigned long long chunks_run, chunks_fast;   // partition chunks written in run form / fast event form
+  unsigned long long part_ticket;       // partition work distribution (blocks of kChunkBlock chunks)
 };
 
 // control record extracted by the partition kernel
@@ -170,6 +172,7 @@ struct PartParams {
   DevStats* st;
   uint32_t n_dev;                         // accelerators (Z24): > 1 puts the device of RT/WT in pos bits 30-31
   uint32_t no_runs;                       // debug (ARB_NO_RUNS): never write the run form
+  uint32_t grid;                          // CTAs (persistent, <= one per SM)
 };
 
 struct ReplayParams {
@@ -233,7 +236,10 @@ cudaError_t launch_partition(const PartParams& p, cudaStream_t s);
 // by (bucket, chunk) (a, b: ping-pong buffers), writes the replay form
 // {chunk, bucket, start | len << 16, exclusive event prefix} to out and each
 // bucket's first entry; cnt: (n / 4096 + 1) * 256 + 4096 u32
-cudaError_t launch_sort_segments(uint2* a, uint2* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
+// The entries of one partition block (kChunkBlock consecutive chunks, one warp) are in
+// chunk order in the input, so a stable sort by (bucket, chunk / kChunkBlock) orders
+// them by (bucket, chunk); n_chunks: chunks of the batch
+cudaError_t launch_sort_segments(uint2* a, uint2* b, uint64_t n, uint64_t n_chunks, uint32_t n_buckets, uint32_t* cnt,
                                  uint32_t* first, uint4* out, cudaStream_t s, int* launches);
 cudaError_t launch_replay(const ReplayParams& p, int n_ctas, cudaStream_t s);
 // K5 phase 2: for every hot bucket {bucket, slices, span, 0} carry the states

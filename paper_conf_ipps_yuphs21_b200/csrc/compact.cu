@@ -6,7 +6,7 @@ namespace arb {
 
 constexpr int kRsThreads = 512, kRsItems = 8, kRsTile = kRsThreads * kRsItems;
 
-struct RsPass { int field; int shift; int bits; };
+struct RsPass { int field; int shift; int bits; uint32_t div = 1; };   // digit of field / div
 constexpr int kRsMaxBits = 11;                    // digits of up to 11 bits (2048 bins)
 constexpr int kRsBins = 1 << kRsMaxBits;
 // digit fields (64-bit): uint4 report candidates {x, y = word, z = record, w = kind}:
@@ -23,7 +23,9 @@ __device__ __forceinline__ uint64_t rs_field(uint2 c, int f) {
 }
 template <class E>
 __device__ __forceinline__ uint32_t rs_digit(E c, RsPass ps) {
-  return (uint32_t)(rs_field(c, ps.field) >> ps.shift) & ((1u << ps.bits) - 1u);
+  uint64_t v = rs_field(c, ps.field);
+  if (ps.div > 1) v /= ps.div;
+  return (uint32_t)(v >> ps.shift) & ((1u << ps.bits) - 1u);
 }
 
 // A block owns `sub` consecutive tiles of kRsTile elements (fewer, larger blocks
@@ -429,11 +431,22 @@ __global__ void __launch_bounds__(kRsThreads) k_seg_cum(const uint2* segs, uint6
   }
 }
 
-cudaError_t launch_sort_segments(uint2* a, uint2* b, uint64_t n, int chunk_bits, uint32_t n_buckets, uint32_t* cnt,
-                                 uint32_t* first, uint4* out, cudaStream_t s, int* launches) {
+cudaError_t launch_sort_segments(uint2* a, uint2* b, uint64_t n, uint64_t n_chunks, uint32_t n_buckets,
+                                 uint32_t* cnt, uint32_t* first, uint4* out, cudaStream_t s, int* launches) {
   RsPass ps[8];
   int np = 0;
-  np = add_field_passes(ps, np, 2, chunk_bits);                // the whole chunk id (<= 22 bits: 2 passes)
+  {
+    // the partition block of the chunk (chunk / kChunkBlock); within a block the input is in chunk order
+    const uint64_t nblocks = (n_chunks + kChunkBlock - 1) / kChunkBlock;
+    int bb = 1;
+    while ((1ull << bb) < nblocks) ++bb;
+    const int k = (bb + kRsMaxBits - 1) / kRsMaxBits;
+    for (int j = 0, sh = 0; j < k; ++j) {
+      const int w = (bb - sh + (k - j) - 1) / (k - j);
+      ps[np++] = RsPass{2, sh, w, kChunkBlock};
+      sh += w;
+    }
+  }
   {
     int nbb = 1;
     while ((1u << nbb) < n_buckets) ++nbb;                      // bucket bits actually used

@@ -353,14 +353,18 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
 
   // the chunk's records arrive in stage k by one TMA bulk copy (lane 0) that
   // completes on bar[k]
-  // the warp's chunks: a contiguous range (consecutive chunks let runs continue
-  // from one chunk into the next, OpenRun)
-  const uint64_t nwarps = (uint64_t)gridDim.x * PW;
-  const uint64_t cpw = (p.n_chunks + nwarps - 1) / nwarps;
-  const uint64_t c_begin = ((uint64_t)blockIdx.x * PW + warp) * cpw;
-  const uint64_t c_end = c_begin + cpw < p.n_chunks ? c_begin + cpw : p.n_chunks;
+  // The warp's chunks: blocks of kChunkBlock consecutive chunks taken from a ticket
+  // counter — consecutive chunks let runs continue from one chunk into the next
+  // (OpenRun), tickets balance the warps (general chunks cost ~10x a run chunk and
+  // cluster in parts of a trace).  The segment sort keys entries by block (chunk /
+  // kChunkBlock): a block's entries are in chunk order in the output.
+  auto take = [&]() -> uint64_t {
+    unsigned long long t = 0;
+    if (lane == 0) t = atomicAdd(&p.st->part_ticket, 1ull);
+    return (uint64_t)__shfl_sync(FULL, t, 0) * kChunkBlock;
+  };
   auto fetch = [&](uint64_t c, uint32_t k) {
-    if (c < c_end && lane == 0) {
+    if (c < p.n_chunks && lane == 0) {
       const uint64_t r0 = c * WREC;
       const uint32_t nv = p.n - r0 < (uint64_t)WREC ? (uint32_t)(p.n - r0) : (uint32_t)WREC;
       mbar_arrive_tx(bar + k, nv * 16u);
@@ -380,12 +384,22 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   OpenRun orun;
   orun.idx = kNoOpen; orun.op = orun.bkt = orun.len = 0; orun.next_word = 0;
 
+  static_assert(NST == 2, "prefetch distance 1 (the next chunk may start another block)");
   uint32_t cur = 0;
-  uint64_t chunk = c_begin;
-#pragma unroll
-  for (int k = 0; k < NST - 1; ++k) fetch(chunk + k, k);
-  for (; chunk < c_end; ++chunk) {
-    fetch(chunk + (NST - 1), cur == 0 ? NST - 1 : cur - 1);
+  uint64_t chunk = take();
+  uint64_t blk_end = chunk + kChunkBlock < p.n_chunks ? chunk + kChunkBlock : p.n_chunks;
+  uint64_t next_blk = take();
+  fetch(chunk, 0);
+  auto advance = [&]() -> uint64_t {           // the warp's next chunk
+    if (chunk + 1 < blk_end) return chunk + 1;
+    const uint64_t c = next_blk;
+    blk_end = c + kChunkBlock < p.n_chunks ? c + kChunkBlock : p.n_chunks;
+    next_blk = take();
+    orun.idx = kNoOpen;                        // not consecutive: no run continues into it
+    return c;
+  };
+  for (; chunk < p.n_chunks; chunk = advance()) {
+    fetch(chunk + 1 < blk_end ? chunk + 1 : next_blk, cur ^ 1u);
     mbar_wait(bar + cur, (phase >> cur) & 1u);
     phase ^= 1u << cur;
     const uint4* st = stage + cur * WREC;
@@ -594,12 +608,7 @@ cudaError_t launch_partition(const PartParams& p, cudaStream_t s) {
   auto kern = p.n_dev > 1 ? k_partition<true> : k_partition<false>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  int dev = 0, sms = 148;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const uint64_t ctas = (p.n_chunks + PW - 1) / PW;
-  const uint32_t grid = (uint32_t)std::min<uint64_t>(ctas, (uint64_t)sms);
-  kern<<<grid, PT, smem, s>>>(p);
+  kern<<<p.grid, PT, smem, s>>>(p);
   return cudaGetLastError();
 }
 
