@@ -218,7 +218,7 @@ class BatchSource:
 
 STAT_KEYS = ("access_words", "range_words", "reports", "records", "ms_partition", "ms_replay", "ms_mir",
              "ms_reports", "ms_control", "ms_total", "ms_sample", "ms_segsort", "ms_host_control", "steps_fast",
-             "steps_sort", "steps_run", "segments", "chunks", "chunks_fast", "chunks_run", "work_items", "hot_buckets", "kernel_launches", "exchanges")
+             "steps_sort", "steps_run", "segments", "chunks", "chunks_fast", "chunks_run", "run_merges", "work_items", "hot_buckets", "kernel_launches", "exchanges")
 
 
 def run_workload(prog, ctx, src, batches, steps, warmup, stream, world, dev, on_batch=None, clocks=None):
@@ -584,6 +584,7 @@ def main():
                                                                 int(s0["steps_run"])],
                            "segments_rank0": int(s0["segments"]),
                            "chunks_all_fast_run_rank0": [int(s0["chunks"]), int(s0["chunks_fast"]), int(s0["chunks_run"])],
+                           "run_merges_rank0": int(s0["run_merges"]),
                            "max_bucket_events_rank0": int(s0["max_bucket_events"]),
                            "replay_work_items_rank0": int(s0["work_items"]),
                            "hot_buckets_rank0": int(s0["hot_buckets"]),

@@ -187,6 +187,7 @@ typedef struct {
                                 stored-event segments)                                        */
   uint64_t chunks, chunks_fast, chunks_run;  /* partition chunks (256 records) of the last flush:
                                 all, on the fast path, written in run form                     */
+  uint64_t run_merges;       /* runs continued from the previous chunk (one entry for both)    */
 } arb_stats;
 
 typedef struct arb_ctx_s* arb_ctx;

@@ -59,7 +59,8 @@ class arb_stats(ctypes.Structure):
                 ("reports_bo", ctypes.c_uint64), ("nccl_ranks", ctypes.c_uint64),
                 ("exchanges", ctypes.c_uint64), ("steps_run", ctypes.c_uint64),
                 ("segments", ctypes.c_uint64), ("chunks", ctypes.c_uint64),
-                ("chunks_fast", ctypes.c_uint64), ("chunks_run", ctypes.c_uint64)]
+                ("chunks_fast", ctypes.c_uint64), ("chunks_run", ctypes.c_uint64),
+                ("run_merges", ctypes.c_uint64)]
 
     def as_dict(self):
         d = {}

@@ -525,7 +525,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   S.reports = 0; std::memset(S.reports_by_kind, 0, sizeof(S.reports_by_kind)); S.ignored_words = 0;
   S.ms_partition = S.ms_control = S.ms_replay = S.ms_mir = S.ms_reports = S.ms_total = 0;
   S.ms_segsort = S.ms_host_control = 0;
-  S.steps_run = S.segments = S.chunks = S.chunks_fast = S.chunks_run = 0;
+  S.steps_run = S.segments = S.chunks = S.chunks_fast = S.chunks_run = S.run_merges = 0;
   S.buckets = ctx->n_buckets; S.bucket_bits = ctx->bucket_bits; S.max_bucket_events = 0;
 
   // Phase A (validation): decode + partition and control resolution.  Nothing
@@ -795,6 +795,7 @@ extern "C" int arb_flush(arb_ctx ctx, void* stream, uint64_t* n_reports_local, u
   S.steps_run = hst.steps_run;
   S.segments = hst.n_segs;
   S.chunks = (n + kChunkRecords - 1) / kChunkRecords; S.chunks_fast = hst.chunks_fast; S.chunks_run = hst.chunks_run;
+  S.run_merges = hst.run_merges;
 
   // ---- A6: MIR join ---------------------------------------------------------------
   uint64_t n_mir = 0;

@@ -121,6 +121,7 @@ struct DevStats {
   unsigned long long steps_run;      // replay steps made only of run segments
   unsigned long long chunks_run, chunks_fast;   // partition chunks written in run form / fast event form
   unsigned long long part_ticket;       // partition work distribution (blocks of kChunkBlock chunks)
+  unsigned long long run_merges;        // runs continued from a warp's previous chunk (entry extended)
 };
 
 // control record extracted by the partition kernel

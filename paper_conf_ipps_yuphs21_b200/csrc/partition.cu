@@ -151,7 +151,7 @@ constexpr uint32_t kMaxRunLen = 0x7FFFu;      // events of a run entry (15-bit l
 template <bool MD>
 __device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p, uint32_t chunk, uint2* out,
                                            uint2* segbuf, uint32_t& nbuf, uint32_t lane, uint16_t* scratch,
-                                           OpenRun& orun) {
+                                           OpenRun& orun, uint32_t& n_merge) {
   const uint4 q0 = st[0];
   const uint64_t w0 = ((uint64_t)((q0.y & 0xFFFFu) >> 3) << 32) | __funnelshift_r(q0.x, q0.y, 3);
   const uint32_t x0w = __funnelshift_r(q0.x, q0.y, 3);        // record 0's word, low 32 bits
@@ -273,6 +273,7 @@ __device__ __forceinline__ bool fast_chunk(const uint4* st, const PartParams& p,
         orun.bkt = __shfl_sync(FULL, split ? bkt + 1 : bkt, L);
         orun.next_word = __shfl_sync(FULL, first + len, L);
         nbuf += nR + __popc(sp) - mg;
+        n_merge += mg;
         return true;
       }
     }
@@ -349,7 +350,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
   fence_mbar_init();
   __syncwarp();
   uint32_t n_acc = 0, n_ign = 0, n_cv = 0, nbuf = 0, phase = 0;   // phase: parity bit of each stage's barrier
-  uint32_t n_fast = 0, n_runc = 0;                                 // chunks: fast path / ending in an open run
+  uint32_t n_fast = 0, n_runc = 0, n_merge = 0;                    // chunks: fast path / ending in an open run
 
   // the chunk's records arrive in stage k by one TMA bulk copy (lane 0) that
   // completes on bar[k]
@@ -423,7 +424,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     }
     if (nvalid < WREC) orun.idx = kNoOpen;
     if (nvalid == WREC && fast_chunk<MD>(st, p, (uint32_t)chunk, p.part_ev + chunk * kChunkCap,
-                                     segbuf, nbuf, lane, tlist, orun)) {
+                                     segbuf, nbuf, lane, tlist, orun, n_merge)) {
       n_fast += 1u;
       n_runc += orun.idx != kNoOpen;
       n_acc += RPL;
@@ -599,6 +600,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
     if (n_cv) atomicAdd(&p.st->n_cv_acc, (unsigned long long)n_cv);
     if (n_fast) atomicAdd(&p.st->chunks_fast, (unsigned long long)n_fast);
     if (n_runc) atomicAdd(&p.st->chunks_run, (unsigned long long)n_runc);
+    if (n_merge) atomicAdd(&p.st->run_merges, (unsigned long long)n_merge);
   }
 }
 
