@@ -71,7 +71,10 @@ constexpr int kSegChunkBits = 21;                    // chunk id bits in the ent
 // a run that continues into the warp's next chunk extends its entry (len < 2^15).
 constexpr uint32_t kRunFlag = 0x8000u;
 constexpr int kMaxChunkRuns = 16;
-constexpr uint32_t kChunkBlock = 16;          // partition work unit: consecutive chunks per ticket
+#ifndef ARB_CHUNK_BLOCK
+#define ARB_CHUNK_BLOCK 64
+#endif
+constexpr uint32_t kChunkBlock = ARB_CHUNK_BLOCK;   // partition work unit: consecutive chunks per ticket
 
 // ---- partition geometry ----------------------------------------------------
 constexpr int kPartThreads = 512;

@@ -354,7 +354,7 @@ __global__ void __launch_bounds__(PT, 1) k_partition(PartParams p) {
 
   // the chunk's records arrive in stage k by one TMA bulk copy (lane 0) that
   // completes on bar[k]
-  // The warp's chunks: blocks of kChunkBlock consecutive chunks taken from a ticket
+  // The warp's chunks: blocks of kChunkBlock (64) consecutive chunks taken from a ticket
   // counter — consecutive chunks let runs continue from one chunk into the next
   // (OpenRun), tickets balance the warps (general chunks cost ~10x a run chunk and
   // cluster in parts of a trace).  The segment sort keys entries by block (chunk /
