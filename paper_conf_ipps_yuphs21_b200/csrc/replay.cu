@@ -26,6 +26,7 @@
 // (ARB_F_DEVICES, 8-bit states, Z24); the mode checks compile away in the others.
 #include "kcommon.cuh"
 #include <algorithm>
+#include <type_traits>
 
 namespace arb {
 
@@ -1001,8 +1002,20 @@ __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t 
 
 // ---- run step -------------------------------------------------------------------------
 // Byte mask of bytes [a, a + n) of a 32-bit group (n = 1..4)
-__device__ __forceinline__ uint32_t byte_mask(uint32_t a, uint32_t n) {
-  return (0xFFFFFFFFu >> (32 - 8 * n)) << (8 * a);
+// Run steps process the shadow in aligned groups of kGW words (kGW states in one
+// GWord, SWAR form): 4 words / 32 bits or 8 words / 64 bits (ARB_RUN_GROUP_WORDS).
+#ifndef ARB_RUN_GROUP_WORDS
+#define ARB_RUN_GROUP_WORDS 8
+#endif
+constexpr uint32_t kGW = ARB_RUN_GROUP_WORDS;
+constexpr uint32_t kGWLog = kGW == 8 ? 3 : 2;
+using GWord = std::conditional<kGW == 8, unsigned long long, uint32_t>::type;
+constexpr GWord kRep = kGW == 8 ? (GWord)0x0101010101010101ull : (GWord)0x01010101u;   // one bit per state byte
+static_assert(kGW == 4 || kGW == 8, "4- or 8-word groups");
+constexpr uint32_t kBytesM = (1u << kGW) - 1u;     // faulting-byte bits of a report slot
+// Byte mask of bytes [a, a + n) of a group (n = 1..kGW)
+__device__ __forceinline__ GWord byte_mask(uint32_t a, uint32_t n) {
+  return ((GWord)~(GWord)0 >> (8 * (kGW - n))) << (8 * a);
 }
 
 // A step made only of runs (each: word A + j, op, position + j for j < count).  No
@@ -1074,7 +1087,7 @@ __device__ void run_setup(RunStage& R, uint32_t nseg, uint32_t cut, uint32_t a3,
   __syncwarp();
   if (lane < nc) {
     const uint4 c = R.cmp[lane];
-    ga = c.x >> 2; gb = (c.y + 3) >> 2;
+    ga = c.x >> kGWLog; gb = (c.y + kGW - 1) >> kGWLog;
   }
   // sort the group intervals by first group (bitonic over the lanes; empty ones last)
   uint32_t sga = ga, sgb = gb, sr = lane;
@@ -1142,8 +1155,8 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
                           bool prepared, RunStage& Rn, uint32_t nsn, uint32_t mn) {
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint64_t bb = S.bucket_base;
-  const uint32_t a3 = (uint32_t)bb & 3u;
-  uint32_t* const gbase = reinterpret_cast<uint32_t*>(p.shadow + (bb - a3));
+  const uint32_t a3 = (uint32_t)bb & (kGW - 1);
+  GWord* const gbase = reinterpret_cast<GWord*>(p.shadow + (bb - a3));
   // the work item's words in A-coordinates: the bucket, or a part of it (kItemPart)
   const uint32_t wlo = a3 + (S.partial ? S.part_lo : 0u), whi = a3 + (S.partial ? S.part_hi : S.span);
   if (!prepared) {                                  // first run step of a stretch, or cut by a range op
@@ -1161,13 +1174,13 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
   const uint32_t nm = R.nm, G = R.G;
   const uint64_t wbase = bb - a3;                    // relative word of A = 0
   // a run's reports in one group, packed: run index (bits 0-4), faulting bytes
-  // (bits 5-8), 2 bits of kind per byte from bit 9 (0 UUM, 1 USD, 2 BO)
+  // (kGW bits from bit 5), 2 bits of kind per byte above them (0 UUM, 1 USD, 2 BO)
   auto emit_one = [&](uint32_t slot, uint32_t w0, unsigned long long base) {
     const uint4 r = R.run[slot & 31u];
 #pragma unroll
-    for (uint32_t b = 0; b < 4; ++b) {
+    for (uint32_t b = 0; b < kGW; ++b) {
       if (!((slot >> (5 + b)) & 1u)) continue;
-      const uint32_t kc = (slot >> (9 + 2 * b)) & 3u;
+      const uint32_t kc = (slot >> (5 + kGW + 2 * b)) & 3u;
       if (base < p.cand_cap) {
         const uint64_t wd = wbase + w0 + b;
         p.cand[base] = make_uint4((uint32_t)wd, (uint32_t)(wd >> 32), r.w + (w0 + b - r.x), kc == 2 ? 4u : kc + 1u);
@@ -1179,7 +1192,8 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
   constexpr uint32_t GU = kRunGroupsInFlight;      // groups per thread whose loads are issued together
   constexpr uint32_t GT = RT - 32;                  // group threads (warps 1..)
   for (uint32_t u00 = 0; u00 < G; u00 += GU * GT) {
-  uint32_t gq[GU], jq[GU], sq[GU];
+  uint32_t gq[GU], jq[GU];
+  GWord sq[GU];
 #pragma unroll
   for (uint32_t q = 0; q < GU; ++q) {
     const uint32_t u = u00 + q * GT + threadIdx.x - 32;
@@ -1201,62 +1215,62 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
     uint32_t w0 = 0;
     if (u < G) {
       const uint32_t j = jq[q], g = gq[q];
-      w0 = 4 * g;
-      uint32_t s = sq[q];
-      uint32_t wr = 0;
+      w0 = kGW * g;
+      GWord s = sq[q];
+      GWord wr = 0;
       for (uint32_t mm = R.mm[j]; mm; mm &= mm - 1) {
         const uint4 cp = R.cmp[__ffs(mm) - 1];
-        const uint32_t lo = max(cp.x, w0), hi = min(cp.y, w0 + 4);
+        const uint32_t lo = max(cp.x, w0), hi = min(cp.y, w0 + kGW);
         if (lo >= hi) continue;
-        const uint32_t M = byte_mask(lo - w0, hi - lo);
+        const GWord M = byte_mask(lo - w0, hi - lo);
         const uint32_t r0 = cp.z & 31u, kn = cp.z >> 5;
         for (uint32_t t = 0; t < kn; ++t) {
         const uint32_t ri = r0 + t;
         const uint32_t o = (cp.w >> (2 * t)) & 3u;
-        uint32_t Me = M, bof = 0;
+        GWord Me = M, bof = 0;
         if (BO && (o & 2u)) {                         // no CV: buffer overflow, no transition (Z20)
-          bof = (~s >> 4) & 0x01010101u & M;
+          bof = (~s >> 4) & kRep & M;
           Me = M & ~(bof * 0xFFu);
         }
-        uint32_t fv = 0;
+        GWord fv = 0;
         if (!(o & 1u)) {
-          fv = (~s >> (o >> 1)) & 0x01010101u & Me;   // RH: OVv (bit 0), RT: CVv (bit 1)
+          fv = (~s >> (o >> 1)) & kRep & Me;        // RH: OVv (bit 0), RT: CVv (bit 1)
         } else {
-          const uint32_t img = UM ? 0x0F0F0F0Fu
-                             : o == OP_WH ? ((s & (BO ? 0x18181818u : 0x08080808u)) | 0x05050505u)
-                                          : ((s & (BO ? 0x14141414u : 0x04040404u)) | 0x0A0A0A0Au);
+          const GWord img = UM ? kRep * 0x0Fu
+                       : o == OP_WH ? ((s & (kRep * (BO ? 0x18u : 0x08u))) | (kRep * 0x05u))
+                                    : ((s & (kRep * (BO ? 0x14u : 0x04u))) | (kRep * 0x0Au));
           s = (s & ~Me) | (img & Me);
           wr |= Me;
         }
         if (fv | bof) {                               // reports (rare)
-          const uint32_t usd = (s >> (2 + (o >> 1))) & 0x01010101u;   // the read side's init bit
+          const GWord usd = (s >> (2 + (o >> 1))) & kRep;   // the read side's init bit
           uint32_t slot = ri;
 #pragma unroll
-          for (uint32_t b = 0; b < 4; ++b) {
+          for (uint32_t b = 0; b < kGW; ++b) {
             if (!(((fv | bof) >> (8 * b)) & 1u)) continue;
-            const uint32_t kc = ((bof >> (8 * b)) & 1u) ? 2u : (usd >> (8 * b)) & 1u;
-            slot |= (1u << (5 + b)) | (kc << (9 + 2 * b));
+            const uint32_t kc = ((bof >> (8 * b)) & 1u) ? 2u : (uint32_t)(usd >> (8 * b)) & 1u;
+            slot |= (1u << (5 + b)) | (kc << (5 + kGW + 2 * b));
           }
           if (ns == 0) fs0 = slot;
           else if (ns == 1) fs1 = slot;
-          else emit_one(slot, w0, atomicAdd(&p.st->n_cand, (unsigned long long)__popc((slot >> 5) & 15u)));
+          else emit_one(slot, w0, atomicAdd(&p.st->n_cand, (unsigned long long)__popc((slot >> 5) & kBytesM)));
           ++ns;
         }
         }
       }
       if (wr) {
-        if (w0 >= wlo && w0 + 4 <= whi) {
+        if (w0 >= wlo && w0 + kGW <= whi) {
           __stcg(gbase + g, s);
         } else {                                      // a group shared with a neighbouring bucket
           uint8_t* gb8 = reinterpret_cast<uint8_t*>(gbase + g);
 #pragma unroll
-          for (uint32_t b = 0; b < 4; ++b)
+          for (uint32_t b = 0; b < kGW; ++b)
             if ((wr >> (8 * b)) & 0xFFu) __stcg(gb8 + b, (uint8_t)(s >> (8 * b)));
         }
       }
     }
     // the reports of each lane's first two faulting runs: one warp-aggregated append
-    const uint32_t k = (ns > 0 ? __popc((fs0 >> 5) & 15u) : 0u) + (ns > 1 ? __popc((fs1 >> 5) & 15u) : 0u);
+    const uint32_t k = (ns > 0 ? __popc((fs0 >> 5) & kBytesM) : 0u) + (ns > 1 ? __popc((fs1 >> 5) & kBytesM) : 0u);
     if (__any_sync(FULL, k != 0)) {
       uint32_t sk = k;
 #pragma unroll
@@ -1268,7 +1282,7 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
       if (lane == 31) base = atomicAdd(&p.st->n_cand, (unsigned long long)sk);
       base = __shfl_sync(FULL, base, 31) + (sk - k);
       if (ns > 0) emit_one(fs0, w0, base);
-      if (ns > 1) emit_one(fs1, w0, base + __popc((fs0 >> 5) & 15u));
+      if (ns > 1) emit_one(fs1, w0, base + __popc((fs0 >> 5) & kBytesM));
     }
   }
   }
