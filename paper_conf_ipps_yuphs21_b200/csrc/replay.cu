@@ -1003,20 +1003,60 @@ __device__ uint32_t issue_gather(ReplaySmem& S, const ReplayParams& p, uint32_t 
 // ---- run step -------------------------------------------------------------------------
 // Byte mask of bytes [a, a + n) of a 32-bit group (n = 1..4)
 // Run steps process the shadow in aligned groups of kGW words (kGW states in one
-// GWord, SWAR form): 4 words / 32 bits or 8 words / 64 bits (ARB_RUN_GROUP_WORDS).
+// GWord, SWAR form): 4 words / 32 bits, 8 words / 64 bits or 16 words / 2 x 64
+// bits (ARB_RUN_GROUP_WORDS).  The SWAR code only shifts right by < 8 bits before
+// masking one bit per byte, so the 128-bit form needs no carries between halves.
 #ifndef ARB_RUN_GROUP_WORDS
-#define ARB_RUN_GROUP_WORDS 8
+#define ARB_RUN_GROUP_WORDS 16
 #endif
 constexpr uint32_t kGW = ARB_RUN_GROUP_WORDS;
-constexpr uint32_t kGWLog = kGW == 8 ? 3 : 2;
-using GWord = std::conditional<kGW == 8, unsigned long long, uint32_t>::type;
-constexpr GWord kRep = kGW == 8 ? (GWord)0x0101010101010101ull : (GWord)0x01010101u;   // one bit per state byte
-static_assert(kGW == 4 || kGW == 8, "4- or 8-word groups");
+constexpr uint32_t kGWLog = kGW == 16 ? 4 : kGW == 8 ? 3 : 2;
+static_assert(kGW == 4 || kGW == 8 || kGW == 16, "4-, 8- or 16-word groups");
+struct W16 {
+  unsigned long long x, y;
+  __host__ __device__ constexpr W16(unsigned long long a = 0) : x(a), y(a) {}     // both halves
+  __host__ __device__ constexpr W16(unsigned long long a, unsigned long long b) : x(a), y(b) {}
+};
+__device__ __forceinline__ W16 operator&(W16 a, W16 b) { return W16(a.x & b.x, a.y & b.y); }
+__device__ __forceinline__ W16 operator|(W16 a, W16 b) { return W16(a.x | b.x, a.y | b.y); }
+__device__ __forceinline__ W16 operator~(W16 a) { return W16(~a.x, ~a.y); }
+__device__ __forceinline__ W16& operator|=(W16& a, W16 b) { a.x |= b.x; a.y |= b.y; return a; }
+__device__ __forceinline__ W16 operator>>(W16 a, uint32_t sh) { return W16(a.x >> sh, a.y >> sh); }  // sh < 8
+__device__ __forceinline__ W16 operator*(W16 a, uint32_t c) { return W16(a.x * c, a.y * c); }       // per byte
+using GWord = std::conditional<kGW == 16, W16, std::conditional<kGW == 8, unsigned long long, uint32_t>::type>::type;
+using Slot = std::conditional<kGW == 16, unsigned long long, uint32_t>::type;   // a report slot (below)
+constexpr GWord kRep = GWord(kGW == 4 ? 0x01010101ull : 0x0101010101010101ull);  // one bit per state byte
 constexpr uint32_t kBytesM = (1u << kGW) - 1u;     // faulting-byte bits of a report slot
+__device__ __forceinline__ bool any(uint32_t v) { return v != 0; }
+__device__ __forceinline__ bool any(unsigned long long v) { return v != 0; }
+__device__ __forceinline__ bool any(W16 v) { return (v.x | v.y) != 0; }
+__device__ __forceinline__ uint32_t byte_of(uint32_t v, uint32_t b) { return (v >> (8 * b)) & 0xFFu; }
+__device__ __forceinline__ uint32_t byte_of(unsigned long long v, uint32_t b) { return (uint32_t)(v >> (8 * b)) & 0xFFu; }
+__device__ __forceinline__ uint32_t byte_of(W16 v, uint32_t b) { return byte_of(b < 8 ? v.x : v.y, b & 7u); }
 // Byte mask of bytes [a, a + n) of a group (n = 1..kGW)
-__device__ __forceinline__ GWord byte_mask(uint32_t a, uint32_t n) {
-  return ((GWord)~(GWord)0 >> (8 * (kGW - n))) << (8 * a);
+__device__ __forceinline__ unsigned long long mask64(uint32_t a, uint32_t n) {   // a + n <= 8
+  return n == 0 ? 0ull : (~0ull >> (8 * (8 - n))) << (8 * a);
 }
+__device__ __forceinline__ uint32_t byte_mask_t(const uint32_t*, uint32_t a, uint32_t n) {
+  return (0xFFFFFFFFu >> (8 * (4 - n))) << (8 * a);
+}
+__device__ __forceinline__ unsigned long long byte_mask_t(const unsigned long long*, uint32_t a, uint32_t n) {
+  return mask64(a, n);
+}
+__device__ __forceinline__ W16 byte_mask_t(const W16*, uint32_t a, uint32_t n) {
+  const uint32_t e = a + n;
+  return W16(a < 8 ? mask64(a, min(e, 8u) - a) : 0ull, e > 8 ? mask64(a > 8 ? a - 8 : 0u, e - max(a, 8u)) : 0ull);
+}
+__device__ __forceinline__ GWord byte_mask(uint32_t a, uint32_t n) { return byte_mask_t((const GWord*)nullptr, a, n); }
+__device__ __forceinline__ uint32_t ld_group(const uint32_t* p) { return __ldcg(p); }
+__device__ __forceinline__ unsigned long long ld_group(const unsigned long long* p) { return __ldcg(p); }
+__device__ __forceinline__ W16 ld_group(const W16* p) {
+  const ulonglong2 v = __ldcg(reinterpret_cast<const ulonglong2*>(p));
+  return W16(v.x, v.y);
+}
+__device__ __forceinline__ void st_group(uint32_t* p, uint32_t v) { __stcg(p, v); }
+__device__ __forceinline__ void st_group(unsigned long long* p, unsigned long long v) { __stcg(p, v); }
+__device__ __forceinline__ void st_group(W16* p, W16 v) { __stcg(reinterpret_cast<ulonglong2*>(p), make_ulonglong2(v.x, v.y)); }
 
 // A step made only of runs (each: word A + j, op, position + j for j < count).  No
 // event is materialised: the shadow is processed in aligned groups of 4 words (one
@@ -1175,12 +1215,12 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
   const uint64_t wbase = bb - a3;                    // relative word of A = 0
   // a run's reports in one group, packed: run index (bits 0-4), faulting bytes
   // (kGW bits from bit 5), 2 bits of kind per byte above them (0 UUM, 1 USD, 2 BO)
-  auto emit_one = [&](uint32_t slot, uint32_t w0, unsigned long long base) {
-    const uint4 r = R.run[slot & 31u];
+  auto emit_one = [&](Slot slot, uint32_t w0, unsigned long long base) {
+    const uint4 r = R.run[(uint32_t)slot & 31u];
 #pragma unroll
     for (uint32_t b = 0; b < kGW; ++b) {
       if (!((slot >> (5 + b)) & 1u)) continue;
-      const uint32_t kc = (slot >> (5 + kGW + 2 * b)) & 3u;
+      const uint32_t kc = (uint32_t)(slot >> (5 + kGW + 2 * b)) & 3u;
       if (base < p.cand_cap) {
         const uint64_t wd = wbase + w0 + b;
         p.cand[base] = make_uint4((uint32_t)wd, (uint32_t)(wd >> 32), r.w + (w0 + b - r.x), kc == 2 ? 4u : kc + 1u);
@@ -1205,13 +1245,14 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
       const uint2 mv = R.mi[j];
       gq[q] = mv.x + (u - mv.y);
       jq[q] = j;
-      sq[q] = __ldcg(gbase + gq[q]);
+      sq[q] = ld_group(gbase + gq[q]);
     }
   }
 #pragma unroll
   for (uint32_t q = 0; q < GU; ++q) {
     const uint32_t u = u00 + q * GT + threadIdx.x - 32;
-    uint32_t ns = 0, fs0 = 0, fs1 = 0;
+    uint32_t ns = 0;
+    Slot fs0 = 0, fs1 = 0;
     uint32_t w0 = 0;
     if (u < G) {
       const uint32_t j = jq[q], g = gq[q];
@@ -1242,35 +1283,36 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
           s = (s & ~Me) | (img & Me);
           wr |= Me;
         }
-        if (fv | bof) {                               // reports (rare)
+        if (any(fv | bof)) {                          // reports (rare)
           const GWord usd = (s >> (2 + (o >> 1))) & kRep;   // the read side's init bit
-          uint32_t slot = ri;
+          Slot slot = ri;
 #pragma unroll
           for (uint32_t b = 0; b < kGW; ++b) {
-            if (!(((fv | bof) >> (8 * b)) & 1u)) continue;
-            const uint32_t kc = ((bof >> (8 * b)) & 1u) ? 2u : (uint32_t)(usd >> (8 * b)) & 1u;
-            slot |= (1u << (5 + b)) | (kc << (5 + kGW + 2 * b));
+            if (!(byte_of(fv | bof, b) & 1u)) continue;
+            const uint32_t kc = (byte_of(bof, b) & 1u) ? 2u : byte_of(usd, b) & 1u;
+            slot |= ((Slot)1 << (5 + b)) | ((Slot)kc << (5 + kGW + 2 * b));
           }
           if (ns == 0) fs0 = slot;
           else if (ns == 1) fs1 = slot;
-          else emit_one(slot, w0, atomicAdd(&p.st->n_cand, (unsigned long long)__popc((slot >> 5) & kBytesM)));
+          else emit_one(slot, w0, atomicAdd(&p.st->n_cand, (unsigned long long)__popc((uint32_t)(slot >> 5) & kBytesM)));
           ++ns;
         }
         }
       }
-      if (wr) {
+      if (any(wr)) {
         if (w0 >= wlo && w0 + kGW <= whi) {
-          __stcg(gbase + g, s);
+          st_group(gbase + g, s);
         } else {                                      // a group shared with a neighbouring bucket
           uint8_t* gb8 = reinterpret_cast<uint8_t*>(gbase + g);
 #pragma unroll
           for (uint32_t b = 0; b < kGW; ++b)
-            if ((wr >> (8 * b)) & 0xFFu) __stcg(gb8 + b, (uint8_t)(s >> (8 * b)));
+            if (byte_of(wr, b)) __stcg(gb8 + b, (uint8_t)byte_of(s, b));
         }
       }
     }
     // the reports of each lane's first two faulting runs: one warp-aggregated append
-    const uint32_t k = (ns > 0 ? __popc((fs0 >> 5) & kBytesM) : 0u) + (ns > 1 ? __popc((fs1 >> 5) & kBytesM) : 0u);
+    const uint32_t k = (ns > 0 ? __popc((uint32_t)(fs0 >> 5) & kBytesM) : 0u) +
+                       (ns > 1 ? __popc((uint32_t)(fs1 >> 5) & kBytesM) : 0u);
     if (__any_sync(FULL, k != 0)) {
       uint32_t sk = k;
 #pragma unroll
@@ -1282,7 +1324,7 @@ __device__ void step_runs(ReplaySmem& S, const ReplayParams& p, RunStage& R, uin
       if (lane == 31) base = atomicAdd(&p.st->n_cand, (unsigned long long)sk);
       base = __shfl_sync(FULL, base, 31) + (sk - k);
       if (ns > 0) emit_one(fs0, w0, base);
-      if (ns > 1) emit_one(fs1, w0, base + __popc((fs0 >> 5) & kBytesM));
+      if (ns > 1) emit_one(fs1, w0, base + __popc((uint32_t)(fs0 >> 5) & kBytesM));
     }
   }
   }
