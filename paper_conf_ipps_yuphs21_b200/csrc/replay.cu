@@ -54,7 +54,7 @@ struct RunStage {
                                              //   4-aligned word below the bucket's first word)
   uint4 cmp[kMaxStepRuns];                   // compounds: adjacent runs on identical words {A, B, first
                                              //   run | runs << 5, their ops (2 bits each, trace order)}
-  uint2 mi[kMaxStepRuns];                    // merged 4-word-group intervals {first group, first unit}
+  uint2 mi[kMaxStepRuns];                    // merged group intervals {first group, first unit}
   uint32_t mm[kMaxStepRuns];                 // the runs overlapping merged interval j
   uint32_t nm, G;                            // merged intervals, groups
 };
@@ -1058,18 +1058,9 @@ __device__ __forceinline__ void st_group(uint32_t* p, uint32_t v) { __stcg(p, v)
 __device__ __forceinline__ void st_group(unsigned long long* p, unsigned long long v) { __stcg(p, v); }
 __device__ __forceinline__ void st_group(W16* p, W16 v) { __stcg(reinterpret_cast<ulonglong2*>(p), make_ulonglong2(v.x, v.y)); }
 
-// A step made only of runs (each: word A + j, op, position + j for j < count).  No
-// event is materialised: the shadow is processed in aligned groups of 4 words (one
-// 32-bit load per group, 4 states in SWAR form), and each group applies, in trace
-// order, every run that overlaps it — reads classify the covered bytes (P:263:
-// read_host needs OVv, read_target CVv; UUM / USD by the init bits), writes
-// take the VSM write image (WH: OVv, OVi set, CVv clear; WT: CVv, CVi set, OVv
-// clear).  Groups are the union of the runs' group intervals, merged so
-// that each group has one owner thread.  Every warp derives the run table and the
-// merged intervals itself (no block barrier).  BO (Z20): a target access to a word
-// without kCVp is a BO report and no transition; UM (Z23): a write makes 0xF.
-// One warp: the step's run table (segments that continue one another joined) and
-// the merged 4-word-group intervals, for the step's first `cut` events.
+// One warp: the step's run table (segments that continue one another joined,
+// adjacent runs on identical words grouped into compounds) and the merged
+// kGW-word-group intervals, for the step's first `cut` events.
 __device__ void run_setup(RunStage& R, uint32_t nseg, uint32_t cut, uint32_t a3, uint32_t plo, uint32_t phi) {
   const uint32_t lane = threadIdx.x & 31;
   constexpr uint32_t kNone = 0xFFFFFFFFu;
@@ -1177,8 +1168,8 @@ __device__ void run_setup(RunStage& R, uint32_t nseg, uint32_t cut, uint32_t a3,
 }
 
 // A step made only of runs (each: word A + j, op, position + j for j < count).  No
-// event is materialised: the shadow is processed in aligned groups of 4 words (one
-// 32-bit load per group, 4 states in SWAR form), and each group applies, in trace
+// event is materialised: the shadow is processed in aligned groups of kGW words (one
+// load per group, kGW states in SWAR form), and each group applies, in trace
 // order, every run that overlaps it — reads classify the covered bytes (P:263:
 // read_host needs OVv, read_target CVv; UUM / USD by the init bits), writes
 // take the VSM write image (WH: OVv, OVi set, CVv clear; WT: CVv, CVi set, OVv
