@@ -694,3 +694,27 @@ def test_runs_fuzz_large(orc, seed):
     cuts = sorted(int(x) for x in np.random.default_rng(seed).choice(rec.shape[0], 4, replace=False))
     rc, got, shadow, st = run_gpu(rec, base, span, flags=flags, flush_points=cuts)
     assert rc == 0 and sorted(got) == exp.triples() and np.array_equal(shadow, exp.shadow)
+
+
+@pytest.mark.parametrize("bb", [0, 9, 12])
+def test_runs_across_4gib_address_blocks(orc, bb):
+    """Runs whose words straddle a 2^32-byte address boundary (the partition's fast
+    decode takes word differences from the low 32 address bits of record 0's block or
+    a neighbouring one), with map / update range ops and sub-word accesses mixed in."""
+    from gen.trace import MAP, OP, UPD, TraceBuilder, encode_np
+    base = (1 << 32) - 3000 * 8                       # 3000 words below the boundary
+    n_words = 8192
+    tb = TraceBuilder()
+    rs = np.random.default_rng(bb)
+    tb.enter(MAP.TOFROM, base, n_words * 8)
+    for k in range(40):
+        lo = int(rs.integers(0, n_words - 1200))
+        ln = int(rs.integers(1, 1200))
+        op = int(rs.choice([OP.RH, OP.WH, OP.RT, OP.WT]))
+        size = 8 if k % 5 else 4
+        tb.add_array(encode_np(op, base + 8 * (lo + np.arange(ln, dtype=np.uint64)), size))
+        if k % 7 == 3:
+            tb.update(int(rs.choice([UPD.TO, UPD.FROM])), base, n_words * 8)
+    tb.exit(MAP.TOFROM, base, n_words * 8)
+    rec = tb.array()
+    check(orc, rec, base, n_words * 8, bucket_bits=bb)
