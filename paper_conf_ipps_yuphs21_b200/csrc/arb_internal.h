@@ -90,7 +90,10 @@ constexpr uint32_t kBucketMask = kMaxBuckets - 1;
 constexpr int kReplayThreads = 256;
 constexpr int kReplayItems = 4;
 constexpr int kStep = kReplayThreads * kReplayItems;  // events per step
-constexpr int kReplayCtasPerSm = 4;
+#ifndef ARB_REPLAY_CTAS_PER_SM
+#define ARB_REPLAY_CTAS_PER_SM 4
+#endif
+constexpr int kReplayCtasPerSm = ARB_REPLAY_CTAS_PER_SM;
 constexpr int kReplayHashBits = 12;                  // fast-step hash: 2^12 slots
 #ifndef ARB_RUN_GROUPS_IN_FLIGHT
 #define ARB_RUN_GROUPS_IN_FLIGHT 1
